@@ -1,0 +1,143 @@
+"""ctypes wrapper of the plain-C oracle ``liblfd_ref.so`` (TEST INFRASTRUCTURE ONLY).
+
+Every function takes NumPy arrays (complex128 / float64, C-contiguous, host memory) in the layouts
+documented at the top of ``oracle/lfd_ref.c`` and mirrors one ``lfd_ref_*`` entry point. Citations
+for the arithmetic are in the C file; this module only marshals arguments.
+"""
+from __future__ import annotations
+
+import ctypes as C
+from dataclasses import dataclass
+
+import numpy as np
+
+from . import build as _build
+
+BC_PERIODIC = 0
+BC_ZERO = 1
+C_LIGHT = 137.035999084  # R1 (atomic units)
+
+
+class _Cfg(C.Structure):
+    _fields_ = [("ndom", C.c_int32), ("nx", C.c_int32), ("ny", C.c_int32), ("nz", C.c_int32),
+                ("hx", C.c_double), ("hy", C.c_double), ("hz", C.c_double), ("bc", C.c_int32),
+                ("norb", C.c_int32), ("nproj", C.c_int32), ("dt", C.c_double)]
+
+
+@dataclass
+class RefConfig:
+    ndom: int
+    nx: int
+    ny: int
+    nz: int
+    hx: float
+    hy: float
+    hz: float
+    bc: int
+    norb: int
+    nproj: int
+    dt: float
+
+    def c(self) -> _Cfg:
+        return _Cfg(self.ndom, self.nx, self.ny, self.nz, self.hx, self.hy, self.hz, self.bc,
+                    self.norb, self.nproj, self.dt)
+
+    @property
+    def ngrid(self) -> int:
+        return self.nx * self.ny * self.nz
+
+    @property
+    def dV(self) -> float:
+        return self.hx * self.hy * self.hz
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        _lib = C.CDLL(_build.build())
+        P = C.c_void_p
+        cfgp = C.POINTER(_Cfg)
+        _lib.lfd_ref_link_sweep.argtypes = [cfgp, P, C.c_int, C.c_int, C.c_double, C.c_double]
+        _lib.lfd_ref_kinetic.argtypes = [cfgp, P, C.c_int, C.c_double, C.c_double]
+        _lib.lfd_ref_local.argtypes = [cfgp, P, P, P]
+        _lib.lfd_ref_nl_half.argtypes = [cfgp, P, P, P]
+        _lib.lfd_ref_step.argtypes = [cfgp, P, P, P, P, P, C.c_int]
+        _lib.lfd_ref_density_current.argtypes = [cfgp, P, P, P, P, P, P]
+        _lib.lfd_ref_kinetic_energy.argtypes = [cfgp, P, P, P]
+        _lib.lfd_ref_kinetic_energy.restype = C.c_double
+        for f in ("link_sweep", "kinetic", "local", "nl_half", "step", "density_current"):
+            getattr(_lib, "lfd_ref_" + f).restype = C.c_int
+    return _lib
+
+
+def _ptr(a: np.ndarray | None, dtype) -> C.c_void_p | None:
+    if a is None:
+        return None
+    if a.dtype != dtype or not a.flags.c_contiguous:
+        raise TypeError(f"expected C-contiguous {dtype}, got {a.dtype}")
+    return C.c_void_p(a.ctypes.data)
+
+
+def _ok(rc: int, what: str) -> None:
+    if rc != 0:
+        raise RuntimeError(f"{what} failed with status {rc}")
+
+
+def link_sweep(cfg: RefConfig, psi: np.ndarray, axis: int, parity: int, tau: float, a: float) -> None:
+    """In place: one E (parity 0) / O (parity 1) sweep of one domain ``psi[nx,ny,nz,norb]``."""
+    c = cfg.c()
+    _ok(lib().lfd_ref_link_sweep(C.byref(c), _ptr(psi, np.complex128), axis, parity, tau, a), "link_sweep")
+
+
+def kinetic(cfg: RefConfig, psi: np.ndarray, axis: int, tau: float, a: float) -> None:
+    c = cfg.c()
+    _ok(lib().lfd_ref_kinetic(C.byref(c), _ptr(psi, np.complex128), axis, tau, a), "kinetic")
+
+
+def local(cfg: RefConfig, psi: np.ndarray, vloc: np.ndarray, A: np.ndarray) -> None:
+    c = cfg.c()
+    _ok(lib().lfd_ref_local(C.byref(c), _ptr(psi, np.complex128), _ptr(vloc, np.float64),
+                            _ptr(np.ascontiguousarray(A, np.float64), np.float64)), "local")
+
+
+def nl_half(cfg: RefConfig, psi: np.ndarray, proj: np.ndarray | None, dnl: np.ndarray | None) -> None:
+    c = cfg.c()
+    _ok(lib().lfd_ref_nl_half(C.byref(c), _ptr(psi, np.complex128), _ptr(proj, np.complex128),
+                              _ptr(dnl, np.float64)), "nl_half")
+
+
+def step(cfg: RefConfig, psi: np.ndarray, proj: np.ndarray | None, dnl: np.ndarray | None,
+         vloc: np.ndarray, A: np.ndarray, nsteps: int = 1) -> None:
+    """In place: ``nsteps`` Eq.-6 steps of every domain with v, A held fixed."""
+    c = cfg.c()
+    A = np.ascontiguousarray(A, np.float64)
+    _ok(lib().lfd_ref_step(C.byref(c), _ptr(psi, np.complex128), _ptr(proj, np.complex128),
+                           _ptr(dnl, np.float64), _ptr(vloc, np.float64), _ptr(A, np.float64), nsteps),
+        "step")
+
+
+def density_current(cfg: RefConfig, psi: np.ndarray, occ: np.ndarray, A: np.ndarray,
+                    want_j: bool = True):
+    """Returns (rho [ndom,ng], j [ndom,3,ng] or None, J [ndom,3])."""
+    c = cfg.c()
+    ng = cfg.ngrid
+    rho = np.zeros((cfg.ndom, ng))
+    j = np.zeros((cfg.ndom, 3, ng)) if want_j else None
+    J = np.zeros((cfg.ndom, 3))
+    A = np.ascontiguousarray(A, np.float64)
+    _ok(lib().lfd_ref_density_current(C.byref(c), _ptr(psi, np.complex128),
+                                      _ptr(np.ascontiguousarray(occ, np.float64), np.float64),
+                                      _ptr(A, np.float64), _ptr(rho, np.float64), _ptr(j, np.float64),
+                                      _ptr(J, np.float64)), "density_current")
+    return rho, j, J
+
+
+def kinetic_energy(cfg: RefConfig, psi: np.ndarray, occ: np.ndarray, A: np.ndarray) -> float:
+    """E_kin of ONE domain (cfg.ndom is ignored beyond the first domain)."""
+    c = cfg.c()
+    return float(lib().lfd_ref_kinetic_energy(C.byref(c), _ptr(psi, np.complex128),
+                                              _ptr(np.ascontiguousarray(occ, np.float64), np.float64),
+                                              _ptr(np.ascontiguousarray(A, np.float64), np.float64)))
