@@ -1,0 +1,367 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 LFD step (driver contract).
+
+One "step" = one pass of the whole hot path of SURVEY §8(a) over one batch of synthetic input:
+  a1 coefficients from A(t_n + Delta/2)  (lfd_set_vector_potential)
+  a2 potential phase from v_loc          (lfd_set_potential)
+  a3-a6 one Eq.-6 LFD step               (lfd_step(1): NL half, local stencil, NL half)
+  a7 density + current + J               (lfd_density_current)
+  a8 (N > 1) the DC recombination: all-gather of every rank's [rho | J] over NCCL.
+Default workload: BASELINE.json configs[1] (= C2: one 70x70x72 domain, 64 orbitals, 64 projectors,
+laser A(t)); under torchrun each rank owns one such domain (C4 weak scaling).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl ours|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = json.load(open(os.path.join(ROOT, "BASELINE.json")))["metric"]
+UNIT = "orbital-gridpoint updates/s"
+PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
+FP64_PEAK_FILE = os.path.join(ROOT, "profiles", "r01_fp64_peaks.jsonl")
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default=None, help="workload name (default C2; C4 under torchrun)")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--seed", type=int, default=1)
+    return ap.parse_args()
+
+
+def peaks():
+    hbm, fp64, src = 6557.1, 37.15, "fallback"
+    if os.path.exists(PEAKS_FILE):
+        p = json.load(open(PEAKS_FILE))
+        hbm = float(p.get("hbm_gbs", hbm))
+        src = "measured (MEASURED_PEAKS.json)"
+    fsrc = "nominal 148 SM x 128 flop/clk x 1.965 GHz"
+    if os.path.exists(FP64_PEAK_FILE):
+        best = 0.0
+        for line in open(FP64_PEAK_FILE):
+            r = json.loads(line)
+            if r.get("kind") == "dmma884":
+                best = max(best, r["tflops"])
+        if best > 0:
+            fp64, fsrc = best, "measured DMMA.8x8x4 issue peak on this pool (profiles/r01_fp64_peaks.jsonl)"
+    return {"hbm_gbs": hbm, "hbm_src": src, "fp64_tflops": fp64, "fp64_src": fsrc}
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region (B200_PROFILING.md clocks line)."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.p = None
+        return self
+
+    def __exit__(self, *a):
+        self.rows = []
+        if self.p is None:
+            return
+        time.sleep(0.25)
+        self.p.terminate()
+        try:
+            out, _ = self.p.communicate(timeout=5)
+        except Exception:
+            self.p.kill()
+            out = ""
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) >= 9:
+                self.rows.append(f)
+
+    def summary(self):
+        if not getattr(self, "rows", None):
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[5 + i] == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def kernel_work(w):
+    """Algorithmic work per launch of each kernel class: (bytes, flops)."""
+    ng, no, npj, nd = w.ngrid, w.norb, w.nproj, w.ndom
+    psi = 16.0 * ng * no * nd
+    bb = 16.0 * ng * npj * nd
+    gemm_flops = 8.0 * ng * no * npj * nd
+    return {
+        "kin_x": (2 * psi + 16.0 * ng * nd, 0.0),
+        "kin_y": (2 * psi, 0.0),
+        "kin_z": (2 * psi + 16.0 * ng * nd, 0.0),
+        "nl_proj": (psi + bb, gemm_flops),
+        "nl_back": (2 * psi + bb, gemm_flops),
+        "density": (psi + 8.0 * ng * nd * 4, 0.0),
+    }
+
+
+def run_reference(args, w, rank, world):
+    """--impl reference: the CPU oracle as it stands, on a bounded sample of the same workload."""
+    out = {"impl": "reference"}
+    if rank != 0:
+        return None
+    from lfd_workloads import make_inputs
+    from lfd_workloads.generate import midpoint_A
+    from oracle import ref
+    x = make_inputs(w, seed=args.seed)
+    # Orbitals evolve independently under Eq. 6 (N and the local factor act column-wise), so a step on
+    # a subset of orbitals is exactly that subset's share of the step: the sample is the first `ns`.
+    ns = min(w.norb, 8)
+    cfg = ref.RefConfig(1, w.nx, w.ny, w.nz, w.hx, w.hy, w.hz, w.bc, ns, w.nproj, w.dt)
+    p = np.ascontiguousarray(x.psi0[:1, ..., :ns])
+    proj = np.ascontiguousarray(x.proj[:1]) if w.nproj else None
+    dnl = np.ascontiguousarray(x.dnl[:1])
+    occ = np.ascontiguousarray(x.occ[:1, :ns])
+    v = np.ascontiguousarray(x.vloc[:1])
+
+    def one(n):
+        A = midpoint_A(w, n)[:1]
+        ref.step(cfg, p, proj, dnl, v, A, 1)
+        ref.density_current(cfg, p, occ, A)
+
+    for n in range(args.warmup):
+        one(n)
+    t0 = time.perf_counter()
+    for n in range(args.steps):
+        one(args.warmup + n)
+    dt = time.perf_counter() - t0
+    ogp = w.ngrid * ns * args.steps
+    val = ogp / dt
+    sample = (f"{args.steps} steps of 1 {w.name} domain ({w.nx}x{w.ny}x{w.nz}, nproj {w.nproj}) restricted to "
+              f"{ns} of {w.norb} orbitals (orbitals evolve independently), incl. density/current")
+    out.update({"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": w.name, "sample_orbitals": ns},
+                "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+                "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}})
+    return out
+
+
+def cpu_baseline(w, seed):
+    """Oracle (single thread, as it stands) on a bounded sample: 1 step of 16 orbitals of the domain."""
+    from lfd_workloads import make_inputs
+    from lfd_workloads.generate import midpoint_A
+    from oracle import ref
+    x = make_inputs(w.with_(ndom=1), seed=seed)
+    ns = min(w.norb, 16)
+    cfg = ref.RefConfig(1, w.nx, w.ny, w.nz, w.hx, w.hy, w.hz, w.bc, ns, w.nproj, w.dt)
+    p = np.ascontiguousarray(x.psi0[..., :ns])
+    A = midpoint_A(w.with_(ndom=1), 0)
+    t0 = time.perf_counter()
+    ref.step(cfg, p, x.proj if w.nproj else None, x.dnl, x.vloc, A, 1)
+    ref.density_current(cfg, p, np.ascontiguousarray(x.occ[:, :ns]), A)
+    dt = time.perf_counter() - t0
+    return {"value": w.ngrid * ns / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"1 step + density of {ns} of {w.norb} orbitals of one {w.name} domain "
+                      f"({w.nx}x{w.ny}x{w.nz}, nproj {w.nproj}); single-threaded plain C, -O2",
+            "seconds": dt}
+
+
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    from lfd_workloads import make_inputs, workload
+    from lfd_workloads.generate import midpoint_A
+    name = args.config or ("C2" if world == 1 else "C4")
+    w = workload(name)
+
+    if args.impl == "reference":
+        out = run_reference(args, w, rank, world)
+        if out is not None:
+            print(json.dumps(out), flush=True)
+        return
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_razakhllknvn24_b200 import Context, lfd
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    x = make_inputs(w, seed=args.seed + rank)
+    stream = torch.cuda.current_stream()
+    psi = torch.from_numpy(x.psi0).to(dev)
+    proj = torch.from_numpy(x.proj).to(dev) if w.nproj else None
+    v_dev = torch.from_numpy(x.vloc).to(dev)
+    ctx = Context(psi, proj, x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc)
+    nd, ng = w.ndom, w.ngrid
+    rho = torch.empty((nd, ng), dtype=torch.float64, device=dev)
+    J = torch.empty((nd, 3), dtype=torch.float64, device=dev)
+    # global gather buffer of the DC recombination: [world][nd*(ng+3)]
+    send = torch.empty(nd * (ng + 3), dtype=torch.float64, device=dev)
+    recv = torch.empty(world * nd * (ng + 3), dtype=torch.float64, device=dev) if world > 1 else None
+    A_seq = [midpoint_A(w, n) for n in range(args.warmup + args.steps)]
+
+    def step(n):
+        lfd.lfd_set_vector_potential(ctx.ctx, A_seq[n])
+        lfd.lfd_set_potential(ctx.ctx, v_dev)
+        lfd.lfd_step(ctx.ctx, 1)
+        if world > 1:
+            lfd.lfd_density_current(ctx.ctx, send[: nd * ng], None, send[nd * ng:])
+            dist.all_gather_into_tensor(recv, send)
+        else:
+            lfd.lfd_density_current(ctx.ctx, rho, None, J)
+
+    for n in range(args.warmup):
+        step(n)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    l0 = lfd.lfd_launch_count(ctx.ctx)
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    with Clocks(local) as clk:
+        e0.record(stream)
+        for n in range(args.steps):
+            step(args.warmup + n)
+        e1.record(stream)
+        torch.cuda.synchronize()
+    launches = lfd.lfd_launch_count(ctx.ctx) - l0
+    ms = e0.elapsed_time(e1)
+    t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item())
+    sec = ms / 1e3
+    ogp = w.ogp_per_step * world * args.steps
+    value = ogp / sec
+
+    # per-kernel device time over an identical second pass (events around every launch, same stream)
+    lfd.lfd_profile_enable(ctx.ctx, True)
+    torch.cuda.synchronize()
+    p0 = time.perf_counter()
+    for n in range(args.steps):
+        step(args.warmup + n)
+    torch.cuda.synchronize()
+    prof = lfd.lfd_profile_read(ctx.ctx)
+    lfd.lfd_profile_enable(ctx.ctx, False)
+    del p0
+    pk = peaks()
+    work = kernel_work(w)
+    kernels = {}
+    total_ms = sum(v[0] for v in prof.values())
+    for k, (kms, cnt) in prof.items():
+        if cnt == 0:
+            continue
+        avg = kms / cnt
+        e = {"ms_per_launch": avg, "launches": cnt, "share": kms / total_ms if total_ms else None}
+        if k in work:
+            b, f = work[k]
+            if f > 0:
+                e.update({"bound": "tensor", "achieved": f / (avg * 1e-3) / 1e12, "unit": "TFLOP/s",
+                          "peak": pk["fp64_tflops"]})
+            else:
+                e.update({"bound": "hbm", "achieved": b / (avg * 1e-3) / 1e9, "unit": "GB/s",
+                          "peak": pk["hbm_gbs"]})
+            e["frac"] = e["achieved"] / e["peak"]
+        kernels[k] = e
+    dom = max((k for k in kernels if "achieved" in kernels[k]), key=lambda k: prof[k][0])
+    d = kernels[dom]
+    roofline = {"kernel": dom, "bound": d["bound"], "achieved": d["achieved"], "peak": d["peak"], "unit": d["unit"],
+                "frac": d["frac"], "traffic": None,
+                "peak_source": pk["fp64_src"] if d["bound"] == "tensor" else pk["hbm_src"],
+                "flops_per_launch" if d["bound"] == "tensor" else "bytes_per_launch":
+                    work[dom][1] if d["bound"] == "tensor" else work[dom][0]}
+
+    # end to end through the C ABI with HOST buffers: pinned v in, pinned rho + J out, every step
+    e2e = None
+    if not args.no_e2e:
+        vh = torch.from_numpy(x.vloc.copy()).pin_memory()
+        rh = torch.empty((nd, ng), dtype=torch.float64).pin_memory()
+        Jh = torch.empty((nd, 3), dtype=torch.float64).pin_memory()
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        f0 = torch.cuda.Event(enable_timing=True)
+        f1 = torch.cuda.Event(enable_timing=True)
+        t0 = time.perf_counter()
+        f0.record(stream)
+        for n in range(args.steps):
+            lfd.lfd_set_vector_potential(ctx.ctx, A_seq[args.warmup + n])
+            lfd.lfd_set_potential_host(ctx.ctx, vh)
+            lfd.lfd_step(ctx.ctx, 1)
+            lfd.lfd_density_current_host(ctx.ctx, rh, Jh)
+            if world > 1:
+                lfd.lfd_density_current(ctx.ctx, send[: nd * ng], None, send[nd * ng:])
+                dist.all_gather_into_tensor(recv, send)
+            lfd.lfd_sync(ctx.ctx)  # the host reads this step's rho / J
+            _ = float(Jh[0, 2])
+        f1.record(stream)
+        torch.cuda.synchronize()
+        ems = max(f0.elapsed_time(f1), 1e3 * (time.perf_counter() - t0))
+        te = torch.tensor([ems], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e2e = {"value": ogp / (float(te.item()) / 1e3), "unit": UNIT, "h2d_bytes_per_step": int(nd * ng * 8),
+               "d2h_bytes_per_step": int(nd * ng * 8 + nd * 3 * 8),
+               "note": "per step: H2D v_loc (pinned) -> a1..a7 -> D2H rho + J (pinned) -> host sync; "
+                       "Psi and B stay resident in HBM (the paper's GPU-resident design, P:216)"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(w, args.seed)
+
+    if rank == 0:
+        out = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "lfd_steps_per_s": world * w.ndom * args.steps / sec,
+            "config": {"workload": name, "ndomains_per_gpu": w.ndom, "grid": [w.nx, w.ny, w.nz], "norb": w.norb,
+                       "nproj": w.nproj, "bc": "periodic" if w.bc == 0 else "zero", "laser": w.laser,
+                       "ogp_per_step_per_gpu": w.ogp_per_step,
+                       "l2": f"inputs exceed L2 (Psi+B = {16 * w.ngrid * (w.norb + w.nproj) * w.ndom / 1e6:.0f} MB "
+                             "per GPU vs 126 MB L2); no explicit flush",
+                       "parallelism": f"domains{world}" if world > 1 else "single"},
+            "gpu_launches": int(launches),
+            "clocks": clk.summary(),
+            "roofline": roofline,
+            "kernels": kernels,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(out), flush=True)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

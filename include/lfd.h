@@ -1,0 +1,171 @@
+/*
+ * lfd.h -- C ABI of the B200-native Local Field Dynamics (LFD) step of DC-MESH.
+ *
+ * What the library computes (PAPER.md = /root/reference/PAPER.md, "P:n" = line n; the readings
+ * R1..R22 are listed in DESIGN.md §3):
+ *   One LFD/QD time step of Eq. 6 for every divide-and-conquer domain (Fig. 1):
+ *       Psi <- N( Local( N(Psi) ) )
+ *   * Local = exp(-i Delta h_loc) of Eq. 5 by the O(N) space-splitting stencil (P:68, P:76-80,
+ *     Alg. 1-5): Psi <- Phi . K_z K_y K_x (Phi . Psi), Phi = e^{-i (Delta/2) v_loc},
+ *     K_d = E_d(Delta/2) O_d(Delta) E_d(Delta/2) (2x2 pair blocks with Peierls phases for A(t); R2-R8).
+ *   * N = the renormalised first-order nonlocal factor (1 - i Delta/2 v_nl)/||...|| of Eq. 6 with the
+ *     scissor projector of Eq. 7, BLASified as in Eq. 9: C = dV B^H Psi,
+ *     Psi <- (Psi - i (Delta/2) B diag(D) C) diag(n), n_s restoring each orbital's norm (R9-R12).
+ *   * Density rho = sum_s f_s |psi_s|^2 and the gauge-consistent link current j, J (R13).
+ *
+ * Conventions (all entry points):
+ *   - Units: atomic units, hbar = m = e = 1, c = 137.035999084 (R1).
+ *   - Layout: complex128 = two doubles (re, im) interleaved; orbital index fastest, then z, y, x,
+ *     then domain:  psi[dom][x][y][z][orb]  (the paper's SoA psi[i][j][k][n]).
+ *     Grid index r = ((x*ny)+y)*nz+z. Orbitals are normalised as dV * sum_r |psi|^2 = 1 (R12).
+ *   - Ownership: the caller owns every buffer (device buffers are typically torch tensors) and keeps
+ *     the borrowed ones (psi, proj, workspace) alive until lfd_destroy. The library owns only the
+ *     context struct. Small HOST arrays are copied (or captured by value) during the call.
+ *   - Streams: all device work is enqueued on the context's CUDA stream, in call order. Calls return
+ *     before the GPU finishes; lfd_sync() waits and reports asynchronous CUDA errors.
+ *   - Errors: every call returns lfd_status. Arguments are validated before anything is enqueued and a
+ *     failed call changes no state. No C++ exception crosses the ABI. lfd_last_error() gives text.
+ *   - Threading: one context = one host thread + one stream. Many contexts may coexist.
+ *   - There is no CPU fallback: without a usable sm_100a device, lfd_init returns LFD_ECUDA.
+ */
+#ifndef LFD_H_
+#define LFD_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define LFD_ABI_VERSION 1
+#define LFD_MAX_DOMAINS 4096
+
+typedef struct lfd_ctx lfd_ctx; /* opaque */
+
+typedef enum {
+  LFD_OK = 0,
+  LFD_EINVAL = -1,       /* bad argument or configuration */
+  LFD_ENOMEM = -2,       /* workspace too small / host allocation failed */
+  LFD_ECUDA = -3,        /* CUDA runtime error (including no sm_100 device) */
+  LFD_ESTATE = -4,       /* call not valid in the current state (e.g. use after destroy) */
+  LFD_EUNSUPPORTED = -5  /* valid request this build does not implement */
+} lfd_status;
+
+typedef enum { LFD_BC_PERIODIC = 0, LFD_BC_ZERO = 1 } lfd_bc; /* reading R8 */
+
+typedef struct {
+  int32_t abi_version; /* must equal LFD_ABI_VERSION */
+  int32_t ndomains;    /* same-shape DC domains batched in this context, 1..LFD_MAX_DOMAINS */
+  int32_t nx, ny, nz;  /* mesh points per domain, each >= 2; even when bc == LFD_BC_PERIODIC */
+  double hx, hy, hz;   /* mesh spacing [bohr], > 0 */
+  int32_t bc;          /* lfd_bc */
+  int32_t norb;        /* propagated KS orbitals per domain, >= 1 */
+  int32_t nproj;       /* projector columns per domain, >= 0 (0 disables the nonlocal factor) */
+  double dt;           /* Delta_QD [a.u.], finite and nonzero (negative = backward in time) */
+  int32_t device;      /* CUDA device ordinal */
+  int32_t flags;       /* reserved, must be 0 */
+} lfd_config;
+
+/* Kernel classes, for lfd_profile_read(). */
+typedef enum {
+  LFD_K_COEF = 0,      /* a1: stencil coefficients from A(t) */
+  LFD_K_PHASE = 1,     /* a2: Phi = exp(-i Delta/2 v_loc) */
+  LFD_K_KIN_X = 2,     /* a6: Phi . K_x (pre-phase fused) */
+  LFD_K_KIN_Y = 3,     /* a6: K_y */
+  LFD_K_KIN_Z = 4,     /* a6: K_z . Phi (post-phase fused) */
+  LFD_K_NL_PROJ = 5,   /* a3: GEMM-1 split-K partials of C = dV B^H Psi + column norms */
+  LFD_K_NL_REDUCE = 6, /* a4: fixed-order split-K reduction, C' = -i(Delta/2) D C */
+  LFD_K_NL_NORM = 7,   /* a4: n_s from the Gram closed form */
+  LFD_K_NL_BACK = 8,   /* a5: GEMM-2 Psi <- (Psi + B C') diag(n), in place */
+  LFD_K_DENSITY = 9,   /* a7: rho, j, per-line partial J */
+  LFD_K_JREDUCE = 10,  /* a7: J = mean of j (fixed order) */
+  LFD_K_COUNT = 11
+} lfd_kernel_id;
+
+/* Bytes of DEVICE workspace lfd_init needs for this configuration. */
+lfd_status lfd_workspace_size(const lfd_config* cfg, size_t* bytes);
+
+/* Create a context.
+ *  psi   DEVICE complex128 [ndom][nx][ny][nz][norb]; borrowed; propagated in place by lfd_step.
+ *  proj  DEVICE complex128 [ndom][nx][ny][nz][nproj]; borrowed, read-only (B = Psi_u(0), the
+ *        unoccupied KS orbitals at t = 0, Eq. 7 P:68 / R9); NULL iff nproj == 0. Need not be
+ *        orthonormal: the Gram matrix G = dV B^H B is computed here (on the device) and used for n_s.
+ *  dnl   HOST double [ndom][nproj] real couplings D_u (paper: all equal Delta_sci of Eq. 8);
+ *        copied. May be NULL iff nproj == 0.
+ *  occ   HOST double [ndom][norb] occupations f_s (not clamped, R14); copied.
+ *  workspace DEVICE, >= lfd_workspace_size bytes, 256-byte aligned; borrowed.
+ *  stream cudaStream_t (NULL = legacy default stream); all work is ordered on it.
+ * Initial state: v_loc = 0 (Phi = 1) and A = 0 until the setters are called.
+ * Errors: LFD_EINVAL (bad config / pointer kind / alignment), LFD_ENOMEM (workspace too small),
+ *         LFD_ECUDA (no sm_100 device or a CUDA failure). *out is set only on LFD_OK. */
+lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const double* dnl,
+                    const double* occ, void* workspace, size_t ws_bytes, void* stream, lfd_ctx** out);
+
+/* v_loc(r) at the step midpoint (Eq. 4; Eq. 5 v_loc), DEVICE double [ndom][nx][ny][nz]
+ * [Hartree]; read in stream order (Phi is computed on the device; the buffer may be reused after the
+ * call's work has run). */
+lfd_status lfd_set_potential(lfd_ctx* ctx, const double* vloc);
+
+/* As lfd_set_potential, but vloc is a HOST buffer (pinned recommended): an async H2D copy into the
+ * workspace is enqueued. The host buffer must stay unchanged until that copy has run (lfd_sync). */
+lfd_status lfd_set_potential_host(lfd_ctx* ctx, const double* vloc_host);
+
+/* A_X(alpha)(t) at the step midpoint (Eq. 2 / Eq. 5; Eq. 4 midpoint), HOST double [ndom][3] a.u.;
+ * captured by value (the coefficient table is rebuilt on the device in stream order). */
+lfd_status lfd_set_vector_potential(lfd_ctx* ctx, const double* A);
+
+/* Enqueue nsteps LFD steps (Eq. 6) with the current v_loc and A. nsteps == 0 is a no-op; < 0 EINVAL. */
+lfd_status lfd_step(lfd_ctx* ctx, int32_t nsteps);
+
+/* Density and current of the current Psi with the current A (kernel 4; R13):
+ *  rho  DEVICE double [ndom][nx][ny][nz]          rho_r = sum_s f_s |psi_rs|^2
+ *  j    DEVICE double [ndom][3][nx][ny][nz] or NULL
+ *       j_d,r = (1/h_d) sum_s f_s Im(e^{i A_d h_d / c} conj(psi_rs) psi_{r+e_d,s}) (left-node link
+ *       current; periodic wrap, or 0 on the last plane for zero BC). Electron-number current.
+ *  Jmac DEVICE double [ndom][3] or NULL            J_d = (1/Ngrid) sum_r j_d,r
+ */
+lfd_status lfd_density_current(lfd_ctx* ctx, double* rho, double* j, double* Jmac);
+
+/* As lfd_density_current, but writes each domain's core into GLOBAL-layout device arrays
+ * rho_g [GX][GY][GZ] and j_g [3][GX][GY][GZ] (j_g may be NULL) at the HOST-given offsets
+ * dom_offset[ndom][3]; domain cores must lie inside gdims[3] and must not overlap. Untouched global
+ * points are left as they are (callers zero them; a SUM all-reduce then assembles the DC
+ * recombination of rho, R18). Jmac as above (per domain, may be NULL). */
+lfd_status lfd_density_current_global(lfd_ctx* ctx, double* rho_g, double* j_g, double* Jmac,
+                                      const int32_t* dom_offset, const int32_t* gdims);
+
+/* As lfd_density_current for rho and Jmac, into HOST buffers (pinned recommended) via async D2H
+ * copies; read them after lfd_sync(). Either pointer may be NULL to skip it. */
+lfd_status lfd_density_current_host(lfd_ctx* ctx, double* rho_host, double* Jmac_host);
+
+/* Replace the occupations f (the QXMD<->LFD shadow-dynamics handshake). HOST [ndom][norb]. */
+lfd_status lfd_set_occupations(lfd_ctx* ctx, const double* occ);
+
+/* Change the stream used by later calls (work already enqueued stays on the old stream). */
+lfd_status lfd_set_stream(lfd_ctx* ctx, void* stream);
+
+/* Wait for all enqueued work; LFD_ECUDA if any asynchronous CUDA error occurred. */
+lfd_status lfd_sync(lfd_ctx* ctx);
+
+/* Number of kernels this context has launched so far (all classes). */
+lfd_status lfd_launch_count(const lfd_ctx* ctx, uint64_t* count);
+
+/* Per-kernel-class device timing with CUDA events on the context stream.
+ * lfd_profile_enable(ctx, 1) starts recording an event pair around every launch;
+ * lfd_profile_read() synchronises, returns accumulated milliseconds and launch counts per class
+ * (arrays of LFD_K_COUNT), and resets the accumulators. enable 0 stops recording. */
+lfd_status lfd_profile_enable(lfd_ctx* ctx, int32_t enable);
+lfd_status lfd_profile_read(lfd_ctx* ctx, double* ms, int64_t* launches);
+
+/* Message of the last error on this context (ctx == NULL: of the last failed lfd_init /
+ * lfd_workspace_size on this thread). Never NULL. */
+const char* lfd_last_error(const lfd_ctx* ctx);
+
+/* Free the context struct (never caller memory). Waits for the context's work first. NULL is OK. */
+lfd_status lfd_destroy(lfd_ctx* ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LFD_H_ */

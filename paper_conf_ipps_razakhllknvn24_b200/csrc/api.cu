@@ -1,0 +1,589 @@
+// api.cu -- the C ABI of include/lfd.h: validation, workspace layout, step sequencing, profiling.
+// Every numerical step runs in the sm_100a kernels of kin.cu / nl.cu / dens.cu; this file only
+// orders them on the context stream. There is no CPU fallback.
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <set>
+#include <string>
+#include <vector>
+
+#include "../../include/lfd.h"
+#include "lfd_internal.h"
+
+using lfd::DomCoef;
+using lfd::Geometry;
+
+namespace {
+
+constexpr size_t kAlign = 256;
+constexpr int kKC1 = 16;  // GEMM-1 rows per chunk (nl.cu)
+
+size_t up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
+
+struct Layout {
+  size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage;
+  size_t total;
+  int nsplit;
+  long long rows_per_split;
+};
+
+thread_local std::string g_tls_error = "no error";
+std::mutex g_live_mu;
+std::set<const void*> g_live;
+
+bool is_live(const void* p) {
+  std::lock_guard<std::mutex> lk(g_live_mu);
+  return g_live.count(p) != 0;
+}
+
+lfd_status validate(const lfd_config* c, std::string& why) {
+  if (!c) { why = "config is NULL"; return LFD_EINVAL; }
+  if (c->abi_version != LFD_ABI_VERSION) { why = "abi_version mismatch"; return LFD_EINVAL; }
+  if (c->ndomains < 1 || c->ndomains > LFD_MAX_DOMAINS) { why = "ndomains out of range"; return LFD_EINVAL; }
+  if (c->nx < 2 || c->ny < 2 || c->nz < 2) { why = "each of nx, ny, nz must be >= 2"; return LFD_EINVAL; }
+  if (c->bc != LFD_BC_PERIODIC && c->bc != LFD_BC_ZERO) { why = "bad bc"; return LFD_EINVAL; }
+  if (c->bc == LFD_BC_PERIODIC && ((c->nx | c->ny | c->nz) & 1)) {
+    why = "periodic boundary needs even nx, ny, nz (pair splitting, reading R8)";
+    return LFD_EINVAL;
+  }
+  if (!(c->hx > 0) || !(c->hy > 0) || !(c->hz > 0) || !std::isfinite(c->hx * c->hy * c->hz)) {
+    why = "spacings must be finite and > 0";
+    return LFD_EINVAL;
+  }
+  if (c->norb < 1) { why = "norb must be >= 1"; return LFD_EINVAL; }
+  if (c->nproj < 0) { why = "nproj must be >= 0"; return LFD_EINVAL; }
+  if (!(c->dt != 0.0) || !std::isfinite(c->dt)) { why = "dt must be finite and nonzero"; return LFD_EINVAL; }
+  if (c->flags != 0) { why = "flags must be 0"; return LFD_EINVAL; }
+  const long long ng = (long long)c->nx * c->ny * c->nz;
+  if (ng * (long long)std::max(c->norb, std::max(c->nproj, 1)) >= (1LL << 31)) {
+    why = "ng * max(norb, nproj) must be < 2^31 per domain";
+    return LFD_EINVAL;
+  }
+  return LFD_OK;
+}
+
+Geometry geometry(const lfd_config* c) {
+  Geometry g;
+  g.ndom = c->ndomains; g.nx = c->nx; g.ny = c->ny; g.nz = c->nz;
+  g.norb = c->norb; g.nproj = c->nproj; g.bc = c->bc;
+  g.hx = c->hx; g.hy = c->hy; g.hz = c->hz; g.dt = c->dt; g.dV = c->hx * c->hy * c->hz;
+  g.ng = (long long)c->nx * c->ny * c->nz;
+  return g;
+}
+
+Layout layout(const Geometry& g, int num_sms) {
+  Layout L{};
+  const int np = g.nproj, no = g.norb, nd = g.ndom;
+  // split-K of GEMM-1: about one CTA per SM in total, each split a multiple of the chunk height
+  int tiles = 0;
+  if (np > 0) {
+    const int t1 = ((np + 63) / 64) * ((no + 63) / 64);
+    const int t2 = ((np + 63) / 64) * ((np + 63) / 64);
+    tiles = std::min(t1, t2) * nd;
+  }
+  int nsplit = tiles > 0 ? std::max(1, num_sms / std::max(tiles, 1)) : 1;
+  long long rps = (g.ng + nsplit - 1) / nsplit;
+  rps = std::max<long long>(kKC1, (rps + kKC1 - 1) / kKC1 * kKC1);
+  nsplit = (int)((g.ng + rps - 1) / rps);
+  L.nsplit = nsplit;
+  L.rows_per_split = rps;
+  const size_t c16 = 16, d8 = 8;
+  const size_t mn = (size_t)std::max(np * no, np * np);
+  size_t o = 0;
+  auto take = [&](size_t bytes) { size_t at = o; o += up(std::max<size_t>(bytes, 1)); return at; };
+  L.phi = take((size_t)nd * g.ng * c16);
+  L.coef = take((size_t)nd * sizeof(DomCoef));
+  L.G = take((size_t)nd * np * np * c16);
+  L.D = take((size_t)nd * np * d8);
+  L.occ = take((size_t)nd * no * d8);
+  L.part = take((size_t)nd * nsplit * mn * c16);
+  L.normp = take((size_t)nd * nsplit * no * d8);
+  L.dc = take((size_t)nd * np * no * c16);
+  L.cprime = take((size_t)nd * np * no * c16);
+  L.s = take((size_t)nd * no * d8);
+  L.nfac = take((size_t)nd * no * d8);
+  L.jline = take((size_t)nd * g.nx * g.ny * 3 * d8);
+  L.base = take((size_t)4 * nd * sizeof(long long));
+  L.vstage = take((size_t)nd * g.ng * d8);
+  L.rhostage = take((size_t)nd * g.ng * d8);
+  L.Jstage = take((size_t)nd * 3 * d8);
+  L.total = o;
+  return L;
+}
+
+int query_sms(int device) {
+  int sms = 0;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) return 0;
+  return sms;
+}
+
+struct ProfSlot {
+  int kid;
+  cudaEvent_t a, b;
+};
+
+}  // namespace
+
+struct lfd_ctx {
+  lfd_config cfg;
+  Geometry g;
+  Layout L;
+  double2* psi;
+  const double2* proj;
+  char* ws;
+  size_t ws_bytes;
+  cudaStream_t stream;
+  int device;
+  int num_sms;
+  uint64_t launches = 0;
+  std::string err = "no error";
+  // density-current global layout cache
+  std::vector<long long> gbase_host;
+  // profiling
+  bool prof = false;
+  std::vector<ProfSlot> slots;
+  size_t nslot = 0;
+  double prof_ms[LFD_K_COUNT] = {0};
+  int64_t prof_n[LFD_K_COUNT] = {0};
+
+  template <class T>
+  T* at(size_t off) const { return reinterpret_cast<T*>(ws + off); }
+  DomCoef* coef() const { return at<DomCoef>(L.coef); }
+  double2* phi() const { return at<double2>(L.phi); }
+};
+
+namespace {
+
+lfd_status fail(lfd_ctx* c, lfd_status st, const std::string& msg) {
+  if (c) c->err = msg; else g_tls_error = msg;
+  return st;
+}
+
+lfd_status cuda_fail(lfd_ctx* c, cudaError_t e, const char* what) {
+  std::string m = std::string(what) + ": " + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ")";
+  return fail(c, LFD_ECUDA, m);
+}
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+void prof_flush(lfd_ctx* c) {
+  if (c->nslot == 0) return;
+  cudaStreamSynchronize(c->stream);
+  for (size_t i = 0; i < c->nslot; ++i) {
+    float ms = 0.f;
+    if (cudaEventElapsedTime(&ms, c->slots[i].a, c->slots[i].b) == cudaSuccess) {
+      c->prof_ms[c->slots[i].kid] += ms;
+      c->prof_n[c->slots[i].kid] += 1;
+    }
+  }
+  c->nslot = 0;
+}
+
+template <class F>
+lfd_status launch(lfd_ctx* c, int kid, const char* name, F&& f) {
+  ProfSlot* s = nullptr;
+  if (c->prof) {
+    if (c->nslot == c->slots.size()) {
+      if (c->slots.size() < 8192) {
+        ProfSlot ns{};
+        if (cudaEventCreate(&ns.a) != cudaSuccess || cudaEventCreate(&ns.b) != cudaSuccess)
+          return fail(c, LFD_ECUDA, "cudaEventCreate failed");
+        c->slots.push_back(ns);
+      } else {
+        prof_flush(c);
+      }
+    }
+    s = &c->slots[c->nslot++];
+    s->kid = kid;
+    cudaEventRecord(s->a, c->stream);
+  }
+  cudaError_t e = f();
+  if (s) cudaEventRecord(s->b, c->stream);
+  c->launches++;
+  if (e != cudaSuccess) return cuda_fail(c, e, name);
+  return LFD_OK;
+}
+
+#define LFD_TRY(x)                 \
+  do {                             \
+    lfd_status st_ = (x);          \
+    if (st_ != LFD_OK) return st_; \
+  } while (0)
+
+lfd_status check_ctx(const lfd_ctx* c) {
+  if (!c) { g_tls_error = "context is NULL"; return LFD_EINVAL; }
+  if (!is_live(c)) { g_tls_error = "context is not live (destroyed or never created)"; return LFD_ESTATE; }
+  return LFD_OK;
+}
+
+bool is_device_ptr(const void* p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+// Eq. 6 nonlocal factor N on every domain (kernels a3, a4, a5).
+lfd_status nl_half(lfd_ctx* c) {
+  const Geometry& g = c->g;
+  lfd::Gemm1Args a1;
+  a1.A = c->proj;
+  a1.X = c->psi;
+  a1.part = c->at<double2>(c->L.part);
+  a1.norms = c->at<double>(c->L.normp);
+  a1.ndom = g.ndom; a1.mrows = g.nproj; a1.ncols = g.norb; a1.nsplit = c->L.nsplit;
+  a1.ng = g.ng; a1.rows_per_split = c->L.rows_per_split;
+  a1.a_dom_stride = g.ng * g.nproj; a1.x_dom_stride = g.ng * g.norb;
+  LFD_TRY(launch(c, LFD_K_NL_PROJ, "k_gemm1", [&] { return lfd::launch_gemm1(a1, c->stream); }));
+  lfd::ReduceArgs r;
+  r.part = a1.part; r.normp = a1.norms;
+  r.D = c->at<double>(c->L.D);
+  r.out = c->at<double2>(c->L.dc);
+  r.cprime = c->at<double2>(c->L.cprime);
+  r.s = c->at<double>(c->L.s);
+  r.ndom = g.ndom; r.mrows = g.nproj; r.ncols = g.norb; r.nsplit = c->L.nsplit;
+  r.scale = g.dV; r.eps = 0.5 * g.dt;
+  LFD_TRY(launch(c, LFD_K_NL_REDUCE, "k_reduce", [&] { return lfd::launch_reduce(r, c->stream); }));
+  LFD_TRY(launch(c, LFD_K_NL_NORM, "k_nlnorm", [&] {
+    return lfd::launch_nlnorm(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), r.out, r.s,
+                              c->at<double>(c->L.nfac), c->stream);
+  }));
+  lfd::Gemm2Args a2;
+  a2.psi = c->psi; a2.B = c->proj; a2.Cp = r.cprime; a2.nfac = c->at<double>(c->L.nfac);
+  a2.ndom = g.ndom; a2.nproj = g.nproj; a2.norb = g.norb; a2.ng = g.ng; a2.num_sms = c->num_sms;
+  return launch(c, LFD_K_NL_BACK, "k_gemm2", [&] { return lfd::launch_gemm2(a2, c->stream); });
+}
+
+lfd_status set_A(lfd_ctx* c, const double* A) {
+  thread_local lfd::CoefParams tp;  // 12 KB kernel-parameter block (A captured by value)
+  for (int d0 = 0; d0 < c->g.ndom; d0 += lfd::kCoefMaxPerLaunch) {
+    const int cnt = std::min(lfd::kCoefMaxPerLaunch, c->g.ndom - d0);
+    for (int i = 0; i < cnt; ++i)
+      for (int d = 0; d < 3; ++d) tp.A[i][d] = A ? A[3 * (d0 + i) + d] : 0.0;
+    LFD_TRY(launch(c, LFD_K_COEF, "k_coef",
+                   [&] { return lfd::launch_coef(c->g, tp, d0, cnt, c->coef(), c->stream); }));
+  }
+  return LFD_OK;
+}
+
+lfd_status density_into(lfd_ctx* c, double* rho, double* j, double* Jmac, const long long* base_dev, long long sx,
+                        long long sy, long long jstride) {
+  lfd::DensArgs a;
+  a.psi = c->psi; a.coef = c->coef(); a.occ = c->at<double>(c->L.occ);
+  a.rho = rho; a.j = j; a.jline = c->at<double>(c->L.jline);
+  a.base = base_dev; a.jbase = base_dev + c->g.ndom; a.sx = sx; a.sy = sy; a.jstride = jstride;
+  LFD_TRY(launch(c, LFD_K_DENSITY, "k_density", [&] { return lfd::launch_density(c->g, a, c->stream); }));
+  if (Jmac)
+    LFD_TRY(launch(c, LFD_K_JREDUCE, "k_jreduce",
+                   [&] { return lfd::launch_jreduce(c->g, a.jline, Jmac, c->stream); }));
+  return LFD_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+lfd_status lfd_workspace_size(const lfd_config* cfg, size_t* bytes) {
+  std::string why;
+  lfd_status st = validate(cfg, why);
+  if (st != LFD_OK) return fail(nullptr, st, why);
+  if (!bytes) return fail(nullptr, LFD_EINVAL, "bytes is NULL");
+  const int sms = query_sms(cfg->device);
+  if (sms <= 0) return fail(nullptr, LFD_ECUDA, "no CUDA device (the LFD library has no CPU fallback)");
+  *bytes = layout(geometry(cfg), sms).total;
+  return LFD_OK;
+}
+
+lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const double* dnl, const double* occ,
+                    void* workspace, size_t ws_bytes, void* stream, lfd_ctx** out) {
+  std::string why;
+  lfd_status st = validate(cfg, why);
+  if (st != LFD_OK) return fail(nullptr, st, why);
+  if (!out) return fail(nullptr, LFD_EINVAL, "out is NULL");
+  if (!psi || !workspace || !occ) return fail(nullptr, LFD_EINVAL, "psi, workspace and occ must be non-NULL");
+  if ((cfg->nproj > 0) != (proj != nullptr)) return fail(nullptr, LFD_EINVAL, "proj must be non-NULL iff nproj > 0");
+  if (cfg->nproj > 0 && !dnl) return fail(nullptr, LFD_EINVAL, "dnl must be non-NULL when nproj > 0");
+  if ((reinterpret_cast<uintptr_t>(psi) | reinterpret_cast<uintptr_t>(proj)) & 15)
+    return fail(nullptr, LFD_EINVAL, "psi / proj must be 16-byte aligned");
+  if (reinterpret_cast<uintptr_t>(workspace) & (kAlign - 1))
+    return fail(nullptr, LFD_EINVAL, "workspace must be 256-byte aligned");
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || cfg->device < 0 || cfg->device >= ndev) {
+    cudaGetLastError();
+    return fail(nullptr, LFD_ECUDA, "no such CUDA device (the LFD library has no CPU fallback)");
+  }
+  cudaDeviceProp prop;
+  if (cudaGetDeviceProperties(&prop, cfg->device) != cudaSuccess) return fail(nullptr, LFD_ECUDA, "cudaGetDeviceProperties failed");
+  if (prop.major != 10) return fail(nullptr, LFD_ECUDA, "this build targets sm_100a (B200) only");
+  DeviceGuard dg(cfg->device);
+  if (!is_device_ptr(psi) || !is_device_ptr(workspace) || (proj && !is_device_ptr(proj)))
+    return fail(nullptr, LFD_EINVAL, "psi, proj and workspace must be device memory");
+  const Geometry g = geometry(cfg);
+  const Layout L = layout(g, prop.multiProcessorCount);
+  if (ws_bytes < L.total) return fail(nullptr, LFD_ENOMEM, "workspace smaller than lfd_workspace_size()");
+  cudaError_t e = lfd::gemm_set_attributes();
+  if (e != cudaSuccess) return cuda_fail(nullptr, e, "cudaFuncSetAttribute");
+
+  lfd_ctx* c = new (std::nothrow) lfd_ctx();
+  if (!c) return fail(nullptr, LFD_ENOMEM, "host allocation failed");
+  c->cfg = *cfg; c->g = g; c->L = L;
+  c->psi = static_cast<double2*>(psi);
+  c->proj = static_cast<const double2*>(proj);
+  c->ws = static_cast<char*>(workspace);
+  c->ws_bytes = ws_bytes;
+  c->stream = static_cast<cudaStream_t>(stream);
+  c->device = cfg->device;
+  c->num_sms = prop.multiProcessorCount;
+  {
+    std::lock_guard<std::mutex> lk(g_live_mu);
+    g_live.insert(c);
+  }
+  auto bail = [&](lfd_status s) {
+    std::string m = c->err;
+    lfd_destroy(c);
+    return fail(nullptr, s, m);
+  };
+  // copies of the small host arrays (pageable H2D copies are staged before the call returns)
+  if (g.nproj > 0) {
+    e = cudaMemcpyAsync(c->at<double>(L.D), dnl, sizeof(double) * g.ndom * g.nproj, cudaMemcpyHostToDevice, c->stream);
+    if (e != cudaSuccess) { cuda_fail(c, e, "copy dnl"); return bail(LFD_ECUDA); }
+  }
+  e = cudaMemcpyAsync(c->at<double>(L.occ), occ, sizeof(double) * g.ndom * g.norb, cudaMemcpyHostToDevice, c->stream);
+  if (e != cudaSuccess) { cuda_fail(c, e, "copy occ"); return bail(LFD_ECUDA); }
+  // local-layout output bases for the density kernel: rho [dom][ng], j [dom][3][ng]
+  std::vector<long long> base(2 * g.ndom);
+  for (int d = 0; d < g.ndom; ++d) {
+    base[d] = (long long)d * g.ng;
+    base[g.ndom + d] = (long long)d * 3 * g.ng;
+  }
+  e = cudaMemcpyAsync(c->at<long long>(L.base), base.data(), sizeof(long long) * base.size(), cudaMemcpyHostToDevice,
+                      c->stream);
+  if (e != cudaSuccess) { cuda_fail(c, e, "copy base"); return bail(LFD_ECUDA); }
+  // initial state: v = 0 (Phi = 1), A = 0
+  e = cudaMemsetAsync(c->at<double>(L.vstage), 0, sizeof(double) * g.ndom * g.ng, c->stream);
+  if (e != cudaSuccess) { cuda_fail(c, e, "memset"); return bail(LFD_ECUDA); }
+  lfd_status s2 = launch(c, LFD_K_PHASE, "k_phase",
+                         [&] { return lfd::launch_phase(g, c->at<double>(L.vstage), c->phi(), c->stream); });
+  if (s2 != LFD_OK) return bail(s2);
+  s2 = set_A(c, nullptr);
+  if (s2 != LFD_OK) return bail(s2);
+  // Gram matrix G = dV B^H B (GEMM-1 with X = B, fixed-order reduction)
+  if (g.nproj > 0) {
+    lfd::Gemm1Args a1;
+    a1.A = c->proj; a1.X = c->proj; a1.part = c->at<double2>(L.part); a1.norms = nullptr;
+    a1.ndom = g.ndom; a1.mrows = g.nproj; a1.ncols = g.nproj; a1.nsplit = L.nsplit;
+    a1.ng = g.ng; a1.rows_per_split = L.rows_per_split;
+    a1.a_dom_stride = g.ng * g.nproj; a1.x_dom_stride = g.ng * g.nproj;
+    s2 = launch(c, LFD_K_NL_PROJ, "k_gemm1(G)", [&] { return lfd::launch_gemm1(a1, c->stream); });
+    if (s2 != LFD_OK) return bail(s2);
+    lfd::ReduceArgs r{};
+    r.part = a1.part; r.normp = nullptr; r.D = nullptr; r.out = c->at<double2>(L.G); r.cprime = nullptr; r.s = nullptr;
+    r.ndom = g.ndom; r.mrows = g.nproj; r.ncols = g.nproj; r.nsplit = L.nsplit; r.scale = g.dV; r.eps = 0;
+    s2 = launch(c, LFD_K_NL_REDUCE, "k_reduce(G)", [&] { return lfd::launch_reduce(r, c->stream); });
+    if (s2 != LFD_OK) return bail(s2);
+  }
+  *out = c;
+  return LFD_OK;
+}
+
+lfd_status lfd_set_potential(lfd_ctx* c, const double* vloc) {
+  LFD_TRY(check_ctx(c));
+  if (!vloc) return fail(c, LFD_EINVAL, "vloc is NULL");
+  DeviceGuard dg(c->device);
+  if (!is_device_ptr(vloc)) return fail(c, LFD_EINVAL, "vloc must be device memory (use lfd_set_potential_host)");
+  return launch(c, LFD_K_PHASE, "k_phase", [&] { return lfd::launch_phase(c->g, vloc, c->phi(), c->stream); });
+}
+
+lfd_status lfd_set_potential_host(lfd_ctx* c, const double* vloc_host) {
+  LFD_TRY(check_ctx(c));
+  if (!vloc_host) return fail(c, LFD_EINVAL, "vloc_host is NULL");
+  DeviceGuard dg(c->device);
+  double* stage = c->at<double>(c->L.vstage);
+  cudaError_t e = cudaMemcpyAsync(stage, vloc_host, sizeof(double) * c->g.ndom * c->g.ng, cudaMemcpyHostToDevice,
+                                  c->stream);
+  if (e != cudaSuccess) return cuda_fail(c, e, "H2D vloc");
+  return launch(c, LFD_K_PHASE, "k_phase", [&] { return lfd::launch_phase(c->g, stage, c->phi(), c->stream); });
+}
+
+lfd_status lfd_set_vector_potential(lfd_ctx* c, const double* A) {
+  LFD_TRY(check_ctx(c));
+  if (!A) return fail(c, LFD_EINVAL, "A is NULL");
+  for (int i = 0; i < 3 * c->g.ndom; ++i)
+    if (!std::isfinite(A[i])) return fail(c, LFD_EINVAL, "A must be finite");
+  DeviceGuard dg(c->device);
+  return set_A(c, A);
+}
+
+lfd_status lfd_step(lfd_ctx* c, int32_t nsteps) {
+  LFD_TRY(check_ctx(c));
+  if (nsteps < 0) return fail(c, LFD_EINVAL, "nsteps must be >= 0");
+  DeviceGuard dg(c->device);
+  for (int it = 0; it < nsteps; ++it) {
+    if (c->g.nproj > 0) LFD_TRY(nl_half(c));
+    LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin(x)",
+                   [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 0, 1, c->stream); }));
+    LFD_TRY(launch(c, LFD_K_KIN_Y, "k_kin(y)",
+                   [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 1, 0, c->stream); }));
+    LFD_TRY(launch(c, LFD_K_KIN_Z, "k_kin(z)",
+                   [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 2, 2, c->stream); }));
+    if (c->g.nproj > 0) LFD_TRY(nl_half(c));
+  }
+  return LFD_OK;
+}
+
+lfd_status lfd_density_current(lfd_ctx* c, double* rho, double* j, double* Jmac) {
+  LFD_TRY(check_ctx(c));
+  if (!rho) return fail(c, LFD_EINVAL, "rho is NULL");
+  DeviceGuard dg(c->device);
+  if (!is_device_ptr(rho) || (j && !is_device_ptr(j)) || (Jmac && !is_device_ptr(Jmac)))
+    return fail(c, LFD_EINVAL, "rho / j / Jmac must be device memory");
+  const Geometry& g = c->g;
+  const long long* base = c->at<long long>(c->L.base);  // [rho bases | j bases]
+  return density_into(c, rho, j, Jmac, base, (long long)g.ny * g.nz, g.nz, g.ng);
+}
+
+lfd_status lfd_density_current_global(lfd_ctx* c, double* rho_g, double* j_g, double* Jmac, const int32_t* off,
+                                      const int32_t* gdims) {
+  LFD_TRY(check_ctx(c));
+  if (!rho_g || !off || !gdims) return fail(c, LFD_EINVAL, "rho_g, dom_offset and gdims must be non-NULL");
+  const Geometry& g = c->g;
+  for (int i = 0; i < 3; ++i)
+    if (gdims[i] < 1) return fail(c, LFD_EINVAL, "gdims must be >= 1");
+  const int nd[3] = {g.nx, g.ny, g.nz};
+  for (int d = 0; d < g.ndom; ++d)
+    for (int i = 0; i < 3; ++i)
+      if (off[3 * d + i] < 0 || off[3 * d + i] + nd[i] > gdims[i])
+        return fail(c, LFD_EINVAL, "domain core outside the global grid");
+  DeviceGuard dg(c->device);
+  if (!is_device_ptr(rho_g) || (j_g && !is_device_ptr(j_g)) || (Jmac && !is_device_ptr(Jmac)))
+    return fail(c, LFD_EINVAL, "rho_g / j_g / Jmac must be device memory");
+  const long long GY = gdims[1], GZ = gdims[2];
+  const long long GN = (long long)gdims[0] * GY * GZ;
+  std::vector<long long> base(2 * g.ndom);
+  for (int d = 0; d < g.ndom; ++d) {
+    base[d] = ((long long)off[3 * d] * GY + off[3 * d + 1]) * GZ + off[3 * d + 2];
+    base[g.ndom + d] = base[d];
+  }
+  long long* bdev = c->at<long long>(c->L.base) + 2 * g.ndom;
+  if (base != c->gbase_host) {
+    cudaError_t e = cudaMemcpyAsync(bdev, base.data(), sizeof(long long) * base.size(), cudaMemcpyHostToDevice, c->stream);
+    if (e != cudaSuccess) return cuda_fail(c, e, "copy global bases");
+    c->gbase_host = base;
+  }
+  return density_into(c, rho_g, j_g, Jmac, bdev, GY * GZ, GZ, GN);
+}
+
+lfd_status lfd_density_current_host(lfd_ctx* c, double* rho_host, double* Jmac_host) {
+  LFD_TRY(check_ctx(c));
+  DeviceGuard dg(c->device);
+  const Geometry& g = c->g;
+  double* rs = c->at<double>(c->L.rhostage);
+  double* Js = c->at<double>(c->L.Jstage);
+  LFD_TRY(density_into(c, rs, nullptr, Js, c->at<long long>(c->L.base), (long long)g.ny * g.nz, g.nz, g.ng));
+  cudaError_t e;
+  if (rho_host) {
+    e = cudaMemcpyAsync(rho_host, rs, sizeof(double) * g.ndom * g.ng, cudaMemcpyDeviceToHost, c->stream);
+    if (e != cudaSuccess) return cuda_fail(c, e, "D2H rho");
+  }
+  if (Jmac_host) {
+    e = cudaMemcpyAsync(Jmac_host, Js, sizeof(double) * g.ndom * 3, cudaMemcpyDeviceToHost, c->stream);
+    if (e != cudaSuccess) return cuda_fail(c, e, "D2H J");
+  }
+  return LFD_OK;
+}
+
+lfd_status lfd_set_occupations(lfd_ctx* c, const double* occ) {
+  LFD_TRY(check_ctx(c));
+  if (!occ) return fail(c, LFD_EINVAL, "occ is NULL");
+  DeviceGuard dg(c->device);
+  cudaError_t e = cudaMemcpyAsync(c->at<double>(c->L.occ), occ, sizeof(double) * c->g.ndom * c->g.norb,
+                                  cudaMemcpyHostToDevice, c->stream);
+  if (e != cudaSuccess) return cuda_fail(c, e, "copy occ");
+  return LFD_OK;
+}
+
+lfd_status lfd_set_stream(lfd_ctx* c, void* stream) {
+  LFD_TRY(check_ctx(c));
+  c->stream = static_cast<cudaStream_t>(stream);
+  return LFD_OK;
+}
+
+lfd_status lfd_sync(lfd_ctx* c) {
+  LFD_TRY(check_ctx(c));
+  DeviceGuard dg(c->device);
+  cudaError_t e = cudaStreamSynchronize(c->stream);
+  if (e == cudaSuccess) e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(c, e, "asynchronous CUDA error");
+  return LFD_OK;
+}
+
+lfd_status lfd_launch_count(const lfd_ctx* c, uint64_t* count) {
+  LFD_TRY(check_ctx(c));
+  if (!count) return LFD_EINVAL;
+  *count = c->launches;
+  return LFD_OK;
+}
+
+lfd_status lfd_profile_enable(lfd_ctx* c, int32_t enable) {
+  LFD_TRY(check_ctx(c));
+  c->prof = enable != 0;
+  return LFD_OK;
+}
+
+lfd_status lfd_profile_read(lfd_ctx* c, double* ms, int64_t* launches) {
+  LFD_TRY(check_ctx(c));
+  DeviceGuard dg(c->device);
+  prof_flush(c);
+  for (int k = 0; k < LFD_K_COUNT; ++k) {
+    if (ms) ms[k] = c->prof_ms[k];
+    if (launches) launches[k] = c->prof_n[k];
+    c->prof_ms[k] = 0;
+    c->prof_n[k] = 0;
+  }
+  return LFD_OK;
+}
+
+const char* lfd_last_error(const lfd_ctx* c) {
+  if (c && is_live(c)) return c->err.c_str();
+  return g_tls_error.c_str();
+}
+
+lfd_status lfd_destroy(lfd_ctx* c) {
+  if (!c) return LFD_OK;
+  {
+    std::lock_guard<std::mutex> lk(g_live_mu);
+    if (!g_live.count(c)) {
+      g_tls_error = "lfd_destroy: context is not live";
+      return LFD_ESTATE;
+    }
+    g_live.erase(c);
+  }
+  {
+    DeviceGuard dg(c->device);
+    cudaStreamSynchronize(c->stream);
+    for (auto& s : c->slots) {
+      cudaEventDestroy(s.a);
+      cudaEventDestroy(s.b);
+    }
+  }
+  delete c;
+  return LFD_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,109 @@
+// lfd_internal.h -- shared (product-only) declarations of the sm_100a kernels and their launchers.
+// Not part of the public ABI (include/lfd.h). Nothing here is shared with oracle/.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace lfd {
+
+constexpr double kCLight = 137.035999084;  // R1: speed of light in atomic units
+
+// Per-domain stencil/current coefficients, rebuilt on the device from A (step a1 of SURVEY §8(a)).
+// For axis d and tau in {Delta/2 (p=0), Delta (p=1)} (p in {Delta_QD/2, Delta_QD}):
+//   alpha = e^{-i tau t_d} cos(tau t_d), up = sigma e^{+i theta_d}, dn = sigma e^{-i theta_d},
+//   onsite = e^{-i tau t_d},  sigma = i e^{-i tau t_d} sin(tau t_d),  t_d = 1/(2 h_d^2),
+//   theta_d = (A_d / c) h_d.   eth[d] = e^{i theta_d} (link current phase, R13).
+struct DomCoef {
+  double2 alpha[3][2];
+  double2 up[3][2];
+  double2 dn[3][2];
+  double2 onsite[3][2];
+  double2 eth[3];
+  double inv_h[3];
+  double pad_;
+};
+
+struct Geometry {
+  int ndom, nx, ny, nz, norb, nproj, bc;
+  double hx, hy, hz, dt, dV;
+  long long ng;  // points per domain
+};
+
+// ---- launchers (each returns the cudaError_t of the launch) -------------------------------------
+constexpr int kCoefMaxPerLaunch = 512;
+struct CoefParams {
+  double A[kCoefMaxPerLaunch][3];
+};
+cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int count, DomCoef* coef,
+                        cudaStream_t st);
+cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, cudaStream_t st);
+
+// One pass of K_axis over every line of every domain, optionally fused with a phase multiply
+// (phase_mode 1: Phi . psi before the sweep; 2: after).
+cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, const double2* phi,
+                       int axis, int phase_mode, cudaStream_t st);
+
+// GEMM-1 split-K: part[dom][split][mrows][ncols] (complex) = sum over the split's grid rows of
+// conj(A[r][m]) X[r][n]; if norms != nullptr also norms[dom][split][n] = sum |X[r][n]|^2.
+// A: [dom][ng][mrows], X: [dom][ng][ncols] complex.
+struct Gemm1Args {
+  const double2* A;
+  const double2* X;
+  double2* part;
+  double* norms;
+  int ndom, mrows, ncols, nsplit;
+  long long ng, rows_per_split;
+  long long a_dom_stride, x_dom_stride;  // in complex elements
+};
+cudaError_t launch_gemm1(const Gemm1Args& a, cudaStream_t st);
+int gemm1_smem_bytes();
+
+// Fixed-order split reduction: out[dom][m][n] = scale * D[m] * sum_split part (D == nullptr -> 1);
+// if cprime != nullptr also cprime = -i eps * out.  Column norms: s[dom][n] = scale * sum_split norms.
+struct ReduceArgs {
+  const double2* part;
+  const double* normp;
+  const double* D;  // [dom][mrows] or nullptr
+  double2* out;     // [dom][mrows][ncols]
+  double2* cprime;  // [dom][mrows][ncols] or nullptr
+  double* s;        // [dom][ncols] or nullptr
+  int ndom, mrows, ncols, nsplit;
+  double scale, eps;
+};
+cudaError_t launch_reduce(const ReduceArgs& a, cudaStream_t st);
+
+// n_s = sqrt( s_s / (s_s + eps^2 * (DC)_s^H G (DC)_s) )   (Gram closed form of the Eq. 6 norm, R11)
+cudaError_t launch_nlnorm(int ndom, int nproj, int norb, double eps, const double2* G,
+                          const double2* DC, const double* s, double* nfac, cudaStream_t st);
+
+// GEMM-2 in place: psi[dom][r][n] <- nfac[dom][n] * (psi[dom][r][n] + sum_m B[dom][r][m] Cp[dom][m][n])
+struct Gemm2Args {
+  double2* psi;
+  const double2* B;
+  const double2* Cp;
+  const double* nfac;
+  int ndom, nproj, norb;
+  long long ng;
+  int num_sms;
+};
+cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st);
+int gemm2_smem_bytes();
+cudaError_t gemm_set_attributes();
+
+// Density / current (a7). Output addressing: out index = base[dom] + x*sx + y*sy + z,
+// j component d at + d*jstride.
+struct DensArgs {
+  const double2* psi;
+  const DomCoef* coef;
+  const double* occ;
+  double* rho;
+  double* j;            // may be nullptr
+  double* jline;        // [dom][nx*ny][3] per-line partial sums of j (for J)
+  const long long* base;   // [dom] device array: rho offset of the domain's (0,0,0)
+  const long long* jbase;  // [dom] device array: j offset of the domain's (0,0,0), component 0
+  long long sx, sy, jstride;
+};
+cudaError_t launch_density(const Geometry& g, const DensArgs& a, cudaStream_t st);
+cudaError_t launch_jreduce(const Geometry& g, const double* jline, double* Jmac, cudaStream_t st);
+
+}  // namespace lfd

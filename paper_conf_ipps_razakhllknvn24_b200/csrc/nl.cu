@@ -1,0 +1,449 @@
+// nl.cu -- the "BLASified" nonlocal factor of Eq. 6/7/9 for sm_100a.
+//
+// Paper: Eq. 7 projects v_nl on the unoccupied KS orbitals at t = 0; §III-D casts it as
+// two BLAS-3 calls on the Ngrid x Norb matrix Psi (Eq. 9); Eq. 6 divides by the norm.
+// Readings R9-R12: C = dV B^H Psi; Psi <- (Psi - i (Delta/2) B diag(D) C) diag(n), with n_s restoring
+// each orbital's norm, computed here from the Gram closed form ||Psi'_s||^2 = s_s + eps^2 (DC)^H G (DC).
+//
+// Both GEMMs are FP64 complex and really are dense contractions, so they run on the FP64 tensor pipe:
+// warp-level DMMA (mma.sync m8n8k4 f64 -> SASS DMMA.8x8x4; tcgen05 has no f64 kind on sm_100a).
+// Complex products use 4 real DMMAs. Operand rows are staged into shared memory by the TMA engine
+// (cp.async.bulk, one bulk copy per row segment, completion on an mbarrier with expect_tx) through a
+// 4-stage ring; rows are padded (66 / 20 complex) so every DMMA fragment load (LDS.128) is
+// bank-conflict free.
+//  * GEMM-1 (k_gemm1): C partials over a fixed split of the grid rows (tall-skinny, K = Ngrid), plus
+//    the column norms s_s from the same operand fragments. Split partials are reduced in a fixed order
+//    (k_reduce) -- deterministic, no atomics.
+//  * GEMM-2 (k_gemm2): persistent CTAs over (domain, 64-row block, 64-column tile); the epilogue fuses
+//    Psi + B C' and the per-orbital renormalisation and writes Psi in place.
+#include "lfd_complex.cuh"
+#include "lfd_internal.h"
+
+namespace lfd {
+
+namespace {
+
+constexpr int kThreads = 256;  // 8 warps: 2 (M) x 4 (N), warp tile 32 x 16 complex
+constexpr int kTile = 64;      // CTA tile 64 x 64 complex
+constexpr int kStages = 4;
+
+// GEMM-1 stage: A rows [KC1][kLd1] (B rows, m along the row) and X rows [KC1][kLd1].
+constexpr int kKC1 = 16;
+constexpr int kLd1 = kTile + 2;
+constexpr int kStage1Bytes = 2 * kKC1 * kLd1 * 16;
+// GEMM-2 stage: A rows [64][kLdA2] (B rows, k = projector along the row) and C' rows [KC2][kLd1].
+constexpr int kKC2 = 16;
+constexpr int kLdA2 = kKC2 + 4;
+constexpr int kStage2Bytes = kTile * kLdA2 * 16 + kKC2 * kLd1 * 16;
+
+__device__ __forceinline__ void dmma(double& c0, double& c1, double a, double b) {
+  asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+      : "+d"(c0), "+d"(c1)
+      : "d"(a), "d"(b));
+}
+
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "LAB_WAIT:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra LAB_WAIT;\n"
+      "}\n" ::"r"(smem_addr(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_row(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_addr(dst)),
+      "l"(src), "r"(bytes), "r"(smem_addr(bar))
+      : "memory");
+}
+
+struct Frag {  // accumulators of one warp: 4 (M) x 2 (N) DMMA tiles, real and imaginary parts
+  double re[4][2][2];
+  double im[4][2][2];
+  __device__ __forceinline__ void zero() {
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 2; ++j) re[i][j][0] = re[i][j][1] = im[i][j][0] = im[i][j][1] = 0.0;
+  }
+};
+
+}  // namespace
+
+// ------------------------------------------------------------------------------------------------
+// GEMM-1: part[dom][split][m][n] = sum_{r in split} conj(A[r][m]) X[r][n];  norms[dom][split][n].
+// grid: (nsplit, mtiles*ntiles, ndom), block 256, dynamic smem kStages*kStage1Bytes + barriers.
+// ------------------------------------------------------------------------------------------------
+template <bool kTail>
+__device__ __forceinline__ void gemm1_chunk(const double2* As, const double2* Xs, int kv, int wm, int wn, int g,
+                                            int t, Frag& acc, double* nrm, bool do_norm) {
+#pragma unroll
+  for (int kk = 0; kk < kKC1; kk += 4) {
+    const int k = kk + t;
+    const bool ok = !kTail || (k < kv);
+    double2 a[4], x[2];
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi) a[mi] = ok ? As[k * kLd1 + wm * 32 + mi * 8 + g] : cz();
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) x[ni] = ok ? Xs[k * kLd1 + wn * 16 + ni * 8 + g] : cz();
+    if (do_norm) {
+#pragma unroll
+      for (int ni = 0; ni < 2; ++ni) nrm[ni] = fma(x[ni].x, x[ni].x, fma(x[ni].y, x[ni].y, nrm[ni]));
+    }
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi) {
+      const double br = a[mi].x, bi = a[mi].y, nbi = -a[mi].y;  // A = conj(B)^T: (br, -bi)
+#pragma unroll
+      for (int ni = 0; ni < 2; ++ni) {
+        dmma(acc.re[mi][ni][0], acc.re[mi][ni][1], br, x[ni].x);   // + br xr
+        dmma(acc.re[mi][ni][0], acc.re[mi][ni][1], bi, x[ni].y);   // + bi xi
+        dmma(acc.im[mi][ni][0], acc.im[mi][ni][1], br, x[ni].y);   // + br xi
+        dmma(acc.im[mi][ni][0], acc.im[mi][ni][1], nbi, x[ni].x);  // - bi xr
+      }
+    }
+  }
+}
+
+__global__ void __launch_bounds__(kThreads, 1) k_gemm1(Gemm1Args p) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kStages * kStage1Bytes);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int g = lane >> 2, t = lane & 3;
+  const int wm = warp >> 2, wn = warp & 3;
+  const int split = blockIdx.x;
+  const int ntn = (p.ncols + kTile - 1) / kTile;
+  const int mt = blockIdx.y / ntn, nt = blockIdx.y - (blockIdx.y / ntn) * ntn;
+  const int dom = blockIdx.z;
+  const int m0 = mt * kTile, n0 = nt * kTile;
+  const int mvalid = min(kTile, p.mrows - m0), nvalid = min(kTile, p.ncols - n0);
+  const long long kbeg = (long long)split * p.rows_per_split;
+  const long long kend = min(p.ng, kbeg + p.rows_per_split);
+  const int nchunks = (kend > kbeg) ? (int)((kend - kbeg + kKC1 - 1) / kKC1) : 0;
+  const double2* Ag = p.A + dom * p.a_dom_stride + m0;
+  const double2* Xg = p.X + dom * p.x_dom_stride + n0;
+
+  if (tid == 0) {
+    for (int s = 0; s < kStages; ++s) mbar_init(&bars[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+
+  auto issue = [&](int chunk, int stage) {  // warp 0 only
+    const long long r0 = kbeg + (long long)chunk * kKC1;
+    const int rows = (int)min((long long)kKC1, kend - r0);
+    double2* As = reinterpret_cast<double2*>(smem + stage * kStage1Bytes);
+    double2* Xs = As + kKC1 * kLd1;
+    if (lane == 0) mbar_expect_tx(&bars[stage], (uint32_t)(rows * (mvalid + nvalid) * 16));
+    __syncwarp();
+    if (lane < rows) {
+      tma_row(As + lane * kLd1, Ag + (r0 + lane) * p.mrows, mvalid * 16, &bars[stage]);
+    } else if (lane >= kKC1 && lane - kKC1 < rows) {
+      const int r = lane - kKC1;
+      tma_row(Xs + r * kLd1, Xg + (r0 + r) * p.ncols, nvalid * 16, &bars[stage]);
+    }
+  };
+
+  if (warp == 0)
+    for (int s = 0; s < kStages && s < nchunks; ++s) issue(s, s);
+
+  Frag acc;
+  acc.zero();
+  double nrm[2] = {0.0, 0.0};
+  const bool do_norm = (p.norms != nullptr) && (mt == 0) && (wm == 0);
+
+  for (int i = 0; i < nchunks; ++i) {
+    const int stage = i % kStages;
+    mbar_wait(&bars[stage], (uint32_t)((i / kStages) & 1));
+    const double2* As = reinterpret_cast<const double2*>(smem + stage * kStage1Bytes);
+    const double2* Xs = As + kKC1 * kLd1;
+    const int kv = (int)min((long long)kKC1, kend - (kbeg + (long long)i * kKC1));
+    if (kv == kKC1)
+      gemm1_chunk<false>(As, Xs, kv, wm, wn, g, t, acc, nrm, do_norm);
+    else
+      gemm1_chunk<true>(As, Xs, kv, wm, wn, g, t, acc, nrm, do_norm);
+    __syncthreads();
+    if (warp == 0 && i + kStages < nchunks) issue(i + kStages, stage);
+  }
+
+  // epilogue: split partials (fixed positions, reduced in order by k_reduce)
+  double2* out = p.part + (((long long)dom * p.nsplit + split) * p.mrows) * p.ncols;
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi) {
+    const int row = wm * 32 + mi * 8 + g;
+    if (row >= mvalid) continue;
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+      for (int c = 0; c < 2; ++c) {
+        const int col = wn * 16 + ni * 8 + 2 * t + c;
+        if (col < nvalid)
+          out[(long long)(m0 + row) * p.ncols + n0 + col] = make_double2(acc.re[mi][ni][c], acc.im[mi][ni][c]);
+      }
+  }
+  if (do_norm) {
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) {
+      double v = nrm[ni];
+      v += __shfl_xor_sync(0xffffffffu, v, 1);
+      v += __shfl_xor_sync(0xffffffffu, v, 2);
+      const int col = wn * 16 + ni * 8 + g;
+      if (t == 0 && col < nvalid)
+        p.norms[((long long)dom * p.nsplit + split) * p.ncols + n0 + col] = v;
+    }
+  }
+}
+
+int gemm1_smem_bytes() { return kStages * kStage1Bytes + kStages * 8; }
+int gemm2_smem_bytes() { return kStages * kStage2Bytes + kStages * 8; }
+
+cudaError_t launch_gemm1(const Gemm1Args& a, cudaStream_t st) {
+  const int tiles = ((a.mrows + kTile - 1) / kTile) * ((a.ncols + kTile - 1) / kTile);
+  dim3 grid(a.nsplit, tiles, a.ndom);
+  k_gemm1<<<grid, kThreads, gemm1_smem_bytes(), st>>>(a);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------------
+// Fixed-order split-K reduction. One thread per (dom, m, n); threads with m == 0 also reduce norms.
+// ------------------------------------------------------------------------------------------------
+__global__ void k_reduce(ReduceArgs p) {
+  const long long per_dom = (long long)p.mrows * p.ncols;
+  const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= per_dom * p.ndom) return;
+  const int dom = (int)(idx / per_dom);
+  const long long e = idx - dom * per_dom;
+  const int m = (int)(e / p.ncols), n = (int)(e - (long long)m * p.ncols);
+  const double2* src = p.part + (long long)dom * p.nsplit * per_dom + e;
+  double sr = 0.0, si = 0.0;
+#pragma unroll 8
+  for (int s = 0; s < p.nsplit; ++s) {
+    const double2 v = src[s * per_dom];
+    sr += v.x;
+    si += v.y;
+  }
+  const double f = p.scale * (p.D ? p.D[(long long)dom * p.mrows + m] : 1.0);
+  const double2 o = make_double2(sr * f, si * f);
+  p.out[idx] = o;
+  if (p.cprime) p.cprime[idx] = make_double2(p.eps * o.y, -p.eps * o.x);  // -i eps (D C)
+  if (p.s && m == 0) {
+    const double* ns = p.normp + (long long)dom * p.nsplit * p.ncols + n;
+    double acc = 0.0;
+    for (int s = 0; s < p.nsplit; ++s) acc += ns[(long long)s * p.ncols];
+    p.s[(long long)dom * p.ncols + n] = p.scale * acc;
+  }
+}
+
+cudaError_t launch_reduce(const ReduceArgs& a, cudaStream_t st) {
+  const long long n = (long long)a.ndom * a.mrows * a.ncols;
+  k_reduce<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(a);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------------
+// n_s = sqrt(s_s / (s_s + eps^2 Re[(DC)_s^H G (DC)_s])). Block = 8 warps = 8 columns; lanes over u.
+// ------------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_nlnorm(int nproj, int norb, double eps2, const double2* __restrict__ G,
+                                                const double2* __restrict__ DC, const double* __restrict__ s,
+                                                double* __restrict__ nfac) {
+  const int dom = blockIdx.y;
+  const int col = blockIdx.x * 8 + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (col >= norb) return;
+  const double2* Gd = G + (long long)dom * nproj * nproj;
+  const double2* Cd = DC + (long long)dom * nproj * norb;
+  double q = 0.0;
+  for (int u = lane; u < nproj; u += 32) {
+    double tr = 0.0, ti = 0.0;
+    const double2* Gu = Gd + (long long)u * nproj;
+    for (int v = 0; v < nproj; ++v) {
+      const double2 gv = Gu[v], c = Cd[(long long)v * norb + col];
+      tr = fma(gv.x, c.x, fma(-gv.y, c.y, tr));
+      ti = fma(gv.x, c.y, fma(gv.y, c.x, ti));
+    }
+    const double2 cu = Cd[(long long)u * norb + col];
+    q = fma(cu.x, tr, fma(cu.y, ti, q));  // Re(conj(cu) * t)
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
+  if (lane == 0) {
+    const double sv = s[(long long)dom * norb + col];
+    nfac[(long long)dom * norb + col] = sqrt(sv / (sv + eps2 * q));
+  }
+}
+
+cudaError_t launch_nlnorm(int ndom, int nproj, int norb, double eps, const double2* G, const double2* DC,
+                          const double* s, double* nfac, cudaStream_t st) {
+  dim3 grid((norb + 7) / 8, ndom);
+  k_nlnorm<<<grid, 256, 0, st>>>(nproj, norb, eps * eps, G, DC, s, nfac);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------------
+// GEMM-2 (persistent): psi[r][n] <- nfac[n] * (psi[r][n] + sum_m B[r][m] Cp[m][n]) for every
+// (dom, 64-row block, 64-column tile) work item; K = nproj in chunks of 16 through the TMA ring.
+// ------------------------------------------------------------------------------------------------
+template <bool kTail>
+__device__ __forceinline__ void gemm2_chunk(const double2* As, const double2* Cs, int kv, int wm, int wn, int g,
+                                            int t, Frag& acc) {
+#pragma unroll
+  for (int kk = 0; kk < kKC2; kk += 4) {
+    const int k = kk + t;
+    const bool ok = !kTail || (k < kv);
+    double2 a[4], c[2];
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi) a[mi] = ok ? As[(wm * 32 + mi * 8 + g) * kLdA2 + k] : cz();
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) c[ni] = ok ? Cs[k * kLd1 + wn * 16 + ni * 8 + g] : cz();
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi) {
+      const double ar = a[mi].x, ai = a[mi].y, nai = -a[mi].y;
+#pragma unroll
+      for (int ni = 0; ni < 2; ++ni) {
+        dmma(acc.re[mi][ni][0], acc.re[mi][ni][1], ar, c[ni].x);   // + ar cr
+        dmma(acc.re[mi][ni][0], acc.re[mi][ni][1], nai, c[ni].y);  // - ai ci
+        dmma(acc.im[mi][ni][0], acc.im[mi][ni][1], ar, c[ni].y);   // + ar ci
+        dmma(acc.im[mi][ni][0], acc.im[mi][ni][1], ai, c[ni].x);   // + ai cr
+      }
+    }
+  }
+}
+
+__global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kStages * kStage2Bytes);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int g = lane >> 2, t = lane & 3;
+  const int wm = warp >> 2, wn = warp & 3;
+  const int rblocks = (int)((p.ng + kTile - 1) / kTile);
+  const int ntn = (p.norb + kTile - 1) / kTile;
+  const long long items = (long long)p.ndom * rblocks * ntn;
+  const int nk = (p.nproj + kKC2 - 1) / kKC2;
+
+  if (tid == 0) {
+    for (int s = 0; s < kStages; ++s) mbar_init(&bars[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+
+  // This CTA's chunk sequence: items blockIdx.x, +gridDim.x, ...; nk chunks each.
+  const long long my_items = (items > blockIdx.x) ? (items - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+  const long long total = my_items * nk;
+
+  auto decode = [&](long long item, int& dom, long long& r0, int& n0) {
+    const long long per_dom = (long long)rblocks * ntn;
+    dom = (int)(item / per_dom);
+    const long long rem = item - dom * per_dom;
+    const long long rb = rem / ntn;
+    r0 = rb * kTile;
+    n0 = (int)(rem - rb * ntn) * kTile;
+  };
+
+  auto issue = [&](long long gc, int stage) {  // warp 0 only
+    const long long item = blockIdx.x + (gc / nk) * gridDim.x;
+    const int kc = (int)(gc % nk);
+    int dom, n0;
+    long long r0;
+    decode(item, dom, r0, n0);
+    const int rows = (int)min((long long)kTile, p.ng - r0);
+    const int k0 = kc * kKC2;
+    const int kv = min(kKC2, p.nproj - k0);
+    const int nvalid = min(kTile, p.norb - n0);
+    double2* As = reinterpret_cast<double2*>(smem + stage * kStage2Bytes);
+    double2* Cs = As + kTile * kLdA2;
+    if (lane == 0) mbar_expect_tx(&bars[stage], (uint32_t)((rows * kv + kv * nvalid) * 16));
+    __syncwarp();
+    const double2* Bg = p.B + (long long)dom * p.ng * p.nproj + k0;
+    for (int r = lane; r < rows; r += 32)
+      tma_row(As + r * kLdA2, Bg + (r0 + r) * p.nproj, kv * 16, &bars[stage]);
+    if (lane < kv)
+      tma_row(Cs + lane * kLd1, p.Cp + ((long long)dom * p.nproj + k0 + lane) * p.norb + n0, nvalid * 16,
+              &bars[stage]);
+  };
+
+  if (warp == 0)
+    for (int s = 0; s < kStages && s < total; ++s) issue(s, s);
+
+  long long gc = 0;
+  for (long long it = 0; it < my_items; ++it) {
+    const long long item = blockIdx.x + it * gridDim.x;
+    int dom, n0;
+    long long r0;
+    decode(item, dom, r0, n0);
+    // prefetch this tile of Psi (consumed in the epilogue; in flight during the K loop)
+    double2* psi = p.psi + (long long)dom * p.ng * p.norb;
+    double2 pv[4][2][2];
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi) {
+      const long long r = r0 + wm * 32 + mi * 8 + g;
+#pragma unroll
+      for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+        for (int c = 0; c < 2; ++c) {
+          const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
+          pv[mi][ni][c] = (r < p.ng && col < p.norb) ? psi[r * p.norb + col] : cz();
+        }
+    }
+    Frag acc;
+    acc.zero();
+    for (int kc = 0; kc < nk; ++kc, ++gc) {
+      const int stage = (int)(gc % kStages);
+      mbar_wait(&bars[stage], (uint32_t)((gc / kStages) & 1));
+      const double2* As = reinterpret_cast<const double2*>(smem + stage * kStage2Bytes);
+      const double2* Cs = As + kTile * kLdA2;
+      const int kv = min(kKC2, p.nproj - kc * kKC2);
+      if (kv == kKC2)
+        gemm2_chunk<false>(As, Cs, kv, wm, wn, g, t, acc);
+      else
+        gemm2_chunk<true>(As, Cs, kv, wm, wn, g, t, acc);
+      __syncthreads();
+      if (warp == 0 && gc + kStages < total) issue(gc + kStages, stage);
+    }
+    // epilogue: Psi <- n_s (Psi + B C')
+    const double* nf = p.nfac + (long long)dom * p.norb;
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+      for (int c = 0; c < 2; ++c) {
+        const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
+        if (col >= p.norb) continue;
+        const double f = nf[col];
+#pragma unroll
+        for (int mi = 0; mi < 4; ++mi) {
+          const long long r = r0 + wm * 32 + mi * 8 + g;
+          if (r < p.ng)
+            psi[r * p.norb + col] =
+                make_double2(f * (pv[mi][ni][c].x + acc.re[mi][ni][c]), f * (pv[mi][ni][c].y + acc.im[mi][ni][c]));
+        }
+      }
+  }
+}
+
+cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
+  const long long rblocks = (a.ng + kTile - 1) / kTile;
+  const long long items = (long long)a.ndom * rblocks * ((a.norb + kTile - 1) / kTile);
+  const int grid = (int)(items < a.num_sms ? items : a.num_sms);
+  k_gemm2<<<grid, kThreads, gemm2_smem_bytes(), st>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t gemm_set_attributes() {
+  cudaError_t e = cudaFuncSetAttribute(k_gemm1, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm1_smem_bytes());
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(k_gemm2, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm2_smem_bytes());
+}
+
+}  // namespace lfd

@@ -1,0 +1,272 @@
+"""Thin ctypes binding of the C ABI in include/lfd.h (argument marshalling only).
+
+Every entry point keeps the C name (``lfd_init``, ``lfd_step``, ...). Device buffers are torch CUDA
+tensors; their data pointers are passed straight to the library and the current torch stream is used
+as the context stream. There is no CPU fallback: if ``liblfd.so`` is missing or no sm_100 device is
+present, the calls raise.
+
+``Context`` is a convenience owner that allocates the workspace and keeps the borrowed tensors alive.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "liblfd.so")
+
+LFD_ABI_VERSION = 1
+LFD_BC_PERIODIC = 0
+LFD_BC_ZERO = 1
+STATUS = {0: "LFD_OK", -1: "LFD_EINVAL", -2: "LFD_ENOMEM", -3: "LFD_ECUDA", -4: "LFD_ESTATE",
+          -5: "LFD_EUNSUPPORTED"}
+KERNELS = ("coef", "phase", "kin_x", "kin_y", "kin_z", "nl_proj", "nl_reduce", "nl_norm", "nl_back",
+           "density", "jreduce")
+EXPORTS = ("lfd_workspace_size", "lfd_init", "lfd_set_potential", "lfd_set_potential_host",
+           "lfd_set_vector_potential", "lfd_step", "lfd_density_current", "lfd_density_current_global",
+           "lfd_density_current_host", "lfd_set_occupations", "lfd_set_stream", "lfd_sync",
+           "lfd_launch_count", "lfd_profile_enable", "lfd_profile_read", "lfd_last_error", "lfd_destroy")
+
+
+class lfd_config(C.Structure):
+    _fields_ = [("abi_version", C.c_int32), ("ndomains", C.c_int32), ("nx", C.c_int32), ("ny", C.c_int32),
+                ("nz", C.c_int32), ("hx", C.c_double), ("hy", C.c_double), ("hz", C.c_double),
+                ("bc", C.c_int32), ("norb", C.c_int32), ("nproj", C.c_int32), ("dt", C.c_double),
+                ("device", C.c_int32), ("flags", C.c_int32)]
+
+
+class LFDError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+_lib = None
+
+
+def load():
+    """Load liblfd.so (raises if it was not built -- there is no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: run `python -c 'import __graft_entry__ as g; g.build()'`")
+    lib = C.CDLL(LIB_PATH)
+    P, I32, D = C.c_void_p, C.c_int32, C.POINTER(C.c_double)
+    cfgp = C.POINTER(lfd_config)
+    sig = {
+        "lfd_workspace_size": [cfgp, C.POINTER(C.c_size_t)],
+        "lfd_init": [cfgp, P, P, P, P, P, C.c_size_t, P, C.POINTER(P)],
+        "lfd_set_potential": [P, P],
+        "lfd_set_potential_host": [P, P],
+        "lfd_set_vector_potential": [P, P],
+        "lfd_step": [P, I32],
+        "lfd_density_current": [P, P, P, P],
+        "lfd_density_current_global": [P, P, P, P, P, P],
+        "lfd_density_current_host": [P, P, P],
+        "lfd_set_occupations": [P, P],
+        "lfd_set_stream": [P, P],
+        "lfd_sync": [P],
+        "lfd_launch_count": [P, C.POINTER(C.c_uint64)],
+        "lfd_profile_enable": [P, I32],
+        "lfd_profile_read": [P, D, C.POINTER(C.c_int64)],
+        "lfd_destroy": [P],
+    }
+    for name, args in sig.items():
+        f = getattr(lib, name)
+        f.argtypes = args
+        f.restype = C.c_int
+    lib.lfd_last_error.argtypes = [P]
+    lib.lfd_last_error.restype = C.c_char_p
+    _lib = lib
+    return lib
+
+
+def _check(rc: int, ctx=None):
+    if rc != 0:
+        msg = load().lfd_last_error(ctx).decode()
+        raise LFDError(rc, msg)
+
+
+def _dptr(t) -> C.c_void_p | None:
+    if t is None:
+        return None
+    if not getattr(t, "is_cuda", False):
+        raise TypeError("expected a CUDA tensor")
+    if not t.is_contiguous():
+        raise TypeError("expected a contiguous tensor")
+    return C.c_void_p(t.data_ptr())
+
+
+def _hptr(a, dtype=np.float64):
+    """Host pointer of a numpy array or CPU tensor; returns (pointer, keepalive)."""
+    if a is None:
+        return None, None
+    if hasattr(a, "data_ptr") and not getattr(a, "is_cuda", False):
+        if not a.is_contiguous():
+            raise TypeError("expected a contiguous host tensor")
+        return C.c_void_p(a.data_ptr()), a
+    arr = np.ascontiguousarray(a, dtype=dtype)
+    return C.c_void_p(arr.ctypes.data), arr
+
+
+def _stream_ptr(stream=None):
+    import torch
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return C.c_void_p(s.cuda_stream)
+
+
+def make_config(ndomains, nx, ny, nz, hx, hy, hz, bc, norb, nproj, dt, device=0) -> lfd_config:
+    return lfd_config(LFD_ABI_VERSION, ndomains, nx, ny, nz, hx, hy, hz, bc, norb, nproj, dt, device, 0)
+
+
+# ---- 1:1 wrappers of the C entry points --------------------------------------------------------
+
+def lfd_workspace_size(cfg: lfd_config) -> int:
+    n = C.c_size_t(0)
+    _check(load().lfd_workspace_size(C.byref(cfg), C.byref(n)))
+    return n.value
+
+
+def lfd_init(cfg, psi, proj, dnl, occ, workspace, stream=None) -> C.c_void_p:
+    pd, _k1 = _hptr(dnl)
+    po, _k2 = _hptr(occ)
+    ctx = C.c_void_p()
+    _check(load().lfd_init(C.byref(cfg), _dptr(psi), _dptr(proj), pd, po, _dptr(workspace),
+                           workspace.numel() * workspace.element_size(), _stream_ptr(stream), C.byref(ctx)))
+    return ctx
+
+
+def lfd_set_potential(ctx, vloc):
+    _check(load().lfd_set_potential(ctx, _dptr(vloc)), ctx)
+
+
+def lfd_set_potential_host(ctx, vloc_host):
+    p, _k = _hptr(vloc_host)
+    _check(load().lfd_set_potential_host(ctx, p), ctx)
+
+
+def lfd_set_vector_potential(ctx, A):
+    p, _k = _hptr(A)
+    _check(load().lfd_set_vector_potential(ctx, p), ctx)
+
+
+def lfd_step(ctx, nsteps: int = 1):
+    _check(load().lfd_step(ctx, int(nsteps)), ctx)
+
+
+def lfd_density_current(ctx, rho, j=None, Jmac=None):
+    _check(load().lfd_density_current(ctx, _dptr(rho), _dptr(j), _dptr(Jmac)), ctx)
+
+
+def lfd_density_current_global(ctx, rho_g, j_g, Jmac, dom_offset, gdims):
+    po, _k1 = _hptr(dom_offset, np.int32)
+    pg, _k2 = _hptr(gdims, np.int32)
+    _check(load().lfd_density_current_global(ctx, _dptr(rho_g), _dptr(j_g), _dptr(Jmac), po, pg), ctx)
+
+
+def lfd_density_current_host(ctx, rho_host=None, Jmac_host=None):
+    pr, _k1 = _hptr(rho_host)
+    pj, _k2 = _hptr(Jmac_host)
+    _check(load().lfd_density_current_host(ctx, pr, pj), ctx)
+
+
+def lfd_set_occupations(ctx, occ):
+    p, _k = _hptr(occ)
+    _check(load().lfd_set_occupations(ctx, p), ctx)
+
+
+def lfd_set_stream(ctx, stream=None):
+    _check(load().lfd_set_stream(ctx, _stream_ptr(stream)), ctx)
+
+
+def lfd_sync(ctx):
+    _check(load().lfd_sync(ctx), ctx)
+
+
+def lfd_launch_count(ctx) -> int:
+    n = C.c_uint64(0)
+    _check(load().lfd_launch_count(ctx, C.byref(n)), ctx)
+    return n.value
+
+
+def lfd_profile_enable(ctx, enable: bool = True):
+    _check(load().lfd_profile_enable(ctx, 1 if enable else 0), ctx)
+
+
+def lfd_profile_read(ctx) -> dict:
+    ms = (C.c_double * len(KERNELS))()
+    n = (C.c_int64 * len(KERNELS))()
+    _check(load().lfd_profile_read(ctx, ms, n), ctx)
+    return {k: (ms[i], n[i]) for i, k in enumerate(KERNELS)}
+
+
+def lfd_last_error(ctx=None) -> str:
+    return load().lfd_last_error(ctx).decode()
+
+
+def lfd_destroy(ctx):
+    _check(load().lfd_destroy(ctx))
+
+
+# ---- convenience owner ---------------------------------------------------------------------------
+
+class Context:
+    """Owns the workspace and keeps psi / proj alive for the context's lifetime.
+
+    psi: CUDA complex128 tensor [ndom, nx, ny, nz, norb] (propagated in place);
+    proj: CUDA complex128 tensor [ndom, nx, ny, nz, nproj] or None; dnl [ndom, nproj]; occ [ndom, norb]
+    (host arrays). h = (hx, hy, hz).
+    """
+
+    def __init__(self, psi, proj, dnl, occ, h, dt, bc=LFD_BC_PERIODIC, stream=None):
+        import torch
+        if psi.dtype != torch.complex128 or psi.dim() != 5:
+            raise TypeError("psi must be complex128 [ndom, nx, ny, nz, norb]")
+        ndom, nx, ny, nz, norb = psi.shape
+        nproj = 0 if proj is None else proj.shape[-1]
+        self.cfg = make_config(ndom, nx, ny, nz, h[0], h[1], h[2], bc, norb, nproj, dt,
+                               device=psi.device.index or 0)
+        self.psi, self.proj = psi, proj
+        ws = lfd_workspace_size(self.cfg)
+        self.workspace = torch.empty(max(ws, 1), dtype=torch.uint8, device=psi.device)
+        self.ctx = lfd_init(self.cfg, psi, proj, None if nproj == 0 else dnl, occ, self.workspace, stream)
+        self.shape = (ndom, nx, ny, nz)
+
+    def set_potential(self, vloc):
+        if getattr(vloc, "is_cuda", False):
+            lfd_set_potential(self.ctx, vloc)
+        else:
+            lfd_set_potential_host(self.ctx, vloc)
+
+    def set_vector_potential(self, A):
+        lfd_set_vector_potential(self.ctx, A)
+
+    def step(self, n: int = 1):
+        lfd_step(self.ctx, n)
+
+    def density_current(self, want_j: bool = True):
+        import torch
+        nd, nx, ny, nz = self.shape
+        dev = self.psi.device
+        rho = torch.empty((nd, nx, ny, nz), dtype=torch.float64, device=dev)
+        j = torch.empty((nd, 3, nx, ny, nz), dtype=torch.float64, device=dev) if want_j else None
+        J = torch.empty((nd, 3), dtype=torch.float64, device=dev)
+        lfd_density_current(self.ctx, rho, j, J)
+        return rho, j, J
+
+    def sync(self):
+        lfd_sync(self.ctx)
+
+    def close(self):
+        if self.ctx is not None:
+            lfd_destroy(self.ctx)
+            self.ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

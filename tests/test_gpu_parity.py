@@ -1,0 +1,260 @@
+"""GPU-vs-oracle parity (the contract of SURVEY §8(c)): the CUDA path through the C ABI against the
+plain-C oracle on identical seeded inputs, element by element.
+
+Criterion (FP64, SURVEY §8(c) "GPU-vs-oracle parity criterion"):
+  ||Psi_gpu - Psi_ref||_F / ||Psi_ref||_F <= 1e-10, the same 2-norm ratio for rho and for j (j's
+  denominator floored at 1e-3 ||rho||_2 / min(h)), and |J_gpu - J_ref| <= 1e-10 mean|j_ref| (floored
+  likewise). Legitimate differences are roundoff only: DMMA / FMA contraction and summation order in the
+  K = Ngrid reductions, the Gram-closed-form norm (GPU) vs direct grid sums (oracle), CUDA sincos vs
+  libm (reading R22).
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+from lfd_workloads import make_inputs, workload
+from lfd_workloads.generate import midpoint_A
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-10
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def run_gpu(w, x, steps, A_fn, dnl=None):
+    torch = _torch()
+    from paper_conf_ipps_razakhllknvn24_b200 import Context
+    dev = torch.device("cuda:0")
+    psi = torch.from_numpy(x.psi0.copy()).to(dev)
+    proj = torch.from_numpy(x.proj).to(dev) if w.nproj > 0 else None
+    ctx = Context(psi, proj, x.dnl if dnl is None else dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc)
+    ctx.set_potential(torch.from_numpy(x.vloc).to(dev))
+    A = np.zeros((w.ndom, 3))
+    for n in range(steps):
+        A = A_fn(n)
+        ctx.set_vector_potential(A)
+        ctx.step(1)
+    ctx.set_vector_potential(A)
+    rho, j, J = ctx.density_current()
+    ctx.sync()
+    out = (psi.cpu().numpy(), rho.cpu().numpy().reshape(w.ndom, -1), j.cpu().numpy().reshape(w.ndom, 3, -1),
+           J.cpu().numpy())
+    ctx.close()
+    return out
+
+
+def run_ref(w, x, steps, A_fn, dnl=None):
+    from oracle import ref
+    cfg = ref.RefConfig(w.ndom, w.nx, w.ny, w.nz, w.hx, w.hy, w.hz, w.bc, w.norb, w.nproj, w.dt)
+    p = x.psi0.copy()
+    A = np.zeros((w.ndom, 3))
+    d = x.dnl if dnl is None else dnl
+    for n in range(steps):
+        A = A_fn(n)
+        ref.step(cfg, p, x.proj if w.nproj else None, d if w.nproj else None, x.vloc, A, 1)
+    rho, j, J = ref.density_current(cfg, p, x.occ, A)
+    return p, rho, j, J
+
+
+def rel(a, b):
+    return np.linalg.norm(a - b) / np.linalg.norm(b)
+
+
+def assert_parity(w, got, want, tol=TOL):
+    psi, rho, j, J = got
+    rpsi, rrho, rj, rJ = want
+    e_psi = rel(psi, rpsi)
+    e_rho = rel(rho, rrho)
+    floor = 1e-3 * np.linalg.norm(rrho) / min(w.hx, w.hy, w.hz)
+    e_j = np.linalg.norm(j - rj) / max(np.linalg.norm(rj), floor)
+    jscale = max(np.abs(rj).mean(), 1e-3 * np.abs(rrho).mean() / min(w.hx, w.hy, w.hz))
+    e_J = np.abs(J - rJ).max() / jscale
+    assert e_psi <= tol and e_rho <= tol and e_j <= tol and e_J <= tol, (e_psi, e_rho, e_j, e_J)
+    return e_psi, e_rho, e_j, e_J
+
+
+def laser(w):
+    return lambda n: midpoint_A(w, n)
+
+
+@pytest.mark.parametrize("name,steps", [("P0", 100), ("P1", 20), ("P2z", 20), ("P3", 5)])
+def test_step_parity_small_shapes(name, steps):
+    w = workload(name)
+    x = make_inputs(w, seed=7)
+    assert_parity(w, run_gpu(w, x, steps, laser(w)), run_ref(w, x, steps, laser(w)))
+
+
+def test_c1_as_specified_10_steps_A0():
+    """BASELINE configs[0]: 1 domain, 24^3, 22 occupied orbitals, 10 steps, A = 0."""
+    w = workload("C1")
+    x = make_inputs(w, seed=1)
+    A0 = lambda n: np.zeros((1, 3))
+    assert_parity(w, run_gpu(w, x, 10, A0), run_ref(w, x, 10, A0))
+
+
+def test_c1_contract_100_steps_laser_and_scissor():
+    """100 steps, A(t) != 0 and D != 0 (C1 shape, laser along a generic direction)."""
+    w = workload("C1").with_(laser=True, pol=(0.3, -0.4, 0.87), e0=0.02)
+    x = make_inputs(w, seed=2)
+    assert_parity(w, run_gpu(w, x, 100, laser(w)), run_ref(w, x, 100, laser(w)))
+
+
+def test_c3_eight_domain_batch():
+    """BASELINE configs[2]: 8 DC domains of the C1 shape batched in one context (20 steps)."""
+    w = workload("C3").with_(a_spread=0.1, vnoise=0.02)
+    x = make_inputs(w, seed=3)
+    assert_parity(w, run_gpu(w, x, 20, laser(w)), run_ref(w, x, 20, laser(w)))
+
+
+def test_local_only_nproj0():
+    w = workload("P0").with_(nproj=0)
+    x = make_inputs(w, seed=4)
+    assert_parity(w, run_gpu(w, x, 50, laser(w)), run_ref(w, x, 50, laser(w)))
+
+
+@pytest.mark.parametrize("dims,bc,norb,nproj", [((2, 4, 2), 0, 1, 1), ((3, 2, 5), 1, 1, 0), ((2, 2, 2), 1, 2, 1),
+                                                ((4, 6, 130), 0, 2, 3), ((130, 4, 2), 0, 3, 2)])
+def test_edge_shapes(dims, bc, norb, nproj):
+    w = workload("P0").with_(nx=dims[0], ny=dims[1], nz=dims[2], bc=bc, norb=norb, nocc=norb, nproj=nproj)
+    x = make_inputs(w, seed=5)
+    assert_parity(w, run_gpu(w, x, 7, laser(w)), run_ref(w, x, 7, laser(w)))
+
+
+def test_ragged_gemm_tiles():
+    """norb and nproj not multiples of the 64-wide tiles / 16-row chunks; several tiles each way."""
+    w = workload("P0").with_(nx=8, ny=10, nz=12, norb=70, nocc=35, nproj=67)
+    x = make_inputs(w, seed=6)
+    assert_parity(w, run_gpu(w, x, 3, laser(w)), run_ref(w, x, 3, laser(w)))
+
+
+def test_nonorthonormal_projectors_and_mixed_D():
+    """B need not be orthonormal (G = dV B^H B is used); D_u of both signs."""
+    w = workload("P3")
+    x = make_inputs(w, seed=8)
+    rng = np.random.default_rng(0)
+    x.proj = np.ascontiguousarray(x.proj * (0.5 + rng.random(x.proj.shape[-1])))
+    d = np.ascontiguousarray(rng.uniform(-0.3, 0.3, size=x.dnl.shape))
+    assert_parity(w, run_gpu(w, x, 5, laser(w), dnl=d), run_ref(w, x, 5, laser(w), dnl=d))
+
+
+def test_c2_full_size_one_step():
+    """BASELINE configs[1] at full size (70x70x72, 64 orbitals, 64 projectors, laser), same launch
+    configuration bench.py times: 2 steps compared element by element with the oracle (~20 s CPU)."""
+    w = workload("C2")
+    x = make_inputs(w, seed=1)
+    assert_parity(w, run_gpu(w, x, 2, laser(w)), run_ref(w, x, 2, laser(w)))
+
+
+def test_deterministic_bitwise():
+    w = workload("P3")
+    x = make_inputs(w, seed=9)
+    a = run_gpu(w, x, 3, laser(w))
+    b = run_gpu(w, x, 3, laser(w))
+    for u, v in zip(a, b):
+        assert np.array_equal(u, v)
+
+
+def test_norm_conservation_on_gpu():
+    w = workload("P0")
+    x = make_inputs(w, seed=10)
+    psi, *_ = run_gpu(w, x, 100, laser(w))
+    P = psi.reshape(-1, w.norb)
+    assert np.abs(w.dV * np.einsum("rs,rs->s", P.conj(), P).real - 1).max() < 1e-12
+
+
+def test_global_layout_and_host_variants():
+    torch = _torch()
+    from paper_conf_ipps_razakhllknvn24_b200 import Context, lfd
+    w = workload("P1")
+    x = make_inputs(w, seed=11)
+    dev = torch.device("cuda:0")
+    psi = torch.from_numpy(x.psi0.copy()).to(dev)
+    ctx = Context(psi, torch.from_numpy(x.proj).to(dev), x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt)
+    ctx.set_potential(x.vloc)  # host path
+    ctx.set_vector_potential(midpoint_A(w, 0))
+    ctx.step(2)
+    rho, j, J = ctx.density_current()
+    gd = np.array([w.nx * 2, w.ny, w.nz], dtype=np.int32)
+    off = np.array([[0, 0, 0], [w.nx, 0, 0]], dtype=np.int32)
+    rg = torch.zeros(tuple(gd), dtype=torch.float64, device=dev)
+    jg = torch.zeros((3,) + tuple(gd), dtype=torch.float64, device=dev)
+    Jg = torch.zeros((2, 3), dtype=torch.float64, device=dev)
+    lfd.lfd_density_current_global(ctx.ctx, rg, jg, Jg, off, gd)
+    rh = torch.empty((2, w.nx, w.ny, w.nz), dtype=torch.float64).pin_memory()
+    Jh = torch.empty((2, 3), dtype=torch.float64).pin_memory()
+    lfd.lfd_density_current_host(ctx.ctx, rh, Jh)
+    ctx.sync()
+    assert torch.equal(rg[: w.nx].cpu(), rho[0].cpu()) and torch.equal(rg[w.nx:].cpu(), rho[1].cpu())
+    assert torch.equal(jg[:, : w.nx].cpu(), j[0].cpu()) and torch.equal(jg[:, w.nx:].cpu(), j[1].cpu())
+    assert torch.equal(Jg.cpu(), J.cpu()) and torch.equal(Jh, J.cpu()) and torch.equal(rh, rho.cpu())
+    # device-path potential gives the same state as the host path
+    psi2 = torch.from_numpy(x.psi0.copy()).to(dev)
+    ctx2 = Context(psi2, torch.from_numpy(x.proj).to(dev), x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt)
+    ctx2.set_potential(torch.from_numpy(x.vloc).to(dev))
+    ctx2.set_vector_potential(midpoint_A(w, 0))
+    ctx2.step(2)
+    ctx2.sync()
+    assert torch.equal(psi, psi2)
+    ctx.close()
+    ctx2.close()
+
+
+def test_abi_errors_change_no_state():
+    torch = _torch()
+    from paper_conf_ipps_razakhllknvn24_b200 import Context, lfd
+    w = workload("P0")
+    x = make_inputs(w, seed=12)
+    dev = torch.device("cuda:0")
+    psi = torch.from_numpy(x.psi0.copy()).to(dev)
+    ctx = Context(psi, torch.from_numpy(x.proj).to(dev), x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt)
+    before = psi.clone()
+    with pytest.raises(lfd.LFDError) as e:
+        lfd.lfd_step(ctx.ctx, -1)
+    assert e.value.status == -1
+    with pytest.raises(lfd.LFDError):
+        lfd.lfd_set_vector_potential(ctx.ctx, np.full((1, 3), np.nan))
+    with pytest.raises(lfd.LFDError):  # host memory where device memory is required
+        lfd._check(lfd.load().lfd_set_potential(ctx.ctx, lfd.C.c_void_p(x.vloc.ctypes.data)), ctx.ctx)
+    ctx.sync()
+    assert torch.equal(psi, before)
+    # workspace too small
+    cfg = ctx.cfg
+    small = torch.empty(256, dtype=torch.uint8, device=dev)
+    with pytest.raises(lfd.LFDError) as e:
+        lfd.lfd_init(cfg, psi, torch.from_numpy(x.proj).to(dev), x.dnl, x.occ, small)
+    assert e.value.status == -2
+    # host psi rejected
+    with pytest.raises(lfd.LFDError):
+        occ = np.ascontiguousarray(x.occ)
+        lfd._check(lfd.load().lfd_init(lfd.C.byref(cfg), lfd.C.c_void_p(x.psi0.ctypes.data),
+                                       lfd.C.c_void_p(x.proj.ctypes.data), lfd.C.c_void_p(x.dnl.ctypes.data),
+                                       lfd.C.c_void_p(occ.ctypes.data), lfd.C.c_void_p(small.data_ptr()),
+                                       1 << 30, None, lfd.C.byref(lfd.C.c_void_p())))
+    h = ctx.ctx
+    ctx.close()
+    with pytest.raises(lfd.LFDError) as e:
+        lfd.lfd_step(h, 1)
+    assert e.value.status == -4  # LFD_ESTATE after destroy
+
+
+def test_launch_count_and_profile():
+    torch = _torch()
+    from paper_conf_ipps_razakhllknvn24_b200 import Context, lfd
+    w = workload("P0")
+    x = make_inputs(w, seed=13)
+    dev = torch.device("cuda:0")
+    psi = torch.from_numpy(x.psi0.copy()).to(dev)
+    ctx = Context(psi, torch.from_numpy(x.proj).to(dev), x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt)
+    n0 = lfd.lfd_launch_count(ctx.ctx)
+    lfd.lfd_profile_enable(ctx.ctx, True)
+    ctx.step(2)
+    prof = lfd.lfd_profile_read(ctx.ctx)
+    assert lfd.lfd_launch_count(ctx.ctx) - n0 == 2 * 11
+    assert prof["kin_x"][1] == 2 and prof["nl_proj"][1] == 4 and prof["nl_back"][1] == 4
+    assert all(v[0] >= 0 for v in prof.values())
+    ctx.close()
