@@ -56,7 +56,7 @@ lfd_status validate(const lfd_config* c, std::string& why) {
     return LFD_EINVAL;
   }
   if (c->norb < 1) { why = "norb must be >= 1"; return LFD_EINVAL; }
-  if (c->nproj < 0) { why = "nproj must be >= 0"; return LFD_EINVAL; }
+  if (c->nproj < 0 || c->nproj > 2048) { why = "nproj must be in [0, 2048]"; return LFD_EINVAL; }
   if (!(c->dt != 0.0) || !std::isfinite(c->dt)) { why = "dt must be finite and nonzero"; return LFD_EINVAL; }
   if (c->flags != 0) { why = "flags must be 0"; return LFD_EINVAL; }
   const long long ng = (long long)c->nx * c->ny * c->nz;
@@ -107,7 +107,7 @@ Layout layout(const Geometry& g, int num_sms) {
   L.cprime = take((size_t)nd * np * no * c16);
   L.s = take((size_t)nd * no * d8);
   L.nfac = take((size_t)nd * no * d8);
-  L.jline = take((size_t)nd * g.nx * g.ny * 3 * d8);
+  L.jline = take((size_t)nd * lfd::density_blocks(g) * 3 * d8);
   L.base = take((size_t)4 * nd * sizeof(long long));
   L.vstage = take((size_t)nd * g.ng * d8);
   L.rhostage = take((size_t)nd * g.ng * d8);

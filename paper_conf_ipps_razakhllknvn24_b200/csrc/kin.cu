@@ -69,7 +69,7 @@ cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, cudaS
 // One K_axis pass. Column c of domain blockIdx.y: outer = c / inner_len, inner = c % inner_len,
 // element offset = outer*outer_stride + inner; successive points of the line are pt_stride apart.
 template <bool kPeriodic, int kPhase>
-__global__ void __launch_bounds__(256) k_kin(double2* __restrict__ psi, const DomCoef* __restrict__ coef,
+__global__ void __launch_bounds__(256, 3) k_kin(double2* __restrict__ psi, const DomCoef* __restrict__ coef,
                                              const double2* __restrict__ phi, int axis, int n, int pt_stride,
                                              int inner_len, int outer_stride, int ncols, int norb,
                                              long long dom_stride, long long ng) {
@@ -99,13 +99,21 @@ __global__ void __launch_bounds__(256) k_kin(double2* __restrict__ psi, const Do
 
   const int P = (n + 1) >> 1;
   double2 E10 = cz(), O1 = cz(), prev_e1 = cz(), prev_oR = cz();
+  // two pairs in flight ahead of the one being combined (memory-level parallelism for the HBM stream)
   double2 na = ld(0), nb = (n > 1) ? ld(1) : cz();
+  double2 nc = cz(), nd = cz();
+  if (P > 1) {
+    nc = ld(2);
+    nd = (3 < n) ? ld(3) : cz();
+  }
   for (int p = 0; p < P; ++p) {
     const double2 a = na, b = nb;
     const bool pair = (2 * p + 1 < n);
-    if (p + 1 < P) {
-      na = ld(2 * p + 2);
-      nb = (2 * p + 3 < n) ? ld(2 * p + 3) : cz();
+    na = nc;
+    nb = nd;
+    if (p + 2 < P) {
+      nc = ld(2 * p + 4);
+      nd = (2 * p + 5 < n) ? ld(2 * p + 5) : cz();
     }
     double2 e0, e1 = cz();
     if (pair) {

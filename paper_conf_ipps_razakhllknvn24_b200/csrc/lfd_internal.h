@@ -98,12 +98,13 @@ struct DensArgs {
   const double* occ;
   double* rho;
   double* j;            // may be nullptr
-  double* jline;        // [dom][nx*ny][3] per-line partial sums of j (for J)
+  double* jline;        // [dom][density_blocks][3] per-CTA partial sums of j (for J)
   const long long* base;   // [dom] device array: rho offset of the domain's (0,0,0)
   const long long* jbase;  // [dom] device array: j offset of the domain's (0,0,0), component 0
   long long sx, sy, jstride;
 };
 cudaError_t launch_density(const Geometry& g, const DensArgs& a, cudaStream_t st);
+int density_blocks(const Geometry& g);
 cudaError_t launch_jreduce(const Geometry& g, const double* jline, double* Jmac, cudaStream_t st);
 
 }  // namespace lfd

@@ -71,16 +71,143 @@ __device__ __forceinline__ void tma_row(void* dst, const void* src, uint32_t byt
       : "memory");
 }
 
-struct Frag {  // accumulators of one warp: 4 (M) x 2 (N) DMMA tiles, real and imaginary parts
-  double re[4][2][2];
-  double im[4][2][2];
+#ifndef LFD_3M
+#define LFD_3M 1  // Gauss/3M complex product: 3 real DMMAs per complex tile instead of 4
+#endif
+
+// Accumulators of one warp: 4 (M) x 2 (N) DMMA tiles. With 3M, for A = a_r + i a_i and
+// B = b_r + i b_i the three real products are T1 = a_r b_r, T2 = a_i b_i, T3 = (a_r + a_i)(b_r + b_i),
+// so Re = T1 - T2 and Im = T3 - T1 - T2 (GEMM-2). GEMM-1 multiplies by conj(A): there T3 uses
+// (a_r - a_i), Re = T1 + T2, Im = T3 - T1 + T2. The flop count reported is always 8 per complex
+// multiply-add ("label any 3M 'effective' rate").
+__device__ __forceinline__ void l2_prefetch(const void* src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+}
+
+struct Frag {
+  double t1[4][2][2];
+  double t2[4][2][2];
+  double t3[4][2][2];
   __device__ __forceinline__ void zero() {
 #pragma unroll
     for (int i = 0; i < 4; ++i)
 #pragma unroll
-      for (int j = 0; j < 2; ++j) re[i][j][0] = re[i][j][1] = im[i][j][0] = im[i][j][1] = 0.0;
+      for (int j = 0; j < 2; ++j)
+#pragma unroll
+        for (int c = 0; c < 2; ++c) t1[i][j][c] = t2[i][j][c] = t3[i][j][c] = 0.0;
+  }
+  // GEMM-2 (plain product) results
+  __device__ __forceinline__ double re(int i, int j, int c) const {
+#if LFD_3M
+    return t1[i][j][c] - t2[i][j][c];
+#else
+    return t1[i][j][c];
+#endif
+  }
+  __device__ __forceinline__ double im(int i, int j, int c) const {
+#if LFD_3M
+    return t3[i][j][c] - t1[i][j][c] - t2[i][j][c];
+#else
+    return t2[i][j][c];
+#endif
+  }
+  // GEMM-1 (conjugated A) results
+  __device__ __forceinline__ double re_conj(int i, int j, int c) const {
+#if LFD_3M
+    return t1[i][j][c] + t2[i][j][c];
+#else
+    return t1[i][j][c];
+#endif
+  }
+  __device__ __forceinline__ double im_conj(int i, int j, int c) const {
+#if LFD_3M
+    return t3[i][j][c] - t1[i][j][c] + t2[i][j][c];
+#else
+    return t2[i][j][c];
+#endif
   }
 };
+
+// acc += a (4 row fragments) * c (2 column fragments), complex. Passes over the 8 tiles keep the
+// updates of one accumulator 8 independent DMMAs apart.
+__device__ __forceinline__ void mma_4x2(Frag& acc, const double2 (&a)[4], const double2 (&c)[2]) {
+#if LFD_3M
+  double as[4], cs[2];
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi) as[mi] = a[mi].x + a[mi].y;
+#pragma unroll
+  for (int ni = 0; ni < 2; ++ni) cs[ni] = c[ni].x + c[ni].y;
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t1[mi][ni][0], acc.t1[mi][ni][1], a[mi].x, c[ni].x);
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t2[mi][ni][0], acc.t2[mi][ni][1], a[mi].y, c[ni].y);
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t3[mi][ni][0], acc.t3[mi][ni][1], as[mi], cs[ni]);
+#else
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t1[mi][ni][0], acc.t1[mi][ni][1], a[mi].x, c[ni].x);  // + ar cr
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t2[mi][ni][0], acc.t2[mi][ni][1], a[mi].x, c[ni].y);  // + ar ci
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t1[mi][ni][0], acc.t1[mi][ni][1], -a[mi].y, c[ni].y);  // - ai ci
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t2[mi][ni][0], acc.t2[mi][ni][1], a[mi].y, c[ni].x);  // + ai cr
+#endif
+}
+
+// acc += conj(a) * x (GEMM-1 orientation: A = conj(B)^T).
+__device__ __forceinline__ void mma_conj_4x2(Frag& acc, const double2 (&a)[4], const double2 (&x)[2]) {
+#if LFD_3M
+  double as[4], xs[2];
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi) as[mi] = a[mi].x - a[mi].y;
+#pragma unroll
+  for (int ni = 0; ni < 2; ++ni) xs[ni] = x[ni].x + x[ni].y;
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t1[mi][ni][0], acc.t1[mi][ni][1], a[mi].x, x[ni].x);
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t2[mi][ni][0], acc.t2[mi][ni][1], a[mi].y, x[ni].y);
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t3[mi][ni][0], acc.t3[mi][ni][1], as[mi], xs[ni]);
+#else
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t1[mi][ni][0], acc.t1[mi][ni][1], a[mi].x, x[ni].x);  // + br xr
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t2[mi][ni][0], acc.t2[mi][ni][1], a[mi].x, x[ni].y);  // + br xi
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t1[mi][ni][0], acc.t1[mi][ni][1], a[mi].y, x[ni].y);  // + bi xi
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni) dmma(acc.t2[mi][ni][0], acc.t2[mi][ni][1], -a[mi].y, x[ni].x);  // - bi xr
+#endif
+}
 
 }  // namespace
 
@@ -104,17 +231,7 @@ __device__ __forceinline__ void gemm1_chunk(const double2* As, const double2* Xs
 #pragma unroll
       for (int ni = 0; ni < 2; ++ni) nrm[ni] = fma(x[ni].x, x[ni].x, fma(x[ni].y, x[ni].y, nrm[ni]));
     }
-#pragma unroll
-    for (int mi = 0; mi < 4; ++mi) {
-      const double br = a[mi].x, bi = a[mi].y, nbi = -a[mi].y;  // A = conj(B)^T: (br, -bi)
-#pragma unroll
-      for (int ni = 0; ni < 2; ++ni) {
-        dmma(acc.re[mi][ni][0], acc.re[mi][ni][1], br, x[ni].x);   // + br xr
-        dmma(acc.re[mi][ni][0], acc.re[mi][ni][1], bi, x[ni].y);   // + bi xi
-        dmma(acc.im[mi][ni][0], acc.im[mi][ni][1], br, x[ni].y);   // + br xi
-        dmma(acc.im[mi][ni][0], acc.im[mi][ni][1], nbi, x[ni].x);  // - bi xr
-      }
-    }
+    mma_conj_4x2(acc, a, x);
   }
 }
 
@@ -191,7 +308,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm1(Gemm1Args p) {
       for (int c = 0; c < 2; ++c) {
         const int col = wn * 16 + ni * 8 + 2 * t + c;
         if (col < nvalid)
-          out[(long long)(m0 + row) * p.ncols + n0 + col] = make_double2(acc.re[mi][ni][c], acc.im[mi][ni][c]);
+          out[(long long)(m0 + row) * p.ncols + n0 + col] = make_double2(acc.re_conj(mi, ni, c), acc.im_conj(mi, ni, c));
       }
   }
   if (do_norm) {
@@ -218,77 +335,115 @@ cudaError_t launch_gemm1(const Gemm1Args& a, cudaStream_t st) {
 }
 
 // ------------------------------------------------------------------------------------------------
-// Fixed-order split-K reduction. One thread per (dom, m, n); threads with m == 0 also reduce norms.
+// Fixed-order split-K reduction. Block = 32 consecutive output elements x 8 split groups: thread
+// (e, sg) sums splits sg, sg+8, ... of element e (coalesced over e), then the 8 group sums are added in
+// group order. Blocks past the element range reduce the column norms the same way. Deterministic.
 // ------------------------------------------------------------------------------------------------
-__global__ void k_reduce(ReduceArgs p) {
+__global__ void __launch_bounds__(256) k_reduce(ReduceArgs p, int eblocks) {
+  __shared__ double2 sh[8][32];
+  const int dom = blockIdx.y;
+  const int el = threadIdx.x & 31, sg = threadIdx.x >> 5;
   const long long per_dom = (long long)p.mrows * p.ncols;
-  const long long idx = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= per_dom * p.ndom) return;
-  const int dom = (int)(idx / per_dom);
-  const long long e = idx - dom * per_dom;
-  const int m = (int)(e / p.ncols), n = (int)(e - (long long)m * p.ncols);
-  const double2* src = p.part + (long long)dom * p.nsplit * per_dom + e;
-  double sr = 0.0, si = 0.0;
-#pragma unroll 8
-  for (int s = 0; s < p.nsplit; ++s) {
-    const double2 v = src[s * per_dom];
-    sr += v.x;
-    si += v.y;
-  }
-  const double f = p.scale * (p.D ? p.D[(long long)dom * p.mrows + m] : 1.0);
-  const double2 o = make_double2(sr * f, si * f);
-  p.out[idx] = o;
-  if (p.cprime) p.cprime[idx] = make_double2(p.eps * o.y, -p.eps * o.x);  // -i eps (D C)
-  if (p.s && m == 0) {
-    const double* ns = p.normp + (long long)dom * p.nsplit * p.ncols + n;
+  if ((int)blockIdx.x < eblocks) {
+    const long long e = (long long)blockIdx.x * 32 + el;
+    double sr = 0.0, si = 0.0;
+    if (e < per_dom) {
+      const double2* src = p.part + (long long)dom * p.nsplit * per_dom + e;
+      for (int s = sg; s < p.nsplit; s += 8) {
+        const double2 v = src[(long long)s * per_dom];
+        sr += v.x;
+        si += v.y;
+      }
+    }
+    sh[sg][el] = make_double2(sr, si);
+    __syncthreads();
+    if (sg == 0 && e < per_dom) {
+      double tr = 0.0, ti = 0.0;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        tr += sh[q][el].x;
+        ti += sh[q][el].y;
+      }
+      const int m = (int)(e / p.ncols);
+      const double f = p.scale * (p.D ? p.D[(long long)dom * p.mrows + m] : 1.0);
+      const double2 o = make_double2(tr * f, ti * f);
+      const long long idx = (long long)dom * per_dom + e;
+      p.out[idx] = o;
+      if (p.cprime) p.cprime[idx] = make_double2(p.eps * o.y, -p.eps * o.x);  // -i eps (D C)
+    }
+  } else {
+    const int n = ((int)blockIdx.x - eblocks) * 32 + el;
     double acc = 0.0;
-    for (int s = 0; s < p.nsplit; ++s) acc += ns[(long long)s * p.ncols];
-    p.s[(long long)dom * p.ncols + n] = p.scale * acc;
+    if (n < p.ncols) {
+      const double* ns = p.normp + (long long)dom * p.nsplit * p.ncols + n;
+      for (int s = sg; s < p.nsplit; s += 8) acc += ns[(long long)s * p.ncols];
+    }
+    sh[sg][el].x = acc;
+    __syncthreads();
+    if (sg == 0 && n < p.ncols) {
+      double t = 0.0;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) t += sh[q][el].x;
+      p.s[(long long)dom * p.ncols + n] = p.scale * t;
+    }
   }
 }
 
 cudaError_t launch_reduce(const ReduceArgs& a, cudaStream_t st) {
-  const long long n = (long long)a.ndom * a.mrows * a.ncols;
-  k_reduce<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(a);
+  const long long per_dom = (long long)a.mrows * a.ncols;
+  const int eblocks = (int)((per_dom + 31) / 32);
+  const int nblocks = a.s ? (a.ncols + 31) / 32 : 0;
+  dim3 grid(eblocks + nblocks, a.ndom);
+  k_reduce<<<grid, 256, 0, st>>>(a, eblocks);
   return cudaGetLastError();
 }
 
 // ------------------------------------------------------------------------------------------------
-// n_s = sqrt(s_s / (s_s + eps^2 Re[(DC)_s^H G (DC)_s])). Block = 8 warps = 8 columns; lanes over u.
+// n_s = sqrt(s_s / (s_s + eps^2 Re[(DC)_s^H G (DC)_s])). Block per (domain, orbital s): warps take
+// projector rows u, lanes run over v (coalesced rows of G), fixed-order warp and block reductions.
 // ------------------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(256) k_nlnorm(int nproj, int norb, double eps2, const double2* __restrict__ G,
                                                 const double2* __restrict__ DC, const double* __restrict__ s,
                                                 double* __restrict__ nfac) {
-  const int dom = blockIdx.y;
-  const int col = blockIdx.x * 8 + (threadIdx.x >> 5);
-  const int lane = threadIdx.x & 31;
-  if (col >= norb) return;
+  extern __shared__ double2 dcs[];  // DC[:, col]
+  __shared__ double wq[8];
+  const int dom = blockIdx.y, col = blockIdx.x;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const double2* Gd = G + (long long)dom * nproj * nproj;
   const double2* Cd = DC + (long long)dom * nproj * norb;
+  for (int u = threadIdx.x; u < nproj; u += blockDim.x) dcs[u] = Cd[(long long)u * norb + col];
+  __syncthreads();
   double q = 0.0;
-  for (int u = lane; u < nproj; u += 32) {
-    double tr = 0.0, ti = 0.0;
+  for (int u = warp; u < nproj; u += 8) {
     const double2* Gu = Gd + (long long)u * nproj;
-    for (int v = 0; v < nproj; ++v) {
-      const double2 gv = Gu[v], c = Cd[(long long)v * norb + col];
+    double tr = 0.0, ti = 0.0;
+    for (int v = lane; v < nproj; v += 32) {
+      const double2 gv = Gu[v], c = dcs[v];
       tr = fma(gv.x, c.x, fma(-gv.y, c.y, tr));
       ti = fma(gv.x, c.y, fma(gv.y, c.x, ti));
     }
-    const double2 cu = Cd[(long long)u * norb + col];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      tr += __shfl_xor_sync(0xffffffffu, tr, o);
+      ti += __shfl_xor_sync(0xffffffffu, ti, o);
+    }
+    const double2 cu = dcs[u];
     q = fma(cu.x, tr, fma(cu.y, ti, q));  // Re(conj(cu) * t)
   }
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
-  if (lane == 0) {
+  if (lane == 0) wq[warp] = q;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double tq = 0.0;
+    for (int w = 0; w < 8; ++w) tq += wq[w];
     const double sv = s[(long long)dom * norb + col];
-    nfac[(long long)dom * norb + col] = sqrt(sv / (sv + eps2 * q));
+    nfac[(long long)dom * norb + col] = sqrt(sv / (sv + eps2 * tq));
   }
 }
 
 cudaError_t launch_nlnorm(int ndom, int nproj, int norb, double eps, const double2* G, const double2* DC,
                           const double* s, double* nfac, cudaStream_t st) {
-  dim3 grid((norb + 7) / 8, ndom);
-  k_nlnorm<<<grid, 256, 0, st>>>(nproj, norb, eps * eps, G, DC, s, nfac);
+  dim3 grid(norb, ndom);
+  k_nlnorm<<<grid, 256, nproj * sizeof(double2), st>>>(nproj, norb, eps * eps, G, DC, s, nfac);
   return cudaGetLastError();
 }
 
@@ -308,17 +463,7 @@ __device__ __forceinline__ void gemm2_chunk(const double2* As, const double2* Cs
     for (int mi = 0; mi < 4; ++mi) a[mi] = ok ? As[(wm * 32 + mi * 8 + g) * kLdA2 + k] : cz();
 #pragma unroll
     for (int ni = 0; ni < 2; ++ni) c[ni] = ok ? Cs[k * kLd1 + wn * 16 + ni * 8 + g] : cz();
-#pragma unroll
-    for (int mi = 0; mi < 4; ++mi) {
-      const double ar = a[mi].x, ai = a[mi].y, nai = -a[mi].y;
-#pragma unroll
-      for (int ni = 0; ni < 2; ++ni) {
-        dmma(acc.re[mi][ni][0], acc.re[mi][ni][1], ar, c[ni].x);   // + ar cr
-        dmma(acc.re[mi][ni][0], acc.re[mi][ni][1], nai, c[ni].y);  // - ai ci
-        dmma(acc.im[mi][ni][0], acc.im[mi][ni][1], ar, c[ni].y);   // + ar ci
-        dmma(acc.im[mi][ni][0], acc.im[mi][ni][1], ai, c[ni].x);   // + ai cr
-      }
-    }
+    mma_4x2(acc, a, c);
   }
 }
 
@@ -426,7 +571,155 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
           const long long r = r0 + wm * 32 + mi * 8 + g;
           if (r < p.ng)
             psi[r * p.norb + col] =
-                make_double2(f * (pv[mi][ni][c].x + acc.re[mi][ni][c]), f * (pv[mi][ni][c].y + acc.im[mi][ni][c]));
+                make_double2(f * (pv[mi][ni][c].x + acc.re(mi, ni, c)), f * (pv[mi][ni][c].y + acc.im(mi, ni, c)));
+        }
+      }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// GEMM-2, full-K variant for nproj <= 64 (the paper-shaped case): the whole K = nproj fits one stage.
+// Each work item's 64 B rows arrive by 64 TMA bulk row copies into a 2-deep ring of padded tiles (row
+// stride = nproj rounded to 4, == 4 mod 8 complex, so the A-fragment LDS.128 are conflict free), and
+// C' for the current (domain, column tile) stays resident in shared memory. Items are ordered
+// (domain, column tile, row block) so C' is reloaded only when a CTA crosses into another
+// (domain, tile). kNP = 64 instantiates a fully unrolled K loop; kNP = 0 handles any nproj <= 64.
+// ------------------------------------------------------------------------------------------------
+constexpr int kFullStages = 2;
+constexpr int kFullLdaMax = 68;
+constexpr int kFullABytes = kTile * kFullLdaMax * 16;     // [64 rows][<=68] complex
+constexpr int kFullCBytes = kTile * kLd1 * 16;            // [<=64 proj][66] complex
+constexpr int kFullSmem = kFullStages * kFullABytes + kFullCBytes + 4 * 8;
+
+__host__ __device__ constexpr int full_lda(int np) { return ((np + 3) / 4 * 4) % 8 == 0 ? (np + 3) / 4 * 4 + 4 : (np + 3) / 4 * 4; }
+
+template <int kNP>
+__global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  double2* Cs = reinterpret_cast<double2*>(smem + kFullStages * kFullABytes);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kFullStages * kFullABytes + kFullCBytes);
+  uint64_t* cbar = bars + kFullStages;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int g = lane >> 2, t = lane & 3;
+  const int wm = warp >> 2, wn = warp & 3;
+  const int np = kNP > 0 ? kNP : p.nproj;
+  const int lda = full_lda(np);
+  const long long rblocks = (p.ng + kTile - 1) / kTile;
+  const int ntn = (p.norb + kTile - 1) / kTile;
+  const long long items = (long long)p.ndom * ntn * rblocks;
+  const long long my_items = (items > blockIdx.x) ? (items - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+  constexpr int kNK4 = kNP > 0 ? (kNP + 3) / 4 : 16;
+  const int nk4 = (np + 3) / 4;
+
+  if (tid == 0) {
+    for (int s = 0; s < kFullStages + 1; ++s) mbar_init(&bars[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+
+  auto decode = [&](long long j, int& dom, int& n0, long long& r0) {
+    const long long item = blockIdx.x + j * gridDim.x;
+    const long long per_dom = (long long)ntn * rblocks;
+    dom = (int)(item / per_dom);
+    const long long rem = item - dom * per_dom;
+    const int nt = (int)(rem / rblocks);
+    n0 = nt * kTile;
+    r0 = (rem - (long long)nt * rblocks) * kTile;
+  };
+  auto issue = [&](long long j, int stage) {  // warp 0
+    int dom, n0;
+    long long r0;
+    decode(j, dom, n0, r0);
+    const int rows = (int)min((long long)kTile, p.ng - r0);
+    if (lane == 0) mbar_expect_tx(&bars[stage], (uint32_t)(rows * np * 16));
+    __syncwarp();
+    double2* As = reinterpret_cast<double2*>(smem + stage * kFullABytes);
+    const double2* src = p.B + ((long long)dom * p.ng + r0) * np;
+    for (int r = lane; r < rows; r += 32) tma_row(As + r * lda, src + (long long)r * np, np * 16, &bars[stage]);
+  };
+
+  if (warp == 0)
+    for (int s = 0; s < kFullStages && s < my_items; ++s) issue(s, s);
+
+  int cur_dom = -1, cur_n0 = -1;
+  uint32_t cphase = 0;
+  for (long long j = 0; j < my_items; ++j) {
+    int dom, n0;
+    long long r0;
+    decode(j, dom, n0, r0);
+    if (dom != cur_dom || n0 != cur_n0) {  // (re)load C'[dom][:, n0:n0+64] (all warps are past Cs)
+      const int nvalid = min(kTile, p.norb - n0);
+      if (warp == 0) {
+        if (lane == 0) mbar_expect_tx(cbar, (uint32_t)(np * nvalid * 16));
+        __syncwarp();
+        for (int r = lane; r < np; r += 32)
+          tma_row(Cs + r * kLd1, p.Cp + ((long long)dom * np + r) * p.norb + n0, nvalid * 16, cbar);
+      }
+      mbar_wait(cbar, cphase);
+      cphase ^= 1;
+      cur_dom = dom;
+      cur_n0 = n0;
+    }
+    double2* psi = p.psi + (long long)dom * p.ng * p.norb;
+    // Psi rows of the NEXT item go to L2 now (the epilogue of this item reads rows prefetched during
+    // the previous one), keeping 64 registers free for fragment pipelining.
+    if (tid == 32 && j + 1 < my_items) {
+      int d1, n1;
+      long long q1;
+      decode(j + 1, d1, n1, q1);
+      const long long rows1 = min((long long)kTile, p.ng - q1);
+      l2_prefetch(p.psi + ((long long)d1 * p.ng + q1) * p.norb, (uint32_t)(rows1 * p.norb * 16));
+    }
+    if (tid == 32 && j == 0) {
+      const long long rows0 = min((long long)kTile, p.ng - r0);
+      l2_prefetch(psi + r0 * p.norb, (uint32_t)(rows0 * p.norb * 16));
+    }
+    const int stage = (int)(j % kFullStages);
+    mbar_wait(&bars[stage], (uint32_t)((j / kFullStages) & 1));
+    const double2* As = reinterpret_cast<const double2*>(smem + stage * kFullABytes);
+    Frag acc;
+    acc.zero();
+#pragma unroll
+    for (int kk = 0; kk < kNK4; ++kk) {
+      if (kNP == 0 && kk >= nk4) break;
+      const int k = kk * 4 + t;
+      const bool ok = (kNP > 0 && kNP % 4 == 0) || k < np;
+      double2 a[4], c[2];
+#pragma unroll
+      for (int mi = 0; mi < 4; ++mi) a[mi] = ok ? As[(wm * 32 + mi * 8 + g) * lda + k] : cz();
+#pragma unroll
+      for (int ni = 0; ni < 2; ++ni) c[ni] = ok ? Cs[k * kLd1 + wn * 16 + ni * 8 + g] : cz();
+      mma_4x2(acc, a, c);
+    }
+    __syncthreads();  // stage and Cs free
+    if (warp == 0 && j + kFullStages < my_items) issue(j + kFullStages, stage);
+    // epilogue: Psi <- n_s (Psi + B C'); all 16 loads (L2 hits, prefetched) are issued before any store
+    const double* nf = p.nfac + (long long)dom * p.norb;
+    double2 pv[4][2][2];
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi) {
+      const long long r = r0 + wm * 32 + mi * 8 + g;
+#pragma unroll
+      for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+        for (int c = 0; c < 2; ++c) {
+          const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
+          pv[mi][ni][c] = (r < p.ng && col < p.norb) ? psi[r * p.norb + col] : cz();
+        }
+    }
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+      for (int c = 0; c < 2; ++c) {
+        const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
+        if (col >= p.norb) continue;
+        const double f = nf[col];
+#pragma unroll
+        for (int mi = 0; mi < 4; ++mi) {
+          const long long r = r0 + wm * 32 + mi * 8 + g;
+          if (r < p.ng)
+            psi[r * p.norb + col] =
+                make_double2(f * (pv[mi][ni][c].x + acc.re(mi, ni, c)), f * (pv[mi][ni][c].y + acc.im(mi, ni, c)));
         }
       }
   }
@@ -436,12 +729,21 @@ cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
   const long long rblocks = (a.ng + kTile - 1) / kTile;
   const long long items = (long long)a.ndom * rblocks * ((a.norb + kTile - 1) / kTile);
   const int grid = (int)(items < a.num_sms ? items : a.num_sms);
-  k_gemm2<<<grid, kThreads, gemm2_smem_bytes(), st>>>(a);
+  if (a.nproj == kTile)
+    k_gemm2_fullk<kTile><<<grid, kThreads, kFullSmem, st>>>(a);
+  else if (a.nproj < kTile)
+    k_gemm2_fullk<0><<<grid, kThreads, kFullSmem, st>>>(a);
+  else
+    k_gemm2<<<grid, kThreads, gemm2_smem_bytes(), st>>>(a);
   return cudaGetLastError();
 }
 
 cudaError_t gemm_set_attributes() {
   cudaError_t e = cudaFuncSetAttribute(k_gemm1, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm1_smem_bytes());
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_gemm2_fullk<kTile>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_gemm2_fullk<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(k_gemm2, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm2_smem_bytes());
 }
