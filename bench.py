@@ -31,13 +31,38 @@ METRIC = json.load(open(os.path.join(ROOT, "BASELINE.json")))["metric"]
 UNIT = "orbital-gridpoint updates/s"
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FP64_PEAK_FILE = os.path.join(ROOT, "profiles", "r01_fp64_peaks.jsonl")
+NCU_SUMMARY = os.path.join(ROOT, "profiles", "latest_ncu_full_summary.csv")
+NCU_NAMES = {"nl_proj": "k_gemm1", "nl_back": "k_gemm2", "kin_x": "k_kin<1, 1>", "kin_y": "k_kin<1, 0>",
+             "kin_z": "k_kin<1, 2>", "density": "k_density"}
+
+
+def ncu_traffic(kernel):
+    """DRAM bytes per launch (read + write) of `kernel` from the committed ncu --set full summary."""
+    import csv
+    if not os.path.exists(NCU_SUMMARY) or kernel not in NCU_NAMES:
+        return None
+    rows = list(csv.reader(open(NCU_SUMMARY)))
+    hdr = rows[0]
+    try:
+        ir = next(i for i, h in enumerate(hdr) if h.startswith("dram__bytes_read.sum"))
+        iw = next(i for i, h in enumerate(hdr) if h.startswith("dram__bytes_write.sum"))
+    except StopIteration:
+        return None
+    scale = {"[byte]": 1.0, "[Kbyte]": 1e3, "[Mbyte]": 1e6, "[Gbyte]": 1e9}
+    vals = []
+    for r in rows[1:]:
+        if r[0].replace("void ", "").startswith(NCU_NAMES[kernel]):
+            sr = next((v for k, v in scale.items() if hdr[ir].endswith(k)), 1.0)
+            sw = next((v for k, v in scale.items() if hdr[iw].endswith(k)), 1.0)
+            vals.append(float(r[ir]) * sr + float(r[iw]) * sw)
+    return sum(vals) / len(vals) if vals else None
 
 
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
-    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--config", default=None, help="workload name (default C2; C4 under torchrun)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -138,7 +163,7 @@ def run_reference(args, w, rank, world):
     x = make_inputs(w, seed=args.seed)
     # Orbitals evolve independently under Eq. 6 (N and the local factor act column-wise), so a step on
     # a subset of orbitals is exactly that subset's share of the step: the sample is the first `ns`.
-    ns = min(w.norb, 8)
+    ns = min(w.norb, 4)
     cfg = ref.RefConfig(1, w.nx, w.ny, w.nz, w.hx, w.hy, w.hz, w.bc, ns, w.nproj, w.dt)
     p = np.ascontiguousarray(x.psi0[:1, ..., :ns])
     proj = np.ascontiguousarray(x.proj[:1]) if w.nproj else None
@@ -295,7 +320,9 @@ def main():
     dom = max((k for k in kernels if "achieved" in kernels[k]), key=lambda k: prof[k][0])
     d = kernels[dom]
     roofline = {"kernel": dom, "bound": d["bound"], "achieved": d["achieved"], "peak": d["peak"], "unit": d["unit"],
-                "frac": d["frac"], "traffic": None,
+                "frac": d["frac"], "traffic": ncu_traffic(dom),
+                "traffic_source": "profiles/latest_ncu_full_summary.csv (dram__bytes_read.sum + dram__bytes_write.sum "
+                                  "per launch, ncu --set full)",
                 "peak_source": pk["fp64_src"] if d["bound"] == "tensor" else pk["hbm_src"],
                 "flops_per_launch" if d["bound"] == "tensor" else "bytes_per_launch":
                     work[dom][1] if d["bound"] == "tensor" else work[dom][0]}

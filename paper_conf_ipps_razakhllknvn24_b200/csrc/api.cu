@@ -86,7 +86,22 @@ Layout layout(const Geometry& g, int num_sms) {
     const int t2 = ((np + 63) / 64) * ((np + 63) / 64);
     tiles = std::min(t1, t2) * nd;
   }
-  int nsplit = tiles > 0 ? std::max(1, num_sms / std::max(tiles, 1)) : 1;
+  // pick the split count with the best wave efficiency (CTAs / (waves * SMs)), preferring fewer
+  // splits unless more splits are clearly better; each split keeps >= 8 chunks of rows
+  int nsplit = 1;
+  if (tiles > 0) {
+    double best = 0.0;
+    const long long max_s = std::max<long long>(1, std::min<long long>(2LL * num_sms, g.ng / (8 * kKC1)));
+    for (long long s = 1; s <= max_s; ++s) {
+      const long long ctas = (long long)tiles * s;
+      const long long waves = (ctas + num_sms - 1) / num_sms;
+      const double eff = (double)ctas / (double)(waves * num_sms);
+      if (eff > best + 0.02) {
+        best = eff;
+        nsplit = (int)s;
+      }
+    }
+  }
   long long rps = (g.ng + nsplit - 1) / nsplit;
   rps = std::max<long long>(kKC1, (rps + kKC1 - 1) / kKC1 * kKC1);
   nsplit = (int)((g.ng + rps - 1) / rps);
@@ -338,6 +353,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   const Layout L = layout(g, prop.multiProcessorCount);
   if (ws_bytes < L.total) return fail(nullptr, LFD_ENOMEM, "workspace smaller than lfd_workspace_size()");
   cudaError_t e = lfd::gemm_set_attributes();
+  if (e == cudaSuccess) e = lfd::density_set_attributes();
   if (e != cudaSuccess) return cuda_fail(nullptr, e, "cudaFuncSetAttribute");
 
   lfd_ctx* c = new (std::nothrow) lfd_ctx();

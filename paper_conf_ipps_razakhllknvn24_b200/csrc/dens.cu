@@ -8,6 +8,7 @@
 // order by k_jreduce (deterministic, no atomics).
 #include "lfd_complex.cuh"
 #include "lfd_internal.h"
+#include "lfd_tma.cuh"
 
 namespace lfd {
 
@@ -111,6 +112,162 @@ __global__ void __launch_bounds__(kDensThreads) k_density(Geometry g, DensArgs a
   }
 }
 
+// ------------------------------------------------------------------------------------------------
+// TMA-staged variant (norb <= 64): the CTA walks its x-chunk plane by plane through a 3-slot ring of
+// shared-memory planes. A plane slot holds rows y0..y0+kTY (the last one is the y+1 halo row) x points
+// z0..z0+kTZ (the last is the z+1 halo point), all orbitals; each row segment is contiguous in HBM and
+// arrives by one cp.async.bulk. Iteration x reads slot(x) and slot(x+1) and then recycles slot(x) for
+// plane x+3, so each row is fetched from HBM about once and every neighbour access is an LDS.
+// ------------------------------------------------------------------------------------------------
+constexpr int kRingSlots = 3;
+constexpr int kMaxNorbTma = 64;
+constexpr int kPlanePts = (kTY + 1) * (kTZ + 1);
+
+__global__ void __launch_bounds__(kDensThreads) k_density_tma(Geometry g, DensArgs a, int ntz, int nty, int nxc) {
+  extern __shared__ __align__(128) unsigned char dsm[];
+  __shared__ __align__(8) uint64_t bars[kRingSlots];
+  __shared__ double jsh[3][kDensThreads / kSub];
+  const int norb = g.norb;
+  const int slot_elems = kPlanePts * norb;  // complex elements per slot
+  double2* ring = reinterpret_cast<double2*>(dsm);
+  const int dom = blockIdx.y;
+  int b = blockIdx.x;
+  const int tz = b % ntz; b /= ntz;
+  const int ty = b % nty; b /= nty;
+  const int xc = b;
+  const int q = threadIdx.x % kSub, pt = threadIdx.x / kSub;
+  const int py = pt / kTZ, pz = pt % kTZ;
+  const int y0 = ty * kTY, z0 = tz * kTZ;
+  const int y = y0 + py, z = z0 + pz;
+  const bool valid = (y < g.ny) && (z < g.nz);
+  const bool per = (g.bc == 0);
+  const bool has_y = valid && (per || y + 1 < g.ny);
+  const bool has_z = valid && (per || z + 1 < g.nz);
+  const double2* P = a.psi + (long long)dom * g.ng * norb;
+  const double* f = a.occ + (long long)dom * norb;
+  const DomCoef* cf = a.coef + dom;
+  const double2 ex = cf->eth[0], ey = cf->eth[1], ez = cf->eth[2];
+  const double ihx = cf->inv_h[0], ihy = cf->inv_h[1], ihz = cf->inv_h[2];
+  const int x0 = xc * nxc, x1 = min(g.nx, x0 + nxc);
+  const int nplanes = x1 - x0 + 1;  // planes x0 .. x1 (x1 is the x+1 neighbour of the last)
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kRingSlots; ++s) mbar_init(&bars[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+
+  // plane x0 + i -> slot i % 3; rows r = 0..kTY are y0 + r (periodic wrap), each kTZ+1 points from z0
+  // (the periodic z halo past nz wraps to z = 0 and needs a second copy). Issued by warp 0.
+  auto issue = [&](int i) {
+    const int xg = x0 + i;
+    const int slot = i % kRingSlots;
+    const bool have_plane = (xg < g.nx) || per;
+    const int xs = (xg < g.nx) ? xg : xg - g.nx;
+    double2* dst = ring + (long long)slot * slot_elems;
+    const int nz_in = min(kTZ + 1, g.nz - z0);       // contiguous part
+    const int nz_wrap = per ? (kTZ + 1 - nz_in) : 0;  // wrapped halo points (z = 0 ..)
+    int nrow = 0;
+    if (have_plane)
+      for (int r = 0; r <= kTY; ++r)
+        if (y0 + r < g.ny || per) ++nrow;
+    const uint32_t bytes = (uint32_t)(nrow * (nz_in + nz_wrap) * norb * 16);
+    if (threadIdx.x == 0) mbar_expect_tx(&bars[slot], bytes);
+    __syncwarp();
+    if (!have_plane) return;
+    const int lane = threadIdx.x & 31;
+    if (lane <= kTY) {
+      const int yy = y0 + lane;
+      if (yy < g.ny || per) {
+        const int ys = yy < g.ny ? yy : yy - g.ny;
+        const long long row0 = ((long long)xs * g.ny + ys) * g.nz;
+        double2* d = dst + (long long)lane * (kTZ + 1) * norb;
+        tma_row(d, P + (row0 + z0) * norb, (uint32_t)(nz_in * norb * 16), &bars[slot]);
+        if (nz_wrap > 0)
+          tma_row(d + (long long)nz_in * norb, P + row0 * norb, (uint32_t)(nz_wrap * norb * 16), &bars[slot]);
+      }
+    }
+  };
+
+  if (threadIdx.x < 32)
+    for (int i = 0; i < kRingSlots && i < nplanes; ++i) issue(i);
+
+  double jsx = 0.0, jsy = 0.0, jsz = 0.0;
+  for (int i = 0; i + 1 < nplanes; ++i) {
+    const int x = x0 + i;
+    mbar_wait(&bars[i % kRingSlots], (uint32_t)((i / kRingSlots) & 1));
+    mbar_wait(&bars[(i + 1) % kRingSlots], (uint32_t)(((i + 1) / kRingSlots) & 1));
+    const double2* S0 = ring + (long long)(i % kRingSlots) * slot_elems;
+    const double2* S1 = ring + (long long)((i + 1) % kRingSlots) * slot_elems;
+    const bool has_x = valid && (per || x + 1 < g.nx);
+    double rho = 0.0, pxr = 0.0, pxi = 0.0, pyr = 0.0, pyi = 0.0, pzr = 0.0, pzi = 0.0;
+    if (valid) {
+      const double2* own = S0 + (py * (kTZ + 1) + pz) * norb;
+      const double2* nx_ = S1 + (py * (kTZ + 1) + pz) * norb;
+      const double2* ny_ = S0 + ((py + 1) * (kTZ + 1) + pz) * norb;
+      const double2* nz_ = S0 + (py * (kTZ + 1) + pz + 1) * norb;
+#pragma unroll 4
+      for (int s = q; s < norb; s += kSub) {
+        const double fs = __ldg(f + s);
+        const double2 v = own[s];
+        rho = fma(fs, fma(v.x, v.x, v.y * v.y), rho);
+        if (has_x) {
+          const double2 w = cconjmul(v, nx_[s]);
+          pxr = fma(fs, w.x, pxr);
+          pxi = fma(fs, w.y, pxi);
+        }
+        if (has_y) {
+          const double2 w = cconjmul(v, ny_[s]);
+          pyr = fma(fs, w.x, pyr);
+          pyi = fma(fs, w.y, pyi);
+        }
+        if (has_z) {
+          const double2 w = cconjmul(v, nz_[s]);
+          pzr = fma(fs, w.x, pzr);
+          pzi = fma(fs, w.y, pzi);
+        }
+      }
+    }
+#pragma unroll
+    for (int o = kSub / 2; o > 0; o >>= 1) {
+      rho += __shfl_xor_sync(0xffffffffu, rho, o);
+      pxr += __shfl_xor_sync(0xffffffffu, pxr, o);
+      pxi += __shfl_xor_sync(0xffffffffu, pxi, o);
+      pyr += __shfl_xor_sync(0xffffffffu, pyr, o);
+      pyi += __shfl_xor_sync(0xffffffffu, pyi, o);
+      pzr += __shfl_xor_sync(0xffffffffu, pzr, o);
+      pzi += __shfl_xor_sync(0xffffffffu, pzi, o);
+    }
+    const double jx = has_x ? (ex.x * pxi + ex.y * pxr) * ihx : 0.0;
+    const double jy = has_y ? (ey.x * pyi + ey.y * pyr) * ihy : 0.0;
+    const double jz = has_z ? (ez.x * pzi + ez.y * pzr) * ihz : 0.0;
+    jsx += jx; jsy += jy; jsz += jz;
+    if (q == 0 && valid) {
+      const long long o = (long long)x * a.sx + (long long)y * a.sy + z;
+      a.rho[a.base[dom] + o] = rho;
+      if (a.j) {
+        const long long oj = a.jbase[dom] + o;
+        a.j[oj] = jx;
+        a.j[oj + a.jstride] = jy;
+        a.j[oj + 2 * a.jstride] = jz;
+      }
+    }
+    __syncthreads();  // slot i % 3 is free
+    if (threadIdx.x < 32 && i + kRingSlots < nplanes) issue(i + kRingSlots);
+  }
+  if (q == 0) {
+    jsh[0][pt] = jsx; jsh[1][pt] = jsy; jsh[2][pt] = jsz;
+  }
+  __syncthreads();
+  if (threadIdx.x < 3) {
+    double t = 0.0;
+    for (int k = 0; k < kDensThreads / kSub; ++k) t += jsh[threadIdx.x][k];
+    a.jline[((long long)dom * gridDim.x + blockIdx.x) * 3 + threadIdx.x] = t;
+  }
+}
+
+int density_smem_bytes(int norb) { return kRingSlots * kPlanePts * norb * 16; }
+
 int density_blocks(const Geometry& g) {
   const int ntz = (g.nz + kTZ - 1) / kTZ, nty = (g.ny + kTY - 1) / kTY, nxc = (g.nx + kXC - 1) / kXC;
   return ntz * nty * nxc;
@@ -119,8 +276,16 @@ int density_blocks(const Geometry& g) {
 cudaError_t launch_density(const Geometry& g, const DensArgs& a, cudaStream_t st) {
   const int ntz = (g.nz + kTZ - 1) / kTZ, nty = (g.ny + kTY - 1) / kTY;
   dim3 grid(density_blocks(g), g.ndom);
-  k_density<<<grid, kDensThreads, 0, st>>>(g, a, ntz, nty, kXC);
+  if (g.norb <= kMaxNorbTma)
+    k_density_tma<<<grid, kDensThreads, density_smem_bytes(g.norb), st>>>(g, a, ntz, nty, kXC);
+  else
+    k_density<<<grid, kDensThreads, 0, st>>>(g, a, ntz, nty, kXC);
   return cudaGetLastError();
+}
+
+cudaError_t density_set_attributes() {
+  return cudaFuncSetAttribute(k_density_tma, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              density_smem_bytes(kMaxNorbTma));
 }
 
 // J_d = (1/Ngrid) sum_lines jline (one block per domain, fixed-order tree over a fixed partition).

@@ -105,6 +105,7 @@ struct DensArgs {
 };
 cudaError_t launch_density(const Geometry& g, const DensArgs& a, cudaStream_t st);
 int density_blocks(const Geometry& g);
+cudaError_t density_set_attributes();
 cudaError_t launch_jreduce(const Geometry& g, const double* jline, double* Jmac, cudaStream_t st);
 
 }  // namespace lfd

@@ -18,6 +18,7 @@
 //    Psi + B C' and the per-orbital renormalisation and writes Psi in place.
 #include "lfd_complex.cuh"
 #include "lfd_internal.h"
+#include "lfd_tma.cuh"
 
 namespace lfd {
 
@@ -32,8 +33,9 @@ constexpr int kKC1 = 16;
 constexpr int kLd1 = kTile + 2;
 constexpr int kStage1Bytes = 2 * kKC1 * kLd1 * 16;
 // GEMM-2 stage: A rows [64][kLdA2] (B rows, k = projector along the row) and C' rows [KC2][kLd1].
-constexpr int kKC2 = 16;
-constexpr int kLdA2 = kKC2 + 4;
+constexpr int kKC2 = 32;
+constexpr int kLdA2 = kKC2 + 4;  // 36 == 4 mod 8: conflict-free A-fragment loads
+constexpr int kStages2 = 3;
 constexpr int kStage2Bytes = kTile * kLdA2 * 16 + kKC2 * kLd1 * 16;
 
 __device__ __forceinline__ void dmma(double& c0, double& c1, double a, double b) {
@@ -42,34 +44,6 @@ __device__ __forceinline__ void dmma(double& c0, double& c1, double a, double b)
       : "d"(a), "d"(b));
 }
 
-__device__ __forceinline__ uint32_t smem_addr(const void* p) {
-  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count));
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(bytes)
-               : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  asm volatile(
-      "{\n"
-      ".reg .pred p;\n"
-      "LAB_WAIT:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      "@!p bra LAB_WAIT;\n"
-      "}\n" ::"r"(smem_addr(bar)),
-      "r"(parity)
-      : "memory");
-}
-__device__ __forceinline__ void tma_row(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-          smem_addr(dst)),
-      "l"(src), "r"(bytes), "r"(smem_addr(bar))
-      : "memory");
-}
 
 #ifndef LFD_3M
 #define LFD_3M 1  // Gauss/3M complex product: 3 real DMMAs per complex tile instead of 4
@@ -80,10 +54,6 @@ __device__ __forceinline__ void tma_row(void* dst, const void* src, uint32_t byt
 // so Re = T1 - T2 and Im = T3 - T1 - T2 (GEMM-2). GEMM-1 multiplies by conj(A): there T3 uses
 // (a_r - a_i), Re = T1 + T2, Im = T3 - T1 + T2. The flop count reported is always 8 per complex
 // multiply-add ("label any 3M 'effective' rate").
-__device__ __forceinline__ void l2_prefetch(const void* src, uint32_t bytes) {
-  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
-}
-
 struct Frag {
   double t1[4][2][2];
   double t2[4][2][2];
@@ -325,7 +295,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm1(Gemm1Args p) {
 }
 
 int gemm1_smem_bytes() { return kStages * kStage1Bytes + kStages * 8; }
-int gemm2_smem_bytes() { return kStages * kStage2Bytes + kStages * 8; }
+int gemm2_smem_bytes() { return kStages2 * kStage2Bytes + kStages2 * 8; }
 
 cudaError_t launch_gemm1(const Gemm1Args& a, cudaStream_t st) {
   const int tiles = ((a.mrows + kTile - 1) / kTile) * ((a.ncols + kTile - 1) / kTile);
@@ -469,7 +439,7 @@ __device__ __forceinline__ void gemm2_chunk(const double2* As, const double2* Cs
 
 __global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
   extern __shared__ __align__(128) unsigned char smem[];
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kStages * kStage2Bytes);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kStages2 * kStage2Bytes);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int g = lane >> 2, t = lane & 3;
   const int wm = warp >> 2, wn = warp & 3;
@@ -479,7 +449,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
   const int nk = (p.nproj + kKC2 - 1) / kKC2;
 
   if (tid == 0) {
-    for (int s = 0; s < kStages; ++s) mbar_init(&bars[s], 1);
+    for (int s = 0; s < kStages2; ++s) mbar_init(&bars[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
@@ -520,7 +490,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
   };
 
   if (warp == 0)
-    for (int s = 0; s < kStages && s < total; ++s) issue(s, s);
+    for (int s = 0; s < kStages2 && s < total; ++s) issue(s, s);
 
   long long gc = 0;
   for (long long it = 0; it < my_items; ++it) {
@@ -528,8 +498,34 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
     int dom, n0;
     long long r0;
     decode(item, dom, r0, n0);
-    // prefetch this tile of Psi (consumed in the epilogue; in flight during the K loop)
     double2* psi = p.psi + (long long)dom * p.ng * p.norb;
+    if (tid == 32) {  // Psi rows of this item (first) and of the next one -> L2, read in the epilogue
+      if (it == 0) l2_prefetch(psi + r0 * p.norb, (uint32_t)(min((long long)kTile, p.ng - r0) * p.norb * 16));
+      if (it + 1 < my_items) {
+        int d1, n1;
+        long long q1;
+        decode(item + gridDim.x, d1, q1, n1);
+        l2_prefetch(p.psi + ((long long)d1 * p.ng + q1) * p.norb,
+                    (uint32_t)(min((long long)kTile, p.ng - q1) * p.norb * 16));
+      }
+    }
+    Frag acc;
+    acc.zero();
+    for (int kc = 0; kc < nk; ++kc, ++gc) {
+      const int stage = (int)(gc % kStages2);
+      mbar_wait(&bars[stage], (uint32_t)((gc / kStages2) & 1));
+      const double2* As = reinterpret_cast<const double2*>(smem + stage * kStage2Bytes);
+      const double2* Cs = As + kTile * kLdA2;
+      const int kv = min(kKC2, p.nproj - kc * kKC2);
+      if (kv == kKC2)
+        gemm2_chunk<false>(As, Cs, kv, wm, wn, g, t, acc);
+      else
+        gemm2_chunk<true>(As, Cs, kv, wm, wn, g, t, acc);
+      __syncthreads();
+      if (warp == 0 && gc + kStages2 < total) issue(gc + kStages2, stage);
+    }
+    // epilogue: Psi <- n_s (Psi + B C'); all 16 loads (L2 hits) are issued before any store
+    const double* nf = p.nfac + (long long)dom * p.norb;
     double2 pv[4][2][2];
 #pragma unroll
     for (int mi = 0; mi < 4; ++mi) {
@@ -542,23 +538,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
           pv[mi][ni][c] = (r < p.ng && col < p.norb) ? psi[r * p.norb + col] : cz();
         }
     }
-    Frag acc;
-    acc.zero();
-    for (int kc = 0; kc < nk; ++kc, ++gc) {
-      const int stage = (int)(gc % kStages);
-      mbar_wait(&bars[stage], (uint32_t)((gc / kStages) & 1));
-      const double2* As = reinterpret_cast<const double2*>(smem + stage * kStage2Bytes);
-      const double2* Cs = As + kTile * kLdA2;
-      const int kv = min(kKC2, p.nproj - kc * kKC2);
-      if (kv == kKC2)
-        gemm2_chunk<false>(As, Cs, kv, wm, wn, g, t, acc);
-      else
-        gemm2_chunk<true>(As, Cs, kv, wm, wn, g, t, acc);
-      __syncthreads();
-      if (warp == 0 && gc + kStages < total) issue(gc + kStages, stage);
-    }
-    // epilogue: Psi <- n_s (Psi + B C')
-    const double* nf = p.nfac + (long long)dom * p.norb;
 #pragma unroll
     for (int ni = 0; ni < 2; ++ni)
 #pragma unroll
@@ -583,13 +562,15 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
 // stride = nproj rounded to 4, == 4 mod 8 complex, so the A-fragment LDS.128 are conflict free), and
 // C' for the current (domain, column tile) stays resident in shared memory. Items are ordered
 // (domain, column tile, row block) so C' is reloaded only when a CTA crosses into another
-// (domain, tile). kNP = 64 instantiates a fully unrolled K loop; kNP = 0 handles any nproj <= 64.
+// (domain, tile). Stages are released per warp through full/empty mbarriers (warp 0 refills them),
+// so there is no CTA-wide barrier per item and each warp's epilogue overlaps the other warps' DMMAs.
+// kNP = 64 instantiates a fully unrolled K loop; kNP = 0 handles any nproj <= 64.
 // ------------------------------------------------------------------------------------------------
 constexpr int kFullStages = 2;
 constexpr int kFullLdaMax = 68;
 constexpr int kFullABytes = kTile * kFullLdaMax * 16;     // [64 rows][<=68] complex
 constexpr int kFullCBytes = kTile * kLd1 * 16;            // [<=64 proj][66] complex
-constexpr int kFullSmem = kFullStages * kFullABytes + kFullCBytes + 4 * 8;
+constexpr int kFullSmem = kFullStages * kFullABytes + kFullCBytes + 8 * 8;
 
 __host__ __device__ constexpr int full_lda(int np) { return ((np + 3) / 4 * 4) % 8 == 0 ? (np + 3) / 4 * 4 + 4 : (np + 3) / 4 * 4; }
 
@@ -597,8 +578,10 @@ template <int kNP>
 __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
   extern __shared__ __align__(128) unsigned char smem[];
   double2* Cs = reinterpret_cast<double2*>(smem + kFullStages * kFullABytes);
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kFullStages * kFullABytes + kFullCBytes);
-  uint64_t* cbar = bars + kFullStages;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kFullStages * kFullABytes + kFullCBytes);
+  uint64_t* empty = full + kFullStages;
+  uint64_t* cfull = empty + kFullStages;
+  uint64_t* cempty = cfull + 1;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int g = lane >> 2, t = lane & 3;
   const int wm = warp >> 2, wn = warp & 3;
@@ -612,12 +595,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
   const int nk4 = (np + 3) / 4;
 
   if (tid == 0) {
-    for (int s = 0; s < kFullStages + 1; ++s) mbar_init(&bars[s], 1);
+    for (int s = 0; s < kFullStages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], kThreads / 32);
+    }
+    mbar_init(cfull, 1);
+    mbar_init(cempty, kThreads / 32);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
 
-  auto decode = [&](long long j, int& dom, int& n0, long long& r0) {
+  // item j of this CTA -> (domain, column tile, row block); the key identifies the C' tile it needs
+  auto decode = [&](long long j, int& dom, int& n0, long long& r0) -> long long {
     const long long item = blockIdx.x + j * gridDim.x;
     const long long per_dom = (long long)ntn * rblocks;
     dom = (int)(item / per_dom);
@@ -625,57 +614,48 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
     const int nt = (int)(rem / rblocks);
     n0 = nt * kTile;
     r0 = (rem - (long long)nt * rblocks) * kTile;
+    return (long long)dom * ntn + nt;
   };
-  auto issue = [&](long long j, int stage) {  // warp 0
+  auto issue = [&](long long j) {  // warp 0: B-row tile of item j into stage j % 2 (+ Psi rows -> L2)
     int dom, n0;
     long long r0;
     decode(j, dom, n0, r0);
+    const int stage = (int)(j % kFullStages);
     const int rows = (int)min((long long)kTile, p.ng - r0);
-    if (lane == 0) mbar_expect_tx(&bars[stage], (uint32_t)(rows * np * 16));
+    if (lane == 0) {
+      mbar_expect_tx(&full[stage], (uint32_t)(rows * np * 16));
+      l2_prefetch(p.psi + ((long long)dom * p.ng + r0) * p.norb, (uint32_t)(rows * p.norb * 16));
+    }
     __syncwarp();
     double2* As = reinterpret_cast<double2*>(smem + stage * kFullABytes);
     const double2* src = p.B + ((long long)dom * p.ng + r0) * np;
-    for (int r = lane; r < rows; r += 32) tma_row(As + r * lda, src + (long long)r * np, np * 16, &bars[stage]);
+    for (int r = lane; r < rows; r += 32) tma_row(As + r * lda, src + (long long)r * np, np * 16, &full[stage]);
   };
 
   if (warp == 0)
-    for (int s = 0; s < kFullStages && s < my_items; ++s) issue(s, s);
+    for (long long s = 0; s < kFullStages && s < my_items; ++s) issue(s);
 
-  int cur_dom = -1, cur_n0 = -1;
-  uint32_t cphase = 0;
+  long long prev = -1;
+  int ver = 0;
   for (long long j = 0; j < my_items; ++j) {
     int dom, n0;
     long long r0;
-    decode(j, dom, n0, r0);
-    if (dom != cur_dom || n0 != cur_n0) {  // (re)load C'[dom][:, n0:n0+64] (all warps are past Cs)
-      const int nvalid = min(kTile, p.norb - n0);
+    const long long key = decode(j, dom, n0, r0);
+    if (key != prev) {  // C'[dom][:, n0:n0+64] for this and the following items of the same tile
       if (warp == 0) {
-        if (lane == 0) mbar_expect_tx(cbar, (uint32_t)(np * nvalid * 16));
+        if (ver > 0) mbar_wait(cempty, (uint32_t)((ver - 1) & 1));  // every warp is done with the old C'
+        const int nvalid = min(kTile, p.norb - n0);
+        if (lane == 0) mbar_expect_tx(cfull, (uint32_t)(np * nvalid * 16));
         __syncwarp();
         for (int r = lane; r < np; r += 32)
-          tma_row(Cs + r * kLd1, p.Cp + ((long long)dom * np + r) * p.norb + n0, nvalid * 16, cbar);
+          tma_row(Cs + r * kLd1, p.Cp + ((long long)dom * np + r) * p.norb + n0, nvalid * 16, cfull);
       }
-      mbar_wait(cbar, cphase);
-      cphase ^= 1;
-      cur_dom = dom;
-      cur_n0 = n0;
-    }
-    double2* psi = p.psi + (long long)dom * p.ng * p.norb;
-    // Psi rows of the NEXT item go to L2 now (the epilogue of this item reads rows prefetched during
-    // the previous one), keeping 64 registers free for fragment pipelining.
-    if (tid == 32 && j + 1 < my_items) {
-      int d1, n1;
-      long long q1;
-      decode(j + 1, d1, n1, q1);
-      const long long rows1 = min((long long)kTile, p.ng - q1);
-      l2_prefetch(p.psi + ((long long)d1 * p.ng + q1) * p.norb, (uint32_t)(rows1 * p.norb * 16));
-    }
-    if (tid == 32 && j == 0) {
-      const long long rows0 = min((long long)kTile, p.ng - r0);
-      l2_prefetch(psi + r0 * p.norb, (uint32_t)(rows0 * p.norb * 16));
+      mbar_wait(cfull, (uint32_t)(ver & 1));
+      ++ver;
+      prev = key;
     }
     const int stage = (int)(j % kFullStages);
-    mbar_wait(&bars[stage], (uint32_t)((j / kFullStages) & 1));
+    mbar_wait(&full[stage], (uint32_t)((j / kFullStages) & 1));
     const double2* As = reinterpret_cast<const double2*>(smem + stage * kFullABytes);
     Frag acc;
     acc.zero();
@@ -691,9 +671,17 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
       for (int ni = 0; ni < 2; ++ni) c[ni] = ok ? Cs[k * kLd1 + wn * 16 + ni * 8 + g] : cz();
       mma_4x2(acc, a, c);
     }
-    __syncthreads();  // stage and Cs free
-    if (warp == 0 && j + kFullStages < my_items) issue(j + kFullStages, stage);
+    // Release the stage (and C' after its last item) per warp: no CTA-wide barrier, so one warp's
+    // epilogue overlaps the other warps' DMMA work.
+    __syncwarp();
+    if (lane == 0) {
+      mbar_arrive(&empty[stage]);
+      int d1, n1;
+      long long q1;
+      if (j + 1 >= my_items || decode(j + 1, d1, n1, q1) != key) mbar_arrive(cempty);
+    }
     // epilogue: Psi <- n_s (Psi + B C'); all 16 loads (L2 hits, prefetched) are issued before any store
+    double2* psi = p.psi + (long long)dom * p.ng * p.norb;
     const double* nf = p.nfac + (long long)dom * p.norb;
     double2 pv[4][2][2];
 #pragma unroll
@@ -722,6 +710,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
                 make_double2(f * (pv[mi][ni][c].x + acc.re(mi, ni, c)), f * (pv[mi][ni][c].y + acc.im(mi, ni, c)));
         }
       }
+    // warp 0 refills this stage with item j + 2 once every warp has released it
+    if (warp == 0 && j + kFullStages < my_items) {
+      mbar_wait(&empty[stage], (uint32_t)((j / kFullStages) & 1));
+      issue(j + kFullStages);
+    }
   }
 }
 
