@@ -26,6 +26,10 @@
  *   lfd_ref_nl_half          pinned: norm closed form; Gram closed form; BLAS (numpy) for C.
  *   lfd_ref_step             pinned: norm / orthonormality conservation; gauge covariance.
  *   lfd_ref_density_current  pinned: plane-wave closed forms; sum rule; J = dE_kin/dA / V.
+ *   lfd_ref_energy           pinned: plane-wave closed forms (kinetic, local = f mean(v)); nonlocal on
+ *                            projector columns = f D_u; O(dt^2) energy drift of the step at A = D = 0.
+ *   lfd_ref_remap_occ        pinned: onto the grid basis it equals rho dV; on the t = 0 basis it gives
+ *                            back f; sum rule over a complete basis.
  *   Faithfulness to the paper's own printed numbers: parity unpinned (the paper prints none).
  */
 #include <complex.h>
@@ -338,4 +342,81 @@ double lfd_ref_kinetic_energy(const lfd_ref_config* c, const double complex* psi
         }
   }
   return e;
+}
+
+/* Public (calc_energy, P:212 / Fig. 5): energy of every domain,
+ * E = sum_s f_s <psi_s| h |psi_s> with h = T(A) + v_loc + v_nl of Eq. 5:
+ *   E[4*dm+0] = kinetic (lfd_ref_kinetic_energy, the FD Peierls form of the propagator),
+ *   E[4*dm+1] = local   = dV sum_r v_r sum_s f_s |psi_rs|^2          (v_loc applies point by point)
+ *   E[4*dm+2] = nonlocal = sum_s f_s sum_u D_u |C_us|^2,  C_us = dV sum_r conj(B_ru) psi_rs
+ *               (<psi| Delta_sci sum_u |B_u><B_u| |psi>, Eq. 7 P:68 with D_u = Delta_sci; R9)
+ *   E[4*dm+3] = total. proj/dnl may be NULL iff nproj == 0. */
+int lfd_ref_energy(const lfd_ref_config* c, const double complex* psi, const double* occ, const double* vloc,
+                   const double* A, const double complex* proj, const double* dnl, double* E) {
+  if (ref_check(c) || !psi || !occ || !vloc || !A || !E) return -1;
+  if (c->nproj > 0 && (!proj || !dnl)) return -1;
+  const size_t ng = (size_t)c->nx * c->ny * c->nz;
+  const int no = c->norb, np = c->nproj;
+  const double dV = c->hx * c->hy * c->hz;
+  lfd_ref_config one = *c;
+  one.ndom = 1;
+  for (int dm = 0; dm < c->ndom; ++dm) {
+    const double complex* p = psi + (size_t)dm * ng * no;
+    const double* f = occ + (size_t)dm * no;
+    const double* v = vloc + (size_t)dm * ng;
+    double ekin = lfd_ref_kinetic_energy(&one, p, f, A + 3 * dm);
+    double eloc = 0.0;
+    for (size_t r = 0; r < ng; ++r) {
+      double rho = 0.0;
+      for (int s = 0; s < no; ++s) rho += f[s] * (creal(p[r * no + s]) * creal(p[r * no + s]) +
+                                                  cimag(p[r * no + s]) * cimag(p[r * no + s]));
+      eloc += v[r] * rho;
+    }
+    eloc *= dV;
+    double enl = 0.0;
+    if (np > 0) {
+      const double complex* b = proj + (size_t)dm * ng * np;
+      const double* d = dnl + (size_t)dm * np;
+      for (int u = 0; u < np; ++u)
+        for (int s = 0; s < no; ++s) {
+          double complex cus = 0.0;
+          for (size_t r = 0; r < ng; ++r) cus += conj(b[r * np + u]) * p[r * no + s];
+          cus *= dV;
+          enl += f[s] * d[u] * (creal(cus) * creal(cus) + cimag(cus) * cimag(cus));
+        }
+    }
+    E[4 * dm + 0] = ekin;
+    E[4 * dm + 1] = eloc;
+    E[4 * dm + 2] = enl;
+    E[4 * dm + 3] = ekin + eloc + enl;
+  }
+  return 0;
+}
+
+/* Public (remap_occ, P:58 / P:212): the shadow-dynamics handshake maps the
+ * propagated orbitals back to occupation numbers of a reference basis (reading: the KS orbitals at
+ * t = 0), out[dm][k] = sum_s f_s |<ref_k | psi_s>|^2 = sum_s f_s |dV sum_r conj(ref_rk) psi_rs|^2.
+ * ref [ndom][nx][ny][nz][nref] complex128. */
+int lfd_ref_remap_occ(const lfd_ref_config* c, const double complex* psi, const double* occ,
+                      const double complex* ref, int nref, double* out) {
+  if (ref_check(c) || !psi || !occ || !ref || nref < 1 || !out) return -1;
+  const size_t ng = (size_t)c->nx * c->ny * c->nz;
+  const int no = c->norb;
+  const double dV = c->hx * c->hy * c->hz;
+  for (int dm = 0; dm < c->ndom; ++dm) {
+    const double complex* p = psi + (size_t)dm * ng * no;
+    const double complex* q = ref + (size_t)dm * ng * nref;
+    const double* f = occ + (size_t)dm * no;
+    for (int k = 0; k < nref; ++k) {
+      double acc = 0.0;
+      for (int s = 0; s < no; ++s) {
+        double complex ov = 0.0;
+        for (size_t r = 0; r < ng; ++r) ov += conj(q[r * nref + k]) * p[r * no + s];
+        ov *= dV;
+        acc += f[s] * (creal(ov) * creal(ov) + cimag(ov) * cimag(ov));
+      }
+      out[(size_t)dm * nref + k] = acc;
+    }
+  }
+  return 0;
 }

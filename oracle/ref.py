@@ -68,6 +68,10 @@ def lib():
         _lib.lfd_ref_density_current.argtypes = [cfgp, P, P, P, P, P, P]
         _lib.lfd_ref_kinetic_energy.argtypes = [cfgp, P, P, P]
         _lib.lfd_ref_kinetic_energy.restype = C.c_double
+        _lib.lfd_ref_energy.argtypes = [cfgp, P, P, P, P, P, P, P]
+        _lib.lfd_ref_energy.restype = C.c_int
+        _lib.lfd_ref_remap_occ.argtypes = [cfgp, P, P, P, C.c_int, P]
+        _lib.lfd_ref_remap_occ.restype = C.c_int
         for f in ("link_sweep", "kinetic", "local", "nl_half", "step", "density_current"):
             getattr(_lib, "lfd_ref_" + f).restype = C.c_int
     return _lib
@@ -141,3 +145,27 @@ def kinetic_energy(cfg: RefConfig, psi: np.ndarray, occ: np.ndarray, A: np.ndarr
     return float(lib().lfd_ref_kinetic_energy(C.byref(c), _ptr(psi, np.complex128),
                                               _ptr(np.ascontiguousarray(occ, np.float64), np.float64),
                                               _ptr(np.ascontiguousarray(A, np.float64), np.float64)))
+
+
+def energy(cfg: RefConfig, psi: np.ndarray, occ: np.ndarray, vloc: np.ndarray, A: np.ndarray,
+           proj: np.ndarray | None = None, dnl: np.ndarray | None = None) -> np.ndarray:
+    """[ndom, 4]: kinetic, local, nonlocal, total (calc_energy)."""
+    c = cfg.c()
+    E = np.zeros((cfg.ndom, 4))
+    _ok(lib().lfd_ref_energy(C.byref(c), _ptr(psi, np.complex128),
+                             _ptr(np.ascontiguousarray(occ, np.float64), np.float64), _ptr(vloc, np.float64),
+                             _ptr(np.ascontiguousarray(A, np.float64), np.float64), _ptr(proj, np.complex128),
+                             _ptr(None if dnl is None else np.ascontiguousarray(dnl, np.float64), np.float64),
+                             _ptr(E, np.float64)), "energy")
+    return E
+
+
+def remap_occ(cfg: RefConfig, psi: np.ndarray, occ: np.ndarray, refb: np.ndarray) -> np.ndarray:
+    """[ndom, nref]: sum_s f_s |<ref_k|psi_s>|^2 (remap_occ)."""
+    c = cfg.c()
+    nref = refb.shape[-1]
+    out = np.zeros((cfg.ndom, nref))
+    _ok(lib().lfd_ref_remap_occ(C.byref(c), _ptr(psi, np.complex128),
+                                _ptr(np.ascontiguousarray(occ, np.float64), np.float64),
+                                _ptr(refb, np.complex128), nref, _ptr(out, np.float64)), "remap_occ")
+    return out
