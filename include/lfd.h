@@ -38,7 +38,7 @@
 extern "C" {
 #endif
 
-#define LFD_ABI_VERSION 1
+#define LFD_ABI_VERSION 2
 #define LFD_MAX_DOMAINS 4096
 
 typedef struct lfd_ctx lfd_ctx; /* opaque */
@@ -61,7 +61,8 @@ typedef struct {
   double hx, hy, hz;   /* mesh spacing [bohr], > 0 */
   int32_t bc;          /* lfd_bc */
   int32_t norb;        /* propagated KS orbitals per domain, >= 1 */
-  int32_t nproj;       /* projector columns per domain, >= 0 (0 disables the nonlocal factor) */
+  int32_t nproj;       /* projector columns per domain, 0..2048 (0 disables the nonlocal factor) */
+  int32_t nref_max;    /* max reference-basis columns for lfd_remap_occ, 0..2048 (0: max(norb, nproj)) */
   double dt;           /* Delta_QD [a.u.], finite and nonzero (negative = backward in time) */
   int32_t device;      /* CUDA device ordinal */
   int32_t flags;       /* reserved, must be 0 */
@@ -80,7 +81,8 @@ typedef enum {
   LFD_K_NL_BACK = 8,   /* a5: GEMM-2 Psi <- (Psi + B C') diag(n), in place */
   LFD_K_DENSITY = 9,   /* a7: rho, j, per-line partial J */
   LFD_K_JREDUCE = 10,  /* a7: J = mean of j (fixed order) */
-  LFD_K_COUNT = 11
+  LFD_K_ENERGY = 11,   /* NEXT f-1: energy / occupation reductions (calc_energy, remap_occ) */
+  LFD_K_COUNT = 12
 } lfd_kernel_id;
 
 /* Bytes of DEVICE workspace lfd_init needs for this configuration. */
@@ -138,6 +140,20 @@ lfd_status lfd_density_current_global(lfd_ctx* ctx, double* rho_g, double* j_g, 
 /* As lfd_density_current for rho and Jmac, into HOST buffers (pinned recommended) via async D2H
  * copies; read them after lfd_sync(). Either pointer may be NULL to skip it. */
 lfd_status lfd_density_current_host(lfd_ctx* ctx, double* rho_host, double* Jmac_host);
+
+/* calc_energy (Fig. 5): E[dom][4] = {kinetic, local, nonlocal,
+ * total} of the current Psi with the current v_loc and A, DEVICE double, stream-ordered:
+ *   kinetic  = sum_s f_s dV sum_d (1/h_d^2) sum_r [ |psi_rs|^2 - Re(e^{i theta_d} conj(psi_rs) psi_{r+e_d,s}) ]
+ *              (the FD Peierls operator the propagator splits; the neighbour term is absent on the last
+ *              plane for zero BC),
+ *   local    = dV sum_r v_loc(r) rho(r),   nonlocal = sum_s f_s sum_u D_u |C_us|^2, C = dV B^H Psi. */
+lfd_status lfd_energy(lfd_ctx* ctx, double* E);
+
+/* remap_occ: occupations of a reference basis (e.g. the KS orbitals
+ * at t = 0), occ_out[dom][k] = sum_s f_s |dV sum_r conj(ref_rk) psi_rs|^2.
+ *  ref     DEVICE complex128 [ndom][nx][ny][nz][nref], 1 <= nref <= nref_max (config); read-only.
+ *  occ_out DEVICE double [ndom][nref]. Stream-ordered. */
+lfd_status lfd_remap_occ(lfd_ctx* ctx, const void* ref, int32_t nref, double* occ_out);
 
 /* Replace the occupations f (the QXMD<->LFD shadow-dynamics handshake). HOST [ndom][norb]. */
 lfd_status lfd_set_occupations(lfd_ctx* ctx, const double* occ);

@@ -26,7 +26,9 @@ constexpr int kKC1 = 16;  // GEMM-1 rows per chunk (nl.cu)
 size_t up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 struct Layout {
-  size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage;
+  size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage, cref,
+      epart;
+  int nref_cap;
   size_t total;
   int nsplit;
   long long rows_per_split;
@@ -59,6 +61,7 @@ lfd_status validate(const lfd_config* c, std::string& why) {
   if (c->nproj < 0 || c->nproj > 2048) { why = "nproj must be in [0, 2048]"; return LFD_EINVAL; }
   if (!(c->dt != 0.0) || !std::isfinite(c->dt)) { why = "dt must be finite and nonzero"; return LFD_EINVAL; }
   if (c->flags != 0) { why = "flags must be 0"; return LFD_EINVAL; }
+  if (c->nref_max < 0 || c->nref_max > 2048) { why = "nref_max must be in [0, 2048]"; return LFD_EINVAL; }
   const long long ng = (long long)c->nx * c->ny * c->nz;
   if (ng * (long long)std::max(c->norb, std::max(c->nproj, 1)) >= (1LL << 31)) {
     why = "ng * max(norb, nproj) must be < 2^31 per domain";
@@ -76,8 +79,9 @@ Geometry geometry(const lfd_config* c) {
   return g;
 }
 
-Layout layout(const Geometry& g, int num_sms) {
+Layout layout(const Geometry& g, int num_sms, int nref_max) {
   Layout L{};
+  L.nref_cap = nref_max > 0 ? nref_max : std::max(g.norb, g.nproj);
   const int np = g.nproj, no = g.norb, nd = g.ndom;
   // split-K of GEMM-1: about one CTA per SM in total, each split a multiple of the chunk height
   int tiles = 0;
@@ -108,7 +112,7 @@ Layout layout(const Geometry& g, int num_sms) {
   L.nsplit = nsplit;
   L.rows_per_split = rps;
   const size_t c16 = 16, d8 = 8;
-  const size_t mn = (size_t)std::max(np * no, np * np);
+  const size_t mn = (size_t)std::max(std::max(np * no, np * np), L.nref_cap * no);
   size_t o = 0;
   auto take = [&](size_t bytes) { size_t at = o; o += up(std::max<size_t>(bytes, 1)); return at; };
   L.phi = take((size_t)nd * g.ng * c16);
@@ -127,6 +131,8 @@ Layout layout(const Geometry& g, int num_sms) {
   L.vstage = take((size_t)nd * g.ng * d8);
   L.rhostage = take((size_t)nd * g.ng * d8);
   L.Jstage = take((size_t)nd * 3 * d8);
+  L.cref = take((size_t)nd * std::max(L.nref_cap, np) * no * c16);
+  L.epart = take((size_t)nd * lfd::density_blocks(g) * 2 * d8);
   L.total = o;
   return L;
 }
@@ -285,6 +291,21 @@ lfd_status nl_half(lfd_ctx* c) {
   return launch(c, LFD_K_NL_BACK, "k_gemm2", [&] { return lfd::launch_gemm2(a2, c->stream); });
 }
 
+// C[dom][m][n] = dV sum_r conj(A[r][m]) Psi[r][n] into out (GEMM-1 + fixed-order reduction).
+lfd_status project(lfd_ctx* c, const double2* A, int mrows, double2* out) {
+  const Geometry& g = c->g;
+  lfd::Gemm1Args a1;
+  a1.A = A; a1.X = c->psi; a1.part = c->at<double2>(c->L.part); a1.norms = nullptr;
+  a1.ndom = g.ndom; a1.mrows = mrows; a1.ncols = g.norb; a1.nsplit = c->L.nsplit;
+  a1.ng = g.ng; a1.rows_per_split = c->L.rows_per_split;
+  a1.a_dom_stride = g.ng * mrows; a1.x_dom_stride = g.ng * g.norb;
+  LFD_TRY(launch(c, LFD_K_NL_PROJ, "k_gemm1", [&] { return lfd::launch_gemm1(a1, c->stream); }));
+  lfd::ReduceArgs r{};
+  r.part = a1.part; r.normp = nullptr; r.D = nullptr; r.out = out; r.cprime = nullptr; r.s = nullptr;
+  r.ndom = g.ndom; r.mrows = mrows; r.ncols = g.norb; r.nsplit = c->L.nsplit; r.scale = g.dV; r.eps = 0;
+  return launch(c, LFD_K_NL_REDUCE, "k_reduce", [&] { return lfd::launch_reduce(r, c->stream); });
+}
+
 lfd_status set_A(lfd_ctx* c, const double* A) {
   thread_local lfd::CoefParams tp;  // 12 KB kernel-parameter block (A captured by value)
   for (int d0 = 0; d0 < c->g.ndom; d0 += lfd::kCoefMaxPerLaunch) {
@@ -298,11 +319,13 @@ lfd_status set_A(lfd_ctx* c, const double* A) {
 }
 
 lfd_status density_into(lfd_ctx* c, double* rho, double* j, double* Jmac, const long long* base_dev, long long sx,
-                        long long sy, long long jstride) {
+                        long long sy, long long jstride, bool energy = false) {
   lfd::DensArgs a;
   a.psi = c->psi; a.coef = c->coef(); a.occ = c->at<double>(c->L.occ);
   a.rho = rho; a.j = j; a.jline = c->at<double>(c->L.jline);
   a.base = base_dev; a.jbase = base_dev + c->g.ndom; a.sx = sx; a.sy = sy; a.jstride = jstride;
+  a.v = energy ? c->at<double>(c->L.vstage) : nullptr;
+  a.epart = energy ? c->at<double>(c->L.epart) : nullptr;
   LFD_TRY(launch(c, LFD_K_DENSITY, "k_density", [&] { return lfd::launch_density(c->g, a, c->stream); }));
   if (Jmac)
     LFD_TRY(launch(c, LFD_K_JREDUCE, "k_jreduce",
@@ -321,7 +344,7 @@ lfd_status lfd_workspace_size(const lfd_config* cfg, size_t* bytes) {
   if (!bytes) return fail(nullptr, LFD_EINVAL, "bytes is NULL");
   const int sms = query_sms(cfg->device);
   if (sms <= 0) return fail(nullptr, LFD_ECUDA, "no CUDA device (the LFD library has no CPU fallback)");
-  *bytes = layout(geometry(cfg), sms).total;
+  *bytes = layout(geometry(cfg), sms, cfg->nref_max).total;
   return LFD_OK;
 }
 
@@ -350,7 +373,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   if (!is_device_ptr(psi) || !is_device_ptr(workspace) || (proj && !is_device_ptr(proj)))
     return fail(nullptr, LFD_EINVAL, "psi, proj and workspace must be device memory");
   const Geometry g = geometry(cfg);
-  const Layout L = layout(g, prop.multiProcessorCount);
+  const Layout L = layout(g, prop.multiProcessorCount, cfg->nref_max);
   if (ws_bytes < L.total) return fail(nullptr, LFD_ENOMEM, "workspace smaller than lfd_workspace_size()");
   cudaError_t e = lfd::gemm_set_attributes();
   if (e == cudaSuccess) e = lfd::density_set_attributes();
@@ -395,7 +418,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   e = cudaMemsetAsync(c->at<double>(L.vstage), 0, sizeof(double) * g.ndom * g.ng, c->stream);
   if (e != cudaSuccess) { cuda_fail(c, e, "memset"); return bail(LFD_ECUDA); }
   lfd_status s2 = launch(c, LFD_K_PHASE, "k_phase",
-                         [&] { return lfd::launch_phase(g, c->at<double>(L.vstage), c->phi(), c->stream); });
+                         [&] { return lfd::launch_phase(g, c->at<double>(L.vstage), c->phi(), c->at<double>(L.vstage), c->stream); });
   if (s2 != LFD_OK) return bail(s2);
   s2 = set_A(c, nullptr);
   if (s2 != LFD_OK) return bail(s2);
@@ -423,7 +446,9 @@ lfd_status lfd_set_potential(lfd_ctx* c, const double* vloc) {
   if (!vloc) return fail(c, LFD_EINVAL, "vloc is NULL");
   DeviceGuard dg(c->device);
   if (!is_device_ptr(vloc)) return fail(c, LFD_EINVAL, "vloc must be device memory (use lfd_set_potential_host)");
-  return launch(c, LFD_K_PHASE, "k_phase", [&] { return lfd::launch_phase(c->g, vloc, c->phi(), c->stream); });
+  return launch(c, LFD_K_PHASE, "k_phase", [&] {
+    return lfd::launch_phase(c->g, vloc, c->phi(), c->at<double>(c->L.vstage), c->stream);
+  });
 }
 
 lfd_status lfd_set_potential_host(lfd_ctx* c, const double* vloc_host) {
@@ -434,7 +459,7 @@ lfd_status lfd_set_potential_host(lfd_ctx* c, const double* vloc_host) {
   cudaError_t e = cudaMemcpyAsync(stage, vloc_host, sizeof(double) * c->g.ndom * c->g.ng, cudaMemcpyHostToDevice,
                                   c->stream);
   if (e != cudaSuccess) return cuda_fail(c, e, "H2D vloc");
-  return launch(c, LFD_K_PHASE, "k_phase", [&] { return lfd::launch_phase(c->g, stage, c->phi(), c->stream); });
+  return launch(c, LFD_K_PHASE, "k_phase", [&] { return lfd::launch_phase(c->g, stage, c->phi(), stage, c->stream); });
 }
 
 lfd_status lfd_set_vector_potential(lfd_ctx* c, const double* A) {
@@ -522,6 +547,39 @@ lfd_status lfd_density_current_host(lfd_ctx* c, double* rho_host, double* Jmac_h
     if (e != cudaSuccess) return cuda_fail(c, e, "D2H J");
   }
   return LFD_OK;
+}
+
+lfd_status lfd_energy(lfd_ctx* c, double* E) {
+  LFD_TRY(check_ctx(c));
+  if (!E) return fail(c, LFD_EINVAL, "E is NULL");
+  DeviceGuard dg(c->device);
+  if (!is_device_ptr(E)) return fail(c, LFD_EINVAL, "E must be device memory");
+  const Geometry& g = c->g;
+  double2* C = nullptr;
+  if (g.nproj > 0) {
+    C = c->at<double2>(c->L.cref);
+    LFD_TRY(project(c, c->proj, g.nproj, C));
+  }
+  LFD_TRY(density_into(c, c->at<double>(c->L.rhostage), nullptr, nullptr, c->at<long long>(c->L.base),
+                       (long long)g.ny * g.nz, g.nz, g.ng, true));
+  return launch(c, LFD_K_ENERGY, "k_energy_final", [&] {
+    return lfd::launch_energy_final(g, c->at<double>(c->L.epart), lfd::density_blocks(g), C,
+                                    c->at<double>(c->L.D), c->at<double>(c->L.occ), E, c->stream);
+  });
+}
+
+lfd_status lfd_remap_occ(lfd_ctx* c, const void* ref, int32_t nref, double* occ_out) {
+  LFD_TRY(check_ctx(c));
+  if (!ref || !occ_out) return fail(c, LFD_EINVAL, "ref and occ_out must be non-NULL");
+  if (nref < 1 || nref > c->L.nref_cap) return fail(c, LFD_EINVAL, "nref must be in [1, nref_max]");
+  if (reinterpret_cast<uintptr_t>(ref) & 15) return fail(c, LFD_EINVAL, "ref must be 16-byte aligned");
+  DeviceGuard dg(c->device);
+  if (!is_device_ptr(ref) || !is_device_ptr(occ_out)) return fail(c, LFD_EINVAL, "ref / occ_out must be device memory");
+  double2* C = c->at<double2>(c->L.cref);
+  LFD_TRY(project(c, static_cast<const double2*>(ref), nref, C));
+  return launch(c, LFD_K_ENERGY, "k_remap", [&] {
+    return lfd::launch_remap(c->g, nref, C, c->at<double>(c->L.occ), occ_out, c->stream);
+  });
 }
 
 lfd_status lfd_set_occupations(lfd_ctx* c, const double* occ) {

@@ -22,7 +22,7 @@ constexpr int kSub = 8, kTY = 2, kTZ = 8, kXC = 10;
 constexpr int kDensThreads = kSub * kTY * kTZ;  // 128
 
 __global__ void __launch_bounds__(kDensThreads) k_density(Geometry g, DensArgs a, int ntz, int nty, int nxc) {
-  __shared__ double jsh[3][kDensThreads / kSub];
+  __shared__ double jsh[5][kDensThreads / kSub];
   const int dom = blockIdx.y;
   int b = blockIdx.x;
   const int tz = b % ntz; b /= ntz;
@@ -43,7 +43,7 @@ __global__ void __launch_bounds__(kDensThreads) k_density(Geometry g, DensArgs a
   const double2 ex = cf->eth[0], ey = cf->eth[1], ez = cf->eth[2];
   const double ihx = cf->inv_h[0], ihy = cf->inv_h[1], ihz = cf->inv_h[2];
   const int x0 = xc * nxc, x1 = min(g.nx, x0 + nxc);
-  double jsx = 0.0, jsy = 0.0, jsz = 0.0;
+  double jsx = 0.0, jsy = 0.0, jsz = 0.0, ekin = 0.0, eloc = 0.0;
   for (int x = x0; x < x1; ++x) {
     const bool has_x = valid && (per || x + 1 < g.nx);
     const int xp = (x + 1 == g.nx) ? 0 : x + 1;
@@ -90,6 +90,15 @@ __global__ void __launch_bounds__(kDensThreads) k_density(Geometry g, DensArgs a
     const double jy = has_y ? (ey.x * pyi + ey.y * pyr) * ihy : 0.0;
     const double jz = has_z ? (ez.x * pzi + ez.y * pzr) * ihz : 0.0;
     jsx += jx; jsy += jy; jsz += jz;
+    if (a.epart && valid) {  // kinetic / local energy densities (lfd_energy), FD Peierls form
+      const double w2x = ihx * ihx, w2y = ihy * ihy, w2z = ihz * ihz;
+      double ek = (w2x + w2y + w2z) * rho;
+      if (has_x) ek -= w2x * (ex.x * pxr - ex.y * pxi);  // Re(e^{i theta} P)
+      if (has_y) ek -= w2y * (ey.x * pyr - ey.y * pyi);
+      if (has_z) ek -= w2z * (ez.x * pzr - ez.y * pzi);
+      ekin += ek;
+      eloc += a.v[(long long)dom * g.ng + ((long long)x * g.ny + y) * g.nz + z] * rho;
+    }
     if (q == 0 && valid) {
       const long long o = (long long)x * a.sx + (long long)y * a.sy + z;
       a.rho[a.base[dom] + o] = rho;
@@ -103,8 +112,14 @@ __global__ void __launch_bounds__(kDensThreads) k_density(Geometry g, DensArgs a
   }
   if (q == 0) {
     jsh[0][pt] = jsx; jsh[1][pt] = jsy; jsh[2][pt] = jsz;
+    jsh[3][pt] = ekin; jsh[4][pt] = eloc;
   }
   __syncthreads();
+  if (a.epart && threadIdx.x >= 32 && threadIdx.x < 34) {
+    double t = 0.0;
+    for (int k = 0; k < kDensThreads / kSub; ++k) t += jsh[3 + threadIdx.x - 32][k];
+    a.epart[((long long)dom * gridDim.x + blockIdx.x) * 2 + threadIdx.x - 32] = t;
+  }
   if (threadIdx.x < 3) {
     double t = 0.0;
     for (int i = 0; i < kDensThreads / kSub; ++i) t += jsh[threadIdx.x][i];
@@ -126,7 +141,7 @@ constexpr int kPlanePts = (kTY + 1) * (kTZ + 1);
 __global__ void __launch_bounds__(kDensThreads) k_density_tma(Geometry g, DensArgs a, int ntz, int nty, int nxc) {
   extern __shared__ __align__(128) unsigned char dsm[];
   __shared__ __align__(8) uint64_t bars[kRingSlots];
-  __shared__ double jsh[3][kDensThreads / kSub];
+  __shared__ double jsh[5][kDensThreads / kSub];
   const int norb = g.norb;
   const int slot_elems = kPlanePts * norb;  // complex elements per slot
   double2* ring = reinterpret_cast<double2*>(dsm);
@@ -192,7 +207,7 @@ __global__ void __launch_bounds__(kDensThreads) k_density_tma(Geometry g, DensAr
   if (threadIdx.x < 32)
     for (int i = 0; i < kRingSlots && i < nplanes; ++i) issue(i);
 
-  double jsx = 0.0, jsy = 0.0, jsz = 0.0;
+  double jsx = 0.0, jsy = 0.0, jsz = 0.0, ekin = 0.0, eloc = 0.0;
   for (int i = 0; i + 1 < nplanes; ++i) {
     const int x = x0 + i;
     mbar_wait(&bars[i % kRingSlots], (uint32_t)((i / kRingSlots) & 1));
@@ -242,6 +257,15 @@ __global__ void __launch_bounds__(kDensThreads) k_density_tma(Geometry g, DensAr
     const double jy = has_y ? (ey.x * pyi + ey.y * pyr) * ihy : 0.0;
     const double jz = has_z ? (ez.x * pzi + ez.y * pzr) * ihz : 0.0;
     jsx += jx; jsy += jy; jsz += jz;
+    if (a.epart && valid) {  // kinetic / local energy densities (lfd_energy), FD Peierls form
+      const double w2x = ihx * ihx, w2y = ihy * ihy, w2z = ihz * ihz;
+      double ek = (w2x + w2y + w2z) * rho;
+      if (has_x) ek -= w2x * (ex.x * pxr - ex.y * pxi);  // Re(e^{i theta} P)
+      if (has_y) ek -= w2y * (ey.x * pyr - ey.y * pyi);
+      if (has_z) ek -= w2z * (ez.x * pzr - ez.y * pzi);
+      ekin += ek;
+      eloc += a.v[(long long)dom * g.ng + ((long long)x * g.ny + y) * g.nz + z] * rho;
+    }
     if (q == 0 && valid) {
       const long long o = (long long)x * a.sx + (long long)y * a.sy + z;
       a.rho[a.base[dom] + o] = rho;
@@ -257,8 +281,14 @@ __global__ void __launch_bounds__(kDensThreads) k_density_tma(Geometry g, DensAr
   }
   if (q == 0) {
     jsh[0][pt] = jsx; jsh[1][pt] = jsy; jsh[2][pt] = jsz;
+    jsh[3][pt] = ekin; jsh[4][pt] = eloc;
   }
   __syncthreads();
+  if (a.epart && threadIdx.x >= 32 && threadIdx.x < 34) {
+    double t = 0.0;
+    for (int k = 0; k < kDensThreads / kSub; ++k) t += jsh[3 + threadIdx.x - 32][k];
+    a.epart[((long long)dom * gridDim.x + blockIdx.x) * 2 + threadIdx.x - 32] = t;
+  }
   if (threadIdx.x < 3) {
     double t = 0.0;
     for (int k = 0; k < kDensThreads / kSub; ++k) t += jsh[threadIdx.x][k];

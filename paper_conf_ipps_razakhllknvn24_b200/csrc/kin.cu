@@ -52,17 +52,21 @@ cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int co
 }
 
 // Phi(r) = e^{-i (Delta/2) v_loc(r)}  (Strang placement of the potential, reading R7).
-__global__ void k_phase(const double* __restrict__ v, double2* __restrict__ phi, long long n, double half_dt) {
+// The kernel also keeps a copy of v_loc for lfd_energy (vcopy may alias v: then it is not written).
+__global__ void k_phase(const double* __restrict__ v, double2* __restrict__ phi, double* vcopy, long long n,
+                        double half_dt) {
   long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
+  const double vi = v[i];
   double s, c;
-  sincos(half_dt * v[i], &s, &c);
+  sincos(half_dt * vi, &s, &c);
   phi[i] = make_double2(c, -s);
+  if (vcopy != v) vcopy[i] = vi;
 }
 
-cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, cudaStream_t st) {
+cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, double* vcopy, cudaStream_t st) {
   long long n = g.ng * g.ndom;
-  k_phase<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(v, phi, n, 0.5 * g.dt);
+  k_phase<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(v, phi, vcopy, n, 0.5 * g.dt);
   return cudaGetLastError();
 }
 

@@ -36,7 +36,7 @@ struct CoefParams {
 };
 cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int count, DomCoef* coef,
                         cudaStream_t st);
-cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, cudaStream_t st);
+cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, double* vcopy, cudaStream_t st);
 
 // One pass of K_axis over every line of every domain, optionally fused with a phase multiply
 // (phase_mode 1: Phi . psi before the sweep; 2: after).
@@ -102,10 +102,18 @@ struct DensArgs {
   const long long* base;   // [dom] device array: rho offset of the domain's (0,0,0)
   const long long* jbase;  // [dom] device array: j offset of the domain's (0,0,0), component 0
   long long sx, sy, jstride;
+  const double* v;      // v_loc copy [dom][ng] when energy partials are wanted, else nullptr
+  double* epart;        // [dom][density_blocks][2] per-CTA sums of (kinetic, local) energy densities
 };
 cudaError_t launch_density(const Geometry& g, const DensArgs& a, cudaStream_t st);
 int density_blocks(const Geometry& g);
 cudaError_t density_set_attributes();
 cudaError_t launch_jreduce(const Geometry& g, const double* jline, double* Jmac, cudaStream_t st);
+
+// calc_energy / remap_occ reductions (energy.cu)
+cudaError_t launch_energy_final(const Geometry& g, const double* epart, int blocks, const double2* C,
+                                const double* D, const double* occ, double* E, cudaStream_t st);
+cudaError_t launch_remap(const Geometry& g, int nref, const double2* C, const double* occ, double* out,
+                         cudaStream_t st);
 
 }  // namespace lfd

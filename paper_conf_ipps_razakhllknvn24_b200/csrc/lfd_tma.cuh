@@ -41,47 +41,4 @@ __device__ __forceinline__ void l2_prefetch(const void* src, uint32_t bytes) {
   asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
 }
 
-// ---- tensor memory (TMEM) as parking space for finished accumulator tiles -------------------------
-__device__ __forceinline__ void tmem_alloc(uint32_t* slot, uint32_t ncols) {  // one full warp
-  asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_addr(slot)), "r"(ncols)
-               : "memory");
-  asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
-}
-__device__ __forceinline__ void tmem_dealloc(uint32_t taddr, uint32_t ncols) {  // the allocating warp
-  asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(taddr), "r"(ncols) : "memory");
-}
-__device__ __forceinline__ void tmem_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
-__device__ __forceinline__ void tmem_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
-
-#define LFD_R8(b) "r"(u[b]), "r"(u[b + 1]), "r"(u[b + 2]), "r"(u[b + 3]), "r"(u[b + 4]), "r"(u[b + 5]), "r"(u[b + 6]), "r"(u[b + 7])
-#define LFD_W8(b) "=r"(u[b]), "=r"(u[b + 1]), "=r"(u[b + 2]), "=r"(u[b + 3]), "=r"(u[b + 4]), "=r"(u[b + 5]), "=r"(u[b + 6]), "=r"(u[b + 7])
-// 32 lanes x 32 consecutive 32-bit columns per call (shape 32x32b, .x32); waits for completion.
-__device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t* u) {
-  asm volatile(
-      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
-      "%15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31, %32};" ::"r"(taddr),
-      LFD_R8(0), LFD_R8(8), LFD_R8(16), LFD_R8(24)
-      : "memory");
-}
-__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t* u) {
-  asm volatile(
-      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15, "
-      "%16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];"
-      : LFD_W8(0), LFD_W8(8), LFD_W8(16), LFD_W8(24)
-      : "r"(taddr)
-      : "memory");
-}
-#undef LFD_R8
-#undef LFD_W8
-__device__ __forceinline__ void tmem_st64(uint32_t taddr, const uint32_t (&u)[64]) {
-  tmem_st32(taddr, u);
-  tmem_st32(taddr + 32, u + 32);
-  asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
-}
-__device__ __forceinline__ void tmem_ld64(uint32_t taddr, uint32_t (&u)[64]) {
-  tmem_ld32(taddr, u);
-  tmem_ld32(taddr + 32, u + 32);
-  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-}
-
 }  // namespace lfd

@@ -562,17 +562,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
 // stride = nproj rounded to 4, == 4 mod 8 complex, so the A-fragment LDS.128 are conflict free), and
 // C' for the current (domain, column tile) stays resident in shared memory. Items are ordered
 // (domain, column tile, row block) so C' is reloaded only when a CTA crosses into another
-// (domain, tile). The epilogue of item j is deferred past the K loop of item j+1: the finished
-// B C' tile is parked in tensor memory (TMEM, tcgen05.st / tcgen05.ld; 64 KB of the SM's 256 KB)
-// while the Psi tile of item j is loaded into registers during item j+1's DMMAs, so the epilogue's
-// global traffic no longer idles the FP64 tensor pipe. kNP = 64 instantiates a fully unrolled K loop; kNP = 0 handles any nproj <= 64.
+// (domain, tile). The Psi rows of the next item are prefetched into L2 (cp.async.bulk.prefetch) so the
+// epilogue's loads hit L2. kNP = 64 instantiates a fully unrolled K loop; kNP = 0 handles any nproj <= 64.
 // ------------------------------------------------------------------------------------------------
 constexpr int kFullStages = 2;
 constexpr int kFullLdaMax = 68;
 constexpr int kFullABytes = kTile * kFullLdaMax * 16;     // [64 rows][<=68] complex
 constexpr int kFullCBytes = kTile * kLd1 * 16;            // [<=64 proj][66] complex
-constexpr int kFullSmem = kFullStages * kFullABytes + kFullCBytes + 8 * 8;
-constexpr uint32_t kTmemCols = 256;  // 2 buffers x (2 warps per lane quarter x 64 columns)
+constexpr int kFullSmem = kFullStages * kFullABytes + kFullCBytes + 4 * 8;
 
 __host__ __device__ constexpr int full_lda(int np) { return ((np + 3) / 4 * 4) % 8 == 0 ? (np + 3) / 4 * 4 + 4 : (np + 3) / 4 * 4; }
 
@@ -580,9 +577,8 @@ template <int kNP>
 __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
   extern __shared__ __align__(128) unsigned char smem[];
   double2* Cs = reinterpret_cast<double2*>(smem + kFullStages * kFullABytes);
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kFullStages * kFullABytes + kFullCBytes);
-  uint64_t* cbar = full + kFullStages;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(cbar + 1);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kFullStages * kFullABytes + kFullCBytes);
+  uint64_t* cbar = bars + kFullStages;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int g = lane >> 2, t = lane & 3;
   const int wm = warp >> 2, wn = warp & 3;
@@ -596,17 +592,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
   const int nk4 = (np + 3) / 4;
 
   if (tid == 0) {
-    for (int s = 0; s < kFullStages; ++s) mbar_init(&full[s], 1);
-    mbar_init(cbar, 1);
+    for (int s = 0; s < kFullStages + 1; ++s) mbar_init(&bars[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == 0) tmem_alloc(tmem_slot, kTmemCols);
-  tmem_fence_before();
   __syncthreads();
-  tmem_fence_after();
-  // TMEM parking for finished tiles: buffer b at columns b*128; warp w uses lanes 32*(w%4).. and
-  // columns +64*(w/4); each lane parks its 32 doubles (re, im of its 16 outputs) as 64 x 32-bit.
-  const uint32_t tmem_base = *tmem_slot + ((uint32_t)(32 * (warp & 3)) << 16) + (uint32_t)(64 * (warp >> 2));
 
   auto decode = [&](long long j, int& dom, int& n0, long long& r0) {
     const long long item = blockIdx.x + j * gridDim.x;
@@ -622,58 +611,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
     long long r0;
     decode(j, dom, n0, r0);
     const int rows = (int)min((long long)kTile, p.ng - r0);
-    if (lane == 0) {
-      mbar_expect_tx(&full[stage], (uint32_t)(rows * np * 16));
-      l2_prefetch(p.psi + ((long long)dom * p.ng + r0) * p.norb, (uint32_t)(rows * p.norb * 16));
-    }
+    if (lane == 0) mbar_expect_tx(&bars[stage], (uint32_t)(rows * np * 16));
     __syncwarp();
     double2* As = reinterpret_cast<double2*>(smem + stage * kFullABytes);
     const double2* src = p.B + ((long long)dom * p.ng + r0) * np;
-    for (int r = lane; r < rows; r += 32) tma_row(As + r * lda, src + (long long)r * np, np * 16, &full[stage]);
-  };
-  // Psi tile of item j -> registers (L2 hits: prefetched when the item's B rows were requested)
-  auto load_psi = [&](long long j, double2 (&pv)[4][2][2]) {
-    int dom, n0;
-    long long r0;
-    decode(j, dom, n0, r0);
-    const double2* psi = p.psi + (long long)dom * p.ng * p.norb;
-#pragma unroll
-    for (int mi = 0; mi < 4; ++mi) {
-      const long long r = r0 + wm * 32 + mi * 8 + g;
-#pragma unroll
-      for (int ni = 0; ni < 2; ++ni)
-#pragma unroll
-        for (int c = 0; c < 2; ++c) {
-          const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
-          pv[mi][ni][c] = (r < p.ng && col < p.norb) ? psi[r * p.norb + col] : cz();
-        }
-    }
-  };
-  // epilogue of item j: Psi <- n_s (Psi + B C'), with B C' parked in TMEM buffer j % 2
-  auto finish = [&](long long j, const double2 (&pv)[4][2][2]) {
-    int dom, n0;
-    long long r0;
-    decode(j, dom, n0, r0);
-    uint32_t u[64];
-    tmem_ld64(tmem_base + (uint32_t)(128 * (j & 1)), u);
-    double2* psi = p.psi + (long long)dom * p.ng * p.norb;
-    const double* nf = p.nfac + (long long)dom * p.norb;
-#pragma unroll
-    for (int ni = 0; ni < 2; ++ni)
-#pragma unroll
-      for (int c = 0; c < 2; ++c) {
-        const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
-        if (col >= p.norb) continue;
-        const double f = nf[col];
-#pragma unroll
-        for (int mi = 0; mi < 4; ++mi) {
-          const long long r = r0 + wm * 32 + mi * 8 + g;
-          const int e = ((mi * 2 + ni) * 2 + c) * 4;
-          const double re = __hiloint2double((int)u[e + 1], (int)u[e]);
-          const double im = __hiloint2double((int)u[e + 3], (int)u[e + 2]);
-          if (r < p.ng) psi[r * p.norb + col] = make_double2(f * (pv[mi][ni][c].x + re), f * (pv[mi][ni][c].y + im));
-        }
-      }
+    for (int r = lane; r < rows; r += 32) tma_row(As + r * lda, src + (long long)r * np, np * 16, &bars[stage]);
   };
 
   if (warp == 0)
@@ -681,12 +623,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
 
   int cur_dom = -1, cur_n0 = -1;
   uint32_t cphase = 0;
-  double2 pv[4][2][2];
   for (long long j = 0; j < my_items; ++j) {
     int dom, n0;
     long long r0;
     decode(j, dom, n0, r0);
-    if (dom != cur_dom || n0 != cur_n0) {  // (re)load C'[dom][:, n0:n0+64]; all warps are past Cs
+    if (dom != cur_dom || n0 != cur_n0) {  // (re)load C'[dom][:, n0:n0+64] (all warps are past Cs)
       const int nvalid = min(kTile, p.norb - n0);
       if (warp == 0) {
         if (lane == 0) mbar_expect_tx(cbar, (uint32_t)(np * nvalid * 16));
@@ -699,9 +640,22 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
       cur_dom = dom;
       cur_n0 = n0;
     }
-    if (j > 0) load_psi(j - 1, pv);  // in flight during this item's K loop
+    double2* psi = p.psi + (long long)dom * p.ng * p.norb;
+    // Psi rows of the NEXT item go to L2 now (the epilogue of this item reads rows prefetched during
+    // the previous one), keeping 64 registers free for fragment pipelining.
+    if (tid == 32 && j + 1 < my_items) {
+      int d1, n1;
+      long long q1;
+      decode(j + 1, d1, n1, q1);
+      const long long rows1 = min((long long)kTile, p.ng - q1);
+      l2_prefetch(p.psi + ((long long)d1 * p.ng + q1) * p.norb, (uint32_t)(rows1 * p.norb * 16));
+    }
+    if (tid == 32 && j == 0) {
+      const long long rows0 = min((long long)kTile, p.ng - r0);
+      l2_prefetch(psi + r0 * p.norb, (uint32_t)(rows0 * p.norb * 16));
+    }
     const int stage = (int)(j % kFullStages);
-    mbar_wait(&full[stage], (uint32_t)((j / kFullStages) & 1));
+    mbar_wait(&bars[stage], (uint32_t)((j / kFullStages) & 1));
     const double2* As = reinterpret_cast<const double2*>(smem + stage * kFullABytes);
     Frag acc;
     acc.zero();
@@ -717,34 +671,38 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
       for (int ni = 0; ni < 2; ++ni) c[ni] = ok ? Cs[k * kLd1 + wn * 16 + ni * 8 + g] : cz();
       mma_4x2(acc, a, c);
     }
-    {  // park this item's B C' in TMEM buffer j % 2 (its epilogue runs after the next K loop)
-      uint32_t u[64];
-#pragma unroll
-      for (int mi = 0; mi < 4; ++mi)
-#pragma unroll
-        for (int ni = 0; ni < 2; ++ni)
-#pragma unroll
-          for (int c = 0; c < 2; ++c) {
-            const int e = ((mi * 2 + ni) * 2 + c) * 4;
-            const double re = acc.re(mi, ni, c), im = acc.im(mi, ni, c);
-            u[e] = (uint32_t)__double2loint(re);
-            u[e + 1] = (uint32_t)__double2hiint(re);
-            u[e + 2] = (uint32_t)__double2loint(im);
-            u[e + 3] = (uint32_t)__double2hiint(im);
-          }
-      tmem_st64(tmem_base + (uint32_t)(128 * (j & 1)), u);
-    }
     __syncthreads();  // stage and Cs free
     if (warp == 0 && j + kFullStages < my_items) issue(j + kFullStages, stage);
-    if (j > 0) finish(j - 1, pv);
+    // epilogue: Psi <- n_s (Psi + B C'); all 16 loads (L2 hits, prefetched) are issued before any store
+    const double* nf = p.nfac + (long long)dom * p.norb;
+    double2 pv[4][2][2];
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi) {
+      const long long r = r0 + wm * 32 + mi * 8 + g;
+#pragma unroll
+      for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+        for (int c = 0; c < 2; ++c) {
+          const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
+          pv[mi][ni][c] = (r < p.ng && col < p.norb) ? psi[r * p.norb + col] : cz();
+        }
+    }
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+      for (int c = 0; c < 2; ++c) {
+        const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
+        if (col >= p.norb) continue;
+        const double f = nf[col];
+#pragma unroll
+        for (int mi = 0; mi < 4; ++mi) {
+          const long long r = r0 + wm * 32 + mi * 8 + g;
+          if (r < p.ng)
+            psi[r * p.norb + col] =
+                make_double2(f * (pv[mi][ni][c].x + acc.re(mi, ni, c)), f * (pv[mi][ni][c].y + acc.im(mi, ni, c)));
+        }
+      }
   }
-  if (my_items > 0) {
-    load_psi(my_items - 1, pv);
-    finish(my_items - 1, pv);
-  }
-  tmem_fence_before();
-  __syncthreads();
-  if (warp == 0) tmem_dealloc(*tmem_slot, kTmemCols);
 }
 
 cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {

@@ -17,24 +17,24 @@ import numpy as np
 HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "liblfd.so")
 
-LFD_ABI_VERSION = 1
+LFD_ABI_VERSION = 2
 LFD_BC_PERIODIC = 0
 LFD_BC_ZERO = 1
 STATUS = {0: "LFD_OK", -1: "LFD_EINVAL", -2: "LFD_ENOMEM", -3: "LFD_ECUDA", -4: "LFD_ESTATE",
           -5: "LFD_EUNSUPPORTED"}
 KERNELS = ("coef", "phase", "kin_x", "kin_y", "kin_z", "nl_proj", "nl_reduce", "nl_norm", "nl_back",
-           "density", "jreduce")
+           "density", "jreduce", "energy")
 EXPORTS = ("lfd_workspace_size", "lfd_init", "lfd_set_potential", "lfd_set_potential_host",
            "lfd_set_vector_potential", "lfd_step", "lfd_density_current", "lfd_density_current_global",
-           "lfd_density_current_host", "lfd_set_occupations", "lfd_set_stream", "lfd_sync",
+           "lfd_density_current_host", "lfd_energy", "lfd_remap_occ", "lfd_set_occupations", "lfd_set_stream", "lfd_sync",
            "lfd_launch_count", "lfd_profile_enable", "lfd_profile_read", "lfd_last_error", "lfd_destroy")
 
 
 class lfd_config(C.Structure):
     _fields_ = [("abi_version", C.c_int32), ("ndomains", C.c_int32), ("nx", C.c_int32), ("ny", C.c_int32),
                 ("nz", C.c_int32), ("hx", C.c_double), ("hy", C.c_double), ("hz", C.c_double),
-                ("bc", C.c_int32), ("norb", C.c_int32), ("nproj", C.c_int32), ("dt", C.c_double),
-                ("device", C.c_int32), ("flags", C.c_int32)]
+                ("bc", C.c_int32), ("norb", C.c_int32), ("nproj", C.c_int32), ("nref_max", C.c_int32),
+                ("dt", C.c_double), ("device", C.c_int32), ("flags", C.c_int32)]
 
 
 class LFDError(RuntimeError):
@@ -66,6 +66,8 @@ def load():
         "lfd_density_current": [P, P, P, P],
         "lfd_density_current_global": [P, P, P, P, P, P],
         "lfd_density_current_host": [P, P, P],
+        "lfd_energy": [P, P],
+        "lfd_remap_occ": [P, P, I32, P],
         "lfd_set_occupations": [P, P],
         "lfd_set_stream": [P, P],
         "lfd_sync": [P],
@@ -118,8 +120,8 @@ def _stream_ptr(stream=None):
     return C.c_void_p(s.cuda_stream)
 
 
-def make_config(ndomains, nx, ny, nz, hx, hy, hz, bc, norb, nproj, dt, device=0) -> lfd_config:
-    return lfd_config(LFD_ABI_VERSION, ndomains, nx, ny, nz, hx, hy, hz, bc, norb, nproj, dt, device, 0)
+def make_config(ndomains, nx, ny, nz, hx, hy, hz, bc, norb, nproj, dt, device=0, nref_max=0) -> lfd_config:
+    return lfd_config(LFD_ABI_VERSION, ndomains, nx, ny, nz, hx, hy, hz, bc, norb, nproj, nref_max, dt, device, 0)
 
 
 # ---- 1:1 wrappers of the C entry points --------------------------------------------------------
@@ -173,6 +175,16 @@ def lfd_density_current_host(ctx, rho_host=None, Jmac_host=None):
     _check(load().lfd_density_current_host(ctx, pr, pj), ctx)
 
 
+def lfd_energy(ctx, E):
+    """E: CUDA float64 [ndom, 4] (kinetic, local, nonlocal, total)."""
+    _check(load().lfd_energy(ctx, _dptr(E)), ctx)
+
+
+def lfd_remap_occ(ctx, ref, occ_out):
+    """ref: CUDA complex128 [ndom, nx, ny, nz, nref]; occ_out: CUDA float64 [ndom, nref]."""
+    _check(load().lfd_remap_occ(ctx, _dptr(ref), int(ref.shape[-1]), _dptr(occ_out)), ctx)
+
+
 def lfd_set_occupations(ctx, occ):
     p, _k = _hptr(occ)
     _check(load().lfd_set_occupations(ctx, p), ctx)
@@ -221,14 +233,14 @@ class Context:
     (host arrays). h = (hx, hy, hz).
     """
 
-    def __init__(self, psi, proj, dnl, occ, h, dt, bc=LFD_BC_PERIODIC, stream=None):
+    def __init__(self, psi, proj, dnl, occ, h, dt, bc=LFD_BC_PERIODIC, stream=None, nref_max=0):
         import torch
         if psi.dtype != torch.complex128 or psi.dim() != 5:
             raise TypeError("psi must be complex128 [ndom, nx, ny, nz, norb]")
         ndom, nx, ny, nz, norb = psi.shape
         nproj = 0 if proj is None else proj.shape[-1]
         self.cfg = make_config(ndom, nx, ny, nz, h[0], h[1], h[2], bc, norb, nproj, dt,
-                               device=psi.device.index or 0)
+                               device=psi.device.index or 0, nref_max=nref_max)
         self.psi, self.proj = psi, proj
         ws = lfd_workspace_size(self.cfg)
         self.workspace = torch.empty(max(ws, 1), dtype=torch.uint8, device=psi.device)
@@ -256,6 +268,18 @@ class Context:
         J = torch.empty((nd, 3), dtype=torch.float64, device=dev)
         lfd_density_current(self.ctx, rho, j, J)
         return rho, j, J
+
+    def energy(self):
+        import torch
+        E = torch.empty((self.shape[0], 4), dtype=torch.float64, device=self.psi.device)
+        lfd_energy(self.ctx, E)
+        return E
+
+    def remap_occ(self, ref):
+        import torch
+        out = torch.empty((self.shape[0], ref.shape[-1]), dtype=torch.float64, device=self.psi.device)
+        lfd_remap_occ(self.ctx, ref, out)
+        return out
 
     def sync(self):
         lfd_sync(self.ctx)
