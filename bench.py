@@ -327,6 +327,27 @@ def main():
                 "flops_per_launch" if d["bound"] == "tensor" else "bytes_per_launch":
                     work[dom][1] if d["bound"] == "tensor" else work[dom][0]}
 
+    # sequence mode: lfd_step_sequence over the same K steps (per-step A, adjacent nonlocal factors
+    # merged, Psi materialised only at the end; one density at the end) -- an additional number for
+    # callers that do not observe Psi between QD steps (e.g. fixed v_loc over an MD step)
+    seq = None
+    if world == 1 and w.nproj > 0:
+        A_arr = np.stack([A_seq[args.warmup + n] for n in range(args.steps)])
+        lfd.lfd_step_sequence(ctx.ctx, A_arr[:3])
+        torch.cuda.synchronize()
+        s0 = torch.cuda.Event(enable_timing=True)
+        s1 = torch.cuda.Event(enable_timing=True)
+        s0.record(stream)
+        lfd.lfd_set_potential(ctx.ctx, v_dev)
+        lfd.lfd_step_sequence(ctx.ctx, A_arr)
+        lfd.lfd_density_current(ctx.ctx, rho, None, J)
+        s1.record(stream)
+        torch.cuda.synchronize()
+        sms = s0.elapsed_time(s1)
+        seq = {"value": w.ogp_per_step * args.steps / (sms / 1e3), "unit": UNIT, "ms_per_step": sms / args.steps,
+               "note": f"lfd_step_sequence of {args.steps} steps (per-step A; N o N merged: {args.steps + 1} "
+                       f"projector GEMM pairs instead of {2 * args.steps}), one density at the end"}
+
     # end to end through the C ABI with HOST buffers: pinned v in, pinned rho + J out, every step
     e2e = None
     if not args.no_e2e:
@@ -382,6 +403,7 @@ def main():
             "roofline": roofline,
             "kernels": kernels,
             "e2e": e2e,
+            "sequence_mode": seq,
             "cpu_baseline": cpu,
         }
         print(json.dumps(out), flush=True)

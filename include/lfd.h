@@ -120,6 +120,15 @@ lfd_status lfd_set_vector_potential(lfd_ctx* ctx, const double* A);
 /* Enqueue nsteps LFD steps (Eq. 6) with the current v_loc and A. nsteps == 0 is a no-op; < 0 EINVAL. */
 lfd_status lfd_step(lfd_ctx* ctx, int32_t nsteps);
 
+/* Enqueue nsteps LFD steps with one vector potential per step, A_seq HOST double [nsteps][ndom][3]
+ * (captured by value; step n uses A_seq[n], Eq. 4 midpoints), and the current v_loc. The result equals
+ * nsteps x (lfd_set_vector_potential(A_seq[n]); lfd_step(1)) up to roundoff: the second nonlocal
+ * factor of step n and the first of step n+1 (Eq. 6; both depend only on Psi, B, D, Delta) are applied
+ * as one combined factor N o N = L^2 renormalised, L^2 = I + B (2cD + c^2 D G D) B^H dV, c = -i Delta/2,
+ * so a sequence costs nsteps + 1 projector GEMM pairs instead of 2 nsteps. Psi is only materialised
+ * at the end. Afterwards the context's A is A_seq[nsteps-1]. */
+lfd_status lfd_step_sequence(lfd_ctx* ctx, int32_t nsteps, const double* A_seq);
+
 /* Density and current of the current Psi with the current A (kernel 4; R13):
  *  rho  DEVICE double [ndom][nx][ny][nz]          rho_r = sum_s f_s |psi_rs|^2
  *  j    DEVICE double [ndom][3][nx][ny][nz] or NULL

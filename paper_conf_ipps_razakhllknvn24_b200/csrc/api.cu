@@ -5,6 +5,7 @@
 
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <new>
@@ -162,6 +163,7 @@ struct lfd_ctx {
   int device;
   int num_sms;
   uint64_t launches = 0;
+  int gemm2_variant = 1;  // internal tuning knob, env LFD_GEMM2_VARIANT (1 measured faster)
   std::string err = "no error";
   // density-current global layout cache
   std::vector<long long> gbase_host;
@@ -260,8 +262,8 @@ bool is_device_ptr(const void* p) {
   return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
-// Eq. 6 nonlocal factor N on every domain (kernels a3, a4, a5).
-lfd_status nl_half(lfd_ctx* c) {
+// Eq. 6 nonlocal factor N on every domain (kernels a3, a4, a5); merged = N o N in one pass.
+lfd_status nl_half(lfd_ctx* c, bool merged = false) {
   const Geometry& g = c->g;
   lfd::Gemm1Args a1;
   a1.A = c->proj;
@@ -281,13 +283,20 @@ lfd_status nl_half(lfd_ctx* c) {
   r.ndom = g.ndom; r.mrows = g.nproj; r.ncols = g.norb; r.nsplit = c->L.nsplit;
   r.scale = g.dV; r.eps = 0.5 * g.dt;
   LFD_TRY(launch(c, LFD_K_NL_REDUCE, "k_reduce", [&] { return lfd::launch_reduce(r, c->stream); }));
-  LFD_TRY(launch(c, LFD_K_NL_NORM, "k_nlnorm", [&] {
-    return lfd::launch_nlnorm(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), r.out, r.s,
-                              c->at<double>(c->L.nfac), c->stream);
-  }));
+  if (merged)
+    LFD_TRY(launch(c, LFD_K_NL_NORM, "k_nlmerge", [&] {
+      return lfd::launch_nlmerge(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), r.D, r.out, r.s,
+                                 r.cprime, c->at<double>(c->L.nfac), c->stream);
+    }));
+  else
+    LFD_TRY(launch(c, LFD_K_NL_NORM, "k_nlnorm", [&] {
+      return lfd::launch_nlnorm(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), r.out, r.s,
+                                c->at<double>(c->L.nfac), c->stream);
+    }));
   lfd::Gemm2Args a2;
   a2.psi = c->psi; a2.B = c->proj; a2.Cp = r.cprime; a2.nfac = c->at<double>(c->L.nfac);
   a2.ndom = g.ndom; a2.nproj = g.nproj; a2.norb = g.norb; a2.ng = g.ng; a2.num_sms = c->num_sms;
+  a2.variant = c->gemm2_variant;
   return launch(c, LFD_K_NL_BACK, "k_gemm2", [&] { return lfd::launch_gemm2(a2, c->stream); });
 }
 
@@ -389,6 +398,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   c->stream = static_cast<cudaStream_t>(stream);
   c->device = cfg->device;
   c->num_sms = prop.multiProcessorCount;
+  if (const char* v = std::getenv("LFD_GEMM2_VARIANT")) c->gemm2_variant = std::atoi(v);
   {
     std::lock_guard<std::mutex> lk(g_live_mu);
     g_live.insert(c);
@@ -484,6 +494,28 @@ lfd_status lfd_step(lfd_ctx* c, int32_t nsteps) {
     LFD_TRY(launch(c, LFD_K_KIN_Z, "k_kin(z)",
                    [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 2, 2, c->stream); }));
     if (c->g.nproj > 0) LFD_TRY(nl_half(c));
+  }
+  return LFD_OK;
+}
+
+lfd_status lfd_step_sequence(lfd_ctx* c, int32_t nsteps, const double* A_seq) {
+  LFD_TRY(check_ctx(c));
+  if (nsteps < 0) return fail(c, LFD_EINVAL, "nsteps must be >= 0");
+  if (nsteps > 0 && !A_seq) return fail(c, LFD_EINVAL, "A_seq is NULL");
+  for (long long i = 0; i < 3LL * c->g.ndom * nsteps; ++i)
+    if (!std::isfinite(A_seq[i])) return fail(c, LFD_EINVAL, "A_seq must be finite");
+  DeviceGuard dg(c->device);
+  const bool nl = c->g.nproj > 0;
+  for (int n = 0; n < nsteps; ++n) {
+    LFD_TRY(set_A(c, A_seq + 3LL * c->g.ndom * n));
+    if (nl && n == 0) LFD_TRY(nl_half(c));  // first factor of the sequence
+    LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin(x)",
+                   [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 0, 1, c->stream); }));
+    LFD_TRY(launch(c, LFD_K_KIN_Y, "k_kin(y)",
+                   [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 1, 0, c->stream); }));
+    LFD_TRY(launch(c, LFD_K_KIN_Z, "k_kin(z)",
+                   [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 2, 2, c->stream); }));
+    if (nl) LFD_TRY(nl_half(c, n + 1 < nsteps));  // N of step n fused with N of step n+1
   }
   return LFD_OK;
 }

@@ -76,6 +76,11 @@ cudaError_t launch_reduce(const ReduceArgs& a, cudaStream_t st);
 cudaError_t launch_nlnorm(int ndom, int nproj, int norb, double eps, const double2* G,
                           const double2* DC, const double* s, double* nfac, cudaStream_t st);
 
+// Combined factor of two consecutive nonlocal halves (lfd_step_sequence): X = (2c D + c^2 D G D) C
+// written to X (the GEMM-2 C'), nfac from the Gram closed form of ||Psi + B X||.
+cudaError_t launch_nlmerge(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
+                           const double2* DC, const double* s, double2* X, double* nfac, cudaStream_t st);
+
 // GEMM-2 in place: psi[dom][r][n] <- nfac[dom][n] * (psi[dom][r][n] + sum_m B[dom][r][m] Cp[dom][m][n])
 struct Gemm2Args {
   double2* psi;
@@ -85,6 +90,7 @@ struct Gemm2Args {
   int ndom, nproj, norb;
   long long ng;
   int num_sms;
+  int variant;  // tuning knob (LFD_GEMM2_VARIANT): 0 = epilogue loads after the K loop, 1 = mid-loop
 };
 cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st);
 int gemm2_smem_bytes();

@@ -418,6 +418,87 @@ cudaError_t launch_nlnorm(int ndom, int nproj, int norb, double eps, const doubl
 }
 
 // ------------------------------------------------------------------------------------------------
+// Two consecutive nonlocal factors N(N(Psi)) as ONE factor (lfd_step_sequence; no Psi is observed
+// between them). With L(Psi) = Psi + c B D C(Psi), c = -i eps, C = dV B^H Psi and G = dV B^H B:
+//   L(L(Psi)) = Psi + B X,   X = M C,   M = 2c D + c^2 D G D,
+// and since each N restores the column norm, N(N(Psi))_s = L^2(Psi)_s * sqrt(s_s / ||L^2 Psi_s||^2) with
+//   ||Psi_s + B X_s||^2 = s_s + 2 Re(C_s^H X_s) + X_s^H G X_s,  2 Re(C^H X) = -2 eps^2 (DC)^H G (DC).
+// Input DC = D C (k_reduce output); writes X to cprime and the factor to nfac. Block per (orbital, dom).
+// ------------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_nlmerge(int nproj, int norb, double eps, const double2* __restrict__ G,
+                                                 const double* __restrict__ D, const double2* __restrict__ DC,
+                                                 const double* __restrict__ s, double2* __restrict__ X,
+                                                 double* __restrict__ nfac) {
+  extern __shared__ double2 sh[];  // dc[np] | x[np]
+  double2* dcs = sh;
+  double2* xs = sh + nproj;
+  __shared__ double wq[2][8];
+  const int dom = blockIdx.y, col = blockIdx.x;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const double2* Gd = G + (long long)dom * nproj * nproj;
+  const double* Dd = D + (long long)dom * nproj;
+  for (int u = threadIdx.x; u < nproj; u += blockDim.x) dcs[u] = DC[((long long)dom * nproj + u) * norb + col];
+  __syncthreads();
+  auto gdot = [&](int u, const double2* vec, double& tr, double& ti) {  // (G vec)_u, warp-wide
+    const double2* Gu = Gd + (long long)u * nproj;
+    tr = 0.0;
+    ti = 0.0;
+    for (int v = lane; v < nproj; v += 32) {
+      const double2 gv = Gu[v], c = vec[v];
+      tr = fma(gv.x, c.x, fma(-gv.y, c.y, tr));
+      ti = fma(gv.x, c.y, fma(gv.y, c.x, ti));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      tr += __shfl_xor_sync(0xffffffffu, tr, o);
+      ti += __shfl_xor_sync(0xffffffffu, ti, o);
+    }
+  };
+  double q1 = 0.0, q2 = 0.0;
+  for (int u = warp; u < nproj; u += 8) {
+    double yr, yi;
+    gdot(u, dcs, yr, yi);
+    const double2 cu = dcs[u];
+    q1 = fma(cu.x, yr, fma(cu.y, yi, q1));  // Re(conj(DC_u) (G DC)_u)
+    const double du = Dd[u];
+    // X_u = -2 i eps DC_u - eps^2 D_u (G DC)_u
+    const double2 x = make_double2(2.0 * eps * cu.y - eps * eps * du * yr, -2.0 * eps * cu.x - eps * eps * du * yi);
+    if (lane == 0) {
+      xs[u] = x;
+      X[((long long)dom * nproj + u) * norb + col] = x;
+    }
+  }
+  __syncthreads();
+  for (int u = warp; u < nproj; u += 8) {
+    double zr, zi;
+    gdot(u, xs, zr, zi);
+    const double2 xu = xs[u];
+    q2 = fma(xu.x, zr, fma(xu.y, zi, q2));  // Re(conj(X_u) (G X)_u)
+  }
+  if (lane == 0) {
+    wq[0][warp] = q1;
+    wq[1][warp] = q2;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double t1 = 0.0, t2 = 0.0;
+    for (int w = 0; w < 8; ++w) {
+      t1 += wq[0][w];
+      t2 += wq[1][w];
+    }
+    const double sv = s[(long long)dom * norb + col];
+    nfac[(long long)dom * norb + col] = sqrt(sv / (sv - 2.0 * eps * eps * t1 + t2));
+  }
+}
+
+cudaError_t launch_nlmerge(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
+                           const double2* DC, const double* s, double2* X, double* nfac, cudaStream_t st) {
+  dim3 grid(norb, ndom);
+  k_nlmerge<<<grid, 256, 2 * nproj * sizeof(double2), st>>>(nproj, norb, eps, G, D, DC, s, X, nfac);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------------
 // GEMM-2 (persistent): psi[r][n] <- nfac[n] * (psi[r][n] + sum_m B[r][m] Cp[m][n]) for every
 // (dom, 64-row block, 64-column tile) work item; K = nproj in chunks of 16 through the TMA ring.
 // ------------------------------------------------------------------------------------------------
@@ -573,7 +654,7 @@ constexpr int kFullSmem = kFullStages * kFullABytes + kFullCBytes + 4 * 8;
 
 __host__ __device__ constexpr int full_lda(int np) { return ((np + 3) / 4 * 4) % 8 == 0 ? (np + 3) / 4 * 4 + 4 : (np + 3) / 4 * 4; }
 
-template <int kNP>
+template <int kNP, bool kPvMid>
 __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
   extern __shared__ __align__(128) unsigned char smem[];
   double2* Cs = reinterpret_cast<double2*>(smem + kFullStages * kFullABytes);
@@ -640,7 +721,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
       cur_dom = dom;
       cur_n0 = n0;
     }
-    double2* psi = p.psi + (long long)dom * p.ng * p.norb;
     // Psi rows of the NEXT item go to L2 now (the epilogue of this item reads rows prefetched during
     // the previous one), keeping 64 registers free for fragment pipelining.
     if (tid == 32 && j + 1 < my_items) {
@@ -652,16 +732,32 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
     }
     if (tid == 32 && j == 0) {
       const long long rows0 = min((long long)kTile, p.ng - r0);
-      l2_prefetch(psi + r0 * p.norb, (uint32_t)(rows0 * p.norb * 16));
+      l2_prefetch(p.psi + ((long long)dom * p.ng + r0) * p.norb, (uint32_t)(rows0 * p.norb * 16));
     }
     const int stage = (int)(j % kFullStages);
     mbar_wait(&bars[stage], (uint32_t)((j / kFullStages) & 1));
     const double2* As = reinterpret_cast<const double2*>(smem + stage * kFullABytes);
     Frag acc;
     acc.zero();
+    double2* psi = p.psi + (long long)dom * p.ng * p.norb;
+    double2 pv[4][2][2];
+    auto load_pv = [&]() {
+#pragma unroll
+      for (int mi = 0; mi < 4; ++mi) {
+        const long long r = r0 + wm * 32 + mi * 8 + g;
+#pragma unroll
+        for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+          for (int c = 0; c < 2; ++c) {
+            const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
+            pv[mi][ni][c] = (r < p.ng && col < p.norb) ? psi[r * p.norb + col] : cz();
+          }
+      }
+    };
 #pragma unroll
     for (int kk = 0; kk < kNK4; ++kk) {
       if (kNP == 0 && kk >= nk4) break;
+      if (kPvMid && kk == kNK4 / 2) load_pv();  // Psi loads in flight during the second half
       const int k = kk * 4 + t;
       const bool ok = (kNP > 0 && kNP % 4 == 0) || k < np;
       double2 a[4], c[2];
@@ -671,22 +767,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
       for (int ni = 0; ni < 2; ++ni) c[ni] = ok ? Cs[k * kLd1 + wn * 16 + ni * 8 + g] : cz();
       mma_4x2(acc, a, c);
     }
+    if (!kPvMid || (kNP == 0 && nk4 <= kNK4 / 2)) load_pv();
     __syncthreads();  // stage and Cs free
     if (warp == 0 && j + kFullStages < my_items) issue(j + kFullStages, stage);
-    // epilogue: Psi <- n_s (Psi + B C'); all 16 loads (L2 hits, prefetched) are issued before any store
+    // epilogue: Psi <- n_s (Psi + B C') (the Psi loads were issued above; L2 hits, prefetched)
     const double* nf = p.nfac + (long long)dom * p.norb;
-    double2 pv[4][2][2];
-#pragma unroll
-    for (int mi = 0; mi < 4; ++mi) {
-      const long long r = r0 + wm * 32 + mi * 8 + g;
-#pragma unroll
-      for (int ni = 0; ni < 2; ++ni)
-#pragma unroll
-        for (int c = 0; c < 2; ++c) {
-          const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
-          pv[mi][ni][c] = (r < p.ng && col < p.norb) ? psi[r * p.norb + col] : cz();
-        }
-    }
 #pragma unroll
     for (int ni = 0; ni < 2; ++ni)
 #pragma unroll
@@ -709,10 +794,12 @@ cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
   const long long rblocks = (a.ng + kTile - 1) / kTile;
   const long long items = (long long)a.ndom * rblocks * ((a.norb + kTile - 1) / kTile);
   const int grid = (int)(items < a.num_sms ? items : a.num_sms);
-  if (a.nproj == kTile)
-    k_gemm2_fullk<kTile><<<grid, kThreads, kFullSmem, st>>>(a);
+  if (a.nproj == kTile && a.variant == 1)
+    k_gemm2_fullk<kTile, true><<<grid, kThreads, kFullSmem, st>>>(a);
+  else if (a.nproj == kTile)
+    k_gemm2_fullk<kTile, false><<<grid, kThreads, kFullSmem, st>>>(a);
   else if (a.nproj < kTile)
-    k_gemm2_fullk<0><<<grid, kThreads, kFullSmem, st>>>(a);
+    k_gemm2_fullk<0, false><<<grid, kThreads, kFullSmem, st>>>(a);
   else
     k_gemm2<<<grid, kThreads, gemm2_smem_bytes(), st>>>(a);
   return cudaGetLastError();
@@ -721,9 +808,11 @@ cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
 cudaError_t gemm_set_attributes() {
   cudaError_t e = cudaFuncSetAttribute(k_gemm1, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm1_smem_bytes());
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_gemm2_fullk<kTile>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
+  e = cudaFuncSetAttribute(k_gemm2_fullk<kTile, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_gemm2_fullk<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
+  e = cudaFuncSetAttribute(k_gemm2_fullk<kTile, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_gemm2_fullk<0, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(k_gemm2, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm2_smem_bytes());
 }

@@ -25,7 +25,7 @@ STATUS = {0: "LFD_OK", -1: "LFD_EINVAL", -2: "LFD_ENOMEM", -3: "LFD_ECUDA", -4: 
 KERNELS = ("coef", "phase", "kin_x", "kin_y", "kin_z", "nl_proj", "nl_reduce", "nl_norm", "nl_back",
            "density", "jreduce", "energy")
 EXPORTS = ("lfd_workspace_size", "lfd_init", "lfd_set_potential", "lfd_set_potential_host",
-           "lfd_set_vector_potential", "lfd_step", "lfd_density_current", "lfd_density_current_global",
+           "lfd_set_vector_potential", "lfd_step", "lfd_step_sequence", "lfd_density_current", "lfd_density_current_global",
            "lfd_density_current_host", "lfd_energy", "lfd_remap_occ", "lfd_set_occupations", "lfd_set_stream", "lfd_sync",
            "lfd_launch_count", "lfd_profile_enable", "lfd_profile_read", "lfd_last_error", "lfd_destroy")
 
@@ -63,6 +63,7 @@ def load():
         "lfd_set_potential_host": [P, P],
         "lfd_set_vector_potential": [P, P],
         "lfd_step": [P, I32],
+        "lfd_step_sequence": [P, I32, P],
         "lfd_density_current": [P, P, P, P],
         "lfd_density_current_global": [P, P, P, P, P, P],
         "lfd_density_current_host": [P, P, P],
@@ -157,6 +158,13 @@ def lfd_set_vector_potential(ctx, A):
 
 def lfd_step(ctx, nsteps: int = 1):
     _check(load().lfd_step(ctx, int(nsteps)), ctx)
+
+
+def lfd_step_sequence(ctx, A_seq):
+    """A_seq: host [nsteps, ndom, 3]; nsteps steps with merged adjacent nonlocal factors."""
+    arr = np.ascontiguousarray(A_seq, dtype=np.float64)
+    p, _k = _hptr(arr)
+    _check(load().lfd_step_sequence(ctx, int(arr.shape[0]), p), ctx)
 
 
 def lfd_density_current(ctx, rho, j=None, Jmac=None):
@@ -258,6 +266,9 @@ class Context:
 
     def step(self, n: int = 1):
         lfd_step(self.ctx, n)
+
+    def step_sequence(self, A_seq):
+        lfd_step_sequence(self.ctx, A_seq)
 
     def density_current(self, want_j: bool = True):
         import torch

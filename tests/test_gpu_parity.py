@@ -258,3 +258,40 @@ def test_launch_count_and_profile():
     assert prof["kin_x"][1] == 2 and prof["nl_proj"][1] == 4 and prof["nl_back"][1] == 4
     assert all(v[0] >= 0 for v in prof.values())
     ctx.close()
+
+
+def run_gpu_sequence(w, x, steps, A_fn, chunk=None):
+    torch = _torch()
+    from paper_conf_ipps_razakhllknvn24_b200 import Context
+    dev = torch.device("cuda:0")
+    psi = torch.from_numpy(x.psi0.copy()).to(dev)
+    proj = torch.from_numpy(x.proj).to(dev) if w.nproj > 0 else None
+    ctx = Context(psi, proj, x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc)
+    ctx.set_potential(torch.from_numpy(x.vloc).to(dev))
+    A_seq = np.stack([A_fn(n) for n in range(steps)])
+    chunk = chunk or steps
+    for s0 in range(0, steps, chunk):
+        ctx.step_sequence(A_seq[s0:s0 + chunk])
+    rho, j, J = ctx.density_current()
+    ctx.sync()
+    out = (psi.cpu().numpy(), rho.cpu().numpy().reshape(w.ndom, -1), j.cpu().numpy().reshape(w.ndom, 3, -1),
+           J.cpu().numpy())
+    ctx.close()
+    return out
+
+
+@pytest.mark.parametrize("name,steps,chunk", [("P0", 100, None), ("P1", 20, 7), ("P2z", 20, None), ("P3", 6, None),
+                                              ("C1", 30, None)])
+def test_step_sequence_parity(name, steps, chunk):
+    """lfd_step_sequence (adjacent nonlocal factors merged, N o N = renormalised L^2) equals the oracle
+    stepping one Eq.-6 step at a time with the same per-step A."""
+    w = workload(name) if name != "C1" else workload("C1").with_(laser=True, e0=0.02, pol=(0.3, -0.4, 0.87))
+    x = make_inputs(w, seed=31)
+    assert_parity(w, run_gpu_sequence(w, x, steps, laser(w), chunk), run_ref(w, x, steps, laser(w)))
+
+
+def test_c2_full_size_sequence():
+    """The merged-factor sequence at the bench size (C2), 3 steps, vs the oracle."""
+    w = workload("C2")
+    x = make_inputs(w, seed=2)
+    assert_parity(w, run_gpu_sequence(w, x, 3, laser(w)), run_ref(w, x, 3, laser(w)))
