@@ -38,7 +38,7 @@
 extern "C" {
 #endif
 
-#define LFD_ABI_VERSION 2
+#define LFD_ABI_VERSION 3
 #define LFD_MAX_DOMAINS 4096
 
 typedef struct lfd_ctx lfd_ctx; /* opaque */
@@ -65,16 +65,22 @@ typedef struct {
   int32_t nref_max;    /* max reference-basis columns for lfd_remap_occ, 0..2048 (0: max(norb, nproj)) */
   double dt;           /* Delta_QD [a.u.], finite and nonzero (negative = backward in time) */
   int32_t device;      /* CUDA device ordinal */
-  int32_t flags;       /* reserved, must be 0 */
+  int32_t flags;       /* 0 or LFD_FLAG_NO_CARRY */
 } lfd_config;
+
+/* lfd_config.flags: disable the projection carry (lfd_step takes the C of each nonlocal factor that
+ * directly follows another one from C_new = (C + G C') diag(n), an exact identity, instead of
+ * recomputing dV B^H Psi by GEMM-1). With the flag every factor runs its GEMM-1; results agree to
+ * roundoff. */
+#define LFD_FLAG_NO_CARRY 1
 
 /* Kernel classes, for lfd_profile_read(). */
 typedef enum {
   LFD_K_COEF = 0,      /* a1: stencil coefficients from A(t) */
   LFD_K_PHASE = 1,     /* a2: Phi = exp(-i Delta/2 v_loc) */
   LFD_K_KIN_X = 2,     /* a6: Phi . K_x (pre-phase fused) */
-  LFD_K_KIN_Y = 3,     /* a6: K_y */
-  LFD_K_KIN_Z = 4,     /* a6: K_z . Phi (post-phase fused) */
+  LFD_K_KIN_Y = 3,     /* a6: K_y (unfused path) */
+  LFD_K_KIN_Z = 4,     /* a6: K_z . Phi (post-phase fused; unfused path) */
   LFD_K_NL_PROJ = 5,   /* a3: GEMM-1 split-K partials of C = dV B^H Psi + column norms */
   LFD_K_NL_REDUCE = 6, /* a4: fixed-order split-K reduction, C' = -i(Delta/2) D C */
   LFD_K_NL_NORM = 7,   /* a4: n_s from the Gram closed form */
@@ -82,14 +88,20 @@ typedef enum {
   LFD_K_DENSITY = 9,   /* a7: rho, j, per-line partial J */
   LFD_K_JREDUCE = 10,  /* a7: J = mean of j (fixed order) */
   LFD_K_ENERGY = 11,   /* NEXT f-1: energy / occupation reductions (calc_energy, remap_occ) */
-  LFD_K_COUNT = 12
+  LFD_K_NL_CARRY = 12, /* a3/a4: projection carry C_new = (C + G C') diag(n) (replaces GEMM-1) */
+  LFD_K_KIN_YZ = 13,   /* a6: K_y K_z . Phi fused in one pass (post-phase fused) */
+  LFD_K_COUNT = 14
 } lfd_kernel_id;
 
 /* Bytes of DEVICE workspace lfd_init needs for this configuration. */
 lfd_status lfd_workspace_size(const lfd_config* cfg, size_t* bytes);
 
 /* Create a context.
- *  psi   DEVICE complex128 [ndom][nx][ny][nz][norb]; borrowed; propagated in place by lfd_step.
+ *  psi   DEVICE complex128 [ndom][nx][ny][nz][norb]; borrowed; propagated in place by lfd_step. Like the
+ *        paper's GPU-resident Psi(t), it belongs to the library while the context is live: the
+ *        caller may read it (after lfd_sync or in stream order) but must call lfd_psi_modified() after
+ *        writing it, because the context keeps the projection C = dV B^H Psi of the last nonlocal
+ *        factor for the next one (see LFD_FLAG_NO_CARRY).
  *  proj  DEVICE complex128 [ndom][nx][ny][nz][nproj]; borrowed, read-only (B = Psi_u(0), the
  *        unoccupied KS orbitals at t = 0, Eq. 7 P:68 / R9); NULL iff nproj == 0. Need not be
  *        orthonormal: the Gram matrix G = dV B^H B is computed here (on the device) and used for n_s.
@@ -163,6 +175,10 @@ lfd_status lfd_energy(lfd_ctx* ctx, double* E);
  *  ref     DEVICE complex128 [ndom][nx][ny][nz][nref], 1 <= nref <= nref_max (config); read-only.
  *  occ_out DEVICE double [ndom][nref]. Stream-ordered. */
 lfd_status lfd_remap_occ(lfd_ctx* ctx, const void* ref, int32_t nref, double* occ_out);
+
+/* Tell the context that the caller wrote psi (drops the kept projection; the next nonlocal factor
+ * recomputes C = dV B^H Psi by GEMM-1). */
+lfd_status lfd_psi_modified(lfd_ctx* ctx);
 
 /* Replace the occupations f (the QXMD<->LFD shadow-dynamics handshake). HOST [ndom][norb]. */
 lfd_status lfd_set_occupations(lfd_ctx* ctx, const double* occ);

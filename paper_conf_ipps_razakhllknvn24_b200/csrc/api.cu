@@ -61,7 +61,7 @@ lfd_status validate(const lfd_config* c, std::string& why) {
   if (c->norb < 1) { why = "norb must be >= 1"; return LFD_EINVAL; }
   if (c->nproj < 0 || c->nproj > 2048) { why = "nproj must be in [0, 2048]"; return LFD_EINVAL; }
   if (!(c->dt != 0.0) || !std::isfinite(c->dt)) { why = "dt must be finite and nonzero"; return LFD_EINVAL; }
-  if (c->flags != 0) { why = "flags must be 0"; return LFD_EINVAL; }
+  if (c->flags & ~LFD_FLAG_NO_CARRY) { why = "unknown flags"; return LFD_EINVAL; }
   if (c->nref_max < 0 || c->nref_max > 2048) { why = "nref_max must be in [0, 2048]"; return LFD_EINVAL; }
   const long long ng = (long long)c->nx * c->ny * c->nz;
   if (ng * (long long)std::max(c->norb, std::max(c->nproj, 1)) >= (1LL << 31)) {
@@ -164,6 +164,12 @@ struct lfd_ctx {
   int num_sms;
   uint64_t launches = 0;
   int gemm2_variant = 1;  // internal tuning knob, env LFD_GEMM2_VARIANT (1 measured faster)
+  // Projection carry: true while the workspace's DC / C' / s / n describe the GEMM-2 that produced the
+  // current Psi, so the next nonlocal factor can take C from the exact identity C_new = (C + G X) n
+  // instead of GEMM-1 (cleared by the local propagator, lfd_psi_modified and LFD_FLAG_NO_CARRY).
+  bool c_valid = false;
+  bool carry = true;
+  bool kin_fused = true;  // Phi.K_y K_z in one pass (env LFD_KIN_FUSED=0: separate y and z passes)
   std::string err = "no error";
   // density-current global layout cache
   std::vector<long long> gbase_host;
@@ -262,9 +268,43 @@ bool is_device_ptr(const void* p) {
   return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
+// GEMM-2 of a nonlocal factor: Psi <- (Psi + B C') diag(n), C' and n from the workspace.
+lfd_status gemm2(lfd_ctx* c) {
+  const Geometry& g = c->g;
+  lfd::Gemm2Args a2;
+  a2.psi = c->psi; a2.B = c->proj; a2.Cp = c->at<double2>(c->L.cprime); a2.nfac = c->at<double>(c->L.nfac);
+  a2.ndom = g.ndom; a2.nproj = g.nproj; a2.norb = g.norb; a2.ng = g.ng; a2.num_sms = c->num_sms;
+  a2.variant = c->gemm2_variant;
+  c->c_valid = false;
+  LFD_TRY(launch(c, LFD_K_NL_BACK, "k_gemm2", [&] { return lfd::launch_gemm2(a2, c->stream); }));
+  c->c_valid = c->carry;
+  return LFD_OK;
+}
+
 // Eq. 6 nonlocal factor N on every domain (kernels a3, a4, a5); merged = N o N in one pass.
 lfd_status nl_half(lfd_ctx* c, bool merged = false) {
   const Geometry& g = c->g;
+  if (c->c_valid) {  // C of the current Psi from the previous factor (no GEMM-1, no reduction)
+    double* D = c->at<double>(c->L.D);
+    double2* DC = c->at<double2>(c->L.dc);
+    double2* X = c->at<double2>(c->L.cprime);
+    double* s = c->at<double>(c->L.s);
+    double* nfac = c->at<double>(c->L.nfac);
+    LFD_TRY(launch(c, LFD_K_NL_CARRY, "k_nlcarry", [&] {
+      return lfd::launch_nlcarry(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), D, DC, X, nfac,
+                                 c->stream);
+    }));
+    if (merged)
+      LFD_TRY(launch(c, LFD_K_NL_NORM, "k_nlmerge", [&] {
+        return lfd::launch_nlmerge(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), D, DC, s, X, nfac,
+                                   c->stream);
+      }));
+    else
+      LFD_TRY(launch(c, LFD_K_NL_NORM, "k_nlnorm", [&] {
+        return lfd::launch_nlnorm(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), DC, s, nfac, c->stream);
+      }));
+    return gemm2(c);
+  }
   lfd::Gemm1Args a1;
   a1.A = c->proj;
   a1.X = c->psi;
@@ -293,11 +333,21 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false) {
       return lfd::launch_nlnorm(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), r.out, r.s,
                                 c->at<double>(c->L.nfac), c->stream);
     }));
-  lfd::Gemm2Args a2;
-  a2.psi = c->psi; a2.B = c->proj; a2.Cp = r.cprime; a2.nfac = c->at<double>(c->L.nfac);
-  a2.ndom = g.ndom; a2.nproj = g.nproj; a2.norb = g.norb; a2.ng = g.ng; a2.num_sms = c->num_sms;
-  a2.variant = c->gemm2_variant;
-  return launch(c, LFD_K_NL_BACK, "k_gemm2", [&] { return lfd::launch_gemm2(a2, c->stream); });
+  return gemm2(c);
+}
+
+// Local factor exp(-i Delta h_loc) of Eq. 6: Psi <- Phi . K_z K_y K_x (Phi . Psi) (kernels a6).
+lfd_status local_prop(lfd_ctx* c) {
+  c->c_valid = false;
+  LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin(x)",
+                 [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 0, 1, c->stream); }));
+  if (c->kin_fused)
+    return launch(c, LFD_K_KIN_YZ, "k_kin_yz",
+                  [&] { return lfd::launch_kin_yz(c->g, c->psi, c->coef(), c->phi(), c->stream); });
+  LFD_TRY(launch(c, LFD_K_KIN_Y, "k_kin(y)",
+                 [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 1, 0, c->stream); }));
+  return launch(c, LFD_K_KIN_Z, "k_kin(z)",
+                [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 2, 2, c->stream); });
 }
 
 // C[dom][m][n] = dV sum_r conj(A[r][m]) Psi[r][n] into out (GEMM-1 + fixed-order reduction).
@@ -386,6 +436,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   if (ws_bytes < L.total) return fail(nullptr, LFD_ENOMEM, "workspace smaller than lfd_workspace_size()");
   cudaError_t e = lfd::gemm_set_attributes();
   if (e == cudaSuccess) e = lfd::density_set_attributes();
+  if (e == cudaSuccess) e = lfd::kin_yz_set_attributes();
   if (e != cudaSuccess) return cuda_fail(nullptr, e, "cudaFuncSetAttribute");
 
   lfd_ctx* c = new (std::nothrow) lfd_ctx();
@@ -399,6 +450,9 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   c->device = cfg->device;
   c->num_sms = prop.multiProcessorCount;
   if (const char* v = std::getenv("LFD_GEMM2_VARIANT")) c->gemm2_variant = std::atoi(v);
+  c->carry = (cfg->flags & LFD_FLAG_NO_CARRY) == 0;
+  if (const char* v = std::getenv("LFD_KIN_FUSED")) c->kin_fused = std::atoi(v) != 0;
+  c->kin_fused = c->kin_fused && lfd::kin_yz_supported(g);
   {
     std::lock_guard<std::mutex> lk(g_live_mu);
     g_live.insert(c);
@@ -487,12 +541,7 @@ lfd_status lfd_step(lfd_ctx* c, int32_t nsteps) {
   DeviceGuard dg(c->device);
   for (int it = 0; it < nsteps; ++it) {
     if (c->g.nproj > 0) LFD_TRY(nl_half(c));
-    LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin(x)",
-                   [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 0, 1, c->stream); }));
-    LFD_TRY(launch(c, LFD_K_KIN_Y, "k_kin(y)",
-                   [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 1, 0, c->stream); }));
-    LFD_TRY(launch(c, LFD_K_KIN_Z, "k_kin(z)",
-                   [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 2, 2, c->stream); }));
+    LFD_TRY(local_prop(c));
     if (c->g.nproj > 0) LFD_TRY(nl_half(c));
   }
   return LFD_OK;
@@ -509,12 +558,7 @@ lfd_status lfd_step_sequence(lfd_ctx* c, int32_t nsteps, const double* A_seq) {
   for (int n = 0; n < nsteps; ++n) {
     LFD_TRY(set_A(c, A_seq + 3LL * c->g.ndom * n));
     if (nl && n == 0) LFD_TRY(nl_half(c));  // first factor of the sequence
-    LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin(x)",
-                   [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 0, 1, c->stream); }));
-    LFD_TRY(launch(c, LFD_K_KIN_Y, "k_kin(y)",
-                   [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 1, 0, c->stream); }));
-    LFD_TRY(launch(c, LFD_K_KIN_Z, "k_kin(z)",
-                   [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 2, 2, c->stream); }));
+    LFD_TRY(local_prop(c));
     if (nl) LFD_TRY(nl_half(c, n + 1 < nsteps));  // N of step n fused with N of step n+1
   }
   return LFD_OK;
@@ -621,6 +665,12 @@ lfd_status lfd_set_occupations(lfd_ctx* c, const double* occ) {
   cudaError_t e = cudaMemcpyAsync(c->at<double>(c->L.occ), occ, sizeof(double) * c->g.ndom * c->g.norb,
                                   cudaMemcpyHostToDevice, c->stream);
   if (e != cudaSuccess) return cuda_fail(c, e, "copy occ");
+  return LFD_OK;
+}
+
+lfd_status lfd_psi_modified(lfd_ctx* c) {
+  LFD_TRY(check_ctx(c));
+  c->c_valid = false;
   return LFD_OK;
 }
 

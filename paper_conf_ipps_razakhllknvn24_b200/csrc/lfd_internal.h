@@ -43,6 +43,12 @@ cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, doubl
 cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, const double2* phi,
                        int axis, int phase_mode, cudaStream_t st);
 
+// Fused pass Psi <- Phi . K_y K_z Psi (one read + write of Psi; nz <= 128).
+bool kin_yz_supported(const Geometry& g);
+cudaError_t launch_kin_yz(const Geometry& g, double2* psi, const DomCoef* coef, const double2* phi,
+                          cudaStream_t st);
+cudaError_t kin_yz_set_attributes();
+
 // GEMM-1 split-K: part[dom][split][mrows][ncols] (complex) = sum over the split's grid rows of
 // conj(A[r][m]) X[r][n]; if norms != nullptr also norms[dom][split][n] = sum |X[r][n]|^2.
 // A: [dom][ng][mrows], X: [dom][ng][ncols] complex.
@@ -80,6 +86,11 @@ cudaError_t launch_nlnorm(int ndom, int nproj, int norb, double eps, const doubl
 // written to X (the GEMM-2 C'), nfac from the Gram closed form of ||Psi + B X||.
 cudaError_t launch_nlmerge(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
                            const double2* DC, const double* s, double2* X, double* nfac, cudaStream_t st);
+
+// Projection carry after a GEMM-2 Psi <- (Psi + B X) diag(n): DC <- (DC + D (G X)) diag(n) and
+// X <- -i eps DC (the C' of the next nonlocal factor), in place; column norms s are unchanged.
+cudaError_t launch_nlcarry(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
+                           double2* DC, double2* X, const double* nfac, cudaStream_t st);
 
 // GEMM-2 in place: psi[dom][r][n] <- nfac[dom][n] * (psi[dom][r][n] + sum_m B[dom][r][m] Cp[dom][m][n])
 struct Gemm2Args {

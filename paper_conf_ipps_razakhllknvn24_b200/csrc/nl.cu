@@ -499,6 +499,60 @@ cudaError_t launch_nlmerge(int ndom, int nproj, int norb, double eps, const doub
 }
 
 // ------------------------------------------------------------------------------------------------
+// Projection carry (no GEMM): the GEMM-2 that just ran wrote Psi_new = (Psi + B X) diag(n), so
+//   C_new = dV B^H Psi_new = (C + G X) diag(n)       (G = dV B^H B, exact identity)
+// and, with DC = D C, DC_new = (DC + D (G X)) diag(n); C'_new = -i eps DC_new. The column norms are
+// unchanged (n restores them), so s is kept. Block per (orbital s, domain); column s only is read and
+// written (X and DC are read into shared memory before any write). Replaces GEMM-1 + k_reduce of the
+// next nonlocal factor when nothing touched Psi in between (lfd_step: N of step n, then N of n+1).
+// ------------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps, const double2* __restrict__ G,
+                                                 const double* __restrict__ D, double2* DC, double2* X,
+                                                 const double* __restrict__ nfac) {
+  extern __shared__ double2 sh[];  // x[np] | dc[np]
+  double2* xs = sh;
+  double2* dcs = sh + nproj;
+  const int dom = blockIdx.y, col = blockIdx.x;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const double2* Gd = G + (long long)dom * nproj * nproj;
+  const double* Dd = D + (long long)dom * nproj;
+  const long long cb = (long long)dom * nproj * norb + col;
+  for (int u = threadIdx.x; u < nproj; u += blockDim.x) {
+    xs[u] = X[cb + (long long)u * norb];
+    dcs[u] = DC[cb + (long long)u * norb];
+  }
+  __syncthreads();
+  const double n = nfac[(long long)dom * norb + col];
+  for (int u = warp; u < nproj; u += 8) {
+    const double2* Gu = Gd + (long long)u * nproj;
+    double tr = 0.0, ti = 0.0;
+    for (int v = lane; v < nproj; v += 32) {
+      const double2 gv = Gu[v], x = xs[v];
+      tr = fma(gv.x, x.x, fma(-gv.y, x.y, tr));
+      ti = fma(gv.x, x.y, fma(gv.y, x.x, ti));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      tr += __shfl_xor_sync(0xffffffffu, tr, o);
+      ti += __shfl_xor_sync(0xffffffffu, ti, o);
+    }
+    if (lane == 0) {
+      const double du = Dd[u];
+      const double2 d = make_double2(n * fma(du, tr, dcs[u].x), n * fma(du, ti, dcs[u].y));
+      DC[cb + (long long)u * norb] = d;
+      X[cb + (long long)u * norb] = make_double2(eps * d.y, -eps * d.x);  // -i eps DC_new
+    }
+  }
+}
+
+cudaError_t launch_nlcarry(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
+                           double2* DC, double2* X, const double* nfac, cudaStream_t st) {
+  dim3 grid(norb, ndom);
+  k_nlcarry<<<grid, 256, 2 * nproj * sizeof(double2), st>>>(nproj, norb, eps, G, D, DC, X, nfac);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------------
 // GEMM-2 (persistent): psi[r][n] <- nfac[n] * (psi[r][n] + sum_m B[r][m] Cp[m][n]) for every
 // (dom, 64-row block, 64-column tile) work item; K = nproj in chunks of 16 through the TMA ring.
 // ------------------------------------------------------------------------------------------------

@@ -17,16 +17,17 @@ import numpy as np
 HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "liblfd.so")
 
-LFD_ABI_VERSION = 2
+LFD_ABI_VERSION = 3
+LFD_FLAG_NO_CARRY = 1
 LFD_BC_PERIODIC = 0
 LFD_BC_ZERO = 1
 STATUS = {0: "LFD_OK", -1: "LFD_EINVAL", -2: "LFD_ENOMEM", -3: "LFD_ECUDA", -4: "LFD_ESTATE",
           -5: "LFD_EUNSUPPORTED"}
 KERNELS = ("coef", "phase", "kin_x", "kin_y", "kin_z", "nl_proj", "nl_reduce", "nl_norm", "nl_back",
-           "density", "jreduce", "energy")
+           "density", "jreduce", "energy", "nl_carry", "kin_yz")
 EXPORTS = ("lfd_workspace_size", "lfd_init", "lfd_set_potential", "lfd_set_potential_host",
            "lfd_set_vector_potential", "lfd_step", "lfd_step_sequence", "lfd_density_current", "lfd_density_current_global",
-           "lfd_density_current_host", "lfd_energy", "lfd_remap_occ", "lfd_set_occupations", "lfd_set_stream", "lfd_sync",
+           "lfd_density_current_host", "lfd_energy", "lfd_remap_occ", "lfd_psi_modified", "lfd_set_occupations", "lfd_set_stream", "lfd_sync",
            "lfd_launch_count", "lfd_profile_enable", "lfd_profile_read", "lfd_last_error", "lfd_destroy")
 
 
@@ -70,6 +71,7 @@ def load():
         "lfd_energy": [P, P],
         "lfd_remap_occ": [P, P, I32, P],
         "lfd_set_occupations": [P, P],
+        "lfd_psi_modified": [P],
         "lfd_set_stream": [P, P],
         "lfd_sync": [P],
         "lfd_launch_count": [P, C.POINTER(C.c_uint64)],
@@ -121,8 +123,10 @@ def _stream_ptr(stream=None):
     return C.c_void_p(s.cuda_stream)
 
 
-def make_config(ndomains, nx, ny, nz, hx, hy, hz, bc, norb, nproj, dt, device=0, nref_max=0) -> lfd_config:
-    return lfd_config(LFD_ABI_VERSION, ndomains, nx, ny, nz, hx, hy, hz, bc, norb, nproj, nref_max, dt, device, 0)
+def make_config(ndomains, nx, ny, nz, hx, hy, hz, bc, norb, nproj, dt, device=0, nref_max=0,
+                flags=0) -> lfd_config:
+    return lfd_config(LFD_ABI_VERSION, ndomains, nx, ny, nz, hx, hy, hz, bc, norb, nproj, nref_max, dt, device,
+                      flags)
 
 
 # ---- 1:1 wrappers of the C entry points --------------------------------------------------------
@@ -193,6 +197,10 @@ def lfd_remap_occ(ctx, ref, occ_out):
     _check(load().lfd_remap_occ(ctx, _dptr(ref), int(ref.shape[-1]), _dptr(occ_out)), ctx)
 
 
+def lfd_psi_modified(ctx):
+    _check(load().lfd_psi_modified(ctx), ctx)
+
+
 def lfd_set_occupations(ctx, occ):
     p, _k = _hptr(occ)
     _check(load().lfd_set_occupations(ctx, p), ctx)
@@ -241,14 +249,14 @@ class Context:
     (host arrays). h = (hx, hy, hz).
     """
 
-    def __init__(self, psi, proj, dnl, occ, h, dt, bc=LFD_BC_PERIODIC, stream=None, nref_max=0):
+    def __init__(self, psi, proj, dnl, occ, h, dt, bc=LFD_BC_PERIODIC, stream=None, nref_max=0, flags=0):
         import torch
         if psi.dtype != torch.complex128 or psi.dim() != 5:
             raise TypeError("psi must be complex128 [ndom, nx, ny, nz, norb]")
         ndom, nx, ny, nz, norb = psi.shape
         nproj = 0 if proj is None else proj.shape[-1]
         self.cfg = make_config(ndom, nx, ny, nz, h[0], h[1], h[2], bc, norb, nproj, dt,
-                               device=psi.device.index or 0, nref_max=nref_max)
+                               device=psi.device.index or 0, nref_max=nref_max, flags=flags)
         self.psi, self.proj = psi, proj
         ws = lfd_workspace_size(self.cfg)
         self.workspace = torch.empty(max(ws, 1), dtype=torch.uint8, device=psi.device)
@@ -291,6 +299,9 @@ class Context:
         out = torch.empty((self.shape[0], ref.shape[-1]), dtype=torch.float64, device=self.psi.device)
         lfd_remap_occ(self.ctx, ref, out)
         return out
+
+    def psi_modified(self):
+        lfd_psi_modified(self.ctx)
 
     def sync(self):
         lfd_sync(self.ctx)

@@ -26,13 +26,14 @@ def _torch():
     return torch
 
 
-def run_gpu(w, x, steps, A_fn, dnl=None):
+def run_gpu(w, x, steps, A_fn, dnl=None, flags=0):
     torch = _torch()
     from paper_conf_ipps_razakhllknvn24_b200 import Context
     dev = torch.device("cuda:0")
     psi = torch.from_numpy(x.psi0.copy()).to(dev)
     proj = torch.from_numpy(x.proj).to(dev) if w.nproj > 0 else None
-    ctx = Context(psi, proj, x.dnl if dnl is None else dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc)
+    ctx = Context(psi, proj, x.dnl if dnl is None else dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc,
+                  flags=flags)
     ctx.set_potential(torch.from_numpy(x.vloc).to(dev))
     A = np.zeros((w.ndom, 3))
     for n in range(steps):
@@ -254,8 +255,11 @@ def test_launch_count_and_profile():
     lfd.lfd_profile_enable(ctx.ctx, True)
     ctx.step(2)
     prof = lfd.lfd_profile_read(ctx.ctx)
-    assert lfd.lfd_launch_count(ctx.ctx) - n0 == 2 * 11
-    assert prof["kin_x"][1] == 2 and prof["nl_proj"][1] == 4 and prof["nl_back"][1] == 4
+    # step 1: N (GEMM-1, reduce, norm, GEMM-2), 3 stencil passes, N; step 2's first N takes C from the
+    # projection carry (carry, norm, GEMM-2) instead of GEMM-1 + reduce
+    assert lfd.lfd_launch_count(ctx.ctx) - n0 == 11 + 10
+    assert prof["kin_x"][1] == 2 and prof["nl_proj"][1] == 3 and prof["nl_back"][1] == 4
+    assert prof["nl_carry"][1] == 1
     assert all(v[0] >= 0 for v in prof.values())
     ctx.close()
 
@@ -295,3 +299,53 @@ def test_c2_full_size_sequence():
     w = workload("C2")
     x = make_inputs(w, seed=2)
     assert_parity(w, run_gpu_sequence(w, x, 3, laser(w)), run_ref(w, x, 3, laser(w)))
+
+
+@pytest.mark.parametrize("name,steps", [("P0", 60), ("P3", 6), ("C1", 12)])
+def test_projection_carry_vs_no_carry(name, steps):
+    """The projection carry (C of a factor that directly follows another from C_new = (C + G C') n)
+    agrees with recomputing C by GEMM-1 every factor (LFD_FLAG_NO_CARRY) to roundoff, and both meet
+    the oracle."""
+    from paper_conf_ipps_razakhllknvn24_b200 import lfd
+    w = workload(name) if name != "C1" else workload("C1").with_(laser=True, e0=0.02, pol=(0.3, -0.4, 0.87))
+    x = make_inputs(w, seed=41)
+    a = run_gpu(w, x, steps, laser(w))
+    b = run_gpu(w, x, steps, laser(w), flags=lfd.LFD_FLAG_NO_CARRY)
+    assert rel(a[0], b[0]) < 1e-13
+    want = run_ref(w, x, steps, laser(w))
+    assert_parity(w, a, want)
+    assert_parity(w, b, want)
+
+
+def test_psi_modified_drops_the_carry():
+    """Writing psi between steps and calling lfd_psi_modified gives the oracle's result from the
+    written state (the kept projection is not reused)."""
+    torch = _torch()
+    from oracle import ref
+    from paper_conf_ipps_razakhllknvn24_b200 import Context
+    w = workload("P0")
+    x = make_inputs(w, seed=42)
+    dev = torch.device("cuda:0")
+    psi = torch.from_numpy(x.psi0.copy()).to(dev)
+    ctx = Context(psi, torch.from_numpy(x.proj).to(dev), x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc)
+    ctx.set_potential(torch.from_numpy(x.vloc).to(dev))
+    cfg = ref.RefConfig(w.ndom, w.nx, w.ny, w.nz, w.hx, w.hy, w.hz, w.bc, w.norb, w.nproj, w.dt)
+    p = x.psi0.copy()
+    phase = np.exp(0.7j * np.arange(w.norb))
+    for n in range(6):
+        A = midpoint_A(w, n)
+        if n == 3:  # the caller rotates every orbital's phase and swaps two orbitals
+            ctx.sync()
+            q = psi.cpu().numpy() * phase
+            q[..., [0, 1]] = q[..., [1, 0]]
+            psi.copy_(torch.from_numpy(np.ascontiguousarray(q)))
+            ctx.psi_modified()
+            p = p * phase
+            p[..., [0, 1]] = p[..., [1, 0]]
+            p = np.ascontiguousarray(p)
+        ctx.set_vector_potential(A)
+        ctx.step(1)
+        ref.step(cfg, p, x.proj, x.dnl, x.vloc, A, 1)
+    ctx.sync()
+    assert rel(psi.cpu().numpy(), p) < TOL
+    ctx.close()
