@@ -33,7 +33,7 @@ PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FP64_PEAK_FILE = os.path.join(ROOT, "profiles", "r01_fp64_peaks.jsonl")
 NCU_SUMMARY = os.path.join(ROOT, "profiles", "latest_ncu_full_summary.csv")
 NCU_NAMES = {"nl_proj": "k_gemm1", "nl_back": "k_gemm2", "kin_x": "k_kin<1, 1>", "kin_y": "k_kin<1, 0>",
-             "kin_z": "k_kin<1, 2>", "density": "k_density"}
+             "kin_z": "k_kin<1, 2>", "kin_yz": "k_kin_yz", "density": "k_density"}
 
 
 def ncu_traffic(kernel):
@@ -146,6 +146,7 @@ def kernel_work(w):
         "kin_x": (2 * psi + 16.0 * ng * nd, 0.0),
         "kin_y": (2 * psi, 0.0),
         "kin_z": (2 * psi + 16.0 * ng * nd, 0.0),
+        "kin_yz": (2 * psi + 16.0 * ng * nd, 0.0),
         "nl_proj": (psi + bb, gemm_flops),
         "nl_back": (2 * psi + bb, gemm_flops),
         "density": (psi + 8.0 * ng * nd * 4, 0.0),

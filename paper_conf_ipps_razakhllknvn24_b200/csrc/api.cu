@@ -170,6 +170,8 @@ struct lfd_ctx {
   bool c_valid = false;
   bool carry = true;
   bool kin_fused = true;  // Phi.K_y K_z in one pass (env LFD_KIN_FUSED=0: separate y and z passes)
+  CUtensorMap psi_tmap;   // TMA descriptor of Psi for the fused pass
+  bool scaled = true;     // scaled pair form of the stencil (env LFD_KIN_SCALED=0: general 2x2 form)
   std::string err = "no error";
   // density-current global layout cache
   std::vector<long long> gbase_host;
@@ -340,14 +342,14 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false) {
 lfd_status local_prop(lfd_ctx* c) {
   c->c_valid = false;
   LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin(x)",
-                 [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 0, 1, c->stream); }));
+                 [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 0, 1, c->scaled, c->stream); }));
   if (c->kin_fused)
     return launch(c, LFD_K_KIN_YZ, "k_kin_yz",
-                  [&] { return lfd::launch_kin_yz(c->g, c->psi, c->coef(), c->phi(), c->stream); });
+                  [&] { return lfd::launch_kin_yz(c->g, &c->psi_tmap, c->psi, c->coef(), c->phi(), c->scaled, c->stream); });
   LFD_TRY(launch(c, LFD_K_KIN_Y, "k_kin(y)",
-                 [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 1, 0, c->stream); }));
+                 [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 1, 0, c->scaled, c->stream); }));
   return launch(c, LFD_K_KIN_Z, "k_kin(z)",
-                [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 2, 2, c->stream); });
+                [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 2, 2, c->scaled, c->stream); });
 }
 
 // C[dom][m][n] = dV sum_r conj(A[r][m]) Psi[r][n] into out (GEMM-1 + fixed-order reduction).
@@ -452,7 +454,13 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   if (const char* v = std::getenv("LFD_GEMM2_VARIANT")) c->gemm2_variant = std::atoi(v);
   c->carry = (cfg->flags & LFD_FLAG_NO_CARRY) == 0;
   if (const char* v = std::getenv("LFD_KIN_FUSED")) c->kin_fused = std::atoi(v) != 0;
+  if (const char* v = std::getenv("LFD_KIN_SCALED")) c->scaled = std::atoi(v) != 0;
+  c->scaled = c->scaled && lfd::kin_scaled_ok(g);
   c->kin_fused = c->kin_fused && lfd::kin_yz_supported(g);
+  if (c->kin_fused && lfd::kin_yz_tensor_map(g, c->psi, &c->psi_tmap) != cudaSuccess) {
+    cudaGetLastError();
+    c->kin_fused = false;  // descriptor not encodable (e.g. alignment): the separate y and z passes
+  }
   {
     std::lock_guard<std::mutex> lk(g_live_mu);
     g_live.insert(c);
@@ -482,7 +490,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   e = cudaMemsetAsync(c->at<double>(L.vstage), 0, sizeof(double) * g.ndom * g.ng, c->stream);
   if (e != cudaSuccess) { cuda_fail(c, e, "memset"); return bail(LFD_ECUDA); }
   lfd_status s2 = launch(c, LFD_K_PHASE, "k_phase",
-                         [&] { return lfd::launch_phase(g, c->at<double>(L.vstage), c->phi(), c->at<double>(L.vstage), c->stream); });
+                         [&] { return lfd::launch_phase(g, c->at<double>(L.vstage), c->phi(), c->at<double>(L.vstage), c->scaled, c->stream); });
   if (s2 != LFD_OK) return bail(s2);
   s2 = set_A(c, nullptr);
   if (s2 != LFD_OK) return bail(s2);
@@ -511,7 +519,7 @@ lfd_status lfd_set_potential(lfd_ctx* c, const double* vloc) {
   DeviceGuard dg(c->device);
   if (!is_device_ptr(vloc)) return fail(c, LFD_EINVAL, "vloc must be device memory (use lfd_set_potential_host)");
   return launch(c, LFD_K_PHASE, "k_phase", [&] {
-    return lfd::launch_phase(c->g, vloc, c->phi(), c->at<double>(c->L.vstage), c->stream);
+    return lfd::launch_phase(c->g, vloc, c->phi(), c->at<double>(c->L.vstage), c->scaled, c->stream);
   });
 }
 
@@ -523,7 +531,7 @@ lfd_status lfd_set_potential_host(lfd_ctx* c, const double* vloc_host) {
   cudaError_t e = cudaMemcpyAsync(stage, vloc_host, sizeof(double) * c->g.ndom * c->g.ng, cudaMemcpyHostToDevice,
                                   c->stream);
   if (e != cudaSuccess) return cuda_fail(c, e, "H2D vloc");
-  return launch(c, LFD_K_PHASE, "k_phase", [&] { return lfd::launch_phase(c->g, stage, c->phi(), stage, c->stream); });
+  return launch(c, LFD_K_PHASE, "k_phase", [&] { return lfd::launch_phase(c->g, stage, c->phi(), stage, c->scaled, c->stream); });
 }
 
 lfd_status lfd_set_vector_potential(lfd_ctx* c, const double* A) {

@@ -3,14 +3,28 @@
 // Paper: Eq. 6 local factor exp(-i Delta h_loc) by the O(N) space-splitting stencil (P:68,
 // P:76-80). Alg. 3-5 stream each line along the stencil axis with one thread team per
 // (other two coordinates, orbital block) and carry the pre-update neighbour (psi_old) so the update is
-// in place. Here: one thread per (domain, other two coordinates, orbital) column; it streams its line
-// in pair-aligned steps, keeping the pre-update values it still needs in registers (the psi_old carry
-// of Alg. 3 l.6), so each pass reads and writes Psi exactly once. Consecutive threads own
-// consecutive orbitals (the paper's orbital-innermost SoA), so every load/store of a warp is a
-// contiguous 512-byte segment.
+// in place. Here the same streaming structure keeps the pre-update values still needed in registers
+// (the psi_old carry of Alg. 3 l.6), so each pass reads and writes Psi exactly once, and lanes
+// run over consecutive orbitals (the paper's orbital-innermost SoA) so every access is coalesced.
 //
 // K_d = E_d(Delta/2) O_d(Delta) E_d(Delta/2) (readings R4/R5): E links (2m,2m+1), O links (2m+1,2m+2)
 // plus the periodic wrap (n-1,0); zero BC turns missing links into the on-site factor e^{-i tau t_d}.
+//
+// Two passes per step:  (1) Psi <- K_x (Phi . Psi)   (k_kin, axis x, pre-phase)
+//                       (2) Psi <- Phi . K_y K_z Psi (k_kin_yz; K_y and K_z commute exactly, R6)
+// (k_kin also runs the y and z passes separately where k_kin_yz does not apply, nz > 80.)
+//
+// Scaled pair form (kS). Every pair block is  e^{-i tau t} [[c, i s e^{i theta}], [i s e^{-i theta}, c]]
+// with c = cos(tau t), s = sin(tau t) (real). Pulling e^{-i tau t} c out of every block leaves
+//     psi'_i = psi_i + w psi_j,   w = i tan(tau t) e^{+-i theta}      (4 DFMA per output instead of 8)
+// and a factor that is the SAME for every grid point: each point sits in exactly one link per sweep,
+// so K_d = e^{-2 i Delta t_d} c1_d^2 c2_d K~_d (c1 = cos(Delta t_d / 2), c2 = cos(Delta t_d)); zero-BC
+// singletons keep their relative factor 1/c. The product over d of those scalars, g, is folded into
+// Phi as sqrt(g) (Phi is applied once before and once after the kinetic sweeps). Exactly the same
+// operator; used when every c >= 1/2 (else the general 2x2 form runs). The FP64 pipe (not tensor) is
+// what bounds these sweeps next to HBM on B200 (DFMA 34 TF/s), so halving the FP64 work matters.
+#include <cmath>
+
 #include "lfd_complex.cuh"
 #include "lfd_internal.h"
 #include "lfd_tma.cuh"
@@ -40,6 +54,10 @@ __global__ void k_coef(CoefParams p, int dom0, int count, double hx, double hy, 
       c.up[d][q] = cmul(sigma, make_double2(ct, st));      // sigma e^{+i theta}
       c.dn[d][q] = cmul(sigma, make_double2(ct, -st));     // sigma e^{-i theta}
       c.onsite[d][q] = ph;
+      const double tn = sp / cp;                           // scaled form: w = i tan(tau t) e^{+-i theta}
+      c.wu[d][q] = make_double2(-tn * st, tn * ct);
+      c.wd[d][q] = make_double2(tn * st, tn * ct);
+      c.rc[d][q] = 1.0 / cp;                               // zero-BC singleton, relative to c
     }
   }
   c.pad_ = 0.0;
@@ -52,28 +70,154 @@ cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int co
   return cudaGetLastError();
 }
 
-// Phi(r) = e^{-i (Delta/2) v_loc(r)}  (Strang placement of the potential, reading R7).
+// Phi(r) = e^{-i (Delta/2) v_loc(r)} (Strang placement of the potential, reading R7), times the
+// constant sqrt(g) of the scaled pair form (1 for the general form).
 // The kernel also keeps a copy of v_loc for lfd_energy (vcopy may alias v: then it is not written).
 __global__ void k_phase(const double* __restrict__ v, double2* __restrict__ phi, double* vcopy, long long n,
-                        double half_dt) {
+                        double half_dt, double2 sg) {
   long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   const double vi = v[i];
   double s, c;
   sincos(half_dt * vi, &s, &c);
-  phi[i] = make_double2(c, -s);
+  phi[i] = cmul(make_double2(c, -s), sg);
   if (vcopy != v) vcopy[i] = vi;
 }
 
-cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, double* vcopy, cudaStream_t st) {
+bool kin_scaled_ok(const Geometry& g) {
+  const double h[3] = {g.hx, g.hy, g.hz};
+  for (int d = 0; d < 3; ++d) {
+    const double t = 1.0 / (2.0 * h[d] * h[d]);
+    if (!(std::cos(0.5 * g.dt * t) >= 0.5) || !(std::cos(g.dt * t) >= 0.5)) return false;
+  }
+  return true;
+}
+
+static double2 scaled_sqrt_g(const Geometry& g) {
+  const double h[3] = {g.hx, g.hy, g.hz};
+  double re = 1.0, im = 0.0;
+  for (int d = 0; d < 3; ++d) {  // prod_d e^{-i Delta t_d} c1_d sqrt(c2_d)
+    const double t = 1.0 / (2.0 * h[d] * h[d]);
+    const double mag = std::cos(0.5 * g.dt * t) * std::sqrt(std::cos(g.dt * t));
+    const double pr = mag * std::cos(g.dt * t), pi = -mag * std::sin(g.dt * t);
+    const double nr = re * pr - im * pi, ni = re * pi + im * pr;
+    re = nr;
+    im = ni;
+  }
+  return make_double2(re, im);
+}
+
+cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, double* vcopy, bool scaled,
+                         cudaStream_t st) {
   long long n = g.ng * g.ndom;
-  k_phase<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(v, phi, vcopy, n, 0.5 * g.dt);
+  const double2 sg = scaled ? scaled_sqrt_g(g) : make_double2(1.0, 0.0);
+  k_phase<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(v, phi, vcopy, n, 0.5 * g.dt, sg);
   return cudaGetLastError();
 }
 
+// ---- pair blocks -------------------------------------------------------------------------------
+// Coefficients of one axis for tau = Delta/2 (1) and Delta (2). General form: a = alpha, u = up,
+// d = dn, s = onsite. Scaled form: u = w_up, d = w_dn, s = (1/c, 0), a unused.
+struct PairCoef {
+  double2 a1, u1, d1, s1, a2, u2, d2, s2;
+};
+
+template <bool kS>
+__device__ __forceinline__ PairCoef pair_coef(const DomCoef* cf, int axis) {
+  PairCoef c;
+  if (kS) {
+    c.a1 = c.a2 = make_double2(1.0, 0.0);
+    c.u1 = cf->wu[axis][0]; c.d1 = cf->wd[axis][0]; c.s1 = make_double2(cf->rc[axis][0], 0.0);
+    c.u2 = cf->wu[axis][1]; c.d2 = cf->wd[axis][1]; c.s2 = make_double2(cf->rc[axis][1], 0.0);
+  } else {
+    c.a1 = cf->alpha[axis][0]; c.u1 = cf->up[axis][0]; c.d1 = cf->dn[axis][0]; c.s1 = cf->onsite[axis][0];
+    c.a2 = cf->alpha[axis][1]; c.u2 = cf->up[axis][1]; c.d2 = cf->dn[axis][1]; c.s2 = cf->onsite[axis][1];
+  }
+  return c;
+}
+
+// x + w y
+__device__ __forceinline__ double2 padd(double2 w, double2 x, double2 y) {
+  return make_double2(fma(w.x, y.x, fma(-w.y, y.y, x.x)), fma(w.x, y.y, fma(w.y, y.x, x.y)));
+}
+// Left / right output of a link (x at the left point, y at the right point) and a singleton.
+template <bool kS>
+__device__ __forceinline__ double2 lk_L(double2 a, double2 u, double2 x, double2 y) {
+  return kS ? padd(u, x, y) : crow(a, x, u, y);
+}
+template <bool kS>
+__device__ __forceinline__ double2 lk_R(double2 a, double2 d, double2 x, double2 y) {
+  return kS ? padd(d, y, x) : crow(d, x, a, y);
+}
+template <bool kS>
+__device__ __forceinline__ double2 lk_S(double2 s, double2 x) {
+  return kS ? make_double2(s.x * x.x, s.x * x.y) : cmul(s, x);
+}
+
+// Streaming K_d along one line, fed one pair (2p, 2p+1) at a time: first E(Delta/2) on the new pair,
+// O(Delta) on the link (2p-1, 2p), second E(Delta/2) on (2p-2, 2p-1) once both its O outputs exist;
+// points 0, 1 wait for the wrap link (n-1, 0) at the end.
+template <bool kS>
+struct LineMarch {
+  double2 E10, O1, prev_e1, prev_oR;
+  __device__ __forceinline__ void init() { E10 = O1 = prev_e1 = prev_oR = cz(); }
+  template <class St>
+  __device__ __forceinline__ void push(const PairCoef& c, int p, double2 a, double2 b, bool pair, St&& st) {
+    double2 e0, e1 = cz();
+    if (pair) {
+      e0 = lk_L<kS>(c.a1, c.u1, a, b);
+      e1 = lk_R<kS>(c.a1, c.d1, a, b);
+    } else {
+      e0 = lk_S<kS>(c.s1, a);  // zero-BC singleton (odd n)
+    }
+    if (p == 0) {
+      E10 = e0;
+    } else {
+      const double2 oL = lk_L<kS>(c.a2, c.u2, prev_e1, e0);
+      const double2 oR = lk_R<kS>(c.a2, c.d2, prev_e1, e0);
+      if (p == 1) {
+        O1 = oL;
+      } else {
+        st(2 * p - 2, lk_L<kS>(c.a1, c.u1, prev_oR, oL));
+        st(2 * p - 1, lk_R<kS>(c.a1, c.d1, prev_oR, oL));
+      }
+      prev_oR = oR;
+    }
+    prev_e1 = e1;
+  }
+  template <bool kPer, class St>
+  __device__ __forceinline__ void finish(const PairCoef& c, int n, St&& st) {
+    if ((n & 1) == 0) {
+      double2 Olast, O0;
+      if (kPer) {  // wrap link (n-1, 0)
+        Olast = lk_L<kS>(c.a2, c.u2, prev_e1, E10);
+        O0 = lk_R<kS>(c.a2, c.d2, prev_e1, E10);
+      } else {
+        Olast = lk_S<kS>(c.s2, prev_e1);
+        O0 = lk_S<kS>(c.s2, E10);
+      }
+      if (n == 2) {
+        st(0, lk_L<kS>(c.a1, c.u1, O0, Olast));
+        st(1, lk_R<kS>(c.a1, c.d1, O0, Olast));
+      } else {
+        st(n - 2, lk_L<kS>(c.a1, c.u1, prev_oR, Olast));
+        st(n - 1, lk_R<kS>(c.a1, c.d1, prev_oR, Olast));
+        st(0, lk_L<kS>(c.a1, c.u1, O0, O1));
+        st(1, lk_R<kS>(c.a1, c.d1, O0, O1));
+      }
+    } else {  // odd n (zero BC): last point is an E singleton; point 0 an O singleton
+      st(n - 1, lk_S<kS>(c.s1, prev_oR));
+      const double2 O0 = lk_S<kS>(c.s2, E10);
+      st(0, lk_L<kS>(c.a1, c.u1, O0, O1));
+      st(1, lk_R<kS>(c.a1, c.d1, O0, O1));
+    }
+  }
+};
+
 // One K_axis pass. Column c of domain blockIdx.y: outer = c / inner_len, inner = c % inner_len,
 // element offset = outer*outer_stride + inner; successive points of the line are pt_stride apart.
-template <bool kPeriodic, int kPhase>
+// Loads run two pairs ahead of the pair being combined (memory-level parallelism for the HBM stream).
+template <bool kPeriodic, int kPhase, bool kS>
 __global__ void __launch_bounds__(256, 3) k_kin(double2* __restrict__ psi, const DomCoef* __restrict__ coef,
                                              const double2* __restrict__ phi, int axis, int n, int pt_stride,
                                              int inner_len, int outer_stride, int ncols, int norb,
@@ -87,10 +231,7 @@ __global__ void __launch_bounds__(256, 3) k_kin(double2* __restrict__ psi, const
   double2* line = psi + dom * dom_stride + off;
   const double2* ph = phi + dom * ng + off / norb;
   const int ph_stride = pt_stride / norb;
-
-  const DomCoef* cf = coef + dom;
-  const double2 a1 = cf->alpha[axis][0], u1 = cf->up[axis][0], d1 = cf->dn[axis][0], s1 = cf->onsite[axis][0];
-  const double2 a2 = cf->alpha[axis][1], u2 = cf->up[axis][1], d2 = cf->dn[axis][1], s2 = cf->onsite[axis][1];
+  const PairCoef cf = pair_coef<kS>(coef + dom, axis);
 
   auto ld = [&](int i) -> double2 {
     double2 v = line[(long long)i * pt_stride];
@@ -103,8 +244,8 @@ __global__ void __launch_bounds__(256, 3) k_kin(double2* __restrict__ psi, const
   };
 
   const int P = (n + 1) >> 1;
-  double2 E10 = cz(), O1 = cz(), prev_e1 = cz(), prev_oR = cz();
-  // two pairs in flight ahead of the one being combined (memory-level parallelism for the HBM stream)
+  LineMarch<kS> L;
+  L.init();
   double2 na = ld(0), nb = (n > 1) ? ld(1) : cz();
   double2 nc = cz(), nd = cz();
   if (P > 1) {
@@ -113,279 +254,222 @@ __global__ void __launch_bounds__(256, 3) k_kin(double2* __restrict__ psi, const
   }
   for (int p = 0; p < P; ++p) {
     const double2 a = na, b = nb;
-    const bool pair = (2 * p + 1 < n);
     na = nc;
     nb = nd;
     if (p + 2 < P) {
       nc = ld(2 * p + 4);
       nd = (2 * p + 5 < n) ? ld(2 * p + 5) : cz();
     }
-    double2 e0, e1 = cz();
-    if (pair) {
-      e0 = crow(a1, a, u1, b);  // first E(Delta/2) on link (2p, 2p+1)
-      e1 = crow(d1, a, a1, b);
-    } else {
-      e0 = cmul(s1, a);  // zero-BC singleton (odd n)
-    }
-    if (p == 0) {
-      E10 = e0;
-    } else {
-      const double2 oL = crow(a2, prev_e1, u2, e0);  // O(Delta) on link (2p-1, 2p)
-      const double2 oR = crow(d2, prev_e1, a2, e0);
-      if (p == 1) {
-        O1 = oL;
-      } else {  // second E(Delta/2) on link (2p-2, 2p-1): both O outputs are now known
-        st(2 * p - 2, crow(a1, prev_oR, u1, oL));
-        st(2 * p - 1, crow(d1, prev_oR, a1, oL));
-      }
-      prev_oR = oR;
-    }
-    prev_e1 = e1;
+    L.push(cf, p, a, b, 2 * p + 1 < n, st);
   }
-  if ((n & 1) == 0) {
-    double2 Olast, O0;
-    if (kPeriodic) {  // wrap link (n-1, 0)
-      Olast = crow(a2, prev_e1, u2, E10);
-      O0 = crow(d2, prev_e1, a2, E10);
-    } else {
-      Olast = cmul(s2, prev_e1);
-      O0 = cmul(s2, E10);
-    }
-    if (n == 2) {
-      st(0, crow(a1, O0, u1, Olast));
-      st(1, crow(d1, O0, a1, Olast));
-    } else {
-      st(n - 2, crow(a1, prev_oR, u1, Olast));
-      st(n - 1, crow(d1, prev_oR, a1, Olast));
-      st(0, crow(a1, O0, u1, O1));
-      st(1, crow(d1, O0, a1, O1));
-    }
-  } else {  // odd n (zero BC): last point is an E singleton; point 0 an O singleton
-    st(n - 1, cmul(s1, prev_oR));
-    const double2 O0 = cmul(s2, E10);
-    st(0, crow(a1, O0, u1, O1));
-    st(1, crow(d1, O0, a1, O1));
-  }
+  L.template finish<kPeriodic>(cf, n, st);
 }
 
 // ------------------------------------------------------------------------------------------------
 // Fused K_y K_z pass with the post-phase:  Psi <- Phi . K_y K_z Psi  (one HBM read + write of Psi).
 // K_y and K_z act on different axes of the tensor grid and commute exactly (reading R6), so the pass
 // applies K_z to each (x, y) z-line as it arrives and streams the K_z-transformed lines through the
-// pair-aligned y-march of K_y (the psi_old carry of Alg. 3, in registers).
-// CTA = (x plane, chunk of kYZW = 8 orbitals, domain); thread (m, o) owns the z pair (2m, 2m+1) of
-// orbital o0 + o. Each (x, y) plane segment [nz][8 orbitals] (nz rows of 128 contiguous bytes) arrives
-// by TMA bulk copies into an S-deep shared-memory ring; K_z's O(Delta) links cross threads and go
-// through a small exchange buffer (double-buffered by pair parity: one __syncthreads per y pair).
+// pair-aligned y-march of K_y.
+// CTA = (x plane, chunk of kYZW = 8 orbitals, domain). A producer warp brings each (x, y) plane segment
+// [nz rows][8 orbitals x 16 B] into an S-deep shared-memory ring with ONE tiled TMA tensor copy
+// (cp.async.bulk.tensor, full/empty mbarriers); consumer thread (m, o) owns the z pair (2m, 2m+1) of
+// orbital o0 + o and recomputes its neighbours' first-E outputs from the ring instead of exchanging
+// them, so consumer warps never synchronise with each other.
 // ------------------------------------------------------------------------------------------------
 constexpr int kYZW = 8;
+constexpr int kYZMaxThreads = 352;  // up to 40 z pairs x 8 orbitals + the producer warp
 
-struct PairCoef {
-  double2 a1, u1, d1, s1, a2, u2, d2, s2;
-};
-
-__device__ __forceinline__ PairCoef pair_coef(const DomCoef* cf, int axis) {
-  PairCoef c;
-  c.a1 = cf->alpha[axis][0]; c.u1 = cf->up[axis][0]; c.d1 = cf->dn[axis][0]; c.s1 = cf->onsite[axis][0];
-  c.a2 = cf->alpha[axis][1]; c.u2 = cf->up[axis][1]; c.d2 = cf->dn[axis][1]; c.s2 = cf->onsite[axis][1];
-  return c;
-}
-
-// Streaming K_d along one line, fed one pair (2p, 2p+1) at a time (same algebra as k_kin's loop).
-struct LineMarch {
-  double2 E10, O1, prev_e1, prev_oR;
-  template <class St>
-  __device__ __forceinline__ void push(const PairCoef& c, int p, double2 a, double2 b, bool pair, St&& st) {
-    double2 e0, e1 = cz();
-    if (pair) {
-      e0 = crow(c.a1, a, c.u1, b);
-      e1 = crow(c.d1, a, c.a1, b);
-    } else {
-      e0 = cmul(c.s1, a);
-    }
-    if (p == 0) {
-      E10 = e0;
-    } else {
-      const double2 oL = crow(c.a2, prev_e1, c.u2, e0);
-      const double2 oR = crow(c.d2, prev_e1, c.a2, e0);
-      if (p == 1) {
-        O1 = oL;
-      } else {
-        st(2 * p - 2, crow(c.a1, prev_oR, c.u1, oL));
-        st(2 * p - 1, crow(c.d1, prev_oR, c.a1, oL));
-      }
-      prev_oR = oR;
-    }
-    prev_e1 = e1;
-  }
-  template <bool kPer, class St>
-  __device__ __forceinline__ void finish(const PairCoef& c, int n, St&& st) {
-    if ((n & 1) == 0) {
-      double2 Olast, O0;
-      if (kPer) {
-        Olast = crow(c.a2, prev_e1, c.u2, E10);
-        O0 = crow(c.d2, prev_e1, c.a2, E10);
-      } else {
-        Olast = cmul(c.s2, prev_e1);
-        O0 = cmul(c.s2, E10);
-      }
-      if (n == 2) {
-        st(0, crow(c.a1, O0, c.u1, Olast));
-        st(1, crow(c.d1, O0, c.a1, Olast));
-      } else {
-        st(n - 2, crow(c.a1, prev_oR, c.u1, Olast));
-        st(n - 1, crow(c.d1, prev_oR, c.a1, Olast));
-        st(0, crow(c.a1, O0, c.u1, O1));
-        st(1, crow(c.d1, O0, c.a1, O1));
-      }
-    } else {
-      st(n - 1, cmul(c.s1, prev_oR));
-      const double2 O0 = cmul(c.s2, E10);
-      st(0, crow(c.a1, O0, c.u1, O1));
-      st(1, crow(c.d1, O0, c.a1, O1));
-    }
-  }
-};
-
-template <bool kPer>
-__global__ void __launch_bounds__(512) k_kin_yz(double2* __restrict__ psi, const DomCoef* __restrict__ coef,
-                                                 const double2* __restrict__ phi, int nx, int ny, int nz, int norb,
-                                                 int nchunks, long long ng, int S) {
+template <bool kPer, bool kS>
+__global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant__ CUtensorMap tmap,
+                                                          double2* __restrict__ psi, const DomCoef* __restrict__ coef,
+                                                          const double2* __restrict__ phi, int nx, int ny, int nz,
+                                                          int norb, int nchunks, long long ng, int S) {
   extern __shared__ __align__(128) unsigned char smem[];
   const int seg = nz * kYZW;  // complex elements per plane segment
   double2* ring = reinterpret_cast<double2*>(smem);
-  double2* xch = ring + (long long)S * seg;               // [2 pair parities][2 planes][nz][8]
-  uint64_t* full = reinterpret_cast<uint64_t*>(xch + 4 * seg);
+  uint64_t* full = reinterpret_cast<uint64_t*>(ring + (long long)S * seg);
+  uint64_t* empty = full + S;
   const int dom = blockIdx.y;
   const int x = blockIdx.x / nchunks, oc = blockIdx.x - (blockIdx.x / nchunks) * nchunks;
   const int o0 = oc * kYZW, wv = min(kYZW, norb - o0);
-  const int tid = threadIdx.x, o = tid % kYZW, m = tid / kYZW;
-  const int z0 = 2 * m, z1 = 2 * m + 1;
-  const bool has1 = z1 < nz;
-  const bool act = o < wv;
-  const long long yst = (long long)nz * norb;  // element stride between y planes
-  double2* base = psi + (long long)dom * ng * norb + (long long)x * ny * yst + o0;
-  const double2* phb = phi + (long long)dom * ng + (long long)x * ny * nz;
-  const DomCoef* cf = coef + dom;
-  const PairCoef cz_ = pair_coef(cf, 2), cy = pair_coef(cf, 1);
-
+  const int npz = (nz + 1) >> 1;                 // z pairs (the last one a singleton for odd nz)
+  const int nconsw = (npz * kYZW + 31) >> 5;     // consumer warps; the next warp is the producer
+  // coefficients live in shared memory (broadcast LDS) to keep registers for the march state
+  __shared__ PairCoef sc[2];
+  const PairCoef& cz_ = sc[0];
+  const PairCoef& cy = sc[1];
+  const int tid = threadIdx.x;
   if (tid == 0) {
-    for (int s = 0; s < S; ++s) mbar_init(&full[s], 1);
+    sc[0] = pair_coef<kS>(coef + dom, 2);
+    sc[1] = pair_coef<kS>(coef + dom, 1);
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], nconsw);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  auto issue = [&](int y) {  // warp 0: plane y -> slot y % S
-    const int s = y % S;
-    const int lane = tid & 31;
-    if (lane == 0) mbar_expect_tx(&full[s], (uint32_t)(nz * wv * 16));
-    __syncwarp();
-    double2* dst = ring + (long long)s * seg;
-    const double2* src = base + (long long)y * yst;
-    for (int z = lane; z < nz; z += 32) tma_row(dst + z * kYZW, src + (long long)z * norb, (uint32_t)(wv * 16), &full[s]);
-  };
-  if (tid < 32)
-    for (int y = 0; y < S && y < ny; ++y) issue(y);
 
-  // first E_z(Delta/2) on (z0, z1) of plane y (from the ring) -> (e0, e1), also into the exchange buffer
-  auto stage_in = [&](int y, double2* xb, double2& e0, double2& e1) {
+  if (tid >= nconsw * 32) {  // producer warp: plane y -> slot y % S, one tensor copy per plane
+    if (tid == nconsw * 32) {
+      const int row0 = (dom * nx + x) * ny;
+      for (int y = 0; y < ny; ++y) {
+        const int s = y % S;
+        if (y >= S) mbar_wait(&empty[s], (uint32_t)(((y / S) - 1) & 1));
+        mbar_expect_tx(&full[s], (uint32_t)(seg * 16));
+        tma_3d(ring + (long long)s * seg, &tmap, 2 * o0, 0, row0 + y, &full[s]);
+      }
+    }
+    return;
+  }
+
+  const int o = tid % kYZW, m = tid / kYZW;
+  const bool live = m < npz;
+  const int z0 = 2 * m, z1 = 2 * m + 1;
+  const bool has1 = z1 < nz;
+  const bool act = live && o < wv;
+  const long long yst = (long long)nz * norb;  // element stride between y planes
+  double2* base = psi + (long long)dom * ng * norb + (long long)x * ny * yst + o0;
+  const double2* phb = phi + (long long)dom * ng + (long long)x * ny * nz;
+
+  // K_z of plane y for this thread's pair: the first E(Delta/2) on pairs m-1, m, m+1 (the neighbours'
+  // outputs recomputed here), O(Delta) on the links (2m-1, 2m) and (2m+1, 2m+2), then the second
+  // E(Delta/2) on (2m, 2m+1). The slot is released to the producer afterwards.
+  auto kz = [&](int y, double2& w0, double2& w1) {
     const int s = y % S;
     mbar_wait(&full[s], (uint32_t)((y / S) & 1));
-    const double2* r = ring + (long long)s * seg;
-    const double2 v0 = r[z0 * kYZW + o];
-    if (has1) {
-      const double2 v1 = r[z1 * kYZW + o];
-      e0 = crow(cz_.a1, v0, cz_.u1, v1);
-      e1 = crow(cz_.d1, v0, cz_.a1, v1);
-      xb[z1 * kYZW + o] = e1;
-    } else {  // zero BC, odd nz: singleton
-      e0 = cmul(cz_.s1, v0);
-      e1 = cz();
+    const double2* r = ring + (long long)s * seg + o;
+    auto v = [&](int z) { return r[z * kYZW]; };
+    w0 = w1 = cz();
+    if (live) {
+      double2 e0, e1 = cz();
+      if (has1) {
+        const double2 a = v(z0), b = v(z1);
+        e0 = lk_L<kS>(cz_.a1, cz_.u1, a, b);
+        e1 = lk_R<kS>(cz_.a1, cz_.d1, a, b);
+      } else {
+        e0 = lk_S<kS>(cz_.s1, v(z0));
+      }
+      double2 q0, q1 = cz();
+      if (m > 0 || kPer) {  // link (2m-1, 2m): E output of z = 2m-1 (pair m-1, its right point)
+        const int zl = (m > 0) ? z0 - 2 : nz - 2;
+        const double2 l1 = lk_R<kS>(cz_.a1, cz_.d1, v(zl), v(zl + 1));
+        q0 = lk_R<kS>(cz_.a2, cz_.d2, l1, e0);
+      } else {
+        q0 = lk_S<kS>(cz_.s2, e0);
+      }
+      if (has1) {
+        if (z1 + 1 < nz || kPer) {  // link (2m+1, 2m+2): E output of z = 2m+2 (pair m+1, its left point)
+          const int zr = (z1 + 1 < nz) ? z1 + 1 : 0;
+          const double2 r0 = (zr + 1 < nz) ? lk_L<kS>(cz_.a1, cz_.u1, v(zr), v(zr + 1)) : lk_S<kS>(cz_.s1, v(zr));
+          q1 = lk_L<kS>(cz_.a2, cz_.u2, e1, r0);
+        } else {
+          q1 = lk_S<kS>(cz_.s2, e1);
+        }
+        w0 = lk_L<kS>(cz_.a1, cz_.u1, q0, q1);
+        w1 = lk_R<kS>(cz_.a1, cz_.d1, q0, q1);
+      } else {
+        w0 = lk_S<kS>(cz_.s1, q0);
+      }
     }
-    xb[z0 * kYZW + o] = e0;
+    __syncwarp();
+    if ((tid & 31) == 0) mbar_arrive(&empty[s]);
   };
-  // O_z(Delta) with the neighbours' E outputs, then the second E_z(Delta/2)
-  auto stage_out = [&](const double2* xb, double2 e0, double2 e1, double2& w0, double2& w1) {
-    double2 q0, q1 = cz();
-    if (m > 0) q0 = crow(cz_.d2, xb[(z0 - 1) * kYZW + o], cz_.a2, e0);
-    else if (kPer) q0 = crow(cz_.d2, xb[(nz - 1) * kYZW + o], cz_.a2, e0);
-    else q0 = cmul(cz_.s2, e0);
-    if (has1) {
-      if (z1 + 1 < nz) q1 = crow(cz_.a2, e1, cz_.u2, xb[(z1 + 1) * kYZW + o]);
-      else if (kPer) q1 = crow(cz_.a2, e1, cz_.u2, xb[o]);
-      else q1 = cmul(cz_.s2, e1);
-      w0 = crow(cz_.a1, q0, cz_.u1, q1);
-      w1 = crow(cz_.d1, q0, cz_.a1, q1);
-    } else {
-      w0 = cmul(cz_.s1, q0);
-      w1 = cz();
-    }
-  };
-  auto st0 = [&](int y, double2 v) {
-    if (act) base[(long long)y * yst + (long long)z0 * norb + o] = cmul(phb[(long long)y * nz + z0], v);
-  };
-  auto st1 = [&](int y, double2 v) {
-    if (act && has1) base[(long long)y * yst + (long long)z1 * norb + o] = cmul(phb[(long long)y * nz + z1], v);
+  auto ph = [&](int y, int z) { return (live && z < nz) ? __ldg(phb + (long long)y * nz + z) : cz(); };
+  auto put = [&](int y, int z, double2 f, double2 v) {
+    if (act && z < nz) base[(long long)y * yst + (long long)z * norb + o] = cmul(f, v);
   };
 
-  LineMarch L0, L1;
-  L0.E10 = L0.O1 = L0.prev_e1 = L0.prev_oR = cz();
-  L1 = L0;
+  // Phi of planes 0 and 1 (stored last, by the wrap) stays in registers
+  const double2 f00 = ph(0, z0), f01 = ph(0, z1), f10 = ph(1, z0), f11 = ph(1, z1);
+  LineMarch<kS> L0, L1;
+  L0.init();
+  L1.init();
   const int npairs = (ny + 1) >> 1;
   for (int p = 0; p < npairs; ++p) {
     const int ya = 2 * p, yb = 2 * p + 1;
     const bool hb = yb < ny;
-    double2* xa = xch + (long long)((p & 1) * 2) * seg;
-    double2* xb = xa + seg;
-    double2 ea0, ea1, eb0 = cz(), eb1 = cz();
-    stage_in(ya, xa, ea0, ea1);
-    if (hb) stage_in(yb, xb, eb0, eb1);
-    __syncthreads();  // exchange buffers written; ring slots of ya, yb consumed
-    if (tid < 32) {
-      if (ya + S < ny) issue(ya + S);
-      if (hb && yb + S < ny) issue(yb + S);
+    // Phi of the two planes this iteration's march step stores (2p-2, 2p-1): loads in flight meanwhile
+    double2 fa0 = cz(), fa1 = cz(), fb0 = cz(), fb1 = cz();
+    if (p >= 2) {
+      fa0 = ph(ya - 2, z0); fa1 = ph(ya - 2, z1);
+      fb0 = ph(ya - 1, z0); fb1 = ph(ya - 1, z1);
     }
     double2 wa0, wa1, wb0 = cz(), wb1 = cz();
-    stage_out(xa, ea0, ea1, wa0, wa1);
-    if (hb) stage_out(xb, eb0, eb1, wb0, wb1);
-    L0.push(cy, p, wa0, wb0, hb, st0);
-    L1.push(cy, p, wa1, wb1, hb, st1);
+    kz(ya, wa0, wa1);
+    if (hb) kz(yb, wb0, wb1);
+    L0.push(cy, p, wa0, wb0, hb, [&](int y, double2 v) { put(y, z0, y == ya - 2 ? fa0 : fb0, v); });
+    L1.push(cy, p, wa1, wb1, hb, [&](int y, double2 v) { put(y, z1, y == ya - 2 ? fa1 : fb1, v); });
   }
-  L0.finish<kPer>(cy, ny, st0);
-  L1.finish<kPer>(cy, ny, st1);
+  // wrap: planes ny-2, ny-1 (or ny-1 for odd ny) and 0, 1
+  const double2 fl0 = ph(ny - 1, z0), fl1 = ph(ny - 1, z1);
+  const double2 fm0 = ph(ny - 2, z0), fm1 = ph(ny - 2, z1);
+  auto pick0 = [&](int y) { return y == 0 ? f00 : y == 1 ? f10 : y == ny - 1 ? fl0 : fm0; };
+  auto pick1 = [&](int y) { return y == 0 ? f01 : y == 1 ? f11 : y == ny - 1 ? fl1 : fm1; };
+  L0.template finish<kPer>(cy, ny, [&](int y, double2 v) { put(y, z0, pick0(y), v); });
+  L1.template finish<kPer>(cy, ny, [&](int y, double2 v) { put(y, z1, pick1(y), v); });
 }
 
 static int yz_stages(int nz) {
   const int seg_bytes = nz * kYZW * 16;
-  int S = (200 * 1024 - 4 * seg_bytes) / seg_bytes;
-  return S > 6 ? 6 : S;
+  int S = (200 * 1024) / seg_bytes;
+  return S > 12 ? 12 : S;
 }
 
-bool kin_yz_supported(const Geometry& g) { return g.nz <= 128 && yz_stages(g.nz) >= 2; }
+bool kin_yz_supported(const Geometry& g) { return g.nz <= 80 && yz_stages(g.nz) >= 2; }
 
-static size_t yz_smem(int nz, int S) { return (size_t)(S + 4) * nz * kYZW * 16 + (size_t)S * 8; }
+static size_t yz_smem(int nz, int S) { return (size_t)S * nz * kYZW * 16 + (size_t)S * 16; }
+
+// Tensor map of Psi for k_kin_yz: 3-D view [ndom*nx*ny planes][nz rows][2*norb doubles], box
+// [1][nz][16 doubles] (one (x, y) plane segment of 8 orbitals), no swizzle (dense rows of 128 B).
+cudaError_t kin_yz_tensor_map(const Geometry& g, double2* psi, CUtensorMap* out) {
+  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+  if (!encode) {
+    cudaDriverEntryPointQueryResult q;
+    void* fn = nullptr;
+    cudaError_t e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q);
+    if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !fn) return e != cudaSuccess ? e : cudaErrorNotSupported;
+    encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  }
+  const cuuint64_t dims[3] = {(cuuint64_t)2 * g.norb, (cuuint64_t)g.nz, (cuuint64_t)g.ndom * g.nx * g.ny};
+  const cuuint64_t strides[2] = {(cuuint64_t)g.norb * 16, (cuuint64_t)g.nz * g.norb * 16};
+  const cuuint32_t box[3] = {2 * kYZW, (cuuint32_t)g.nz, 1};
+  const cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = encode(out, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, psi, dims, strides, box, estr,
+                      CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
+}
 
 cudaError_t kin_yz_set_attributes() {
-  cudaError_t e = cudaFuncSetAttribute(k_kin_yz<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-  if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(k_kin_yz<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+  const int sm = 220 * 1024;
+  cudaError_t e = cudaFuncSetAttribute(k_kin_yz<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(k_kin_yz<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(k_kin_yz<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(k_kin_yz<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+  return e;
 }
 
-cudaError_t launch_kin_yz(const Geometry& g, double2* psi, const DomCoef* coef, const double2* phi,
-                          cudaStream_t st) {
+cudaError_t launch_kin_yz(const Geometry& g, const CUtensorMap* tmap, double2* psi, const DomCoef* coef,
+                          const double2* phi, bool scaled, cudaStream_t st) {
   const int nchunks = (g.norb + kYZW - 1) / kYZW;
   const int S = yz_stages(g.nz);
-  const int threads = ((g.nz + 1) / 2) * kYZW;
+  const int threads = ((((g.nz + 1) / 2) * kYZW + 31) / 32 + 1) * 32;  // consumer warps + producer warp
   dim3 grid(g.nx * nchunks, g.ndom);
   const size_t sm = yz_smem(g.nz, S);
-  if (g.bc == 0)
-    k_kin_yz<true><<<grid, threads, sm, st>>>(psi, coef, phi, g.nx, g.ny, g.nz, g.norb, nchunks, g.ng, S);
-  else
-    k_kin_yz<false><<<grid, threads, sm, st>>>(psi, coef, phi, g.nx, g.ny, g.nz, g.norb, nchunks, g.ng, S);
+#define LFD_KYZ(P, K) \
+  k_kin_yz<P, K><<<grid, threads, sm, st>>>(*tmap, psi, coef, phi, g.nx, g.ny, g.nz, g.norb, nchunks, g.ng, S)
+  if (g.bc == 0) {
+    if (scaled) LFD_KYZ(true, true); else LFD_KYZ(true, false);
+  } else {
+    if (scaled) LFD_KYZ(false, true); else LFD_KYZ(false, false);
+  }
+#undef LFD_KYZ
   return cudaGetLastError();
 }
 
 cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, const double2* phi, int axis,
-                       int phase_mode, cudaStream_t st) {
+                       int phase_mode, bool scaled, cudaStream_t st) {
   const int nd[3] = {g.nx, g.ny, g.nz};
   const int norb = g.norb;
   int pt_stride, inner_len, outer_stride;
@@ -406,15 +490,17 @@ cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, con
   const int ncols = (int)(g.ng / n) * norb;
   dim3 grid((ncols + 255) / 256, g.ndom);
   const long long dom_stride = g.ng * norb;
-  const bool per = (g.bc == 0);
-#define LFD_KIN(P, M)                                                                                    \
-  k_kin<P, M><<<grid, 256, 0, st>>>(psi, coef, phi, axis, n, pt_stride, inner_len, outer_stride, ncols, \
-                                    norb, dom_stride, g.ng)
-  if (per) {
-    if (phase_mode == 1) LFD_KIN(true, 1); else if (phase_mode == 2) LFD_KIN(true, 2); else LFD_KIN(true, 0);
+#define LFD_KIN(P, M, K)                                                                                    \
+  k_kin<P, M, K><<<grid, 256, 0, st>>>(psi, coef, phi, axis, n, pt_stride, inner_len, outer_stride, ncols, \
+                                       norb, dom_stride, g.ng)
+#define LFD_KIN_M(P, K) \
+  if (phase_mode == 1) LFD_KIN(P, 1, K); else if (phase_mode == 2) LFD_KIN(P, 2, K); else LFD_KIN(P, 0, K)
+  if (g.bc == 0) {
+    if (scaled) { LFD_KIN_M(true, true); } else { LFD_KIN_M(true, false); }
   } else {
-    if (phase_mode == 1) LFD_KIN(false, 1); else if (phase_mode == 2) LFD_KIN(false, 2); else LFD_KIN(false, 0);
+    if (scaled) { LFD_KIN_M(false, true); } else { LFD_KIN_M(false, false); }
   }
+#undef LFD_KIN_M
 #undef LFD_KIN
   return cudaGetLastError();
 }

@@ -1,6 +1,8 @@
 // lfd_internal.h -- shared (product-only) declarations of the sm_100a kernels and their launchers.
 // Not part of the public ABI (include/lfd.h). Nothing here is shared with oracle/.
 #pragma once
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -21,6 +23,11 @@ struct DomCoef {
   double2 eth[3];
   double inv_h[3];
   double pad_;
+  // scaled pair form (kin.cu): w_up = i tan(tau t_d) e^{+i theta_d}, w_dn = i tan(tau t_d) e^{-i theta_d},
+  // rc = 1 / cos(tau t_d) (zero-BC singletons)
+  double2 wu[3][2];
+  double2 wd[3][2];
+  double rc[3][2];
 };
 
 struct Geometry {
@@ -36,17 +43,22 @@ struct CoefParams {
 };
 cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int count, DomCoef* coef,
                         cudaStream_t st);
-cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, double* vcopy, cudaStream_t st);
+// Phi = e^{-i (Delta/2) v} (times sqrt(g) when the scaled pair form is used, kin.cu).
+cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, double* vcopy, bool scaled,
+                         cudaStream_t st);
+// True when the scaled pair form applies (cos(tau t_d) >= 1/2 for every axis and tau).
+bool kin_scaled_ok(const Geometry& g);
 
 // One pass of K_axis over every line of every domain, optionally fused with a phase multiply
 // (phase_mode 1: Phi . psi before the sweep; 2: after).
 cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, const double2* phi,
-                       int axis, int phase_mode, cudaStream_t st);
+                       int axis, int phase_mode, bool scaled, cudaStream_t st);
 
-// Fused pass Psi <- Phi . K_y K_z Psi (one read + write of Psi; nz <= 128).
+// Fused pass Psi <- Phi . K_y K_z Psi (one read + write of Psi; nz <= 80).
 bool kin_yz_supported(const Geometry& g);
-cudaError_t launch_kin_yz(const Geometry& g, double2* psi, const DomCoef* coef, const double2* phi,
-                          cudaStream_t st);
+cudaError_t kin_yz_tensor_map(const Geometry& g, double2* psi, CUtensorMap* out);
+cudaError_t launch_kin_yz(const Geometry& g, const CUtensorMap* tmap, double2* psi, const DomCoef* coef,
+                          const double2* phi, bool scaled, cudaStream_t st);
 cudaError_t kin_yz_set_attributes();
 
 // GEMM-1 split-K: part[dom][split][mrows][ncols] (complex) = sum over the split's grid rows of

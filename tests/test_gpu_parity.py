@@ -255,10 +255,11 @@ def test_launch_count_and_profile():
     lfd.lfd_profile_enable(ctx.ctx, True)
     ctx.step(2)
     prof = lfd.lfd_profile_read(ctx.ctx)
-    # step 1: N (GEMM-1, reduce, norm, GEMM-2), 3 stencil passes, N; step 2's first N takes C from the
-    # projection carry (carry, norm, GEMM-2) instead of GEMM-1 + reduce
-    assert lfd.lfd_launch_count(ctx.ctx) - n0 == 11 + 10
-    assert prof["kin_x"][1] == 2 and prof["nl_proj"][1] == 3 and prof["nl_back"][1] == 4
+    # step 1: N (GEMM-1, reduce, norm, GEMM-2), the stencil passes (Phi.K_x, then Phi.K_y K_z fused), N;
+    # step 2's first N takes C from the projection carry (carry, norm, GEMM-2) instead of GEMM-1 + reduce
+    assert prof["kin_x"][1] == 2 and prof["kin_yz"][1] == 2 and prof["kin_y"][1] == 0
+    assert lfd.lfd_launch_count(ctx.ctx) - n0 == sum(v[1] for v in prof.values()) == 10 + 9
+    assert prof["nl_proj"][1] == 3 and prof["nl_back"][1] == 4
     assert prof["nl_carry"][1] == 1
     assert all(v[0] >= 0 for v in prof.values())
     ctx.close()
