@@ -423,22 +423,10 @@ static size_t yz_smem(int nz, int S) { return (size_t)S * nz * kYZW * 16 + (size
 // Tensor map of Psi for k_kin_yz: 3-D view [ndom*nx*ny planes][nz rows][2*norb doubles], box
 // [1][nz][16 doubles] (one (x, y) plane segment of 8 orbitals), no swizzle (dense rows of 128 B).
 cudaError_t kin_yz_tensor_map(const Geometry& g, double2* psi, CUtensorMap* out) {
-  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
-  if (!encode) {
-    cudaDriverEntryPointQueryResult q;
-    void* fn = nullptr;
-    cudaError_t e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q);
-    if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !fn) return e != cudaSuccess ? e : cudaErrorNotSupported;
-    encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
-  }
-  const cuuint64_t dims[3] = {(cuuint64_t)2 * g.norb, (cuuint64_t)g.nz, (cuuint64_t)g.ndom * g.nx * g.ny};
-  const cuuint64_t strides[2] = {(cuuint64_t)g.norb * 16, (cuuint64_t)g.nz * g.norb * 16};
-  const cuuint32_t box[3] = {2 * kYZW, (cuuint32_t)g.nz, 1};
-  const cuuint32_t estr[3] = {1, 1, 1};
-  CUresult r = encode(out, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, psi, dims, strides, box, estr,
-                      CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
+  const uint64_t dims[3] = {(uint64_t)2 * g.norb, (uint64_t)g.nz, (uint64_t)g.ndom * g.nx * g.ny};
+  const uint64_t strides[2] = {(uint64_t)g.norb * 16, (uint64_t)g.nz * g.norb * 16};
+  const uint32_t box[3] = {2 * kYZW, (uint32_t)g.nz, 1};
+  return encode_tmap_f64(out, 3, psi, dims, strides, box);
 }
 
 cudaError_t kin_yz_set_attributes() {

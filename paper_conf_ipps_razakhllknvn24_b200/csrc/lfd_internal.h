@@ -36,6 +36,11 @@ struct Geometry {
   long long ng;  // points per domain
 };
 
+// TMA tensor map of a float64 tensor (dims innermost first, in elements; strides of dims 1.. in bytes;
+// box in elements), no swizzle, zero fill out of bounds (tmap.cu).
+cudaError_t encode_tmap_f64(CUtensorMap* out, int rank, const void* base, const uint64_t* dims,
+                            const uint64_t* strides_bytes, const uint32_t* box);
+
 // ---- launchers (each returns the cudaError_t of the launch) -------------------------------------
 constexpr int kCoefMaxPerLaunch = 512;
 struct CoefParams {

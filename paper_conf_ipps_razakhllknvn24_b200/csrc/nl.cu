@@ -29,9 +29,12 @@ constexpr int kTile = 64;      // CTA tile 64 x 64 complex
 constexpr int kStages = 4;
 
 // GEMM-1 stage: A rows [KC1][kLd1] (B rows, m along the row) and X rows [KC1][kLd1].
-constexpr int kKC1 = 16;
+constexpr int kKC1 = 32;
 constexpr int kLd1 = kTile + 2;
 constexpr int kStage1Bytes = 2 * kKC1 * kLd1 * 16;
+constexpr int kStages1 = 3;
+constexpr int kConsWarps1 = 8;
+constexpr int kThreads1 = kConsWarps1 * 32 + 32;  // + producer warp
 // GEMM-2 stage: A rows [64][kLdA2] (B rows, k = projector along the row) and C' rows [KC2][kLd1].
 constexpr int kKC2 = 32;
 constexpr int kLdA2 = kKC2 + 4;  // 36 == 4 mod 8: conflict-free A-fragment loads
@@ -183,87 +186,84 @@ __device__ __forceinline__ void mma_conj_4x2(Frag& acc, const double2 (&a)[4], c
 
 // ------------------------------------------------------------------------------------------------
 // GEMM-1: part[dom][split][m][n] = sum_{r in split} conj(A[r][m]) X[r][n];  norms[dom][split][n].
-// grid: (nsplit, mtiles*ntiles, ndom), block 256, dynamic smem kStages*kStage1Bytes + barriers.
+// grid: (nsplit, mtiles*ntiles, ndom), block 8 consumer warps (2 x 4, warp tile 32 x 16 complex) + 1
+// producer warp. Per chunk of kKC1 grid rows the producer issues TWO tiled TMA tensor copies (the A and
+// X row blocks, box [kKC1 rows][66 complex]: the 2 columns past a 64-wide tile are the next tile's or
+// zero fill, which pads every smem row to 66 complex so the DMMA fragment LDS.128 are bank-conflict
+// free) into a kStages1-deep ring with full/empty mbarriers; consumer warps release a stage when done
+// with it (no CTA-wide barrier in the K loop). Rows past the domain end are zero-filled by the TMA
+// (rows_per_split is a multiple of kKC1, so every other chunk is whole). The column norms s_s are
+// accumulated from the X fragments, the k-steps split between the two M-warps of a column slice.
 // ------------------------------------------------------------------------------------------------
-template <bool kTail>
-__device__ __forceinline__ void gemm1_chunk(const double2* As, const double2* Xs, int kv, int wm, int wn, int g,
-                                            int t, Frag& acc, double* nrm, bool do_norm) {
-#pragma unroll
-  for (int kk = 0; kk < kKC1; kk += 4) {
-    const int k = kk + t;
-    const bool ok = !kTail || (k < kv);
-    double2 a[4], x[2];
-#pragma unroll
-    for (int mi = 0; mi < 4; ++mi) a[mi] = ok ? As[k * kLd1 + wm * 32 + mi * 8 + g] : cz();
-#pragma unroll
-    for (int ni = 0; ni < 2; ++ni) x[ni] = ok ? Xs[k * kLd1 + wn * 16 + ni * 8 + g] : cz();
-    if (do_norm) {
-#pragma unroll
-      for (int ni = 0; ni < 2; ++ni) nrm[ni] = fma(x[ni].x, x[ni].x, fma(x[ni].y, x[ni].y, nrm[ni]));
-    }
-    mma_conj_4x2(acc, a, x);
-  }
-}
-
-__global__ void __launch_bounds__(kThreads, 1) k_gemm1(Gemm1Args p) {
+__global__ void __launch_bounds__(kThreads1, 1) k_gemm1(const __grid_constant__ CUtensorMap tA,
+                                                         const __grid_constant__ CUtensorMap tX, Gemm1Args p) {
   extern __shared__ __align__(128) unsigned char smem[];
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kStages * kStage1Bytes);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages1 * kStage1Bytes);
+  uint64_t* empty = full + kStages1;
+  __shared__ double nsh[2][kTile];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int g = lane >> 2, t = lane & 3;
-  const int wm = warp >> 2, wn = warp & 3;
   const int split = blockIdx.x;
   const int ntn = (p.ncols + kTile - 1) / kTile;
   const int mt = blockIdx.y / ntn, nt = blockIdx.y - (blockIdx.y / ntn) * ntn;
   const int dom = blockIdx.z;
   const int m0 = mt * kTile, n0 = nt * kTile;
-  const int mvalid = min(kTile, p.mrows - m0), nvalid = min(kTile, p.ncols - n0);
   const long long kbeg = (long long)split * p.rows_per_split;
   const long long kend = min(p.ng, kbeg + p.rows_per_split);
   const int nchunks = (kend > kbeg) ? (int)((kend - kbeg + kKC1 - 1) / kKC1) : 0;
-  const double2* Ag = p.A + dom * p.a_dom_stride + m0;
-  const double2* Xg = p.X + dom * p.x_dom_stride + n0;
 
   if (tid == 0) {
-    for (int s = 0; s < kStages; ++s) mbar_init(&bars[s], 1);
+    for (int s = 0; s < kStages1; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], kConsWarps1);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
 
-  auto issue = [&](int chunk, int stage) {  // warp 0 only
-    const long long r0 = kbeg + (long long)chunk * kKC1;
-    const int rows = (int)min((long long)kKC1, kend - r0);
-    double2* As = reinterpret_cast<double2*>(smem + stage * kStage1Bytes);
-    double2* Xs = As + kKC1 * kLd1;
-    if (lane == 0) mbar_expect_tx(&bars[stage], (uint32_t)(rows * (mvalid + nvalid) * 16));
-    __syncwarp();
-    if (lane < rows) {
-      tma_row(As + lane * kLd1, Ag + (r0 + lane) * p.mrows, mvalid * 16, &bars[stage]);
-    } else if (lane >= kKC1 && lane - kKC1 < rows) {
-      const int r = lane - kKC1;
-      tma_row(Xs + r * kLd1, Xg + (r0 + r) * p.ncols, nvalid * 16, &bars[stage]);
+  if (warp == kConsWarps1) {  // producer warp
+    if (lane == 0) {
+      for (int i = 0; i < nchunks; ++i) {
+        const int s = i % kStages1;
+        if (i >= kStages1) mbar_wait(&empty[s], (uint32_t)(((i / kStages1) - 1) & 1));
+        mbar_expect_tx(&full[s], (uint32_t)kStage1Bytes);
+        double2* As = reinterpret_cast<double2*>(smem + s * kStage1Bytes);
+        const int r0 = (int)(kbeg + (long long)i * kKC1);
+        tma_3d(As, &tA, 2 * m0, r0, dom, &full[s]);
+        tma_3d(As + kKC1 * kLd1, &tX, 2 * n0, r0, dom, &full[s]);
+      }
     }
-  };
+    return;
+  }
 
-  if (warp == 0)
-    for (int s = 0; s < kStages && s < nchunks; ++s) issue(s, s);
-
+  const int g = lane >> 2, t = lane & 3;
+  const int wm = warp >> 2, wn = warp & 3;
+  const int mvalid = min(kTile, p.mrows - m0), nvalid = min(kTile, p.ncols - n0);
   Frag acc;
   acc.zero();
   double nrm[2] = {0.0, 0.0};
-  const bool do_norm = (p.norms != nullptr) && (mt == 0) && (wm == 0);
+  const bool do_norm = (p.norms != nullptr) && (mt == 0);
 
   for (int i = 0; i < nchunks; ++i) {
-    const int stage = i % kStages;
-    mbar_wait(&bars[stage], (uint32_t)((i / kStages) & 1));
-    const double2* As = reinterpret_cast<const double2*>(smem + stage * kStage1Bytes);
+    const int s = i % kStages1;
+    mbar_wait(&full[s], (uint32_t)((i / kStages1) & 1));
+    const double2* As = reinterpret_cast<const double2*>(smem + s * kStage1Bytes);
     const double2* Xs = As + kKC1 * kLd1;
-    const int kv = (int)min((long long)kKC1, kend - (kbeg + (long long)i * kKC1));
-    if (kv == kKC1)
-      gemm1_chunk<false>(As, Xs, kv, wm, wn, g, t, acc, nrm, do_norm);
-    else
-      gemm1_chunk<true>(As, Xs, kv, wm, wn, g, t, acc, nrm, do_norm);
-    __syncthreads();
-    if (warp == 0 && i + kStages < nchunks) issue(i + kStages, stage);
+#pragma unroll
+    for (int kk = 0; kk < kKC1; kk += 4) {
+      const int k = kk + t;
+      double2 a[4], x[2];
+#pragma unroll
+      for (int mi = 0; mi < 4; ++mi) a[mi] = As[k * kLd1 + wm * 32 + mi * 8 + g];
+#pragma unroll
+      for (int ni = 0; ni < 2; ++ni) x[ni] = Xs[k * kLd1 + wn * 16 + ni * 8 + g];
+      if (do_norm && ((kk >> 2) & 1) == wm) {
+#pragma unroll
+        for (int ni = 0; ni < 2; ++ni) nrm[ni] = fma(x[ni].x, x[ni].x, fma(x[ni].y, x[ni].y, nrm[ni]));
+      }
+      mma_conj_4x2(acc, a, x);
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[s]);
   }
 
   // epilogue: split partials (fixed positions, reduced in order by k_reduce)
@@ -287,20 +287,36 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm1(Gemm1Args p) {
       double v = nrm[ni];
       v += __shfl_xor_sync(0xffffffffu, v, 1);
       v += __shfl_xor_sync(0xffffffffu, v, 2);
-      const int col = wn * 16 + ni * 8 + g;
-      if (t == 0 && col < nvalid)
-        p.norms[((long long)dom * p.nsplit + split) * p.ncols + n0 + col] = v;
+      if (t == 0) nsh[wm][wn * 16 + ni * 8 + g] = v;
     }
+    asm volatile("bar.sync 1, %0;" ::"n"(kConsWarps1 * 32));  // consumer warps only
+    if (tid < nvalid)
+      p.norms[((long long)dom * p.nsplit + split) * p.ncols + n0 + tid] = nsh[0][tid] + nsh[1][tid];
   }
 }
 
-int gemm1_smem_bytes() { return kStages * kStage1Bytes + kStages * 8; }
+// A [dom][ng][mrows] / X [dom][ng][ncols] complex as 3-D float64 tensors, box [1][kKC1][2*kLd1].
+static cudaError_t gemm1_maps(const Gemm1Args& a, CUtensorMap* tA, CUtensorMap* tX) {
+  const uint32_t box[3] = {2 * kLd1, kKC1, 1};
+  const uint64_t dA[3] = {(uint64_t)2 * a.mrows, (uint64_t)a.ng, (uint64_t)a.ndom};
+  const uint64_t sA[2] = {(uint64_t)a.mrows * 16, (uint64_t)a.a_dom_stride * 16};
+  cudaError_t e = encode_tmap_f64(tA, 3, a.A, dA, sA, box);
+  if (e != cudaSuccess) return e;
+  const uint64_t dX[3] = {(uint64_t)2 * a.ncols, (uint64_t)a.ng, (uint64_t)a.ndom};
+  const uint64_t sX[2] = {(uint64_t)a.ncols * 16, (uint64_t)a.x_dom_stride * 16};
+  return encode_tmap_f64(tX, 3, a.X, dX, sX, box);
+}
+
+int gemm1_smem_bytes() { return kStages1 * kStage1Bytes + 2 * kStages1 * 8; }
 int gemm2_smem_bytes() { return kStages2 * kStage2Bytes + kStages2 * 8; }
 
 cudaError_t launch_gemm1(const Gemm1Args& a, cudaStream_t st) {
   const int tiles = ((a.mrows + kTile - 1) / kTile) * ((a.ncols + kTile - 1) / kTile);
   dim3 grid(a.nsplit, tiles, a.ndom);
-  k_gemm1<<<grid, kThreads, gemm1_smem_bytes(), st>>>(a);
+  CUtensorMap tA, tX;
+  cudaError_t e = gemm1_maps(a, &tA, &tX);
+  if (e != cudaSuccess) return e;
+  k_gemm1<<<grid, kThreads1, gemm1_smem_bytes(), st>>>(tA, tX, a);
   return cudaGetLastError();
 }
 
@@ -844,11 +860,172 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
   }
 }
 
+// ------------------------------------------------------------------------------------------------
+// GEMM-2, TMA tensor-map variant for nproj <= 64 (the paper-shaped case). Thread 0 issues, per work item,
+// ONE tiled tensor copy of the item's 64 B rows (box [64 rows][lda complex]; the columns past nproj are
+// zero fill, which pads the smem rows to lda == 4 mod 8 complex so the A-fragment LDS.128 are
+// conflict free) into a 2-deep ring (full/empty mbarriers), plus an L2 prefetch of the item's Psi rows
+// for the epilogue. C' of the current (domain, column tile) stays resident (one tensor
+// copy when it changes), the K loop is fully unrolled for nproj = 64, the epilogue's Psi loads are
+// issued mid-loop and Psi <- n_s (Psi + B C') is written in place.
+// ------------------------------------------------------------------------------------------------
+template <int kNP>
+__global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant__ CUtensorMap tB,
+                                                             const __grid_constant__ CUtensorMap tC, Gemm2Args p) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  double2* Cs = reinterpret_cast<double2*>(smem + kFullStages * kFullABytes);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kFullStages * kFullABytes + kFullCBytes);
+  uint64_t* empty = full + kFullStages;
+  uint64_t* cbar = empty + kFullStages;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int np = kNP > 0 ? kNP : p.nproj;
+  const int lda = full_lda(np);
+  const long long rblocks = (p.ng + kTile - 1) / kTile;
+  const int ntn = (p.norb + kTile - 1) / kTile;
+  const long long items = (long long)p.ndom * ntn * rblocks;
+  const long long my_items = (items > blockIdx.x) ? (items - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+  constexpr int kNK4 = kNP > 0 ? (kNP + 3) / 4 : 16;
+  const int nk4 = (np + 3) / 4;
+
+  if (tid == 0) {
+    for (int s = 0; s < kFullStages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], kConsWarps1);
+    }
+    mbar_init(cbar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+
+  auto decode = [&](long long j, int& dom, int& n0, long long& r0) {
+    const long long item = blockIdx.x + j * gridDim.x;
+    const long long per_dom = (long long)ntn * rblocks;
+    dom = (int)(item / per_dom);
+    const long long rem = item - dom * per_dom;
+    const int nt = (int)(rem / rblocks);
+    n0 = nt * kTile;
+    r0 = (rem - (long long)nt * rblocks) * kTile;
+  };
+
+  // item j -> stage j % kFullStages: ONE tensor copy of its B rows + L2 prefetch of its Psi rows
+  auto issue = [&](long long j) {
+    const int s = (int)(j % kFullStages);
+    int dom, n0;
+    long long r0;
+    decode(j, dom, n0, r0);
+    mbar_expect_tx(&full[s], (uint32_t)(kTile * lda * 16));
+    tma_3d(smem + s * kFullABytes, &tB, 0, (int)r0, dom, &full[s]);
+    const long long rows = min((long long)kTile, p.ng - r0);
+    l2_prefetch(p.psi + ((long long)dom * p.ng + r0) * p.norb, (uint32_t)(rows * p.norb * 16));
+  };
+  if (tid == 0)
+    for (long long j = 0; j < kFullStages && j < my_items; ++j) issue(j);
+
+  const int g = lane >> 2, t = lane & 3;
+  const int wm = warp >> 2, wn = warp & 3;
+  int cur_dom = -1, cur_n0 = -1;
+  uint32_t cphase = 0;
+  for (long long j = 0; j < my_items; ++j) {
+    int dom, n0;
+    long long r0;
+    decode(j, dom, n0, r0);
+    if (dom != cur_dom || n0 != cur_n0) {  // (re)load C'[dom][:, n0:n0+64] once every consumer is past Cs
+      asm volatile("bar.sync 1, %0;" ::"n"(kConsWarps1 * 32));
+      if (tid == 0) {
+        mbar_expect_tx(cbar, (uint32_t)(np * kLd1 * 16));
+        tma_3d(Cs, &tC, 2 * n0, 0, dom, cbar);
+      }
+      mbar_wait(cbar, cphase);
+      cphase ^= 1;
+      cur_dom = dom;
+      cur_n0 = n0;
+    }
+    const int s = (int)(j % kFullStages);
+    mbar_wait(&full[s], (uint32_t)((j / kFullStages) & 1));
+    const double2* As = reinterpret_cast<const double2*>(smem + s * kFullABytes);
+    Frag acc;
+    acc.zero();
+    double2* psi = p.psi + (long long)dom * p.ng * p.norb;
+    double2 pv[4][2][2];
+    auto load_pv = [&]() {
+#pragma unroll
+      for (int mi = 0; mi < 4; ++mi) {
+        const long long r = r0 + wm * 32 + mi * 8 + g;
+#pragma unroll
+        for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+          for (int c = 0; c < 2; ++c) {
+            const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
+            pv[mi][ni][c] = (r < p.ng && col < p.norb) ? psi[r * p.norb + col] : cz();
+          }
+      }
+    };
+#pragma unroll
+    for (int kk = 0; kk < kNK4; ++kk) {
+      if (kNP == 0 && kk >= nk4) break;
+      if (kk == kNK4 / 2) load_pv();  // Psi loads (L2 hits) in flight during the second half
+      const int k = kk * 4 + t;
+      double2 a[4], c[2];
+#pragma unroll
+      for (int mi = 0; mi < 4; ++mi) a[mi] = As[(wm * 32 + mi * 8 + g) * lda + k];
+#pragma unroll
+      for (int ni = 0; ni < 2; ++ni) c[ni] = Cs[k * kLd1 + wn * 16 + ni * 8 + g];
+      mma_4x2(acc, a, c);
+    }
+    if (kNP == 0 && nk4 <= kNK4 / 2) load_pv();
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[s]);
+    if (tid == 0 && j + kFullStages < my_items) {  // refill the stage once every warp has released it
+      mbar_wait(&empty[s], (uint32_t)((j / kFullStages) & 1));
+      issue(j + kFullStages);
+    }
+    // epilogue: Psi <- n_s (Psi + B C')
+    const double* nf = p.nfac + (long long)dom * p.norb;
+#pragma unroll
+    for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+      for (int c = 0; c < 2; ++c) {
+        const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
+        if (col >= p.norb) continue;
+        const double f = nf[col];
+#pragma unroll
+        for (int mi = 0; mi < 4; ++mi) {
+          const long long r = r0 + wm * 32 + mi * 8 + g;
+          if (r < p.ng)
+            psi[r * p.norb + col] =
+                make_double2(f * (pv[mi][ni][c].x + acc.re(mi, ni, c)), f * (pv[mi][ni][c].y + acc.im(mi, ni, c)));
+        }
+      }
+  }
+}
+
+// B [dom][ng][nproj] (box [1][64 rows][lda]) and C' [dom][nproj][norb] (box [1][nproj][kLd1]).
+static cudaError_t gemm2_maps(const Gemm2Args& a, CUtensorMap* tB, CUtensorMap* tC) {
+  const int lda = full_lda(a.nproj);
+  const uint64_t dB[3] = {(uint64_t)2 * a.nproj, (uint64_t)a.ng, (uint64_t)a.ndom};
+  const uint64_t sB[2] = {(uint64_t)a.nproj * 16, (uint64_t)a.ng * a.nproj * 16};
+  const uint32_t bB[3] = {(uint32_t)(2 * lda), kTile, 1};
+  cudaError_t e = encode_tmap_f64(tB, 3, a.B, dB, sB, bB);
+  if (e != cudaSuccess) return e;
+  const uint64_t dC[3] = {(uint64_t)2 * a.norb, (uint64_t)a.nproj, (uint64_t)a.ndom};
+  const uint64_t sC[2] = {(uint64_t)a.norb * 16, (uint64_t)a.nproj * a.norb * 16};
+  const uint32_t bC[3] = {2 * kLd1, (uint32_t)a.nproj, 1};
+  return encode_tmap_f64(tC, 3, a.Cp, dC, sC, bC);
+}
+
 cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
   const long long rblocks = (a.ng + kTile - 1) / kTile;
   const long long items = (long long)a.ndom * rblocks * ((a.norb + kTile - 1) / kTile);
   const int grid = (int)(items < a.num_sms ? items : a.num_sms);
-  if (a.nproj == kTile && a.variant == 1)
+  if (a.nproj <= kTile && a.variant == 2) {
+    CUtensorMap tB, tC;
+    cudaError_t e = gemm2_maps(a, &tB, &tC);
+    if (e != cudaSuccess) return e;
+    if (a.nproj == kTile)
+      k_gemm2_tma<kTile><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+    else
+      k_gemm2_tma<0><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+  } else if (a.nproj == kTile && a.variant == 1)
     k_gemm2_fullk<kTile, true><<<grid, kThreads, kFullSmem, st>>>(a);
   else if (a.nproj == kTile)
     k_gemm2_fullk<kTile, false><<<grid, kThreads, kFullSmem, st>>>(a);
@@ -867,6 +1044,10 @@ cudaError_t gemm_set_attributes() {
   e = cudaFuncSetAttribute(k_gemm2_fullk<kTile, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_gemm2_fullk<0, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_gemm2_tma<kTile>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem + 16);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_gemm2_tma<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem + 16);
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(k_gemm2, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm2_smem_bytes());
 }
