@@ -278,17 +278,18 @@ __global__ void __launch_bounds__(256, 3) k_kin(double2* __restrict__ psi, const
 // ------------------------------------------------------------------------------------------------
 constexpr int kYZW = 8;
 constexpr int kYZMaxThreads = 352;  // up to 40 z pairs x 8 orbitals + the producer warp
+constexpr int kYZS = 8;             // ring depth (planes)
 
 template <bool kPer, bool kS>
 __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant__ CUtensorMap tmap,
                                                           double2* __restrict__ psi, const DomCoef* __restrict__ coef,
                                                           const double2* __restrict__ phi, int nx, int ny, int nz,
-                                                          int norb, int nchunks, long long ng, int S) {
+                                                          int norb, int nchunks, long long ng) {
   extern __shared__ __align__(128) unsigned char smem[];
   const int seg = nz * kYZW;  // complex elements per plane segment
   double2* ring = reinterpret_cast<double2*>(smem);
-  uint64_t* full = reinterpret_cast<uint64_t*>(ring + (long long)S * seg);
-  uint64_t* empty = full + S;
+  uint64_t* full = reinterpret_cast<uint64_t*>(ring + kYZS * seg);
+  uint64_t* empty = full + kYZS;
   const int dom = blockIdx.y;
   const int x = blockIdx.x / nchunks, oc = blockIdx.x - (blockIdx.x / nchunks) * nchunks;
   const int o0 = oc * kYZW, wv = min(kYZW, norb - o0);
@@ -302,7 +303,7 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
   if (tid == 0) {
     sc[0] = pair_coef<kS>(coef + dom, 2);
     sc[1] = pair_coef<kS>(coef + dom, 1);
-    for (int s = 0; s < S; ++s) {
+    for (int s = 0; s < kYZS; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], nconsw);
     }
@@ -310,14 +311,16 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
   }
   __syncthreads();
 
-  if (tid >= nconsw * 32) {  // producer warp: plane y -> slot y % S, one tensor copy per plane
+  if (tid >= nconsw * 32) {  // producer warp: plane y -> slot y % kYZS, one tensor copy per plane
     if (tid == nconsw * 32) {
       const int row0 = (dom * nx + x) * ny;
+      int s = 0;
+      uint32_t ph = 0;
       for (int y = 0; y < ny; ++y) {
-        const int s = y % S;
-        if (y >= S) mbar_wait(&empty[s], (uint32_t)(((y / S) - 1) & 1));
+        if (y >= kYZS) mbar_wait(&empty[s], ph ^ 1);
         mbar_expect_tx(&full[s], (uint32_t)(seg * 16));
-        tma_3d(ring + (long long)s * seg, &tmap, 2 * o0, 0, row0 + y, &full[s]);
+        tma_3d(ring + s * seg, &tmap, 2 * o0, 0, row0 + y, &full[s]);
+        if (++s == kYZS) { s = 0; ph ^= 1; }
       }
     }
     return;
@@ -326,99 +329,97 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
   const int o = tid % kYZW, m = tid / kYZW;
   const bool live = m < npz;
   const int z0 = 2 * m, z1 = 2 * m + 1;
-  const bool has1 = z1 < nz;
+  const bool has1 = live && z1 < nz;
   const bool act = live && o < wv;
-  const long long yst = (long long)nz * norb;  // element stride between y planes
-  double2* base = psi + (long long)dom * ng * norb + (long long)x * ny * yst + o0;
-  const double2* phb = phi + (long long)dom * ng + (long long)x * ny * nz;
+  // ring offsets (complex elements within a slot) of the six points this thread's K_z reads
+  const int zl = (m > 0) ? z0 - 2 : nz - 2;                    // pair m-1 (periodic wrap for m == 0)
+  const int zr = (z1 + 1 < nz) ? z1 + 1 : 0;                   // pair m+1 (periodic wrap at the end)
+  const bool has_l = live && (m > 0 || kPer);                  // link (2m-1, 2m) exists
+  const bool has_r = has1 && (z1 + 1 < nz || kPer);            // link (2m+1, 2m+2) exists
+  const bool r_single = zr + 1 >= nz;                          // pair m+1 is a zero-BC singleton
+  const int oz0 = live ? z0 * kYZW + o : o, oz1 = has1 ? z1 * kYZW + o : o;
+  const int ozl = has_l ? zl * kYZW + o : o, ozl1 = has_l ? (zl + 1) * kYZW + o : o;
+  const int ozr = has_r ? zr * kYZW + o : o, ozr1 = (has_r && !r_single) ? (zr + 1) * kYZW + o : o;
+  const int yst = nz * norb;  // element stride between y planes (< 2^31 per domain, validated)
+  double2* out0 = psi + (long long)dom * ng * norb + (long long)x * ny * yst + o0 + z0 * norb + o;
+  double2* out1 = out0 + norb;
+  const double2* ph0 = phi + (long long)dom * ng + (long long)x * ny * nz + z0;  // Phi(x, y=0, z0)
 
-  // K_z of plane y for this thread's pair: the first E(Delta/2) on pairs m-1, m, m+1 (the neighbours'
-  // outputs recomputed here), O(Delta) on the links (2m-1, 2m) and (2m+1, 2m+2), then the second
-  // E(Delta/2) on (2m, 2m+1). The slot is released to the producer afterwards.
-  auto kz = [&](int y, double2& w0, double2& w1) {
-    const int s = y % S;
-    mbar_wait(&full[s], (uint32_t)((y / S) & 1));
-    const double2* r = ring + (long long)s * seg + o;
-    auto v = [&](int z) { return r[z * kYZW]; };
-    w0 = w1 = cz();
-    if (live) {
-      double2 e0, e1 = cz();
-      if (has1) {
-        const double2 a = v(z0), b = v(z1);
-        e0 = lk_L<kS>(cz_.a1, cz_.u1, a, b);
-        e1 = lk_R<kS>(cz_.a1, cz_.d1, a, b);
-      } else {
-        e0 = lk_S<kS>(cz_.s1, v(z0));
-      }
-      double2 q0, q1 = cz();
-      if (m > 0 || kPer) {  // link (2m-1, 2m): E output of z = 2m-1 (pair m-1, its right point)
-        const int zl = (m > 0) ? z0 - 2 : nz - 2;
-        const double2 l1 = lk_R<kS>(cz_.a1, cz_.d1, v(zl), v(zl + 1));
-        q0 = lk_R<kS>(cz_.a2, cz_.d2, l1, e0);
-      } else {
-        q0 = lk_S<kS>(cz_.s2, e0);
-      }
-      if (has1) {
-        if (z1 + 1 < nz || kPer) {  // link (2m+1, 2m+2): E output of z = 2m+2 (pair m+1, its left point)
-          const int zr = (z1 + 1 < nz) ? z1 + 1 : 0;
-          const double2 r0 = (zr + 1 < nz) ? lk_L<kS>(cz_.a1, cz_.u1, v(zr), v(zr + 1)) : lk_S<kS>(cz_.s1, v(zr));
-          q1 = lk_L<kS>(cz_.a2, cz_.u2, e1, r0);
-        } else {
-          q1 = lk_S<kS>(cz_.s2, e1);
-        }
-        w0 = lk_L<kS>(cz_.a1, cz_.u1, q0, q1);
-        w1 = lk_R<kS>(cz_.a1, cz_.d1, q0, q1);
-      } else {
-        w0 = lk_S<kS>(cz_.s1, q0);
-      }
-    }
+  int slot = 0;
+  uint32_t phase = 0;
+  // K_z of the next plane (in y order) for this thread's pair: the first E(Delta/2) on pairs m-1, m,
+  // m+1 (the neighbours' outputs recomputed here), O(Delta) on the links (2m-1, 2m), (2m+1, 2m+2), then
+  // the second E(Delta/2) on (2m, 2m+1). The slot is released to the producer afterwards.
+  auto kz = [&](double2& w0, double2& w1) {
+    mbar_wait(&full[slot], phase);
+    const double2* r = ring + slot * seg;
+    const double2 a = r[oz0], b = r[oz1], vl = r[ozl], vl1 = r[ozl1], vr = r[ozr], vr1 = r[ozr1];
     __syncwarp();
-    if ((tid & 31) == 0) mbar_arrive(&empty[s]);
+    if ((tid & 31) == 0) mbar_arrive(&empty[slot]);
+    if (++slot == kYZS) { slot = 0; phase ^= 1; }
+    double2 e0, e1 = cz();
+    if (has1) {
+      e0 = lk_L<kS>(cz_.a1, cz_.u1, a, b);
+      e1 = lk_R<kS>(cz_.a1, cz_.d1, a, b);
+    } else {
+      e0 = lk_S<kS>(cz_.s1, a);
+    }
+    const double2 q0 = has_l ? lk_R<kS>(cz_.a2, cz_.d2, lk_R<kS>(cz_.a1, cz_.d1, vl, vl1), e0) : lk_S<kS>(cz_.s2, e0);
+    if (has1) {
+      double2 q1;
+      if (has_r) {
+        const double2 r0 = r_single ? lk_S<kS>(cz_.s1, vr) : lk_L<kS>(cz_.a1, cz_.u1, vr, vr1);
+        q1 = lk_L<kS>(cz_.a2, cz_.u2, e1, r0);
+      } else {
+        q1 = lk_S<kS>(cz_.s2, e1);
+      }
+      w0 = lk_L<kS>(cz_.a1, cz_.u1, q0, q1);
+      w1 = lk_R<kS>(cz_.a1, cz_.d1, q0, q1);
+    } else {
+      w0 = lk_S<kS>(cz_.s1, q0);
+      w1 = cz();
+    }
   };
-  auto ph = [&](int y, int z) { return (live && z < nz) ? __ldg(phb + (long long)y * nz + z) : cz(); };
-  auto put = [&](int y, int z, double2 f, double2 v) {
-    if (act && z < nz) base[(long long)y * yst + (long long)z * norb + o] = cmul(f, v);
+  auto ph = [&](int y, int dz) { return live ? __ldg(ph0 + y * nz + dz) : cz(); };
+  auto put0 = [&](int y, double2 f, double2 v) {
+    if (act) out0[y * yst] = cmul(f, v);
+  };
+  auto put1 = [&](int y, double2 f, double2 v) {
+    if (act && has1) out1[y * yst] = cmul(f, v);
   };
 
-  // Phi of planes 0 and 1 (stored last, by the wrap) stays in registers
-  const double2 f00 = ph(0, z0), f01 = ph(0, z1), f10 = ph(1, z0), f11 = ph(1, z1);
   LineMarch<kS> L0, L1;
   L0.init();
   L1.init();
   const int npairs = (ny + 1) >> 1;
   for (int p = 0; p < npairs; ++p) {
-    const int ya = 2 * p, yb = 2 * p + 1;
-    const bool hb = yb < ny;
+    const int ya = 2 * p;
+    const bool hb = ya + 1 < ny;
     // Phi of the two planes this iteration's march step stores (2p-2, 2p-1): loads in flight meanwhile
     double2 fa0 = cz(), fa1 = cz(), fb0 = cz(), fb1 = cz();
     if (p >= 2) {
-      fa0 = ph(ya - 2, z0); fa1 = ph(ya - 2, z1);
-      fb0 = ph(ya - 1, z0); fb1 = ph(ya - 1, z1);
+      fa0 = ph(ya - 2, 0); fa1 = ph(ya - 2, 1);
+      fb0 = ph(ya - 1, 0); fb1 = ph(ya - 1, 1);
     }
     double2 wa0, wa1, wb0 = cz(), wb1 = cz();
-    kz(ya, wa0, wa1);
-    if (hb) kz(yb, wb0, wb1);
-    L0.push(cy, p, wa0, wb0, hb, [&](int y, double2 v) { put(y, z0, y == ya - 2 ? fa0 : fb0, v); });
-    L1.push(cy, p, wa1, wb1, hb, [&](int y, double2 v) { put(y, z1, y == ya - 2 ? fa1 : fb1, v); });
+    kz(wa0, wa1);
+    if (hb) kz(wb0, wb1);
+    L0.push(cy, p, wa0, wb0, hb, [&](int y, double2 v) { put0(y, y == ya - 2 ? fa0 : fb0, v); });
+    L1.push(cy, p, wa1, wb1, hb, [&](int y, double2 v) { put1(y, y == ya - 2 ? fa1 : fb1, v); });
   }
   // wrap: planes ny-2, ny-1 (or ny-1 for odd ny) and 0, 1
-  const double2 fl0 = ph(ny - 1, z0), fl1 = ph(ny - 1, z1);
-  const double2 fm0 = ph(ny - 2, z0), fm1 = ph(ny - 2, z1);
+  const double2 f00 = ph(0, 0), f01 = ph(0, 1), f10 = ph(1, 0), f11 = ph(1, 1);
+  const double2 fl0 = ph(ny - 1, 0), fl1 = ph(ny - 1, 1);
+  const double2 fm0 = ph(ny - 2, 0), fm1 = ph(ny - 2, 1);
   auto pick0 = [&](int y) { return y == 0 ? f00 : y == 1 ? f10 : y == ny - 1 ? fl0 : fm0; };
   auto pick1 = [&](int y) { return y == 0 ? f01 : y == 1 ? f11 : y == ny - 1 ? fl1 : fm1; };
-  L0.template finish<kPer>(cy, ny, [&](int y, double2 v) { put(y, z0, pick0(y), v); });
-  L1.template finish<kPer>(cy, ny, [&](int y, double2 v) { put(y, z1, pick1(y), v); });
+  L0.template finish<kPer>(cy, ny, [&](int y, double2 v) { put0(y, pick0(y), v); });
+  L1.template finish<kPer>(cy, ny, [&](int y, double2 v) { put1(y, pick1(y), v); });
 }
 
-static int yz_stages(int nz) {
-  const int seg_bytes = nz * kYZW * 16;
-  int S = (200 * 1024) / seg_bytes;
-  return S > 12 ? 12 : S;
-}
+bool kin_yz_supported(const Geometry& g) { return g.nz <= 80; }
 
-bool kin_yz_supported(const Geometry& g) { return g.nz <= 80 && yz_stages(g.nz) >= 2; }
-
-static size_t yz_smem(int nz, int S) { return (size_t)S * nz * kYZW * 16 + (size_t)S * 16; }
+static size_t yz_smem(int nz) { return (size_t)kYZS * nz * kYZW * 16 + (size_t)kYZS * 16; }
 
 // Tensor map of Psi for k_kin_yz: 3-D view [ndom*nx*ny planes][nz rows][2*norb doubles], box
 // [1][nz][16 doubles] (one (x, y) plane segment of 8 orbitals), no swizzle (dense rows of 128 B).
@@ -441,12 +442,11 @@ cudaError_t kin_yz_set_attributes() {
 cudaError_t launch_kin_yz(const Geometry& g, const CUtensorMap* tmap, double2* psi, const DomCoef* coef,
                           const double2* phi, bool scaled, cudaStream_t st) {
   const int nchunks = (g.norb + kYZW - 1) / kYZW;
-  const int S = yz_stages(g.nz);
   const int threads = ((((g.nz + 1) / 2) * kYZW + 31) / 32 + 1) * 32;  // consumer warps + producer warp
   dim3 grid(g.nx * nchunks, g.ndom);
-  const size_t sm = yz_smem(g.nz, S);
+  const size_t sm = yz_smem(g.nz);
 #define LFD_KYZ(P, K) \
-  k_kin_yz<P, K><<<grid, threads, sm, st>>>(*tmap, psi, coef, phi, g.nx, g.ny, g.nz, g.norb, nchunks, g.ng, S)
+  k_kin_yz<P, K><<<grid, threads, sm, st>>>(*tmap, psi, coef, phi, g.nx, g.ny, g.nz, g.norb, nchunks, g.ng)
   if (g.bc == 0) {
     if (scaled) LFD_KYZ(true, true); else LFD_KYZ(true, false);
   } else {
