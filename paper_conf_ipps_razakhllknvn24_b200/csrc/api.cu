@@ -171,6 +171,7 @@ struct lfd_ctx {
   bool carry = true;
   bool kin_fused = true;  // Phi.K_y K_z in one pass (env LFD_KIN_FUSED=0: separate y and z passes)
   CUtensorMap psi_tmap;   // TMA descriptor of Psi for the fused pass
+  lfd::DensMaps* dmaps = nullptr;  // TMA descriptors of Psi for the density kernel
   bool scaled = true;     // scaled pair form of the stencil (env LFD_KIN_SCALED=0: general 2x2 form)
   std::string err = "no error";
   // density-current global layout cache
@@ -387,7 +388,7 @@ lfd_status density_into(lfd_ctx* c, double* rho, double* j, double* Jmac, const 
   a.base = base_dev; a.jbase = base_dev + c->g.ndom; a.sx = sx; a.sy = sy; a.jstride = jstride;
   a.v = energy ? c->at<double>(c->L.vstage) : nullptr;
   a.epart = energy ? c->at<double>(c->L.epart) : nullptr;
-  LFD_TRY(launch(c, LFD_K_DENSITY, "k_density", [&] { return lfd::launch_density(c->g, a, c->stream); }));
+  LFD_TRY(launch(c, LFD_K_DENSITY, "k_density", [&] { return lfd::launch_density(c->g, a, c->dmaps, c->stream); }));
   if (Jmac)
     LFD_TRY(launch(c, LFD_K_JREDUCE, "k_jreduce",
                    [&] { return lfd::launch_jreduce(c->g, a.jline, Jmac, c->stream); }));
@@ -457,6 +458,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   if (const char* v = std::getenv("LFD_KIN_SCALED")) c->scaled = std::atoi(v) != 0;
   c->scaled = c->scaled && lfd::kin_scaled_ok(g);
   c->kin_fused = c->kin_fused && lfd::kin_yz_supported(g);
+  c->dmaps = lfd::density_maps_create(g, c->psi);
   if (c->kin_fused && lfd::kin_yz_tensor_map(g, c->psi, &c->psi_tmap) != cudaSuccess) {
     cudaGetLastError();
     c->kin_fused = false;  // descriptor not encodable (e.g. alignment): the separate y and z passes
@@ -746,6 +748,7 @@ lfd_status lfd_destroy(lfd_ctx* c) {
       cudaEventDestroy(s.b);
     }
   }
+  lfd::density_maps_destroy(c->dmaps);
   delete c;
   return LFD_OK;
 }

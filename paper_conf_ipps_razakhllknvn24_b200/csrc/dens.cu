@@ -10,6 +10,8 @@
 #include "lfd_internal.h"
 #include "lfd_tma.cuh"
 
+#include <new>
+
 namespace lfd {
 
 // Tiling: a CTA owns a (kTY x kTZ) tile of (y, z) points and a chunk of kXC x-planes, which it walks in
@@ -296,16 +298,251 @@ __global__ void __launch_bounds__(kDensThreads) k_density_tma(Geometry g, DensAr
   }
 }
 
+// ------------------------------------------------------------------------------------------------
+// y-marching variant (norb <= 128; the bench shape). CTA = (x plane, z chunk of zc points, domain): it
+// walks y and needs, at step y, the z-line segment of its own points (x, y, z0..z0+zc) plus the z+1
+// halo point, the next line (x, y+1) for the y links and the line (x+1, y) for the x links. A producer
+// warp brings each segment with one tiled TMA tensor copy (all orbitals of zc points; the halo point is
+// a second, 1-point copy) into two
+// rings (own lines: 3 slots, x+1 lines: 2 slots) with full/empty mbarriers; the own line y+1 stays
+// resident for the next step, and the x+1 lines are the next CTA's own lines, read about when that CTA
+// reads them (L2 hits). kSub lanes per point split the orbitals and the 7 per-point sums are shuffle
+// reductions with the occupation weights (kept in shared memory).
+// ------------------------------------------------------------------------------------------------
+constexpr int kYOwn = 3, kYXp = 2;
+constexpr int kYMaxThreads = 544;  // up to 64 points x kSub + the producer warp
+
+struct DensMaps {
+  CUtensorMap seg;   // box [1][zc][2*norb]: a z-line segment of zc points, all orbitals
+  CUtensorMap one;   // box [1][1][2*norb]: the z+1 halo point
+  int zc;            // points per CTA (divides nz)
+};
+
+// shared-memory layout of the y-marching kernel (every TMA destination 128-byte aligned)
+struct YLayout {
+  size_t seg_b, halo_b, own_b, xp_b, fsh_off, bar_off, total;
+  __host__ __device__ YLayout(int zc, int norb) {
+    seg_b = ((size_t)zc * norb * 16 + 127) & ~(size_t)127;
+    halo_b = ((size_t)norb * 16 + 127) & ~(size_t)127;
+    own_b = seg_b + halo_b;
+    xp_b = seg_b;
+    fsh_off = kYOwn * own_b + kYXp * xp_b;
+    bar_off = fsh_off + (((size_t)norb * 8 + 15) & ~(size_t)15);
+    total = bar_off + (2 * kYOwn + 2 * kYXp) * 8;
+  }
+};
+
+static int ymarch_zc(const Geometry& g) {
+  if (g.norb > 128) return 0;
+  const size_t per_pt = (size_t)g.norb * 16;
+  for (int nzc = 1; nzc <= g.nz; ++nzc) {
+    if (g.nz % nzc) continue;
+    const int zc = g.nz / nzc;
+    if (zc > 64) continue;
+    (void)per_pt;
+    if (YLayout(zc, g.norb).total <= 200 * 1024) return zc;
+  }
+  return 0;
+}
+
+__global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constant__ DensMaps mp, Geometry g,
+                                                            DensArgs a) {
+  extern __shared__ __align__(128) unsigned char dsm[];
+  const int norb = g.norb, zc = mp.zc;
+  const YLayout Ly(zc, norb);
+  auto own_slot = [&](int s) { return reinterpret_cast<double2*>(dsm + s * Ly.own_b); };
+  auto halo_of = [&](int s) { return reinterpret_cast<double2*>(dsm + s * Ly.own_b + Ly.seg_b); };
+  auto xp_slot = [&](int s) { return reinterpret_cast<double2*>(dsm + kYOwn * Ly.own_b + s * Ly.xp_b); };
+  double* fsh = reinterpret_cast<double*>(dsm + Ly.fsh_off);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(dsm + Ly.bar_off);
+  uint64_t *ofull = bars, *oempty = bars + kYOwn, *xfull = bars + 2 * kYOwn, *xempty = xfull + kYXp;
+  __shared__ double jsh[5][kYMaxThreads / kSub];
+  const int dom = blockIdx.y;
+  const int nzc = g.nz / zc;
+  const int x = blockIdx.x / nzc, z0 = (blockIdx.x - x * nzc) * zc;
+  const bool per = (g.bc == 0);
+  const bool has_x = per || x + 1 < g.nx;
+  const int xp = (x + 1 == g.nx) ? 0 : x + 1;
+  const bool last_chunk = z0 + zc == g.nz;
+  const int nconsw = (zc * kSub + 31) >> 5;
+  const int tid = threadIdx.x;
+  const int nown = per ? g.ny + 1 : g.ny;  // own lines y = 0..ny-1 (+ y = 0 again for the periodic wrap)
+  if (tid == 0) {
+    for (int s = 0; s < kYOwn; ++s) { mbar_init(&ofull[s], 1); mbar_init(&oempty[s], nconsw); }
+    for (int s = 0; s < kYXp; ++s) { mbar_init(&xfull[s], 1); mbar_init(&xempty[s], nconsw); }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  for (int s = tid; s < norb; s += blockDim.x) fsh[s] = a.occ[(long long)dom * norb + s];
+  __syncthreads();
+
+  if (tid >= nconsw * 32) {  // producer warp
+    if (tid == nconsw * 32) {
+      const int rowx = (dom * g.nx + x) * g.ny, rowxp = (dom * g.nx + xp) * g.ny;
+      auto issue_own = [&](int k) {  // own line k (k == ny: plane 0 again)
+        const int s = k % kYOwn;
+        if (k >= kYOwn) mbar_wait(&oempty[s], (uint32_t)(((k / kYOwn) - 1) & 1));
+        const int yy = (k == g.ny) ? 0 : k;
+        const bool halo = !last_chunk || per;  // z+1 halo point: z0 + zc, or z = 0 (periodic wrap)
+        mbar_expect_tx(&ofull[s], (uint32_t)((zc + (halo ? 1 : 0)) * norb * 16));
+        tma_3d(own_slot(s), &mp.seg, 0, z0, rowx + yy, &ofull[s]);
+        if (halo) tma_3d(halo_of(s), &mp.one, 0, last_chunk ? 0 : z0 + zc, rowx + yy, &ofull[s]);
+      };
+      auto issue_xp = [&](int k) {
+        const int s = k % kYXp;
+        if (k >= kYXp) mbar_wait(&xempty[s], (uint32_t)(((k / kYXp) - 1) & 1));
+        mbar_expect_tx(&xfull[s], (uint32_t)(zc * norb * 16));
+        tma_3d(xp_slot(s), &mp.seg, 0, z0, rowxp + k, &xfull[s]);
+      };
+      issue_own(0);
+      if (nown > 1) issue_own(1);
+      for (int y = 0; y < g.ny; ++y) {
+        if (has_x) issue_xp(y);
+        if (y + 2 < nown) issue_own(y + 2);
+      }
+    }
+    return;
+  }
+
+  const int q = tid % kSub, pt = tid / kSub;
+  const bool valid = pt < zc;
+  const int z = z0 + pt;
+  const bool has_z = valid && (per || z + 1 < g.nz);
+  const DomCoef* cf = a.coef + dom;
+  const double2 ex = cf->eth[0], ey = cf->eth[1], ez = cf->eth[2];
+  const double ihx = cf->inv_h[0], ihy = cf->inv_h[1], ihz = cf->inv_h[2];
+  const int ptr = valid ? pt : 0;
+  double jsx = 0.0, jsy = 0.0, jsz = 0.0, ekin = 0.0, eloc = 0.0;
+  for (int y = 0; y < g.ny; ++y) {
+    const bool has_y = valid && (per || y + 1 < g.ny);
+    const int so = y % kYOwn, sn = (y + 1) % kYOwn, sx = y % kYXp;
+    mbar_wait(&ofull[so], (uint32_t)((y / kYOwn) & 1));
+    if (y + 1 < nown) mbar_wait(&ofull[sn], (uint32_t)(((y + 1) / kYOwn) & 1));
+    if (has_x) mbar_wait(&xfull[sx], (uint32_t)((y / kYXp) & 1));
+    const double2* O = own_slot(so) + ptr * norb;
+    const double2* Oz = (ptr + 1 < zc) ? O + norb : halo_of(so);  // point z+1
+    const double2* N = own_slot(sn) + ptr * norb;
+    const double2* X = xp_slot(sx) + ptr * norb;
+    double rho = 0.0, pxr = 0.0, pxi = 0.0, pyr = 0.0, pyi = 0.0, pzr = 0.0, pzi = 0.0;
+    if (valid) {
+#pragma unroll 4
+      for (int s = q; s < norb; s += kSub) {
+        const double fs = fsh[s];
+        const double2 v = O[s];
+        rho = fma(fs, fma(v.x, v.x, v.y * v.y), rho);
+        if (has_x) {
+          const double2 w = cconjmul(v, X[s]);
+          pxr = fma(fs, w.x, pxr);
+          pxi = fma(fs, w.y, pxi);
+        }
+        if (has_y) {
+          const double2 w = cconjmul(v, N[s]);
+          pyr = fma(fs, w.x, pyr);
+          pyi = fma(fs, w.y, pyi);
+        }
+        if (has_z) {
+          const double2 w = cconjmul(v, Oz[s]);
+          pzr = fma(fs, w.x, pzr);
+          pzi = fma(fs, w.y, pzi);
+        }
+      }
+    }
+    __syncwarp();
+    if ((tid & 31) == 0) {  // this warp is done with own line y and x+1 line y
+      mbar_arrive(&oempty[so]);
+      if (has_x) mbar_arrive(&xempty[sx]);
+    }
+#pragma unroll
+    for (int o = kSub / 2; o > 0; o >>= 1) {
+      rho += __shfl_xor_sync(0xffffffffu, rho, o);
+      pxr += __shfl_xor_sync(0xffffffffu, pxr, o);
+      pxi += __shfl_xor_sync(0xffffffffu, pxi, o);
+      pyr += __shfl_xor_sync(0xffffffffu, pyr, o);
+      pyi += __shfl_xor_sync(0xffffffffu, pyi, o);
+      pzr += __shfl_xor_sync(0xffffffffu, pzr, o);
+      pzi += __shfl_xor_sync(0xffffffffu, pzi, o);
+    }
+    const double jx = (valid && has_x) ? (ex.x * pxi + ex.y * pxr) * ihx : 0.0;
+    const double jy = has_y ? (ey.x * pyi + ey.y * pyr) * ihy : 0.0;
+    const double jz = has_z ? (ez.x * pzi + ez.y * pzr) * ihz : 0.0;
+    jsx += jx; jsy += jy; jsz += jz;
+    if (a.epart && valid) {  // kinetic / local energy densities (lfd_energy), FD Peierls form
+      const double w2x = ihx * ihx, w2y = ihy * ihy, w2z = ihz * ihz;
+      double ek = (w2x + w2y + w2z) * rho;
+      if (has_x) ek -= w2x * (ex.x * pxr - ex.y * pxi);  // Re(e^{i theta} P)
+      if (has_y) ek -= w2y * (ey.x * pyr - ey.y * pyi);
+      if (has_z) ek -= w2z * (ez.x * pzr - ez.y * pzi);
+      ekin += ek;
+      eloc += a.v[(long long)dom * g.ng + ((long long)x * g.ny + y) * g.nz + z] * rho;
+    }
+    if (q == 0 && valid) {
+      const long long o = (long long)x * a.sx + (long long)y * a.sy + z;
+      a.rho[a.base[dom] + o] = rho;
+      if (a.j) {
+        const long long oj = a.jbase[dom] + o;
+        a.j[oj] = jx;
+        a.j[oj + a.jstride] = jy;
+        a.j[oj + 2 * a.jstride] = jz;
+      }
+    }
+  }
+  const int pts = nconsw * 32 / kSub;
+  if (q == 0) {
+    jsh[0][pt] = jsx; jsh[1][pt] = jsy; jsh[2][pt] = jsz;
+    jsh[3][pt] = ekin; jsh[4][pt] = eloc;
+  }
+  asm volatile("bar.sync 1, %0;" ::"r"(nconsw * 32));  // consumer warps only
+  if (a.epart && tid >= 3 && tid < 5) {  // (warp 0: there may be a single consumer warp)
+    double t = 0.0;
+    for (int k = 0; k < pts; ++k) t += jsh[tid][k];
+    a.epart[((long long)dom * gridDim.x + blockIdx.x) * 2 + tid - 3] = t;
+  }
+  if (tid < 3) {
+    double t = 0.0;
+    for (int k = 0; k < pts; ++k) t += jsh[tid][k];
+    a.jline[((long long)dom * gridDim.x + blockIdx.x) * 3 + tid] = t;
+  }
+}
+
+static size_t ymarch_smem(const Geometry& g, int zc) { return YLayout(zc, g.norb).total; }
+
+DensMaps* density_maps_create(const Geometry& g, const double2* psi) {
+  const int zc = ymarch_zc(g);
+  if (zc == 0) return nullptr;
+  DensMaps* m = new (std::nothrow) DensMaps;
+  if (!m) return nullptr;
+  m->zc = zc;
+  const uint64_t dims[3] = {(uint64_t)2 * g.norb, (uint64_t)g.nz, (uint64_t)g.ndom * g.nx * g.ny};
+  const uint64_t str[2] = {(uint64_t)g.norb * 16, (uint64_t)g.nz * g.norb * 16};
+  const uint32_t b2[3] = {(uint32_t)(2 * g.norb), (uint32_t)zc, 1};
+  const uint32_t b3[3] = {(uint32_t)(2 * g.norb), 1, 1};
+  if (encode_tmap_f64(&m->seg, 3, psi, dims, str, b2) != cudaSuccess ||
+      encode_tmap_f64(&m->one, 3, psi, dims, str, b3) != cudaSuccess) {
+    delete m;
+    return nullptr;
+  }
+  return m;
+}
+
+void density_maps_destroy(DensMaps* m) { delete m; }
+
 int density_smem_bytes(int norb) { return kRingSlots * kPlanePts * norb * 16; }
 
 int density_blocks(const Geometry& g) {
+  const int zc = ymarch_zc(g);
+  if (zc > 0) return g.nx * (g.nz / zc);
   const int ntz = (g.nz + kTZ - 1) / kTZ, nty = (g.ny + kTY - 1) / kTY, nxc = (g.nx + kXC - 1) / kXC;
   return ntz * nty * nxc;
 }
 
-cudaError_t launch_density(const Geometry& g, const DensArgs& a, cudaStream_t st) {
-  const int ntz = (g.nz + kTZ - 1) / kTZ, nty = (g.ny + kTY - 1) / kTY;
+cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps* maps, cudaStream_t st) {
   dim3 grid(density_blocks(g), g.ndom);
+  if (maps) {
+    const int threads = ((maps->zc * kSub + 31) / 32 + 1) * 32;
+    k_density_y<<<grid, threads, ymarch_smem(g, maps->zc), st>>>(*maps, g, a);
+    return cudaGetLastError();
+  }
+  if (ymarch_zc(g) > 0) return cudaErrorInvalidValue;  // the block layout expects the y-marching kernel
+  const int ntz = (g.nz + kTZ - 1) / kTZ, nty = (g.ny + kTY - 1) / kTY;
   if (g.norb <= kMaxNorbTma)
     k_density_tma<<<grid, kDensThreads, density_smem_bytes(g.norb), st>>>(g, a, ntz, nty, kXC);
   else
@@ -314,8 +551,10 @@ cudaError_t launch_density(const Geometry& g, const DensArgs& a, cudaStream_t st
 }
 
 cudaError_t density_set_attributes() {
-  return cudaFuncSetAttribute(k_density_tma, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              density_smem_bytes(kMaxNorbTma));
+  cudaError_t e = cudaFuncSetAttribute(k_density_tma, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       density_smem_bytes(kMaxNorbTma));
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(k_density_y, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024);
 }
 
 // J_d = (1/Ngrid) sum_lines jline (one block per domain, fixed-order tree over a fixed partition).

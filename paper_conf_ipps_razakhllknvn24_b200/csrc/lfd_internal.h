@@ -139,7 +139,10 @@ struct DensArgs {
   const double* v;      // v_loc copy [dom][ng] when energy partials are wanted, else nullptr
   double* epart;        // [dom][density_blocks][2] per-CTA sums of (kinetic, local) energy densities
 };
-cudaError_t launch_density(const Geometry& g, const DensArgs& a, cudaStream_t st);
+struct DensMaps;  // TMA descriptors of Psi for the y-marching density kernel (dens.cu)
+DensMaps* density_maps_create(const Geometry& g, const double2* psi);  // nullptr: generic kernel
+void density_maps_destroy(DensMaps* m);
+cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps* maps, cudaStream_t st);
 int density_blocks(const Geometry& g);
 cudaError_t density_set_attributes();
 cudaError_t launch_jreduce(const Geometry& g, const double* jline, double* Jmac, cudaStream_t st);
