@@ -163,7 +163,7 @@ struct lfd_ctx {
   int device;
   int num_sms;
   uint64_t launches = 0;
-  int gemm2_variant = 2;  // internal tuning knob, env LFD_GEMM2_VARIANT (2 = TMA tensor-map variant)
+  int gemm2_variant = 3;  // internal tuning knob, env LFD_GEMM2_VARIANT (3 = TMA tensor maps + warp-half skew)
   // Projection carry: true while the workspace's DC / C' / s / n describe the GEMM-2 that produced the
   // current Psi, so the next nonlocal factor can take C from the exact identity C_new = (C + G X) n
   // instead of GEMM-1 (cleared by the local propagator, lfd_psi_modified and LFD_FLAG_NO_CARRY).

@@ -869,7 +869,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
 // copy when it changes), the K loop is fully unrolled for nproj = 64, the epilogue's Psi loads are
 // issued mid-loop and Psi <- n_s (Psi + B C') is written in place.
 // ------------------------------------------------------------------------------------------------
-template <int kNP>
+template <int kNP, bool kSkew>
 __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant__ CUtensorMap tB,
                                                              const __grid_constant__ CUtensorMap tC, Gemm2Args p) {
   extern __shared__ __align__(128) unsigned char smem[];
@@ -886,6 +886,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant
   const long long my_items = (items > blockIdx.x) ? (items - 1 - blockIdx.x) / gridDim.x + 1 : 0;
   constexpr int kNK4 = kNP > 0 ? (kNP + 3) / 4 : 16;
   const int nk4 = (np + 3) / 4;
+  const int kmid = (kNP > 0 ? kNK4 : nk4) / 2;  // k step at which the epilogue's Psi loads are issued
 
   if (tid == 0) {
     for (int s = 0; s < kFullStages; ++s) {
@@ -940,6 +941,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant
       cur_dom = dom;
       cur_n0 = n0;
     }
+    // skew: the second M-half of the warps starts half a K loop late, so each half's epilogue overlaps
+    // the other half's DMMAs (the halves share only the B stage and C')
+    if (kSkew && j == 0 && wm == 1) asm volatile("bar.sync 2, %0;" ::"n"(kThreads));
     const int s = (int)(j % kFullStages);
     mbar_wait(&full[s], (uint32_t)((j / kFullStages) & 1));
     const double2* As = reinterpret_cast<const double2*>(smem + s * kFullABytes);
@@ -963,7 +967,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant
 #pragma unroll
     for (int kk = 0; kk < kNK4; ++kk) {
       if (kNP == 0 && kk >= nk4) break;
-      if (kk == kNK4 / 2) load_pv();  // Psi loads (L2 hits) in flight during the second half
+      if (kk == kmid) {
+        load_pv();  // Psi loads (L2 hits) in flight during the second half
+        if (kSkew && j == 0 && wm == 0) asm volatile("bar.arrive 2, %0;" ::"n"(kThreads));
+      }
       const int k = kk * 4 + t;
       double2 a[4], c[2];
 #pragma unroll
@@ -972,7 +979,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant
       for (int ni = 0; ni < 2; ++ni) c[ni] = Cs[k * kLd1 + wn * 16 + ni * 8 + g];
       mma_4x2(acc, a, c);
     }
-    if (kNP == 0 && nk4 <= kNK4 / 2) load_pv();
     __syncwarp();
     if (lane == 0) mbar_arrive(&empty[s]);
     if (tid == 0 && j + kFullStages < my_items) {  // refill the stage once every warp has released it
@@ -1022,9 +1028,17 @@ cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
     cudaError_t e = gemm2_maps(a, &tB, &tC);
     if (e != cudaSuccess) return e;
     if (a.nproj == kTile)
-      k_gemm2_tma<kTile><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+      k_gemm2_tma<kTile, false><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
     else
-      k_gemm2_tma<0><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+      k_gemm2_tma<0, false><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+  } else if (a.nproj <= kTile && a.variant == 3) {
+    CUtensorMap tB, tC;
+    cudaError_t e = gemm2_maps(a, &tB, &tC);
+    if (e != cudaSuccess) return e;
+    if (a.nproj == kTile)
+      k_gemm2_tma<kTile, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+    else
+      k_gemm2_tma<0, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
   } else if (a.nproj == kTile && a.variant == 1)
     k_gemm2_fullk<kTile, true><<<grid, kThreads, kFullSmem, st>>>(a);
   else if (a.nproj == kTile)
@@ -1045,10 +1059,10 @@ cudaError_t gemm_set_attributes() {
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_gemm2_fullk<0, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_gemm2_tma<kTile>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem + 16);
-  if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_gemm2_tma<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem + 16);
-  if (e != cudaSuccess) return e;
+  for (auto f : {k_gemm2_tma<kTile, false>, k_gemm2_tma<0, false>, k_gemm2_tma<kTile, true>, k_gemm2_tma<0, true>}) {
+    e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem + 16);
+    if (e != cudaSuccess) return e;
+  }
   return cudaFuncSetAttribute(k_gemm2, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm2_smem_bytes());
 }
 
