@@ -294,17 +294,13 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false) {
     double* s = c->at<double>(c->L.s);
     double* nfac = c->at<double>(c->L.nfac);
     LFD_TRY(launch(c, LFD_K_NL_CARRY, "k_nlcarry", [&] {
-      return lfd::launch_nlcarry(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), D, DC, X, nfac,
-                                 c->stream);
+      return lfd::launch_nlcarry(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), D, DC, X, s, nfac,
+                                 !merged, c->stream);
     }));
     if (merged)
       LFD_TRY(launch(c, LFD_K_NL_NORM, "k_nlmerge", [&] {
         return lfd::launch_nlmerge(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), D, DC, s, X, nfac,
                                    c->stream);
-      }));
-    else
-      LFD_TRY(launch(c, LFD_K_NL_NORM, "k_nlnorm", [&] {
-        return lfd::launch_nlnorm(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), DC, s, nfac, c->stream);
       }));
     return gemm2(c);
   }

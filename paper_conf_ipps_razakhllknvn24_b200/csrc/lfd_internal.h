@@ -106,8 +106,9 @@ cudaError_t launch_nlmerge(int ndom, int nproj, int norb, double eps, const doub
 
 // Projection carry after a GEMM-2 Psi <- (Psi + B X) diag(n): DC <- (DC + D (G X)) diag(n) and
 // X <- -i eps DC (the C' of the next nonlocal factor), in place; column norms s are unchanged.
+// with_norm: also the next factor's n_s (as launch_nlnorm) in the same kernel (nfac is overwritten).
 cudaError_t launch_nlcarry(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
-                           double2* DC, double2* X, const double* nfac, cudaStream_t st);
+                           double2* DC, double2* X, const double* s, double* nfac, bool with_norm, cudaStream_t st);
 
 // GEMM-2 in place: psi[dom][r][n] <- nfac[dom][n] * (psi[dom][r][n] + sum_m B[dom][r][m] Cp[dom][m][n])
 struct Gemm2Args {

@@ -522,12 +522,14 @@ cudaError_t launch_nlmerge(int ndom, int nproj, int norb, double eps, const doub
 // written (X and DC are read into shared memory before any write). Replaces GEMM-1 + k_reduce of the
 // next nonlocal factor when nothing touched Psi in between (lfd_step: N of step n, then N of n+1).
 // ------------------------------------------------------------------------------------------------
+template <bool kNorm>
 __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps, const double2* __restrict__ G,
                                                  const double* __restrict__ D, double2* DC, double2* X,
-                                                 const double* __restrict__ nfac) {
-  extern __shared__ double2 sh[];  // x[np] | dc[np]
+                                                 const double* __restrict__ s, double* nfac) {
+  extern __shared__ double2 sh[];  // x[np] | dc[np] (dc is overwritten with DC_new)
   double2* xs = sh;
   double2* dcs = sh + nproj;
+  __shared__ double wq[8];
   const int dom = blockIdx.y, col = blockIdx.x;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const double2* Gd = G + (long long)dom * nproj * nproj;
@@ -539,11 +541,13 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
   }
   __syncthreads();
   const double n = nfac[(long long)dom * norb + col];
-  for (int u = warp; u < nproj; u += 8) {
+  // (G v)_u, warp-wide (lanes over the row of G), fixed-order shuffle tree
+  auto gdot = [&](int u, const double2* v, double& tr, double& ti) {
     const double2* Gu = Gd + (long long)u * nproj;
-    double tr = 0.0, ti = 0.0;
-    for (int v = lane; v < nproj; v += 32) {
-      const double2 gv = Gu[v], x = xs[v];
+    tr = 0.0;
+    ti = 0.0;
+    for (int w = lane; w < nproj; w += 32) {
+      const double2 gv = Gu[w], x = v[w];
       tr = fma(gv.x, x.x, fma(-gv.y, x.y, tr));
       ti = fma(gv.x, x.y, fma(gv.y, x.x, ti));
     }
@@ -552,19 +556,45 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
       tr += __shfl_xor_sync(0xffffffffu, tr, o);
       ti += __shfl_xor_sync(0xffffffffu, ti, o);
     }
+  };
+  for (int u = warp; u < nproj; u += 8) {
+    double tr, ti;
+    gdot(u, xs, tr, ti);
     if (lane == 0) {
       const double du = Dd[u];
       const double2 d = make_double2(n * fma(du, tr, dcs[u].x), n * fma(du, ti, dcs[u].y));
       DC[cb + (long long)u * norb] = d;
       X[cb + (long long)u * norb] = make_double2(eps * d.y, -eps * d.x);  // -i eps DC_new
+      dcs[u] = d;  // only this lane reads dcs[u] above
     }
+  }
+  if (!kNorm) return;
+  // n_s of the next factor from the Gram closed form (as k_nlnorm), on DC_new
+  __syncthreads();
+  double q = 0.0;
+  for (int u = warp; u < nproj; u += 8) {
+    double tr, ti;
+    gdot(u, dcs, tr, ti);
+    const double2 cu = dcs[u];
+    q = fma(cu.x, tr, fma(cu.y, ti, q));  // Re(conj(cu) (G DC)_u)
+  }
+  if (lane == 0) wq[warp] = q;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double tq = 0.0;
+    for (int w = 0; w < 8; ++w) tq += wq[w];
+    const double sv = s[(long long)dom * norb + col];
+    nfac[(long long)dom * norb + col] = sqrt(sv / (sv + eps * eps * tq));
   }
 }
 
 cudaError_t launch_nlcarry(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
-                           double2* DC, double2* X, const double* nfac, cudaStream_t st) {
+                           double2* DC, double2* X, const double* s, double* nfac, bool with_norm, cudaStream_t st) {
   dim3 grid(norb, ndom);
-  k_nlcarry<<<grid, 256, 2 * nproj * sizeof(double2), st>>>(nproj, norb, eps, G, D, DC, X, nfac);
+  if (with_norm)
+    k_nlcarry<true><<<grid, 256, 2 * nproj * sizeof(double2), st>>>(nproj, norb, eps, G, D, DC, X, s, nfac);
+  else
+    k_nlcarry<false><<<grid, 256, 2 * nproj * sizeof(double2), st>>>(nproj, norb, eps, G, D, DC, X, s, nfac);
   return cudaGetLastError();
 }
 

@@ -256,10 +256,10 @@ def test_launch_count_and_profile():
     ctx.step(2)
     prof = lfd.lfd_profile_read(ctx.ctx)
     # step 1: N (GEMM-1, reduce, norm, GEMM-2), the stencil passes (Phi.K_x, then Phi.K_y K_z fused), N;
-    # step 2's first N takes C from the projection carry (carry, norm, GEMM-2) instead of GEMM-1 + reduce
+    # step 2's first N takes C and n from the projection carry (one kernel) instead of GEMM-1 + reduce + norm
     assert prof["kin_x"][1] == 2 and prof["kin_yz"][1] == 2 and prof["kin_y"][1] == 0
-    assert lfd.lfd_launch_count(ctx.ctx) - n0 == sum(v[1] for v in prof.values()) == 10 + 9
-    assert prof["nl_proj"][1] == 3 and prof["nl_back"][1] == 4
+    assert lfd.lfd_launch_count(ctx.ctx) - n0 == sum(v[1] for v in prof.values()) == 10 + 8
+    assert prof["nl_proj"][1] == 3 and prof["nl_back"][1] == 4 and prof["nl_norm"][1] == 3
     assert prof["nl_carry"][1] == 1
     assert all(v[0] >= 0 for v in prof.values())
     ctx.close()
