@@ -185,6 +185,27 @@ struct LineMarch {
     }
     prev_e1 = e1;
   }
+  // The three phases of push() without the p tests (p == 0, p == 1, p >= 2 with a full pair).
+  __device__ __forceinline__ void first(const PairCoef& c, double2 a, double2 b) {
+    E10 = lk_L<kS>(c.a1, c.u1, a, b);
+    prev_e1 = lk_R<kS>(c.a1, c.d1, a, b);
+  }
+  __device__ __forceinline__ void second(const PairCoef& c, double2 a, double2 b) {
+    const double2 e0 = lk_L<kS>(c.a1, c.u1, a, b);
+    O1 = lk_L<kS>(c.a2, c.u2, prev_e1, e0);
+    prev_oR = lk_R<kS>(c.a2, c.d2, prev_e1, e0);
+    prev_e1 = lk_R<kS>(c.a1, c.d1, a, b);
+  }
+  template <class St>
+  __device__ __forceinline__ void steady(const PairCoef& c, double2 a, double2 b, St&& st) {
+    const double2 e0 = lk_L<kS>(c.a1, c.u1, a, b);
+    const double2 oL = lk_L<kS>(c.a2, c.u2, prev_e1, e0);
+    const double2 oR = lk_R<kS>(c.a2, c.d2, prev_e1, e0);
+    st(0, lk_L<kS>(c.a1, c.u1, prev_oR, oL));
+    st(1, lk_R<kS>(c.a1, c.d1, prev_oR, oL));
+    prev_oR = oR;
+    prev_e1 = lk_R<kS>(c.a1, c.d1, a, b);
+  }
   template <bool kPer, class St>
   __device__ __forceinline__ void finish(const PairCoef& c, int n, St&& st) {
     if ((n & 1) == 0) {
@@ -278,17 +299,24 @@ __global__ void __launch_bounds__(256, 3) k_kin(double2* __restrict__ psi, const
 // ------------------------------------------------------------------------------------------------
 constexpr int kYZW = 8;
 constexpr int kYZMaxThreads = 352;  // up to 40 z pairs x 8 orbitals + the producer warp
-constexpr int kYZS = 8;             // ring depth (planes)
+constexpr int kYZS = 10;            // ring depth (planes); even, so a y pair never straddles the wrap
+
+// bytes of one ring slot: the Psi segment [nz][8 orbitals] + the Phi row [nz], 128-byte aligned
+__host__ __device__ __forceinline__ int yz_slot_bytes(int nz) { return (nz * kYZW * 16 + nz * 16 + 127) & ~127; }
 
 template <bool kPer, bool kS>
 __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant__ CUtensorMap tmap,
                                                           double2* __restrict__ psi, const DomCoef* __restrict__ coef,
                                                           const double2* __restrict__ phi, int nx, int ny, int nz,
                                                           int norb, int nchunks, long long ng) {
+  // periodic => nz even (validated), so every thread owns a full pair and every link exists
+  constexpr bool kFull = kPer;
   extern __shared__ __align__(128) unsigned char smem[];
-  const int seg = nz * kYZW;  // complex elements per plane segment
-  double2* ring = reinterpret_cast<double2*>(smem);
-  uint64_t* full = reinterpret_cast<uint64_t*>(ring + kYZS * seg);
+  const int seg = nz * kYZW;                               // complex elements of the Psi segment
+  const int slot_b = yz_slot_bytes(nz);                    // Psi segment + Phi row, 128-byte aligned
+  auto slot_psi = [&](int s) { return reinterpret_cast<const double2*>(smem + s * slot_b); };
+  auto slot_phi = [&](int s) { return reinterpret_cast<const double2*>(smem + s * slot_b + seg * 16); };
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kYZS * slot_b);
   uint64_t* empty = full + kYZS;
   const int dom = blockIdx.y;
   const int x = blockIdx.x / nchunks, oc = blockIdx.x - (blockIdx.x / nchunks) * nchunks;
@@ -310,16 +338,18 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
+  const double2* phx = phi + (long long)dom * ng + (long long)x * ny * nz;  // Phi(x, y = 0, z = 0)
 
-  if (tid >= nconsw * 32) {  // producer warp: plane y -> slot y % kYZS, one tensor copy per plane
+  if (tid >= nconsw * 32) {  // producer warp: plane y -> slot y % kYZS (Psi: one tensor copy; Phi: one row)
     if (tid == nconsw * 32) {
       const int row0 = (dom * nx + x) * ny;
       int s = 0;
       uint32_t ph = 0;
       for (int y = 0; y < ny; ++y) {
         if (y >= kYZS) mbar_wait(&empty[s], ph ^ 1);
-        mbar_expect_tx(&full[s], (uint32_t)(seg * 16));
-        tma_3d(ring + s * seg, &tmap, 2 * o0, 0, row0 + y, &full[s]);
+        mbar_expect_tx(&full[s], (uint32_t)(seg * 16 + nz * 16));
+        tma_3d(smem + s * slot_b, &tmap, 2 * o0, 0, row0 + y, &full[s]);
+        tma_row(smem + s * slot_b + seg * 16, phx + (long long)y * nz, (uint32_t)(nz * 16), &full[s]);
         if (++s == kYZS) { s = 0; ph ^= 1; }
       }
     }
@@ -329,34 +359,28 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
   const int o = tid % kYZW, m = tid / kYZW;
   const bool live = m < npz;
   const int z0 = 2 * m, z1 = 2 * m + 1;
-  const bool has1 = live && z1 < nz;
+  const bool has1 = kFull ? live : (live && z1 < nz);
   const bool act = live && o < wv;
   // ring offsets (complex elements within a slot) of the six points this thread's K_z reads
   const int zl = (m > 0) ? z0 - 2 : nz - 2;                    // pair m-1 (periodic wrap for m == 0)
   const int zr = (z1 + 1 < nz) ? z1 + 1 : 0;                   // pair m+1 (periodic wrap at the end)
-  const bool has_l = live && (m > 0 || kPer);                  // link (2m-1, 2m) exists
-  const bool has_r = has1 && (z1 + 1 < nz || kPer);            // link (2m+1, 2m+2) exists
-  const bool r_single = zr + 1 >= nz;                          // pair m+1 is a zero-BC singleton
+  const bool has_l = kFull ? live : (live && m > 0);           // link (2m-1, 2m) exists
+  const bool has_r = kFull ? live : (has1 && z1 + 1 < nz);     // link (2m+1, 2m+2) exists
+  const bool r_single = kFull ? false : (zr + 1 >= nz);        // pair m+1 is a zero-BC singleton
   const int oz0 = live ? z0 * kYZW + o : o, oz1 = has1 ? z1 * kYZW + o : o;
   const int ozl = has_l ? zl * kYZW + o : o, ozl1 = has_l ? (zl + 1) * kYZW + o : o;
   const int ozr = has_r ? zr * kYZW + o : o, ozr1 = (has_r && !r_single) ? (zr + 1) * kYZW + o : o;
+  const int pz0 = live ? z0 : 0, pz1 = has1 ? z1 : 0;          // Phi offsets in the slot's Phi row
   const int yst = nz * norb;  // element stride between y planes (< 2^31 per domain, validated)
   double2* out0 = psi + (long long)dom * ng * norb + (long long)x * ny * yst + o0 + z0 * norb + o;
   double2* out1 = out0 + norb;
-  const double2* ph0 = phi + (long long)dom * ng + (long long)x * ny * nz + z0;  // Phi(x, y=0, z0)
 
-  int slot = 0;
-  uint32_t phase = 0;
-  // K_z of the next plane (in y order) for this thread's pair: the first E(Delta/2) on pairs m-1, m,
-  // m+1 (the neighbours' outputs recomputed here), O(Delta) on the links (2m-1, 2m), (2m+1, 2m+2), then
-  // the second E(Delta/2) on (2m, 2m+1). The slot is released to the producer afterwards.
-  auto kz = [&](double2& w0, double2& w1) {
-    mbar_wait(&full[slot], phase);
-    const double2* r = ring + slot * seg;
+  // K_z of plane y (slot s) for this thread's pair: the first E(Delta/2) on pairs m-1, m, m+1 (the
+  // neighbours' outputs recomputed here), O(Delta) on the links (2m-1, 2m), (2m+1, 2m+2), then the
+  // second E(Delta/2) on (2m, 2m+1).
+  auto kz = [&](int s, double2& w0, double2& w1) {
+    const double2* r = slot_psi(s);
     const double2 a = r[oz0], b = r[oz1], vl = r[ozl], vl1 = r[ozl1], vr = r[ozr], vr1 = r[ozr1];
-    __syncwarp();
-    if ((tid & 31) == 0) mbar_arrive(&empty[slot]);
-    if (++slot == kYZS) { slot = 0; phase ^= 1; }
     double2 e0, e1 = cz();
     if (has1) {
       e0 = lk_L<kS>(cz_.a1, cz_.u1, a, b);
@@ -380,7 +404,10 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
       w1 = cz();
     }
   };
-  auto ph = [&](int y, int dz) { return live ? __ldg(ph0 + y * nz + dz) : cz(); };
+  auto release = [&](int s) {
+    __syncwarp();
+    if ((tid & 31) == 0) mbar_arrive(&empty[s]);
+  };
   auto put0 = [&](int y, double2 f, double2 v) {
     if (act) out0[y * yst] = cmul(f, v);
   };
@@ -392,22 +419,96 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
   L0.init();
   L1.init();
   const int npairs = (ny + 1) >> 1;
-  for (int p = 0; p < npairs; ++p) {
-    const int ya = 2 * p;
-    const bool hb = ya + 1 < ny;
-    // Phi of the two planes this iteration's march step stores (2p-2, 2p-1): loads in flight meanwhile
-    double2 fa0 = cz(), fa1 = cz(), fb0 = cz(), fb1 = cz();
-    if (p >= 2) {
-      fa0 = ph(ya - 2, 0); fa1 = ph(ya - 2, 1);
-      fb0 = ph(ya - 1, 0); fb1 = ph(ya - 1, 1);
+  if (kFull && ny >= 4) {
+    // periodic (even ny): pairs 0 and 1 peeled, then a steady loop without p / parity tests
+    double2 wa0, wa1, wb0, wb1;
+    mbar_wait(&full[0], 0);
+    kz(0, wa0, wa1);
+    mbar_wait(&full[1], 0);
+    kz(1, wb0, wb1);
+    release(0);
+    release(1);
+    L0.first(cy, wa0, wb0);
+    L1.first(cy, wa1, wb1);
+    mbar_wait(&full[2], 0);
+    kz(2, wa0, wa1);
+    mbar_wait(&full[3], 0);
+    kz(3, wb0, wb1);
+    L0.second(cy, wa0, wb0);
+    L1.second(cy, wa1, wb1);
+    int s_prev = 2, s_a = 4;  // slot of plane 2p-2 and of plane 2p (kYZS is even: pairs never straddle)
+    uint32_t ph_a = 0;
+    double2* o0p = out0 + 2 * yst;  // plane 2p-2
+    for (int p = 2; p < npairs; ++p) {
+      mbar_wait(&full[s_a], ph_a);
+      kz(s_a, wa0, wa1);
+      mbar_wait(&full[s_a + 1], ph_a);
+      kz(s_a + 1, wb0, wb1);
+      const double2* pa = slot_phi(s_prev);
+      const double2* pb = slot_phi(s_prev + 1);
+      const double2 fa0 = pa[pz0], fa1 = pa[pz1], fb0 = pb[pz0], fb1 = pb[pz1];
+      L0.steady(cy, wa0, wb0, [&](int k, double2 v) {
+        if (act) o0p[k * yst] = cmul(k == 0 ? fa0 : fb0, v);
+      });
+      L1.steady(cy, wa1, wb1, [&](int k, double2 v) {
+        if (act) o0p[k * yst + norb] = cmul(k == 0 ? fa1 : fb1, v);
+      });
+      release(s_prev);
+      release(s_prev + 1);
+      o0p += 2 * yst;
+      s_prev = s_a;
+      s_a += 2;
+      if (s_a == kYZS) { s_a = 0; ph_a ^= 1; }
     }
-    double2 wa0, wa1, wb0 = cz(), wb1 = cz();
-    kz(wa0, wa1);
-    if (hb) kz(wb0, wb1);
-    L0.push(cy, p, wa0, wb0, hb, [&](int y, double2 v) { put0(y, y == ya - 2 ? fa0 : fb0, v); });
-    L1.push(cy, p, wa1, wb1, hb, [&](int y, double2 v) { put1(y, y == ya - 2 ? fa1 : fb1, v); });
+  } else {
+    // ring bookkeeping: plane y sits in slot y % kYZS (phase (y / kYZS) & 1). Planes >= 2 are released
+    // after their store (their Phi row is read then); planes 0 and 1 (stored last, by the wrap) right
+    // after K_z -- their Phi comes from global memory at the end.
+    int s_a = 0;
+    uint32_t ph_a = 0;
+    int s_prev = 0;  // slot of plane 2p-2
+    for (int p = 0; p < npairs; ++p) {
+      const int ya = 2 * p;
+      const bool hb = ya + 1 < ny;
+      int s_b = s_a + 1;
+      uint32_t ph_b = ph_a;
+      if (s_b == kYZS) { s_b = 0; ph_b ^= 1; }
+      double2 wa0, wa1, wb0 = cz(), wb1 = cz();
+      mbar_wait(&full[s_a], ph_a);
+      kz(s_a, wa0, wa1);
+      if (hb) {
+        mbar_wait(&full[s_b], ph_b);
+        kz(s_b, wb0, wb1);
+      }
+      if (p == 0) {
+        release(s_a);
+        if (hb) release(s_b);
+      }
+      // Phi of the planes this march step stores (2p-2 in slot s_prev, 2p-1 in the next slot)
+      int s_pb = s_prev + 1;
+      if (s_pb == kYZS) s_pb = 0;
+      double2 fa0 = cz(), fa1 = cz(), fb0 = cz(), fb1 = cz();
+      if (p >= 2) {
+        const double2* pa = slot_phi(s_prev);
+        const double2* pb = slot_phi(s_pb);
+        fa0 = pa[pz0]; fa1 = pa[pz1];
+        fb0 = pb[pz0]; fb1 = pb[pz1];
+      }
+      L0.push(cy, p, wa0, wb0, hb, [&](int y, double2 v) { put0(y, y == ya - 2 ? fa0 : fb0, v); });
+      L1.push(cy, p, wa1, wb1, hb, [&](int y, double2 v) { put1(y, y == ya - 2 ? fa1 : fb1, v); });
+      if (p >= 2) {
+        release(s_prev);
+        release(s_pb);
+      }
+      s_prev = s_a;
+      s_a = s_b + 1;
+      ph_a = ph_b;
+      if (s_a == kYZS) { s_a = 0; ph_a ^= 1; }
+    }
   }
-  // wrap: planes ny-2, ny-1 (or ny-1 for odd ny) and 0, 1
+  // wrap: planes ny-2, ny-1 (or ny-1 for odd ny; their slots are released at the end) and 0, 1
+  const double2* phb = phx + pz0;
+  auto ph = [&](int y, int dz) { return live ? __ldg(phb + y * nz + dz) : cz(); };
   const double2 f00 = ph(0, 0), f01 = ph(0, 1), f10 = ph(1, 0), f11 = ph(1, 1);
   const double2 fl0 = ph(ny - 1, 0), fl1 = ph(ny - 1, 1);
   const double2 fm0 = ph(ny - 2, 0), fm1 = ph(ny - 2, 1);
@@ -419,7 +520,7 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
 
 bool kin_yz_supported(const Geometry& g) { return g.nz <= 80; }
 
-static size_t yz_smem(int nz) { return (size_t)kYZS * nz * kYZW * 16 + (size_t)kYZS * 16; }
+static size_t yz_smem(int nz) { return (size_t)kYZS * yz_slot_bytes(nz) + (size_t)kYZS * 16; }
 
 // Tensor map of Psi for k_kin_yz: 3-D view [ndom*nx*ny planes][nz rows][2*norb doubles], box
 // [1][nz][16 doubles] (one (x, y) plane segment of 8 orbitals), no swizzle (dense rows of 128 B).
