@@ -267,6 +267,20 @@ __global__ void __launch_bounds__(256, 3) k_kin(double2* __restrict__ psi, const
   const int P = (n + 1) >> 1;
   LineMarch<kS> L;
   L.init();
+  if (kPeriodic && n >= 6) {  // periodic (even n): first two pairs peeled, then a test-free steady loop
+    double2 a0 = ld(0), b0 = ld(1), a1 = ld(2), b1 = ld(3), a2 = ld(4), b2 = ld(5);
+    L.first(cf, a0, b0);
+    a0 = a1; b0 = b1; a1 = a2; b1 = b2;
+    if (3 < P) { a2 = ld(6); b2 = ld(7); }
+    L.second(cf, a0, b0);
+    for (int p = 2; p < P; ++p) {
+      a0 = a1; b0 = b1; a1 = a2; b1 = b2;
+      if (p + 2 < P) { a2 = ld(2 * p + 4); b2 = ld(2 * p + 5); }
+      L.steady(cf, a0, b0, [&](int k, double2 v) { st(2 * p - 2 + k, v); });
+    }
+    L.template finish<kPeriodic>(cf, n, st);
+    return;
+  }
   double2 na = ld(0), nb = (n > 1) ? ld(1) : cz();
   double2 nc = cz(), nd = cz();
   if (P > 1) {
