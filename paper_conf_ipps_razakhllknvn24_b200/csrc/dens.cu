@@ -310,7 +310,7 @@ __global__ void __launch_bounds__(kDensThreads) k_density_tma(Geometry g, DensAr
 // reductions with the occupation weights (kept in shared memory).
 // ------------------------------------------------------------------------------------------------
 constexpr int kYOwn = 3, kYXp = 2;
-constexpr int kYMaxThreads = 544;  // up to 64 points x kSub + the producer warp
+constexpr int kYMaxThreads = 352;  // up to 40 points x kSub + the producer warp
 
 struct DensMaps {
   CUtensorMap seg;   // box [1][zc][2*norb]: a z-line segment of zc points, all orbitals
@@ -338,13 +338,14 @@ static int ymarch_zc(const Geometry& g) {
   for (int nzc = 1; nzc <= g.nz; ++nzc) {
     if (g.nz % nzc) continue;
     const int zc = g.nz / nzc;
-    if (zc > 64) continue;
+    if (zc > 40) continue;
     (void)per_pt;
     if (YLayout(zc, g.norb).total <= 200 * 1024) return zc;
   }
   return 0;
 }
 
+template <bool kPer, int kIt>
 __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constant__ DensMaps mp, Geometry g,
                                                             DensArgs a) {
   extern __shared__ __align__(128) unsigned char dsm[];
@@ -360,7 +361,7 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
   const int dom = blockIdx.y;
   const int nzc = g.nz / zc;
   const int x = blockIdx.x / nzc, z0 = (blockIdx.x - x * nzc) * zc;
-  const bool per = (g.bc == 0);
+  const bool per = kPer;
   const bool has_x = per || x + 1 < g.nx;
   const int xp = (x + 1 == g.nx) ? 0 : x + 1;
   const bool last_chunk = z0 + zc == g.nz;
@@ -406,14 +407,23 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
   const int q = tid % kSub, pt = tid / kSub;
   const bool valid = pt < zc;
   const int z = z0 + pt;
-  const bool has_z = valid && (per || z + 1 < g.nz);
+  const bool has_z = valid && (kPer || z + 1 < g.nz);
   const DomCoef* cf = a.coef + dom;
   const double2 ex = cf->eth[0], ey = cf->eth[1], ez = cf->eth[2];
   const double ihx = cf->inv_h[0], ihy = cf->inv_h[1], ihz = cf->inv_h[2];
+  const double w2x = ihx * ihx, w2y = ihy * ihy, w2z = ihz * ihz;
   const int ptr = valid ? pt : 0;
-  double jsx = 0.0, jsy = 0.0, jsz = 0.0, ekin = 0.0, eloc = 0.0;
+  // occupations of this lane's orbitals s = q, q + kSub, ... in registers
+  constexpr int kItMax = 128 / kSub;
+  const int nit = (norb - q + kSub - 1) / kSub;
+  double fr[kIt > 0 ? kIt : kItMax];
+#pragma unroll
+  for (int i = 0; i < (kIt > 0 ? kIt : kItMax); ++i) fr[i] = (i < nit) ? fsh[q + i * kSub] : 0.0;
+  // lane q of a point ends up holding the full sum of value q >> 1: 0 rho, 1 jx, 2 jy, 3 jz
+  const int vsel = q >> 1;
+  double jacc = 0.0, ekin = 0.0, eloc = 0.0;
   for (int y = 0; y < g.ny; ++y) {
-    const bool has_y = valid && (per || y + 1 < g.ny);
+    const bool has_y = valid && (kPer || y + 1 < g.ny);
     const int so = y % kYOwn, sn = (y + 1) % kYOwn, sx = y % kYXp;
     mbar_wait(&ofull[so], (uint32_t)((y / kYOwn) & 1));
     if (y + 1 < nown) mbar_wait(&ofull[sn], (uint32_t)(((y + 1) / kYOwn) & 1));
@@ -422,27 +432,31 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
     const double2* Oz = (ptr + 1 < zc) ? O + norb : halo_of(so);  // point z+1
     const double2* N = own_slot(sn) + ptr * norb;
     const double2* X = xp_slot(sx) + ptr * norb;
+    // per-lane partial sums over this lane's orbitals: rho and the three link products P_d = sum f
+    // conj(psi_r) psi_{r+e_d} (f folded into fv = f psi_r)
     double rho = 0.0, pxr = 0.0, pxi = 0.0, pyr = 0.0, pyi = 0.0, pzr = 0.0, pzi = 0.0;
     if (valid) {
-#pragma unroll 4
-      for (int s = q; s < norb; s += kSub) {
-        const double fs = fsh[s];
-        const double2 v = O[s];
-        rho = fma(fs, fma(v.x, v.x, v.y * v.y), rho);
-        if (has_x) {
-          const double2 w = cconjmul(v, X[s]);
-          pxr = fma(fs, w.x, pxr);
-          pxi = fma(fs, w.y, pxi);
+#pragma unroll
+      for (int i = 0; i < (kIt > 0 ? kIt : kItMax); ++i) {
+        if (kIt == 0 && i >= nit) break;
+        const int sidx = q + i * kSub;
+        const double2 v = O[sidx];
+        const double2 fv = make_double2(fr[i] * v.x, fr[i] * v.y);
+        rho = fma(fv.x, v.x, fma(fv.y, v.y, rho));
+        if (kPer || has_x) {
+          const double2 w = X[sidx];
+          pxr = fma(fv.x, w.x, fma(fv.y, w.y, pxr));
+          pxi = fma(fv.x, w.y, fma(-fv.y, w.x, pxi));
         }
-        if (has_y) {
-          const double2 w = cconjmul(v, N[s]);
-          pyr = fma(fs, w.x, pyr);
-          pyi = fma(fs, w.y, pyi);
+        if (kPer || has_y) {
+          const double2 w = N[sidx];
+          pyr = fma(fv.x, w.x, fma(fv.y, w.y, pyr));
+          pyi = fma(fv.x, w.y, fma(-fv.y, w.x, pyi));
         }
-        if (has_z) {
-          const double2 w = cconjmul(v, Oz[s]);
-          pzr = fma(fs, w.x, pzr);
-          pzi = fma(fs, w.y, pzi);
+        if (kPer || has_z) {
+          const double2 w = Oz[sidx];
+          pzr = fma(fv.x, w.x, fma(fv.y, w.y, pzr));
+          pzi = fma(fv.x, w.y, fma(-fv.y, w.x, pzi));
         }
       }
     }
@@ -451,44 +465,56 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
       mbar_arrive(&oempty[so]);
       if (has_x) mbar_arrive(&xempty[sx]);
     }
-#pragma unroll
-    for (int o = kSub / 2; o > 0; o >>= 1) {
-      rho += __shfl_xor_sync(0xffffffffu, rho, o);
-      pxr += __shfl_xor_sync(0xffffffffu, pxr, o);
-      pxi += __shfl_xor_sync(0xffffffffu, pxi, o);
-      pyr += __shfl_xor_sync(0xffffffffu, pyr, o);
-      pyi += __shfl_xor_sync(0xffffffffu, pyi, o);
-      pzr += __shfl_xor_sync(0xffffffffu, pzr, o);
-      pzi += __shfl_xor_sync(0xffffffffu, pzi, o);
-    }
-    const double jx = (valid && has_x) ? (ex.x * pxi + ex.y * pxr) * ihx : 0.0;
-    const double jy = has_y ? (ey.x * pyi + ey.y * pyr) * ihy : 0.0;
-    const double jz = has_z ? (ez.x * pzi + ez.y * pzr) * ihz : 0.0;
-    jsx += jx; jsy += jy; jsz += jz;
-    if (a.epart && valid) {  // kinetic / local energy densities (lfd_energy), FD Peierls form
-      const double w2x = ihx * ihx, w2y = ihy * ihy, w2z = ihz * ihz;
+    // the currents and the kinetic energy density are linear in the P_d: form them per lane first
+    // (Im(e^{i theta} P) = cos Im P + sin Re P, Re(e^{i theta} P) = cos Re P - sin Im P)
+    const double jx = (kPer || has_x) ? (ex.x * pxi + ex.y * pxr) * ihx : 0.0;
+    const double jy = (kPer || has_y) ? (ey.x * pyi + ey.y * pyr) * ihy : 0.0;
+    const double jz = (kPer || has_z) ? (ez.x * pzi + ez.y * pzr) * ihz : 0.0;
+    if (a.epart) {  // kinetic energy density (FD Peierls form) summed per lane; reduced per CTA at the end
       double ek = (w2x + w2y + w2z) * rho;
-      if (has_x) ek -= w2x * (ex.x * pxr - ex.y * pxi);  // Re(e^{i theta} P)
-      if (has_y) ek -= w2y * (ey.x * pyr - ey.y * pyi);
-      if (has_z) ek -= w2z * (ez.x * pzr - ez.y * pzi);
+      if (kPer || has_x) ek -= w2x * (ex.x * pxr - ex.y * pxi);
+      if (kPer || has_y) ek -= w2y * (ey.x * pyr - ey.y * pyi);
+      if (kPer || has_z) ek -= w2z * (ez.x * pzr - ez.y * pzi);
       ekin += ek;
-      eloc += a.v[(long long)dom * g.ng + ((long long)x * g.ny + y) * g.nz + z] * rho;
     }
-    if (q == 0 && valid) {
+    // reduce-scatter of (rho, jx, jy, jz) over the kSub = 8 lanes of the point (fixed order)
+    double u0, u1;
+    {
+      const bool hi = (q & 4) != 0;  // lanes 4..7 keep (jy, jz), lanes 0..3 keep (rho, jx)
+      const double s0 = hi ? rho : jy, s1 = hi ? jx : jz;
+      const double k0 = hi ? jy : rho, k1 = hi ? jz : jx;
+      u0 = k0 + __shfl_xor_sync(0xffffffffu, s0, 4);
+      u1 = k1 + __shfl_xor_sync(0xffffffffu, s1, 4);
+    }
+    double val;
+    {
+      const bool hi = (q & 2) != 0;  // keep the second of the two
+      const double sd = hi ? u0 : u1, kp = hi ? u1 : u0;
+      val = kp + __shfl_xor_sync(0xffffffffu, sd, 2);
+    }
+    val += __shfl_xor_sync(0xffffffffu, val, 1);
+    // lanes 2v, 2v+1 now hold value v: 0 rho, 1 jx, 2 jy, 3 jz
+    if (valid && (q & 1) == 0) {
       const long long o = (long long)x * a.sx + (long long)y * a.sy + z;
-      a.rho[a.base[dom] + o] = rho;
-      if (a.j) {
-        const long long oj = a.jbase[dom] + o;
-        a.j[oj] = jx;
-        a.j[oj + a.jstride] = jy;
-        a.j[oj + 2 * a.jstride] = jz;
+      if (vsel == 0) {
+        a.rho[a.base[dom] + o] = val;
+        if (a.epart) eloc += a.v[(long long)dom * g.ng + ((long long)x * g.ny + y) * g.nz + z] * val;
+      } else {
+        jacc += val;
+        if (a.j) a.j[a.jbase[dom] + o + (vsel - 1) * a.jstride] = val;
       }
     }
   }
+  // per-CTA sums in a fixed order: J components from lanes q = 2, 4, 6 of every point, energies from all
   const int pts = nconsw * 32 / kSub;
+  if (q == 2 || q == 4 || q == 6) jsh[q / 2 - 1][pt] = jacc;
+  double ekp = ekin;  // sum the kinetic partials over the 8 lanes of the point (fixed tree)
+  ekp += __shfl_xor_sync(0xffffffffu, ekp, 4);
+  ekp += __shfl_xor_sync(0xffffffffu, ekp, 2);
+  ekp += __shfl_xor_sync(0xffffffffu, ekp, 1);
   if (q == 0) {
-    jsh[0][pt] = jsx; jsh[1][pt] = jsy; jsh[2][pt] = jsz;
-    jsh[3][pt] = ekin; jsh[4][pt] = eloc;
+    jsh[3][pt] = ekp;
+    jsh[4][pt] = eloc;
   }
   asm volatile("bar.sync 1, %0;" ::"r"(nconsw * 32));  // consumer warps only
   if (a.epart && tid >= 3 && tid < 5) {  // (warp 0: there may be a single consumer warp)
@@ -538,7 +564,13 @@ cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps*
   dim3 grid(density_blocks(g), g.ndom);
   if (maps) {
     const int threads = ((maps->zc * kSub + 31) / 32 + 1) * 32;
-    k_density_y<<<grid, threads, ymarch_smem(g, maps->zc), st>>>(*maps, g, a);
+    const size_t sm = ymarch_smem(g, maps->zc);
+    if (g.bc == 0 && g.norb == 64)
+      k_density_y<true, 8><<<grid, threads, sm, st>>>(*maps, g, a);
+    else if (g.bc == 0)
+      k_density_y<true, 0><<<grid, threads, sm, st>>>(*maps, g, a);
+    else
+      k_density_y<false, 0><<<grid, threads, sm, st>>>(*maps, g, a);
     return cudaGetLastError();
   }
   if (ymarch_zc(g) > 0) return cudaErrorInvalidValue;  // the block layout expects the y-marching kernel
@@ -554,7 +586,11 @@ cudaError_t density_set_attributes() {
   cudaError_t e = cudaFuncSetAttribute(k_density_tma, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        density_smem_bytes(kMaxNorbTma));
   if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(k_density_y, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024);
+  for (auto f : {k_density_y<true, 8>, k_density_y<true, 0>, k_density_y<false, 0>}) {
+    e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
 }
 
 // J_d = (1/Ngrid) sum_lines jline (one block per domain, fixed-order tree over a fixed partition).
