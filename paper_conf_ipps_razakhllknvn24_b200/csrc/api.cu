@@ -330,7 +330,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false) {
   else
     LFD_TRY(launch(c, LFD_K_NL_NORM, "k_nlnorm", [&] {
       return lfd::launch_nlnorm(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), r.out, r.s,
-                                c->at<double>(c->L.nfac), c->stream);
+                                c->at<double>(c->L.nfac), r.cprime, c->stream);
     }));
   return gemm2(c);
 }

@@ -95,22 +95,25 @@ struct ReduceArgs {
 };
 cudaError_t launch_reduce(const ReduceArgs& a, cudaStream_t st);
 
-// n_s = sqrt( s_s / (s_s + eps^2 * (DC)_s^H G (DC)_s) )   (Gram closed form of the Eq. 6 norm, R11)
+// n_s = sqrt( s_s / (s_s + eps^2 * (DC)_s^H G (DC)_s) )   (Gram closed form of the Eq. 6 norm, R11),
+// then C'_s <- C'_s n_s in place: the GEMM-2 coefficient is always C'' = C' diag(n), so its epilogue is
+// Psi n + B C'' (and the projection carry uses DC_new = n DC + D G C'').
 cudaError_t launch_nlnorm(int ndom, int nproj, int norb, double eps, const double2* G,
-                          const double2* DC, const double* s, double* nfac, cudaStream_t st);
+                          const double2* DC, const double* s, double* nfac, double2* Cp, cudaStream_t st);
 
-// Combined factor of two consecutive nonlocal halves (lfd_step_sequence): X = (2c D + c^2 D G D) C
-// written to X (the GEMM-2 C'), nfac from the Gram closed form of ||Psi + B X||.
+// Combined factor of two consecutive nonlocal halves (lfd_step_sequence): X = (2c D + c^2 D G D) C,
+// nfac from the Gram closed form of ||Psi + B X||; X diag(n) is written (the GEMM-2 coefficient).
 cudaError_t launch_nlmerge(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
                            const double2* DC, const double* s, double2* X, double* nfac, cudaStream_t st);
 
-// Projection carry after a GEMM-2 Psi <- (Psi + B X) diag(n): DC <- (DC + D (G X)) diag(n) and
-// X <- -i eps DC (the C' of the next nonlocal factor), in place; column norms s are unchanged.
+// Projection carry after a GEMM-2 Psi <- Psi diag(n) + B X'' (X'' = X diag(n)): DC <- n DC + D (G X'')
+// and X <- -i eps DC (the C' of the next nonlocal factor), in place; column norms s are unchanged.
 // with_norm: also the next factor's n_s (as launch_nlnorm) in the same kernel (nfac is overwritten).
 cudaError_t launch_nlcarry(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
                            double2* DC, double2* X, const double* s, double* nfac, bool with_norm, cudaStream_t st);
 
-// GEMM-2 in place: psi[dom][r][n] <- nfac[dom][n] * (psi[dom][r][n] + sum_m B[dom][r][m] Cp[dom][m][n])
+// GEMM-2 in place: psi[dom][r][n] <- nfac[dom][n] * psi[dom][r][n] + sum_m B[dom][r][m] Cp[dom][m][n]
+// (Cp = C'' = C' diag(n), scaled by the norm / merge / carry kernels)
 struct Gemm2Args {
   double2* psi;
   const double2* B;

@@ -390,7 +390,7 @@ cudaError_t launch_reduce(const ReduceArgs& a, cudaStream_t st) {
 // ------------------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(256) k_nlnorm(int nproj, int norb, double eps2, const double2* __restrict__ G,
                                                 const double2* __restrict__ DC, const double* __restrict__ s,
-                                                double* __restrict__ nfac) {
+                                                double* __restrict__ nfac, double2* __restrict__ Cp) {
   extern __shared__ double2 dcs[];  // DC[:, col]
   __shared__ double wq[8];
   const int dom = blockIdx.y, col = blockIdx.x;
@@ -422,14 +422,22 @@ __global__ void __launch_bounds__(256) k_nlnorm(int nproj, int norb, double eps2
     double tq = 0.0;
     for (int w = 0; w < 8; ++w) tq += wq[w];
     const double sv = s[(long long)dom * norb + col];
-    nfac[(long long)dom * norb + col] = sqrt(sv / (sv + eps2 * tq));
+    const double n = sqrt(sv / (sv + eps2 * tq));
+    nfac[(long long)dom * norb + col] = n;
+    wq[0] = n;
+  }
+  __syncthreads();
+  const double n = wq[0];  // C'' = C' n (the GEMM-2 epilogue is then Psi n + B C'')
+  for (int u = threadIdx.x; u < nproj; u += blockDim.x) {
+    double2& c = Cp[((long long)dom * nproj + u) * norb + col];
+    c = make_double2(c.x * n, c.y * n);
   }
 }
 
 cudaError_t launch_nlnorm(int ndom, int nproj, int norb, double eps, const double2* G, const double2* DC,
-                          const double* s, double* nfac, cudaStream_t st) {
+                          const double* s, double* nfac, double2* Cp, cudaStream_t st) {
   dim3 grid(norb, ndom);
-  k_nlnorm<<<grid, 256, nproj * sizeof(double2), st>>>(nproj, norb, eps * eps, G, DC, s, nfac);
+  k_nlnorm<<<grid, 256, nproj * sizeof(double2), st>>>(nproj, norb, eps * eps, G, DC, s, nfac, Cp);
   return cudaGetLastError();
 }
 
@@ -479,10 +487,7 @@ __global__ void __launch_bounds__(256) k_nlmerge(int nproj, int norb, double eps
     const double du = Dd[u];
     // X_u = -2 i eps DC_u - eps^2 D_u (G DC)_u
     const double2 x = make_double2(2.0 * eps * cu.y - eps * eps * du * yr, -2.0 * eps * cu.x - eps * eps * du * yi);
-    if (lane == 0) {
-      xs[u] = x;
-      X[((long long)dom * nproj + u) * norb + col] = x;
-    }
+    if (lane == 0) xs[u] = x;
   }
   __syncthreads();
   for (int u = warp; u < nproj; u += 8) {
@@ -503,8 +508,14 @@ __global__ void __launch_bounds__(256) k_nlmerge(int nproj, int norb, double eps
       t2 += wq[1][w];
     }
     const double sv = s[(long long)dom * norb + col];
-    nfac[(long long)dom * norb + col] = sqrt(sv / (sv - 2.0 * eps * eps * t1 + t2));
+    const double n = sqrt(sv / (sv - 2.0 * eps * eps * t1 + t2));
+    nfac[(long long)dom * norb + col] = n;
+    wq[0][0] = n;
   }
+  __syncthreads();
+  const double n = wq[0][0];  // X'' = X n (the GEMM-2 epilogue is then Psi n + B X'')
+  for (int u = threadIdx.x; u < nproj; u += blockDim.x)
+    X[((long long)dom * nproj + u) * norb + col] = make_double2(xs[u].x * n, xs[u].y * n);
 }
 
 cudaError_t launch_nlmerge(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
@@ -562,9 +573,9 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
     gdot(u, xs, tr, ti);
     if (lane == 0) {
       const double du = Dd[u];
-      const double2 d = make_double2(n * fma(du, tr, dcs[u].x), n * fma(du, ti, dcs[u].y));
+      const double2 d = make_double2(fma(n, dcs[u].x, du * tr), fma(n, dcs[u].y, du * ti));
       DC[cb + (long long)u * norb] = d;
-      X[cb + (long long)u * norb] = make_double2(eps * d.y, -eps * d.x);  // -i eps DC_new
+      if (!kNorm) X[cb + (long long)u * norb] = make_double2(eps * d.y, -eps * d.x);  // -i eps DC_new
       dcs[u] = d;  // only this lane reads dcs[u] above
     }
   }
@@ -584,8 +595,14 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
     double tq = 0.0;
     for (int w = 0; w < 8; ++w) tq += wq[w];
     const double sv = s[(long long)dom * norb + col];
-    nfac[(long long)dom * norb + col] = sqrt(sv / (sv + eps * eps * tq));
+    const double nn = sqrt(sv / (sv + eps * eps * tq));
+    nfac[(long long)dom * norb + col] = nn;
+    wq[0] = nn;
   }
+  __syncthreads();
+  const double nn = wq[0];  // C'' = -i eps DC_new n_new
+  for (int u = threadIdx.x; u < nproj; u += blockDim.x)
+    X[cb + (long long)u * norb] = make_double2(eps * dcs[u].y * nn, -eps * dcs[u].x * nn);
 }
 
 cudaError_t launch_nlcarry(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
@@ -731,7 +748,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
           const long long r = r0 + wm * 32 + mi * 8 + g;
           if (r < p.ng)
             psi[r * p.norb + col] =
-                make_double2(f * (pv[mi][ni][c].x + acc.re(mi, ni, c)), f * (pv[mi][ni][c].y + acc.im(mi, ni, c)));
+                make_double2(fma(f, pv[mi][ni][c].x, acc.re(mi, ni, c)), fma(f, pv[mi][ni][c].y, acc.im(mi, ni, c)));
         }
       }
   }
@@ -884,7 +901,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
           const long long r = r0 + wm * 32 + mi * 8 + g;
           if (r < p.ng)
             psi[r * p.norb + col] =
-                make_double2(f * (pv[mi][ni][c].x + acc.re(mi, ni, c)), f * (pv[mi][ni][c].y + acc.im(mi, ni, c)));
+                make_double2(fma(f, pv[mi][ni][c].x, acc.re(mi, ni, c)), fma(f, pv[mi][ni][c].y, acc.im(mi, ni, c)));
         }
       }
   }
@@ -1029,7 +1046,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant
           const long long r = r0 + wm * 32 + mi * 8 + g;
           if (r < p.ng)
             psi[r * p.norb + col] =
-                make_double2(f * (pv[mi][ni][c].x + acc.re(mi, ni, c)), f * (pv[mi][ni][c].y + acc.im(mi, ni, c)));
+                make_double2(fma(f, pv[mi][ni][c].x, acc.re(mi, ni, c)), fma(f, pv[mi][ni][c].y, acc.im(mi, ni, c)));
         }
       }
   }
