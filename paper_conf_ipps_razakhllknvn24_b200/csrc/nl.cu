@@ -308,7 +308,7 @@ static cudaError_t gemm1_maps(const Gemm1Args& a, CUtensorMap* tA, CUtensorMap* 
 }
 
 int gemm1_smem_bytes() { return kStages1 * kStage1Bytes + 2 * kStages1 * 8; }
-int gemm2_smem_bytes() { return kStages2 * kStage2Bytes + kStages2 * 8; }
+int gemm2_smem_bytes() { return kStages2 * kStage2Bytes + 2 * kStages2 * 8; }
 
 cudaError_t launch_gemm1(const Gemm1Args& a, cudaStream_t st) {
   const int tiles = ((a.mrows + kTile - 1) / kTile) * ((a.ncols + kTile - 1) / kTile);
@@ -616,8 +616,9 @@ cudaError_t launch_nlcarry(int ndom, int nproj, int norb, double eps, const doub
 }
 
 // ------------------------------------------------------------------------------------------------
-// GEMM-2 (persistent): psi[r][n] <- nfac[n] * (psi[r][n] + sum_m B[r][m] Cp[m][n]) for every
-// (dom, 64-row block, 64-column tile) work item; K = nproj in chunks of 16 through the TMA ring.
+// GEMM-2 (persistent, any nproj): psi[r][n] <- nfac[n] psi[r][n] + sum_m B[r][m] Cp[m][n] for every
+// (dom, 64-row block, 64-column tile) work item; K = nproj in chunks of kKC2 through a TMA tensor-map
+// ring (full/empty mbarriers; thread 0 refills a stage once every warp has released it).
 // ------------------------------------------------------------------------------------------------
 template <bool kTail>
 __device__ __forceinline__ void gemm2_chunk(const double2* As, const double2* Cs, int kv, int wm, int wn, int g,
@@ -635,9 +636,11 @@ __device__ __forceinline__ void gemm2_chunk(const double2* As, const double2* Cs
   }
 }
 
-__global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
+__global__ void __launch_bounds__(kThreads, 1) k_gemm2(const __grid_constant__ CUtensorMap tA,
+                                                       const __grid_constant__ CUtensorMap tC, Gemm2Args p) {
   extern __shared__ __align__(128) unsigned char smem[];
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kStages2 * kStage2Bytes);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages2 * kStage2Bytes);
+  uint64_t* empty = full + kStages2;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int g = lane >> 2, t = lane & 3;
   const int wm = warp >> 2, wn = warp & 3;
@@ -647,7 +650,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
   const int nk = (p.nproj + kKC2 - 1) / kKC2;
 
   if (tid == 0) {
-    for (int s = 0; s < kStages2; ++s) mbar_init(&bars[s], 1);
+    for (int s = 0; s < kStages2; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], kConsWarps1);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
@@ -665,30 +671,24 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
     n0 = (int)(rem - rb * ntn) * kTile;
   };
 
-  auto issue = [&](long long gc, int stage) {  // warp 0 only
+  // chunk gc -> stage gc % kStages2: two tiled tensor copies, the B block [64 rows][kKC2 + 4 complex]
+  // (columns past nproj and rows past ng are zero fill) and the C'' block [kKC2 rows][66 complex]
+  auto issue = [&](long long gc) {  // thread 0 only
+    const int stage = (int)(gc % kStages2);
     const long long item = blockIdx.x + (gc / nk) * gridDim.x;
     const int kc = (int)(gc % nk);
     int dom, n0;
     long long r0;
     decode(item, dom, r0, n0);
-    const int rows = (int)min((long long)kTile, p.ng - r0);
-    const int k0 = kc * kKC2;
-    const int kv = min(kKC2, p.nproj - k0);
-    const int nvalid = min(kTile, p.norb - n0);
     double2* As = reinterpret_cast<double2*>(smem + stage * kStage2Bytes);
     double2* Cs = As + kTile * kLdA2;
-    if (lane == 0) mbar_expect_tx(&bars[stage], (uint32_t)((rows * kv + kv * nvalid) * 16));
-    __syncwarp();
-    const double2* Bg = p.B + (long long)dom * p.ng * p.nproj + k0;
-    for (int r = lane; r < rows; r += 32)
-      tma_row(As + r * kLdA2, Bg + (r0 + r) * p.nproj, kv * 16, &bars[stage]);
-    if (lane < kv)
-      tma_row(Cs + lane * kLd1, p.Cp + ((long long)dom * p.nproj + k0 + lane) * p.norb + n0, nvalid * 16,
-              &bars[stage]);
+    mbar_expect_tx(&full[stage], (uint32_t)kStage2Bytes);
+    tma_3d(As, &tA, 2 * kc * kKC2, (int)r0, dom, &full[stage]);
+    tma_3d(Cs, &tC, 2 * n0, kc * kKC2, dom, &full[stage]);
   };
 
-  if (warp == 0)
-    for (int s = 0; s < kStages2 && s < total; ++s) issue(s, s);
+  if (tid == 0)
+    for (long long s = 0; s < kStages2 && s < total; ++s) issue(s);
 
   long long gc = 0;
   for (long long it = 0; it < my_items; ++it) {
@@ -711,16 +711,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(Gemm2Args p) {
     acc.zero();
     for (int kc = 0; kc < nk; ++kc, ++gc) {
       const int stage = (int)(gc % kStages2);
-      mbar_wait(&bars[stage], (uint32_t)((gc / kStages2) & 1));
+      mbar_wait(&full[stage], (uint32_t)((gc / kStages2) & 1));
       const double2* As = reinterpret_cast<const double2*>(smem + stage * kStage2Bytes);
       const double2* Cs = As + kTile * kLdA2;
-      const int kv = min(kKC2, p.nproj - kc * kKC2);
-      if (kv == kKC2)
-        gemm2_chunk<false>(As, Cs, kv, wm, wn, g, t, acc);
-      else
-        gemm2_chunk<true>(As, Cs, kv, wm, wn, g, t, acc);
-      __syncthreads();
-      if (warp == 0 && gc + kStages2 < total) issue(gc + kStages2, stage);
+      gemm2_chunk<false>(As, Cs, kKC2, wm, wn, g, t, acc);  // the K tail is zero fill
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[stage]);
+      if (tid == 0 && gc + kStages2 < total) {  // refill once every warp has released the stage
+        mbar_wait(&empty[stage], (uint32_t)((gc / kStages2) & 1));
+        issue(gc + kStages2);
+      }
     }
     // epilogue: Psi <- n_s (Psi + B C'); all 16 loads (L2 hits) are issued before any store
     const double* nf = p.nfac + (long long)dom * p.norb;
@@ -1092,8 +1092,21 @@ cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
     k_gemm2_fullk<kTile, false><<<grid, kThreads, kFullSmem, st>>>(a);
   else if (a.nproj < kTile)
     k_gemm2_fullk<0, false><<<grid, kThreads, kFullSmem, st>>>(a);
-  else
-    k_gemm2<<<grid, kThreads, gemm2_smem_bytes(), st>>>(a);
+  else {
+    // B [dom][ng][nproj] (box [1][64 rows][kKC2 + 4 complex]) and C'' [dom][nproj][norb] (box [1][kKC2][66])
+    CUtensorMap tA, tC;
+    const uint64_t dA[3] = {(uint64_t)2 * a.nproj, (uint64_t)a.ng, (uint64_t)a.ndom};
+    const uint64_t sA[2] = {(uint64_t)a.nproj * 16, (uint64_t)a.ng * a.nproj * 16};
+    const uint32_t bA[3] = {2 * kLdA2, kTile, 1};
+    cudaError_t e = encode_tmap_f64(&tA, 3, a.B, dA, sA, bA);
+    if (e != cudaSuccess) return e;
+    const uint64_t dC[3] = {(uint64_t)2 * a.norb, (uint64_t)a.nproj, (uint64_t)a.ndom};
+    const uint64_t sC[2] = {(uint64_t)a.norb * 16, (uint64_t)a.nproj * a.norb * 16};
+    const uint32_t bC[3] = {2 * kLd1, kKC2, 1};
+    e = encode_tmap_f64(&tC, 3, a.Cp, dC, sC, bC);
+    if (e != cudaSuccess) return e;
+    k_gemm2<<<grid, kThreads, gemm2_smem_bytes(), st>>>(tA, tC, a);
+  }
   return cudaGetLastError();
 }
 
