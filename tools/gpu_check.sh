@@ -11,6 +11,6 @@ timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${TA
 timeout 600 python bench.py > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_bench.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv \
    python bench.py --steps 3 --warmup 1 --no-cpu-baseline --no-e2e > gpurun_out/${TAG}_ncu_bench.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:"${KREGEX:-k_gemm1|k_gemm2|k_kin|k_density}" -s ${KSKIP:-20} -c ${KCOUNT:-6} \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"${KREGEX:-k_gemm1|k_gemm2|k_kin|k_density}" -s ${KSKIP:-8} -c ${KCOUNT:-6} \
    -o gpurun_out/${TAG}_prof -f python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e > gpurun_out/${TAG}_ncu_full.log 2>&1
 echo done
