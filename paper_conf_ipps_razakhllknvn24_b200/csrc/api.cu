@@ -96,7 +96,7 @@ Layout layout(const Geometry& g, int num_sms, int nref_max) {
   int nsplit = 1;
   if (tiles > 0) {
     double best = 0.0;
-    const long long max_s = std::max<long long>(1, std::min<long long>(2LL * num_sms, g.ng / (8 * kKC1)));
+    const long long max_s = std::max<long long>(1, std::min<long long>(2LL * num_sms, g.ng / (2 * kKC1)));
     for (long long s = 1; s <= max_s; ++s) {
       const long long ctas = (long long)tiles * s;
       const long long waves = (ctas + num_sms - 1) / num_sms;

@@ -31,7 +31,6 @@ constexpr int kStages = 4;
 // GEMM-1 stage: A rows [KC1][kLd1] (B rows, m along the row) and X rows [KC1][kLd1].
 constexpr int kKC1 = 32;
 constexpr int kLd1 = kTile + 2;
-constexpr int kStage1Bytes = 2 * kKC1 * kLd1 * 16;
 constexpr int kStages1 = 3;
 constexpr int kConsWarps1 = 8;
 constexpr int kThreads1 = kConsWarps1 * 32 + 32;  // + producer warp
@@ -142,63 +141,73 @@ __device__ __forceinline__ void mma_4x2(Frag& acc, const double2 (&a)[4], const 
 #endif
 }
 
-// acc += conj(a) * x (GEMM-1 orientation: A = conj(B)^T).
-__device__ __forceinline__ void mma_conj_4x2(Frag& acc, const double2 (&a)[4], const double2 (&x)[2]) {
-#if LFD_3M
-  double as[4], xs[2];
-#pragma unroll
-  for (int mi = 0; mi < 4; ++mi) as[mi] = a[mi].x - a[mi].y;
-#pragma unroll
-  for (int ni = 0; ni < 2; ++ni) xs[ni] = x[ni].x + x[ni].y;
-#pragma unroll
-  for (int mi = 0; mi < 4; ++mi)
-#pragma unroll
-    for (int ni = 0; ni < 2; ++ni) dmma(acc.t1[mi][ni][0], acc.t1[mi][ni][1], a[mi].x, x[ni].x);
-#pragma unroll
-  for (int mi = 0; mi < 4; ++mi)
-#pragma unroll
-    for (int ni = 0; ni < 2; ++ni) dmma(acc.t2[mi][ni][0], acc.t2[mi][ni][1], a[mi].y, x[ni].y);
-#pragma unroll
-  for (int mi = 0; mi < 4; ++mi)
-#pragma unroll
-    for (int ni = 0; ni < 2; ++ni) dmma(acc.t3[mi][ni][0], acc.t3[mi][ni][1], as[mi], xs[ni]);
-#else
-#pragma unroll
-  for (int mi = 0; mi < 4; ++mi)
-#pragma unroll
-    for (int ni = 0; ni < 2; ++ni) dmma(acc.t1[mi][ni][0], acc.t1[mi][ni][1], a[mi].x, x[ni].x);  // + br xr
-#pragma unroll
-  for (int mi = 0; mi < 4; ++mi)
-#pragma unroll
-    for (int ni = 0; ni < 2; ++ni) dmma(acc.t2[mi][ni][0], acc.t2[mi][ni][1], a[mi].x, x[ni].y);  // + br xi
-#pragma unroll
-  for (int mi = 0; mi < 4; ++mi)
-#pragma unroll
-    for (int ni = 0; ni < 2; ++ni) dmma(acc.t1[mi][ni][0], acc.t1[mi][ni][1], a[mi].y, x[ni].y);  // + bi xi
-#pragma unroll
-  for (int mi = 0; mi < 4; ++mi)
-#pragma unroll
-    for (int ni = 0; ni < 2; ++ni) dmma(acc.t2[mi][ni][0], acc.t2[mi][ni][1], -a[mi].y, x[ni].x);  // - bi xr
-#endif
-}
-
 }  // namespace
 
 // ------------------------------------------------------------------------------------------------
 // GEMM-1: part[dom][split][m][n] = sum_{r in split} conj(A[r][m]) X[r][n];  norms[dom][split][n].
-// grid: (nsplit, mtiles*ntiles, ndom), block 8 consumer warps (2 x 4, warp tile 32 x 16 complex) + 1
-// producer warp. Per chunk of kKC1 grid rows the producer issues TWO tiled TMA tensor copies (the A and
-// X row blocks, box [kKC1 rows][66 complex]: the 2 columns past a 64-wide tile are the next tile's or
-// zero fill, which pads every smem row to 66 complex so the DMMA fragment LDS.128 are bank-conflict
-// free) into a kStages1-deep ring with full/empty mbarriers; consumer warps release a stage when done
-// with it (no CTA-wide barrier in the K loop). Rows past the domain end are zero-filled by the TMA
-// (rows_per_split is a multiple of kKC1, so every other chunk is whole). The column norms s_s are
-// accumulated from the X fragments, the k-steps split between the two M-warps of a column slice.
+// grid: (nsplit, mtiles*ntiles, ndom), block 8 consumer warps + 1 producer warp. CTA tile kMT x 64
+// complex: kMT = 64 uses 2 x 4 warps (warp tile 32 x 16); kMT = 32 / 16 (few projectors, e.g. the
+// paper-timing-consistent nproj = 16, R20) use 1 x 8 warps (warp tile kMT x 8) so no DMMA work is spent
+// on empty projector rows. Per chunk of kKC1 grid rows the producer issues TWO tiled TMA tensor copies
+// (the A and X row blocks, box [kKC1 rows][tile + 2 complex]: the 2 extra columns are the next tile's
+// data or zero fill, which pads every smem row to == 2 mod 8 complex so the DMMA fragment LDS.128 are
+// bank-conflict free) into a kStages1-deep ring with full/empty mbarriers; consumer warps release a
+// stage when done with it (no CTA-wide barrier in the K loop). Rows past the domain end are zero-filled
+// by the TMA (rows_per_split is a multiple of kKC1, so every other chunk is whole). The column norms s_s
+// are accumulated from the X fragments, the k-steps split between the M-warps of a column slice.
 // ------------------------------------------------------------------------------------------------
+template <int MI, int NI>
+struct FragT {
+  double t1[MI][NI][2], t2[MI][NI][2], t3[MI][NI][2];
+  __device__ __forceinline__ void zero() {
+#pragma unroll
+    for (int i = 0; i < MI; ++i)
+#pragma unroll
+      for (int j = 0; j < NI; ++j)
+#pragma unroll
+        for (int c = 0; c < 2; ++c) t1[i][j][c] = t2[i][j][c] = t3[i][j][c] = 0.0;
+  }
+};
+
+// acc += conj(a) * x, 3M (see Frag): T1 = ar xr, T2 = ai xi, T3 = (ar - ai)(xr + xi)
+template <int MI, int NI>
+__device__ __forceinline__ void mma_conj(FragT<MI, NI>& acc, const double2 (&a)[MI], const double2 (&x)[NI]) {
+  double as[MI], xs[NI];
+#pragma unroll
+  for (int mi = 0; mi < MI; ++mi) as[mi] = a[mi].x - a[mi].y;
+#pragma unroll
+  for (int ni = 0; ni < NI; ++ni) xs[ni] = x[ni].x + x[ni].y;
+#pragma unroll
+  for (int mi = 0; mi < MI; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < NI; ++ni) dmma(acc.t1[mi][ni][0], acc.t1[mi][ni][1], a[mi].x, x[ni].x);
+#pragma unroll
+  for (int mi = 0; mi < MI; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < NI; ++ni) dmma(acc.t2[mi][ni][0], acc.t2[mi][ni][1], a[mi].y, x[ni].y);
+#pragma unroll
+  for (int mi = 0; mi < MI; ++mi)
+#pragma unroll
+    for (int ni = 0; ni < NI; ++ni) dmma(acc.t3[mi][ni][0], acc.t3[mi][ni][1], as[mi], xs[ni]);
+}
+
+template <int kMT>
+struct G1Shape {
+  static constexpr int WM = kMT == 64 ? 2 : 1;   // warps along M
+  static constexpr int WN = 8 / WM;              // warps along N
+  static constexpr int MI = kMT / WM / 8;        // 8-row fragments per warp
+  static constexpr int NI = kTile / WN / 8;      // 8-column fragments per warp
+  static constexpr int LDA = kMT + 2;            // smem row pitch of the A block (complex)
+  static constexpr int ABytes = kKC1 * LDA * 16;
+  static constexpr int StageBytes = ABytes + kKC1 * kLd1 * 16;
+};
+
+template <int kMT>
 __global__ void __launch_bounds__(kThreads1, 1) k_gemm1(const __grid_constant__ CUtensorMap tA,
                                                          const __grid_constant__ CUtensorMap tX, Gemm1Args p) {
+  using S = G1Shape<kMT>;
   extern __shared__ __align__(128) unsigned char smem[];
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages1 * kStage1Bytes);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages1 * S::StageBytes);
   uint64_t* empty = full + kStages1;
   __shared__ double nsh[2][kTile];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -206,7 +215,7 @@ __global__ void __launch_bounds__(kThreads1, 1) k_gemm1(const __grid_constant__ 
   const int ntn = (p.ncols + kTile - 1) / kTile;
   const int mt = blockIdx.y / ntn, nt = blockIdx.y - (blockIdx.y / ntn) * ntn;
   const int dom = blockIdx.z;
-  const int m0 = mt * kTile, n0 = nt * kTile;
+  const int m0 = mt * kMT, n0 = nt * kTile;
   const long long kbeg = (long long)split * p.rows_per_split;
   const long long kend = min(p.ng, kbeg + p.rows_per_split);
   const int nchunks = (kend > kbeg) ? (int)((kend - kbeg + kKC1 - 1) / kKC1) : 0;
@@ -225,98 +234,115 @@ __global__ void __launch_bounds__(kThreads1, 1) k_gemm1(const __grid_constant__ 
       for (int i = 0; i < nchunks; ++i) {
         const int s = i % kStages1;
         if (i >= kStages1) mbar_wait(&empty[s], (uint32_t)(((i / kStages1) - 1) & 1));
-        mbar_expect_tx(&full[s], (uint32_t)kStage1Bytes);
-        double2* As = reinterpret_cast<double2*>(smem + s * kStage1Bytes);
+        mbar_expect_tx(&full[s], (uint32_t)S::StageBytes);
+        unsigned char* st = smem + s * S::StageBytes;
         const int r0 = (int)(kbeg + (long long)i * kKC1);
-        tma_3d(As, &tA, 2 * m0, r0, dom, &full[s]);
-        tma_3d(As + kKC1 * kLd1, &tX, 2 * n0, r0, dom, &full[s]);
+        tma_3d(st, &tA, 2 * m0, r0, dom, &full[s]);
+        tma_3d(st + S::ABytes, &tX, 2 * n0, r0, dom, &full[s]);
       }
     }
     return;
   }
 
   const int g = lane >> 2, t = lane & 3;
-  const int wm = warp >> 2, wn = warp & 3;
-  const int mvalid = min(kTile, p.mrows - m0), nvalid = min(kTile, p.ncols - n0);
-  Frag acc;
+  const int wm = warp / S::WN, wn = warp - (warp / S::WN) * S::WN;
+  const int mvalid = min(kMT, p.mrows - m0), nvalid = min(kTile, p.ncols - n0);
+  FragT<S::MI, S::NI> acc;
   acc.zero();
-  double nrm[2] = {0.0, 0.0};
+  double nrm[S::NI];
+#pragma unroll
+  for (int ni = 0; ni < S::NI; ++ni) nrm[ni] = 0.0;
   const bool do_norm = (p.norms != nullptr) && (mt == 0);
 
   for (int i = 0; i < nchunks; ++i) {
     const int s = i % kStages1;
     mbar_wait(&full[s], (uint32_t)((i / kStages1) & 1));
-    const double2* As = reinterpret_cast<const double2*>(smem + s * kStage1Bytes);
-    const double2* Xs = As + kKC1 * kLd1;
+    const double2* As = reinterpret_cast<const double2*>(smem + s * S::StageBytes);
+    const double2* Xs = reinterpret_cast<const double2*>(smem + s * S::StageBytes + S::ABytes);
 #pragma unroll
     for (int kk = 0; kk < kKC1; kk += 4) {
       const int k = kk + t;
-      double2 a[4], x[2];
+      double2 a[S::MI], x[S::NI];
 #pragma unroll
-      for (int mi = 0; mi < 4; ++mi) a[mi] = As[k * kLd1 + wm * 32 + mi * 8 + g];
+      for (int mi = 0; mi < S::MI; ++mi) a[mi] = As[k * S::LDA + wm * (kMT / S::WM) + mi * 8 + g];
 #pragma unroll
-      for (int ni = 0; ni < 2; ++ni) x[ni] = Xs[k * kLd1 + wn * 16 + ni * 8 + g];
-      if (do_norm && ((kk >> 2) & 1) == wm) {
+      for (int ni = 0; ni < S::NI; ++ni) x[ni] = Xs[k * kLd1 + wn * (kTile / S::WN) + ni * 8 + g];
+      if (do_norm && ((kk >> 2) % S::WM) == wm) {
 #pragma unroll
-        for (int ni = 0; ni < 2; ++ni) nrm[ni] = fma(x[ni].x, x[ni].x, fma(x[ni].y, x[ni].y, nrm[ni]));
+        for (int ni = 0; ni < S::NI; ++ni) nrm[ni] = fma(x[ni].x, x[ni].x, fma(x[ni].y, x[ni].y, nrm[ni]));
       }
-      mma_conj_4x2(acc, a, x);
+      mma_conj(acc, a, x);
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(&empty[s]);
   }
 
-  // epilogue: split partials (fixed positions, reduced in order by k_reduce)
+  // epilogue: split partials (fixed positions, reduced in order by k_reduce); 3M recombination for
+  // conj(A): Re = T1 + T2, Im = T3 - T1 + T2
   double2* out = p.part + (((long long)dom * p.nsplit + split) * p.mrows) * p.ncols;
 #pragma unroll
-  for (int mi = 0; mi < 4; ++mi) {
-    const int row = wm * 32 + mi * 8 + g;
+  for (int mi = 0; mi < S::MI; ++mi) {
+    const int row = wm * (kMT / S::WM) + mi * 8 + g;
     if (row >= mvalid) continue;
 #pragma unroll
-    for (int ni = 0; ni < 2; ++ni)
+    for (int ni = 0; ni < S::NI; ++ni)
 #pragma unroll
       for (int c = 0; c < 2; ++c) {
-        const int col = wn * 16 + ni * 8 + 2 * t + c;
-        if (col < nvalid)
-          out[(long long)(m0 + row) * p.ncols + n0 + col] = make_double2(acc.re_conj(mi, ni, c), acc.im_conj(mi, ni, c));
+        const int col = wn * (kTile / S::WN) + ni * 8 + 2 * t + c;
+        if (col < nvalid) {
+          const double t1 = acc.t1[mi][ni][c], t2 = acc.t2[mi][ni][c], t3 = acc.t3[mi][ni][c];
+          out[(long long)(m0 + row) * p.ncols + n0 + col] = make_double2(t1 + t2, t3 - t1 + t2);
+        }
       }
   }
   if (do_norm) {
 #pragma unroll
-    for (int ni = 0; ni < 2; ++ni) {
+    for (int ni = 0; ni < S::NI; ++ni) {
       double v = nrm[ni];
       v += __shfl_xor_sync(0xffffffffu, v, 1);
       v += __shfl_xor_sync(0xffffffffu, v, 2);
-      if (t == 0) nsh[wm][wn * 16 + ni * 8 + g] = v;
+      if (t == 0) nsh[wm][wn * (kTile / S::WN) + ni * 8 + g] = v;
     }
     asm volatile("bar.sync 1, %0;" ::"n"(kConsWarps1 * 32));  // consumer warps only
-    if (tid < nvalid)
-      p.norms[((long long)dom * p.nsplit + split) * p.ncols + n0 + tid] = nsh[0][tid] + nsh[1][tid];
+    if (tid < nvalid) {
+      double v = nsh[0][tid];
+      if (S::WM == 2) v += nsh[1][tid];
+      p.norms[((long long)dom * p.nsplit + split) * p.ncols + n0 + tid] = v;
+    }
   }
 }
 
-// A [dom][ng][mrows] / X [dom][ng][ncols] complex as 3-D float64 tensors, box [1][kKC1][2*kLd1].
-static cudaError_t gemm1_maps(const Gemm1Args& a, CUtensorMap* tA, CUtensorMap* tX) {
-  const uint32_t box[3] = {2 * kLd1, kKC1, 1};
+static int gemm1_mt(int mrows) { return mrows <= 16 ? 16 : mrows <= 32 ? 32 : 64; }
+
+// A [dom][ng][mrows] / X [dom][ng][ncols] complex as 3-D float64 tensors, boxes [1][kKC1][tile + 2].
+static cudaError_t gemm1_maps(const Gemm1Args& a, int mt, CUtensorMap* tA, CUtensorMap* tX) {
+  const uint32_t boxA[3] = {(uint32_t)(2 * (mt + 2)), kKC1, 1};
+  const uint32_t boxX[3] = {2 * kLd1, kKC1, 1};
   const uint64_t dA[3] = {(uint64_t)2 * a.mrows, (uint64_t)a.ng, (uint64_t)a.ndom};
   const uint64_t sA[2] = {(uint64_t)a.mrows * 16, (uint64_t)a.a_dom_stride * 16};
-  cudaError_t e = encode_tmap_f64(tA, 3, a.A, dA, sA, box);
+  cudaError_t e = encode_tmap_f64(tA, 3, a.A, dA, sA, boxA);
   if (e != cudaSuccess) return e;
   const uint64_t dX[3] = {(uint64_t)2 * a.ncols, (uint64_t)a.ng, (uint64_t)a.ndom};
   const uint64_t sX[2] = {(uint64_t)a.ncols * 16, (uint64_t)a.x_dom_stride * 16};
-  return encode_tmap_f64(tX, 3, a.X, dX, sX, box);
+  return encode_tmap_f64(tX, 3, a.X, dX, sX, boxX);
 }
 
-int gemm1_smem_bytes() { return kStages1 * kStage1Bytes + 2 * kStages1 * 8; }
+int gemm1_smem_bytes() { return kStages1 * G1Shape<64>::StageBytes + 2 * kStages1 * 8; }
 int gemm2_smem_bytes() { return kStages2 * kStage2Bytes + 2 * kStages2 * 8; }
 
 cudaError_t launch_gemm1(const Gemm1Args& a, cudaStream_t st) {
-  const int tiles = ((a.mrows + kTile - 1) / kTile) * ((a.ncols + kTile - 1) / kTile);
+  const int mt = gemm1_mt(a.mrows);
+  const int tiles = ((a.mrows + mt - 1) / mt) * ((a.ncols + kTile - 1) / kTile);
   dim3 grid(a.nsplit, tiles, a.ndom);
   CUtensorMap tA, tX;
-  cudaError_t e = gemm1_maps(a, &tA, &tX);
+  cudaError_t e = gemm1_maps(a, mt, &tA, &tX);
   if (e != cudaSuccess) return e;
-  k_gemm1<<<grid, kThreads1, gemm1_smem_bytes(), st>>>(tA, tX, a);
+  if (mt == 16)
+    k_gemm1<16><<<grid, kThreads1, kStages1 * G1Shape<16>::StageBytes + 2 * kStages1 * 8, st>>>(tA, tX, a);
+  else if (mt == 32)
+    k_gemm1<32><<<grid, kThreads1, kStages1 * G1Shape<32>::StageBytes + 2 * kStages1 * 8, st>>>(tA, tX, a);
+  else
+    k_gemm1<64><<<grid, kThreads1, gemm1_smem_bytes(), st>>>(tA, tX, a);
   return cudaGetLastError();
 }
 
@@ -980,7 +1006,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant
     if (dom != cur_dom || n0 != cur_n0) {  // (re)load C'[dom][:, n0:n0+64] once every consumer is past Cs
       asm volatile("bar.sync 1, %0;" ::"n"(kConsWarps1 * 32));
       if (tid == 0) {
-        mbar_expect_tx(cbar, (uint32_t)(np * kLd1 * 16));
+        mbar_expect_tx(cbar, (uint32_t)(nk4 * 4 * kLd1 * 16));
         tma_3d(Cs, &tC, 2 * n0, 0, dom, cbar);
       }
       mbar_wait(cbar, cphase);
@@ -1062,7 +1088,8 @@ static cudaError_t gemm2_maps(const Gemm2Args& a, CUtensorMap* tB, CUtensorMap* 
   if (e != cudaSuccess) return e;
   const uint64_t dC[3] = {(uint64_t)2 * a.norb, (uint64_t)a.nproj, (uint64_t)a.ndom};
   const uint64_t sC[2] = {(uint64_t)a.norb * 16, (uint64_t)a.nproj * a.norb * 16};
-  const uint32_t bC[3] = {2 * kLd1, (uint32_t)a.nproj, 1};
+  // rows up to the K loop's multiple of 4: the rows past nproj are zero fill (never stale smem)
+  const uint32_t bC[3] = {2 * kLd1, (uint32_t)((a.nproj + 3) / 4 * 4), 1};
   return encode_tmap_f64(tC, 3, a.Cp, dC, sC, bC);
 }
 
@@ -1111,7 +1138,11 @@ cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
 }
 
 cudaError_t gemm_set_attributes() {
-  cudaError_t e = cudaFuncSetAttribute(k_gemm1, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm1_smem_bytes());
+  cudaError_t e = cudaFuncSetAttribute(k_gemm1<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm1_smem_bytes());
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_gemm1<32>, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm1_smem_bytes());
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_gemm1<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm1_smem_bytes());
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_gemm2_fullk<kTile, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
   if (e != cudaSuccess) return e;
