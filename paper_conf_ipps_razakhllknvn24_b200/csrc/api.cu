@@ -256,6 +256,19 @@ lfd_status launch(lfd_ctx* c, int kid, const char* name, F&& f) {
     if (st_ != LFD_OK) return st_; \
   } while (0)
 
+// 1 + the last orbital index with a nonzero occupation in any domain (at least 1): the density kernel
+// reads only these (f = 0 orbitals add exactly zero to rho, j and the energies).
+int active_orbitals(const Geometry& g, const double* occ) {
+  int n = 1;
+  for (int d = 0; d < g.ndom; ++d)
+    for (int s = g.norb - 1; s >= n; --s)
+      if (occ[(long long)d * g.norb + s] != 0.0) {
+        n = s + 1;
+        break;
+      }
+  return n;
+}
+
 lfd_status check_ctx(const lfd_ctx* c) {
   if (!c) { g_tls_error = "context is NULL"; return LFD_EINVAL; }
   if (!is_live(c)) { g_tls_error = "context is not live (destroyed or never created)"; return LFD_ESTATE; }
@@ -454,7 +467,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   if (const char* v = std::getenv("LFD_KIN_SCALED")) c->scaled = std::atoi(v) != 0;
   c->scaled = c->scaled && lfd::kin_scaled_ok(g);
   c->kin_fused = c->kin_fused && lfd::kin_yz_supported(g);
-  c->dmaps = lfd::density_maps_create(g, c->psi);
+  c->dmaps = lfd::density_maps_create(g, c->psi, active_orbitals(g, occ));
   if (c->kin_fused && lfd::kin_yz_tensor_map(g, c->psi, &c->psi_tmap) != cudaSuccess) {
     cudaGetLastError();
     c->kin_fused = false;  // descriptor not encodable (e.g. alignment): the separate y and z passes
@@ -671,6 +684,8 @@ lfd_status lfd_set_occupations(lfd_ctx* c, const double* occ) {
   cudaError_t e = cudaMemcpyAsync(c->at<double>(c->L.occ), occ, sizeof(double) * c->g.ndom * c->g.norb,
                                   cudaMemcpyHostToDevice, c->stream);
   if (e != cudaSuccess) return cuda_fail(c, e, "copy occ");
+  e = lfd::density_maps_set_active(c->dmaps, c->g, c->psi, active_orbitals(c->g, occ));
+  if (e != cudaSuccess) return cuda_fail(c, e, "density tensor map");
   return LFD_OK;
 }
 

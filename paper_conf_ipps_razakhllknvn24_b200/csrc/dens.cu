@@ -10,6 +10,7 @@
 #include "lfd_internal.h"
 #include "lfd_tma.cuh"
 
+#include <algorithm>
 #include <new>
 
 namespace lfd {
@@ -313,9 +314,10 @@ constexpr int kYOwn = 3, kYXp = 2;
 constexpr int kYMaxThreads = 352;  // up to 40 points x kSub + the producer warp
 
 struct DensMaps {
-  CUtensorMap seg;   // box [1][zc][2*norb]: a z-line segment of zc points, all orbitals
-  CUtensorMap one;   // box [1][1][2*norb]: the z+1 halo point
+  CUtensorMap seg;   // box [1][zc][2*nact]: a z-line segment of zc points, the active orbitals
+  CUtensorMap one;   // box [1][1][2*nact]: the z+1 halo point
   int zc;            // points per CTA (divides nz)
+  int nact;          // active orbitals: 1 + the last index with f != 0 (f = 0 contributes exactly 0)
 };
 
 // shared-memory layout of the y-marching kernel (every TMA destination 128-byte aligned)
@@ -349,7 +351,7 @@ template <bool kPer, int kIt>
 __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constant__ DensMaps mp, Geometry g,
                                                             DensArgs a) {
   extern __shared__ __align__(128) unsigned char dsm[];
-  const int norb = g.norb, zc = mp.zc;
+  const int norb = mp.nact, zc = mp.zc;  // smem rows hold the nact active orbitals of each point
   const YLayout Ly(zc, norb);
   auto own_slot = [&](int s) { return reinterpret_cast<double2*>(dsm + s * Ly.own_b); };
   auto halo_of = [&](int s) { return reinterpret_cast<double2*>(dsm + s * Ly.own_b + Ly.seg_b); };
@@ -373,7 +375,7 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
     for (int s = 0; s < kYXp; ++s) { mbar_init(&xfull[s], 1); mbar_init(&xempty[s], nconsw); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  for (int s = tid; s < norb; s += blockDim.x) fsh[s] = a.occ[(long long)dom * norb + s];
+  for (int s = tid; s < norb; s += blockDim.x) fsh[s] = a.occ[(long long)dom * g.norb + s];
   __syncthreads();
 
   if (tid >= nconsw * 32) {  // producer warp
@@ -529,24 +531,36 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
   }
 }
 
-static size_t ymarch_smem(const Geometry& g, int zc) { return YLayout(zc, g.norb).total; }
+static size_t ymarch_smem(int zc, int nact) { return YLayout(zc, nact).total; }
 
-DensMaps* density_maps_create(const Geometry& g, const double2* psi) {
+static cudaError_t density_maps_encode(DensMaps* m, const Geometry& g, const double2* psi, int nact) {
+  const uint64_t dims[3] = {(uint64_t)2 * g.norb, (uint64_t)g.nz, (uint64_t)g.ndom * g.nx * g.ny};
+  const uint64_t str[2] = {(uint64_t)g.norb * 16, (uint64_t)g.nz * g.norb * 16};
+  const uint32_t b2[3] = {(uint32_t)(2 * nact), (uint32_t)m->zc, 1};
+  const uint32_t b3[3] = {(uint32_t)(2 * nact), 1, 1};
+  cudaError_t e = encode_tmap_f64(&m->seg, 3, psi, dims, str, b2);
+  if (e == cudaSuccess) e = encode_tmap_f64(&m->one, 3, psi, dims, str, b3);
+  if (e == cudaSuccess) m->nact = nact;
+  return e;
+}
+
+DensMaps* density_maps_create(const Geometry& g, const double2* psi, int nact) {
   const int zc = ymarch_zc(g);
   if (zc == 0) return nullptr;
   DensMaps* m = new (std::nothrow) DensMaps;
   if (!m) return nullptr;
   m->zc = zc;
-  const uint64_t dims[3] = {(uint64_t)2 * g.norb, (uint64_t)g.nz, (uint64_t)g.ndom * g.nx * g.ny};
-  const uint64_t str[2] = {(uint64_t)g.norb * 16, (uint64_t)g.nz * g.norb * 16};
-  const uint32_t b2[3] = {(uint32_t)(2 * g.norb), (uint32_t)zc, 1};
-  const uint32_t b3[3] = {(uint32_t)(2 * g.norb), 1, 1};
-  if (encode_tmap_f64(&m->seg, 3, psi, dims, str, b2) != cudaSuccess ||
-      encode_tmap_f64(&m->one, 3, psi, dims, str, b3) != cudaSuccess) {
+  if (density_maps_encode(m, g, psi, std::min(std::max(nact, 1), g.norb)) != cudaSuccess) {
     delete m;
     return nullptr;
   }
   return m;
+}
+
+cudaError_t density_maps_set_active(DensMaps* m, const Geometry& g, const double2* psi, int nact) {
+  nact = std::min(std::max(nact, 1), g.norb);
+  if (!m || m->nact == nact) return cudaSuccess;
+  return density_maps_encode(m, g, psi, nact);
 }
 
 void density_maps_destroy(DensMaps* m) { delete m; }
@@ -564,9 +578,11 @@ cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps*
   dim3 grid(density_blocks(g), g.ndom);
   if (maps) {
     const int threads = ((maps->zc * kSub + 31) / 32 + 1) * 32;
-    const size_t sm = ymarch_smem(g, maps->zc);
-    if (g.bc == 0 && g.norb == 64)
+    const size_t sm = ymarch_smem(maps->zc, maps->nact);
+    if (g.bc == 0 && maps->nact == 64)
       k_density_y<true, 8><<<grid, threads, sm, st>>>(*maps, g, a);
+    else if (g.bc == 0 && maps->nact == 32)
+      k_density_y<true, 4><<<grid, threads, sm, st>>>(*maps, g, a);
     else if (g.bc == 0)
       k_density_y<true, 0><<<grid, threads, sm, st>>>(*maps, g, a);
     else
@@ -586,7 +602,7 @@ cudaError_t density_set_attributes() {
   cudaError_t e = cudaFuncSetAttribute(k_density_tma, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        density_smem_bytes(kMaxNorbTma));
   if (e != cudaSuccess) return e;
-  for (auto f : {k_density_y<true, 8>, k_density_y<true, 0>, k_density_y<false, 0>}) {
+  for (auto f : {k_density_y<true, 8>, k_density_y<true, 4>, k_density_y<true, 0>, k_density_y<false, 0>}) {
     e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024);
     if (e != cudaSuccess) return e;
   }

@@ -144,7 +144,9 @@ struct DensArgs {
   double* epart;        // [dom][density_blocks][2] per-CTA sums of (kinetic, local) energy densities
 };
 struct DensMaps;  // TMA descriptors of Psi for the y-marching density kernel (dens.cu)
-DensMaps* density_maps_create(const Geometry& g, const double2* psi);  // nullptr: generic kernel
+// nact: active orbitals (1 + last index with f != 0); f = 0 orbitals add exactly zero to rho, j, E
+DensMaps* density_maps_create(const Geometry& g, const double2* psi, int nact);  // nullptr: generic kernel
+cudaError_t density_maps_set_active(DensMaps* m, const Geometry& g, const double2* psi, int nact);
 void density_maps_destroy(DensMaps* m);
 cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps* maps, cudaStream_t st);
 int density_blocks(const Geometry& g);

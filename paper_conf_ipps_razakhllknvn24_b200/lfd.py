@@ -303,6 +303,9 @@ class Context:
     def psi_modified(self):
         lfd_psi_modified(self.ctx)
 
+    def set_occupations(self, occ):
+        lfd_set_occupations(self.ctx, occ)
+
     def sync(self):
         lfd_sync(self.ctx)
 

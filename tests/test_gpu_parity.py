@@ -350,3 +350,35 @@ def test_psi_modified_drops_the_carry():
     ctx.sync()
     assert rel(psi.cpu().numpy(), p) < TOL
     ctx.close()
+
+
+def test_set_occupations_changes_active_orbitals():
+    """The density reads only orbitals up to the last nonzero occupation; lfd_set_occupations moves
+    that bound (here from 20 to all 33 orbitals of P1 and back to 5) and the results follow the
+    oracle's full sums exactly as before."""
+    torch = _torch()
+    from oracle import ref
+    from paper_conf_ipps_razakhllknvn24_b200 import Context
+    w = workload("P1")
+    x = make_inputs(w, seed=43)
+    dev = torch.device("cuda:0")
+    psi = torch.from_numpy(x.psi0.copy()).to(dev)
+    ctx = Context(psi, torch.from_numpy(x.proj).to(dev), x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc)
+    ctx.set_potential(torch.from_numpy(x.vloc).to(dev))
+    A = midpoint_A(w, 0)
+    ctx.set_vector_potential(A)
+    ctx.step(2)
+    cfg = ref.RefConfig(w.ndom, w.nx, w.ny, w.nz, w.hx, w.hy, w.hz, w.bc, w.norb, w.nproj, w.dt)
+    p = x.psi0.copy()
+    ref.step(cfg, p, x.proj, x.dnl, x.vloc, A, 2)
+    rng = np.random.default_rng(1)
+    for occ in (rng.uniform(0.0, 2.0, size=(w.ndom, w.norb)), np.pad(np.full((w.ndom, 5), 2.0), ((0, 0), (0, w.norb - 5))),
+                x.occ):
+        occ = np.ascontiguousarray(occ)
+        ctx.set_occupations(occ)
+        rho, j, J = ctx.density_current()
+        ctx.sync()
+        rr, jr, Jr = ref.density_current(cfg, p, occ, A)
+        assert rel(rho.cpu().numpy().reshape(rr.shape), rr) < TOL
+        assert np.linalg.norm(j.cpu().numpy().reshape(jr.shape) - jr) <= TOL * max(np.linalg.norm(jr), 1e-3 * np.linalg.norm(rr))
+    ctx.close()
