@@ -24,6 +24,9 @@
  *   lfd_ref_kinetic          pinned: plane-wave closed form; O(dt^2) convergence; commutation.
  *   lfd_ref_local            pinned: product of dense expms on a tiny 3-D grid; time reversal.
  *   lfd_ref_nl_half          pinned: norm closed form; Gram closed form; BLAS (numpy) for C.
+ *   lfd_ref_nl_half_exact    pinned: dense scipy expm of -i(Delta/2) B D B^H dV; projector columns get
+ *                            e^{-i(Delta/2)D_u}; span(B)-orthogonal part unchanged; unitary.
+ *   lfd_ref_step_exact       pinned: Gram matrix (orthonormality) conserved for D != 0.
  *   lfd_ref_step             pinned: norm / orthonormality conservation; gauge covariance.
  *   lfd_ref_density_current  pinned: plane-wave closed forms; sum rule; J = dE_kin/dA / V.
  *   lfd_ref_energy           pinned: plane-wave closed forms (kinetic, local = f mean(v)); nonlocal on
@@ -223,6 +226,64 @@ int lfd_ref_nl_half(const lfd_ref_config* c, double complex* psi, const double c
     for (size_t r = 0; r < ng; ++r) psi[r * no + s] *= f;
   }
   free(C); free(n0); free(n1); free(row);
+  return 0;
+}
+
+/* Public: the EXACTLY UNITARY nonlocal factor, for projector
+ * columns that are dV-orthonormal (dV B^H B = I). Then v_nl = B diag(D) B^H dV has the spectral form
+ * sum_u D_u P_u with orthogonal projectors P_u = |B_u><B_u| dV, so the factor of Eq. 6 taken exactly
+ * instead of to first order,  exp(-i (Delta/2) v_nl) = 1 + sum_u (e^{-i (Delta/2) D_u} - 1) P_u,  is
+ *   C_us    = dV sum_r conj(B_ru) Psi_rs
+ *   Psi'_rs = Psi_rs + sum_u B_ru (e^{-i (Delta/2) D_u} - 1) C_us
+ * and needs no renormalisation (the ||.|| denominator of Eq. 6 is 1). One domain (c->ndom ignored). */
+int lfd_ref_nl_half_exact(const lfd_ref_config* c, double complex* psi, const double complex* proj,
+                          const double* dnl) {
+  if (ref_check(c) || !psi) return -1;
+  if (c->nproj == 0) return 0;
+  if (!proj || !dnl) return -1;
+  const size_t ng = (size_t)c->nx * c->ny * c->nz;
+  const int no = c->norb, np = c->nproj;
+  const double dV = c->hx * c->hy * c->hz;
+  const double eps = 0.5 * c->dt;
+  double complex* C = calloc((size_t)np * no, sizeof(double complex));
+  double complex* row = malloc((size_t)no * sizeof(double complex));
+  if (!C || !row) { free(C); free(row); return -2; }
+  for (size_t r = 0; r < ng; ++r)
+    for (int u = 0; u < np; ++u) {
+      double complex bc = conj(proj[r * np + u]);
+      for (int s = 0; s < no; ++s) C[(size_t)u * no + s] += bc * psi[r * no + s];
+    }
+  for (size_t k = 0; k < (size_t)np * no; ++k) C[k] *= dV;
+  for (size_t r = 0; r < ng; ++r) {
+    for (int s = 0; s < no; ++s) row[s] = 0.0;
+    for (int u = 0; u < np; ++u) {
+      double complex b = proj[r * np + u] * (cexp(-I * eps * dnl[u]) - 1.0);
+      for (int s = 0; s < no; ++s) row[s] += b * C[(size_t)u * no + s];
+    }
+    for (int s = 0; s < no; ++s) psi[r * no + s] += row[s];
+  }
+  free(C); free(row);
+  return 0;
+}
+
+/* Public: nsteps LFD steps with the exactly unitary nonlocal factor (N_exact o Local o N_exact). */
+int lfd_ref_step_exact(const lfd_ref_config* c, double complex* psi, const double complex* proj,
+                       const double* dnl, const double* vloc, const double* A, int nsteps) {
+  if (ref_check(c) || !psi || !vloc || !A || nsteps < 0) return -1;
+  if (c->nproj > 0 && (!proj || !dnl)) return -1;
+  const size_t ng = (size_t)c->nx * c->ny * c->nz;
+  lfd_ref_config one = *c;
+  one.ndom = 1;
+  for (int it = 0; it < nsteps; ++it)
+    for (int dm = 0; dm < c->ndom; ++dm) {
+      double complex* p = psi + (size_t)dm * ng * c->norb;
+      const double complex* b = proj ? proj + (size_t)dm * ng * c->nproj : NULL;
+      const double* d = dnl ? dnl + (size_t)dm * c->nproj : NULL;
+      int e = lfd_ref_nl_half_exact(&one, p, b, d);
+      e |= lfd_ref_local(&one, p, vloc + (size_t)dm * ng, A + 3 * dm);
+      e |= lfd_ref_nl_half_exact(&one, p, b, d);
+      if (e) return -1;
+    }
   return 0;
 }
 

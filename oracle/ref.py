@@ -65,6 +65,8 @@ def lib():
         _lib.lfd_ref_local.argtypes = [cfgp, P, P, P]
         _lib.lfd_ref_nl_half.argtypes = [cfgp, P, P, P]
         _lib.lfd_ref_step.argtypes = [cfgp, P, P, P, P, P, C.c_int]
+        _lib.lfd_ref_nl_half_exact.argtypes = [cfgp, P, P, P]
+        _lib.lfd_ref_step_exact.argtypes = [cfgp, P, P, P, P, P, C.c_int]
         _lib.lfd_ref_density_current.argtypes = [cfgp, P, P, P, P, P, P]
         _lib.lfd_ref_kinetic_energy.argtypes = [cfgp, P, P, P]
         _lib.lfd_ref_kinetic_energy.restype = C.c_double
@@ -72,7 +74,8 @@ def lib():
         _lib.lfd_ref_energy.restype = C.c_int
         _lib.lfd_ref_remap_occ.argtypes = [cfgp, P, P, P, C.c_int, P]
         _lib.lfd_ref_remap_occ.restype = C.c_int
-        for f in ("link_sweep", "kinetic", "local", "nl_half", "step", "density_current"):
+        for f in ("link_sweep", "kinetic", "local", "nl_half", "step", "density_current", "nl_half_exact",
+                  "step_exact"):
             getattr(_lib, "lfd_ref_" + f).restype = C.c_int
     return _lib
 
@@ -111,6 +114,23 @@ def nl_half(cfg: RefConfig, psi: np.ndarray, proj: np.ndarray | None, dnl: np.nd
     c = cfg.c()
     _ok(lib().lfd_ref_nl_half(C.byref(c), _ptr(psi, np.complex128), _ptr(proj, np.complex128),
                               _ptr(dnl, np.float64)), "nl_half")
+
+
+def nl_half_exact(cfg: RefConfig, psi: np.ndarray, proj: np.ndarray | None, dnl: np.ndarray | None) -> None:
+    """In place: the exactly unitary nonlocal factor (dV-orthonormal projector columns)."""
+    c = cfg.c()
+    _ok(lib().lfd_ref_nl_half_exact(C.byref(c), _ptr(psi, np.complex128), _ptr(proj, np.complex128),
+                                    _ptr(dnl, np.float64)), "nl_half_exact")
+
+
+def step_exact(cfg: RefConfig, psi: np.ndarray, proj: np.ndarray | None, dnl: np.ndarray | None,
+               vloc: np.ndarray, A: np.ndarray, nsteps: int = 1) -> None:
+    """In place: ``nsteps`` steps N_exact o Local o N_exact of every domain."""
+    c = cfg.c()
+    A = np.ascontiguousarray(A, np.float64)
+    _ok(lib().lfd_ref_step_exact(C.byref(c), _ptr(psi, np.complex128), _ptr(proj, np.complex128),
+                                 _ptr(dnl, np.float64), _ptr(vloc, np.float64), _ptr(A, np.float64), nsteps),
+        "step_exact")
 
 
 def step(cfg: RefConfig, psi: np.ndarray, proj: np.ndarray | None, dnl: np.ndarray | None,

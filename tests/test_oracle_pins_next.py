@@ -100,3 +100,74 @@ def test_remap_on_initial_basis_returns_occupations(seed):
     occ = ref.remap_occ(cfg, p, x.occ, basis)
     assert abs(occ.sum() - x.occ.sum()) < 1e-11
     assert occ[0, 3:].sum() > 0  # light and scissor excite into the unoccupied block
+
+
+# --- exactly unitary nonlocal factor -------------------------------------
+
+def _onb(rng, ng, k, dV):
+    z = rng.standard_normal((ng, k)) + 1j * rng.standard_normal((ng, k))
+    q, _ = np.linalg.qr(z)
+    return q / np.sqrt(dV)
+
+
+def test_exact_nl_equals_dense_matrix_exponential():
+    """N_exact = expm(-i (dt/2) B diag(D) B^H dV) (scipy dense matrix exponential on a tiny grid),
+    for dV-orthonormal B and distinct D_u of both signs; any psi (not only span(B))."""
+    from scipy.linalg import expm
+    rng = np.random.default_rng(31)
+    dims = (4, 4, 2)
+    ng = 32
+    cfg = ref.RefConfig(1, *dims, 0.4, 0.5, 0.6, 0, 3, 4, 0.37)
+    dV = cfg.dV
+    B = _onb(rng, ng, 4, dV)
+    Dn = np.array([0.9, -1.7, 0.35, 2.2])
+    psi = rng.standard_normal((ng, 3)) + 1j * rng.standard_normal((ng, 3))
+    H = (B * Dn) @ B.conj().T * dV
+    want = expm(-1j * 0.5 * cfg.dt * H) @ psi
+    out = np.ascontiguousarray(psi.reshape(dims + (3,)))
+    ref.nl_half_exact(cfg, out, np.ascontiguousarray(B.reshape(dims + (4,))), Dn)
+    assert np.abs(out.reshape(ng, 3) - want).max() < 1e-13 * np.abs(want).max()
+
+
+def test_exact_nl_projector_columns_and_complement():
+    """psi = B_u gets exactly e^{-i (dt/2) D_u} B_u; the part orthogonal to span(B) is unchanged."""
+    rng = np.random.default_rng(32)
+    dims = (4, 2, 4)
+    ng = 32
+    cfg = ref.RefConfig(1, *dims, 0.3, 0.3, 0.3, 0, 3, 3, 0.8)
+    Q = _onb(rng, ng, 6, cfg.dV)
+    B = Q[:, :3]
+    Dn = np.array([0.5, -2.0, 1.25])
+    cols = [2, 0, 1]
+    psi = np.ascontiguousarray(B[:, cols].reshape(dims + (3,)))
+    out = psi.copy()
+    ref.nl_half_exact(cfg, out, np.ascontiguousarray(B.reshape(dims + (3,))), Dn)
+    assert np.abs(out - psi * np.exp(-0.5j * cfg.dt * Dn[cols])).max() < 1e-14
+    perp = np.ascontiguousarray(Q[:, 3:].reshape(dims + (3,)))
+    out = perp.copy()
+    ref.nl_half_exact(cfg, out, np.ascontiguousarray(B.reshape(dims + (3,))), Dn)
+    assert np.abs(out - perp).max() < 1e-14
+
+
+def test_exact_step_conserves_orthonormality_with_scissor():
+    """With the exact factor the whole step is unitary, so dV Psi^H Psi = I is kept for D != 0
+    (the first-order factor of Eq. 6 drifts at O(eps^2) there)."""
+    from lfd_workloads import make_inputs, workload
+    from lfd_workloads.generate import midpoint_A
+    w = workload("P0")
+    x = make_inputs(w, seed=33)
+    cfg = ref.RefConfig(w.ndom, w.nx, w.ny, w.nz, w.hx, w.hy, w.hz, w.bc, w.norb, w.nproj, w.dt)
+    p = x.psi0.copy()
+    q = x.psi0.copy()
+    for n in range(60):
+        A = midpoint_A(w, n)
+        ref.step_exact(cfg, p, x.proj, x.dnl * 20.0, x.vloc, A, 1)
+        ref.step(cfg, q, x.proj, x.dnl * 20.0, x.vloc, A, 1)
+    P = p.reshape(-1, w.norb)
+    Q = q.reshape(-1, w.norb)
+    S_exact = w.dV * P.conj().T @ P
+    S_first = w.dV * Q.conj().T @ Q
+    assert np.abs(S_exact - np.eye(w.norb)).max() < 1e-12
+    # the two factors agree to O(eps^2) per step, and the first-order one loses orthonormality
+    assert np.abs(S_first - np.eye(w.norb)).max() > 1e-8
+    assert np.linalg.norm(p - q) / np.linalg.norm(p) < 1e-2
