@@ -68,6 +68,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--exact-nl", action="store_true",
+                    help="exactly unitary nonlocal factor (LFD_FLAG_EXACT_NL, SURVEY §8(f) rank 4)")
     return ap.parse_args()
 
 
@@ -252,7 +254,8 @@ def main():
     psi = torch.from_numpy(x.psi0).to(dev)
     proj = torch.from_numpy(x.proj).to(dev) if w.nproj else None
     v_dev = torch.from_numpy(x.vloc).to(dev)
-    ctx = Context(psi, proj, x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc)
+    ctx = Context(psi, proj, x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc,
+                  flags=lfd.LFD_FLAG_EXACT_NL if args.exact_nl else 0)
     nd, ng = w.ndom, w.ngrid
     rho = torch.empty((nd, ng), dtype=torch.float64, device=dev)
     J = torch.empty((nd, 3), dtype=torch.float64, device=dev)
@@ -402,6 +405,7 @@ def main():
             "lfd_steps_per_s": world * w.ndom * args.steps / sec,
             "config": {"workload": name, "ndomains_per_gpu": w.ndom, "grid": [w.nx, w.ny, w.nz], "norb": w.norb,
                        "nproj": w.nproj, "bc": "periodic" if w.bc == 0 else "zero", "laser": w.laser,
+                       "nonlocal": "exact-unitary" if args.exact_nl else "eq6-first-order",
                        "ogp_per_step_per_gpu": w.ogp_per_step,
                        "l2": f"inputs exceed L2 (Psi+B = {16 * w.ngrid * (w.norb + w.nproj) * w.ndom / 1e6:.0f} MB "
                              "per GPU vs 126 MB L2); no explicit flush",

@@ -65,7 +65,7 @@ typedef struct {
   int32_t nref_max;    /* max reference-basis columns for lfd_remap_occ, 0..2048 (0: max(norb, nproj)) */
   double dt;           /* Delta_QD [a.u.], finite and nonzero (negative = backward in time) */
   int32_t device;      /* CUDA device ordinal */
-  int32_t flags;       /* 0 or LFD_FLAG_NO_CARRY */
+  int32_t flags;       /* 0 or LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL */
 } lfd_config;
 
 /* lfd_config.flags: disable the projection carry (lfd_step takes the C of each nonlocal factor that
@@ -73,6 +73,11 @@ typedef struct {
  * recomputing dV B^H Psi by GEMM-1). With the flag every factor runs its GEMM-1; results agree to
  * roundoff. */
 #define LFD_FLAG_NO_CARRY 1
+/* lfd_config.flags: the EXACTLY UNITARY nonlocal factor instead of Eq. 6's
+ * renormalised first-order one: for dV-orthonormal projector columns (dV B^H B = I, checked at lfd_init:
+ * LFD_EINVAL otherwise) exp(-i (Delta/2) B diag(D) B^H dV) = 1 + B diag(e^{-i (Delta/2) D} - 1) B^H dV,
+ * which keeps every orbital's norm and the orthonormality of Psi exactly (no renormalisation). */
+#define LFD_FLAG_EXACT_NL 2
 
 /* Kernel classes, for lfd_profile_read(). */
 typedef enum {

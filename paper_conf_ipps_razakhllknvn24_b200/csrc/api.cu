@@ -3,6 +3,7 @@
 // orders them on the context stream. There is no CPU fallback.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
@@ -28,7 +29,7 @@ size_t up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 struct Layout {
   size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage, cref,
-      epart;
+      epart, W, ones;
   int nref_cap;
   size_t total;
   int nsplit;
@@ -61,7 +62,7 @@ lfd_status validate(const lfd_config* c, std::string& why) {
   if (c->norb < 1) { why = "norb must be >= 1"; return LFD_EINVAL; }
   if (c->nproj < 0 || c->nproj > 2048) { why = "nproj must be in [0, 2048]"; return LFD_EINVAL; }
   if (!(c->dt != 0.0) || !std::isfinite(c->dt)) { why = "dt must be finite and nonzero"; return LFD_EINVAL; }
-  if (c->flags & ~LFD_FLAG_NO_CARRY) { why = "unknown flags"; return LFD_EINVAL; }
+  if (c->flags & ~(LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL)) { why = "unknown flags"; return LFD_EINVAL; }
   if (c->nref_max < 0 || c->nref_max > 2048) { why = "nref_max must be in [0, 2048]"; return LFD_EINVAL; }
   const long long ng = (long long)c->nx * c->ny * c->nz;
   if (ng * (long long)std::max(c->norb, std::max(c->nproj, 1)) >= (1LL << 31)) {
@@ -134,6 +135,8 @@ Layout layout(const Geometry& g, int num_sms, int nref_max) {
   L.Jstage = take((size_t)nd * 3 * d8);
   L.cref = take((size_t)nd * std::max(L.nref_cap, np) * no * c16);
   L.epart = take((size_t)nd * lfd::density_blocks(g) * 2 * d8);
+  L.W = take((size_t)2 * nd * np * c16);
+  L.ones = take((size_t)nd * std::max(np, no) * d8);
   L.total = o;
   return L;
 }
@@ -169,6 +172,7 @@ struct lfd_ctx {
   // instead of GEMM-1 (cleared by the local propagator, lfd_psi_modified and LFD_FLAG_NO_CARRY).
   bool c_valid = false;
   bool carry = true;
+  bool exact = false;     // LFD_FLAG_EXACT_NL: exactly unitary nonlocal factor (orthonormal B)
   bool kin_fused = true;  // Phi.K_y K_z in one pass (env LFD_KIN_FUSED=0: separate y and z passes)
   CUtensorMap psi_tmap;   // TMA descriptor of Psi for the fused pass
   lfd::DensMaps* dmaps = nullptr;  // TMA descriptors of Psi for the density kernel
@@ -297,6 +301,11 @@ lfd_status gemm2(lfd_ctx* c) {
   return LFD_OK;
 }
 
+// Exact-factor coefficients: W1 = e^{-i (Delta/2) D} - 1 (one factor), W2 = e^{-i Delta D} - 1 (two merged).
+const double2* exact_w(lfd_ctx* c, bool merged) {
+  return c->at<double2>(c->L.W) + (merged ? (size_t)c->g.ndom * c->g.nproj : 0);
+}
+
 // Eq. 6 nonlocal factor N on every domain (kernels a3, a4, a5); merged = N o N in one pass.
 lfd_status nl_half(lfd_ctx* c, bool merged = false) {
   const Geometry& g = c->g;
@@ -306,9 +315,16 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false) {
     double2* X = c->at<double2>(c->L.cprime);
     double* s = c->at<double>(c->L.s);
     double* nfac = c->at<double>(c->L.nfac);
+    if (c->exact) {  // exactly unitary factor: C_new = C + G X, X = W C_new (n stays 1)
+      LFD_TRY(launch(c, LFD_K_NL_CARRY, "k_nlcarry", [&] {
+        return lfd::launch_nlcarry(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G),
+                                   c->at<double>(c->L.ones), DC, X, s, nfac, false, exact_w(c, merged), c->stream);
+      }));
+      return gemm2(c);
+    }
     LFD_TRY(launch(c, LFD_K_NL_CARRY, "k_nlcarry", [&] {
       return lfd::launch_nlcarry(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), D, DC, X, s, nfac,
-                                 !merged, c->stream);
+                                 !merged, nullptr, c->stream);
     }));
     if (merged)
       LFD_TRY(launch(c, LFD_K_NL_NORM, "k_nlmerge", [&] {
@@ -334,6 +350,12 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false) {
   r.s = c->at<double>(c->L.s);
   r.ndom = g.ndom; r.mrows = g.nproj; r.ncols = g.norb; r.nsplit = c->L.nsplit;
   r.scale = g.dV; r.eps = 0.5 * g.dt;
+  if (c->exact) {  // C (undecorated) and C'' = W C; n == 1 (set at init)
+    r.D = nullptr;
+    r.W = exact_w(c, merged);
+    LFD_TRY(launch(c, LFD_K_NL_REDUCE, "k_reduce", [&] { return lfd::launch_reduce(r, c->stream); }));
+    return gemm2(c);
+  }
   LFD_TRY(launch(c, LFD_K_NL_REDUCE, "k_reduce", [&] { return lfd::launch_reduce(r, c->stream); }));
   if (merged)
     LFD_TRY(launch(c, LFD_K_NL_NORM, "k_nlmerge", [&] {
@@ -519,6 +541,47 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
     r.ndom = g.ndom; r.mrows = g.nproj; r.ncols = g.nproj; r.nsplit = L.nsplit; r.scale = g.dV; r.eps = 0;
     s2 = launch(c, LFD_K_NL_REDUCE, "k_reduce(G)", [&] { return lfd::launch_reduce(r, c->stream); });
     if (s2 != LFD_OK) return bail(s2);
+  }
+  if (cfg->flags & LFD_FLAG_EXACT_NL) {
+    // exactly unitary nonlocal factor: needs dV B^H B = I (checked on G), then
+    // exp(-i (Delta/2) B D B^H dV) = 1 + B diag(e^{-i (Delta/2) D} - 1) B^H dV with n = 1
+    c->exact = true;
+    if (g.nproj > 0) {
+      std::vector<double2> Gh((size_t)g.ndom * g.nproj * g.nproj);
+      e = cudaMemcpyAsync(Gh.data(), c->at<double2>(L.G), Gh.size() * sizeof(double2), cudaMemcpyDeviceToHost,
+                          c->stream);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
+      if (e != cudaSuccess) { cuda_fail(c, e, "copy G"); return bail(LFD_ECUDA); }
+      double dev = 0.0;
+      for (int d = 0; d < g.ndom; ++d)
+        for (int u = 0; u < g.nproj; ++u)
+          for (int v = 0; v < g.nproj; ++v) {
+            const double2 x = Gh[((size_t)d * g.nproj + u) * g.nproj + v];
+            dev = std::max(dev, std::hypot(x.x - (u == v ? 1.0 : 0.0), x.y));
+          }
+      if (dev > 1e-9) {
+        c->err = "LFD_FLAG_EXACT_NL needs dV-orthonormal projector columns (max |dV B^H B - I| = " +
+                 std::to_string(dev) + ")";
+        return bail(LFD_EINVAL);
+      }
+      std::vector<double2> Wh((size_t)2 * g.ndom * g.nproj);
+      for (size_t i = 0; i < (size_t)g.ndom * g.nproj; ++i)
+        for (int k = 0; k < 2; ++k) {  // k = 0: one factor (tau = Delta/2), 1: two merged (tau = Delta)
+          const double ph = -(k + 1) * 0.5 * g.dt * dnl[i];
+          Wh[k * (size_t)g.ndom * g.nproj + i] = make_double2(std::cos(ph) - 1.0, std::sin(ph));
+        }
+      e = cudaMemcpyAsync(c->at<double2>(L.W), Wh.data(), Wh.size() * sizeof(double2), cudaMemcpyHostToDevice,
+                          c->stream);
+      std::vector<double> ones((size_t)g.ndom * std::max(g.nproj, g.norb), 1.0);
+      if (e == cudaSuccess)
+        e = cudaMemcpyAsync(c->at<double>(L.ones), ones.data(), ones.size() * sizeof(double), cudaMemcpyHostToDevice,
+                            c->stream);
+      if (e == cudaSuccess)
+        e = cudaMemcpyAsync(c->at<double>(L.nfac), ones.data(), sizeof(double) * g.ndom * g.norb,
+                            cudaMemcpyHostToDevice, c->stream);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);  // host staging vectors go out of scope
+      if (e != cudaSuccess) { cuda_fail(c, e, "copy exact-factor coefficients"); return bail(LFD_ECUDA); }
+    }
   }
   *out = c;
   return LFD_OK;

@@ -92,6 +92,7 @@ struct ReduceArgs {
   double* s;        // [dom][ncols] or nullptr
   int ndom, mrows, ncols, nsplit;
   double scale, eps;
+  const double2* W = nullptr;  // [dom][mrows]: cprime = W out instead of -i eps out (exact factor)
 };
 cudaError_t launch_reduce(const ReduceArgs& a, cudaStream_t st);
 
@@ -109,8 +110,10 @@ cudaError_t launch_nlmerge(int ndom, int nproj, int norb, double eps, const doub
 // Projection carry after a GEMM-2 Psi <- Psi diag(n) + B X'' (X'' = X diag(n)): DC <- n DC + D (G X'')
 // and X <- -i eps DC (the C' of the next nonlocal factor), in place; column norms s are unchanged.
 // with_norm: also the next factor's n_s (as launch_nlnorm) in the same kernel (nfac is overwritten).
+// W != nullptr (exactly unitary factor; D == 1 and n == 1 passed): X <- W C_new, no norm.
 cudaError_t launch_nlcarry(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
-                           double2* DC, double2* X, const double* s, double* nfac, bool with_norm, cudaStream_t st);
+                           double2* DC, double2* X, const double* s, double* nfac, bool with_norm,
+                           const double2* W, cudaStream_t st);
 
 // GEMM-2 in place: psi[dom][r][n] <- nfac[dom][n] * psi[dom][r][n] + sum_m B[dom][r][m] Cp[dom][m][n]
 // (Cp = C'' = C' diag(n), scaled by the norm / merge / carry kernels)

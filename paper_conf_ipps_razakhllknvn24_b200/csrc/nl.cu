@@ -381,7 +381,14 @@ __global__ void __launch_bounds__(256) k_reduce(ReduceArgs p, int eblocks) {
       const double2 o = make_double2(tr * f, ti * f);
       const long long idx = (long long)dom * per_dom + e;
       p.out[idx] = o;
-      if (p.cprime) p.cprime[idx] = make_double2(p.eps * o.y, -p.eps * o.x);  // -i eps (D C)
+      if (p.cprime) {
+        if (p.W) {  // exactly unitary factor: C'' = (e^{-i eps D_m} - 1) C (W precomputed)
+          const double2 w = p.W[(long long)dom * p.mrows + m];
+          p.cprime[idx] = make_double2(w.x * o.x - w.y * o.y, w.x * o.y + w.y * o.x);
+        } else {
+          p.cprime[idx] = make_double2(p.eps * o.y, -p.eps * o.x);  // -i eps (D C)
+        }
+      }
     }
   } else {
     const int n = ((int)blockIdx.x - eblocks) * 32 + el;
@@ -562,7 +569,8 @@ cudaError_t launch_nlmerge(int ndom, int nproj, int norb, double eps, const doub
 template <bool kNorm>
 __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps, const double2* __restrict__ G,
                                                  const double* __restrict__ D, double2* DC, double2* X,
-                                                 const double* __restrict__ s, double* nfac) {
+                                                 const double* __restrict__ s, double* nfac,
+                                                 const double2* __restrict__ W) {
   extern __shared__ double2 sh[];  // x[np] | dc[np] (dc is overwritten with DC_new)
   double2* xs = sh;
   double2* dcs = sh + nproj;
@@ -601,7 +609,12 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
       const double du = Dd[u];
       const double2 d = make_double2(fma(n, dcs[u].x, du * tr), fma(n, dcs[u].y, du * ti));
       DC[cb + (long long)u * norb] = d;
-      if (!kNorm) X[cb + (long long)u * norb] = make_double2(eps * d.y, -eps * d.x);  // -i eps DC_new
+      if (W) {  // exactly unitary factor (D == 1 passed, n == 1): C''_new = W C_new
+        const double2 w = W[(long long)dom * nproj + u];
+        X[cb + (long long)u * norb] = make_double2(w.x * d.x - w.y * d.y, w.x * d.y + w.y * d.x);
+      } else if (!kNorm) {
+        X[cb + (long long)u * norb] = make_double2(eps * d.y, -eps * d.x);  // -i eps DC_new
+      }
       dcs[u] = d;  // only this lane reads dcs[u] above
     }
   }
@@ -632,12 +645,13 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
 }
 
 cudaError_t launch_nlcarry(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
-                           double2* DC, double2* X, const double* s, double* nfac, bool with_norm, cudaStream_t st) {
+                           double2* DC, double2* X, const double* s, double* nfac, bool with_norm,
+                           const double2* W, cudaStream_t st) {
   dim3 grid(norb, ndom);
-  if (with_norm)
-    k_nlcarry<true><<<grid, 256, 2 * nproj * sizeof(double2), st>>>(nproj, norb, eps, G, D, DC, X, s, nfac);
+  if (with_norm && !W)
+    k_nlcarry<true><<<grid, 256, 2 * nproj * sizeof(double2), st>>>(nproj, norb, eps, G, D, DC, X, s, nfac, W);
   else
-    k_nlcarry<false><<<grid, 256, 2 * nproj * sizeof(double2), st>>>(nproj, norb, eps, G, D, DC, X, s, nfac);
+    k_nlcarry<false><<<grid, 256, 2 * nproj * sizeof(double2), st>>>(nproj, norb, eps, G, D, DC, X, s, nfac, W);
   return cudaGetLastError();
 }
 

@@ -19,6 +19,7 @@ LIB_PATH = os.path.join(HERE, "liblfd.so")
 
 LFD_ABI_VERSION = 3
 LFD_FLAG_NO_CARRY = 1
+LFD_FLAG_EXACT_NL = 2
 LFD_BC_PERIODIC = 0
 LFD_BC_ZERO = 1
 STATUS = {0: "LFD_OK", -1: "LFD_EINVAL", -2: "LFD_ENOMEM", -3: "LFD_ECUDA", -4: "LFD_ESTATE",
