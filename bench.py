@@ -162,6 +162,17 @@ def kernel_work(w):
     }
 
 
+def run_config(w, world, exact):
+    """The `config` object of the JSON line (the same for our arm and the reference arm)."""
+    return {"workload": w.name, "ndomains_per_gpu": w.ndom, "grid": [w.nx, w.ny, w.nz], "norb": w.norb,
+            "nproj": w.nproj, "bc": "periodic" if w.bc == 0 else "zero", "laser": w.laser,
+            "nonlocal": "exact-unitary" if exact else "eq6-first-order",
+            "ogp_per_step_per_gpu": w.ogp_per_step,
+            "l2": f"inputs exceed L2 (Psi+B = {16 * w.ngrid * (w.norb + w.nproj) * w.ndom / 1e6:.0f} MB "
+                  "per GPU vs 126 MB L2); no explicit flush",
+            "parallelism": f"domains{world}" if world > 1 else "single"}
+
+
 def run_reference(args, w, rank, world):
     """--impl reference: the CPU oracle as it stands, on a bounded sample of the same workload."""
     out = {"impl": "reference"}
@@ -199,7 +210,7 @@ def run_reference(args, w, rank, world):
     out.update({"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-                "config": {"workload": w.name, "sample_orbitals": ns},
+                "config": dict(run_config(w, world, exact=False), sample_orbitals=ns),
                 "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
                 "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}})
     return out
@@ -403,13 +414,7 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "lfd_steps_per_s": world * w.ndom * args.steps / sec,
-            "config": {"workload": name, "ndomains_per_gpu": w.ndom, "grid": [w.nx, w.ny, w.nz], "norb": w.norb,
-                       "nproj": w.nproj, "bc": "periodic" if w.bc == 0 else "zero", "laser": w.laser,
-                       "nonlocal": "exact-unitary" if args.exact_nl else "eq6-first-order",
-                       "ogp_per_step_per_gpu": w.ogp_per_step,
-                       "l2": f"inputs exceed L2 (Psi+B = {16 * w.ngrid * (w.norb + w.nproj) * w.ndom / 1e6:.0f} MB "
-                             "per GPU vs 126 MB L2); no explicit flush",
-                       "parallelism": f"domains{world}" if world > 1 else "single"},
+            "config": run_config(w, world, args.exact_nl),
             "gpu_launches": int(launches),
             "clocks": clk.summary(),
             "roofline": roofline,
