@@ -5,5 +5,5 @@ orbitals and projectors, occupations, the laser vector potential). It contains n
 arithmetic (no propagator, no projection, no density) -- see DESIGN.md §5 for the recipe and its
 citations.
 """
-from .configs import WORKLOADS, Workload, workload  # noqa: F401
+from .configs import WORKLOADS, Workload, domain_tiling, workload  # noqa: F401
 from .generate import Inputs, laser_A, make_inputs  # noqa: F401

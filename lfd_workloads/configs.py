@@ -98,3 +98,26 @@ def workload(name: str) -> Workload:
 # C5: nonlocal-projector sweep (GEMM shapes only; Ngrid = 352,800).
 C5_NORB = (32, 64, 128, 256, 512)
 C5_NPROJ = (64, 128, 256, 512, 1024)
+
+
+def domain_tiling(ndom: int, dims) -> tuple:
+    """Place ndom same-shape domains on a global grid (R18: cores tile it, buffer b = 0).
+
+    Domains are laid out as a (px, py, pz) block grid, px * py * pz == ndom, filled x first
+    (ndom = 8 -> 2x2x2 as the 2x2x2 PbTiO3 supercell of C3; 2 -> 2x1x1; 4 -> 2x2x1). Returns
+    (offsets [ndom][3] int32, gdims (GX, GY, GZ)). Pure geometry, no arithmetic of the method.
+    """
+    import numpy as np
+
+    p = [1, 1, 1]
+    n, axis = ndom, 0
+    while n > 1:
+        f = 2 if n % 2 == 0 else n
+        p[axis] *= f
+        n //= f
+        axis = (axis + 1) % 3
+    offsets = np.zeros((ndom, 3), dtype=np.int32)
+    for dm in range(ndom):
+        ix, iy, iz = dm % p[0], (dm // p[0]) % p[1], dm // (p[0] * p[1])
+        offsets[dm] = (ix * dims[0], iy * dims[1], iz * dims[2])
+    return offsets, (p[0] * dims[0], p[1] * dims[1], p[2] * dims[2])
