@@ -68,6 +68,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--no-sc", action="store_true", help="skip the self-consistent-step measurement (sc_mode)")
+    ap.add_argument("--sc-corr", type=int, default=1, help="corrector sweeps of the sc_mode measurement")
     ap.add_argument("--exact-nl", action="store_true",
                     help="exactly unitary nonlocal factor (LFD_FLAG_EXACT_NL, SURVEY §8(f) rank 4)")
     return ap.parse_args()
@@ -236,6 +238,63 @@ def cpu_baseline(w, seed):
             "seconds": dt}
 
 
+def run_sc_mode(args, w, ctx, x, dev, stream, rank, world):
+    import torch
+    import torch.distributed as dist
+    from lfd_workloads import domain_tiling
+    from lfd_workloads.generate import laser_A
+    from paper_conf_ipps_razakhllknvn24_b200 import lfd
+    nd = w.ndom
+    offs_all, gd = domain_tiling(nd * world, (w.nx, w.ny, w.nz))
+    offs = offs_all[rank * nd:(rank + 1) * nd]
+    uid = None
+    if world > 1:
+        obj = [lfd.lfd_comm_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+    steps = min(args.steps, 50)
+    Ah = np.stack([laser_A(w, 0.5 * k * w.dt)[0] for k in range(2 * (args.warmup + steps) + 1)])
+    ctx.psi_modified()
+    ctx.sc_init(gd, offs, torch.from_numpy(x.vloc).to(dev), n_corr=args.sc_corr, Aext0=Ah[0],
+                nranks=world, rank=rank, comm_id=uid)
+    lfd.lfd_sc_step(ctx.ctx, Ah[: 2 * args.warmup + 1])
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    l0 = lfd.lfd_launch_count(ctx.ctx)
+    lfd.lfd_profile_enable(ctx.ctx, True)
+    lfd.lfd_profile_read(ctx.ctx)
+    lfd.lfd_profile_enable(ctx.ctx, False)
+    s0 = torch.cuda.Event(enable_timing=True)
+    s1 = torch.cuda.Event(enable_timing=True)
+    s0.record(stream)
+    lfd.lfd_sc_step(ctx.ctx, Ah[2 * args.warmup: 2 * (args.warmup + steps) + 1])
+    s1.record(stream)
+    torch.cuda.synchronize()
+    launches = lfd.lfd_launch_count(ctx.ctx) - l0
+    t = torch.tensor([s0.elapsed_time(s1)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item())
+    # per-class shares over a second identical run (events around every launch)
+    lfd.lfd_profile_enable(ctx.ctx, True)
+    lfd.lfd_sc_step(ctx.ctx, Ah[2 * args.warmup: 2 * (args.warmup + steps) + 1])
+    prof = lfd.lfd_profile_read(ctx.ctx)
+    lfd.lfd_profile_enable(ctx.ctx, False)
+    tot = sum(v[0] for v in prof.values()) or 1.0
+    st = torch.empty(9, dtype=torch.float64, device=dev)
+    lfd.lfd_sc_read(ctx.ctx, st)
+    torch.cuda.synchronize()
+    return {"value": w.ogp_per_step * world * steps / (ms / 1e3), "unit": UNIT, "ms_per_step": ms / steps,
+            "steps": steps, "n_corr": args.sc_corr, "flags": "hartree+xc+maxwell", "global_grid": list(gd),
+            "launches": int(launches),
+            "shares": {k: round(v[0] / tot, 4) for k, v in prof.items() if v[1]},
+            "A_ind_end": [float(a) for a in st[:3].cpu()],
+            "note": f"lfd_sc_step: {1 + args.sc_corr} propagations + {1 + args.sc_corr} global densities / "
+                    "Hartree (cuFFT) / exchange per QD step, Maxwell Verlet; [rho_g | Jbar] all-reduced over "
+                    "NCCL when world > 1; value counts one physical step (ndom x Ngrid x norb ogp)"}
+
+
 def main():
     args = parse()
     rank = int(os.environ.get("RANK", "0"))
@@ -370,6 +429,16 @@ def main():
                "note": f"lfd_step_sequence of {args.steps} steps (per-step A; N o N merged: {args.steps + 1} "
                        f"projector GEMM pairs instead of {2 * args.steps}), one density at the end"}
 
+    # self-consistent mode (lfd_sc_step): Hartree (cuFFT on the global grid of all
+    # ranks' domains) + LDA exchange + Maxwell, predictor + n_corr corrector sweeps, the [rho_g | Jbar]
+    # SUM all-reduce over NCCL inside the step when world > 1 -- the full LFD subprogram per QD step
+    scm = None
+    if not args.no_sc:
+        try:
+            scm = run_sc_mode(args, w, ctx, x, dev, stream, rank, world)
+        except Exception as ex:  # reported, never fatal for the main measurement
+            scm = {"error": f"{type(ex).__name__}: {ex}"}
+
     # end to end through the C ABI with HOST buffers: pinned v in, pinned rho + J out, every step
     e2e = None
     if not args.no_e2e:
@@ -421,6 +490,7 @@ def main():
             "kernels": kernels,
             "e2e": e2e,
             "sequence_mode": seq,
+            "sc_mode": scm,
             "cpu_baseline": cpu,
         }
         print(json.dumps(out), flush=True)

@@ -38,7 +38,7 @@
 extern "C" {
 #endif
 
-#define LFD_ABI_VERSION 3
+#define LFD_ABI_VERSION 4
 #define LFD_MAX_DOMAINS 4096
 
 typedef struct lfd_ctx lfd_ctx; /* opaque */
@@ -95,7 +95,9 @@ typedef enum {
   LFD_K_ENERGY = 11,   /* NEXT f-1: energy / occupation reductions (calc_energy, remap_occ) */
   LFD_K_NL_CARRY = 12, /* a3/a4: projection carry C_new = (C + G C') diag(n) (replaces GEMM-1) */
   LFD_K_KIN_YZ = 13,   /* a6: K_y K_z . Phi fused in one pass (post-phase fused) */
-  LFD_K_COUNT = 14
+  LFD_K_SC = 14,       /* self-consistent step: Maxwell, potential gather, Poisson filter, v_Hxc */
+  LFD_K_FFT = 15,      /* self-consistent step: cuFFT D2Z / Z2D of the Hartree solve (library kernels) */
+  LFD_K_COUNT = 16
 } lfd_kernel_id;
 
 /* Bytes of DEVICE workspace lfd_init needs for this configuration. */
@@ -180,6 +182,62 @@ lfd_status lfd_energy(lfd_ctx* ctx, double* E);
  *  ref     DEVICE complex128 [ndom][nx][ny][nz][nref], 1 <= nref <= nref_max (config); read-only.
  *  occ_out DEVICE double [ndom][nref]. Stream-ordered. */
 lfd_status lfd_remap_occ(lfd_ctx* ctx, const void* ref, int32_t nref, double* occ_out);
+
+/* ---- Self-consistent LFD step (readings R23-R28 in DESIGN.md §3) -----------------
+ * Eq. 5 puts the Hartree and local xc potentials of the propagated density into v_loc, A_X(alpha)
+ * obeys Maxwell's equation, and each QD step is "self-consistent, time-reversible". With the
+ * SC state initialised, one lfd_sc_step does, for every step n (all on the context stream):
+ *   A: velocity-Verlet half kick and drift of the induced field with Jbar(t_n) (R25/R26),
+ *      A_mid = A_ext(t_n + Delta/2) + (A_ind(t_n) + A_ind(t_n+1)) / 2, A_end = A_ext(t_n+1) + A_ind(t_n+1);
+ *   v: v_loc = v_ion + 3/2 v_Hxc(t_n) - 1/2 v_Hxc(t_n-1) (predictor, R27);
+ *   for k = 0..n_corr: Psi <- Eq.-6 step of Psi(t_n) with (v_loc, A_mid); rho, Jbar of Psi with A_end on the
+ *      GLOBAL grid (domain cores, R18; SUM all-reduce over ranks when nranks > 1); v_Hxc = v_H + v_x (R23,
+ *      R24; Hartree by cuFFT on the global grid); if k < n_corr: v_loc = v_ion + (v_Hxc(t_n) + v_Hxc)/2;
+ *   A: second half kick with Jbar(t_n+1).
+ * Afterwards the context's A (lfd_density_current) is A_end of the last step. */
+#define LFD_SC_HARTREE 1 /* v_H[rho] in v_loc (R23) */
+#define LFD_SC_XC 2      /* LDA exchange v_x[rho] in v_loc (R24) */
+#define LFD_SC_MAXWELL 4 /* induced A_ind from the macroscopic current (R25) */
+
+typedef struct {
+  int32_t flags;            /* LFD_SC_* (0 = v_ion and A_ext only: the plain step with midpoint inputs) */
+  int32_t n_corr;           /* corrector sweeps per step, 0..16 (each re-propagates Psi(t_n) once) */
+  int32_t gdims[3];         /* global grid the domain cores of ALL ranks tile (periodic cell of v_H) */
+  int32_t nranks, rank;     /* processes sharing the global grid (1, 0 for one process) */
+  const int32_t* dom_offset; /* HOST [ndom][3] global offsets of this context's domains (copied) */
+} lfd_sc_config;
+
+/* Bytes of DEVICE workspace lfd_sc_init needs (includes a copy of Psi when n_corr > 0 and the cuFFT
+ * work area; the library allocates nothing). */
+lfd_status lfd_sc_workspace_size(const lfd_ctx* ctx, const lfd_sc_config* sc, size_t* bytes);
+
+/* Initialise the SC state at t_0 from the current Psi: rho(t_0), Jbar(t_0) with A(t_0) = Aext0 + A_ind0,
+ * v_Hxc(t_0) (= v_Hxc(t_-1)).
+ *  vion    DEVICE double [ndom][nx][ny][nz] local pseudopotential (borrowed, read every step), or NULL = 0
+ *  ws      DEVICE >= lfd_sc_workspace_size bytes, 256-byte aligned (borrowed until lfd_destroy)
+ *  Aext0   HOST double[3]; A_ind0, Adot0 HOST double[3] or NULL (= 0)
+ * With nranks == 1 the domains must tile gdims exactly; with nranks > 1 lfd_sc_comm_init must come first
+ * (each rank's domains must lie inside gdims without overlap; the ranks together must tile it).
+ * Errors: LFD_EINVAL (config), LFD_ENOMEM (ws too small), LFD_ESTATE (nranks > 1 without a communicator),
+ * LFD_ECUDA / LFD_EUNSUPPORTED (cuFFT / NCCL failures). Calling it again re-initialises. */
+lfd_status lfd_sc_init(lfd_ctx* ctx, const lfd_sc_config* sc, const double* vion, void* ws, size_t ws_bytes,
+                       const double* Aext0, const double* A_ind0, const double* Adot0);
+
+/* Enqueue nsteps self-consistent steps. Aext HOST double [2*nsteps+1][3]: A_ext at t_n, t_n + Delta/2,
+ * t_n+1, ... (R28), one vector for all domains; captured by value. */
+lfd_status lfd_sc_step(lfd_ctx* ctx, int32_t nsteps, const double* Aext);
+
+/* Copy the SC state out (stream-ordered, DEVICE pointers, each may be NULL):
+ *  state DEVICE double[9] = {A_ind[3], dA_ind/dt[3], Jbar[3]} at the current time,
+ *  rho_g DEVICE double [GX][GY][GZ] global density, vhxc DEVICE double [GX][GY][GZ] v_Hxc(t_n). */
+lfd_status lfd_sc_read(lfd_ctx* ctx, double* state, double* rho_g, double* vhxc);
+
+/* Multi-process SC: lfd_comm_unique_id fills 128 bytes on ONE rank (broadcast them to the others, e.g.
+ * with torch.distributed); every rank then calls lfd_sc_comm_init with the same bytes. The library loads
+ * NCCL (libnccl.so.2) at this call and all-reduces the [rho_g | Jbar] buffer over it on the context stream.
+ * LFD_EUNSUPPORTED if NCCL cannot be loaded. */
+lfd_status lfd_comm_unique_id(void* id128);
+lfd_status lfd_sc_comm_init(lfd_ctx* ctx, int32_t nranks, int32_t rank, const void* id128);
 
 /* Tell the context that the caller wrote psi (drops the kept projection; the next nonlocal factor
  * recomputes C = dV B^H Psi by GEMM-1). */

@@ -2,6 +2,8 @@
 // Every numerical step runs in the sm_100a kernels of kin.cu / nl.cu / dens.cu; this file only
 // orders them on the context stream. There is no CPU fallback.
 #include <cuda_runtime.h>
+#include <cufft.h>
+#include <dlfcn.h>
 
 #include <algorithm>
 #include <cmath>
@@ -152,6 +154,75 @@ struct ProfSlot {
   cudaEvent_t a, b;
 };
 
+// ---- self-consistent step state (lfd_sc_*; sc.cu) ----------------------------------------------------
+// Minimal NCCL declarations (the library is loaded with dlopen at lfd_sc_comm_init; no link dependency).
+typedef struct {
+  char internal[128];
+} nccl_unique_id;
+typedef void* nccl_comm;
+typedef int (*nccl_get_unique_id_fn)(nccl_unique_id*);
+typedef int (*nccl_comm_init_rank_fn)(nccl_comm*, int, nccl_unique_id, int);
+typedef int (*nccl_all_reduce_fn)(const void*, void*, size_t, int, int, nccl_comm, cudaStream_t);
+typedef int (*nccl_comm_destroy_fn)(nccl_comm);
+typedef const char* (*nccl_error_string_fn)(int);
+constexpr int kNcclFloat64 = 8, kNcclSum = 0;
+
+struct Nccl {
+  void* h = nullptr;
+  nccl_get_unique_id_fn get_unique_id = nullptr;
+  nccl_comm_init_rank_fn comm_init_rank = nullptr;
+  nccl_all_reduce_fn all_reduce = nullptr;
+  nccl_comm_destroy_fn comm_destroy = nullptr;
+  nccl_error_string_fn error_string = nullptr;
+};
+
+const Nccl* nccl_load(std::string& why) {
+  static Nccl n;
+  static bool tried = false;
+  static std::mutex mu;
+  std::lock_guard<std::mutex> lk(mu);
+  if (!tried) {
+    tried = true;
+    n.h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (n.h) {
+      n.get_unique_id = (nccl_get_unique_id_fn)dlsym(n.h, "ncclGetUniqueId");
+      n.comm_init_rank = (nccl_comm_init_rank_fn)dlsym(n.h, "ncclCommInitRank");
+      n.all_reduce = (nccl_all_reduce_fn)dlsym(n.h, "ncclAllReduce");
+      n.comm_destroy = (nccl_comm_destroy_fn)dlsym(n.h, "ncclCommDestroy");
+      n.error_string = (nccl_error_string_fn)dlsym(n.h, "ncclGetErrorString");
+    }
+  }
+  if (!n.h || !n.get_unique_id || !n.comm_init_rank || !n.all_reduce || !n.comm_destroy) {
+    why = std::string("NCCL (libnccl.so.2) could not be loaded: ") + (n.h ? "missing symbols" : dlerror() ? dlerror() : "dlopen failed");
+    return nullptr;
+  }
+  return &n;
+}
+
+struct ScLayout {
+  size_t pack, vh0, vh1, vh2, spec, state, coef_end, gbase, off, jtmp, snap_dc, snap_cp, snap_s, snap_n, fftwork,
+      psi_save, total;
+  size_t fft_bytes;
+};
+
+struct ScState {
+  bool ready = false;
+  int flags = 0, n_corr = 0, nranks = 1, rank = 0;
+  int gd[3] = {0, 0, 0};
+  long long GN = 0;
+  ScLayout L{};
+  char* ws = nullptr;
+  const double* vion = nullptr;
+  int vi[3] = {0, 1, 2};  // rotation of the three global v_Hxc buffers: [t_n, t_n-1, new]
+  cufftHandle plan_f = 0, plan_b = 0;
+  bool plans = false;
+  nccl_comm comm = nullptr;
+  int comm_nranks = 1, comm_rank = 0;
+  template <class T>
+  T* at(size_t off) const { return reinterpret_cast<T*>(ws + off); }
+  double* vh(int k) const { return at<double>(k == 0 ? L.vh0 : k == 1 ? L.vh1 : L.vh2); }
+};
+
 }  // namespace
 
 struct lfd_ctx {
@@ -186,6 +257,7 @@ struct lfd_ctx {
   size_t nslot = 0;
   double prof_ms[LFD_K_COUNT] = {0};
   int64_t prof_n[LFD_K_COUNT] = {0};
+  ScState sc;  // self-consistent step (lfd_sc_*)
 
   template <class T>
   T* at(size_t off) const { return reinterpret_cast<T*>(ws + off); }
@@ -412,9 +484,9 @@ lfd_status set_A(lfd_ctx* c, const double* A) {
 }
 
 lfd_status density_into(lfd_ctx* c, double* rho, double* j, double* Jmac, const long long* base_dev, long long sx,
-                        long long sy, long long jstride, bool energy = false) {
+                        long long sy, long long jstride, bool energy = false, const DomCoef* coef = nullptr) {
   lfd::DensArgs a;
-  a.psi = c->psi; a.coef = c->coef(); a.occ = c->at<double>(c->L.occ);
+  a.psi = c->psi; a.coef = coef ? coef : c->coef(); a.occ = c->at<double>(c->L.occ);
   a.rho = rho; a.j = j; a.jline = c->at<double>(c->L.jline);
   a.base = base_dev; a.jbase = base_dev + c->g.ndom; a.sx = sx; a.sy = sy; a.jstride = jstride;
   a.v = energy ? c->at<double>(c->L.vstage) : nullptr;
@@ -424,6 +496,158 @@ lfd_status density_into(lfd_ctx* c, double* rho, double* j, double* Jmac, const 
     LFD_TRY(launch(c, LFD_K_JREDUCE, "k_jreduce",
                    [&] { return lfd::launch_jreduce(c->g, a.jline, Jmac, c->stream); }));
   return LFD_OK;
+}
+
+
+// ---- self-consistent step helpers --------------------------------------------------------------------
+lfd_status sc_validate(const lfd_ctx* c, const lfd_sc_config* sc, std::string& why) {
+  if (!sc) { why = "sc config is NULL"; return LFD_EINVAL; }
+  if (sc->flags & ~(LFD_SC_HARTREE | LFD_SC_XC | LFD_SC_MAXWELL)) { why = "unknown SC flags"; return LFD_EINVAL; }
+  if (sc->n_corr < 0 || sc->n_corr > 16) { why = "n_corr must be in [0, 16]"; return LFD_EINVAL; }
+  for (int i = 0; i < 3; ++i)
+    if (sc->gdims[i] < 1) { why = "gdims must be >= 1"; return LFD_EINVAL; }
+  if (sc->nranks < 1 || sc->rank < 0 || sc->rank >= sc->nranks) { why = "bad nranks / rank"; return LFD_EINVAL; }
+  if (!sc->dom_offset) { why = "dom_offset is NULL"; return LFD_EINVAL; }
+  const Geometry& g = c->g;
+  const long long GN = (long long)sc->gdims[0] * sc->gdims[1] * sc->gdims[2];
+  if (GN >= (1LL << 31)) { why = "global grid too large"; return LFD_EINVAL; }
+  const int nd[3] = {g.nx, g.ny, g.nz};
+  for (int d = 0; d < g.ndom; ++d)
+    for (int i = 0; i < 3; ++i)
+      if (sc->dom_offset[3 * d + i] < 0 || sc->dom_offset[3 * d + i] + nd[i] > sc->gdims[i]) {
+        why = "domain core outside the global grid";
+        return LFD_EINVAL;
+      }
+  for (int a = 0; a < g.ndom; ++a)  // own cores must not overlap (boxes of equal shape)
+    for (int b = a + 1; b < g.ndom; ++b) {
+      bool sep = false;
+      for (int i = 0; i < 3; ++i)
+        sep = sep || std::abs(sc->dom_offset[3 * a + i] - sc->dom_offset[3 * b + i]) >= nd[i];
+      if (!sep) { why = "domain cores overlap"; return LFD_EINVAL; }
+    }
+  if (sc->nranks == 1 && (long long)g.ndom * g.ng != GN) {
+    why = "with nranks == 1 the domain cores must tile gdims exactly";
+    return LFD_EINVAL;
+  }
+  return LFD_OK;
+}
+
+cudaError_t fft_work_bytes(const int* gd, size_t* bytes) {
+  size_t wf = 0, wb = 0;
+  cufftHandle pf, pb;
+  if (cufftCreate(&pf) != CUFFT_SUCCESS) return cudaErrorUnknown;
+  if (cufftCreate(&pb) != CUFFT_SUCCESS) { cufftDestroy(pf); return cudaErrorUnknown; }
+  cufftSetAutoAllocation(pf, 0);
+  cufftSetAutoAllocation(pb, 0);
+  cufftResult r1 = cufftMakePlan3d(pf, gd[0], gd[1], gd[2], CUFFT_D2Z, &wf);
+  cufftResult r2 = cufftMakePlan3d(pb, gd[0], gd[1], gd[2], CUFFT_Z2D, &wb);
+  cufftDestroy(pf);
+  cufftDestroy(pb);
+  if (r1 != CUFFT_SUCCESS || r2 != CUFFT_SUCCESS) return cudaErrorUnknown;
+  *bytes = std::max(wf, wb);
+  return cudaSuccess;
+}
+
+ScLayout sc_layout(const Geometry& g, const lfd_sc_config* sc, size_t fft_bytes) {
+  ScLayout L{};
+  const long long GN = (long long)sc->gdims[0] * sc->gdims[1] * sc->gdims[2];
+  const long long GH = (long long)sc->gdims[0] * sc->gdims[1] * (sc->gdims[2] / 2 + 1);
+  const size_t d8 = 8, c16 = 16;
+  size_t o = 0;
+  auto take = [&](size_t bytes) { size_t at = o; o += up(std::max<size_t>(bytes, 1)); return at; };
+  L.pack = take((size_t)(GN + 3) * d8);
+  L.vh0 = take((size_t)GN * d8);
+  L.vh1 = take((size_t)GN * d8);
+  L.vh2 = take((size_t)GN * d8);
+  L.spec = take((size_t)GH * c16);
+  L.state = take(32 * d8);
+  L.coef_end = take((size_t)g.ndom * sizeof(DomCoef));
+  L.gbase = take((size_t)2 * g.ndom * sizeof(long long));
+  L.off = take((size_t)3 * g.ndom * sizeof(int));
+  L.jtmp = take((size_t)3 * g.ndom * d8);
+  L.snap_dc = take((size_t)g.ndom * g.nproj * g.norb * c16);
+  L.snap_cp = take((size_t)g.ndom * g.nproj * g.norb * c16);
+  L.snap_s = take((size_t)g.ndom * g.norb * d8);
+  L.snap_n = take((size_t)g.ndom * g.norb * d8);
+  L.fft_bytes = fft_bytes;
+  L.fftwork = take(fft_bytes);
+  L.psi_save = sc->n_corr > 0 ? take((size_t)g.ndom * g.ng * g.norb * c16) : 0;
+  L.total = o;
+  return L;
+}
+
+// Eq.-6 step of every domain with the context's current Phi and coefficients.
+lfd_status one_step(lfd_ctx* c) {
+  if (c->g.nproj > 0) LFD_TRY(nl_half(c));
+  LFD_TRY(local_prop(c));
+  if (c->g.nproj > 0) LFD_TRY(nl_half(c));
+  return LFD_OK;
+}
+
+// rho (global layout) and this rank's Jbar share into the pack buffer; SUM all-reduce over ranks.
+lfd_status sc_density(lfd_ctx* c) {
+  ScState& S = c->sc;
+  const Geometry& g = c->g;
+  double* pack = S.at<double>(S.L.pack);
+  if (S.comm) {
+    cudaError_t e = cudaMemsetAsync(pack, 0, sizeof(double) * (S.GN + 3), c->stream);
+    if (e != cudaSuccess) return cuda_fail(c, e, "memset rho_g");
+  }
+  LFD_TRY(density_into(c, pack, nullptr, S.at<double>(S.L.jtmp), S.at<long long>(S.L.gbase),
+                       (long long)S.gd[1] * S.gd[2], S.gd[2], S.GN, false, S.at<DomCoef>(S.L.coef_end)));
+  LFD_TRY(launch(c, LFD_K_SC, "k_sc_jbar", [&] {
+    return lfd::launch_sc_jbar(S.at<double>(S.L.jtmp), g.ndom, (double)g.ng / (double)S.GN, pack + S.GN, c->stream);
+  }));
+  if (S.comm) {  // the communicator of lfd_sc_comm_init (also used with nranks == 1 when set)
+    std::string why;
+    const Nccl* n = nccl_load(why);
+    if (!n) return fail(c, LFD_EUNSUPPORTED, why);
+    int r = n->all_reduce(pack, pack, (size_t)(S.GN + 3), kNcclFloat64, kNcclSum, S.comm, c->stream);
+    if (r != 0) return fail(c, LFD_ECUDA, std::string("ncclAllReduce: ") + (n->error_string ? n->error_string(r) : "error"));
+  }
+  return LFD_OK;
+}
+
+// v_Hxc[rho_g] into the global buffer `out` (R23 Hartree by cuFFT, R24 exchange).
+lfd_status sc_vhxc(lfd_ctx* c, double* out) {
+  ScState& S = c->sc;
+  const double* rho = S.at<double>(S.L.pack);
+  const bool H = S.flags & LFD_SC_HARTREE, X = S.flags & LFD_SC_XC;
+  if (H) {
+    double2* spec = S.at<double2>(S.L.spec);
+    cufftSetStream(S.plan_f, c->stream);
+    cufftSetStream(S.plan_b, c->stream);
+    LFD_TRY(launch(c, LFD_K_FFT, "cufftExecD2Z", [&] {
+      return cufftExecD2Z(S.plan_f, const_cast<double*>(rho), reinterpret_cast<cufftDoubleComplex*>(spec)) == CUFFT_SUCCESS
+                 ? cudaGetLastError() : cudaErrorUnknown;
+    }));
+    LFD_TRY(launch(c, LFD_K_SC, "k_sc_poisson", [&] { return lfd::launch_sc_poisson(spec, S.gd, c->g, c->stream); }));
+    LFD_TRY(launch(c, LFD_K_FFT, "cufftExecZ2D", [&] {
+      return cufftExecZ2D(S.plan_b, reinterpret_cast<cufftDoubleComplex*>(spec), out) == CUFFT_SUCCESS
+                 ? cudaGetLastError() : cudaErrorUnknown;
+    }));
+  }
+  return launch(c, LFD_K_SC, "k_sc_vhxc", [&] { return lfd::launch_sc_vhxc(rho, out, S.GN, H, X, c->stream); });
+}
+
+// v_loc = v_ion + wa va + wb vb (global buffers gathered per domain point), then Phi.
+lfd_status sc_set_v(lfd_ctx* c, const double* va, double wa, const double* vb, double wb) {
+  ScState& S = c->sc;
+  double* vst = c->at<double>(c->L.vstage);
+  LFD_TRY(launch(c, LFD_K_SC, "k_sc_vmid", [&] {
+    return lfd::launch_sc_vmid(c->g, S.vion, va, vb, wa, wb, S.at<int>(S.L.off), S.gd[1], S.gd[2], vst, c->stream);
+  }));
+  return launch(c, LFD_K_PHASE, "k_phase",
+                [&] { return lfd::launch_phase(c->g, vst, c->phi(), vst, c->scaled, c->stream); });
+}
+
+void sc_release(ScState& S) {
+  if (S.plans) {
+    cufftDestroy(S.plan_f);
+    cufftDestroy(S.plan_b);
+    S.plans = false;
+  }
+  S.ready = false;
 }
 
 }  // namespace
@@ -752,6 +976,224 @@ lfd_status lfd_set_occupations(lfd_ctx* c, const double* occ) {
   return LFD_OK;
 }
 
+lfd_status lfd_sc_workspace_size(const lfd_ctx* c, const lfd_sc_config* sc, size_t* bytes) {
+  LFD_TRY(check_ctx(c));
+  std::string why;
+  lfd_status st = sc_validate(c, sc, why);
+  if (st != LFD_OK) return fail(const_cast<lfd_ctx*>(c), st, why);
+  if (!bytes) return fail(const_cast<lfd_ctx*>(c), LFD_EINVAL, "bytes is NULL");
+  DeviceGuard dg(c->device);
+  size_t fb = 0;
+  if (fft_work_bytes(sc->gdims, &fb) != cudaSuccess) return fail(const_cast<lfd_ctx*>(c), LFD_ECUDA, "cuFFT plan failed");
+  *bytes = sc_layout(c->g, sc, fb).total;
+  return LFD_OK;
+}
+
+lfd_status lfd_sc_init(lfd_ctx* c, const lfd_sc_config* sc, const double* vion, void* ws, size_t ws_bytes,
+                       const double* Aext0, const double* A_ind0, const double* Adot0) {
+  LFD_TRY(check_ctx(c));
+  std::string why;
+  lfd_status st = sc_validate(c, sc, why);
+  if (st != LFD_OK) return fail(c, st, why);
+  if (!ws || !Aext0) return fail(c, LFD_EINVAL, "ws and Aext0 must be non-NULL");
+  if (reinterpret_cast<uintptr_t>(ws) & (kAlign - 1)) return fail(c, LFD_EINVAL, "ws must be 256-byte aligned");
+  for (int i = 0; i < 3; ++i)
+    if (!std::isfinite(Aext0[i]) || (A_ind0 && !std::isfinite(A_ind0[i])) || (Adot0 && !std::isfinite(Adot0[i])))
+      return fail(c, LFD_EINVAL, "Aext0 / A_ind0 / Adot0 must be finite");
+  if ((sc->nranks > 1 || c->sc.comm) &&
+      (!c->sc.comm || c->sc.comm_nranks != sc->nranks || c->sc.comm_rank != sc->rank))
+    return fail(c, LFD_ESTATE, "nranks > 1 needs lfd_sc_comm_init with the same nranks / rank first");
+  DeviceGuard dg(c->device);
+  if (!is_device_ptr(ws) || (vion && !is_device_ptr(vion))) return fail(c, LFD_EINVAL, "ws / vion must be device memory");
+  size_t fb = 0;
+  if (fft_work_bytes(sc->gdims, &fb) != cudaSuccess) return fail(c, LFD_ECUDA, "cuFFT plan failed");
+  const ScLayout L = sc_layout(c->g, sc, fb);
+  if (ws_bytes < L.total) return fail(c, LFD_ENOMEM, "SC workspace smaller than lfd_sc_workspace_size()");
+  ScState& S = c->sc;
+  sc_release(S);
+  S.flags = sc->flags; S.n_corr = sc->n_corr; S.nranks = sc->nranks; S.rank = sc->rank;
+  for (int i = 0; i < 3; ++i) S.gd[i] = sc->gdims[i];
+  S.GN = (long long)S.gd[0] * S.gd[1] * S.gd[2];
+  S.L = L; S.ws = static_cast<char*>(ws); S.vion = vion;
+  S.vi[0] = 0; S.vi[1] = 1; S.vi[2] = 2;
+  // cuFFT plans on the caller's workspace (the library allocates nothing)
+  size_t w1 = 0, w2 = 0;
+  if (cufftCreate(&S.plan_f) != CUFFT_SUCCESS) return fail(c, LFD_ECUDA, "cufftCreate");
+  if (cufftCreate(&S.plan_b) != CUFFT_SUCCESS) { cufftDestroy(S.plan_f); return fail(c, LFD_ECUDA, "cufftCreate"); }
+  S.plans = true;
+  cufftSetAutoAllocation(S.plan_f, 0);
+  cufftSetAutoAllocation(S.plan_b, 0);
+  if (cufftMakePlan3d(S.plan_f, S.gd[0], S.gd[1], S.gd[2], CUFFT_D2Z, &w1) != CUFFT_SUCCESS ||
+      cufftMakePlan3d(S.plan_b, S.gd[0], S.gd[1], S.gd[2], CUFFT_Z2D, &w2) != CUFFT_SUCCESS ||
+      cufftSetWorkArea(S.plan_f, S.at<void>(L.fftwork)) != CUFFT_SUCCESS ||
+      cufftSetWorkArea(S.plan_b, S.at<void>(L.fftwork)) != CUFFT_SUCCESS) {
+    sc_release(S);
+    return fail(c, LFD_ECUDA, "cuFFT plan setup failed");
+  }
+  // host-side tables: global output bases of the domain cores and their offsets
+  const Geometry& g = c->g;
+  std::vector<long long> base(2 * g.ndom);
+  std::vector<int> off(3 * g.ndom);
+  for (int d = 0; d < g.ndom; ++d) {
+    for (int i = 0; i < 3; ++i) off[3 * d + i] = sc->dom_offset[3 * d + i];
+    base[d] = ((long long)off[3 * d] * S.gd[1] + off[3 * d + 1]) * S.gd[2] + off[3 * d + 2];
+    base[g.ndom + d] = base[d];
+  }
+  double st0[32] = {0};
+  for (int i = 0; i < 3; ++i) {
+    st0[i] = A_ind0 ? A_ind0[i] : 0.0;
+    st0[3 + i] = Adot0 ? Adot0[i] : 0.0;
+  }
+  cudaError_t e = cudaMemcpyAsync(S.at<long long>(L.gbase), base.data(), sizeof(long long) * base.size(),
+                                  cudaMemcpyHostToDevice, c->stream);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(S.at<int>(L.off), off.data(), sizeof(int) * off.size(), cudaMemcpyHostToDevice, c->stream);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(S.at<double>(L.state), st0, sizeof(st0), cudaMemcpyHostToDevice, c->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);  // host staging goes out of scope
+  if (e != cudaSuccess) { sc_release(S); return cuda_fail(c, e, "SC init copies"); }
+  // state at t_0: coefficients of A(t_0) = A_ext(t_0) + A_ind(t_0), rho, Jbar, v_Hxc(t_0) = v_Hxc(t_-1)
+  const double A0[3] = {Aext0[0] + st0[0], Aext0[1] + st0[1], Aext0[2] + st0[2]};
+  double* state = S.at<double>(L.state);
+  lfd_status r = launch(c, LFD_K_SC, "k_sc_maxwell_begin", [&] {
+    return lfd::launch_sc_maxwell_begin(state, A0, A0, g.dt, false, g, c->coef(), S.at<DomCoef>(L.coef_end), c->stream);
+  });
+  if (r == LFD_OK) r = sc_density(c);
+  if (r == LFD_OK) r = sc_vhxc(c, S.vh(S.vi[0]));
+  if (r == LFD_OK) {
+    e = cudaMemcpyAsync(S.vh(S.vi[1]), S.vh(S.vi[0]), sizeof(double) * S.GN, cudaMemcpyDeviceToDevice, c->stream);
+    if (e != cudaSuccess) r = cuda_fail(c, e, "copy v_Hxc");
+  }
+  if (r == LFD_OK)
+    r = launch(c, LFD_K_SC, "k_sc_maxwell_end", [&] {
+      return lfd::launch_sc_maxwell_end(state, S.at<double>(L.pack) + S.GN, g.dt, false, c->stream);
+    });
+  if (r != LFD_OK) { sc_release(S); return r; }
+  S.ready = true;
+  return LFD_OK;
+}
+
+lfd_status lfd_sc_step(lfd_ctx* c, int32_t nsteps, const double* Aext) {
+  LFD_TRY(check_ctx(c));
+  ScState& S = c->sc;
+  if (!S.ready) return fail(c, LFD_ESTATE, "lfd_sc_init has not been called");
+  if (nsteps < 0) return fail(c, LFD_EINVAL, "nsteps must be >= 0");
+  if (nsteps == 0) return LFD_OK;
+  if (!Aext) return fail(c, LFD_EINVAL, "Aext is NULL");
+  for (long long i = 0; i < 3LL * (2LL * nsteps + 1); ++i)
+    if (!std::isfinite(Aext[i])) return fail(c, LFD_EINVAL, "Aext must be finite");
+  DeviceGuard dg(c->device);
+  const Geometry& g = c->g;
+  const bool maxwell = S.flags & LFD_SC_MAXWELL;
+  double* state = S.at<double>(S.L.state);
+  const size_t psi_bytes = (size_t)g.ndom * g.ng * g.norb * 16;
+  const size_t cbytes = (size_t)g.ndom * g.nproj * g.norb * 16, nbytes = (size_t)g.ndom * g.norb * 8;
+  auto cpy = [&](void* dst, const void* src, size_t n) -> lfd_status {
+    cudaError_t e = cudaMemcpyAsync(dst, src, n, cudaMemcpyDeviceToDevice, c->stream);
+    return e == cudaSuccess ? LFD_OK : cuda_fail(c, e, "SC device copy");
+  };
+  for (int n = 0; n < nsteps; ++n) {
+    const double* a_mid = Aext + 3 * (2 * n + 1);
+    const double* a_end = Aext + 3 * (2 * n + 2);
+    LFD_TRY(launch(c, LFD_K_SC, "k_sc_maxwell_begin", [&] {
+      return lfd::launch_sc_maxwell_begin(state, a_mid, a_end, g.dt, maxwell, g, c->coef(), S.at<DomCoef>(S.L.coef_end),
+                                          c->stream);
+    }));
+    double* vn = S.vh(S.vi[0]);
+    double* vp = S.vh(S.vi[1]);
+    double* vnew = S.vh(S.vi[2]);
+    LFD_TRY(sc_set_v(c, vn, 1.5, vp, -0.5));  // predictor (R27)
+    bool snap_valid = false;
+    if (S.n_corr > 0) {
+      LFD_TRY(cpy(S.at<void>(S.L.psi_save), c->psi, psi_bytes));
+      snap_valid = c->c_valid;
+      if (snap_valid) {  // the projection carry of Psi(t_n), reused by every sweep
+        LFD_TRY(cpy(S.at<void>(S.L.snap_dc), c->at<void>(c->L.dc), cbytes));
+        LFD_TRY(cpy(S.at<void>(S.L.snap_cp), c->at<void>(c->L.cprime), cbytes));
+        LFD_TRY(cpy(S.at<void>(S.L.snap_s), c->at<void>(c->L.s), nbytes));
+        LFD_TRY(cpy(S.at<void>(S.L.snap_n), c->at<void>(c->L.nfac), nbytes));
+      }
+    }
+    for (int k = 0; k <= S.n_corr; ++k) {
+      if (k > 0) {
+        LFD_TRY(cpy(c->psi, S.at<void>(S.L.psi_save), psi_bytes));
+        c->c_valid = snap_valid;
+        if (snap_valid) {
+          LFD_TRY(cpy(c->at<void>(c->L.dc), S.at<void>(S.L.snap_dc), cbytes));
+          LFD_TRY(cpy(c->at<void>(c->L.cprime), S.at<void>(S.L.snap_cp), cbytes));
+          LFD_TRY(cpy(c->at<void>(c->L.s), S.at<void>(S.L.snap_s), nbytes));
+          LFD_TRY(cpy(c->at<void>(c->L.nfac), S.at<void>(S.L.snap_n), nbytes));
+        }
+      }
+      LFD_TRY(one_step(c));
+      LFD_TRY(sc_density(c));
+      LFD_TRY(sc_vhxc(c, vnew));
+      if (k < S.n_corr) LFD_TRY(sc_set_v(c, vn, 0.5, vnew, 0.5));  // corrector (R27)
+    }
+    LFD_TRY(launch(c, LFD_K_SC, "k_sc_maxwell_end", [&] {
+      return lfd::launch_sc_maxwell_end(state, S.at<double>(S.L.pack) + S.GN, g.dt, maxwell, c->stream);
+    }));
+    const int old_prev = S.vi[1];
+    S.vi[1] = S.vi[0];
+    S.vi[0] = S.vi[2];
+    S.vi[2] = old_prev;
+  }
+  // the context's A is now A(t_end): the density / energy calls use its coefficients
+  return cpy(c->coef(), S.at<void>(S.L.coef_end), sizeof(DomCoef) * g.ndom);
+}
+
+lfd_status lfd_sc_read(lfd_ctx* c, double* state, double* rho_g, double* vhxc) {
+  LFD_TRY(check_ctx(c));
+  ScState& S = c->sc;
+  if (!S.ready) return fail(c, LFD_ESTATE, "lfd_sc_init has not been called");
+  DeviceGuard dg(c->device);
+  if ((state && !is_device_ptr(state)) || (rho_g && !is_device_ptr(rho_g)) || (vhxc && !is_device_ptr(vhxc)))
+    return fail(c, LFD_EINVAL, "state / rho_g / vhxc must be device memory");
+  cudaError_t e = cudaSuccess;
+  if (state) e = cudaMemcpyAsync(state, S.at<double>(S.L.state), 9 * sizeof(double), cudaMemcpyDeviceToDevice, c->stream);
+  if (e == cudaSuccess && rho_g)
+    e = cudaMemcpyAsync(rho_g, S.at<double>(S.L.pack), S.GN * sizeof(double), cudaMemcpyDeviceToDevice, c->stream);
+  if (e == cudaSuccess && vhxc)
+    e = cudaMemcpyAsync(vhxc, S.vh(S.vi[0]), S.GN * sizeof(double), cudaMemcpyDeviceToDevice, c->stream);
+  if (e != cudaSuccess) return cuda_fail(c, e, "SC read");
+  return LFD_OK;
+}
+
+lfd_status lfd_comm_unique_id(void* id128) {
+  if (!id128) { g_tls_error = "id128 is NULL"; return LFD_EINVAL; }
+  std::string why;
+  const Nccl* n = nccl_load(why);
+  if (!n) { g_tls_error = why; return LFD_EUNSUPPORTED; }
+  nccl_unique_id id;
+  int r = n->get_unique_id(&id);
+  if (r != 0) { g_tls_error = "ncclGetUniqueId failed"; return LFD_ECUDA; }
+  std::memcpy(id128, id.internal, sizeof(id.internal));
+  return LFD_OK;
+}
+
+lfd_status lfd_sc_comm_init(lfd_ctx* c, int32_t nranks, int32_t rank, const void* id128) {
+  LFD_TRY(check_ctx(c));
+  if (nranks < 1 || rank < 0 || rank >= nranks || !id128) return fail(c, LFD_EINVAL, "bad nranks / rank / id");
+  std::string why;
+  const Nccl* n = nccl_load(why);
+  if (!n) return fail(c, LFD_EUNSUPPORTED, why);
+  DeviceGuard dg(c->device);
+  if (c->sc.comm) {
+    n->comm_destroy(c->sc.comm);
+    c->sc.comm = nullptr;
+  }
+  nccl_unique_id id;
+  std::memcpy(id.internal, id128, sizeof(id.internal));
+  int r = n->comm_init_rank(&c->sc.comm, nranks, id, rank);
+  if (r != 0) {
+    c->sc.comm = nullptr;
+    return fail(c, LFD_ECUDA, std::string("ncclCommInitRank: ") + (n->error_string ? n->error_string(r) : "error"));
+  }
+  c->sc.comm_nranks = nranks;
+  c->sc.comm_rank = rank;
+  return LFD_OK;
+}
+
 lfd_status lfd_psi_modified(lfd_ctx* c) {
   LFD_TRY(check_ctx(c));
   c->c_valid = false;
@@ -823,6 +1265,11 @@ lfd_status lfd_destroy(lfd_ctx* c) {
     }
   }
   lfd::density_maps_destroy(c->dmaps);
+  sc_release(c->sc);
+  if (c->sc.comm) {
+    std::string why;
+    if (const Nccl* n = nccl_load(why)) n->comm_destroy(c->sc.comm);
+  }
   delete c;
   return LFD_OK;
 }

@@ -25,6 +25,7 @@
 // what bounds these sweeps next to HBM on B200 (DFMA 34 TF/s), so halving the FP64 work matters.
 #include <cmath>
 
+#include "lfd_coef.cuh"
 #include "lfd_complex.cuh"
 #include "lfd_internal.h"
 #include "lfd_tma.cuh"
@@ -35,33 +36,7 @@ __global__ void k_coef(CoefParams p, int dom0, int count, double hx, double hy, 
                        DomCoef* __restrict__ coef) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= count) return;
-  const double h[3] = {hx, hy, hz};
-  DomCoef c;
-  for (int d = 0; d < 3; ++d) {
-    double t = 1.0 / (2.0 * h[d] * h[d]);
-    double theta = (p.A[i][d] / kCLight) * h[d];
-    double st, ct;
-    sincos(theta, &st, &ct);
-    c.eth[d] = make_double2(ct, st);
-    c.inv_h[d] = 1.0 / h[d];
-    for (int q = 0; q < 2; ++q) {
-      double tau = (q == 0) ? 0.5 * dt : dt;
-      double sp, cp;
-      sincos(tau * t, &sp, &cp);
-      double2 ph = make_double2(cp, -sp);                  // e^{-i tau t}
-      double2 sigma = make_double2(sp * sp, sp * cp);      // i e^{-i tau t} sin(tau t)
-      c.alpha[d][q] = make_double2(cp * cp, -sp * cp);     // e^{-i tau t} cos(tau t)
-      c.up[d][q] = cmul(sigma, make_double2(ct, st));      // sigma e^{+i theta}
-      c.dn[d][q] = cmul(sigma, make_double2(ct, -st));     // sigma e^{-i theta}
-      c.onsite[d][q] = ph;
-      const double tn = sp / cp;                           // scaled form: w = i tan(tau t) e^{+-i theta}
-      c.wu[d][q] = make_double2(-tn * st, tn * ct);
-      c.wd[d][q] = make_double2(tn * st, tn * ct);
-      c.rc[d][q] = 1.0 / cp;                               // zero-BC singleton, relative to c
-    }
-  }
-  c.pad_ = 0.0;
-  coef[dom0 + i] = c;
+  coef[dom0 + i] = make_coef(p.A[i], hx, hy, hz, dt);
 }
 
 cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int count, DomCoef* coef,

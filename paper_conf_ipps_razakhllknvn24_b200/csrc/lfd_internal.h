@@ -162,4 +162,14 @@ cudaError_t launch_energy_final(const Geometry& g, const double* epart, int bloc
 cudaError_t launch_remap(const Geometry& g, int nref, const double2* C, const double* occ, double* out,
                          cudaStream_t st);
 
+// Self-consistent step kernels (sc.cu, readings R23-R28).
+cudaError_t launch_sc_maxwell_begin(double* st, const double* a_mid, const double* a_end, double dt, bool maxwell,
+                                    const Geometry& g, DomCoef* coef_mid, DomCoef* coef_end, cudaStream_t s);
+cudaError_t launch_sc_maxwell_end(double* st, const double* jbar, double dt, bool maxwell, cudaStream_t s);
+cudaError_t launch_sc_jbar(const double* Jmac, int ndom, double w, double* out, cudaStream_t s);
+cudaError_t launch_sc_vmid(const Geometry& g, const double* vion, const double* va, const double* vb, double wa,
+                           double wb, const int* off, int GY, int GZ, double* vout, cudaStream_t s);
+cudaError_t launch_sc_poisson(double2* spec, const int* gdims, const Geometry& g, cudaStream_t s);
+cudaError_t launch_sc_vhxc(const double* rho, double* v, long long n, bool hartree, bool xc, cudaStream_t s);
+
 }  // namespace lfd

@@ -17,7 +17,7 @@ import numpy as np
 HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "liblfd.so")
 
-LFD_ABI_VERSION = 3
+LFD_ABI_VERSION = 4
 LFD_FLAG_NO_CARRY = 1
 LFD_FLAG_EXACT_NL = 2
 LFD_BC_PERIODIC = 0
@@ -25,11 +25,16 @@ LFD_BC_ZERO = 1
 STATUS = {0: "LFD_OK", -1: "LFD_EINVAL", -2: "LFD_ENOMEM", -3: "LFD_ECUDA", -4: "LFD_ESTATE",
           -5: "LFD_EUNSUPPORTED"}
 KERNELS = ("coef", "phase", "kin_x", "kin_y", "kin_z", "nl_proj", "nl_reduce", "nl_norm", "nl_back",
-           "density", "jreduce", "energy", "nl_carry", "kin_yz")
+           "density", "jreduce", "energy", "nl_carry", "kin_yz", "sc", "fft")
+LFD_SC_HARTREE = 1
+LFD_SC_XC = 2
+LFD_SC_MAXWELL = 4
 EXPORTS = ("lfd_workspace_size", "lfd_init", "lfd_set_potential", "lfd_set_potential_host",
            "lfd_set_vector_potential", "lfd_step", "lfd_step_sequence", "lfd_density_current", "lfd_density_current_global",
            "lfd_density_current_host", "lfd_energy", "lfd_remap_occ", "lfd_psi_modified", "lfd_set_occupations", "lfd_set_stream", "lfd_sync",
-           "lfd_launch_count", "lfd_profile_enable", "lfd_profile_read", "lfd_last_error", "lfd_destroy")
+           "lfd_launch_count", "lfd_profile_enable", "lfd_profile_read", "lfd_last_error", "lfd_destroy",
+           "lfd_sc_workspace_size", "lfd_sc_init", "lfd_sc_step", "lfd_sc_read", "lfd_comm_unique_id",
+           "lfd_sc_comm_init")
 
 
 class lfd_config(C.Structure):
@@ -37,6 +42,11 @@ class lfd_config(C.Structure):
                 ("nz", C.c_int32), ("hx", C.c_double), ("hy", C.c_double), ("hz", C.c_double),
                 ("bc", C.c_int32), ("norb", C.c_int32), ("nproj", C.c_int32), ("nref_max", C.c_int32),
                 ("dt", C.c_double), ("device", C.c_int32), ("flags", C.c_int32)]
+
+
+class lfd_sc_config(C.Structure):
+    _fields_ = [("flags", C.c_int32), ("n_corr", C.c_int32), ("gdims", C.c_int32 * 3), ("nranks", C.c_int32),
+                ("rank", C.c_int32), ("dom_offset", C.c_void_p)]
 
 
 class LFDError(RuntimeError):
@@ -79,6 +89,12 @@ def load():
         "lfd_profile_enable": [P, I32],
         "lfd_profile_read": [P, D, C.POINTER(C.c_int64)],
         "lfd_destroy": [P],
+        "lfd_sc_workspace_size": [P, C.POINTER(lfd_sc_config), C.POINTER(C.c_size_t)],
+        "lfd_sc_init": [P, C.POINTER(lfd_sc_config), P, P, C.c_size_t, P, P, P],
+        "lfd_sc_step": [P, I32, P],
+        "lfd_sc_read": [P, P, P, P],
+        "lfd_comm_unique_id": [P],
+        "lfd_sc_comm_init": [P, I32, I32, P],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -240,6 +256,52 @@ def lfd_destroy(ctx):
     _check(load().lfd_destroy(ctx))
 
 
+def make_sc_config(flags, n_corr, gdims, dom_offset, nranks=1, rank=0):
+    """Returns (config, keepalive): dom_offset host int32 [ndom, 3]."""
+    off = np.ascontiguousarray(dom_offset, dtype=np.int32)
+    cfg = lfd_sc_config(int(flags), int(n_corr), (C.c_int32 * 3)(*[int(g) for g in gdims]), int(nranks), int(rank),
+                        C.c_void_p(off.ctypes.data))
+    return cfg, off
+
+
+def lfd_sc_workspace_size(ctx, sccfg) -> int:
+    n = C.c_size_t(0)
+    _check(load().lfd_sc_workspace_size(ctx, C.byref(sccfg), C.byref(n)), ctx)
+    return n.value
+
+
+def lfd_sc_init(ctx, sccfg, vion, ws, Aext0, A_ind0=None, Adot0=None):
+    pa, _k1 = _hptr(Aext0)
+    pi, _k2 = _hptr(A_ind0)
+    pd, _k3 = _hptr(Adot0)
+    _check(load().lfd_sc_init(ctx, C.byref(sccfg), _dptr(vion), _dptr(ws), ws.numel() * ws.element_size(), pa, pi,
+                              pd), ctx)
+
+
+def lfd_sc_step(ctx, Aext):
+    """Aext: host [2*nsteps+1, 3] (A_ext at t_n, t_n + dt/2, t_n+1, ...)."""
+    arr = np.ascontiguousarray(Aext, dtype=np.float64).reshape(-1, 3)
+    if arr.shape[0] % 2 != 1:
+        raise ValueError("Aext needs 2*nsteps+1 rows")
+    p, _k = _hptr(arr)
+    _check(load().lfd_sc_step(ctx, int((arr.shape[0] - 1) // 2), p), ctx)
+
+
+def lfd_sc_read(ctx, state=None, rho_g=None, vhxc=None):
+    _check(load().lfd_sc_read(ctx, _dptr(state), _dptr(rho_g), _dptr(vhxc)), ctx)
+
+
+def lfd_comm_unique_id() -> bytes:
+    buf = (C.c_char * 128)()
+    _check(load().lfd_comm_unique_id(buf))
+    return bytes(buf)
+
+
+def lfd_sc_comm_init(ctx, nranks: int, rank: int, uid: bytes):
+    buf = (C.c_char * 128).from_buffer_copy(uid)
+    _check(load().lfd_sc_comm_init(ctx, int(nranks), int(rank), buf), ctx)
+
+
 # ---- convenience owner ---------------------------------------------------------------------------
 
 class Context:
@@ -300,6 +362,33 @@ class Context:
         out = torch.empty((self.shape[0], ref.shape[-1]), dtype=torch.float64, device=self.psi.device)
         lfd_remap_occ(self.ctx, ref, out)
         return out
+
+    def sc_init(self, gdims, dom_offset, vion=None, flags=LFD_SC_HARTREE | LFD_SC_XC | LFD_SC_MAXWELL, n_corr=1,
+                Aext0=(0.0, 0.0, 0.0), A_ind0=None, Adot0=None, nranks=1, rank=0, comm_id=None):
+        """Self-consistent step state (lfd_sc_*). vion: CUDA float64 [ndom, nx, ny, nz] or None.
+        With nranks > 1, comm_id = the 128 bytes of lfd_comm_unique_id() from one rank."""
+        import torch
+        if nranks > 1:
+            lfd_sc_comm_init(self.ctx, nranks, rank, comm_id)
+        self.sc_cfg, self._sc_off = make_sc_config(flags, n_corr, gdims, dom_offset, nranks, rank)
+        n = lfd_sc_workspace_size(self.ctx, self.sc_cfg)
+        self.sc_ws = torch.empty(max(n, 1), dtype=torch.uint8, device=self.psi.device)
+        self.vion = vion
+        lfd_sc_init(self.ctx, self.sc_cfg, vion, self.sc_ws, Aext0, A_ind0, Adot0)
+        self.gdims = tuple(int(g) for g in gdims)
+
+    def sc_step(self, Aext):
+        lfd_sc_step(self.ctx, Aext)
+
+    def sc_read(self):
+        """(state [9] = A_ind, dA_ind/dt, Jbar; rho_g [GX,GY,GZ]; v_Hxc [GX,GY,GZ]) as CUDA tensors."""
+        import torch
+        dev = self.psi.device
+        st = torch.empty(9, dtype=torch.float64, device=dev)
+        rho = torch.empty(self.gdims, dtype=torch.float64, device=dev)
+        v = torch.empty(self.gdims, dtype=torch.float64, device=dev)
+        lfd_sc_read(self.ctx, st, rho, v)
+        return st, rho, v
 
     def psi_modified(self):
         lfd_psi_modified(self.ctx)
