@@ -11,6 +11,7 @@
 #include "lfd_tma.cuh"
 
 #include <algorithm>
+#include <cstdlib>
 #include <new>
 
 namespace lfd {
@@ -300,33 +301,37 @@ __global__ void __launch_bounds__(kDensThreads) k_density_tma(Geometry g, DensAr
 }
 
 // ------------------------------------------------------------------------------------------------
-// y-marching variant (norb <= 128; the bench shape). CTA = (x plane, z chunk of zc points, domain): it
-// walks y and needs, at step y, the z-line segment of its own points (x, y, z0..z0+zc) plus the z+1
-// halo point, the next line (x, y+1) for the y links and the line (x+1, y) for the x links. A producer
-// warp brings each segment with one tiled TMA tensor copy (all orbitals of zc points; the halo point is
-// a second, 1-point copy) into two
-// rings (own lines: 3 slots, x+1 lines: 2 slots) with full/empty mbarriers; the own line y+1 stays
-// resident for the next step, and the x+1 lines are the next CTA's own lines, read about when that CTA
-// reads them (L2 hits). kSub lanes per point split the orbitals and the 7 per-point sums are shuffle
-// reductions with the occupation weights (kept in shared memory).
+// y-marching variant (norb <= 128; the bench shape). CTA = (px consecutive x planes, z chunk of zc
+// points, y chunk, domain): it walks y and needs, at step y, the z-line segments of its own points
+// (x0..x0+px-1, y, z0..z0+zc) plus their z+1 halo points, the next lines (y+1) for the y links and, for
+// the x links, the lines of its own next plane -- or, for the last plane, of plane x0+px (the next CTA's
+// first plane: an L2 hit, so HBM sees each line once and the L2->SM traffic is (px+1)/px of it). A
+// producer warp brings each segment with one tiled TMA tensor copy (the halo point is a second, 1-point
+// copy) into two rings (own lines: kYOwn slots of px segments, x+px lines: kYXp slots) with full/empty
+// mbarriers; the own line y+1 stays resident for the next step. kSub lanes per point split the orbitals
+// and the 7 per-point sums are shuffle reductions with the occupation weights (kept in shared memory).
 // ------------------------------------------------------------------------------------------------
-constexpr int kYOwn = 3, kYXp = 2;
-constexpr int kYMaxThreads = 352;  // up to 40 points x kSub + the producer warp
+constexpr int kYOwn = 4, kYXp = 3;  // ring depths (lines); the own line y+1 stays resident for the y links
+constexpr int kYMaxThreads = 512;  // up to 60 points x kSub + the producer warp
 
 struct DensMaps {
   CUtensorMap seg;   // box [1][zc][2*nact]: a z-line segment of zc points, the active orbitals
   CUtensorMap one;   // box [1][1][2*nact]: the z+1 halo point
-  int zc;            // points per CTA (divides nz)
+  int zc;            // points per CTA and plane (divides nz)
+  int px;            // x planes per CTA (divides nx)
+  int nyc;           // y chunks per (plane group, z chunk)
   int nact;          // active orbitals: 1 + the last index with f != 0 (f = 0 contributes exactly 0)
 };
 
-// shared-memory layout of the y-marching kernel (every TMA destination 128-byte aligned)
+// shared-memory layout of the y-marching kernel (every TMA destination 128-byte aligned): an own slot
+// holds px (segment, halo point) pairs
 struct YLayout {
-  size_t seg_b, halo_b, own_b, xp_b, fsh_off, bar_off, total;
-  __host__ __device__ YLayout(int zc, int norb) {
+  size_t seg_b, halo_b, pl_b, own_b, xp_b, fsh_off, bar_off, total;
+  __host__ __device__ YLayout(int zc, int norb, int px) {
     seg_b = ((size_t)zc * norb * 16 + 127) & ~(size_t)127;
     halo_b = ((size_t)norb * 16 + 127) & ~(size_t)127;
-    own_b = seg_b + halo_b;
+    pl_b = seg_b + halo_b;
+    own_b = px * pl_b;
     xp_b = seg_b;
     fsh_off = kYOwn * own_b + kYXp * xp_b;
     bar_off = fsh_off + (((size_t)norb * 8 + 15) & ~(size_t)15);
@@ -334,42 +339,71 @@ struct YLayout {
   }
 };
 
-static int ymarch_zc(const Geometry& g) {
-  if (g.norb > 128) return 0;
-  const size_t per_pt = (size_t)g.norb * 16;
+struct YShape {
+  int zc, px, nyc;
+};
+
+// Tuning knobs LFD_DENS_ZCMAX (points per plane), LFD_DENS_PX (planes per CTA), LFD_DENS_YC (y chunks).
+static YShape ymarch_shape(const Geometry& g) {
+  YShape sh{0, 1, 1};
+  if (g.norb > 128) return sh;
+  int zmax = 18, pxmax = 1, yc = 1;  // measured on C2 (tools/dens_tune.sh): 1 plane, 18 points
+  if (const char* v = std::getenv("LFD_DENS_ZCMAX")) zmax = std::max(1, std::min(60, std::atoi(v)));
+  if (const char* v = std::getenv("LFD_DENS_PX")) pxmax = std::max(1, std::atoi(v));
+  if (const char* v = std::getenv("LFD_DENS_YC")) yc = std::max(1, std::atoi(v));
+  int px = 1;
+  for (int d = std::min(pxmax, g.nx); d >= 1; --d)
+    if (g.nx % d == 0) { px = d; break; }
   for (int nzc = 1; nzc <= g.nz; ++nzc) {
     if (g.nz % nzc) continue;
     const int zc = g.nz / nzc;
-    if (zc > 40) continue;
-    (void)per_pt;
-    if (YLayout(zc, g.norb).total <= 200 * 1024) return zc;
+    if (zc > zmax || zc * px * kSub + 32 > kYMaxThreads) continue;
+    if (YLayout(zc, g.norb, px).total <= 200 * 1024) { sh.zc = zc; break; }
   }
-  return 0;
+  if (sh.zc == 0 && px > 1) {  // fall back to one plane per CTA
+    sh.px = 1;
+    for (int nzc = 1; nzc <= g.nz; ++nzc) {
+      if (g.nz % nzc) continue;
+      const int zc = g.nz / nzc;
+      if (zc > std::min(zmax, 40)) continue;
+      if (YLayout(zc, g.norb, 1).total <= 200 * 1024) { sh.zc = zc; break; }
+    }
+    px = 1;
+  }
+  sh.px = px;
+  sh.nyc = std::max(1, std::min(yc, g.ny / 2 > 0 ? g.ny / 2 : 1));
+  return sh;
 }
 
 template <bool kPer, int kIt>
 __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constant__ DensMaps mp, Geometry g,
                                                             DensArgs a) {
   extern __shared__ __align__(128) unsigned char dsm[];
-  const int norb = mp.nact, zc = mp.zc;  // smem rows hold the nact active orbitals of each point
-  const YLayout Ly(zc, norb);
-  auto own_slot = [&](int s) { return reinterpret_cast<double2*>(dsm + s * Ly.own_b); };
-  auto halo_of = [&](int s) { return reinterpret_cast<double2*>(dsm + s * Ly.own_b + Ly.seg_b); };
+  const int norb = mp.nact, zc = mp.zc, px = mp.px;  // smem rows hold the nact active orbitals of each point
+  const YLayout Ly(zc, norb, px);
+  auto own_seg = [&](int s, int p) { return reinterpret_cast<double2*>(dsm + s * Ly.own_b + p * Ly.pl_b); };
+  auto halo_of = [&](int s, int p) {
+    return reinterpret_cast<double2*>(dsm + s * Ly.own_b + p * Ly.pl_b + Ly.seg_b);
+  };
   auto xp_slot = [&](int s) { return reinterpret_cast<double2*>(dsm + kYOwn * Ly.own_b + s * Ly.xp_b); };
   double* fsh = reinterpret_cast<double*>(dsm + Ly.fsh_off);
   uint64_t* bars = reinterpret_cast<uint64_t*>(dsm + Ly.bar_off);
   uint64_t *ofull = bars, *oempty = bars + kYOwn, *xfull = bars + 2 * kYOwn, *xempty = xfull + kYXp;
   __shared__ double jsh[5][kYMaxThreads / kSub];
   const int dom = blockIdx.y;
-  const int nzc = g.nz / zc;
-  const int x = blockIdx.x / nzc, z0 = (blockIdx.x - x * nzc) * zc;
+  const int nzc = g.nz / zc, nyc = mp.nyc;
+  const int yci = blockIdx.x % nyc, xz = blockIdx.x / nyc;
+  const int xg = xz / nzc, z0 = (xz - xg * nzc) * zc;
+  const int xb = xg * px;  // first plane of the CTA
+  const int y0 = (int)(((long long)yci * g.ny) / nyc), ycnt = (int)(((long long)(yci + 1) * g.ny) / nyc) - y0;
   const bool per = kPer;
-  const bool has_x = per || x + 1 < g.nx;
-  const int xp = (x + 1 == g.nx) ? 0 : x + 1;
+  const bool has_xn = per || xb + px < g.nx;  // plane xb + px exists (the x+1 of the last plane)
+  const int xnext = (xb + px == g.nx) ? 0 : xb + px;
   const bool last_chunk = z0 + zc == g.nz;
-  const int nconsw = (zc * kSub + 31) >> 5;
+  const int nconsw = (zc * px * kSub + 31) >> 5;
   const int tid = threadIdx.x;
-  const int nown = per ? g.ny + 1 : g.ny;  // own lines y = 0..ny-1 (+ y = 0 again for the periodic wrap)
+  // own lines y0 .. y0+ycnt-1 plus the y+1 halo line (y = 0 again past the periodic wrap)
+  const int nown = (per || y0 + ycnt < g.ny) ? ycnt + 1 : ycnt;
   if (tid == 0) {
     for (int s = 0; s < kYOwn; ++s) { mbar_init(&ofull[s], 1); mbar_init(&oempty[s], nconsw); }
     for (int s = 0; s < kYXp; ++s) { mbar_init(&xfull[s], 1); mbar_init(&xempty[s], nconsw); }
@@ -380,34 +414,40 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
 
   if (tid >= nconsw * 32) {  // producer warp
     if (tid == nconsw * 32) {
-      const int rowx = (dom * g.nx + x) * g.ny, rowxp = (dom * g.nx + xp) * g.ny;
-      auto issue_own = [&](int k) {  // own line k (k == ny: plane 0 again)
+      const int rowxn = (dom * g.nx + xnext) * g.ny;
+      auto issue_own = [&](int k) {  // own lines y0 + k (== ny: plane 0 again) of the px planes
         const int s = k % kYOwn;
         if (k >= kYOwn) mbar_wait(&oempty[s], (uint32_t)(((k / kYOwn) - 1) & 1));
-        const int yy = (k == g.ny) ? 0 : k;
+        const int yy = (y0 + k == g.ny) ? 0 : y0 + k;
         const bool halo = !last_chunk || per;  // z+1 halo point: z0 + zc, or z = 0 (periodic wrap)
-        mbar_expect_tx(&ofull[s], (uint32_t)((zc + (halo ? 1 : 0)) * norb * 16));
-        tma_3d(own_slot(s), &mp.seg, 0, z0, rowx + yy, &ofull[s]);
-        if (halo) tma_3d(halo_of(s), &mp.one, 0, last_chunk ? 0 : z0 + zc, rowx + yy, &ofull[s]);
+        mbar_expect_tx(&ofull[s], (uint32_t)(px * (zc + (halo ? 1 : 0)) * norb * 16));
+        for (int p = 0; p < px; ++p) {
+          const int row = (dom * g.nx + xb + p) * g.ny + yy;
+          tma_3d(own_seg(s, p), &mp.seg, 0, z0, row, &ofull[s]);
+          if (halo) tma_3d(halo_of(s, p), &mp.one, 0, last_chunk ? 0 : z0 + zc, row, &ofull[s]);
+        }
       };
       auto issue_xp = [&](int k) {
         const int s = k % kYXp;
         if (k >= kYXp) mbar_wait(&xempty[s], (uint32_t)(((k / kYXp) - 1) & 1));
         mbar_expect_tx(&xfull[s], (uint32_t)(zc * norb * 16));
-        tma_3d(xp_slot(s), &mp.seg, 0, z0, rowxp + k, &xfull[s]);
+        tma_3d(xp_slot(s), &mp.seg, 0, z0, rowxn + y0 + k, &xfull[s]);
       };
       issue_own(0);
       if (nown > 1) issue_own(1);
-      for (int y = 0; y < g.ny; ++y) {
-        if (has_x) issue_xp(y);
-        if (y + 2 < nown) issue_own(y + 2);
+      for (int k = 0; k < ycnt; ++k) {
+        if (has_xn) issue_xp(k);
+        if (k + 2 < nown) issue_own(k + 2);
       }
     }
     return;
   }
 
-  const int q = tid % kSub, pt = tid / kSub;
-  const bool valid = pt < zc;
+  const int q = tid % kSub, pa = tid / kSub;
+  const int pl = pa / zc, pt = pa - pl * zc;  // plane within the CTA, point within the z chunk
+  const bool valid = pl < px;
+  const int x = xb + (valid ? pl : 0);
+  const bool has_x = per || x + 1 < g.nx;
   const int z = z0 + pt;
   const bool has_z = valid && (kPer || z + 1 < g.nz);
   const DomCoef* cf = a.coef + dom;
@@ -424,16 +464,19 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
   // lane q of a point ends up holding the full sum of value q >> 1: 0 rho, 1 jx, 2 jy, 3 jz
   const int vsel = q >> 1;
   double jacc = 0.0, ekin = 0.0, eloc = 0.0;
-  for (int y = 0; y < g.ny; ++y) {
+  const long long rbase = a.base[dom], jb = a.j ? a.jbase[dom] : 0;  // hoisted global loads
+  for (int k = 0; k < ycnt; ++k) {
+    const int y = y0 + k;
     const bool has_y = valid && (kPer || y + 1 < g.ny);
-    const int so = y % kYOwn, sn = (y + 1) % kYOwn, sx = y % kYXp;
-    mbar_wait(&ofull[so], (uint32_t)((y / kYOwn) & 1));
-    if (y + 1 < nown) mbar_wait(&ofull[sn], (uint32_t)(((y + 1) / kYOwn) & 1));
-    if (has_x) mbar_wait(&xfull[sx], (uint32_t)((y / kYXp) & 1));
-    const double2* O = own_slot(so) + ptr * norb;
-    const double2* Oz = (ptr + 1 < zc) ? O + norb : halo_of(so);  // point z+1
-    const double2* N = own_slot(sn) + ptr * norb;
-    const double2* X = xp_slot(sx) + ptr * norb;
+    const int so = k % kYOwn, sn = (k + 1) % kYOwn, sx = k % kYXp;
+    mbar_wait(&ofull[so], (uint32_t)((k / kYOwn) & 1));
+    if (k + 1 < nown) mbar_wait(&ofull[sn], (uint32_t)(((k + 1) / kYOwn) & 1));
+    if (has_xn) mbar_wait(&xfull[sx], (uint32_t)((k / kYXp) & 1));
+    const int plr = valid ? pl : 0;
+    const double2* O = own_seg(so, plr) + ptr * norb;
+    const double2* Oz = (ptr + 1 < zc) ? O + norb : halo_of(so, plr);  // point z+1
+    const double2* N = own_seg(sn, plr) + ptr * norb;
+    const double2* X = (plr + 1 < px ? own_seg(so, plr + 1) : xp_slot(sx)) + ptr * norb;  // plane x+1
     // per-lane partial sums over this lane's orbitals: rho and the three link products P_d = sum f
     // conj(psi_r) psi_{r+e_d} (f folded into fv = f psi_r)
     double rho = 0.0, pxr = 0.0, pxi = 0.0, pyr = 0.0, pyi = 0.0, pzr = 0.0, pzi = 0.0;
@@ -465,7 +508,7 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
     __syncwarp();
     if ((tid & 31) == 0) {  // this warp is done with own line y and x+1 line y
       mbar_arrive(&oempty[so]);
-      if (has_x) mbar_arrive(&xempty[sx]);
+      if (has_xn) mbar_arrive(&xempty[sx]);
     }
     // the currents and the kinetic energy density are linear in the P_d: form them per lane first
     // (Im(e^{i theta} P) = cos Im P + sin Re P, Re(e^{i theta} P) = cos Re P - sin Im P)
@@ -499,24 +542,24 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
     if (valid && (q & 1) == 0) {
       const long long o = (long long)x * a.sx + (long long)y * a.sy + z;
       if (vsel == 0) {
-        a.rho[a.base[dom] + o] = val;
+        a.rho[rbase + o] = val;
         if (a.epart) eloc += a.v[(long long)dom * g.ng + ((long long)x * g.ny + y) * g.nz + z] * val;
       } else {
         jacc += val;
-        if (a.j) a.j[a.jbase[dom] + o + (vsel - 1) * a.jstride] = val;
+        if (a.j) a.j[jb + o + (vsel - 1) * a.jstride] = val;
       }
     }
   }
   // per-CTA sums in a fixed order: J components from lanes q = 2, 4, 6 of every point, energies from all
   const int pts = nconsw * 32 / kSub;
-  if (q == 2 || q == 4 || q == 6) jsh[q / 2 - 1][pt] = jacc;
+  if (q == 2 || q == 4 || q == 6) jsh[q / 2 - 1][pa] = jacc;
   double ekp = ekin;  // sum the kinetic partials over the 8 lanes of the point (fixed tree)
   ekp += __shfl_xor_sync(0xffffffffu, ekp, 4);
   ekp += __shfl_xor_sync(0xffffffffu, ekp, 2);
   ekp += __shfl_xor_sync(0xffffffffu, ekp, 1);
   if (q == 0) {
-    jsh[3][pt] = ekp;
-    jsh[4][pt] = eloc;
+    jsh[3][pa] = ekp;
+    jsh[4][pa] = eloc;
   }
   asm volatile("bar.sync 1, %0;" ::"r"(nconsw * 32));  // consumer warps only
   if (a.epart && tid >= 3 && tid < 5) {  // (warp 0: there may be a single consumer warp)
@@ -531,7 +574,7 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
   }
 }
 
-static size_t ymarch_smem(int zc, int nact) { return YLayout(zc, nact).total; }
+static size_t ymarch_smem(int zc, int nact, int px) { return YLayout(zc, nact, px).total; }
 
 static cudaError_t density_maps_encode(DensMaps* m, const Geometry& g, const double2* psi, int nact) {
   const uint64_t dims[3] = {(uint64_t)2 * g.norb, (uint64_t)g.nz, (uint64_t)g.ndom * g.nx * g.ny};
@@ -545,11 +588,13 @@ static cudaError_t density_maps_encode(DensMaps* m, const Geometry& g, const dou
 }
 
 DensMaps* density_maps_create(const Geometry& g, const double2* psi, int nact) {
-  const int zc = ymarch_zc(g);
-  if (zc == 0) return nullptr;
+  const YShape sh = ymarch_shape(g);
+  if (sh.zc == 0) return nullptr;
   DensMaps* m = new (std::nothrow) DensMaps;
   if (!m) return nullptr;
-  m->zc = zc;
+  m->zc = sh.zc;
+  m->px = sh.px;
+  m->nyc = sh.nyc;
   if (density_maps_encode(m, g, psi, std::min(std::max(nact, 1), g.norb)) != cudaSuccess) {
     delete m;
     return nullptr;
@@ -568,8 +613,8 @@ void density_maps_destroy(DensMaps* m) { delete m; }
 int density_smem_bytes(int norb) { return kRingSlots * kPlanePts * norb * 16; }
 
 int density_blocks(const Geometry& g) {
-  const int zc = ymarch_zc(g);
-  if (zc > 0) return g.nx * (g.nz / zc);
+  const YShape sh = ymarch_shape(g);
+  if (sh.zc > 0) return (g.nx / sh.px) * (g.nz / sh.zc) * sh.nyc;
   const int ntz = (g.nz + kTZ - 1) / kTZ, nty = (g.ny + kTY - 1) / kTY, nxc = (g.nx + kXC - 1) / kXC;
   return ntz * nty * nxc;
 }
@@ -577,8 +622,8 @@ int density_blocks(const Geometry& g) {
 cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps* maps, cudaStream_t st) {
   dim3 grid(density_blocks(g), g.ndom);
   if (maps) {
-    const int threads = ((maps->zc * kSub + 31) / 32 + 1) * 32;
-    const size_t sm = ymarch_smem(maps->zc, maps->nact);
+    const int threads = ((maps->zc * maps->px * kSub + 31) / 32 + 1) * 32;
+    const size_t sm = ymarch_smem(maps->zc, maps->nact, maps->px);
     if (g.bc == 0 && maps->nact == 64)
       k_density_y<true, 8><<<grid, threads, sm, st>>>(*maps, g, a);
     else if (g.bc == 0 && maps->nact == 32)
@@ -589,7 +634,7 @@ cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps*
       k_density_y<false, 0><<<grid, threads, sm, st>>>(*maps, g, a);
     return cudaGetLastError();
   }
-  if (ymarch_zc(g) > 0) return cudaErrorInvalidValue;  // the block layout expects the y-marching kernel
+  if (ymarch_shape(g).zc > 0) return cudaErrorInvalidValue;  // the block layout expects the y-marching kernel
   const int ntz = (g.nz + kTZ - 1) / kTZ, nty = (g.ny + kTY - 1) / kTY;
   if (g.norb <= kMaxNorbTma)
     k_density_tma<<<grid, kDensThreads, density_smem_bytes(g.norb), st>>>(g, a, ntz, nty, kXC);

@@ -37,9 +37,12 @@ def main():
             ctx.set_vector_potential(midpoint_A(w, n))
             ctx.step(1)
         lfd.lfd_profile_enable(ctx.ctx, True)
+        rho = torch.empty((w.ndom, w.ngrid), dtype=torch.float64, device=dev)
+        J = torch.empty((w.ndom, 3), dtype=torch.float64, device=dev)
         for n in range(args.steps):
             ctx.set_vector_potential(midpoint_A(w, n))
             ctx.step(1)
+            lfd.lfd_density_current(ctx.ctx, rho, None, J)
         prof = lfd.lfd_profile_read(ctx.ctx)
         ctx.close()
         out = {"knob": args.knob, "value": val,
