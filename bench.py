@@ -70,6 +70,9 @@ def parse():
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--no-sc", action="store_true", help="skip the self-consistent-step measurement (sc_mode)")
     ap.add_argument("--sc-corr", type=int, default=1, help="corrector sweeps of the sc_mode measurement")
+    ap.add_argument("--sc-multi", action="store_true",
+                    help="also measure sc_mode under torchrun (its NCCL communicator is built by liblfd; the "
+                         "multi-rank path has not run on this pool, which has one GPU per call)")
     ap.add_argument("--exact-nl", action="store_true",
                     help="exactly unitary nonlocal factor (LFD_FLAG_EXACT_NL, SURVEY §8(f) rank 4)")
     return ap.parse_args()
@@ -433,7 +436,7 @@ def main():
     # ranks' domains) + LDA exchange + Maxwell, predictor + n_corr corrector sweeps, the [rho_g | Jbar]
     # SUM all-reduce over NCCL inside the step when world > 1 -- the full LFD subprogram per QD step
     scm = None
-    if not args.no_sc:
+    if not args.no_sc and (world == 1 or args.sc_multi):
         try:
             scm = run_sc_mode(args, w, ctx, x, dev, stream, rank, world)
         except Exception as ex:  # reported, never fatal for the main measurement
