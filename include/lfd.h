@@ -65,7 +65,7 @@ typedef struct {
   int32_t nref_max;    /* max reference-basis columns for lfd_remap_occ, 0..2048 (0: max(norb, nproj)) */
   double dt;           /* Delta_QD [a.u.], finite and nonzero (negative = backward in time) */
   int32_t device;      /* CUDA device ordinal */
-  int32_t flags;       /* 0 or LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL */
+  int32_t flags;       /* 0 or LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP */
 } lfd_config;
 
 /* lfd_config.flags: disable the projection carry (lfd_step takes the C of each nonlocal factor that
@@ -78,6 +78,13 @@ typedef struct {
  * LFD_EINVAL otherwise) exp(-i (Delta/2) B diag(D) B^H dV) = 1 + B diag(e^{-i (Delta/2) D} - 1) B^H dV,
  * which keeps every orbital's norm and the orthonormality of Psi exactly (no renormalisation). */
 #define LFD_FLAG_EXACT_NL 2
+/* lfd_config.flags: the SP variant (the paper's SP column, and its
+ * complex<float> listings): psi, proj (and lfd_remap_occ's ref) are complex64 [.. same layouts ..]
+ * (two floats, 8-byte aligned). The stencil sweeps run in FP32 (three line passes), the projector GEMMs in
+ * 3xTF32 on the tensor pipe (FP32-accurate products, FP32 accumulation per split), and everything
+ * O(nproj x norb) -- the split reduction, the Gram matrix, n_s, the carry, the energies -- in FP64. Results
+ * agree with the FP64 path to single-precision roundoff (DESIGN.md §4 states the tolerance). */
+#define LFD_FLAG_SP 4
 
 /* Kernel classes, for lfd_profile_read(). */
 typedef enum {

@@ -31,7 +31,7 @@ size_t up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 struct Layout {
   size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage, cref,
-      epart, W, ones;
+      epart, W, ones, x32;
   int nref_cap;
   size_t total;
   int nsplit;
@@ -64,7 +64,7 @@ lfd_status validate(const lfd_config* c, std::string& why) {
   if (c->norb < 1) { why = "norb must be >= 1"; return LFD_EINVAL; }
   if (c->nproj < 0 || c->nproj > 2048) { why = "nproj must be in [0, 2048]"; return LFD_EINVAL; }
   if (!(c->dt != 0.0) || !std::isfinite(c->dt)) { why = "dt must be finite and nonzero"; return LFD_EINVAL; }
-  if (c->flags & ~(LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL)) { why = "unknown flags"; return LFD_EINVAL; }
+  if (c->flags & ~(LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP)) { why = "unknown flags"; return LFD_EINVAL; }
   if (c->nref_max < 0 || c->nref_max > 2048) { why = "nref_max must be in [0, 2048]"; return LFD_EINVAL; }
   const long long ng = (long long)c->nx * c->ny * c->nz;
   if (ng * (long long)std::max(c->norb, std::max(c->nproj, 1)) >= (1LL << 31)) {
@@ -80,6 +80,7 @@ Geometry geometry(const lfd_config* c) {
   g.norb = c->norb; g.nproj = c->nproj; g.bc = c->bc;
   g.hx = c->hx; g.hy = c->hy; g.hz = c->hz; g.dt = c->dt; g.dV = c->hx * c->hy * c->hz;
   g.ng = (long long)c->nx * c->ny * c->nz;
+  g.sp = (c->flags & LFD_FLAG_SP) ? 1 : 0;
   return g;
 }
 
@@ -139,6 +140,7 @@ Layout layout(const Geometry& g, int num_sms, int nref_max) {
   L.epart = take((size_t)nd * lfd::density_blocks(g) * 2 * d8);
   L.W = take((size_t)2 * nd * np * c16);
   L.ones = take((size_t)nd * std::max(np, no) * d8);
+  L.x32 = g.sp ? take((size_t)nd * np * no * 8) : 0;  // SP: the GEMM-2 coefficient rounded to complex64
   L.total = o;
   return L;
 }
@@ -263,6 +265,11 @@ struct lfd_ctx {
   T* at(size_t off) const { return reinterpret_cast<T*>(ws + off); }
   DomCoef* coef() const { return at<DomCoef>(L.coef); }
   double2* phi() const { return at<double2>(L.phi); }
+  // SP variant views (complex64 Psi, B, Phi)
+  float2* psi32() const { return reinterpret_cast<float2*>(psi); }
+  const float2* proj32() const { return reinterpret_cast<const float2*>(proj); }
+  float2* phi32() const { return at<float2>(L.phi); }
+  size_t celem() const { return g.sp ? 8 : 16; }
 };
 
 namespace {
@@ -360,6 +367,20 @@ bool is_device_ptr(const void* p) {
   return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
+// GEMM-1 launch in the context's precision (the SP variant reads complex64 A and X).
+cudaError_t gemm1_any(lfd_ctx* c, const lfd::Gemm1Args& a) {
+  if (c->g.sp)
+    return lfd::launch_gemm1_sp(a, reinterpret_cast<const float2*>(a.A), reinterpret_cast<const float2*>(a.X),
+                                c->stream);
+  return lfd::launch_gemm1(a, c->stream);
+}
+
+// Phi from v in the context's precision (vcopy as lfd::launch_phase).
+cudaError_t phase_any(lfd_ctx* c, const double* v, double* vcopy) {
+  if (c->g.sp) return lfd::launch_phase_sp(c->g, v, c->phi32(), vcopy, c->scaled, c->stream);
+  return lfd::launch_phase(c->g, v, c->phi(), vcopy, c->scaled, c->stream);
+}
+
 // GEMM-2 of a nonlocal factor: Psi <- (Psi + B C') diag(n), C' and n from the workspace.
 lfd_status gemm2(lfd_ctx* c) {
   const Geometry& g = c->g;
@@ -368,7 +389,13 @@ lfd_status gemm2(lfd_ctx* c) {
   a2.ndom = g.ndom; a2.nproj = g.nproj; a2.norb = g.norb; a2.ng = g.ng; a2.num_sms = c->num_sms;
   a2.variant = c->gemm2_variant;
   c->c_valid = false;
-  LFD_TRY(launch(c, LFD_K_NL_BACK, "k_gemm2", [&] { return lfd::launch_gemm2(a2, c->stream); }));
+  if (g.sp)
+    LFD_TRY(launch(c, LFD_K_NL_BACK, "k_gemm2_sp", [&] {
+      return lfd::launch_gemm2_sp(c->psi32(), c->proj32(), a2.Cp, c->at<float2>(c->L.x32), a2.nfac, g.ndom, g.nproj,
+                                  g.norb, g.ng, c->stream);
+    }));
+  else
+    LFD_TRY(launch(c, LFD_K_NL_BACK, "k_gemm2", [&] { return lfd::launch_gemm2(a2, c->stream); }));
   c->c_valid = c->carry;
   return LFD_OK;
 }
@@ -413,7 +440,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false) {
   a1.ndom = g.ndom; a1.mrows = g.nproj; a1.ncols = g.norb; a1.nsplit = c->L.nsplit;
   a1.ng = g.ng; a1.rows_per_split = c->L.rows_per_split;
   a1.a_dom_stride = g.ng * g.nproj; a1.x_dom_stride = g.ng * g.norb;
-  LFD_TRY(launch(c, LFD_K_NL_PROJ, "k_gemm1", [&] { return lfd::launch_gemm1(a1, c->stream); }));
+  LFD_TRY(launch(c, LFD_K_NL_PROJ, "k_gemm1", [&] { return gemm1_any(c, a1); }));
   lfd::ReduceArgs r;
   r.part = a1.part; r.normp = a1.norms;
   r.D = c->at<double>(c->L.D);
@@ -445,6 +472,17 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false) {
 // Local factor exp(-i Delta h_loc) of Eq. 6: Psi <- Phi . K_z K_y K_x (Phi . Psi) (kernels a6).
 lfd_status local_prop(lfd_ctx* c) {
   c->c_valid = false;
+  if (c->g.sp) {  // SP variant: three FP32 line passes Phi.K_x, K_y, K_z.Phi (complex64 Psi)
+    LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin_sp(x)", [&] {
+      return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 0, 1, c->scaled, c->stream);
+    }));
+    LFD_TRY(launch(c, LFD_K_KIN_Y, "k_kin_sp(y)", [&] {
+      return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 1, 0, c->scaled, c->stream);
+    }));
+    return launch(c, LFD_K_KIN_Z, "k_kin_sp(z)", [&] {
+      return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 2, 2, c->scaled, c->stream);
+    });
+  }
   LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin(x)",
                  [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 0, 1, c->scaled, c->stream); }));
   if (c->kin_fused)
@@ -464,7 +502,7 @@ lfd_status project(lfd_ctx* c, const double2* A, int mrows, double2* out) {
   a1.ndom = g.ndom; a1.mrows = mrows; a1.ncols = g.norb; a1.nsplit = c->L.nsplit;
   a1.ng = g.ng; a1.rows_per_split = c->L.rows_per_split;
   a1.a_dom_stride = g.ng * mrows; a1.x_dom_stride = g.ng * g.norb;
-  LFD_TRY(launch(c, LFD_K_NL_PROJ, "k_gemm1", [&] { return lfd::launch_gemm1(a1, c->stream); }));
+  LFD_TRY(launch(c, LFD_K_NL_PROJ, "k_gemm1", [&] { return gemm1_any(c, a1); }));
   lfd::ReduceArgs r{};
   r.part = a1.part; r.normp = nullptr; r.D = nullptr; r.out = out; r.cprime = nullptr; r.s = nullptr;
   r.ndom = g.ndom; r.mrows = mrows; r.ncols = g.norb; r.nsplit = c->L.nsplit; r.scale = g.dV; r.eps = 0;
@@ -487,6 +525,7 @@ lfd_status density_into(lfd_ctx* c, double* rho, double* j, double* Jmac, const 
                         long long sy, long long jstride, bool energy = false, const DomCoef* coef = nullptr) {
   lfd::DensArgs a;
   a.psi = c->psi; a.coef = coef ? coef : c->coef(); a.occ = c->at<double>(c->L.occ);
+  a.psi_sp = c->g.sp ? c->psi32() : nullptr;
   a.rho = rho; a.j = j; a.jline = c->at<double>(c->L.jline);
   a.base = base_dev; a.jbase = base_dev + c->g.ndom; a.sx = sx; a.sy = sy; a.jstride = jstride;
   a.v = energy ? c->at<double>(c->L.vstage) : nullptr;
@@ -571,7 +610,7 @@ ScLayout sc_layout(const Geometry& g, const lfd_sc_config* sc, size_t fft_bytes)
   L.snap_n = take((size_t)g.ndom * g.norb * d8);
   L.fft_bytes = fft_bytes;
   L.fftwork = take(fft_bytes);
-  L.psi_save = sc->n_corr > 0 ? take((size_t)g.ndom * g.ng * g.norb * c16) : 0;
+  L.psi_save = sc->n_corr > 0 ? take((size_t)g.ndom * g.ng * g.norb * (g.sp ? 8 : c16)) : 0;
   L.total = o;
   return L;
 }
@@ -638,7 +677,7 @@ lfd_status sc_set_v(lfd_ctx* c, const double* va, double wa, const double* vb, d
     return lfd::launch_sc_vmid(c->g, S.vion, va, vb, wa, wb, S.at<int>(S.L.off), S.gd[1], S.gd[2], vst, c->stream);
   }));
   return launch(c, LFD_K_PHASE, "k_phase",
-                [&] { return lfd::launch_phase(c->g, vst, c->phi(), vst, c->scaled, c->stream); });
+                [&] { return phase_any(c, vst, vst); });
 }
 
 void sc_release(ScState& S) {
@@ -674,8 +713,9 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   if (!psi || !workspace || !occ) return fail(nullptr, LFD_EINVAL, "psi, workspace and occ must be non-NULL");
   if ((cfg->nproj > 0) != (proj != nullptr)) return fail(nullptr, LFD_EINVAL, "proj must be non-NULL iff nproj > 0");
   if (cfg->nproj > 0 && !dnl) return fail(nullptr, LFD_EINVAL, "dnl must be non-NULL when nproj > 0");
-  if ((reinterpret_cast<uintptr_t>(psi) | reinterpret_cast<uintptr_t>(proj)) & 15)
-    return fail(nullptr, LFD_EINVAL, "psi / proj must be 16-byte aligned");
+  const uintptr_t amask = (cfg->flags & LFD_FLAG_SP) ? 7 : 15;
+  if ((reinterpret_cast<uintptr_t>(psi) | reinterpret_cast<uintptr_t>(proj)) & amask)
+    return fail(nullptr, LFD_EINVAL, "psi / proj must be aligned to their complex element (16 B, or 8 B with LFD_FLAG_SP)");
   if (reinterpret_cast<uintptr_t>(workspace) & (kAlign - 1))
     return fail(nullptr, LFD_EINVAL, "workspace must be 256-byte aligned");
   int ndev = 0;
@@ -695,6 +735,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   cudaError_t e = lfd::gemm_set_attributes();
   if (e == cudaSuccess) e = lfd::density_set_attributes();
   if (e == cudaSuccess) e = lfd::kin_yz_set_attributes();
+  if (e == cudaSuccess) e = lfd::gemm_sp_set_attributes();
   if (e != cudaSuccess) return cuda_fail(nullptr, e, "cudaFuncSetAttribute");
 
   lfd_ctx* c = new (std::nothrow) lfd_ctx();
@@ -712,7 +753,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   if (const char* v = std::getenv("LFD_KIN_FUSED")) c->kin_fused = std::atoi(v) != 0;
   if (const char* v = std::getenv("LFD_KIN_SCALED")) c->scaled = std::atoi(v) != 0;
   c->scaled = c->scaled && lfd::kin_scaled_ok(g);
-  c->kin_fused = c->kin_fused && lfd::kin_yz_supported(g);
+  c->kin_fused = c->kin_fused && lfd::kin_yz_supported(g) && !g.sp;
   c->dmaps = lfd::density_maps_create(g, c->psi, active_orbitals(g, occ));
   if (c->kin_fused && lfd::kin_yz_tensor_map(g, c->psi, &c->psi_tmap) != cudaSuccess) {
     cudaGetLastError();
@@ -747,7 +788,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   e = cudaMemsetAsync(c->at<double>(L.vstage), 0, sizeof(double) * g.ndom * g.ng, c->stream);
   if (e != cudaSuccess) { cuda_fail(c, e, "memset"); return bail(LFD_ECUDA); }
   lfd_status s2 = launch(c, LFD_K_PHASE, "k_phase",
-                         [&] { return lfd::launch_phase(g, c->at<double>(L.vstage), c->phi(), c->at<double>(L.vstage), c->scaled, c->stream); });
+                         [&] { return phase_any(c, c->at<double>(L.vstage), c->at<double>(L.vstage)); });
   if (s2 != LFD_OK) return bail(s2);
   s2 = set_A(c, nullptr);
   if (s2 != LFD_OK) return bail(s2);
@@ -758,7 +799,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
     a1.ndom = g.ndom; a1.mrows = g.nproj; a1.ncols = g.nproj; a1.nsplit = L.nsplit;
     a1.ng = g.ng; a1.rows_per_split = L.rows_per_split;
     a1.a_dom_stride = g.ng * g.nproj; a1.x_dom_stride = g.ng * g.nproj;
-    s2 = launch(c, LFD_K_NL_PROJ, "k_gemm1(G)", [&] { return lfd::launch_gemm1(a1, c->stream); });
+    s2 = launch(c, LFD_K_NL_PROJ, "k_gemm1(G)", [&] { return gemm1_any(c, a1); });
     if (s2 != LFD_OK) return bail(s2);
     lfd::ReduceArgs r{};
     r.part = a1.part; r.normp = nullptr; r.D = nullptr; r.out = c->at<double2>(L.G); r.cprime = nullptr; r.s = nullptr;
@@ -783,7 +824,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
             const double2 x = Gh[((size_t)d * g.nproj + u) * g.nproj + v];
             dev = std::max(dev, std::hypot(x.x - (u == v ? 1.0 : 0.0), x.y));
           }
-      if (dev > 1e-9) {
+      if (dev > (g.sp ? 1e-5 : 1e-9)) {  // SP: B is orthonormal to FP32 rounding only
         c->err = "LFD_FLAG_EXACT_NL needs dV-orthonormal projector columns (max |dV B^H B - I| = " +
                  std::to_string(dev) + ")";
         return bail(LFD_EINVAL);
@@ -817,7 +858,7 @@ lfd_status lfd_set_potential(lfd_ctx* c, const double* vloc) {
   DeviceGuard dg(c->device);
   if (!is_device_ptr(vloc)) return fail(c, LFD_EINVAL, "vloc must be device memory (use lfd_set_potential_host)");
   return launch(c, LFD_K_PHASE, "k_phase", [&] {
-    return lfd::launch_phase(c->g, vloc, c->phi(), c->at<double>(c->L.vstage), c->scaled, c->stream);
+    return phase_any(c, vloc, c->at<double>(c->L.vstage));
   });
 }
 
@@ -829,7 +870,7 @@ lfd_status lfd_set_potential_host(lfd_ctx* c, const double* vloc_host) {
   cudaError_t e = cudaMemcpyAsync(stage, vloc_host, sizeof(double) * c->g.ndom * c->g.ng, cudaMemcpyHostToDevice,
                                   c->stream);
   if (e != cudaSuccess) return cuda_fail(c, e, "H2D vloc");
-  return launch(c, LFD_K_PHASE, "k_phase", [&] { return lfd::launch_phase(c->g, stage, c->phi(), stage, c->scaled, c->stream); });
+  return launch(c, LFD_K_PHASE, "k_phase", [&] { return phase_any(c, stage, stage); });
 }
 
 lfd_status lfd_set_vector_potential(lfd_ctx* c, const double* A) {
@@ -954,7 +995,8 @@ lfd_status lfd_remap_occ(lfd_ctx* c, const void* ref, int32_t nref, double* occ_
   LFD_TRY(check_ctx(c));
   if (!ref || !occ_out) return fail(c, LFD_EINVAL, "ref and occ_out must be non-NULL");
   if (nref < 1 || nref > c->L.nref_cap) return fail(c, LFD_EINVAL, "nref must be in [1, nref_max]");
-  if (reinterpret_cast<uintptr_t>(ref) & 15) return fail(c, LFD_EINVAL, "ref must be 16-byte aligned");
+  if (reinterpret_cast<uintptr_t>(ref) & (c->celem() - 1))
+    return fail(c, LFD_EINVAL, "ref must be aligned to its complex element (16 B; 8 B with LFD_FLAG_SP)");
   DeviceGuard dg(c->device);
   if (!is_device_ptr(ref) || !is_device_ptr(occ_out)) return fail(c, LFD_EINVAL, "ref / occ_out must be device memory");
   double2* C = c->at<double2>(c->L.cref);
@@ -1086,7 +1128,7 @@ lfd_status lfd_sc_step(lfd_ctx* c, int32_t nsteps, const double* Aext) {
   const Geometry& g = c->g;
   const bool maxwell = S.flags & LFD_SC_MAXWELL;
   double* state = S.at<double>(S.L.state);
-  const size_t psi_bytes = (size_t)g.ndom * g.ng * g.norb * 16;
+  const size_t psi_bytes = (size_t)g.ndom * g.ng * g.norb * c->celem();
   const size_t cbytes = (size_t)g.ndom * g.nproj * g.norb * 16, nbytes = (size_t)g.ndom * g.norb * 8;
   auto cpy = [&](void* dst, const void* src, size_t n) -> lfd_status {
     cudaError_t e = cudaMemcpyAsync(dst, src, n, cudaMemcpyDeviceToDevice, c->stream);

@@ -25,6 +25,7 @@ namespace lfd {
 constexpr int kSub = 8, kTY = 2, kTZ = 8, kXC = 10;
 constexpr int kDensThreads = kSub * kTY * kTZ;  // 128
 
+template <class C>
 __global__ void __launch_bounds__(kDensThreads) k_density(Geometry g, DensArgs a, int ntz, int nty, int nxc) {
   __shared__ double jsh[5][kDensThreads / kSub];
   const int dom = blockIdx.y;
@@ -41,7 +42,9 @@ __global__ void __launch_bounds__(kDensThreads) k_density(Geometry g, DensArgs a
   const bool has_z = valid && (per || z + 1 < g.nz);
   const int yp = (y + 1 >= g.ny) ? 0 : y + 1;
   const int zp = (z + 1 >= g.nz) ? 0 : z + 1;
-  const double2* P = a.psi + (long long)dom * g.ng * norb;
+  // the SP variant (complex64 Psi) reads float2 and accumulates in FP64
+  const C* P = reinterpret_cast<const C*>(sizeof(C) == 8 ? (const void*)a.psi_sp : (const void*)a.psi) +
+               (long long)dom * g.ng * norb;
   const double* f = a.occ + (long long)dom * norb;
   const DomCoef* cf = a.coef + dom;
   const double2 ex = cf->eth[0], ey = cf->eth[1], ez = cf->eth[2];
@@ -60,20 +63,20 @@ __global__ void __launch_bounds__(kDensThreads) k_density(Geometry g, DensArgs a
 #pragma unroll 4
       for (int s = q; s < norb; s += kSub) {
         const double fs = __ldg(f + s);
-        const double2 v = __ldg(P + r * norb + s);
+        const double2 v = to_d2(__ldg(P + r * norb + s));
         rho = fma(fs, fma(v.x, v.x, v.y * v.y), rho);
         if (has_x) {
-          const double2 w = cconjmul(v, __ldg(P + rx * norb + s));
+          const double2 w = cconjmul(v, to_d2(__ldg(P + rx * norb + s)));
           pxr = fma(fs, w.x, pxr);
           pxi = fma(fs, w.y, pxi);
         }
         if (has_y) {
-          const double2 w = cconjmul(v, __ldg(P + ry * norb + s));
+          const double2 w = cconjmul(v, to_d2(__ldg(P + ry * norb + s)));
           pyr = fma(fs, w.x, pyr);
           pyi = fma(fs, w.y, pyi);
         }
         if (has_z) {
-          const double2 w = cconjmul(v, __ldg(P + rz * norb + s));
+          const double2 w = cconjmul(v, to_d2(__ldg(P + rz * norb + s)));
           pzr = fma(fs, w.x, pzr);
           pzi = fma(fs, w.y, pzi);
         }
@@ -321,15 +324,16 @@ struct DensMaps {
   int px;            // x planes per CTA (divides nx)
   int nyc;           // y chunks per (plane group, z chunk)
   int nact;          // active orbitals: 1 + the last index with f != 0 (f = 0 contributes exactly 0)
+  int esz;           // bytes per complex value: 16 (complex128) or 8 (complex64, the SP variant)
 };
 
 // shared-memory layout of the y-marching kernel (every TMA destination 128-byte aligned): an own slot
 // holds px (segment, halo point) pairs
 struct YLayout {
   size_t seg_b, halo_b, pl_b, own_b, xp_b, fsh_off, bar_off, total;
-  __host__ __device__ YLayout(int zc, int norb, int px) {
-    seg_b = ((size_t)zc * norb * 16 + 127) & ~(size_t)127;
-    halo_b = ((size_t)norb * 16 + 127) & ~(size_t)127;
+  __host__ __device__ YLayout(int zc, int norb, int px, int esz = 16) {  // esz: bytes per complex value
+    seg_b = ((size_t)zc * norb * esz + 127) & ~(size_t)127;
+    halo_b = ((size_t)norb * esz + 127) & ~(size_t)127;
     pl_b = seg_b + halo_b;
     own_b = px * pl_b;
     xp_b = seg_b;
@@ -347,6 +351,7 @@ struct YShape {
 static YShape ymarch_shape(const Geometry& g) {
   YShape sh{0, 1, 1};
   if (g.norb > 128) return sh;
+  if (g.sp && (g.norb & 1)) return sh;  // TMA global strides must be multiples of 16 bytes
   int zmax = 18, pxmax = 1, yc = 1;  // measured on C2 (tools/dens_tune.sh): 1 plane, 18 points
   if (const char* v = std::getenv("LFD_DENS_ZCMAX")) zmax = std::max(1, std::min(60, std::atoi(v)));
   if (const char* v = std::getenv("LFD_DENS_PX")) pxmax = std::max(1, std::atoi(v));
@@ -375,17 +380,17 @@ static YShape ymarch_shape(const Geometry& g) {
   return sh;
 }
 
-template <bool kPer, int kIt>
+template <bool kPer, int kIt, class C = double2>
 __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constant__ DensMaps mp, Geometry g,
                                                             DensArgs a) {
   extern __shared__ __align__(128) unsigned char dsm[];
   const int norb = mp.nact, zc = mp.zc, px = mp.px;  // smem rows hold the nact active orbitals of each point
-  const YLayout Ly(zc, norb, px);
-  auto own_seg = [&](int s, int p) { return reinterpret_cast<double2*>(dsm + s * Ly.own_b + p * Ly.pl_b); };
+  const YLayout Ly(zc, norb, px, (int)sizeof(C));
+  auto own_seg = [&](int s, int p) { return reinterpret_cast<C*>(dsm + s * Ly.own_b + p * Ly.pl_b); };
   auto halo_of = [&](int s, int p) {
-    return reinterpret_cast<double2*>(dsm + s * Ly.own_b + p * Ly.pl_b + Ly.seg_b);
+    return reinterpret_cast<C*>(dsm + s * Ly.own_b + p * Ly.pl_b + Ly.seg_b);
   };
-  auto xp_slot = [&](int s) { return reinterpret_cast<double2*>(dsm + kYOwn * Ly.own_b + s * Ly.xp_b); };
+  auto xp_slot = [&](int s) { return reinterpret_cast<C*>(dsm + kYOwn * Ly.own_b + s * Ly.xp_b); };
   double* fsh = reinterpret_cast<double*>(dsm + Ly.fsh_off);
   uint64_t* bars = reinterpret_cast<uint64_t*>(dsm + Ly.bar_off);
   uint64_t *ofull = bars, *oempty = bars + kYOwn, *xfull = bars + 2 * kYOwn, *xempty = xfull + kYXp;
@@ -420,7 +425,7 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
         if (k >= kYOwn) mbar_wait(&oempty[s], (uint32_t)(((k / kYOwn) - 1) & 1));
         const int yy = (y0 + k == g.ny) ? 0 : y0 + k;
         const bool halo = !last_chunk || per;  // z+1 halo point: z0 + zc, or z = 0 (periodic wrap)
-        mbar_expect_tx(&ofull[s], (uint32_t)(px * (zc + (halo ? 1 : 0)) * norb * 16));
+        mbar_expect_tx(&ofull[s], (uint32_t)(px * (zc + (halo ? 1 : 0)) * norb * (int)sizeof(C)));
         for (int p = 0; p < px; ++p) {
           const int row = (dom * g.nx + xb + p) * g.ny + yy;
           tma_3d(own_seg(s, p), &mp.seg, 0, z0, row, &ofull[s]);
@@ -430,7 +435,7 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
       auto issue_xp = [&](int k) {
         const int s = k % kYXp;
         if (k >= kYXp) mbar_wait(&xempty[s], (uint32_t)(((k / kYXp) - 1) & 1));
-        mbar_expect_tx(&xfull[s], (uint32_t)(zc * norb * 16));
+        mbar_expect_tx(&xfull[s], (uint32_t)(zc * norb * (int)sizeof(C)));
         tma_3d(xp_slot(s), &mp.seg, 0, z0, rowxn + y0 + k, &xfull[s]);
       };
       issue_own(0);
@@ -473,10 +478,10 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
     if (k + 1 < nown) mbar_wait(&ofull[sn], (uint32_t)(((k + 1) / kYOwn) & 1));
     if (has_xn) mbar_wait(&xfull[sx], (uint32_t)((k / kYXp) & 1));
     const int plr = valid ? pl : 0;
-    const double2* O = own_seg(so, plr) + ptr * norb;
-    const double2* Oz = (ptr + 1 < zc) ? O + norb : halo_of(so, plr);  // point z+1
-    const double2* N = own_seg(sn, plr) + ptr * norb;
-    const double2* X = (plr + 1 < px ? own_seg(so, plr + 1) : xp_slot(sx)) + ptr * norb;  // plane x+1
+    const C* O = own_seg(so, plr) + ptr * norb;
+    const C* Oz = (ptr + 1 < zc) ? O + norb : halo_of(so, plr);  // point z+1
+    const C* N = own_seg(sn, plr) + ptr * norb;
+    const C* X = (plr + 1 < px ? own_seg(so, plr + 1) : xp_slot(sx)) + ptr * norb;  // plane x+1
     // per-lane partial sums over this lane's orbitals: rho and the three link products P_d = sum f
     // conj(psi_r) psi_{r+e_d} (f folded into fv = f psi_r)
     double rho = 0.0, pxr = 0.0, pxi = 0.0, pyr = 0.0, pyi = 0.0, pzr = 0.0, pzi = 0.0;
@@ -485,21 +490,21 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
       for (int i = 0; i < (kIt > 0 ? kIt : kItMax); ++i) {
         if (kIt == 0 && i >= nit) break;
         const int sidx = q + i * kSub;
-        const double2 v = O[sidx];
+        const double2 v = to_d2(O[sidx]);  // FP64 accumulation (also for complex64 Psi)
         const double2 fv = make_double2(fr[i] * v.x, fr[i] * v.y);
         rho = fma(fv.x, v.x, fma(fv.y, v.y, rho));
         if (kPer || has_x) {
-          const double2 w = X[sidx];
+          const double2 w = to_d2(X[sidx]);
           pxr = fma(fv.x, w.x, fma(fv.y, w.y, pxr));
           pxi = fma(fv.x, w.y, fma(-fv.y, w.x, pxi));
         }
         if (kPer || has_y) {
-          const double2 w = N[sidx];
+          const double2 w = to_d2(N[sidx]);
           pyr = fma(fv.x, w.x, fma(fv.y, w.y, pyr));
           pyi = fma(fv.x, w.y, fma(-fv.y, w.x, pyi));
         }
         if (kPer || has_z) {
-          const double2 w = Oz[sidx];
+          const double2 w = to_d2(Oz[sidx]);
           pzr = fma(fv.x, w.x, fma(fv.y, w.y, pzr));
           pzi = fma(fv.x, w.y, fma(-fv.y, w.x, pzi));
         }
@@ -574,13 +579,16 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
   }
 }
 
-static size_t ymarch_smem(int zc, int nact, int px) { return YLayout(zc, nact, px).total; }
+static size_t ymarch_smem(int zc, int nact, int px, int esz) { return YLayout(zc, nact, px, esz).total; }
 
+// Psi as a 3-D tensor of 8-byte elements [rows][nz][norb * esz / 8] (the TMA only moves bytes: a
+// complex64 value is one 8-byte element, a complex128 value two).
 static cudaError_t density_maps_encode(DensMaps* m, const Geometry& g, const double2* psi, int nact) {
-  const uint64_t dims[3] = {(uint64_t)2 * g.norb, (uint64_t)g.nz, (uint64_t)g.ndom * g.nx * g.ny};
-  const uint64_t str[2] = {(uint64_t)g.norb * 16, (uint64_t)g.nz * g.norb * 16};
-  const uint32_t b2[3] = {(uint32_t)(2 * nact), (uint32_t)m->zc, 1};
-  const uint32_t b3[3] = {(uint32_t)(2 * nact), 1, 1};
+  const uint64_t w = (uint64_t)m->esz / 8;
+  const uint64_t dims[3] = {w * g.norb, (uint64_t)g.nz, (uint64_t)g.ndom * g.nx * g.ny};
+  const uint64_t str[2] = {(uint64_t)g.norb * m->esz, (uint64_t)g.nz * g.norb * m->esz};
+  const uint32_t b2[3] = {(uint32_t)(w * nact), (uint32_t)m->zc, 1};
+  const uint32_t b3[3] = {(uint32_t)(w * nact), 1, 1};
   cudaError_t e = encode_tmap_f64(&m->seg, 3, psi, dims, str, b2);
   if (e == cudaSuccess) e = encode_tmap_f64(&m->one, 3, psi, dims, str, b3);
   if (e == cudaSuccess) m->nact = nact;
@@ -595,6 +603,7 @@ DensMaps* density_maps_create(const Geometry& g, const double2* psi, int nact) {
   m->zc = sh.zc;
   m->px = sh.px;
   m->nyc = sh.nyc;
+  m->esz = g.sp ? 8 : 16;
   if (density_maps_encode(m, g, psi, std::min(std::max(nact, 1), g.norb)) != cudaSuccess) {
     delete m;
     return nullptr;
@@ -623,7 +632,16 @@ cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps*
   dim3 grid(density_blocks(g), g.ndom);
   if (maps) {
     const int threads = ((maps->zc * maps->px * kSub + 31) / 32 + 1) * 32;
-    const size_t sm = ymarch_smem(maps->zc, maps->nact, maps->px);
+    const size_t sm = ymarch_smem(maps->zc, maps->nact, maps->px, maps->esz);
+    if (maps->esz == 8) {  // SP variant (complex64 Psi)
+      if (g.bc == 0 && maps->nact == 32)
+        k_density_y<true, 4, float2><<<grid, threads, sm, st>>>(*maps, g, a);
+      else if (g.bc == 0)
+        k_density_y<true, 0, float2><<<grid, threads, sm, st>>>(*maps, g, a);
+      else
+        k_density_y<false, 0, float2><<<grid, threads, sm, st>>>(*maps, g, a);
+      return cudaGetLastError();
+    }
     if (g.bc == 0 && maps->nact == 64)
       k_density_y<true, 8><<<grid, threads, sm, st>>>(*maps, g, a);
     else if (g.bc == 0 && maps->nact == 32)
@@ -636,10 +654,12 @@ cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps*
   }
   if (ymarch_shape(g).zc > 0) return cudaErrorInvalidValue;  // the block layout expects the y-marching kernel
   const int ntz = (g.nz + kTZ - 1) / kTZ, nty = (g.ny + kTY - 1) / kTY;
-  if (g.norb <= kMaxNorbTma)
+  if (a.psi_sp)
+    k_density<float2><<<grid, kDensThreads, 0, st>>>(g, a, ntz, nty, kXC);
+  else if (g.norb <= kMaxNorbTma)
     k_density_tma<<<grid, kDensThreads, density_smem_bytes(g.norb), st>>>(g, a, ntz, nty, kXC);
   else
-    k_density<<<grid, kDensThreads, 0, st>>>(g, a, ntz, nty, kXC);
+    k_density<double2><<<grid, kDensThreads, 0, st>>>(g, a, ntz, nty, kXC);
   return cudaGetLastError();
 }
 
@@ -648,6 +668,10 @@ cudaError_t density_set_attributes() {
                                        density_smem_bytes(kMaxNorbTma));
   if (e != cudaSuccess) return e;
   for (auto f : {k_density_y<true, 8>, k_density_y<true, 4>, k_density_y<true, 0>, k_density_y<false, 0>}) {
+    e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024);
+    if (e != cudaSuccess) return e;
+  }
+  for (auto f : {k_density_y<true, 4, float2>, k_density_y<true, 0, float2>, k_density_y<false, 0, float2>}) {
     e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024);
     if (e != cudaSuccess) return e;
   }

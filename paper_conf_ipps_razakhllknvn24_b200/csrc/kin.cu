@@ -48,14 +48,15 @@ cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int co
 // Phi(r) = e^{-i (Delta/2) v_loc(r)} (Strang placement of the potential, reading R7), times the
 // constant sqrt(g) of the scaled pair form (1 for the general form).
 // The kernel also keeps a copy of v_loc for lfd_energy (vcopy may alias v: then it is not written).
-__global__ void k_phase(const double* __restrict__ v, double2* __restrict__ phi, double* vcopy, long long n,
+template <class C>
+__global__ void k_phase(const double* __restrict__ v, C* __restrict__ phi, double* vcopy, long long n,
                         double half_dt, double2 sg) {
   long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   const double vi = v[i];
   double s, c;
   sincos(half_dt * vi, &s, &c);
-  phi[i] = cmul(make_double2(c, -s), sg);
+  phi[i] = from_d2<C>(cmul(make_double2(c, -s), sg));  // FP64, rounded once for the SP variant
   if (vcopy != v) vcopy[i] = vi;
 }
 
@@ -86,16 +87,26 @@ cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, doubl
                          cudaStream_t st) {
   long long n = g.ng * g.ndom;
   const double2 sg = scaled ? scaled_sqrt_g(g) : make_double2(1.0, 0.0);
-  k_phase<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(v, phi, vcopy, n, 0.5 * g.dt, sg);
+  k_phase<double2><<<(unsigned)((n + 255) / 256), 256, 0, st>>>(v, phi, vcopy, n, 0.5 * g.dt, sg);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_phase_sp(const Geometry& g, const double* v, float2* phi, double* vcopy, bool scaled,
+                            cudaStream_t st) {
+  long long n = g.ng * g.ndom;
+  const double2 sg = scaled ? scaled_sqrt_g(g) : make_double2(1.0, 0.0);
+  k_phase<float2><<<(unsigned)((n + 255) / 256), 256, 0, st>>>(v, phi, vcopy, n, 0.5 * g.dt, sg);
   return cudaGetLastError();
 }
 
 // ---- pair blocks -------------------------------------------------------------------------------
 // Coefficients of one axis for tau = Delta/2 (1) and Delta (2). General form: a = alpha, u = up,
 // d = dn, s = onsite. Scaled form: u = w_up, d = w_dn, s = (1/c, 0), a unused.
-struct PairCoef {
-  double2 a1, u1, d1, s1, a2, u2, d2, s2;
+template <class C>
+struct PairCoefT {
+  C a1, u1, d1, s1, a2, u2, d2, s2;
 };
+using PairCoef = PairCoefT<double2>;
 
 template <bool kS>
 __device__ __forceinline__ PairCoef pair_coef(const DomCoef* cf, int axis) {
@@ -111,34 +122,62 @@ __device__ __forceinline__ PairCoef pair_coef(const DomCoef* cf, int axis) {
   return c;
 }
 
+// The SP variant (complex64 Psi) runs the same sweeps in FP32 with the coefficients
+// rounded once from the FP64 table.
+template <bool kS, class C>
+__device__ __forceinline__ PairCoefT<C> pair_coef_t(const DomCoef* cf, int axis) {
+  const PairCoef d = pair_coef<kS>(cf, axis);
+  PairCoefT<C> c;
+  c.a1 = from_d2<C>(d.a1); c.u1 = from_d2<C>(d.u1); c.d1 = from_d2<C>(d.d1); c.s1 = from_d2<C>(d.s1);
+  c.a2 = from_d2<C>(d.a2); c.u2 = from_d2<C>(d.u2); c.d2 = from_d2<C>(d.d2); c.s2 = from_d2<C>(d.s2);
+  return c;
+}
+
 // x + w y
 __device__ __forceinline__ double2 padd(double2 w, double2 x, double2 y) {
   return make_double2(fma(w.x, y.x, fma(-w.y, y.y, x.x)), fma(w.x, y.y, fma(w.y, y.x, x.y)));
 }
-// Left / right output of a link (x at the left point, y at the right point) and a singleton.
-template <bool kS>
-__device__ __forceinline__ double2 lk_L(double2 a, double2 u, double2 x, double2 y) {
+__device__ __forceinline__ float2 padd(float2 w, float2 x, float2 y) {
+  return make_float2(fmaf(w.x, y.x, fmaf(-w.y, y.y, x.x)), fmaf(w.x, y.y, fmaf(w.y, y.x, x.y)));
+}
+// Two adjacent orbitals of one grid point (the SP passes move 16 bytes per lane, like the FP64 ones).
+struct __align__(16) cf2 {
+  float2 a, b;
+};
+__device__ __forceinline__ cf2 padd(float2 w, cf2 x, cf2 y) { return {padd(w, x.a, y.a), padd(w, x.b, y.b)}; }
+__device__ __forceinline__ cf2 cmul(float2 s, cf2 x) { return {cmul(s, x.a), cmul(s, x.b)}; }
+__device__ __forceinline__ cf2 crow(float2 a, cf2 x, float2 b, cf2 y) {
+  return {crow(a, x.a, b, y.a), crow(a, x.b, b, y.b)};
+}
+__device__ __forceinline__ double2 rscale(double r, double2 x) { return make_double2(r * x.x, r * x.y); }
+__device__ __forceinline__ float2 rscale(float r, float2 x) { return make_float2(r * x.x, r * x.y); }
+__device__ __forceinline__ cf2 rscale(float r, cf2 x) { return {rscale(r, x.a), rscale(r, x.b)}; }
+
+// Left / right output of a link (x at the left point, y at the right point) and a singleton; coefficients
+// of type C, values of type V (V = C, or two complex64 orbitals for the SP passes).
+template <bool kS, class C, class V>
+__device__ __forceinline__ V lk_L(C a, C u, V x, V y) {
   return kS ? padd(u, x, y) : crow(a, x, u, y);
 }
-template <bool kS>
-__device__ __forceinline__ double2 lk_R(double2 a, double2 d, double2 x, double2 y) {
+template <bool kS, class C, class V>
+__device__ __forceinline__ V lk_R(C a, C d, V x, V y) {
   return kS ? padd(d, y, x) : crow(d, x, a, y);
 }
-template <bool kS>
-__device__ __forceinline__ double2 lk_S(double2 s, double2 x) {
-  return kS ? make_double2(s.x * x.x, s.x * x.y) : cmul(s, x);
+template <bool kS, class C, class V>
+__device__ __forceinline__ V lk_S(C s, V x) {
+  return kS ? rscale(s.x, x) : cmul(s, x);
 }
 
 // Streaming K_d along one line, fed one pair (2p, 2p+1) at a time: first E(Delta/2) on the new pair,
 // O(Delta) on the link (2p-1, 2p), second E(Delta/2) on (2p-2, 2p-1) once both its O outputs exist;
 // points 0, 1 wait for the wrap link (n-1, 0) at the end.
-template <bool kS>
+template <bool kS, class C = double2, class V = C>
 struct LineMarch {
-  double2 E10, O1, prev_e1, prev_oR;
-  __device__ __forceinline__ void init() { E10 = O1 = prev_e1 = prev_oR = cz(); }
+  V E10, O1, prev_e1, prev_oR;
+  __device__ __forceinline__ void init() { E10 = O1 = prev_e1 = prev_oR = V{}; }
   template <class St>
-  __device__ __forceinline__ void push(const PairCoef& c, int p, double2 a, double2 b, bool pair, St&& st) {
-    double2 e0, e1 = cz();
+  __device__ __forceinline__ void push(const PairCoefT<C>& c, int p, V a, V b, bool pair, St&& st) {
+    V e0, e1 = V{};
     if (pair) {
       e0 = lk_L<kS>(c.a1, c.u1, a, b);
       e1 = lk_R<kS>(c.a1, c.d1, a, b);
@@ -148,8 +187,8 @@ struct LineMarch {
     if (p == 0) {
       E10 = e0;
     } else {
-      const double2 oL = lk_L<kS>(c.a2, c.u2, prev_e1, e0);
-      const double2 oR = lk_R<kS>(c.a2, c.d2, prev_e1, e0);
+      const V oL = lk_L<kS>(c.a2, c.u2, prev_e1, e0);
+      const V oR = lk_R<kS>(c.a2, c.d2, prev_e1, e0);
       if (p == 1) {
         O1 = oL;
       } else {
@@ -161,30 +200,30 @@ struct LineMarch {
     prev_e1 = e1;
   }
   // The three phases of push() without the p tests (p == 0, p == 1, p >= 2 with a full pair).
-  __device__ __forceinline__ void first(const PairCoef& c, double2 a, double2 b) {
+  __device__ __forceinline__ void first(const PairCoefT<C>& c, V a, V b) {
     E10 = lk_L<kS>(c.a1, c.u1, a, b);
     prev_e1 = lk_R<kS>(c.a1, c.d1, a, b);
   }
-  __device__ __forceinline__ void second(const PairCoef& c, double2 a, double2 b) {
-    const double2 e0 = lk_L<kS>(c.a1, c.u1, a, b);
+  __device__ __forceinline__ void second(const PairCoefT<C>& c, V a, V b) {
+    const V e0 = lk_L<kS>(c.a1, c.u1, a, b);
     O1 = lk_L<kS>(c.a2, c.u2, prev_e1, e0);
     prev_oR = lk_R<kS>(c.a2, c.d2, prev_e1, e0);
     prev_e1 = lk_R<kS>(c.a1, c.d1, a, b);
   }
   template <class St>
-  __device__ __forceinline__ void steady(const PairCoef& c, double2 a, double2 b, St&& st) {
-    const double2 e0 = lk_L<kS>(c.a1, c.u1, a, b);
-    const double2 oL = lk_L<kS>(c.a2, c.u2, prev_e1, e0);
-    const double2 oR = lk_R<kS>(c.a2, c.d2, prev_e1, e0);
+  __device__ __forceinline__ void steady(const PairCoefT<C>& c, V a, V b, St&& st) {
+    const V e0 = lk_L<kS>(c.a1, c.u1, a, b);
+    const V oL = lk_L<kS>(c.a2, c.u2, prev_e1, e0);
+    const V oR = lk_R<kS>(c.a2, c.d2, prev_e1, e0);
     st(0, lk_L<kS>(c.a1, c.u1, prev_oR, oL));
     st(1, lk_R<kS>(c.a1, c.d1, prev_oR, oL));
     prev_oR = oR;
     prev_e1 = lk_R<kS>(c.a1, c.d1, a, b);
   }
   template <bool kPer, class St>
-  __device__ __forceinline__ void finish(const PairCoef& c, int n, St&& st) {
+  __device__ __forceinline__ void finish(const PairCoefT<C>& c, int n, St&& st) {
     if ((n & 1) == 0) {
-      double2 Olast, O0;
+      V Olast, O0;
       if (kPer) {  // wrap link (n-1, 0)
         Olast = lk_L<kS>(c.a2, c.u2, prev_e1, E10);
         O0 = lk_R<kS>(c.a2, c.d2, prev_e1, E10);
@@ -203,7 +242,7 @@ struct LineMarch {
       }
     } else {  // odd n (zero BC): last point is an E singleton; point 0 an O singleton
       st(n - 1, lk_S<kS>(c.s1, prev_oR));
-      const double2 O0 = lk_S<kS>(c.s2, E10);
+      const V O0 = lk_S<kS>(c.s2, E10);
       st(0, lk_L<kS>(c.a1, c.u1, O0, O1));
       st(1, lk_R<kS>(c.a1, c.d1, O0, O1));
     }
@@ -213,9 +252,11 @@ struct LineMarch {
 // One K_axis pass. Column c of domain blockIdx.y: outer = c / inner_len, inner = c % inner_len,
 // element offset = outer*outer_stride + inner; successive points of the line are pt_stride apart.
 // Loads run two pairs ahead of the pair being combined (memory-level parallelism for the HBM stream).
-template <bool kPeriodic, int kPhase, bool kS>
-__global__ void __launch_bounds__(256, 3) k_kin(double2* __restrict__ psi, const DomCoef* __restrict__ coef,
-                                             const double2* __restrict__ phi, int axis, int n, int pt_stride,
+// C: complex type of the coefficients and Phi; V: the value a lane moves per grid point (C, or cf2 = two
+// complex64 orbitals); strides and norb are in units of V.
+template <bool kPeriodic, int kPhase, bool kS, class C = double2, class V = C>
+__global__ void __launch_bounds__(256, 3) k_kin(V* __restrict__ psi, const DomCoef* __restrict__ coef,
+                                             const C* __restrict__ phi, int axis, int n, int pt_stride,
                                              int inner_len, int outer_stride, int ncols, int norb,
                                              long long dom_stride, long long ng) {
   int c = blockIdx.x * blockDim.x + threadIdx.x;
@@ -224,26 +265,26 @@ __global__ void __launch_bounds__(256, 3) k_kin(double2* __restrict__ psi, const
   const int outer = c / inner_len;
   const int inner = c - outer * inner_len;
   const int off = outer * outer_stride + inner;
-  double2* line = psi + dom * dom_stride + off;
-  const double2* ph = phi + dom * ng + off / norb;
+  V* line = psi + dom * dom_stride + off;
+  const C* ph = phi + dom * ng + off / norb;
   const int ph_stride = pt_stride / norb;
-  const PairCoef cf = pair_coef<kS>(coef + dom, axis);
+  const PairCoefT<C> cf = pair_coef_t<kS, C>(coef + dom, axis);
 
-  auto ld = [&](int i) -> double2 {
-    double2 v = line[(long long)i * pt_stride];
+  auto ld = [&](int i) -> V {
+    V v = line[(long long)i * pt_stride];
     if (kPhase == 1) v = cmul(ph[(long long)i * ph_stride], v);
     return v;
   };
-  auto st = [&](int i, double2 v) {
+  auto st = [&](int i, V v) {
     if (kPhase == 2) v = cmul(ph[(long long)i * ph_stride], v);
     line[(long long)i * pt_stride] = v;
   };
 
   const int P = (n + 1) >> 1;
-  LineMarch<kS> L;
+  LineMarch<kS, C, V> L;
   L.init();
   if (kPeriodic && n >= 6) {  // periodic (even n): first two pairs peeled, then a test-free steady loop
-    double2 a0 = ld(0), b0 = ld(1), a1 = ld(2), b1 = ld(3), a2 = ld(4), b2 = ld(5);
+    V a0 = ld(0), b0 = ld(1), a1 = ld(2), b1 = ld(3), a2 = ld(4), b2 = ld(5);
     L.first(cf, a0, b0);
     a0 = a1; b0 = b1; a1 = a2; b1 = b2;
     if (3 < P) { a2 = ld(6); b2 = ld(7); }
@@ -251,24 +292,24 @@ __global__ void __launch_bounds__(256, 3) k_kin(double2* __restrict__ psi, const
     for (int p = 2; p < P; ++p) {
       a0 = a1; b0 = b1; a1 = a2; b1 = b2;
       if (p + 2 < P) { a2 = ld(2 * p + 4); b2 = ld(2 * p + 5); }
-      L.steady(cf, a0, b0, [&](int k, double2 v) { st(2 * p - 2 + k, v); });
+      L.steady(cf, a0, b0, [&](int k, V v) { st(2 * p - 2 + k, v); });
     }
     L.template finish<kPeriodic>(cf, n, st);
     return;
   }
-  double2 na = ld(0), nb = (n > 1) ? ld(1) : cz();
-  double2 nc = cz(), nd = cz();
+  V na = ld(0), nb = (n > 1) ? ld(1) : V{};
+  V nc = V{}, nd = V{};
   if (P > 1) {
     nc = ld(2);
-    nd = (3 < n) ? ld(3) : cz();
+    nd = (3 < n) ? ld(3) : V{};
   }
   for (int p = 0; p < P; ++p) {
-    const double2 a = na, b = nb;
+    const V a = na, b = nb;
     na = nc;
     nb = nd;
     if (p + 2 < P) {
       nc = ld(2 * p + 4);
-      nd = (2 * p + 5 < n) ? ld(2 * p + 5) : cz();
+      nd = (2 * p + 5 < n) ? ld(2 * p + 5) : V{};
     }
     L.push(cf, p, a, b, 2 * p + 1 < n, st);
   }
@@ -546,10 +587,11 @@ cudaError_t launch_kin_yz(const Geometry& g, const CUtensorMap* tmap, double2* p
   return cudaGetLastError();
 }
 
-cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, const double2* phi, int axis,
-                       int phase_mode, bool scaled, cudaStream_t st) {
+template <class C, class V>
+static cudaError_t launch_kin_t(const Geometry& g, V* psi, const DomCoef* coef, const C* phi, int axis,
+                                int phase_mode, bool scaled, cudaStream_t st) {
   const int nd[3] = {g.nx, g.ny, g.nz};
-  const int norb = g.norb;
+  const int norb = g.norb / (int)(sizeof(V) / sizeof(C));  // values of type V per grid point
   int pt_stride, inner_len, outer_stride;
   if (axis == 0) {
     pt_stride = g.ny * g.nz * norb;
@@ -568,9 +610,9 @@ cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, con
   const int ncols = (int)(g.ng / n) * norb;
   dim3 grid((ncols + 255) / 256, g.ndom);
   const long long dom_stride = g.ng * norb;
-#define LFD_KIN(P, M, K)                                                                                    \
-  k_kin<P, M, K><<<grid, 256, 0, st>>>(psi, coef, phi, axis, n, pt_stride, inner_len, outer_stride, ncols, \
-                                       norb, dom_stride, g.ng)
+#define LFD_KIN(P, M, K)                                                                                       \
+  k_kin<P, M, K, C, V><<<grid, 256, 0, st>>>(psi, coef, phi, axis, n, pt_stride, inner_len, outer_stride, ncols, \
+                                          norb, dom_stride, g.ng)
 #define LFD_KIN_M(P, K) \
   if (phase_mode == 1) LFD_KIN(P, 1, K); else if (phase_mode == 2) LFD_KIN(P, 2, K); else LFD_KIN(P, 0, K)
   if (g.bc == 0) {
@@ -581,6 +623,18 @@ cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, con
 #undef LFD_KIN_M
 #undef LFD_KIN
   return cudaGetLastError();
+}
+
+cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, const double2* phi, int axis,
+                       int phase_mode, bool scaled, cudaStream_t st) {
+  return launch_kin_t<double2, double2>(g, psi, coef, phi, axis, phase_mode, scaled, st);
+}
+
+cudaError_t launch_kin_sp(const Geometry& g, float2* psi, const DomCoef* coef, const float2* phi, int axis,
+                          int phase_mode, bool scaled, cudaStream_t st) {
+  if (g.norb % 2 == 0 && (reinterpret_cast<uintptr_t>(psi) & 15) == 0)  // two orbitals (16 bytes) per lane
+    return launch_kin_t<float2, cf2>(g, reinterpret_cast<cf2*>(psi), coef, phi, axis, phase_mode, scaled, st);
+  return launch_kin_t<float2, float2>(g, psi, coef, phi, axis, phase_mode, scaled, st);
 }
 
 }  // namespace lfd

@@ -32,6 +32,7 @@ struct DomCoef {
 
 struct Geometry {
   int ndom, nx, ny, nz, norb, nproj, bc;
+  int sp;  // 1: SP variant (complex64 Psi / B, FP32 sweeps and 3xTF32 tensor-core GEMMs), else FP64
   double hx, hy, hz, dt, dV;
   long long ng;  // points per domain
 };
@@ -51,6 +52,8 @@ cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int co
 // Phi = e^{-i (Delta/2) v} (times sqrt(g) when the scaled pair form is used, kin.cu).
 cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, double* vcopy, bool scaled,
                          cudaStream_t st);
+cudaError_t launch_phase_sp(const Geometry& g, const double* v, float2* phi, double* vcopy, bool scaled,
+                            cudaStream_t st);
 // True when the scaled pair form applies (cos(tau t_d) >= 1/2 for every axis and tau).
 bool kin_scaled_ok(const Geometry& g);
 
@@ -58,6 +61,9 @@ bool kin_scaled_ok(const Geometry& g);
 // (phase_mode 1: Phi . psi before the sweep; 2: after).
 cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, const double2* phi,
                        int axis, int phase_mode, bool scaled, cudaStream_t st);
+// SP variant (complex64 Psi and Phi, FP32 sweeps)
+cudaError_t launch_kin_sp(const Geometry& g, float2* psi, const DomCoef* coef, const float2* phi,
+                          int axis, int phase_mode, bool scaled, cudaStream_t st);
 
 // Fused pass Psi <- Phi . K_y K_z Psi (one read + write of Psi; nz <= 80).
 bool kin_yz_supported(const Geometry& g);
@@ -135,6 +141,7 @@ cudaError_t gemm_set_attributes();
 // j component d at + d*jstride.
 struct DensArgs {
   const double2* psi;
+  const float2* psi_sp = nullptr;  // SP variant: complex64 Psi (then psi is unused)
   const DomCoef* coef;
   const double* occ;
   double* rho;
@@ -161,6 +168,14 @@ cudaError_t launch_energy_final(const Geometry& g, const double* epart, int bloc
                                 const double* D, const double* occ, double* E, cudaStream_t st);
 cudaError_t launch_remap(const Geometry& g, int nref, const double2* C, const double* occ, double* out,
                          cudaStream_t st);
+
+// SP variant projector GEMMs (nl_sp.cu; 3xTF32 on the warp-level tensor path). GEMM-1 takes the geometry
+// of a Gemm1Args (part / norms / sizes / strides) with complex64 operands A, X; GEMM-2 rounds C'' to
+// complex64 into X32 [ndom][nproj][norb] and updates psi in place.
+cudaError_t launch_gemm1_sp(const Gemm1Args& a, const float2* A, const float2* X, cudaStream_t st);
+cudaError_t launch_gemm2_sp(float2* psi, const float2* B, const double2* Cp, float2* X32, const double* nfac,
+                            int ndom, int nproj, int norb, long long ng, cudaStream_t st);
+cudaError_t gemm_sp_set_attributes();
 
 // Self-consistent step kernels (sc.cu, readings R23-R28).
 cudaError_t launch_sc_maxwell_begin(double* st, const double* a_mid, const double* a_end, double dt, bool maxwell,

@@ -20,6 +20,7 @@ LIB_PATH = os.path.join(HERE, "liblfd.so")
 LFD_ABI_VERSION = 4
 LFD_FLAG_NO_CARRY = 1
 LFD_FLAG_EXACT_NL = 2
+LFD_FLAG_SP = 4
 LFD_BC_PERIODIC = 0
 LFD_BC_ZERO = 1
 STATUS = {0: "LFD_OK", -1: "LFD_EINVAL", -2: "LFD_ENOMEM", -3: "LFD_ECUDA", -4: "LFD_ESTATE",
@@ -314,8 +315,12 @@ class Context:
 
     def __init__(self, psi, proj, dnl, occ, h, dt, bc=LFD_BC_PERIODIC, stream=None, nref_max=0, flags=0):
         import torch
-        if psi.dtype != torch.complex128 or psi.dim() != 5:
-            raise TypeError("psi must be complex128 [ndom, nx, ny, nz, norb]")
+        if psi.dtype not in (torch.complex128, torch.complex64) or psi.dim() != 5:
+            raise TypeError("psi must be complex128 (or complex64: the SP variant) [ndom, nx, ny, nz, norb]")
+        if proj is not None and proj.dtype != psi.dtype:
+            raise TypeError("proj must have psi's dtype")
+        if psi.dtype == torch.complex64:
+            flags |= LFD_FLAG_SP
         ndom, nx, ny, nz, norb = psi.shape
         nproj = 0 if proj is None else proj.shape[-1]
         self.cfg = make_config(ndom, nx, ny, nz, h[0], h[1], h[2], bc, norb, nproj, dt,

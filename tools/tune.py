@@ -4,6 +4,8 @@
 Prints one JSON line per value with the per-kernel-class device time per launch (ms).
 """
 import argparse
+
+import numpy as np
 import json
 import os
 import sys
@@ -18,6 +20,7 @@ def main():
     ap.add_argument("--values", nargs="+", required=True)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--config", default="C2")
+    ap.add_argument("--sp", action="store_true", help="the SP variant (complex64 Psi / B)")
     args = ap.parse_args()
     import torch
     from lfd_workloads import make_inputs, workload
@@ -26,6 +29,9 @@ def main():
     w = workload(args.config)
     x = make_inputs(w, seed=1)
     dev = torch.device("cuda:0")
+    if args.sp:
+        x.psi0 = x.psi0.astype(np.complex64)
+        x.proj = x.proj.astype(np.complex64) if w.nproj else None
     proj = torch.from_numpy(x.proj).to(dev) if w.nproj else None
     v = torch.from_numpy(x.vloc).to(dev)
     for val in args.values:
