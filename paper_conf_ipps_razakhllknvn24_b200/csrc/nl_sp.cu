@@ -5,10 +5,10 @@
 //   GEMM-2  psi[r][n] <- nfac[n] psi[r][n] + sum_m B[r][m] Xc[m][n]
 // in single precision on the tensor pipe: B200 has no FP32 tensor-core kind, so every real product runs as
 // 3xTF32 on the warp-level HMMA path (mma.sync m16n8k8 tf32, 279 TF/s measured on this pool vs 72 TF/s
-// FFMA, profiles/r01_sp_peaks.txt): x = hi + lo with hi = tf32(x), lo = tf32(x - hi), and
-// a b ~ hi_a hi_b + hi_a lo_b + lo_a hi_b (the dropped lo lo term is ~2^-22 relative), FP32 accumulation --
-// the accuracy of an FP32 GEMM. Complex products use 4 real products (the 3M form's extra cancellation is not
-// worth it at 24-bit precision). GEMM-1 writes its split partials in FP64, so the split reduction, the
+// FFMA, profiles/r01_sp_peaks.txt): x = hi + lo with hi = trunc_tf32(x), lo = x - hi, and
+// a b ~ hi_a hi_b + hi_a lo_b + lo_a hi_b (relative error ~2^-20 per product), FP32 accumulation -- close to
+// the accuracy of an FP32 GEMM. Complex products use the 3M form (3 real products; 9 HMMA per complex
+// tile-step instead of 12). GEMM-1 writes its split partials in FP64, so the split reduction, the
 // norm / carry / merge kernels and everything downstream of them are the FP64 kernels of nl.cu; GEMM-2
 // reads the coefficient X'' rounded to complex64 once per call (k_to_c64).
 // Operands are staged in shared memory by cp.async (8-byte, zero fill past the edges) in a 2-deep ring
@@ -35,16 +35,17 @@ __device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_grou
 __device__ __forceinline__ void cp_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
 __device__ __forceinline__ void cp_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 
+// 3xTF32 split of an FP32 operand: the tensor core reads only the top 19 bits of a tf32 operand (the low 13
+// mantissa bits are ignored: truncation), so hi = x itself acts as trunc(x), and lo = x - trunc(x) is exact
+// in FP32 (one LOP3 + one FADD per value).
 struct TF {
   unsigned hi, lo;
 };
 __device__ __forceinline__ TF split_tf32(float x) {
-  unsigned h, l;
-  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(h) : "f"(x));
-  const float r = x - __uint_as_float(h);
-  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(l) : "f"(r));
-  return {h, l};
+  const unsigned xb = __float_as_uint(x);
+  return {xb, __float_as_uint(x - __uint_as_float(xb & 0xffffe000u))};
 }
+__device__ __forceinline__ TF neg(TF v) { return {v.hi ^ 0x80000000u, v.lo ^ 0x80000000u}; }
 // Not volatile: the compiler may interleave the independent HMMAs of different accumulators.
 __device__ __forceinline__ void hmma(float* c, unsigned a0, unsigned a1, unsigned a2, unsigned a3, unsigned b0,
                                      unsigned b1) {
@@ -54,55 +55,52 @@ __device__ __forceinline__ void hmma(float* c, unsigned a0, unsigned a1, unsigne
       : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
 }
 
-// One k8 step of a warp tile of MT x NT (16 x 8) tiles, complex, 4 real products per complex product, each
-// in 3xTF32: a b ~ lo_a hi_b + hi_a lo_b + hi_a hi_b (small terms first).
+// One k8 step of a warp tile of MT x NT (16 x 8) tiles, complex, in the 3M form (three real products per
+// complex product), each real product in 3xTF32: a b ~ lo_a hi_b + hi_a lo_b + hi_a hi_b (small terms
+// first; lo_a lo_b ~ 2^-20 |ab| dropped).
 // a[mi][0..3]: complex A fragment (rows g, g+8, cols t, t+4), b[ni][0..1]: complex B fragment (k t, t+4).
-// kConj: A is conjugated (GEMM-1). Re += Ar Br -/+ Ai Bi, Im += Ar Bi +/- Ai Br.
-// Issue order: term-major, then product, then tile -- consecutive HMMAs update different accumulators
-// (2 MT NT of them), so the dependent updates of one accumulator are that many instructions apart.
+//   plain (GEMM-2): T1 = Ar Br, T2 = Ai Bi, T3 = (Ar + Ai)(Br + Bi);  Re = T1 - T2, Im = T3 - T1 - T2
+//   kConj (GEMM-1): T1 = Ar Br, T2 = Ai Bi, T3 = (Ar - Ai)(Br + Bi);  Re = T1 + T2, Im = T3 - T1 + T2
+// (cmma_finish forms Re, Im.) Issue order: term-major, then product, then tile, so consecutive HMMAs update
+// different accumulators.
 template <int MT, int NT, bool kConj>
-__device__ __forceinline__ void cmma_k8(float (&re)[MT][NT][4], float (&im)[MT][NT][4], const float2 (&a)[MT][4],
-                                        const float2 (&b)[NT][2]) {
-  TF ar[MT][4], ai[MT][4], br[NT][2], bi[NT][2];
+__device__ __forceinline__ void cmma_k8(float (&acc)[3][MT][NT][4], const float2 (&a)[MT][4], const float2 (&b)[NT][2]) {
+  TF as[3][MT][4], bs[3][NT][2];
 #pragma unroll
   for (int mi = 0; mi < MT; ++mi)
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
-      ar[mi][q] = split_tf32(a[mi][q].x);
-      ai[mi][q] = split_tf32(a[mi][q].y);
+      as[0][mi][q] = split_tf32(a[mi][q].x);
+      as[1][mi][q] = split_tf32(a[mi][q].y);
+      as[2][mi][q] = split_tf32(kConj ? a[mi][q].x - a[mi][q].y : a[mi][q].x + a[mi][q].y);
     }
 #pragma unroll
   for (int ni = 0; ni < NT; ++ni)
 #pragma unroll
     for (int q = 0; q < 2; ++q) {
-      br[ni][q] = split_tf32(b[ni][q].x);
-      bi[ni][q] = split_tf32(b[ni][q].y);
+      bs[0][ni][q] = split_tf32(b[ni][q].x);
+      bs[1][ni][q] = split_tf32(b[ni][q].y);
+      bs[2][ni][q] = split_tf32(b[ni][q].x + b[ni][q].y);
     }
-  constexpr unsigned kNeg = 0x80000000u;
-  const unsigned n_ib = kConj ? 0u : kNeg;  // sign of Ai Bi in Re
-  const unsigned n_ir = kConj ? kNeg : 0u;  // sign of Ai Br in Im
 #pragma unroll
-  for (int term = 0; term < 3; ++term) {  // 0: lo_a hi_b, 1: hi_a lo_b, 2: hi_a hi_b
+  for (int term = 0; term < 3; ++term)  // 0: lo_a hi_b, 1: hi_a lo_b, 2: hi_a hi_b
 #pragma unroll
-    for (int prod = 0; prod < 2; ++prod) {  // 0: (Ar Br, Ar Bi), 1: (+-Ai Bi, +-Ai Br)
+    for (int p = 0; p < 3; ++p)
 #pragma unroll
       for (int mi = 0; mi < MT; ++mi)
 #pragma unroll
         for (int ni = 0; ni < NT; ++ni) {
-          const TF* A = prod == 0 ? ar[mi] : ai[mi];
-          const TF* Bre = prod == 0 ? br[ni] : bi[ni];  // the operand that goes to Re
-          const TF* Bim = prod == 0 ? bi[ni] : br[ni];  // ... and to Im
-          const unsigned sr = prod == 0 ? 0u : n_ib, si = prod == 0 ? 0u : n_ir;
-          unsigned a0, a1, a2, a3;
-          if (term == 0) { a0 = A[0].lo; a1 = A[1].lo; a2 = A[2].lo; a3 = A[3].lo; }
-          else { a0 = A[0].hi; a1 = A[1].hi; a2 = A[2].hi; a3 = A[3].hi; }
-          const unsigned b0r = term == 1 ? Bre[0].lo : Bre[0].hi, b1r = term == 1 ? Bre[1].lo : Bre[1].hi;
-          const unsigned b0i = term == 1 ? Bim[0].lo : Bim[0].hi, b1i = term == 1 ? Bim[1].lo : Bim[1].hi;
-          hmma(re[mi][ni], a0 ^ sr, a1 ^ sr, a2 ^ sr, a3 ^ sr, b0r, b1r);
-          hmma(im[mi][ni], a0 ^ si, a1 ^ si, a2 ^ si, a3 ^ si, b0i, b1i);
+          const TF* A = as[p][mi];
+          const TF* B = bs[p][ni];
+          if (term == 0) hmma(acc[p][mi][ni], A[0].lo, A[1].lo, A[2].lo, A[3].lo, B[0].hi, B[1].hi);
+          else if (term == 1) hmma(acc[p][mi][ni], A[0].hi, A[1].hi, A[2].hi, A[3].hi, B[0].lo, B[1].lo);
+          else hmma(acc[p][mi][ni], A[0].hi, A[1].hi, A[2].hi, A[3].hi, B[0].hi, B[1].hi);
         }
-    }
-  }
+}
+
+template <bool kConj>
+__device__ __forceinline__ float2 cmma_finish(float t1, float t2, float t3) {
+  return kConj ? make_float2(t1 + t2, t3 - t1 + t2) : make_float2(t1 - t2, t3 - t1 - t2);
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -138,13 +136,15 @@ __global__ void __launch_bounds__(kSpThreads) k_gemm1_sp(const float2* __restric
     cp_commit();
   };
 
-  float acc_re[2][2][4], acc_im[2][2][4];
+  float acc[3][2][2][4];
 #pragma unroll
-  for (int mi = 0; mi < 2; ++mi)
+  for (int p = 0; p < 3; ++p)
 #pragma unroll
-    for (int ni = 0; ni < 2; ++ni)
+    for (int mi = 0; mi < 2; ++mi)
 #pragma unroll
-      for (int q = 0; q < 4; ++q) acc_re[mi][ni][q] = acc_im[mi][ni][q] = 0.f;
+      for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+        for (int q = 0; q < 4; ++q) acc[p][mi][ni][q] = 0.f;
   float nrm[2] = {0.f, 0.f};  // |X|^2 of columns (wn*16 + ni*8 + g), k = t, t+4 (warps wm == 0)
 
   if (nchunks > 0) load(0, 0);
@@ -178,7 +178,7 @@ __global__ void __launch_bounds__(kSpThreads) k_gemm1_sp(const float2* __restric
           nrm[ni] += b[ni][0].x * b[ni][0].x + b[ni][0].y * b[ni][0].y + b[ni][1].x * b[ni][1].x +
                      b[ni][1].y * b[ni][1].y;
       }
-      cmma_k8<2, 2, true>(acc_re, acc_im, a, b);
+      cmma_k8<2, 2, true>(acc, a, b);
     }
     __syncthreads();
   }
@@ -192,7 +192,10 @@ __global__ void __launch_bounds__(kSpThreads) k_gemm1_sp(const float2* __restric
       for (int q = 0; q < 4; ++q) {
         const int m = m0 + wm * 32 + mi * 16 + g + (q >> 1) * 8;
         const int n = n0 + wn * 16 + ni * 8 + 2 * t + (q & 1);
-        if (m < mrows && n < ncols) P[(long long)m * ncols + n] = make_double2(acc_re[mi][ni][q], acc_im[mi][ni][q]);
+        if (m < mrows && n < ncols) {
+          const float2 v = cmma_finish<true>(acc[0][mi][ni][q], acc[1][mi][ni][q], acc[2][mi][ni][q]);
+          P[(long long)m * ncols + n] = make_double2(v.x, v.y);
+        }
       }
   if (norms && wm == 0 && blockIdx.y < ntn) {  // first M tile only (the norms do not depend on m)
 #pragma unroll
@@ -225,6 +228,11 @@ __global__ void __launch_bounds__(kSpThreads) k_gemm2_sp(float2* __restrict__ ps
   const float2* Xd = Xc + (long long)dom * np * norb;
   float2* Pd = psi + (long long)dom * ng * norb;
   const int nchunks = (np + kSpKC - 1) / kSpKC;
+  {  // the epilogue's Psi tile to L2 now (one 128-byte line per thread covers rows x 64 columns)
+    const int rr = tid / 4, cc = n0 + (tid % 4) * 16;
+    if (r0 + rr < ng && cc < norb)
+      asm volatile("prefetch.global.L2 [%0];" ::"l"(Pd + (r0 + rr) * norb + cc));
+  }
 
   auto load = [&](int c, int st) {
     const int k0 = c * kSpKC;
@@ -237,13 +245,15 @@ __global__ void __launch_bounds__(kSpThreads) k_gemm2_sp(float2* __restrict__ ps
     cp_commit();
   };
 
-  float acc_re[2][2][4], acc_im[2][2][4];
+  float acc[3][2][2][4];
 #pragma unroll
-  for (int mi = 0; mi < 2; ++mi)
+  for (int p = 0; p < 3; ++p)
 #pragma unroll
-    for (int ni = 0; ni < 2; ++ni)
+    for (int mi = 0; mi < 2; ++mi)
 #pragma unroll
-      for (int q = 0; q < 4; ++q) acc_re[mi][ni][q] = acc_im[mi][ni][q] = 0.f;
+      for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+        for (int q = 0; q < 4; ++q) acc[p][mi][ni][q] = 0.f;
 
   load(0, 0);
   for (int c = 0; c < nchunks; ++c) {
@@ -273,7 +283,7 @@ __global__ void __launch_bounds__(kSpThreads) k_gemm2_sp(float2* __restrict__ ps
         b[ni][0] = Xs[st][k][n];
         b[ni][1] = Xs[st][k + 4][n];
       }
-      cmma_k8<2, 2, false>(acc_re, acc_im, a, b);
+      cmma_k8<2, 2, false>(acc, a, b);
     }
     __syncthreads();
   }
@@ -291,7 +301,8 @@ __global__ void __launch_bounds__(kSpThreads) k_gemm2_sp(float2* __restrict__ ps
           const float f = (float)nf[n];
           float2* p = Pd + r * norb + n;
           const float2 v = *p;
-          *p = make_float2(fmaf(f, v.x, acc_re[mi][ni][q]), fmaf(f, v.y, acc_im[mi][ni][q]));
+          const float2 u = cmma_finish<false>(acc[0][mi][ni][q], acc[1][mi][ni][q], acc[2][mi][ni][q]);
+          *p = make_float2(fmaf(f, v.x, u.x), fmaf(f, v.y, u.y));
         }
       }
 }
