@@ -69,6 +69,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--no-sc", action="store_true", help="skip the self-consistent-step measurement (sc_mode)")
+    ap.add_argument("--no-sp", action="store_true", help="skip the single-precision measurement (sp_mode)")
     ap.add_argument("--sc-corr", type=int, default=1, help="corrector sweeps of the sc_mode measurement")
     ap.add_argument("--sc-multi", action="store_true",
                     help="also measure sc_mode under torchrun (its NCCL communicator is built by liblfd; the "
@@ -96,7 +97,7 @@ def peaks():
     # The complex GEMMs use the 3M (Gauss) product: 3 real DMMAs per complex multiply-add, while flops
     # are counted as 8 per complex multiply-add. Their roofline peak is therefore the DMMA peak x 4/3, so
     # that frac = the fraction of the DMMA pipe the kernel keeps busy.
-    return {"hbm_gbs": hbm, "hbm_src": src, "fp64_tflops": fp64, "fp64_src": fsrc,
+    return {"hbm_gbs": hbm, "hbm_src": src, "fp64_tflops": fp64, "fp64_src": fsrc, "tf32_tflops": 278.9,
             "zgemm3m_tflops": fp64 * 4.0 / 3.0,
             "zgemm3m_src": fsrc + " x 4/3 (3M complex product: 3 real DMMA per complex MAC, 8 flops counted)"}
 
@@ -298,6 +299,69 @@ def run_sc_mode(args, w, ctx, x, dev, stream, rank, world):
                     "NCCL when world > 1; value counts one physical step (ndom x Ngrid x norb ogp)"}
 
 
+def run_sp_mode(args, w, x, dev, stream, pk):
+    """The same step loop on the SP variant (LFD_FLAG_SP: complex64 Psi / B)."""
+    import torch
+    from paper_conf_ipps_razakhllknvn24_b200 import Context, lfd
+    from lfd_workloads.generate import midpoint_A
+    psi = torch.from_numpy(x.psi0.astype(np.complex64)).to(dev)
+    proj = torch.from_numpy(x.proj.astype(np.complex64)).to(dev) if w.nproj else None
+    v_dev = torch.from_numpy(x.vloc).to(dev)
+    ctx = Context(psi, proj, x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc)
+    nd, ng = w.ndom, w.ngrid
+    rho = torch.empty((nd, ng), dtype=torch.float64, device=dev)
+    J = torch.empty((nd, 3), dtype=torch.float64, device=dev)
+
+    def step(n):
+        lfd.lfd_set_vector_potential(ctx.ctx, midpoint_A(w, n))
+        lfd.lfd_set_potential(ctx.ctx, v_dev)
+        lfd.lfd_step(ctx.ctx, 1)
+        lfd.lfd_density_current(ctx.ctx, rho, None, J)
+
+    for n in range(args.warmup):
+        step(n)
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for n in range(args.steps):
+        step(args.warmup + n)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    lfd.lfd_profile_enable(ctx.ctx, True)
+    for n in range(args.steps):
+        step(args.warmup + n)
+    prof = lfd.lfd_profile_read(ctx.ctx)
+    ctx.close()
+    del psi, proj
+    tot = sum(v[0] for v in prof.values()) or 1.0
+    work = kernel_work(w)
+    kern = {}
+    # 3xTF32 3M: 3 real products x 3 TF32 terms = 18 HMMA flops per complex MAC, 8 counted
+    tpeak = pk["tf32_tflops"] * 8.0 / 18.0
+    for k, (kms, cnt) in prof.items():
+        if not cnt:
+            continue
+        avg = kms / cnt
+        e = {"ms_per_launch": avg, "launches": cnt, "share": round(kms / tot, 4)}
+        if k in work:
+            b, f = work[k]
+            if f > 0:
+                e.update({"bound": "tensor", "achieved": f / (avg * 1e-3) / 1e12, "unit": "TFLOP/s", "peak": tpeak})
+            else:
+                e.update({"bound": "hbm", "achieved": 0.5 * b / (avg * 1e-3) / 1e9, "unit": "GB/s",
+                          "peak": pk["hbm_gbs"]})
+            e["frac"] = e["achieved"] / e["peak"]
+        kern[k] = e
+    return {"value": w.ogp_per_step * args.steps / (ms / 1e3), "unit": UNIT, "ms_per_step": ms / args.steps,
+            "dtype": "c64 (FP32 sweeps, 3xTF32 tensor-core GEMMs, FP64 reductions)", "kernels": kern,
+            "tensor_peak_source": f"measured mma.sync tf32 {pk['tf32_tflops']} TF/s (profiles/r01_sp_peaks.txt) "
+                                  "x 8/18 (3M x 3xTF32)",
+            "note": "same step loop as the headline on complex64 copies of Psi / B (LFD_FLAG_SP); parity vs the "
+                    "FP64 oracle within n*30*2^-24 (tests/test_gpu_sp.py)"}
+
+
 def main():
     args = parse()
     rank = int(os.environ.get("RANK", "0"))
@@ -432,6 +496,13 @@ def main():
                "note": f"lfd_step_sequence of {args.steps} steps (per-step A; N o N merged: {args.steps + 1} "
                        f"projector GEMM pairs instead of {2 * args.steps}), one density at the end"}
 
+    spm = None
+    if not args.no_sp and world == 1:
+        try:
+            spm = run_sp_mode(args, w, x, dev, stream, pk)
+        except Exception as ex:
+            spm = {"error": f"{type(ex).__name__}: {ex}"}
+
     # self-consistent mode (lfd_sc_step): Hartree (cuFFT on the global grid of all
     # ranks' domains) + LDA exchange + Maxwell, predictor + n_corr corrector sweeps, the [rho_g | Jbar]
     # SUM all-reduce over NCCL inside the step when world > 1 -- the full LFD subprogram per QD step
@@ -494,6 +565,7 @@ def main():
             "e2e": e2e,
             "sequence_mode": seq,
             "sc_mode": scm,
+            "sp_mode": spm,
             "cpu_baseline": cpu,
         }
         print(json.dumps(out), flush=True)
