@@ -32,7 +32,7 @@ UNIT = "orbital-gridpoint updates/s"
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FP64_PEAK_FILE = os.path.join(ROOT, "profiles", "r01_fp64_peaks.jsonl")
 NCU_SUMMARY = os.path.join(ROOT, "profiles", "latest_ncu_full_summary.csv")
-NCU_NAMES = {"nl_proj": "k_gemm1", "nl_back": "k_gemm2", "kin_x": "k_kin<1, 1>", "kin_y": "k_kin<1, 0>",
+NCU_NAMES = {"nl_proj": "k_gemm1", "nl_back": "k_gemm2", "kin_x": "k_kin<1, 1, 1", "kin_y": "k_kin<1, 0",
              "kin_z": "k_kin<1, 2>", "kin_yz": "k_kin_yz", "density": "k_density"}
 
 
