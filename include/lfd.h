@@ -197,7 +197,8 @@ lfd_status lfd_remap_occ(lfd_ctx* ctx, const void* ref, int32_t nref, double* oc
  *   A: velocity-Verlet half kick and drift of the induced field with Jbar(t_n) (R25/R26),
  *      A_mid = A_ext(t_n + Delta/2) + (A_ind(t_n) + A_ind(t_n+1)) / 2, A_end = A_ext(t_n+1) + A_ind(t_n+1);
  *   v: v_loc = v_ion + 3/2 v_Hxc(t_n) - 1/2 v_Hxc(t_n-1) (predictor, R27);
- *   for k = 0..n_corr: Psi <- Eq.-6 step of Psi(t_n) with (v_loc, A_mid); rho, Jbar of Psi with A_end on the
+ *   S = N(Psi(t_n)) (the first Eq.-6 nonlocal factor does not depend on v or A: applied once per step);
+ *   for k = 0..n_corr: Psi <- N(Local(S)) with (v_loc, A_mid); rho, Jbar of Psi with A_end on the
  *      GLOBAL grid (domain cores, R18; SUM all-reduce over ranks when nranks > 1); v_Hxc = v_H + v_x (R23,
  *      R24; Hartree by cuFFT on the global grid); if k < n_corr: v_loc = v_ion + (v_Hxc(t_n) + v_Hxc)/2;
  *   A: second half kick with Jbar(t_n+1).
@@ -214,7 +215,7 @@ typedef struct {
   const int32_t* dom_offset; /* HOST [ndom][3] global offsets of this context's domains (copied) */
 } lfd_sc_config;
 
-/* Bytes of DEVICE workspace lfd_sc_init needs (includes a copy of Psi when n_corr > 0 and the cuFFT
+/* Bytes of DEVICE workspace lfd_sc_init needs (includes a buffer of Psi's size for N(Psi(t_n)) and the cuFFT
  * work area; the library allocates nothing). */
 lfd_status lfd_sc_workspace_size(const lfd_ctx* ctx, const lfd_sc_config* sc, size_t* bytes);
 

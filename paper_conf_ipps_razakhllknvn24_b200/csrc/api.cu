@@ -202,8 +202,7 @@ const Nccl* nccl_load(std::string& why) {
 }
 
 struct ScLayout {
-  size_t pack, vh0, vh1, vh2, spec, state, coef_end, gbase, off, jtmp, snap_dc, snap_cp, snap_s, snap_n, fftwork,
-      psi_save, total;
+  size_t pack, vh0, vh1, vh2, spec, state, coef_end, gbase, off, jtmp, fftwork, psi_save, total;
   size_t fft_bytes;
 };
 
@@ -381,18 +380,20 @@ cudaError_t phase_any(lfd_ctx* c, const double* v, double* vcopy) {
   return lfd::launch_phase(c->g, v, c->phi(), vcopy, c->scaled, c->stream);
 }
 
-// GEMM-2 of a nonlocal factor: Psi <- (Psi + B C') diag(n), C' and n from the workspace.
-lfd_status gemm2(lfd_ctx* c) {
+// GEMM-2 of a nonlocal factor: Psi <- (Psi + B C') diag(n), C' and n from the workspace; with out != nullptr
+// the result goes to `out` (same layout) and Psi is only read.
+lfd_status gemm2(lfd_ctx* c, double2* out = nullptr) {
   const Geometry& g = c->g;
   lfd::Gemm2Args a2;
   a2.psi = c->psi; a2.B = c->proj; a2.Cp = c->at<double2>(c->L.cprime); a2.nfac = c->at<double>(c->L.nfac);
   a2.ndom = g.ndom; a2.nproj = g.nproj; a2.norb = g.norb; a2.ng = g.ng; a2.num_sms = c->num_sms;
   a2.variant = c->gemm2_variant;
+  a2.psi_out = out;
   c->c_valid = false;
   if (g.sp)
     LFD_TRY(launch(c, LFD_K_NL_BACK, "k_gemm2_sp", [&] {
       return lfd::launch_gemm2_sp(c->psi32(), c->proj32(), a2.Cp, c->at<float2>(c->L.x32), a2.nfac, g.ndom, g.nproj,
-                                  g.norb, g.ng, c->stream);
+                                  g.norb, g.ng, c->stream, reinterpret_cast<float2*>(out));
     }));
   else
     LFD_TRY(launch(c, LFD_K_NL_BACK, "k_gemm2", [&] { return lfd::launch_gemm2(a2, c->stream); }));
@@ -406,7 +407,7 @@ const double2* exact_w(lfd_ctx* c, bool merged) {
 }
 
 // Eq. 6 nonlocal factor N on every domain (kernels a3, a4, a5); merged = N o N in one pass.
-lfd_status nl_half(lfd_ctx* c, bool merged = false) {
+lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
   const Geometry& g = c->g;
   if (c->c_valid) {  // C of the current Psi from the previous factor (no GEMM-1, no reduction)
     double* D = c->at<double>(c->L.D);
@@ -419,7 +420,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false) {
         return lfd::launch_nlcarry(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G),
                                    c->at<double>(c->L.ones), DC, X, s, nfac, false, exact_w(c, merged), c->stream);
       }));
-      return gemm2(c);
+      return gemm2(c, out);
     }
     LFD_TRY(launch(c, LFD_K_NL_CARRY, "k_nlcarry", [&] {
       return lfd::launch_nlcarry(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), D, DC, X, s, nfac,
@@ -430,7 +431,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false) {
         return lfd::launch_nlmerge(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), D, DC, s, X, nfac,
                                    c->stream);
       }));
-    return gemm2(c);
+    return gemm2(c, out);
   }
   lfd::Gemm1Args a1;
   a1.A = c->proj;
@@ -453,7 +454,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false) {
     r.D = nullptr;
     r.W = exact_w(c, merged);
     LFD_TRY(launch(c, LFD_K_NL_REDUCE, "k_reduce", [&] { return lfd::launch_reduce(r, c->stream); }));
-    return gemm2(c);
+    return gemm2(c, out);
   }
   LFD_TRY(launch(c, LFD_K_NL_REDUCE, "k_reduce", [&] { return lfd::launch_reduce(r, c->stream); }));
   if (merged)
@@ -466,15 +467,17 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false) {
       return lfd::launch_nlnorm(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), r.out, r.s,
                                 c->at<double>(c->L.nfac), r.cprime, c->stream);
     }));
-  return gemm2(c);
+  return gemm2(c, out);
 }
 
 // Local factor exp(-i Delta h_loc) of Eq. 6: Psi <- Phi . K_z K_y K_x (Phi . Psi) (kernels a6).
-lfd_status local_prop(lfd_ctx* c) {
+// src != nullptr: the first pass reads src (same layout) and writes Psi (out of place).
+lfd_status local_prop(lfd_ctx* c, const double2* src = nullptr) {
   c->c_valid = false;
   if (c->g.sp) {  // SP variant: three FP32 line passes Phi.K_x, K_y, K_z.Phi (complex64 Psi)
     LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin_sp(x)", [&] {
-      return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 0, 1, c->scaled, c->stream);
+      return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 0, 1, c->scaled, c->stream,
+                                reinterpret_cast<const float2*>(src));
     }));
     LFD_TRY(launch(c, LFD_K_KIN_Y, "k_kin_sp(y)", [&] {
       return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 1, 0, c->scaled, c->stream);
@@ -484,7 +487,7 @@ lfd_status local_prop(lfd_ctx* c) {
     });
   }
   LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin(x)",
-                 [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 0, 1, c->scaled, c->stream); }));
+                 [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 0, 1, c->scaled, c->stream, src); }));
   if (c->kin_fused)
     return launch(c, LFD_K_KIN_YZ, "k_kin_yz",
                   [&] { return lfd::launch_kin_yz(c->g, &c->psi_tmap, c->psi, c->coef(), c->phi(), c->scaled, c->stream); });
@@ -526,6 +529,7 @@ lfd_status density_into(lfd_ctx* c, double* rho, double* j, double* Jmac, const 
   lfd::DensArgs a;
   a.psi = c->psi; a.coef = coef ? coef : c->coef(); a.occ = c->at<double>(c->L.occ);
   a.psi_sp = c->g.sp ? c->psi32() : nullptr;
+  if (const char* v = std::getenv("LFD_DENS_DBG")) a.dbg_nocompute = std::atoi(v);
   a.rho = rho; a.j = j; a.jline = c->at<double>(c->L.jline);
   a.base = base_dev; a.jbase = base_dev + c->g.ndom; a.sx = sx; a.sy = sy; a.jstride = jstride;
   a.v = energy ? c->at<double>(c->L.vstage) : nullptr;
@@ -604,13 +608,9 @@ ScLayout sc_layout(const Geometry& g, const lfd_sc_config* sc, size_t fft_bytes)
   L.gbase = take((size_t)2 * g.ndom * sizeof(long long));
   L.off = take((size_t)3 * g.ndom * sizeof(int));
   L.jtmp = take((size_t)3 * g.ndom * d8);
-  L.snap_dc = take((size_t)g.ndom * g.nproj * g.norb * c16);
-  L.snap_cp = take((size_t)g.ndom * g.nproj * g.norb * c16);
-  L.snap_s = take((size_t)g.ndom * g.norb * d8);
-  L.snap_n = take((size_t)g.ndom * g.norb * d8);
   L.fft_bytes = fft_bytes;
   L.fftwork = take(fft_bytes);
-  L.psi_save = sc->n_corr > 0 ? take((size_t)g.ndom * g.ng * g.norb * (g.sp ? 8 : c16)) : 0;
+  L.psi_save = take((size_t)g.ndom * g.ng * g.norb * (g.sp ? 8 : c16));  // S = N(Psi(t_n)) (lfd_sc_step)
   L.total = o;
   return L;
 }
@@ -1129,11 +1129,16 @@ lfd_status lfd_sc_step(lfd_ctx* c, int32_t nsteps, const double* Aext) {
   const bool maxwell = S.flags & LFD_SC_MAXWELL;
   double* state = S.at<double>(S.L.state);
   const size_t psi_bytes = (size_t)g.ndom * g.ng * g.norb * c->celem();
-  const size_t cbytes = (size_t)g.ndom * g.nproj * g.norb * 16, nbytes = (size_t)g.ndom * g.norb * 8;
   auto cpy = [&](void* dst, const void* src, size_t n) -> lfd_status {
     cudaError_t e = cudaMemcpyAsync(dst, src, n, cudaMemcpyDeviceToDevice, c->stream);
     return e == cudaSuccess ? LFD_OK : cuda_fail(c, e, "SC device copy");
   };
+  // Psi(t_n) lives in the caller's buffer P. The first nonlocal factor of Eq. 6 depends on Psi(t_n), B and
+  // D only (not on v or A), so it is applied ONCE per step, out of place into the SC buffer S = N(Psi(t_n));
+  // every sweep then runs the local factor from S into P (the first stencil pass reads S, writes P) and the
+  // second nonlocal factor in place on P. S is never overwritten, so the corrector needs no copies, and the
+  // last sweep leaves Psi(t_n+1) in P with the projection carry of its second factor for the next step.
+  double2* Sbuf = S.at<double2>(S.L.psi_save);
   for (int n = 0; n < nsteps; ++n) {
     const double* a_mid = Aext + 3 * (2 * n + 1);
     const double* a_end = Aext + 3 * (2 * n + 2);
@@ -1145,29 +1150,15 @@ lfd_status lfd_sc_step(lfd_ctx* c, int32_t nsteps, const double* Aext) {
     double* vp = S.vh(S.vi[1]);
     double* vnew = S.vh(S.vi[2]);
     LFD_TRY(sc_set_v(c, vn, 1.5, vp, -0.5));  // predictor (R27)
-    bool snap_valid = false;
-    if (S.n_corr > 0) {
-      LFD_TRY(cpy(S.at<void>(S.L.psi_save), c->psi, psi_bytes));
-      snap_valid = c->c_valid;
-      if (snap_valid) {  // the projection carry of Psi(t_n), reused by every sweep
-        LFD_TRY(cpy(S.at<void>(S.L.snap_dc), c->at<void>(c->L.dc), cbytes));
-        LFD_TRY(cpy(S.at<void>(S.L.snap_cp), c->at<void>(c->L.cprime), cbytes));
-        LFD_TRY(cpy(S.at<void>(S.L.snap_s), c->at<void>(c->L.s), nbytes));
-        LFD_TRY(cpy(S.at<void>(S.L.snap_n), c->at<void>(c->L.nfac), nbytes));
-      }
+    if (g.nproj > 0) {
+      LFD_TRY(nl_half(c, false, Sbuf));  // S = N(Psi(t_n))
+    } else {
+      cudaError_t e = cudaMemcpyAsync(Sbuf, c->psi, psi_bytes, cudaMemcpyDeviceToDevice, c->stream);
+      if (e != cudaSuccess) return cuda_fail(c, e, "SC device copy");
     }
     for (int k = 0; k <= S.n_corr; ++k) {
-      if (k > 0) {
-        LFD_TRY(cpy(c->psi, S.at<void>(S.L.psi_save), psi_bytes));
-        c->c_valid = snap_valid;
-        if (snap_valid) {
-          LFD_TRY(cpy(c->at<void>(c->L.dc), S.at<void>(S.L.snap_dc), cbytes));
-          LFD_TRY(cpy(c->at<void>(c->L.cprime), S.at<void>(S.L.snap_cp), cbytes));
-          LFD_TRY(cpy(c->at<void>(c->L.s), S.at<void>(S.L.snap_s), nbytes));
-          LFD_TRY(cpy(c->at<void>(c->L.nfac), S.at<void>(S.L.snap_n), nbytes));
-        }
-      }
-      LFD_TRY(one_step(c));
+      LFD_TRY(local_prop(c, Sbuf));
+      if (g.nproj > 0) LFD_TRY(nl_half(c));
       LFD_TRY(sc_density(c));
       LFD_TRY(sc_vhxc(c, vnew));
       if (k < S.n_corr) LFD_TRY(sc_set_v(c, vn, 0.5, vnew, 0.5));  // corrector (R27)

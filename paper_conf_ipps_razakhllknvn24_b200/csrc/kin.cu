@@ -254,8 +254,11 @@ struct LineMarch {
 // Loads run two pairs ahead of the pair being combined (memory-level parallelism for the HBM stream).
 // C: complex type of the coefficients and Phi; V: the value a lane moves per grid point (C, or cf2 = two
 // complex64 orbitals); strides and norb are in units of V.
+// src: the input (== psi for the usual in-place pass; another buffer for the out-of-place first pass of the
+// self-consistent sweeps). In place is safe: each line belongs to one lane, whose reads of a point precede
+// its write of that point.
 template <bool kPeriodic, int kPhase, bool kS, class C = double2, class V = C>
-__global__ void __launch_bounds__(256, 3) k_kin(V* __restrict__ psi, const DomCoef* __restrict__ coef,
+__global__ void __launch_bounds__(256, 3) k_kin(V* psi, const V* src, const DomCoef* __restrict__ coef,
                                              const C* __restrict__ phi, int axis, int n, int pt_stride,
                                              int inner_len, int outer_stride, int ncols, int norb,
                                              long long dom_stride, long long ng) {
@@ -266,12 +269,13 @@ __global__ void __launch_bounds__(256, 3) k_kin(V* __restrict__ psi, const DomCo
   const int inner = c - outer * inner_len;
   const int off = outer * outer_stride + inner;
   V* line = psi + dom * dom_stride + off;
+  const V* sline = src + dom * dom_stride + off;
   const C* ph = phi + dom * ng + off / norb;
   const int ph_stride = pt_stride / norb;
   const PairCoefT<C> cf = pair_coef_t<kS, C>(coef + dom, axis);
 
   auto ld = [&](int i) -> V {
-    V v = line[(long long)i * pt_stride];
+    V v = sline[(long long)i * pt_stride];
     if (kPhase == 1) v = cmul(ph[(long long)i * ph_stride], v);
     return v;
   };
@@ -589,7 +593,8 @@ cudaError_t launch_kin_yz(const Geometry& g, const CUtensorMap* tmap, double2* p
 
 template <class C, class V>
 static cudaError_t launch_kin_t(const Geometry& g, V* psi, const DomCoef* coef, const C* phi, int axis,
-                                int phase_mode, bool scaled, cudaStream_t st) {
+                                int phase_mode, bool scaled, cudaStream_t st, const V* src) {
+  if (!src) src = psi;
   const int nd[3] = {g.nx, g.ny, g.nz};
   const int norb = g.norb / (int)(sizeof(V) / sizeof(C));  // values of type V per grid point
   int pt_stride, inner_len, outer_stride;
@@ -611,7 +616,7 @@ static cudaError_t launch_kin_t(const Geometry& g, V* psi, const DomCoef* coef, 
   dim3 grid((ncols + 255) / 256, g.ndom);
   const long long dom_stride = g.ng * norb;
 #define LFD_KIN(P, M, K)                                                                                       \
-  k_kin<P, M, K, C, V><<<grid, 256, 0, st>>>(psi, coef, phi, axis, n, pt_stride, inner_len, outer_stride, ncols, \
+  k_kin<P, M, K, C, V><<<grid, 256, 0, st>>>(psi, src, coef, phi, axis, n, pt_stride, inner_len, outer_stride, ncols, \
                                           norb, dom_stride, g.ng)
 #define LFD_KIN_M(P, K) \
   if (phase_mode == 1) LFD_KIN(P, 1, K); else if (phase_mode == 2) LFD_KIN(P, 2, K); else LFD_KIN(P, 0, K)
@@ -626,15 +631,17 @@ static cudaError_t launch_kin_t(const Geometry& g, V* psi, const DomCoef* coef, 
 }
 
 cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, const double2* phi, int axis,
-                       int phase_mode, bool scaled, cudaStream_t st) {
-  return launch_kin_t<double2, double2>(g, psi, coef, phi, axis, phase_mode, scaled, st);
+                       int phase_mode, bool scaled, cudaStream_t st, const double2* src) {
+  return launch_kin_t<double2, double2>(g, psi, coef, phi, axis, phase_mode, scaled, st, src);
 }
 
 cudaError_t launch_kin_sp(const Geometry& g, float2* psi, const DomCoef* coef, const float2* phi, int axis,
-                          int phase_mode, bool scaled, cudaStream_t st) {
-  if (g.norb % 2 == 0 && (reinterpret_cast<uintptr_t>(psi) & 15) == 0)  // two orbitals (16 bytes) per lane
-    return launch_kin_t<float2, cf2>(g, reinterpret_cast<cf2*>(psi), coef, phi, axis, phase_mode, scaled, st);
-  return launch_kin_t<float2, float2>(g, psi, coef, phi, axis, phase_mode, scaled, st);
+                          int phase_mode, bool scaled, cudaStream_t st, const float2* src) {
+  if (!src) src = psi;
+  if (g.norb % 2 == 0 && ((reinterpret_cast<uintptr_t>(psi) | reinterpret_cast<uintptr_t>(src)) & 15) == 0)
+    return launch_kin_t<float2, cf2>(g, reinterpret_cast<cf2*>(psi), coef, phi, axis, phase_mode, scaled, st,
+                                     reinterpret_cast<const cf2*>(src));  // two orbitals (16 bytes) per lane
+  return launch_kin_t<float2, float2>(g, psi, coef, phi, axis, phase_mode, scaled, st, src);
 }
 
 }  // namespace lfd

@@ -60,10 +60,10 @@ bool kin_scaled_ok(const Geometry& g);
 // One pass of K_axis over every line of every domain, optionally fused with a phase multiply
 // (phase_mode 1: Phi . psi before the sweep; 2: after).
 cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, const double2* phi,
-                       int axis, int phase_mode, bool scaled, cudaStream_t st);
+                       int axis, int phase_mode, bool scaled, cudaStream_t st, const double2* src = nullptr);
 // SP variant (complex64 Psi and Phi, FP32 sweeps)
 cudaError_t launch_kin_sp(const Geometry& g, float2* psi, const DomCoef* coef, const float2* phi,
-                          int axis, int phase_mode, bool scaled, cudaStream_t st);
+                          int axis, int phase_mode, bool scaled, cudaStream_t st, const float2* src = nullptr);
 
 // Fused pass Psi <- Phi . K_y K_z Psi (one read + write of Psi; nz <= 80).
 bool kin_yz_supported(const Geometry& g);
@@ -125,6 +125,7 @@ cudaError_t launch_nlcarry(int ndom, int nproj, int norb, double eps, const doub
 // (Cp = C'' = C' diag(n), scaled by the norm / merge / carry kernels)
 struct Gemm2Args {
   double2* psi;
+  double2* psi_out = nullptr;  // nullptr: in place; else the result goes here (psi is only read)
   const double2* B;
   const double2* Cp;
   const double* nfac;
@@ -142,6 +143,7 @@ cudaError_t gemm_set_attributes();
 struct DensArgs {
   const double2* psi;
   const float2* psi_sp = nullptr;  // SP variant: complex64 Psi (then psi is unused)
+  int dbg_nocompute = 0;           // diagnostics only (env LFD_DENS_DBG=1): skip the per-point sums
   const DomCoef* coef;
   const double* occ;
   double* rho;
@@ -174,7 +176,7 @@ cudaError_t launch_remap(const Geometry& g, int nref, const double2* C, const do
 // complex64 into X32 [ndom][nproj][norb] and updates psi in place.
 cudaError_t launch_gemm1_sp(const Gemm1Args& a, const float2* A, const float2* X, cudaStream_t st);
 cudaError_t launch_gemm2_sp(float2* psi, const float2* B, const double2* Cp, float2* X32, const double* nfac,
-                            int ndom, int nproj, int norb, long long ng, cudaStream_t st);
+                            int ndom, int nproj, int norb, long long ng, cudaStream_t st, float2* psi_out = nullptr);
 cudaError_t gemm_sp_set_attributes();
 
 // Self-consistent step kernels (sc.cu, readings R23-R28).

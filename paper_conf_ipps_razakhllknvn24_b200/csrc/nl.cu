@@ -736,7 +736,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(const __grid_constant__ C
     int dom, n0;
     long long r0;
     decode(item, dom, r0, n0);
-    double2* psi = p.psi + (long long)dom * p.ng * p.norb;
+    const double2* psi = p.psi + (long long)dom * p.ng * p.norb;
+    double2* pout = (p.psi_out ? p.psi_out : p.psi) + (long long)dom * p.ng * p.norb;
     if (tid == 32) {  // Psi rows of this item (first) and of the next one -> L2, read in the epilogue
       if (it == 0) l2_prefetch(psi + r0 * p.norb, (uint32_t)(min((long long)kTile, p.ng - r0) * p.norb * 16));
       if (it + 1 < my_items) {
@@ -787,7 +788,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(const __grid_constant__ C
         for (int mi = 0; mi < 4; ++mi) {
           const long long r = r0 + wm * 32 + mi * 8 + g;
           if (r < p.ng)
-            psi[r * p.norb + col] =
+            pout[r * p.norb + col] =
                 make_double2(fma(f, pv[mi][ni][c].x, acc.re(mi, ni, c)), fma(f, pv[mi][ni][c].y, acc.im(mi, ni, c)));
         }
       }
@@ -896,7 +897,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
     const double2* As = reinterpret_cast<const double2*>(smem + stage * kFullABytes);
     Frag acc;
     acc.zero();
-    double2* psi = p.psi + (long long)dom * p.ng * p.norb;
+    const double2* psi = p.psi + (long long)dom * p.ng * p.norb;
+    double2* pout = (p.psi_out ? p.psi_out : p.psi) + (long long)dom * p.ng * p.norb;
     double2 pv[4][2][2];
     auto load_pv = [&]() {
 #pragma unroll
@@ -940,7 +942,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
         for (int mi = 0; mi < 4; ++mi) {
           const long long r = r0 + wm * 32 + mi * 8 + g;
           if (r < p.ng)
-            psi[r * p.norb + col] =
+            pout[r * p.norb + col] =
                 make_double2(fma(f, pv[mi][ni][c].x, acc.re(mi, ni, c)), fma(f, pv[mi][ni][c].y, acc.im(mi, ni, c)));
         }
       }
@@ -956,7 +958,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
 // copy when it changes), the K loop is fully unrolled for nproj = 64, the epilogue's Psi loads are
 // issued mid-loop and Psi <- n_s (Psi + B C') is written in place.
 // ------------------------------------------------------------------------------------------------
-template <int kNP, bool kSkew>
+template <int kNP, bool kSkew, bool kOut = false>
 __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant__ CUtensorMap tB,
                                                              const __grid_constant__ CUtensorMap tC, Gemm2Args p) {
   extern __shared__ __align__(128) unsigned char smem[];
@@ -1036,7 +1038,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant
     const double2* As = reinterpret_cast<const double2*>(smem + s * kFullABytes);
     Frag acc;
     acc.zero();
+    // kOut: out of place (psi_out); else the in-place code path reads and writes one pointer
     double2* psi = p.psi + (long long)dom * p.ng * p.norb;
+    double2* pout = kOut ? p.psi_out + (long long)dom * p.ng * p.norb : psi;
     double2 pv[4][2][2];
     auto load_pv = [&]() {
 #pragma unroll
@@ -1085,7 +1089,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant
         for (int mi = 0; mi < 4; ++mi) {
           const long long r = r0 + wm * 32 + mi * 8 + g;
           if (r < p.ng)
-            psi[r * p.norb + col] =
+            pout[r * p.norb + col] =
                 make_double2(fma(f, pv[mi][ni][c].x, acc.re(mi, ni, c)), fma(f, pv[mi][ni][c].y, acc.im(mi, ni, c)));
         }
       }
@@ -1115,18 +1119,26 @@ cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
     CUtensorMap tB, tC;
     cudaError_t e = gemm2_maps(a, &tB, &tC);
     if (e != cudaSuccess) return e;
-    if (a.nproj == kTile)
-      k_gemm2_tma<kTile, false><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
-    else
-      k_gemm2_tma<0, false><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+    const bool o = a.psi_out != nullptr;  // out of place (the self-consistent step's first factor)
+    if (a.nproj == kTile) {
+      if (o) k_gemm2_tma<kTile, false, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+      else k_gemm2_tma<kTile, false><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+    } else {
+      if (o) k_gemm2_tma<0, false, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+      else k_gemm2_tma<0, false><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+    }
   } else if (a.nproj <= kTile && a.variant == 3) {
     CUtensorMap tB, tC;
     cudaError_t e = gemm2_maps(a, &tB, &tC);
     if (e != cudaSuccess) return e;
-    if (a.nproj == kTile)
-      k_gemm2_tma<kTile, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
-    else
-      k_gemm2_tma<0, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+    const bool o = a.psi_out != nullptr;
+    if (a.nproj == kTile) {
+      if (o) k_gemm2_tma<kTile, true, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+      else k_gemm2_tma<kTile, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+    } else {
+      if (o) k_gemm2_tma<0, true, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+      else k_gemm2_tma<0, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+    }
   } else if (a.nproj == kTile && a.variant == 1)
     k_gemm2_fullk<kTile, true><<<grid, kThreads, kFullSmem, st>>>(a);
   else if (a.nproj == kTile)
@@ -1164,7 +1176,9 @@ cudaError_t gemm_set_attributes() {
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_gemm2_fullk<0, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
   if (e != cudaSuccess) return e;
-  for (auto f : {k_gemm2_tma<kTile, false>, k_gemm2_tma<0, false>, k_gemm2_tma<kTile, true>, k_gemm2_tma<0, true>}) {
+  for (auto f : {k_gemm2_tma<kTile, false>, k_gemm2_tma<0, false>, k_gemm2_tma<kTile, true>, k_gemm2_tma<0, true>,
+                 k_gemm2_tma<kTile, false, true>, k_gemm2_tma<kTile, true, true>, k_gemm2_tma<0, false, true>,
+                 k_gemm2_tma<0, true, true>}) {
     e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem + 16);
     if (e != cudaSuccess) return e;
   }

@@ -213,7 +213,7 @@ __global__ void __launch_bounds__(kSpThreads) k_gemm1_sp(const float2* __restric
 // GEMM-2 (SP). grid (row blocks of 64, column tiles of 64, ndom); K = nproj in chunks of 32.
 // smem per stage: Bs[m][k] (B rows), Xs[k][n] (the complex64 coefficient X'').
 // ------------------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kSpThreads) k_gemm2_sp(float2* __restrict__ psi, const float2* __restrict__ B,
+__global__ void __launch_bounds__(kSpThreads) k_gemm2_sp(const float2* psi, float2* pout, const float2* __restrict__ B,
                                                           const float2* __restrict__ Xc, const double* __restrict__ nfac,
                                                           int np, int norb, long long ng) {
   extern __shared__ __align__(16) float2 sp_smem[];
@@ -226,7 +226,8 @@ __global__ void __launch_bounds__(kSpThreads) k_gemm2_sp(float2* __restrict__ ps
   const int wm = warp >> 2, wn = warp & 3;
   const float2* Bd = B + (long long)dom * ng * np;
   const float2* Xd = Xc + (long long)dom * np * norb;
-  float2* Pd = psi + (long long)dom * ng * norb;
+  const float2* Pd = psi + (long long)dom * ng * norb;
+  float2* Po = pout + (long long)dom * ng * norb;
   const int nchunks = (np + kSpKC - 1) / kSpKC;
   {  // the epilogue's Psi tile to L2 now (one 128-byte line per thread covers rows x 64 columns)
     const int rr = tid / 4, cc = n0 + (tid % 4) * 16;
@@ -299,10 +300,9 @@ __global__ void __launch_bounds__(kSpThreads) k_gemm2_sp(float2* __restrict__ ps
         const int n = n0 + wn * 16 + ni * 8 + 2 * t + (q & 1);
         if (r < ng && n < norb) {
           const float f = (float)nf[n];
-          float2* p = Pd + r * norb + n;
-          const float2 v = *p;
+          const float2 v = Pd[r * norb + n];
           const float2 u = cmma_finish<false>(acc[0][mi][ni][q], acc[1][mi][ni][q], acc[2][mi][ni][q]);
-          *p = make_float2(fmaf(f, v.x, u.x), fmaf(f, v.y, u.y));
+          Po[r * norb + n] = make_float2(fmaf(f, v.x, u.x), fmaf(f, v.y, u.y));
         }
       }
 }
@@ -332,13 +332,13 @@ cudaError_t launch_gemm1_sp(const Gemm1Args& a, const float2* A, const float2* X
 }
 
 cudaError_t launch_gemm2_sp(float2* psi, const float2* B, const double2* Cp, float2* X32, const double* nfac,
-                            int ndom, int nproj, int norb, long long ng, cudaStream_t st) {
+                            int ndom, int nproj, int norb, long long ng, cudaStream_t st, float2* psi_out) {
   const long long n = (long long)ndom * nproj * norb;
   k_to_c64<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(Cp, X32, n);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   dim3 grid((unsigned)((ng + kSpT - 1) / kSpT), (norb + kSpT - 1) / kSpT, ndom);
-  k_gemm2_sp<<<grid, kSpThreads, kSmem2, st>>>(psi, B, X32, nfac, nproj, norb, ng);
+  k_gemm2_sp<<<grid, kSpThreads, kSmem2, st>>>(psi, psi_out ? psi_out : psi, B, X32, nfac, nproj, norb, ng);
   return cudaGetLastError();
 }
 
