@@ -155,6 +155,18 @@ lfd_status lfd_step(lfd_ctx* ctx, int32_t nsteps);
  * at the end. Afterwards the context's A is A_seq[nsteps-1]. */
 lfd_status lfd_step_sequence(lfd_ctx* ctx, int32_t nsteps, const double* A_seq);
 
+/* nsteps x (lfd_set_vector_potential(A_seq[n]); lfd_step(1); [density]) executed as CUDA graphs: chunks of up
+ * to 32 steps are captured once (on a private stream, on first use; keyed by chunk length, the projection-carry
+ * state and the outputs) and replayed with the chunk's A values uploaded to the workspace, so the host cost is
+ * one graph launch per 32 steps instead of ~12 kernel launches per step (latency-bound shapes such as C1 / C3).
+ * Results are bitwise those of the per-step calls (same kernels, same order).
+ *  A_seq     HOST double [nsteps][ndom][3] (copied during the call), the step midpoints (Eq. 4)
+ *  rho       DEVICE double [ndom][nx][ny][nz] or NULL: the density after each step (the last one remains)
+ *  Jmac_seq  DEVICE double [nsteps][ndom][3] or NULL: J of every step (the current response time series)
+ * Density and J use each step's own A, as lfd_density_current after that step. With lfd_profile_enable on, the
+ * same kernels run eagerly (per-launch events). Afterwards the context's A is A_seq[nsteps-1]. */
+lfd_status lfd_step_graph(lfd_ctx* ctx, int32_t nsteps, const double* A_seq, double* rho, double* Jmac_seq);
+
 /* Density and current of the current Psi with the current A (kernel 4; R13):
  *  rho  DEVICE double [ndom][nx][ny][nz]          rho_r = sum_s f_s |psi_rs|^2
  *  j    DEVICE double [ndom][3][nx][ny][nz] or NULL

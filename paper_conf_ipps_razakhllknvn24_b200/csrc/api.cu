@@ -25,13 +25,14 @@ using lfd::Geometry;
 namespace {
 
 constexpr size_t kAlign = 256;
+constexpr int kGraphChunk = 32;  // steps per captured CUDA graph (lfd_step_graph)
 constexpr int kKC1 = 32;  // GEMM-1 rows per chunk (nl.cu)
 
 size_t up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 struct Layout {
   size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage, cref,
-      epart, W, ones, x32;
+      epart, W, ones, x32, aseq, jseq;
   int nref_cap;
   size_t total;
   int nsplit;
@@ -141,6 +142,8 @@ Layout layout(const Geometry& g, int num_sms, int nref_max) {
   L.W = take((size_t)2 * nd * np * c16);
   L.ones = take((size_t)nd * std::max(np, no) * d8);
   L.x32 = g.sp ? take((size_t)nd * np * no * 8) : 0;  // SP: the GEMM-2 coefficient rounded to complex64
+  L.aseq = take((size_t)kGraphChunk * nd * 3 * d8);   // lfd_step_graph: A of the chunk's steps
+  L.jseq = take((size_t)kGraphChunk * nd * 3 * d8);   // lfd_step_graph: J of the chunk's steps
   L.total = o;
   return L;
 }
@@ -259,6 +262,17 @@ struct lfd_ctx {
   double prof_ms[LFD_K_COUNT] = {0};
   int64_t prof_n[LFD_K_COUNT] = {0};
   ScState sc;  // self-consistent step (lfd_sc_*)
+  // lfd_step_graph: captured CUDA graphs of K steps (+ density), keyed by what changes the launch sequence
+  struct Graph {
+    cudaGraphExec_t exec = nullptr;
+    int K = 0;
+    bool cv0 = false, cv1 = false;  // projection carry valid before / after the chunk
+    double* rho = nullptr;
+    bool dens = false;
+    uint64_t nlaunch = 0;  // kernels per replay
+  };
+  std::vector<Graph> graphs;
+  cudaStream_t cap_stream = nullptr;  // private stream for capture only (the legacy stream cannot capture)
 
   template <class T>
   T* at(size_t off) const { return reinterpret_cast<T*>(ws + off); }
@@ -689,6 +703,69 @@ void sc_release(ScState& S) {
   S.ready = false;
 }
 
+
+// ---- lfd_step_graph: K steps (+ density) as one CUDA graph ---------------------------------------------
+// The body every replay runs: per step k, the coefficient table from A in the workspace (aseq[k]), the
+// Eq.-6 step, and (if requested) the density into rho and J into jseq[k].
+lfd_status graph_body(lfd_ctx* c, int K, double* rho, bool dens) {
+  const Geometry& g = c->g;
+  for (int k = 0; k < K; ++k) {
+    LFD_TRY(launch(c, LFD_K_COEF, "k_coef_dev", [&] {
+      return lfd::launch_coef_dev(g, c->at<double>(c->L.aseq) + (size_t)k * g.ndom * 3, c->coef(), c->stream);
+    }));
+    LFD_TRY(one_step(c));
+    if (dens)
+      LFD_TRY(density_into(c, rho ? rho : c->at<double>(c->L.rhostage), nullptr,
+                           c->at<double>(c->L.jseq) + (size_t)k * g.ndom * 3, c->at<long long>(c->L.base),
+                           (long long)g.ny * g.nz, g.nz, g.ng));
+  }
+  return LFD_OK;
+}
+
+// The cached graph for (K, carry state, outputs), captured on first use.
+lfd_status get_graph(lfd_ctx* c, int K, double* rho, bool dens, lfd_ctx::Graph** out) {
+  for (auto& gr : c->graphs)
+    if (gr.K == K && gr.cv0 == c->c_valid && gr.rho == rho && gr.dens == dens) {
+      *out = &gr;
+      return LFD_OK;
+    }
+  if (!c->cap_stream) {
+    cudaError_t e = cudaStreamCreateWithFlags(&c->cap_stream, cudaStreamNonBlocking);
+    if (e != cudaSuccess) return cuda_fail(c, e, "cudaStreamCreate (graph capture)");
+  }
+  lfd_ctx::Graph gr;
+  gr.K = K; gr.cv0 = c->c_valid; gr.rho = rho; gr.dens = dens;
+  cudaStream_t orig = c->stream;
+  const uint64_t l0 = c->launches;
+  c->stream = c->cap_stream;
+  cudaError_t e = cudaStreamBeginCapture(c->cap_stream, cudaStreamCaptureModeThreadLocal);
+  if (e != cudaSuccess) { c->stream = orig; return cuda_fail(c, e, "cudaStreamBeginCapture"); }
+  lfd_status st = graph_body(c, K, rho, dens);
+  cudaGraph_t graph = nullptr;
+  e = cudaStreamEndCapture(c->cap_stream, &graph);
+  c->stream = orig;
+  if (st != LFD_OK) { if (graph) cudaGraphDestroy(graph); c->c_valid = gr.cv0; return st; }
+  if (e != cudaSuccess) { c->c_valid = gr.cv0; return cuda_fail(c, e, "cudaStreamEndCapture"); }
+  e = cudaGraphInstantiate(&gr.exec, graph, 0);
+  cudaGraphDestroy(graph);
+  if (e != cudaSuccess) { c->c_valid = gr.cv0; return cuda_fail(c, e, "cudaGraphInstantiate"); }
+  gr.cv1 = c->c_valid;  // the host-side carry logic ran during capture
+  c->c_valid = gr.cv0;
+  gr.nlaunch = c->launches - l0;
+  c->launches = l0;
+  c->graphs.push_back(gr);
+  *out = &c->graphs.back();
+  return LFD_OK;
+}
+
+void release_graphs(lfd_ctx* c) {
+  for (auto& gr : c->graphs)
+    if (gr.exec) cudaGraphExecDestroy(gr.exec);
+  c->graphs.clear();
+  if (c->cap_stream) cudaStreamDestroy(c->cap_stream);
+  c->cap_stream = nullptr;
+}
+
 }  // namespace
 
 extern "C" {
@@ -911,6 +988,42 @@ lfd_status lfd_step_sequence(lfd_ctx* c, int32_t nsteps, const double* A_seq) {
   return LFD_OK;
 }
 
+lfd_status lfd_step_graph(lfd_ctx* c, int32_t nsteps, const double* A_seq, double* rho, double* Jmac_seq) {
+  LFD_TRY(check_ctx(c));
+  if (nsteps < 0) return fail(c, LFD_EINVAL, "nsteps must be >= 0");
+  if (nsteps > 0 && !A_seq) return fail(c, LFD_EINVAL, "A_seq is NULL");
+  for (long long i = 0; i < 3LL * c->g.ndom * nsteps; ++i)
+    if (!std::isfinite(A_seq[i])) return fail(c, LFD_EINVAL, "A_seq must be finite");
+  DeviceGuard dg(c->device);
+  if ((rho && !is_device_ptr(rho)) || (Jmac_seq && !is_device_ptr(Jmac_seq)))
+    return fail(c, LFD_EINVAL, "rho / Jmac_seq must be device memory");
+  const Geometry& g = c->g;
+  const bool dens = rho || Jmac_seq;
+  const size_t ab = (size_t)g.ndom * 3 * sizeof(double);
+  for (int s0 = 0; s0 < nsteps; s0 += kGraphChunk) {
+    const int K = std::min(kGraphChunk, nsteps - s0);
+    cudaError_t e = cudaMemcpyAsync(c->at<double>(c->L.aseq), A_seq + (size_t)s0 * g.ndom * 3, ab * K,
+                                    cudaMemcpyHostToDevice, c->stream);
+    if (e != cudaSuccess) return cuda_fail(c, e, "H2D A_seq");
+    if (c->prof) {  // per-kernel timing needs events around every launch: run the same body eagerly
+      LFD_TRY(graph_body(c, K, rho, dens));
+    } else {
+      lfd_ctx::Graph* gr = nullptr;
+      LFD_TRY(get_graph(c, K, rho, dens, &gr));
+      e = cudaGraphLaunch(gr->exec, c->stream);
+      if (e != cudaSuccess) return cuda_fail(c, e, "cudaGraphLaunch");
+      c->launches += gr->nlaunch;
+      c->c_valid = gr->cv1;
+    }
+    if (Jmac_seq) {
+      e = cudaMemcpyAsync(Jmac_seq + (size_t)s0 * g.ndom * 3, c->at<double>(c->L.jseq), ab * K,
+                          cudaMemcpyDeviceToDevice, c->stream);
+      if (e != cudaSuccess) return cuda_fail(c, e, "copy J");
+    }
+  }
+  return LFD_OK;  // the coefficient table (the context's A) now holds A_seq[nsteps-1]
+}
+
 lfd_status lfd_density_current(lfd_ctx* c, double* rho, double* j, double* Jmac) {
   LFD_TRY(check_ctx(c));
   if (!rho) return fail(c, LFD_EINVAL, "rho is NULL");
@@ -1015,6 +1128,7 @@ lfd_status lfd_set_occupations(lfd_ctx* c, const double* occ) {
   if (e != cudaSuccess) return cuda_fail(c, e, "copy occ");
   e = lfd::density_maps_set_active(c->dmaps, c->g, c->psi, active_orbitals(c->g, occ));
   if (e != cudaSuccess) return cuda_fail(c, e, "density tensor map");
+  release_graphs(c);  // captured graphs hold the density kernel's tensor maps by value
   return LFD_OK;
 }
 
@@ -1299,6 +1413,7 @@ lfd_status lfd_destroy(lfd_ctx* c) {
   }
   lfd::density_maps_destroy(c->dmaps);
   sc_release(c->sc);
+  release_graphs(c);
   if (c->sc.comm) {
     std::string why;
     if (const Nccl* n = nccl_load(why)) n->comm_destroy(c->sc.comm);

@@ -39,6 +39,21 @@ __global__ void k_coef(CoefParams p, int dom0, int count, double hx, double hy, 
   coef[dom0 + i] = make_coef(p.A[i], hx, hy, hz, dt);
 }
 
+// The same table from A in DEVICE memory ([ndom][3]): step-invariant kernel parameters, so a captured CUDA
+// graph of several steps replays with new A values (lfd_step_graph).
+__global__ void k_coef_dev(const double* __restrict__ A, int ndom, double hx, double hy, double hz, double dt,
+                           DomCoef* __restrict__ coef) {
+  int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= ndom) return;
+  const double a[3] = {A[3 * i], A[3 * i + 1], A[3 * i + 2]};
+  coef[i] = make_coef(a, hx, hy, hz, dt);
+}
+
+cudaError_t launch_coef_dev(const Geometry& g, const double* A, DomCoef* coef, cudaStream_t st) {
+  k_coef_dev<<<(g.ndom + 127) / 128, 128, 0, st>>>(A, g.ndom, g.hx, g.hy, g.hz, g.dt, coef);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int count, DomCoef* coef,
                         cudaStream_t st) {
   k_coef<<<(count + 127) / 128, 128, 0, st>>>(p, dom0, count, g.hx, g.hy, g.hz, g.dt, coef);

@@ -49,6 +49,7 @@ struct CoefParams {
 };
 cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int count, DomCoef* coef,
                         cudaStream_t st);
+cudaError_t launch_coef_dev(const Geometry& g, const double* A, DomCoef* coef, cudaStream_t st);
 // Phi = e^{-i (Delta/2) v} (times sqrt(g) when the scaled pair form is used, kin.cu).
 cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, double* vcopy, bool scaled,
                          cudaStream_t st);

@@ -35,7 +35,7 @@ EXPORTS = ("lfd_workspace_size", "lfd_init", "lfd_set_potential", "lfd_set_poten
            "lfd_density_current_host", "lfd_energy", "lfd_remap_occ", "lfd_psi_modified", "lfd_set_occupations", "lfd_set_stream", "lfd_sync",
            "lfd_launch_count", "lfd_profile_enable", "lfd_profile_read", "lfd_last_error", "lfd_destroy",
            "lfd_sc_workspace_size", "lfd_sc_init", "lfd_sc_step", "lfd_sc_read", "lfd_comm_unique_id",
-           "lfd_sc_comm_init")
+           "lfd_sc_comm_init", "lfd_step_graph")
 
 
 class lfd_config(C.Structure):
@@ -96,6 +96,7 @@ def load():
         "lfd_sc_read": [P, P, P, P],
         "lfd_comm_unique_id": [P],
         "lfd_sc_comm_init": [P, I32, I32, P],
+        "lfd_step_graph": [P, I32, P, P, P],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -187,6 +188,13 @@ def lfd_step_sequence(ctx, A_seq):
     arr = np.ascontiguousarray(A_seq, dtype=np.float64)
     p, _k = _hptr(arr)
     _check(load().lfd_step_sequence(ctx, int(arr.shape[0]), p), ctx)
+
+
+def lfd_step_graph(ctx, A_seq, rho=None, Jmac_seq=None):
+    """A_seq: host [nsteps, ndom, 3]; the steps as captured CUDA graphs (chunks of 32), optional density / J."""
+    arr = np.ascontiguousarray(A_seq, dtype=np.float64)
+    p, _k = _hptr(arr)
+    _check(load().lfd_step_graph(ctx, int(arr.shape[0]), p, _dptr(rho), _dptr(Jmac_seq)), ctx)
 
 
 def lfd_density_current(ctx, rho, j=None, Jmac=None):
