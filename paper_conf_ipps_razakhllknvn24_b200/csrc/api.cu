@@ -740,7 +740,9 @@ lfd_status get_graph(lfd_ctx* c, int K, double* rho, bool dens, lfd_ctx::Graph**
   c->stream = c->cap_stream;
   cudaError_t e = cudaStreamBeginCapture(c->cap_stream, cudaStreamCaptureModeThreadLocal);
   if (e != cudaSuccess) { c->stream = orig; return cuda_fail(c, e, "cudaStreamBeginCapture"); }
+  lfd::pdl_suspend(true);
   lfd_status st = graph_body(c, K, rho, dens);
+  lfd::pdl_suspend(false);
   cudaGraph_t graph = nullptr;
   e = cudaStreamEndCapture(c->cap_stream, &graph);
   c->stream = orig;

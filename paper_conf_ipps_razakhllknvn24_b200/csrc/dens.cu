@@ -27,6 +27,8 @@ constexpr int kDensThreads = kSub * kTY * kTZ;  // 128
 
 template <class C>
 __global__ void __launch_bounds__(kDensThreads) k_density(Geometry g, DensArgs a, int ntz, int nty, int nxc) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   __shared__ double jsh[5][kDensThreads / kSub];
   const int dom = blockIdx.y;
   int b = blockIdx.x;
@@ -146,6 +148,8 @@ constexpr int kMaxNorbTma = 64;
 constexpr int kPlanePts = (kTY + 1) * (kTZ + 1);
 
 __global__ void __launch_bounds__(kDensThreads) k_density_tma(Geometry g, DensArgs a, int ntz, int nty, int nxc) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   extern __shared__ __align__(128) unsigned char dsm[];
   __shared__ __align__(8) uint64_t bars[kRingSlots];
   __shared__ double jsh[5][kDensThreads / kSub];
@@ -383,6 +387,8 @@ static YShape ymarch_shape(const Geometry& g) {
 template <bool kPer, int kIt, class C = double2>
 __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constant__ DensMaps mp, Geometry g,
                                                             DensArgs a) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   extern __shared__ __align__(128) unsigned char dsm[];
   const int norb = mp.nact, zc = mp.zc, px = mp.px;  // smem rows hold the nact active orbitals of each point
   const YLayout Ly(zc, norb, px, (int)sizeof(C));
@@ -635,31 +641,31 @@ cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps*
     const size_t sm = ymarch_smem(maps->zc, maps->nact, maps->px, maps->esz);
     if (maps->esz == 8) {  // SP variant (complex64 Psi)
       if (g.bc == 0 && maps->nact == 32)
-        k_density_y<true, 4, float2><<<grid, threads, sm, st>>>(*maps, g, a);
+        launch_k(k_density_y<true, 4, float2>, grid, threads, sm, st, *maps, g, a);
       else if (g.bc == 0)
-        k_density_y<true, 0, float2><<<grid, threads, sm, st>>>(*maps, g, a);
+        launch_k(k_density_y<true, 0, float2>, grid, threads, sm, st, *maps, g, a);
       else
-        k_density_y<false, 0, float2><<<grid, threads, sm, st>>>(*maps, g, a);
+        launch_k(k_density_y<false, 0, float2>, grid, threads, sm, st, *maps, g, a);
       return cudaGetLastError();
     }
     if (g.bc == 0 && maps->nact == 64)
-      k_density_y<true, 8><<<grid, threads, sm, st>>>(*maps, g, a);
+      launch_k(k_density_y<true, 8>, grid, threads, sm, st, *maps, g, a);
     else if (g.bc == 0 && maps->nact == 32)
-      k_density_y<true, 4><<<grid, threads, sm, st>>>(*maps, g, a);
+      launch_k(k_density_y<true, 4>, grid, threads, sm, st, *maps, g, a);
     else if (g.bc == 0)
-      k_density_y<true, 0><<<grid, threads, sm, st>>>(*maps, g, a);
+      launch_k(k_density_y<true, 0>, grid, threads, sm, st, *maps, g, a);
     else
-      k_density_y<false, 0><<<grid, threads, sm, st>>>(*maps, g, a);
+      launch_k(k_density_y<false, 0>, grid, threads, sm, st, *maps, g, a);
     return cudaGetLastError();
   }
   if (ymarch_shape(g).zc > 0) return cudaErrorInvalidValue;  // the block layout expects the y-marching kernel
   const int ntz = (g.nz + kTZ - 1) / kTZ, nty = (g.ny + kTY - 1) / kTY;
   if (a.psi_sp)
-    k_density<float2><<<grid, kDensThreads, 0, st>>>(g, a, ntz, nty, kXC);
+    launch_k(k_density<float2>, grid, kDensThreads, 0, st, g, a, ntz, nty, kXC);
   else if (g.norb <= kMaxNorbTma)
-    k_density_tma<<<grid, kDensThreads, density_smem_bytes(g.norb), st>>>(g, a, ntz, nty, kXC);
+    launch_k(k_density_tma, grid, kDensThreads, density_smem_bytes(g.norb), st, g, a, ntz, nty, kXC);
   else
-    k_density<double2><<<grid, kDensThreads, 0, st>>>(g, a, ntz, nty, kXC);
+    launch_k(k_density<double2>, grid, kDensThreads, 0, st, g, a, ntz, nty, kXC);
   return cudaGetLastError();
 }
 
@@ -681,6 +687,8 @@ cudaError_t density_set_attributes() {
 // J_d = (1/Ngrid) sum_lines jline (one block per domain, fixed-order tree over a fixed partition).
 __global__ void __launch_bounds__(256) k_jreduce(const double* __restrict__ jline, int lines, double inv_ng,
                                                  double* __restrict__ Jmac) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   __shared__ double sh[3][256];
   const int dom = blockIdx.x;
   double s[3] = {0.0, 0.0, 0.0};
@@ -697,7 +705,7 @@ __global__ void __launch_bounds__(256) k_jreduce(const double* __restrict__ jlin
 }
 
 cudaError_t launch_jreduce(const Geometry& g, const double* jline, double* Jmac, cudaStream_t st) {
-  k_jreduce<<<g.ndom, 256, 0, st>>>(jline, density_blocks(g), 1.0 / (double)g.ng, Jmac);
+  launch_k(k_jreduce, g.ndom, 256, 0, st, jline, density_blocks(g), 1.0 / (double)g.ng, Jmac);
   return cudaGetLastError();
 }
 

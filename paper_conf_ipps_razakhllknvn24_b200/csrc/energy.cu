@@ -14,6 +14,8 @@ __global__ void __launch_bounds__(256) k_energy_final(const double* __restrict__
                                                       const double2* __restrict__ C, const double* __restrict__ D,
                                                       const double* __restrict__ occ, int nproj, int norb, double dV,
                                                       double* __restrict__ E) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   __shared__ double sh[3][256];
   const int dom = blockIdx.x, tid = threadIdx.x;
   double ek = 0.0, el = 0.0, en = 0.0;
@@ -49,13 +51,15 @@ __global__ void __launch_bounds__(256) k_energy_final(const double* __restrict__
 
 cudaError_t launch_energy_final(const Geometry& g, const double* epart, int blocks, const double2* C,
                                 const double* D, const double* occ, double* E, cudaStream_t st) {
-  k_energy_final<<<g.ndom, 256, 0, st>>>(epart, blocks, C, D, occ, g.nproj, g.norb, g.dV, E);
+  launch_k(k_energy_final, g.ndom, 256, 0, st, epart, blocks, C, D, occ, g.nproj, g.norb, g.dV, E);
   return cudaGetLastError();
 }
 
 // occ_out[dom][k] = sum_s f_s |C[dom][k][s]|^2 : one warp per (dom, k), lanes over s, fixed-order tree.
 __global__ void __launch_bounds__(256) k_remap(int ndom, int nref, int norb, const double2* __restrict__ C,
                                                const double* __restrict__ occ, double* __restrict__ out) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   const long long w = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
   if (w >= (long long)ndom * nref) return;
@@ -75,7 +79,7 @@ __global__ void __launch_bounds__(256) k_remap(int ndom, int nref, int norb, con
 cudaError_t launch_remap(const Geometry& g, int nref, const double2* C, const double* occ, double* out,
                          cudaStream_t st) {
   const long long threads = (long long)g.ndom * nref * 32;
-  k_remap<<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(g.ndom, nref, g.norb, C, occ, out);
+  launch_k(k_remap, (unsigned)((threads + 255) / 256), 256, 0, st, g.ndom, nref, g.norb, C, occ, out);
   return cudaGetLastError();
 }
 

@@ -34,6 +34,8 @@ namespace lfd {
 
 __global__ void k_coef(CoefParams p, int dom0, int count, double hx, double hy, double hz, double dt,
                        DomCoef* __restrict__ coef) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= count) return;
   coef[dom0 + i] = make_coef(p.A[i], hx, hy, hz, dt);
@@ -43,6 +45,8 @@ __global__ void k_coef(CoefParams p, int dom0, int count, double hx, double hy, 
 // graph of several steps replays with new A values (lfd_step_graph).
 __global__ void k_coef_dev(const double* __restrict__ A, int ndom, double hx, double hy, double hz, double dt,
                            DomCoef* __restrict__ coef) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= ndom) return;
   const double a[3] = {A[3 * i], A[3 * i + 1], A[3 * i + 2]};
@@ -50,13 +54,13 @@ __global__ void k_coef_dev(const double* __restrict__ A, int ndom, double hx, do
 }
 
 cudaError_t launch_coef_dev(const Geometry& g, const double* A, DomCoef* coef, cudaStream_t st) {
-  k_coef_dev<<<(g.ndom + 127) / 128, 128, 0, st>>>(A, g.ndom, g.hx, g.hy, g.hz, g.dt, coef);
+  launch_k(k_coef_dev, (g.ndom + 127) / 128, 128, 0, st, A, g.ndom, g.hx, g.hy, g.hz, g.dt, coef);
   return cudaGetLastError();
 }
 
 cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int count, DomCoef* coef,
                         cudaStream_t st) {
-  k_coef<<<(count + 127) / 128, 128, 0, st>>>(p, dom0, count, g.hx, g.hy, g.hz, g.dt, coef);
+  launch_k(k_coef, (count + 127) / 128, 128, 0, st, p, dom0, count, g.hx, g.hy, g.hz, g.dt, coef);
   return cudaGetLastError();
 }
 
@@ -66,6 +70,8 @@ cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int co
 template <class C>
 __global__ void k_phase(const double* __restrict__ v, C* __restrict__ phi, double* vcopy, long long n,
                         double half_dt, double2 sg) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   const double vi = v[i];
@@ -102,7 +108,7 @@ cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, doubl
                          cudaStream_t st) {
   long long n = g.ng * g.ndom;
   const double2 sg = scaled ? scaled_sqrt_g(g) : make_double2(1.0, 0.0);
-  k_phase<double2><<<(unsigned)((n + 255) / 256), 256, 0, st>>>(v, phi, vcopy, n, 0.5 * g.dt, sg);
+  launch_k(k_phase<double2>, (unsigned)((n + 255) / 256), 256, 0, st, v, phi, vcopy, n, 0.5 * g.dt, sg);
   return cudaGetLastError();
 }
 
@@ -110,7 +116,7 @@ cudaError_t launch_phase_sp(const Geometry& g, const double* v, float2* phi, dou
                             cudaStream_t st) {
   long long n = g.ng * g.ndom;
   const double2 sg = scaled ? scaled_sqrt_g(g) : make_double2(1.0, 0.0);
-  k_phase<float2><<<(unsigned)((n + 255) / 256), 256, 0, st>>>(v, phi, vcopy, n, 0.5 * g.dt, sg);
+  launch_k(k_phase<float2>, (unsigned)((n + 255) / 256), 256, 0, st, v, phi, vcopy, n, 0.5 * g.dt, sg);
   return cudaGetLastError();
 }
 
@@ -277,6 +283,8 @@ __global__ void __launch_bounds__(256, 3) k_kin(V* psi, const V* src, const DomC
                                              const C* __restrict__ phi, int axis, int n, int pt_stride,
                                              int inner_len, int outer_stride, int ncols, int norb,
                                              long long dom_stride, long long ng) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   int c = blockIdx.x * blockDim.x + threadIdx.x;
   if (c >= ncols) return;
   const int dom = blockIdx.y;
@@ -358,6 +366,8 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
                                                           double2* __restrict__ psi, const DomCoef* __restrict__ coef,
                                                           const double2* __restrict__ phi, int nx, int ny, int nz,
                                                           int norb, int nchunks, long long ng) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   // periodic => nz even (validated), so every thread owns a full pair and every link exists
   constexpr bool kFull = kPer;
   extern __shared__ __align__(128) unsigned char smem[];
@@ -596,7 +606,7 @@ cudaError_t launch_kin_yz(const Geometry& g, const CUtensorMap* tmap, double2* p
   dim3 grid(g.nx * nchunks, g.ndom);
   const size_t sm = yz_smem(g.nz);
 #define LFD_KYZ(P, K) \
-  k_kin_yz<P, K><<<grid, threads, sm, st>>>(*tmap, psi, coef, phi, g.nx, g.ny, g.nz, g.norb, nchunks, g.ng)
+  launch_k(k_kin_yz<P, K>, grid, threads, sm, st, *tmap, psi, coef, phi, g.nx, g.ny, g.nz, g.norb, nchunks, g.ng)
   if (g.bc == 0) {
     if (scaled) LFD_KYZ(true, true); else LFD_KYZ(true, false);
   } else {
@@ -631,7 +641,7 @@ static cudaError_t launch_kin_t(const Geometry& g, V* psi, const DomCoef* coef, 
   dim3 grid((ncols + 255) / 256, g.ndom);
   const long long dom_stride = g.ng * norb;
 #define LFD_KIN(P, M, K)                                                                                       \
-  k_kin<P, M, K, C, V><<<grid, 256, 0, st>>>(psi, src, coef, phi, axis, n, pt_stride, inner_len, outer_stride, ncols, \
+  launch_k(k_kin<P, M, K, C, V>, grid, 256, 0, st, psi, src, coef, phi, axis, n, pt_stride, inner_len, outer_stride, ncols, \
                                           norb, dom_stride, g.ng)
 #define LFD_KIN_M(P, K) \
   if (phase_mode == 1) LFD_KIN(P, 1, K); else if (phase_mode == 2) LFD_KIN(P, 2, K); else LFD_KIN(P, 0, K)

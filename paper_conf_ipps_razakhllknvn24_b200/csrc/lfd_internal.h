@@ -10,6 +10,31 @@ namespace lfd {
 
 constexpr double kCLight = 137.035999084;  // R1: speed of light in atomic units
 
+// ---- programmatic dependent launch (PDL) -----------------------------------------------------------------
+// Every kernel starts with pdl_wait() (griddepcontrol.wait: returns once the previous kernel in the stream has
+// completed and its writes are visible; a no-op when launched without the PDL attribute) and pdl_trigger()
+// (griddepcontrol.launch_dependents: once every CTA of this grid has started, the next kernel may launch).
+// So each launch, block scheduling and prologue overlaps the previous kernel's last wave, with the same
+// ordering guarantees as plain stream order. LFD_PDL=0 in the environment disables the attribute.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+bool pdl_enabled();
+void pdl_suspend(bool s);  // graph capture: plain stream edges (measured faster inside graphs than PDL edges)
+template <typename... KArgs, typename... Args>
+cudaError_t launch_k(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+}
+
 // Per-domain stencil/current coefficients, rebuilt on the device from A (step a1 of SURVEY §8(a)).
 // For axis d and tau in {Delta/2 (p=0), Delta (p=1)} (p in {Delta_QD/2, Delta_QD}):
 //   alpha = e^{-i tau t_d} cos(tau t_d), up = sigma e^{+i theta_d}, dn = sigma e^{-i theta_d},

@@ -205,6 +205,8 @@ struct G1Shape {
 template <int kMT>
 __global__ void __launch_bounds__(kThreads1, 1) k_gemm1(const __grid_constant__ CUtensorMap tA,
                                                          const __grid_constant__ CUtensorMap tX, Gemm1Args p) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   using S = G1Shape<kMT>;
   extern __shared__ __align__(128) unsigned char smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages1 * S::StageBytes);
@@ -338,11 +340,11 @@ cudaError_t launch_gemm1(const Gemm1Args& a, cudaStream_t st) {
   cudaError_t e = gemm1_maps(a, mt, &tA, &tX);
   if (e != cudaSuccess) return e;
   if (mt == 16)
-    k_gemm1<16><<<grid, kThreads1, kStages1 * G1Shape<16>::StageBytes + 2 * kStages1 * 8, st>>>(tA, tX, a);
+    launch_k(k_gemm1<16>, grid, kThreads1, kStages1 * G1Shape<16>::StageBytes + 2 * kStages1 * 8, st, tA, tX, a);
   else if (mt == 32)
-    k_gemm1<32><<<grid, kThreads1, kStages1 * G1Shape<32>::StageBytes + 2 * kStages1 * 8, st>>>(tA, tX, a);
+    launch_k(k_gemm1<32>, grid, kThreads1, kStages1 * G1Shape<32>::StageBytes + 2 * kStages1 * 8, st, tA, tX, a);
   else
-    k_gemm1<64><<<grid, kThreads1, gemm1_smem_bytes(), st>>>(tA, tX, a);
+    launch_k(k_gemm1<64>, grid, kThreads1, gemm1_smem_bytes(), st, tA, tX, a);
   return cudaGetLastError();
 }
 
@@ -352,6 +354,8 @@ cudaError_t launch_gemm1(const Gemm1Args& a, cudaStream_t st) {
 // group order. Blocks past the element range reduce the column norms the same way. Deterministic.
 // ------------------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(256) k_reduce(ReduceArgs p, int eblocks) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   __shared__ double2 sh[8][32];
   const int dom = blockIdx.y;
   const int el = threadIdx.x & 31, sg = threadIdx.x >> 5;
@@ -413,7 +417,7 @@ cudaError_t launch_reduce(const ReduceArgs& a, cudaStream_t st) {
   const int eblocks = (int)((per_dom + 31) / 32);
   const int nblocks = a.s ? (a.ncols + 31) / 32 : 0;
   dim3 grid(eblocks + nblocks, a.ndom);
-  k_reduce<<<grid, 256, 0, st>>>(a, eblocks);
+  launch_k(k_reduce, grid, 256, 0, st, a, eblocks);
   return cudaGetLastError();
 }
 
@@ -424,6 +428,8 @@ cudaError_t launch_reduce(const ReduceArgs& a, cudaStream_t st) {
 __global__ void __launch_bounds__(256) k_nlnorm(int nproj, int norb, double eps2, const double2* __restrict__ G,
                                                 const double2* __restrict__ DC, const double* __restrict__ s,
                                                 double* __restrict__ nfac, double2* __restrict__ Cp) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   extern __shared__ double2 dcs[];  // DC[:, col]
   __shared__ double wq[8];
   const int dom = blockIdx.y, col = blockIdx.x;
@@ -470,7 +476,7 @@ __global__ void __launch_bounds__(256) k_nlnorm(int nproj, int norb, double eps2
 cudaError_t launch_nlnorm(int ndom, int nproj, int norb, double eps, const double2* G, const double2* DC,
                           const double* s, double* nfac, double2* Cp, cudaStream_t st) {
   dim3 grid(norb, ndom);
-  k_nlnorm<<<grid, 256, nproj * sizeof(double2), st>>>(nproj, norb, eps * eps, G, DC, s, nfac, Cp);
+  launch_k(k_nlnorm, grid, 256, nproj * sizeof(double2), st, nproj, norb, eps * eps, G, DC, s, nfac, Cp);
   return cudaGetLastError();
 }
 
@@ -486,6 +492,8 @@ __global__ void __launch_bounds__(256) k_nlmerge(int nproj, int norb, double eps
                                                  const double* __restrict__ D, const double2* __restrict__ DC,
                                                  const double* __restrict__ s, double2* __restrict__ X,
                                                  double* __restrict__ nfac) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   extern __shared__ double2 sh[];  // dc[np] | x[np]
   double2* dcs = sh;
   double2* xs = sh + nproj;
@@ -554,7 +562,7 @@ __global__ void __launch_bounds__(256) k_nlmerge(int nproj, int norb, double eps
 cudaError_t launch_nlmerge(int ndom, int nproj, int norb, double eps, const double2* G, const double* D,
                            const double2* DC, const double* s, double2* X, double* nfac, cudaStream_t st) {
   dim3 grid(norb, ndom);
-  k_nlmerge<<<grid, 256, 2 * nproj * sizeof(double2), st>>>(nproj, norb, eps, G, D, DC, s, X, nfac);
+  launch_k(k_nlmerge, grid, 256, 2 * nproj * sizeof(double2), st, nproj, norb, eps, G, D, DC, s, X, nfac);
   return cudaGetLastError();
 }
 
@@ -571,6 +579,8 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
                                                  const double* __restrict__ D, double2* DC, double2* X,
                                                  const double* __restrict__ s, double* nfac,
                                                  const double2* __restrict__ W) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   extern __shared__ double2 sh[];  // x[np] | dc[np] (dc is overwritten with DC_new)
   double2* xs = sh;
   double2* dcs = sh + nproj;
@@ -649,9 +659,9 @@ cudaError_t launch_nlcarry(int ndom, int nproj, int norb, double eps, const doub
                            const double2* W, cudaStream_t st) {
   dim3 grid(norb, ndom);
   if (with_norm && !W)
-    k_nlcarry<true><<<grid, 256, 2 * nproj * sizeof(double2), st>>>(nproj, norb, eps, G, D, DC, X, s, nfac, W);
+    launch_k(k_nlcarry<true>, grid, 256, 2 * nproj * sizeof(double2), st, nproj, norb, eps, G, D, DC, X, s, nfac, W);
   else
-    k_nlcarry<false><<<grid, 256, 2 * nproj * sizeof(double2), st>>>(nproj, norb, eps, G, D, DC, X, s, nfac, W);
+    launch_k(k_nlcarry<false>, grid, 256, 2 * nproj * sizeof(double2), st, nproj, norb, eps, G, D, DC, X, s, nfac, W);
   return cudaGetLastError();
 }
 
@@ -678,6 +688,8 @@ __device__ __forceinline__ void gemm2_chunk(const double2* As, const double2* Cs
 
 __global__ void __launch_bounds__(kThreads, 1) k_gemm2(const __grid_constant__ CUtensorMap tA,
                                                        const __grid_constant__ CUtensorMap tC, Gemm2Args p) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   extern __shared__ __align__(128) unsigned char smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages2 * kStage2Bytes);
   uint64_t* empty = full + kStages2;
@@ -814,6 +826,8 @@ __host__ __device__ constexpr int full_lda(int np) { return ((np + 3) / 4 * 4) %
 
 template <int kNP, bool kPvMid>
 __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   extern __shared__ __align__(128) unsigned char smem[];
   double2* Cs = reinterpret_cast<double2*>(smem + kFullStages * kFullABytes);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kFullStages * kFullABytes + kFullCBytes);
@@ -961,6 +975,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
 template <int kNP, bool kSkew, bool kOut = false>
 __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant__ CUtensorMap tB,
                                                              const __grid_constant__ CUtensorMap tC, Gemm2Args p) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   extern __shared__ __align__(128) unsigned char smem[];
   double2* Cs = reinterpret_cast<double2*>(smem + kFullStages * kFullABytes);
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + kFullStages * kFullABytes + kFullCBytes);
@@ -1121,11 +1137,11 @@ cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
     if (e != cudaSuccess) return e;
     const bool o = a.psi_out != nullptr;  // out of place (the self-consistent step's first factor)
     if (a.nproj == kTile) {
-      if (o) k_gemm2_tma<kTile, false, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
-      else k_gemm2_tma<kTile, false><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+      if (o) launch_k(k_gemm2_tma<kTile, false, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
+      else launch_k(k_gemm2_tma<kTile, false>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
     } else {
-      if (o) k_gemm2_tma<0, false, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
-      else k_gemm2_tma<0, false><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+      if (o) launch_k(k_gemm2_tma<0, false, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
+      else launch_k(k_gemm2_tma<0, false>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
     }
   } else if (a.nproj <= kTile && a.variant == 3) {
     CUtensorMap tB, tC;
@@ -1133,18 +1149,18 @@ cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
     if (e != cudaSuccess) return e;
     const bool o = a.psi_out != nullptr;
     if (a.nproj == kTile) {
-      if (o) k_gemm2_tma<kTile, true, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
-      else k_gemm2_tma<kTile, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+      if (o) launch_k(k_gemm2_tma<kTile, true, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
+      else launch_k(k_gemm2_tma<kTile, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
     } else {
-      if (o) k_gemm2_tma<0, true, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
-      else k_gemm2_tma<0, true><<<grid, kThreads, kFullSmem + 16, st>>>(tB, tC, a);
+      if (o) launch_k(k_gemm2_tma<0, true, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
+      else launch_k(k_gemm2_tma<0, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
     }
   } else if (a.nproj == kTile && a.variant == 1)
-    k_gemm2_fullk<kTile, true><<<grid, kThreads, kFullSmem, st>>>(a);
+    launch_k(k_gemm2_fullk<kTile, true>, grid, kThreads, kFullSmem, st, a);
   else if (a.nproj == kTile)
-    k_gemm2_fullk<kTile, false><<<grid, kThreads, kFullSmem, st>>>(a);
+    launch_k(k_gemm2_fullk<kTile, false>, grid, kThreads, kFullSmem, st, a);
   else if (a.nproj < kTile)
-    k_gemm2_fullk<0, false><<<grid, kThreads, kFullSmem, st>>>(a);
+    launch_k(k_gemm2_fullk<0, false>, grid, kThreads, kFullSmem, st, a);
   else {
     // B [dom][ng][nproj] (box [1][64 rows][kKC2 + 4 complex]) and C'' [dom][nproj][norb] (box [1][kKC2][66])
     CUtensorMap tA, tC;
@@ -1158,7 +1174,7 @@ cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
     const uint32_t bC[3] = {2 * kLd1, kKC2, 1};
     e = encode_tmap_f64(&tC, 3, a.Cp, dC, sC, bC);
     if (e != cudaSuccess) return e;
-    k_gemm2<<<grid, kThreads, gemm2_smem_bytes(), st>>>(tA, tC, a);
+    launch_k(k_gemm2, grid, kThreads, gemm2_smem_bytes(), st, tA, tC, a);
   }
   return cudaGetLastError();
 }

@@ -111,6 +111,8 @@ __global__ void __launch_bounds__(kSpThreads) k_gemm1_sp(const float2* __restric
                                                           double2* __restrict__ part, double* __restrict__ norms,
                                                           int mrows, int ncols, int nsplit, long long ng,
                                                           long long rps, long long a_ds, long long x_ds) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   extern __shared__ __align__(16) float2 sp_smem[];
   auto As = reinterpret_cast<float2(*)[kSpKC][kSpLdA]>(sp_smem);                       // [2][KC][LdA]
   auto Xs = reinterpret_cast<float2(*)[kSpKC][kSpLdA]>(sp_smem + 2 * kSpKC * kSpLdA);  // [2][KC][LdA]
@@ -216,6 +218,8 @@ __global__ void __launch_bounds__(kSpThreads) k_gemm1_sp(const float2* __restric
 __global__ void __launch_bounds__(kSpThreads) k_gemm2_sp(const float2* psi, float2* pout, const float2* __restrict__ B,
                                                           const float2* __restrict__ Xc, const double* __restrict__ nfac,
                                                           int np, int norb, long long ng) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   extern __shared__ __align__(16) float2 sp_smem[];
   auto Bs = reinterpret_cast<float2(*)[kSpT][kSpLdK]>(sp_smem);                        // [2][T][LdK]
   auto Xs = reinterpret_cast<float2(*)[kSpKC][kSpLdA]>(sp_smem + 2 * kSpT * kSpLdK);   // [2][KC][LdA]
@@ -308,6 +312,8 @@ __global__ void __launch_bounds__(kSpThreads) k_gemm2_sp(const float2* psi, floa
 }
 
 __global__ void k_to_c64(const double2* __restrict__ in, float2* __restrict__ out, long long n) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) out[i] = make_float2((float)in[i].x, (float)in[i].y);
 }
@@ -326,7 +332,7 @@ cudaError_t gemm_sp_set_attributes() {
 cudaError_t launch_gemm1_sp(const Gemm1Args& a, const float2* A, const float2* X, cudaStream_t st) {
   const int mt = (a.mrows + kSpT - 1) / kSpT, nt = (a.ncols + kSpT - 1) / kSpT;
   dim3 grid(a.nsplit, mt * nt, a.ndom);
-  k_gemm1_sp<<<grid, kSpThreads, kSmem1, st>>>(A, X, a.part, a.norms, a.mrows, a.ncols, a.nsplit, a.ng, a.rows_per_split,
+  launch_k(k_gemm1_sp, grid, kSpThreads, kSmem1, st, A, X, a.part, a.norms, a.mrows, a.ncols, a.nsplit, a.ng, a.rows_per_split,
                                           a.a_dom_stride, a.x_dom_stride);
   return cudaGetLastError();
 }
@@ -334,11 +340,11 @@ cudaError_t launch_gemm1_sp(const Gemm1Args& a, const float2* A, const float2* X
 cudaError_t launch_gemm2_sp(float2* psi, const float2* B, const double2* Cp, float2* X32, const double* nfac,
                             int ndom, int nproj, int norb, long long ng, cudaStream_t st, float2* psi_out) {
   const long long n = (long long)ndom * nproj * norb;
-  k_to_c64<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(Cp, X32, n);
+  launch_k(k_to_c64, (unsigned)((n + 255) / 256), 256, 0, st, Cp, X32, n);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   dim3 grid((unsigned)((ng + kSpT - 1) / kSpT), (norb + kSpT - 1) / kSpT, ndom);
-  k_gemm2_sp<<<grid, kSpThreads, kSmem2, st>>>(psi, psi_out ? psi_out : psi, B, X32, nfac, nproj, norb, ng);
+  launch_k(k_gemm2_sp, grid, kSpThreads, kSmem2, st, psi, psi_out ? psi_out : psi, B, X32, nfac, nproj, norb, ng);
   return cudaGetLastError();
 }
 

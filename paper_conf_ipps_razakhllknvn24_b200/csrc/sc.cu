@@ -27,6 +27,8 @@ constexpr double kPi = 3.141592653589793238462643383279502884;
 __global__ void k_sc_maxwell_begin(double* __restrict__ st, double3 a_mid, double3 a_end, double dt, int maxwell,
                                    int ndom, double hx, double hy, double hz, DomCoef* __restrict__ coef_mid,
                                    DomCoef* __restrict__ coef_end) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   __shared__ double Am[3], Ae[3];
   if (threadIdx.x == 0) {
     const double am[3] = {a_mid.x, a_mid.y, a_mid.z}, ae[3] = {a_end.x, a_end.y, a_end.z};
@@ -58,6 +60,8 @@ __global__ void k_sc_maxwell_begin(double* __restrict__ st, double3 a_mid, doubl
 // End of a step: Jbar(t_n+1) from the (all-reduced) density buffer; A_ind <- A_ind(t_n+1) and the second
 // half kick dA/dt <- dA/dt(n+1/2) - 2 pi c dt Jbar(t_n+1).
 __global__ void k_sc_maxwell_end(double* __restrict__ st, const double* __restrict__ jbar, double dt, int maxwell) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   const int d = threadIdx.x;
   if (d >= 3) return;
   const double J = jbar[d];
@@ -70,6 +74,8 @@ __global__ void k_sc_maxwell_end(double* __restrict__ st, const double* __restri
 
 // Jbar = sum_dom J_dom * (ng / GN): this rank's share of the global-grid mean current (fixed order).
 __global__ void k_sc_jbar(const double* __restrict__ Jmac, int ndom, double w, double* __restrict__ out) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   const int d = threadIdx.x;
   if (d >= 3) return;
   double s = 0.0;
@@ -81,6 +87,8 @@ __global__ void k_sc_jbar(const double* __restrict__ Jmac, int ndom, double w, d
 __global__ void k_sc_vmid(const double* __restrict__ vion, const double* __restrict__ va,
                           const double* __restrict__ vb, double wa, double wb, const int* __restrict__ off,
                           int nx, int ny, int nz, int GY, int GZ, long long total, double* __restrict__ vout) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= total) return;
   const long long ng = (long long)nx * ny * nz;
@@ -99,6 +107,8 @@ __global__ void k_sc_vmid(const double* __restrict__ vion, const double* __restr
 // rho_G -> 4 pi / |G|^2 rho_G / GN (G = 0 dropped: neutralising background), on the D2Z half spectrum
 // [GX][GY][GZ/2+1]; |m_d| = min(k, N_d - k) (the Nyquist term of an even N_d is its own mirror).
 __global__ void k_sc_poisson(double2* __restrict__ spec, int GX, int GY, int GZ, double hx, double hy, double hz) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   const int GZh = GZ / 2 + 1;
   const long long n = (long long)GX * GY * GZh;
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
@@ -116,6 +126,8 @@ __global__ void k_sc_poisson(double2* __restrict__ spec, int GX, int GY, int GZ,
 
 // v_Hxc[g] = (hartree ? v_H[g] : 0) + (xc ? -(3 rho / pi)^{1/3} : 0), in place on v (v_H from the Z2D).
 __global__ void k_sc_vhxc(const double* __restrict__ rho, double* __restrict__ v, long long n, int hartree, int xc) {
+  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
+  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   double r = hartree ? v[i] : 0.0;
@@ -126,38 +138,38 @@ __global__ void k_sc_vhxc(const double* __restrict__ rho, double* __restrict__ v
 // ---- launchers ------------------------------------------------------------------------------------
 cudaError_t launch_sc_maxwell_begin(double* st, const double* a_mid, const double* a_end, double dt, bool maxwell,
                                     const Geometry& g, DomCoef* coef_mid, DomCoef* coef_end, cudaStream_t s) {
-  k_sc_maxwell_begin<<<1, 256, 0, s>>>(st, make_double3(a_mid[0], a_mid[1], a_mid[2]),
+  launch_k(k_sc_maxwell_begin, 1, 256, 0, s, st, make_double3(a_mid[0], a_mid[1], a_mid[2]),
                                        make_double3(a_end[0], a_end[1], a_end[2]), dt, maxwell ? 1 : 0, g.ndom,
                                        g.hx, g.hy, g.hz, coef_mid, coef_end);
   return cudaGetLastError();
 }
 
 cudaError_t launch_sc_maxwell_end(double* st, const double* jbar, double dt, bool maxwell, cudaStream_t s) {
-  k_sc_maxwell_end<<<1, 32, 0, s>>>(st, jbar, dt, maxwell ? 1 : 0);
+  launch_k(k_sc_maxwell_end, 1, 32, 0, s, st, jbar, dt, maxwell ? 1 : 0);
   return cudaGetLastError();
 }
 
 cudaError_t launch_sc_jbar(const double* Jmac, int ndom, double w, double* out, cudaStream_t s) {
-  k_sc_jbar<<<1, 32, 0, s>>>(Jmac, ndom, w, out);
+  launch_k(k_sc_jbar, 1, 32, 0, s, Jmac, ndom, w, out);
   return cudaGetLastError();
 }
 
 cudaError_t launch_sc_vmid(const Geometry& g, const double* vion, const double* va, const double* vb, double wa,
                            double wb, const int* off, int GY, int GZ, double* vout, cudaStream_t s) {
   const long long total = (long long)g.ndom * g.ng;
-  k_sc_vmid<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(vion, va, vb, wa, wb, off, g.nx, g.ny, g.nz, GY, GZ,
+  launch_k(k_sc_vmid, (unsigned)((total + 255) / 256), 256, 0, s, vion, va, vb, wa, wb, off, g.nx, g.ny, g.nz, GY, GZ,
                                                             total, vout);
   return cudaGetLastError();
 }
 
 cudaError_t launch_sc_poisson(double2* spec, const int* gd, const Geometry& g, cudaStream_t s) {
   const long long n = (long long)gd[0] * gd[1] * (gd[2] / 2 + 1);
-  k_sc_poisson<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(spec, gd[0], gd[1], gd[2], g.hx, g.hy, g.hz);
+  launch_k(k_sc_poisson, (unsigned)((n + 255) / 256), 256, 0, s, spec, gd[0], gd[1], gd[2], g.hx, g.hy, g.hz);
   return cudaGetLastError();
 }
 
 cudaError_t launch_sc_vhxc(const double* rho, double* v, long long n, bool hartree, bool xc, cudaStream_t s) {
-  k_sc_vhxc<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(rho, v, n, hartree ? 1 : 0, xc ? 1 : 0);
+  launch_k(k_sc_vhxc, (unsigned)((n + 255) / 256), 256, 0, s, rho, v, n, hartree ? 1 : 0, xc ? 1 : 0);
   return cudaGetLastError();
 }
 

@@ -2,7 +2,21 @@
 // entry point, so the library needs no libcuda link). Used by the stencil and GEMM kernels.
 #include "lfd_internal.h"
 
+#include <cstdlib>
+
 namespace lfd {
+
+thread_local bool g_pdl_suspended = false;  // set while a CUDA graph is captured (plain edges measured faster)
+
+bool pdl_enabled() {
+  static const bool on = [] {
+    const char* v = std::getenv("LFD_PDL");
+    return !(v && v[0] == '0');
+  }();
+  return on && !g_pdl_suspended;
+}
+
+void pdl_suspend(bool s) { g_pdl_suspended = s; }
 
 cudaError_t encode_tmap_f64(CUtensorMap* out, int rank, const void* base, const uint64_t* dims,
                             const uint64_t* strides_bytes, const uint32_t* box) {
