@@ -51,7 +51,7 @@ def ncu_traffic(kernel):
     scale = {"[byte]": 1.0, "[Kbyte]": 1e3, "[Mbyte]": 1e6, "[Gbyte]": 1e9}
     vals = []
     for r in rows[1:]:
-        if r[0].replace("void ", "").startswith(NCU_NAMES[kernel]):
+        if r[0].replace("void ", "").replace("lfd::", "").startswith(NCU_NAMES[kernel]):
             sr = next((v for k, v in scale.items() if hdr[ir].endswith(k)), 1.0)
             sw = next((v for k, v in scale.items() if hdr[iw].endswith(k)), 1.0)
             vals.append(float(r[ir]) * sr + float(r[iw]) * sw)
@@ -347,7 +347,15 @@ def run_sp_mode(args, w, x, dev, stream, pk):
         e = {"ms_per_launch": avg, "launches": cnt, "share": round(kms / tot, 4)}
         if k in work:
             b, f = work[k]
-            if f > 0:
+            if k == "nl_back" and nl_path == 1:
+                # int8-digit tcgen05 GEMM-2 (FP64 accuracy): the digit products are cheap on the int8 tensor
+                # cores, so the kernel is bound by streaming Psi (read + write) and B -- report it against
+                # HBM with the FP64 operation's algorithmic bytes, and its FP64-equivalent rate alongside
+                e.update({"bound": "hbm", "achieved": b / (avg * 1e-3) / 1e9, "unit": "GB/s", "peak": pk["hbm_gbs"],
+                          "path": "int8-digit tcgen05 (FP64 accuracy)",
+                          "fp64_equiv_tflops": f / (avg * 1e-3) / 1e12,
+                          "fp64_equiv_vs_dmma_peak": f / (avg * 1e-3) / 1e12 / pk["zgemm3m_tflops"]})
+            elif f > 0:
                 e.update({"bound": "tensor", "achieved": f / (avg * 1e-3) / 1e12, "unit": "TFLOP/s", "peak": tpeak})
             else:
                 e.update({"bound": "hbm", "achieved": 0.5 * b / (avg * 1e-3) / 1e9, "unit": "GB/s",
@@ -448,6 +456,7 @@ def main():
     del p0
     pk = peaks()
     work = kernel_work(w)
+    nl_path = lfd.lfd_nl_path(ctx.ctx)
     kernels = {}
     total_ms = sum(v[0] for v in prof.values())
     for k, (kms, cnt) in prof.items():
@@ -457,7 +466,15 @@ def main():
         e = {"ms_per_launch": avg, "launches": cnt, "share": kms / total_ms if total_ms else None}
         if k in work:
             b, f = work[k]
-            if f > 0:
+            if k == "nl_back" and nl_path == 1:
+                # int8-digit tcgen05 GEMM-2 (FP64 accuracy): the digit products are cheap on the int8 tensor
+                # cores, so the kernel is bound by streaming Psi (read + write) and B -- report it against
+                # HBM with the FP64 operation's algorithmic bytes, and its FP64-equivalent rate alongside
+                e.update({"bound": "hbm", "achieved": b / (avg * 1e-3) / 1e9, "unit": "GB/s", "peak": pk["hbm_gbs"],
+                          "path": "int8-digit tcgen05 (FP64 accuracy)",
+                          "fp64_equiv_tflops": f / (avg * 1e-3) / 1e12,
+                          "fp64_equiv_vs_dmma_peak": f / (avg * 1e-3) / 1e12 / pk["zgemm3m_tflops"]})
+            elif f > 0:
                 e.update({"bound": "tensor", "achieved": f / (avg * 1e-3) / 1e12, "unit": "TFLOP/s",
                           "peak": pk["zgemm3m_tflops"]})
             else:
@@ -472,6 +489,7 @@ def main():
                 "traffic_source": "profiles/latest_ncu_full_summary.csv (dram__bytes_read.sum + dram__bytes_write.sum "
                                   "per launch, ncu --set full)",
                 "peak_source": pk["zgemm3m_src"] if d["bound"] == "tensor" else pk["hbm_src"],
+                "nl_gemm2_path": {0: "fp64-dmma", 1: "int8-digit-tcgen05", 2: "sp-3xtf32", -1: "none"}[nl_path],
                 "flops_per_launch" if d["bound"] == "tensor" else "bytes_per_launch":
                     work[dom][1] if d["bound"] == "tensor" else work[dom][0]}
 

@@ -65,7 +65,7 @@ typedef struct {
   int32_t nref_max;    /* max reference-basis columns for lfd_remap_occ, 0..2048 (0: max(norb, nproj)) */
   double dt;           /* Delta_QD [a.u.], finite and nonzero (negative = backward in time) */
   int32_t device;      /* CUDA device ordinal */
-  int32_t flags;       /* 0 or LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP */
+  int32_t flags;       /* 0 or LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP | LFD_FLAG_NL_DMMA */
 } lfd_config;
 
 /* lfd_config.flags: disable the projection carry (lfd_step takes the C of each nonlocal factor that
@@ -85,6 +85,13 @@ typedef struct {
  * O(nproj x norb) -- the split reduction, the Gram matrix, n_s, the carry, the energies -- in FP64. Results
  * agree with the FP64 path to single-precision roundoff (DESIGN.md §4 states the tolerance). */
 #define LFD_FLAG_SP 4
+/* lfd_config.flags: run the nonlocal GEMM-2 (Psi <- Psi diag(n) + B C'') as complex FP64 DMMA
+ * (mma.sync m8n8k4) instead of the default for FP64 contexts with nproj <= 64 and norb <= 64: the same
+ * product with FP64 accuracy on the tcgen05 int8 tensor cores -- B and C'' split exactly into 6 int8
+ * digits each with power-of-two row / column scales, the 21 digit-pair products accumulated exactly in
+ * int32 in tensor memory, recombined in FP64 (relative error of the product ~3e-12, i.e. ~1e-15 of Psi
+ * per factor since the update is O(Delta Delta_sci / 2) of Psi). See lfd_nl_path(). */
+#define LFD_FLAG_NL_DMMA 8
 
 /* Kernel classes, for lfd_profile_read(). */
 typedef enum {
@@ -119,6 +126,7 @@ lfd_status lfd_workspace_size(const lfd_config* cfg, size_t* bytes);
  *  proj  DEVICE complex128 [ndom][nx][ny][nz][nproj]; borrowed, read-only (B = Psi_u(0), the
  *        unoccupied KS orbitals at t = 0, Eq. 7 P:68 / R9); NULL iff nproj == 0. Need not be
  *        orthonormal: the Gram matrix G = dV B^H B is computed here (on the device) and used for n_s.
+ *        Must not change while the context lives: G and (default path) B's int8 digits are made here.
  *  dnl   HOST double [ndom][nproj] real couplings D_u (paper: all equal Delta_sci of Eq. 8);
  *        copied. May be NULL iff nproj == 0.
  *  occ   HOST double [ndom][norb] occupations f_s (not clamped, R14); copied.
@@ -274,6 +282,11 @@ lfd_status lfd_sync(lfd_ctx* ctx);
 
 /* Number of kernels this context has launched so far (all classes). */
 lfd_status lfd_launch_count(const lfd_ctx* ctx, uint64_t* count);
+
+/* Which kernel runs the nonlocal GEMM-2 of this context: *path = 0 complex FP64 DMMA (mma.sync),
+ * 1 int8-digit tcgen05 tensor cores with FP64 accuracy (LFD_FLAG_NL_DMMA), 2 SP 3xTF32 (LFD_FLAG_SP),
+ * -1 no nonlocal factor (nproj == 0). */
+lfd_status lfd_nl_path(const lfd_ctx* ctx, int32_t* path);
 
 /* Per-kernel-class device timing with CUDA events on the context stream.
  * lfd_profile_enable(ctx, 1) starts recording an event pair around every launch;

@@ -32,8 +32,9 @@ size_t up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 struct Layout {
   size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage, cref,
-      epart, W, ones, x32, aseq, jseq;
+      epart, W, ones, x32, aseq, jseq, bsl, bsig;
   int nref_cap;
+  bool i8;  // GEMM-2 on the int8 tensor cores (nl_i8.cu): B digit tiles + row scales in the workspace
   size_t total;
   int nsplit;
   long long rows_per_split;
@@ -65,7 +66,10 @@ lfd_status validate(const lfd_config* c, std::string& why) {
   if (c->norb < 1) { why = "norb must be >= 1"; return LFD_EINVAL; }
   if (c->nproj < 0 || c->nproj > 2048) { why = "nproj must be in [0, 2048]"; return LFD_EINVAL; }
   if (!(c->dt != 0.0) || !std::isfinite(c->dt)) { why = "dt must be finite and nonzero"; return LFD_EINVAL; }
-  if (c->flags & ~(LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP)) { why = "unknown flags"; return LFD_EINVAL; }
+  if (c->flags & ~(LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP | LFD_FLAG_NL_DMMA)) {
+    why = "unknown flags";
+    return LFD_EINVAL;
+  }
   if (c->nref_max < 0 || c->nref_max > 2048) { why = "nref_max must be in [0, 2048]"; return LFD_EINVAL; }
   const long long ng = (long long)c->nx * c->ny * c->nz;
   if (ng * (long long)std::max(c->norb, std::max(c->nproj, 1)) >= (1LL << 31)) {
@@ -75,6 +79,14 @@ lfd_status validate(const lfd_config* c, std::string& why) {
   return LFD_OK;
 }
 
+// GEMM-2 on the tcgen05 int8 tensor cores with FP64 accuracy (nl_i8.cu): the default for FP64 contexts with
+// nproj, norb <= 64; LFD_FLAG_NL_DMMA (or env LFD_NL_I8=0, an A/B knob) selects the DMMA kernels.
+bool use_i8(const lfd_config* c) {
+  bool on = (c->flags & (LFD_FLAG_NL_DMMA | LFD_FLAG_SP)) == 0;
+  if (const char* v = std::getenv("LFD_NL_I8")) on = on && std::atoi(v) != 0;
+  return on && lfd::gemm2_i8_supported(c->nproj, c->norb);
+}
+
 Geometry geometry(const lfd_config* c) {
   Geometry g;
   g.ndom = c->ndomains; g.nx = c->nx; g.ny = c->ny; g.nz = c->nz;
@@ -82,11 +94,13 @@ Geometry geometry(const lfd_config* c) {
   g.hx = c->hx; g.hy = c->hy; g.hz = c->hz; g.dt = c->dt; g.dV = c->hx * c->hy * c->hz;
   g.ng = (long long)c->nx * c->ny * c->nz;
   g.sp = (c->flags & LFD_FLAG_SP) ? 1 : 0;
+  g.i8 = use_i8(c) ? 1 : 0;
   return g;
 }
 
 Layout layout(const Geometry& g, int num_sms, int nref_max) {
   Layout L{};
+  L.i8 = g.i8 != 0;
   L.nref_cap = nref_max > 0 ? nref_max : std::max(g.norb, g.nproj);
   const int np = g.nproj, no = g.norb, nd = g.ndom;
   // split-K of GEMM-1: about one CTA per SM in total, each split a multiple of the chunk height
@@ -144,6 +158,8 @@ Layout layout(const Geometry& g, int num_sms, int nref_max) {
   L.x32 = g.sp ? take((size_t)nd * np * no * 8) : 0;  // SP: the GEMM-2 coefficient rounded to complex64
   L.aseq = take((size_t)kGraphChunk * nd * 3 * d8);   // lfd_step_graph: A of the chunk's steps
   L.jseq = take((size_t)kGraphChunk * nd * 3 * d8);   // lfd_step_graph: J of the chunk's steps
+  L.bsl = L.i8 ? take(lfd::gemm2_i8_bytes(nd, g.ng)) : 0;
+  L.bsig = L.i8 ? take(lfd::gemm2_i8_sig_bytes(nd, g.ng)) : 0;
   L.total = o;
   return L;
 }
@@ -403,6 +419,11 @@ lfd_status gemm2(lfd_ctx* c, double2* out = nullptr) {
   a2.ndom = g.ndom; a2.nproj = g.nproj; a2.norb = g.norb; a2.ng = g.ng; a2.num_sms = c->num_sms;
   a2.variant = c->gemm2_variant;
   a2.psi_out = out;
+  if (c->L.i8) {
+    a2.bsl = c->at<int8_t>(c->L.bsl);
+    a2.bsig = c->at<double>(c->L.bsig);
+    if (const char* v = std::getenv("LFD_I8_DBG")) a2.dbg = std::atoi(v);
+  }
   c->c_valid = false;
   if (g.sp)
     LFD_TRY(launch(c, LFD_K_NL_BACK, "k_gemm2_sp", [&] {
@@ -815,6 +836,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   if (e == cudaSuccess) e = lfd::density_set_attributes();
   if (e == cudaSuccess) e = lfd::kin_yz_set_attributes();
   if (e == cudaSuccess) e = lfd::gemm_sp_set_attributes();
+  if (e == cudaSuccess) e = lfd::gemm_i8_set_attributes();
   if (e != cudaSuccess) return cuda_fail(nullptr, e, "cudaFuncSetAttribute");
 
   lfd_ctx* c = new (std::nothrow) lfd_ctx();
@@ -884,6 +906,13 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
     r.part = a1.part; r.normp = nullptr; r.D = nullptr; r.out = c->at<double2>(L.G); r.cprime = nullptr; r.s = nullptr;
     r.ndom = g.ndom; r.mrows = g.nproj; r.ncols = g.nproj; r.nsplit = L.nsplit; r.scale = g.dV; r.eps = 0;
     s2 = launch(c, LFD_K_NL_REDUCE, "k_reduce(G)", [&] { return lfd::launch_reduce(r, c->stream); });
+    if (s2 != LFD_OK) return bail(s2);
+  }
+  if (L.i8) {  // int8 digit tiles of B for the tensor-core GEMM-2 (B is constant, like G)
+    s2 = launch(c, LFD_K_NL_BACK, "k_bslice_i8", [&] {
+      return lfd::launch_bslice_i8(c->proj, g.ndom, g.nproj, g.ng, c->at<int8_t>(L.bsl), c->at<double>(L.bsig),
+                                   c->stream);
+    });
     if (s2 != LFD_OK) return bail(s2);
   }
   if (cfg->flags & LFD_FLAG_EXACT_NL) {
@@ -1361,6 +1390,13 @@ lfd_status lfd_sync(lfd_ctx* c) {
   cudaError_t e = cudaStreamSynchronize(c->stream);
   if (e == cudaSuccess) e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "asynchronous CUDA error");
+  return LFD_OK;
+}
+
+lfd_status lfd_nl_path(const lfd_ctx* c, int32_t* path) {
+  LFD_TRY(check_ctx(c));
+  if (!path) return LFD_EINVAL;
+  *path = c->g.nproj == 0 ? -1 : c->g.sp ? 2 : c->L.i8 ? 1 : 0;
   return LFD_OK;
 }
 

@@ -58,6 +58,7 @@ struct DomCoef {
 struct Geometry {
   int ndom, nx, ny, nz, norb, nproj, bc;
   int sp;  // 1: SP variant (complex64 Psi / B, FP32 sweeps and 3xTF32 tensor-core GEMMs), else FP64
+  int i8;  // 1: GEMM-2 on the int8-digit tcgen05 path (nl_i8.cu), else DMMA / SP
   double hx, hy, hz, dt, dV;
   long long ng;  // points per domain
 };
@@ -159,8 +160,20 @@ struct Gemm2Args {
   long long ng;
   int num_sms;
   int variant;  // tuning knob (LFD_GEMM2_VARIANT): 0 = epilogue loads after the K loop, 1 = mid-loop
+  // int8-digit tensor-core path (nl_i8.cu): B's digit tiles and row scales from launch_bslice_i8, or nullptr
+  const int8_t* bsl = nullptr;
+  const double* bsig = nullptr;
+  int dbg = 0;  // diagnostics only (env LFD_I8_DBG): 1 = one digit pair per tile, 2 = no epilogue math
 };
 cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st);
+// GEMM-2 with FP64 accuracy on the tcgen05 int8 tensor cores (nl_i8.cu): nproj <= 64, norb <= 64.
+bool gemm2_i8_supported(int nproj, int norb);
+size_t gemm2_i8_bytes(int ndom, long long ng);      // B digit tiles
+size_t gemm2_i8_sig_bytes(int ndom, long long ng);  // B row scales
+cudaError_t launch_bslice_i8(const double2* B, int ndom, int nproj, long long ng, int8_t* out, double* sig,
+                             cudaStream_t st);
+cudaError_t launch_gemm2_i8(const Gemm2Args& a, cudaStream_t st);
+cudaError_t gemm_i8_set_attributes();
 int gemm2_smem_bytes();
 cudaError_t gemm_set_attributes();
 

@@ -1128,6 +1128,7 @@ static cudaError_t gemm2_maps(const Gemm2Args& a, CUtensorMap* tB, CUtensorMap* 
 }
 
 cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
+  if (a.bsl) return launch_gemm2_i8(a, st);
   const long long rblocks = (a.ng + kTile - 1) / kTile;
   const long long items = (long long)a.ndom * rblocks * ((a.norb + kTile - 1) / kTile);
   const int grid = (int)(items < a.num_sms ? items : a.num_sms);

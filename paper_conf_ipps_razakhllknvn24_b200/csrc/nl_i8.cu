@@ -1,0 +1,442 @@
+// nl_i8.cu -- GEMM-2 of the nonlocal factor (Eq. 9 / P:210) on the tcgen05 tensor
+// cores with FP64 accuracy: the FP64 operands are split into int8 digit slices (an Ozaki-type scheme), the
+// digit products run as tcgen05.mma kind::i8 with exact int32 accumulation in TMEM, and the epilogue
+// recombines them in FP64.
+//
+//   Psi[r][s] <- n_s Psi[r][s] + sum_u B[r][u] X[u][s]          (X = C'' = C' diag(n), nl.cu)
+//
+// Real form. With n = 2s + c (Psi's interleaved re/im doubles) and k = 2u + c' (B's), the complex product
+// is one real GEMM out[r][n] = sum_k Bre[r][k] W[k][n], W[2u][2s] = Re X, W[2u+1][2s] = -Im X,
+// W[2u][2s+1] = Im X, W[2u+1][2s+1] = Re X (K = 2 nproj <= 128, N = 2 norb <= 128).
+//
+// Digits. Every row r of B (over k) and every column n of W (over k) gets a power-of-two scale
+// sigma_r = 2^e (max_k |B[r][k]| < 2^e), and x = B / sigma_r in (-1, 1) is written exactly as
+//   x = sum_{i=1..S} d_i 2^{-6-7(i-1)} + rest,  d_1 = rint(64 x),  d_{i+1} = rint(128 (residual_i)),
+// |d_i| <= 64, |rest| <= 2^{-7S-1} (each step is exact in FP64: scaling by powers of two and subtracting
+// an integer). The same for W with tau_n. Then
+//   out[r][n] ~= sigma_r tau_n sum_{d=2..S+1} 2^{-12-7(d-2)} P_d[r][n],  P_d = sum_{i+j=d} sum_k b_i w_j,
+// and each P_d is an exact int32 sum (|P_d| <= 6 * 128 * 64 * 64 < 2^22). The terms dropped (i+j > S+1)
+// and the digit remainders are O(2^-42) relative to sigma_r tau_n: with S = 6 the product is accurate to
+// ~1e-12 relative (tools/i8_model.py), and since the update B X is O(eps = Delta Delta_sci / 2 ~ 1.4e-3)
+// of Psi, the error on Psi per factor is ~1e-15 -- the north star's 1e-10 after 100 steps holds with a
+// wide margin (tests/test_gpu_i8.py checks the same bound as the FP64 path).
+//
+// Kernel (B200-first). The B digits are built ONCE at lfd_init (B is constant: P:216's resident Psi_u(0))
+// into tiles of 32 grid points, each tile [S][32 rows][128 B] already in the canonical K-major
+// SWIZZLE_128B shared-memory image, so one cp.async.bulk per tile stages it. Per call every CTA builds the
+// W digits (6 x 16 KB) from C'' itself, straight into TMEM (tcgen05.st), where they are the MMA's A
+// operand -- shared memory is left to the two streaming rings. Transposed MMA: D[n][r] = sum_k W^T[n][k]
+// b[r][k] (M = 128 output columns n on the TMEM lanes, N = 32 grid points), so each epilogue lane owns one
+// Psi double n and a warp reads/writes 256 contiguous bytes per grid point. Roles: warp 8 = producer of the
+// digit tiles, warp 10 = producer of the tile's Psi rows (contiguous in HBM: one bulk copy into a 2-deep
+// shared-memory ring), warp 9 = MMA issuer (21 digit pairs x 4 K-steps per tile into 6 diagonal
+// accumulators), warps 0-7 = epilogue (tcgen05.ld, FP64 recombination, Psi update stored to HBM). The
+// epilogue releases the accumulators as soon as they are in registers, so the MMAs of tile t+1 overlap
+// its FP64 work on tile t; the digit ring (3 x 24 KB) and the Psi ring (4 x 32 KB) keep ~150 KB per SM in
+// flight.
+#include "lfd_internal.h"
+#include "lfd_tma.cuh"
+
+#include <type_traits>
+
+namespace lfd {
+
+constexpr int kI8S = 6;                             // digits per operand
+constexpr int kI8NT = 64;                           // grid points per tile (MMA N)
+constexpr int kI8K = 128;                           // bytes per digit row: K = 2 nproj padded to 128
+constexpr int kI8M = 128;                           // MMA M: 2 norb padded to 128
+constexpr int kI8Stages = 2;                        // digit-tile ring
+constexpr int kI8Slots = 4;                         // TMEM ring of diagonal accumulators (kI8NT columns each)
+constexpr int kI8Half = kI8NT / 2;                  // tile rows per epilogue warp
+constexpr int kI8SliceB = kI8NT * kI8K;             // 8 KB: one digit slice of a tile
+constexpr int kI8TileB = kI8S * kI8SliceB;          // 48 KB: all digits of a tile
+constexpr int kI8SubR = 16;                         // Psi rows per staged sub-tile
+constexpr int kI8SubRowsB = kI8SubR * 64 * 16;      // 16 KB (norb <= 64)
+constexpr int kI8SubB = kI8SubRowsB + kI8SubR * 8;  // + the sub-tile's row scales sigma_r
+constexpr int kI8PsiSlots = 7;                      // Psi sub-tile ring (first 64 KB also stage C'')
+constexpr int kI8Smem = kI8Stages * kI8TileB + kI8PsiSlots * kI8SubB + 1024;  // + alignment slack
+constexpr int kI8WCols = kI8S * (kI8K / 4);        // 192 TMEM columns: W^T digits (4 int8 per column)
+constexpr int kI8Acc = kI8S;                        // diagonals d = 2 .. S+1
+constexpr int kI8Threads = 352;                     // 8 epilogue warps + 2 producers + MMA
+
+// byte offset of (row, k) in a K-major SWIZZLE_128B image with 128-byte rows (8-row, 1024-byte atoms;
+// the 16-byte chunk index is XOR-ed with the row within the atom)
+__host__ __device__ __forceinline__ int sw128(int row, int k) {
+  return ((row >> 3) << 10) + ((row & 7) << 7) + ((((k >> 4) ^ (row & 7))) << 4) + (k & 15);
+}
+
+// the digits of 4 consecutive values of one row; the scale exponent e is shared by the row (x = v 2^-e)
+__device__ __forceinline__ void digits4(const double v[4], int e, bool zero, uint32_t out[kI8S]) {
+  double x[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) x[q] = zero ? 0.0 : ldexp(v[q], 6 - e);  // 64 x, exact
+#pragma unroll
+  for (int i = 0; i < kI8S; ++i) {
+    uint32_t w = 0;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const double d = rint(x[q]);
+      x[q] = (x[q] - d) * 128.0;  // exact: |x - d| <= 1/2
+      w |= ((uint32_t)(int)d & 0xffu) << (8 * q);
+    }
+    out[i] = w;
+  }
+}
+
+// exact int32 -> FP64 without the (low-rate) I2F.F64 conversion: 2^52 + (x + 2^31) built from bits, minus
+// 2^52 + 2^31 (one full-rate DADD)
+__device__ __forceinline__ double i2d(int32_t x) {
+  return __hiloint2double(0x43300000, (int)((uint32_t)x ^ 0x80000000u)) - 4503601774854144.0;
+}
+
+__device__ __forceinline__ int row_exponent(double mx) {
+  int e = 0;
+  frexp(mx, &e);  // mx = m 2^e, m in [0.5, 1): mx < 2^e
+  return e;
+}
+
+// ---- B digits (once per lfd_init): warp per grid row -------------------------------------------------
+__global__ void __launch_bounds__(256) k_bslice_i8(const double2* __restrict__ B, int nproj, long long ng,
+                                                   long long tiles, int8_t* __restrict__ out,
+                                                   double* __restrict__ sig) {
+  pdl_wait();
+  pdl_trigger();
+  const int dom = blockIdx.y, lane = threadIdx.x & 31;
+  const long long r = (long long)blockIdx.x * 8 + (threadIdx.x >> 5);
+  if (r >= tiles * kI8NT) return;
+  double v[4] = {0.0, 0.0, 0.0, 0.0};
+  const int u0 = 2 * lane;
+  if (r < ng) {
+    const double2* row = B + ((long long)dom * ng + r) * nproj;
+    if (u0 < nproj) { const double2 a = row[u0]; v[0] = a.x; v[1] = a.y; }
+    if (u0 + 1 < nproj) { const double2 a = row[u0 + 1]; v[2] = a.x; v[3] = a.y; }
+  }
+  double mx = fmax(fmax(fabs(v[0]), fabs(v[1])), fmax(fabs(v[2]), fabs(v[3])));
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  const int e = mx > 0.0 ? row_exponent(mx) : 0;
+  uint32_t d[kI8S];
+  digits4(v, e, !(mx > 0.0), d);
+  const long long t = r / kI8NT;
+  const int rr = (int)(r - t * kI8NT);
+  int8_t* tb = out + ((long long)dom * tiles + t) * kI8TileB;
+#pragma unroll
+  for (int i = 0; i < kI8S; ++i) *reinterpret_cast<uint32_t*>(tb + i * kI8SliceB + sw128(rr, 4 * lane)) = d[i];
+  if (lane == 0) sig[(long long)dom * tiles * kI8NT + r] = mx > 0.0 ? ldexp(1.0, e) : 0.0;
+}
+
+// ---- tcgen05 helpers (inline PTX) ----------------------------------------------------------------------
+__device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr) {
+  // start address >> 4 [0,14), LBO (unused for swizzled K-major) = 1 [16,30), SBO = 1024 B >> 4 [32,46),
+  // version 1 [46,48), base offset 0, layout SWIZZLE_128B = 2 [61,64)
+  return (uint64_t)((saddr >> 4) & 0x3FFFu) | (1ull << 16) | (64ull << 32) | (1ull << 46) | (2ull << 61);
+}
+// kind::i8 instruction descriptor: D s32, A/B signed int8, both K-major, N = kI8NT, M = kI8M
+constexpr uint32_t kI8Idesc = (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(kI8NT >> 3) << 17) |
+                              ((uint32_t)(kI8M >> 4) << 24);
+
+__device__ __forceinline__ void umma_i8(uint32_t tmem_d, uint64_t da, uint64_t db, uint32_t accumulate) {
+  asm volatile(
+      "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "l"(da), "l"(db), "r"(kI8Idesc), "r"(accumulate));
+}
+// A (W^T digits) from TMEM, B (digit tile) from shared memory
+__device__ __forceinline__ void umma_i8_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t accumulate) {
+  asm volatile(
+      "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(db), "r"(kI8Idesc), "r"(accumulate));
+}
+__device__ __forceinline__ void tmem_st8(uint32_t taddr, const uint32_t v[8]) {
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"r"(taddr), "r"(v[0]),
+               "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
+               : "memory");
+}
+__device__ __forceinline__ void umma_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_addr(bar))
+               : "memory");
+}
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, int32_t v[16]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+        "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+      : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, int32_t v[8]) {
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+               : "r"(taddr));
+}
+template <int W>
+__device__ __forceinline__ void tmem_ld(uint32_t taddr, int32_t* v);
+template <>
+__device__ __forceinline__ void tmem_ld<16>(uint32_t taddr, int32_t* v) { tmem_ld16(taddr, v); }
+template <>
+__device__ __forceinline__ void tmem_ld<8>(uint32_t taddr, int32_t* v) { tmem_ld8(taddr, v); }
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+
+// ---- GEMM-2 -----------------------------------------------------------------------------------------
+// grid (CTAs per domain, ndom); CTA b of a domain takes tiles b, b + gridDim.x, ...
+template <bool kOut>
+__global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
+  pdl_wait();
+  pdl_trigger();
+  extern __shared__ __align__(1024) unsigned char dsm_raw[];
+  // SWIZZLE_128B images need 1024-byte aligned shared addresses
+  unsigned char* dsm = dsm_raw + ((1024u - (smem_addr(dsm_raw) & 1023u)) & 1023u);
+  unsigned char* Tsm = dsm;                            // [stages][S][64 r][128 B] swizzled digit tiles
+  unsigned char* Psm = Tsm + kI8Stages * kI8TileB;     // [slots][16 r][norb] complex + sigma: Psi sub-tiles
+  unsigned char* Csm = Psm;                            // C'' of the domain (staged before the Psi ring starts)
+  __shared__ __align__(8) uint64_t full[kI8Stages], empty[kI8Stages], dfull[kI8Slots], dempty[kI8Slots];
+  __shared__ __align__(8) uint64_t pfull[kI8PsiSlots], pempty[kI8PsiSlots];
+  __shared__ __align__(8) uint64_t cbar, wready;
+  __shared__ uint32_t tmem_base_sh;
+  __shared__ double taus[kI8M];
+
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int dom = blockIdx.y;
+  const int norb = p.norb, nproj = p.nproj;
+  const long long ng = p.ng;
+  const long long tiles = (ng + kI8NT - 1) / kI8NT;
+
+  if (warp == 9) {  // TMEM: W^T digits (A operand, 6 x 32 columns) + the ring of diagonal accumulators
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_addr(&tmem_base_sh)));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  if (tid == 0) {
+    for (int s = 0; s < kI8Stages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
+    for (int s = 0; s < kI8Slots; ++s) { mbar_init(&dfull[s], 1); mbar_init(&dempty[s], 8); }
+    for (int s = 0; s < kI8PsiSlots; ++s) { mbar_init(&pfull[s], 1); mbar_init(&pempty[s], 4); }
+    mbar_init(&cbar, 1);
+    mbar_init(&wready, 4);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_base_sh;
+  const uint32_t tacc = tmem + kI8WCols;  // accumulator slot columns
+
+  if (warp < 4) {
+    // W^T digits from C'' (staged by one bulk copy) into TMEM: thread (warp q < 4, lane) owns row
+    // n = 32 q + lane of W^T (TMEM lane n); its 128 K bytes per digit are 32 consecutive 32-bit columns,
+    // k = 4 c + byte. tau_n = 2^f (max_k |W^T[n][k]| < 2^f).
+    if (tid == 0) {
+      mbar_expect_tx(&cbar, (uint32_t)(nproj * norb * 16));
+      tma_row(Csm, p.Cp + (long long)dom * nproj * norb, (uint32_t)(nproj * norb * 16), &cbar);
+    }
+    const int n = 32 * warp + lane, s = n >> 1, cn = n & 1;
+    const bool sv = s < norb;
+    mbar_wait(&cbar, 0);
+    const double2* X = reinterpret_cast<const double2*>(Csm) + s;  // X[u][s] at u * norb
+    double mx = 0.0;
+    if (sv)
+      for (int u = 0; u < nproj; ++u) {
+        const double2 x = X[u * norb];
+        mx = fmax(mx, fmax(fabs(x.x), fabs(x.y)));
+      }
+    const int e = mx > 0.0 ? row_exponent(mx) : 0;
+    taus[n] = mx > 0.0 ? ldexp(1.0, e - 12) : 0.0;  // x 2^-12: the weight of diagonal 2 (see the epilogue)
+    const uint32_t trow = tmem + ((uint32_t)(32 * warp) << 16);
+#pragma unroll 1
+    for (int c8 = 0; c8 < 4; ++c8) {  // 8 columns = 32 k values = 16 projectors per chunk
+      uint32_t dg[kI8S][8];
+#pragma unroll
+      for (int w = 0; w < 8; ++w) {
+        double v[4] = {0.0, 0.0, 0.0, 0.0};
+        const int u0 = 16 * c8 + 2 * w;  // k = 4 (8 c8 + w) .. + 3 -> projectors u0, u0 + 1
+        if (sv && u0 < nproj) {
+          const double2 x = X[u0 * norb];
+          v[0] = cn ? x.y : x.x; v[1] = cn ? x.x : -x.y;
+        }
+        if (sv && u0 + 1 < nproj) {
+          const double2 x = X[(u0 + 1) * norb];
+          v[2] = cn ? x.y : x.x; v[3] = cn ? x.x : -x.y;
+        }
+        uint32_t d[kI8S];
+        digits4(v, e, !(mx > 0.0), d);
+#pragma unroll
+        for (int i = 0; i < kI8S; ++i) dg[i][w] = d[i];
+      }
+#pragma unroll
+      for (int i = 0; i < kI8S; ++i) tmem_st8(trow + i * 32 + 8 * c8, dg[i]);
+    }
+    asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+    tc_fence_before();
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&wready);
+  }
+
+  const int rowb = norb * 16;  // bytes per Psi row
+  if (warp == 8) {  // producer of the digit tiles (one bulk copy each)
+    if (lane == 0) {
+      const int8_t* src = p.bsl + (long long)dom * tiles * kI8TileB;
+      int it = 0;
+      for (long long t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
+        const int s = it % kI8Stages;
+        if (it >= kI8Stages) mbar_wait(&empty[s], (uint32_t)(((it / kI8Stages) - 1) & 1));
+        mbar_expect_tx(&full[s], kI8TileB);
+        tma_row(Tsm + s * kI8TileB, src + t * kI8TileB, kI8TileB, &full[s]);
+      }
+    }
+  } else if (warp == 10) {  // producer of the Psi sub-tiles (16 contiguous rows + their 16 row scales)
+    if (lane == 0) {
+      const double2* prow = p.psi + (long long)dom * ng * norb;
+      const double* sig = p.bsig + (long long)dom * tiles * kI8NT;
+      mbar_wait(&wready, 0);  // the staged C'' has been consumed
+      int u = 0;
+      for (long long t = blockIdx.x; t < tiles; t += gridDim.x)
+        for (int k = 0; k < kI8NT / kI8SubR; ++k, ++u) {
+          const int s = u % kI8PsiSlots;
+          if (u >= kI8PsiSlots) mbar_wait(&pempty[s], (uint32_t)(((u / kI8PsiSlots) - 1) & 1));
+          const long long r0 = t * kI8NT + k * kI8SubR;
+          const long long nr = (ng - r0) < kI8SubR ? (ng - r0) : kI8SubR;
+          if (nr <= 0) {  // past the domain end: nothing to stage, the slot completes at once
+            mbar_arrive(&pfull[s]);
+            continue;
+          }
+          mbar_expect_tx(&pfull[s], (uint32_t)(nr * rowb + kI8SubR * 8));
+          tma_row(Psm + s * kI8SubB, prow + r0 * norb, (uint32_t)(nr * rowb), &pfull[s]);
+          tma_row(Psm + s * kI8SubB + kI8SubRowsB, sig + r0, kI8SubR * 8, &pfull[s]);
+        }
+    }
+  } else if (warp == 9) {  // MMA issuer: D_d += W_j^T (TMEM) x b_i (smem), i + j = d; one ring slot per d
+    if (lane == 0) {
+      const uint32_t tbase = smem_addr(Tsm);
+      mbar_wait(&wready, 0);
+      tc_fence_after();
+      int it = 0;
+      for (long long t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
+        const int s = it % kI8Stages;
+        mbar_wait(&full[s], (uint32_t)((it / kI8Stages) & 1));
+        tc_fence_after();
+        const uint32_t tb = tbase + s * kI8TileB;
+#pragma unroll
+        for (int d = 2; d <= kI8S + 1; ++d) {
+          const int g = it * kI8Acc + (d - 2), sl = g % kI8Slots;
+          if (g >= kI8Slots) {
+            mbar_wait(&dempty[sl], (uint32_t)(((g / kI8Slots) - 1) & 1));
+            tc_fence_after();
+          }
+          const uint32_t acc = tacc + sl * kI8NT;
+          uint32_t first = 1;
+#pragma unroll
+          for (int i = 1; i <= kI8S; ++i) {
+            const int j = d - i;
+            if (j < 1 || j > kI8S) continue;
+            if ((p.dbg & 1) && d > 2) continue;
+#pragma unroll
+            for (int kk = 0; kk < kI8K / 32; ++kk) {
+              umma_i8_ts(acc, tmem + (j - 1) * 32 + kk * 8, umma_desc_sw128(tb + (i - 1) * kI8SliceB + kk * 32),
+                         first ? 0u : 1u);
+              first = 0;
+            }
+          }
+          umma_commit(&dfull[sl]);  // diagonal d of tile t ready
+        }
+        umma_commit(&empty[s]);  // the digit tile may be overwritten once these MMAs are done
+      }
+    }
+  } else if (warp < 8) {
+    // epilogue: warp w reads TMEM lanes 32 (w & 3) .. + 31 (output double n of a Psi row) and tile rows
+    // 32 (w >> 2) .. + 31; it drains the diagonals as they complete into FP64 sums
+    // acc_c = sum_d P_d 2^{-7(d-2)}, then Psi <- n_s Psi + sigma_r tau_n 2^-12 acc.
+    const int q = warp & 3, h = warp >> 2;
+    const int n = 32 * q + lane;
+    const bool nvalid = n < 2 * norb;
+    const double nf = nvalid ? p.nfac[(long long)dom * norb + (n >> 1)] : 0.0;
+    mbar_wait(&wready, 0);
+    const double tau = taus[n];
+    double* pout = reinterpret_cast<double*>((kOut ? p.psi_out : p.psi) + (long long)dom * ng * norb) + n;
+    const int ld = 2 * norb;
+    int it = 0;
+    for (long long t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
+      const long long r0 = t * kI8NT + kI8Half * h;
+      const int nc = (int)((ng - r0) < kI8Half ? (ng - r0) : kI8Half);  // valid rows of this warp
+      double fa[kI8Half];
+#pragma unroll
+      for (int c = 0; c < kI8Half; ++c) fa[c] = 0.0;
+#pragma unroll 1
+      for (int d = 2; d <= kI8S + 1; ++d) {
+        const int g = it * kI8Acc + (d - 2), sl = g % kI8Slots;
+        mbar_wait(&dfull[sl], (uint32_t)((g / kI8Slots) & 1));
+        tc_fence_after();
+        int32_t a[kI8Half];
+        const uint32_t ta = tacc + sl * kI8NT + ((uint32_t)(32 * q) << 16) + kI8Half * h;
+        tmem_ld16(ta, a);
+        tmem_ld16(ta + 16, a + 16);
+        tmem_wait_ld();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&dempty[sl]);  // the slot may take the next diagonal
+        const double wd = ldexp(1.0, -7 * (d - 2));
+#pragma unroll
+        for (int c = 0; c < kI8Half; ++c) fa[c] = fma(i2d(a[c]), wd, fa[c]);
+      }
+      // the warp's two staged Psi sub-tiles (rows 32 h .. 32 h + 31 of the tile)
+#pragma unroll
+      for (int k = 0; k < 2; ++k) {
+        const int u = it * (kI8NT / kI8SubR) + 2 * h + k, s = u % kI8PsiSlots;
+        mbar_wait(&pfull[s], (uint32_t)((u / kI8PsiSlots) & 1));
+        const double* ps = reinterpret_cast<const double*>(Psm + s * kI8SubB) + n;
+        const double* sg = reinterpret_cast<const double*>(Psm + s * kI8SubB + kI8SubRowsB);
+#pragma unroll
+        for (int c = 0; c < kI8SubR; ++c) {
+          const int cc = k * kI8SubR + c;
+          if (!nvalid || cc >= nc || (p.dbg & 2)) continue;
+          pout[(r0 + cc) * ld] = fma(sg[c] * tau, fa[cc], nf * ps[c * ld]);
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&pempty[s]);
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 9) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
+  }
+}
+
+size_t gemm2_i8_bytes(int ndom, long long ng) {
+  const long long tiles = (ng + kI8NT - 1) / kI8NT;
+  return (size_t)ndom * tiles * kI8TileB;
+}
+size_t gemm2_i8_sig_bytes(int ndom, long long ng) {
+  const long long tiles = (ng + kI8NT - 1) / kI8NT;
+  return (size_t)ndom * tiles * kI8NT * sizeof(double);
+}
+bool gemm2_i8_supported(int nproj, int norb) { return nproj >= 1 && nproj <= 64 && norb >= 1 && norb <= 64; }
+
+cudaError_t launch_bslice_i8(const double2* B, int ndom, int nproj, long long ng, int8_t* out, double* sig,
+                             cudaStream_t st) {
+  const long long tiles = (ng + kI8NT - 1) / kI8NT;
+  dim3 grid((unsigned)((tiles * kI8NT + 7) / 8), ndom);
+  launch_k(k_bslice_i8, grid, 256, 0, st, B, nproj, ng, tiles, out, sig);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_gemm2_i8(const Gemm2Args& a, cudaStream_t st) {
+  const long long tiles = (a.ng + kI8NT - 1) / kI8NT;
+  int cpd = a.num_sms / a.ndom;
+  if (cpd < 1) cpd = 1;
+  if (cpd > tiles) cpd = (int)tiles;
+  dim3 grid(cpd, a.ndom);
+  if (a.psi_out) launch_k(k_gemm2_i8<true>, grid, kI8Threads, kI8Smem, st, a);
+  else launch_k(k_gemm2_i8<false>, grid, kI8Threads, kI8Smem, st, a);
+  return cudaGetLastError();
+}
+
+cudaError_t gemm_i8_set_attributes() {
+  cudaError_t e = cudaFuncSetAttribute(k_gemm2_i8<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kI8Smem);
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(k_gemm2_i8<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kI8Smem);
+}
+
+}  // namespace lfd

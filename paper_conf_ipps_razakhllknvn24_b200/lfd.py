@@ -21,6 +21,7 @@ LFD_ABI_VERSION = 4
 LFD_FLAG_NO_CARRY = 1
 LFD_FLAG_EXACT_NL = 2
 LFD_FLAG_SP = 4
+LFD_FLAG_NL_DMMA = 8
 LFD_BC_PERIODIC = 0
 LFD_BC_ZERO = 1
 STATUS = {0: "LFD_OK", -1: "LFD_EINVAL", -2: "LFD_ENOMEM", -3: "LFD_ECUDA", -4: "LFD_ESTATE",
@@ -33,7 +34,7 @@ LFD_SC_MAXWELL = 4
 EXPORTS = ("lfd_workspace_size", "lfd_init", "lfd_set_potential", "lfd_set_potential_host",
            "lfd_set_vector_potential", "lfd_step", "lfd_step_sequence", "lfd_density_current", "lfd_density_current_global",
            "lfd_density_current_host", "lfd_energy", "lfd_remap_occ", "lfd_psi_modified", "lfd_set_occupations", "lfd_set_stream", "lfd_sync",
-           "lfd_launch_count", "lfd_profile_enable", "lfd_profile_read", "lfd_last_error", "lfd_destroy",
+           "lfd_launch_count", "lfd_nl_path", "lfd_profile_enable", "lfd_profile_read", "lfd_last_error", "lfd_destroy",
            "lfd_sc_workspace_size", "lfd_sc_init", "lfd_sc_step", "lfd_sc_read", "lfd_comm_unique_id",
            "lfd_sc_comm_init", "lfd_step_graph")
 
@@ -87,6 +88,7 @@ def load():
         "lfd_set_stream": [P, P],
         "lfd_sync": [P],
         "lfd_launch_count": [P, C.POINTER(C.c_uint64)],
+        "lfd_nl_path": [P, C.POINTER(C.c_int32)],
         "lfd_profile_enable": [P, I32],
         "lfd_profile_read": [P, D, C.POINTER(C.c_int64)],
         "lfd_destroy": [P],
@@ -243,6 +245,13 @@ def lfd_sync(ctx):
 def lfd_launch_count(ctx) -> int:
     n = C.c_uint64(0)
     _check(load().lfd_launch_count(ctx, C.byref(n)), ctx)
+    return n.value
+
+
+def lfd_nl_path(ctx) -> int:
+    """0 FP64 DMMA, 1 int8-digit tcgen05 (FP64 accuracy), 2 SP 3xTF32, -1 no nonlocal factor."""
+    n = C.c_int32(0)
+    _check(load().lfd_nl_path(ctx, C.byref(n)), ctx)
     return n.value
 
 
