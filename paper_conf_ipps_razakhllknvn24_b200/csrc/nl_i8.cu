@@ -194,7 +194,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
   unsigned char* Csm = Psm;                            // C'' of the domain (staged before the Psi ring starts)
   __shared__ __align__(8) uint64_t full[kI8Stages], empty[kI8Stages], dfull[kI8Slots], dempty[kI8Slots];
   __shared__ __align__(8) uint64_t pfull[kI8PsiSlots], pempty[kI8PsiSlots];
-  __shared__ __align__(8) uint64_t cbar, wready;
+  __shared__ __align__(8) uint64_t cbar;
   __shared__ uint32_t tmem_base_sh;
   __shared__ double taus[kI8M];
 
@@ -213,7 +213,6 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
     for (int s = 0; s < kI8Slots; ++s) { mbar_init(&dfull[s], 1); mbar_init(&dempty[s], 8); }
     for (int s = 0; s < kI8PsiSlots; ++s) { mbar_init(&pfull[s], 1); mbar_init(&pempty[s], 4); }
     mbar_init(&cbar, 1);
-    mbar_init(&wready, 4);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   tc_fence_before();
@@ -267,9 +266,13 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
       for (int i = 0; i < kI8S; ++i) tmem_st8(trow + i * 32 + 8 * c8, dg[i]);
     }
     asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+  }
+  // W ready (TMEM digits, taus[]) and the staged C'' consumed: named barrier 1 over every warp except the
+  // digit producer (warp 8), which streams from the start
+  if (warp != 8) {
     tc_fence_before();
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&wready);
+    asm volatile("bar.sync 1, %0;" ::"n"(kI8Threads - 32) : "memory");
+    tc_fence_after();
   }
 
   const int rowb = norb * 16;  // bytes per Psi row
@@ -288,7 +291,6 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
     if (lane == 0) {
       const double2* prow = p.psi + (long long)dom * ng * norb;
       const double* sig = p.bsig + (long long)dom * tiles * kI8NT;
-      mbar_wait(&wready, 0);  // the staged C'' has been consumed
       int u = 0;
       for (long long t = blockIdx.x; t < tiles; t += gridDim.x)
         for (int k = 0; k < kI8NT / kI8SubR; ++k, ++u) {
@@ -308,8 +310,6 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
   } else if (warp == 9) {  // MMA issuer: D_d += W_j^T (TMEM) x b_i (smem), i + j = d; one ring slot per d
     if (lane == 0) {
       const uint32_t tbase = smem_addr(Tsm);
-      mbar_wait(&wready, 0);
-      tc_fence_after();
       int it = 0;
       for (long long t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
         const int s = it % kI8Stages;
@@ -350,7 +350,6 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
     const int n = 32 * q + lane;
     const bool nvalid = n < 2 * norb;
     const double nf = nvalid ? p.nfac[(long long)dom * norb + (n >> 1)] : 0.0;
-    mbar_wait(&wready, 0);
     const double tau = taus[n];
     double* pout = reinterpret_cast<double*>((kOut ? p.psi_out : p.psi) + (long long)dom * ng * norb) + n;
     const int ld = 2 * norb;
