@@ -423,6 +423,25 @@ lfd_status gemm2(lfd_ctx* c, double2* out = nullptr) {
     a2.bsl = c->at<int8_t>(c->L.bsl);
     a2.bsig = c->at<double>(c->L.bsig);
     if (const char* v = std::getenv("LFD_I8_DBG")) a2.dbg = std::atoi(v);
+    if (std::getenv("LFD_I8_TIMING")) {  // diagnostics: role wait cycles, printed per call (one domain)
+      static long long* buf = nullptr;
+      if (!buf) cudaMallocManaged(&buf, 8 * 1024 * sizeof(long long));
+      cudaStreamSynchronize(c->stream);
+      for (int i = 0; i < 8 * 1024; ++i) buf[i] = 0;
+      a2.dbgbuf = buf;
+      lfd_status st = LFD_OK;
+      LFD_TRY(launch(c, LFD_K_NL_BACK, "k_gemm2", [&] { return lfd::launch_gemm2(a2, c->stream); }));
+      cudaStreamSynchronize(c->stream);
+      double s[7] = {0, 0, 0, 0, 0, 0, 0};
+      for (int b = 0; b < c->num_sms; ++b)
+        for (int k = 0; k < 7; ++k) s[k] += (double)buf[b * 8 + k];
+      std::fprintf(stderr, "i8 timing (avg cycles per CTA): prologue %.0f  mma loop %.0f  kernel %.0f  mma-wait-digits %.0f  "
+                   "mma-wait-slot %.0f  epi-wait-diag %.0f (per warp)  epi-wait-psi %.0f (per warp)\n",
+                   s[5] / c->num_sms, s[2] / c->num_sms, s[6] / c->num_sms, s[0] / c->num_sms, s[1] / c->num_sms,
+                   s[3] / c->num_sms / 16, s[4] / c->num_sms / 16);
+      c->c_valid = c->carry;
+      return st;
+    }
   }
   c->c_valid = false;
   if (g.sp)

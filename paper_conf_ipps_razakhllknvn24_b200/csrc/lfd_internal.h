@@ -164,6 +164,7 @@ struct Gemm2Args {
   const int8_t* bsl = nullptr;
   const double* bsig = nullptr;
   int dbg = 0;  // diagnostics only (env LFD_I8_DBG): 1 = one digit pair per tile, 2 = no epilogue math
+  long long* dbgbuf = nullptr;  // diagnostics only (env LFD_I8_TIMING): per-CTA wait cycles of each role
 };
 cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st);
 // GEMM-2 with FP64 accuracy on the tcgen05 int8 tensor cores (nl_i8.cu): nproj <= 64, norb <= 64.

@@ -46,18 +46,20 @@ constexpr int kI8NT = 64;                           // grid points per tile (MMA
 constexpr int kI8K = 128;                           // bytes per digit row: K = 2 nproj padded to 128
 constexpr int kI8M = 128;                           // MMA M: 2 norb padded to 128
 constexpr int kI8Stages = 2;                        // digit-tile ring
-constexpr int kI8Slots = 4;                         // TMEM ring of diagonal accumulators (kI8NT columns each)
-constexpr int kI8Half = kI8NT / 2;                  // tile rows per epilogue warp
+constexpr int kI8Slots = 5;                         // TMEM ring of diagonal accumulators (kI8NT columns each)
+constexpr int kI8EpiWarps = 16;                     // epilogue warps: 4 lane quarters x 4 row quarters
+constexpr int kI8Rows = kI8NT / 4;                  // tile rows per epilogue warp
 constexpr int kI8SliceB = kI8NT * kI8K;             // 8 KB: one digit slice of a tile
 constexpr int kI8TileB = kI8S * kI8SliceB;          // 48 KB: all digits of a tile
-constexpr int kI8SubR = 16;                         // Psi rows per staged sub-tile
+constexpr int kI8SubR = 16;                         // Psi rows per staged sub-tile (= rows per epilogue warp)
 constexpr int kI8SubRowsB = kI8SubR * 64 * 16;      // 16 KB (norb <= 64)
 constexpr int kI8SubB = kI8SubRowsB + kI8SubR * 8;  // + the sub-tile's row scales sigma_r
-constexpr int kI8PsiSlots = 7;                      // Psi sub-tile ring (first 64 KB also stage C'')
+constexpr int kI8PsiSlots = 7;                      // Psi sub-tile ring (the first 64 KB also stage C'')
 constexpr int kI8Smem = kI8Stages * kI8TileB + kI8PsiSlots * kI8SubB + 1024;  // + alignment slack
 constexpr int kI8WCols = kI8S * (kI8K / 4);        // 192 TMEM columns: W^T digits (4 int8 per column)
 constexpr int kI8Acc = kI8S;                        // diagonals d = 2 .. S+1
-constexpr int kI8Threads = 352;                     // 8 epilogue warps + 2 producers + MMA
+constexpr int kI8Threads = (kI8EpiWarps + 3) * 32;  // epilogue warps + 2 producers + MMA
+constexpr int kWDig = kI8EpiWarps, kWMma = kI8EpiWarps + 1, kWPsi = kI8EpiWarps + 2;  // role warps
 
 // byte offset of (row, k) in a K-major SWIZZLE_128B image with 128-byte rows (8-row, 1024-byte atoms;
 // the 16-byte chunk index is XOR-ed with the row within the atom)
@@ -87,6 +89,18 @@ __device__ __forceinline__ void digits4(const double v[4], int e, bool zero, uin
 // 2^52 + 2^31 (one full-rate DADD)
 __device__ __forceinline__ double i2d(int32_t x) {
   return __hiloint2double(0x43300000, (int)((uint32_t)x ^ 0x80000000u)) - 4503601774854144.0;
+}
+
+// exact int64 -> FP64 for |x| < 2^51: (1.5 2^52 + x) built from bits, minus 1.5 2^52 (one DADD)
+__device__ __forceinline__ double l2d(long long x) {
+  return __longlong_as_double(x + 0x4338000000000000LL) - 6755399441055744.0;
+}
+
+// product of two powers of two (or zeros) by exponent arithmetic on the bits: no FP64 multiply
+__device__ __forceinline__ double pow2mul(double a, double b) {
+  const int ea = (__double2hiint(a) >> 20) & 0x7ff, eb = (__double2hiint(b) >> 20) & 0x7ff;
+  const int e = ea + eb - 1023;
+  return (ea == 0 || eb == 0 || e <= 0) ? 0.0 : __hiloint2double(e << 20, 0);
 }
 
 __device__ __forceinline__ int row_exponent(double mx) {
@@ -203,14 +217,15 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
   const int norb = p.norb, nproj = p.nproj;
   const long long ng = p.ng;
   const long long tiles = (ng + kI8NT - 1) / kI8NT;
+  const long long t_entry = clock64();
 
-  if (warp == 9) {  // TMEM: W^T digits (A operand, 6 x 32 columns) + the ring of diagonal accumulators
+  if (warp == kWMma) {  // TMEM: W^T digits (A operand, 6 x 32 columns) + the ring of diagonal accumulators
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_addr(&tmem_base_sh)));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   if (tid == 0) {
     for (int s = 0; s < kI8Stages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
-    for (int s = 0; s < kI8Slots; ++s) { mbar_init(&dfull[s], 1); mbar_init(&dempty[s], 8); }
+    for (int s = 0; s < kI8Slots; ++s) { mbar_init(&dfull[s], 1); mbar_init(&dempty[s], kI8EpiWarps); }
     for (int s = 0; s < kI8PsiSlots; ++s) { mbar_init(&pfull[s], 1); mbar_init(&pempty[s], 4); }
     mbar_init(&cbar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -221,15 +236,16 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
   const uint32_t tmem = tmem_base_sh;
   const uint32_t tacc = tmem + kI8WCols;  // accumulator slot columns
 
-  if (warp < 4) {
-    // W^T digits from C'' (staged by one bulk copy) into TMEM: thread (warp q < 4, lane) owns row
-    // n = 32 q + lane of W^T (TMEM lane n); its 128 K bytes per digit are 32 consecutive 32-bit columns,
-    // k = 4 c + byte. tau_n = 2^f (max_k |W^T[n][k]| < 2^f).
+  if (warp < kI8EpiWarps) {
+    // W^T digits from C'' (staged by one bulk copy) into TMEM: thread (warp w, lane) owns row
+    // n = 32 (w & 3) + lane of W^T (TMEM lane n) and the 8 columns (32 K bytes, projectors 16 c8 ..
+    // 16 c8 + 15) of chunk c8 = w >> 2 of each digit; k = 4 c + byte. tau_n = 2^f, max_k |W^T[n][k]| < 2^f.
     if (tid == 0) {
       mbar_expect_tx(&cbar, (uint32_t)(nproj * norb * 16));
       tma_row(Csm, p.Cp + (long long)dom * nproj * norb, (uint32_t)(nproj * norb * 16), &cbar);
     }
-    const int n = 32 * warp + lane, s = n >> 1, cn = n & 1;
+    const int q = warp & 3, c8 = warp >> 2;
+    const int n = 32 * q + lane, s = n >> 1, cn = n & 1;
     const bool sv = s < norb;
     mbar_wait(&cbar, 0);
     const double2* X = reinterpret_cast<const double2*>(Csm) + s;  // X[u][s] at u * norb
@@ -240,43 +256,40 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
         mx = fmax(mx, fmax(fabs(x.x), fabs(x.y)));
       }
     const int e = mx > 0.0 ? row_exponent(mx) : 0;
-    taus[n] = mx > 0.0 ? ldexp(1.0, e - 12) : 0.0;  // x 2^-12: the weight of diagonal 2 (see the epilogue)
-    const uint32_t trow = tmem + ((uint32_t)(32 * warp) << 16);
-#pragma unroll 1
-    for (int c8 = 0; c8 < 4; ++c8) {  // 8 columns = 32 k values = 16 projectors per chunk
-      uint32_t dg[kI8S][8];
+    if (c8 == 0) taus[n] = mx > 0.0 ? ldexp(1.0, e - 12) : 0.0;  // x 2^-12: the weight of diagonal 2
+    const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
+    uint32_t dg[kI8S][8];
 #pragma unroll
-      for (int w = 0; w < 8; ++w) {
-        double v[4] = {0.0, 0.0, 0.0, 0.0};
-        const int u0 = 16 * c8 + 2 * w;  // k = 4 (8 c8 + w) .. + 3 -> projectors u0, u0 + 1
-        if (sv && u0 < nproj) {
-          const double2 x = X[u0 * norb];
-          v[0] = cn ? x.y : x.x; v[1] = cn ? x.x : -x.y;
-        }
-        if (sv && u0 + 1 < nproj) {
-          const double2 x = X[(u0 + 1) * norb];
-          v[2] = cn ? x.y : x.x; v[3] = cn ? x.x : -x.y;
-        }
-        uint32_t d[kI8S];
-        digits4(v, e, !(mx > 0.0), d);
-#pragma unroll
-        for (int i = 0; i < kI8S; ++i) dg[i][w] = d[i];
+    for (int w = 0; w < 8; ++w) {
+      double v[4] = {0.0, 0.0, 0.0, 0.0};
+      const int u0 = 16 * c8 + 2 * w;  // k = 4 (8 c8 + w) .. + 3 -> projectors u0, u0 + 1
+      if (sv && u0 < nproj) {
+        const double2 x = X[u0 * norb];
+        v[0] = cn ? x.y : x.x; v[1] = cn ? x.x : -x.y;
       }
+      if (sv && u0 + 1 < nproj) {
+        const double2 x = X[(u0 + 1) * norb];
+        v[2] = cn ? x.y : x.x; v[3] = cn ? x.x : -x.y;
+      }
+      uint32_t d[kI8S];
+      digits4(v, e, !(mx > 0.0), d);
 #pragma unroll
-      for (int i = 0; i < kI8S; ++i) tmem_st8(trow + i * 32 + 8 * c8, dg[i]);
+      for (int i = 0; i < kI8S; ++i) dg[i][w] = d[i];
     }
+#pragma unroll
+    for (int i = 0; i < kI8S; ++i) tmem_st8(trow + i * 32 + 8 * c8, dg[i]);
     asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
   }
   // W ready (TMEM digits, taus[]) and the staged C'' consumed: named barrier 1 over every warp except the
   // digit producer (warp 8), which streams from the start
-  if (warp != 8) {
+  if (warp != kWDig) {
     tc_fence_before();
     asm volatile("bar.sync 1, %0;" ::"n"(kI8Threads - 32) : "memory");
     tc_fence_after();
   }
 
   const int rowb = norb * 16;  // bytes per Psi row
-  if (warp == 8) {  // producer of the digit tiles (one bulk copy each)
+  if (warp == kWDig) {  // producer of the digit tiles (one bulk copy each)
     if (lane == 0) {
       const int8_t* src = p.bsl + (long long)dom * tiles * kI8TileB;
       int it = 0;
@@ -287,7 +300,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
         tma_row(Tsm + s * kI8TileB, src + t * kI8TileB, kI8TileB, &full[s]);
       }
     }
-  } else if (warp == 10) {  // producer of the Psi sub-tiles (16 contiguous rows + their 16 row scales)
+  } else if (warp == kWPsi) {  // producer of the Psi sub-tiles (16 contiguous rows + their 16 row scales)
     if (lane == 0) {
       const double2* prow = p.psi + (long long)dom * ng * norb;
       const double* sig = p.bsig + (long long)dom * tiles * kI8NT;
@@ -307,20 +320,26 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
           tma_row(Psm + s * kI8SubB + kI8SubRowsB, sig + r0, kI8SubR * 8, &pfull[s]);
         }
     }
-  } else if (warp == 9) {  // MMA issuer: D_d += W_j^T (TMEM) x b_i (smem), i + j = d; one ring slot per d
+  } else if (warp == kWMma) {  // MMA issuer: D_d += W_j^T (TMEM) x b_i (smem), i + j = d; one ring slot per d
     if (lane == 0) {
       const uint32_t tbase = smem_addr(Tsm);
+      long long w_full = 0, w_slot = 0;
+      const long long t_start = clock64();
       int it = 0;
       for (long long t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
         const int s = it % kI8Stages;
+        long long c0 = clock64();
         mbar_wait(&full[s], (uint32_t)((it / kI8Stages) & 1));
+        w_full += clock64() - c0;
         tc_fence_after();
-        const uint32_t tb = tbase + s * kI8TileB;
+        const uint64_t db0 = umma_desc_sw128(tbase + s * kI8TileB);
 #pragma unroll
         for (int d = 2; d <= kI8S + 1; ++d) {
           const int g = it * kI8Acc + (d - 2), sl = g % kI8Slots;
           if (g >= kI8Slots) {
+            long long c1 = clock64();
             mbar_wait(&dempty[sl], (uint32_t)(((g / kI8Slots) - 1) & 1));
+            w_slot += clock64() - c1;
             tc_fence_after();
           }
           const uint32_t acc = tacc + sl * kI8NT;
@@ -332,7 +351,9 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
             if ((p.dbg & 1) && d > 2) continue;
 #pragma unroll
             for (int kk = 0; kk < kI8K / 32; ++kk) {
-              umma_i8_ts(acc, tmem + (j - 1) * 32 + kk * 8, umma_desc_sw128(tb + (i - 1) * kI8SliceB + kk * 32),
+              // descriptor arithmetic is linear in the (>> 4) start address: one add per MMA (the issuing
+              // warp shares its scheduler with four epilogue warps, so its instruction count matters)
+              umma_i8_ts(acc, tmem + (j - 1) * 32 + kk * 8, db0 + (uint64_t)(((i - 1) * kI8SliceB + kk * 32) >> 4),
                          first ? 0u : 1u);
               first = 0;
             }
@@ -341,63 +362,81 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
         }
         umma_commit(&empty[s]);  // the digit tile may be overwritten once these MMAs are done
       }
+      if (p.dbgbuf) {
+        p.dbgbuf[blockIdx.x * 8 + 0] = w_full;
+        p.dbgbuf[blockIdx.x * 8 + 1] = w_slot;
+        p.dbgbuf[blockIdx.x * 8 + 2] = clock64() - t_start;
+        p.dbgbuf[blockIdx.x * 8 + 5] = t_start - t_entry;
+      }
     }
-  } else if (warp < 8) {
+  } else if (warp < kI8EpiWarps) {
     // epilogue: warp w reads TMEM lanes 32 (w & 3) .. + 31 (output double n of a Psi row) and tile rows
-    // 32 (w >> 2) .. + 31; it drains the diagonals as they complete into FP64 sums
-    // acc_c = sum_d P_d 2^{-7(d-2)}, then Psi <- n_s Psi + sigma_r tau_n 2^-12 acc.
+    // 16 (w >> 2) .. + 15; it drains the diagonals two at a time as they complete, (P_d 2^7 + P_{d+1}) an
+    // exact int32, into FP64 sums acc_c = sum_d P_d 2^{-7(d-2)}; then Psi <- n_s Psi + sigma_r tau_n 2^-12 acc.
     const int q = warp & 3, h = warp >> 2;
     const int n = 32 * q + lane;
     const bool nvalid = n < 2 * norb;
     const double nf = nvalid ? p.nfac[(long long)dom * norb + (n >> 1)] : 0.0;
     const double tau = taus[n];
+    long long w_dfull = 0, w_pfull = 0;
     double* pout = reinterpret_cast<double*>((kOut ? p.psi_out : p.psi) + (long long)dom * ng * norb) + n;
     const int ld = 2 * norb;
     int it = 0;
     for (long long t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
-      const long long r0 = t * kI8NT + kI8Half * h;
-      const int nc = (int)((ng - r0) < kI8Half ? (ng - r0) : kI8Half);  // valid rows of this warp
-      double fa[kI8Half];
+      const long long r0 = t * kI8NT + kI8Rows * h;
+      const int nc = (int)((ng - r0) < kI8Rows ? (ng - r0) : kI8Rows);  // valid rows of this warp
+      double fa[kI8Rows];
 #pragma unroll
-      for (int c = 0; c < kI8Half; ++c) fa[c] = 0.0;
+      for (int c = 0; c < kI8Rows; ++c) fa[c] = 0.0;
 #pragma unroll 1
-      for (int d = 2; d <= kI8S + 1; ++d) {
-        const int g = it * kI8Acc + (d - 2), sl = g % kI8Slots;
-        mbar_wait(&dfull[sl], (uint32_t)((g / kI8Slots) & 1));
+      for (int dp = 0; dp < kI8Acc / 2; ++dp) {  // diagonals d = 2 + 2 dp and d + 1
+        const int g = it * kI8Acc + 2 * dp, s0 = g % kI8Slots, s1 = (g + 1) % kI8Slots;
+        long long c2 = clock64();
+        mbar_wait(&dfull[s0], (uint32_t)((g / kI8Slots) & 1));
+        mbar_wait(&dfull[s1], (uint32_t)(((g + 1) / kI8Slots) & 1));
+        w_dfull += clock64() - c2;
         tc_fence_after();
-        int32_t a[kI8Half];
-        const uint32_t ta = tacc + sl * kI8NT + ((uint32_t)(32 * q) << 16) + kI8Half * h;
-        tmem_ld16(ta, a);
-        tmem_ld16(ta + 16, a + 16);
+        int32_t a0[kI8Rows], a1[kI8Rows];
+        const uint32_t lb = ((uint32_t)(32 * q) << 16) + kI8Rows * h;
+        tmem_ld16(tacc + s0 * kI8NT + lb, a0);
+        tmem_ld16(tacc + s1 * kI8NT + lb, a1);
         tmem_wait_ld();
         tc_fence_before();
         __syncwarp();
-        if (lane == 0) mbar_arrive(&dempty[sl]);  // the slot may take the next diagonal
-        const double wd = ldexp(1.0, -7 * (d - 2));
+        if (lane == 0) {  // the slots may take the next diagonals
+          mbar_arrive(&dempty[s0]);
+          mbar_arrive(&dempty[s1]);
+        }
+        const double wd = ldexp(1.0, -14 * dp - 7);
 #pragma unroll
-        for (int c = 0; c < kI8Half; ++c) fa[c] = fma(i2d(a[c]), wd, fa[c]);
+        for (int c = 0; c < kI8Rows; ++c) fa[c] = fma(i2d(a0[c] * 128 + a1[c]), wd, fa[c]);
       }
-      // the warp's two staged Psi sub-tiles (rows 32 h .. 32 h + 31 of the tile)
-#pragma unroll
-      for (int k = 0; k < 2; ++k) {
-        const int u = it * (kI8NT / kI8SubR) + 2 * h + k, s = u % kI8PsiSlots;
+      // the warp's staged Psi sub-tile (rows 16 h .. 16 h + 15 of the tile)
+      {
+        const int u = it * (kI8NT / kI8SubR) + h, s = u % kI8PsiSlots;
+        long long c3 = clock64();
         mbar_wait(&pfull[s], (uint32_t)((u / kI8PsiSlots) & 1));
+        w_pfull += clock64() - c3;
         const double* ps = reinterpret_cast<const double*>(Psm + s * kI8SubB) + n;
         const double* sg = reinterpret_cast<const double*>(Psm + s * kI8SubB + kI8SubRowsB);
 #pragma unroll
-        for (int c = 0; c < kI8SubR; ++c) {
-          const int cc = k * kI8SubR + c;
-          if (!nvalid || cc >= nc || (p.dbg & 2)) continue;
-          pout[(r0 + cc) * ld] = fma(sg[c] * tau, fa[cc], nf * ps[c * ld]);
+        for (int c = 0; c < kI8Rows; ++c) {
+          if (!nvalid || c >= nc || (p.dbg & 2)) continue;
+          pout[(r0 + c) * ld] = fma(nf, ps[c * ld], pow2mul(sg[c], tau) * fa[c]);
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&pempty[s]);
       }
     }
+    if (p.dbgbuf && lane == 0) {
+      atomicAdd((unsigned long long*)&p.dbgbuf[blockIdx.x * 8 + 3], (unsigned long long)w_dfull);
+      atomicAdd((unsigned long long*)&p.dbgbuf[blockIdx.x * 8 + 4], (unsigned long long)w_pfull);
+    }
   }
   tc_fence_before();
   __syncthreads();
-  if (warp == 9) {
+  if (p.dbgbuf && tid == 0) p.dbgbuf[blockIdx.x * 8 + 6] = clock64() - t_entry;
+  if (warp == kWMma) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
   }
