@@ -32,9 +32,11 @@ size_t up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 struct Layout {
   size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage, cref,
-      epart, W, ones, x32, aseq, jseq, bsl, bsig;
+      epart, W, ones, x32, aseq, jseq, bsl, bsig, bsl1, bexp, colE, g1cnt;
   int nref_cap;
   bool i8;  // GEMM-2 on the int8 tensor cores (nl_i8.cu): B digit tiles + row scales in the workspace
+  int nsplit_i8;           // GEMM-1 on the int8 tensor cores: splits of rows_per_split_i8 rows
+  long long rows_per_split_i8;
   size_t total;
   int nsplit;
   long long rows_per_split;
@@ -140,8 +142,13 @@ Layout layout(const Geometry& g, int num_sms, int nref_max) {
   L.G = take((size_t)nd * np * np * c16);
   L.D = take((size_t)nd * np * d8);
   L.occ = take((size_t)nd * no * d8);
-  L.part = take((size_t)nd * nsplit * mn * c16);
-  L.normp = take((size_t)nd * nsplit * no * d8);
+  if (L.i8) {
+    L.rows_per_split_i8 = lfd::gemm1_i8_rows_per_split(g.ng, nd, num_sms);
+    L.nsplit_i8 = (int)((g.ng + L.rows_per_split_i8 - 1) / L.rows_per_split_i8);
+  }
+  const int nsplit_cap = std::max(nsplit, L.i8 ? L.nsplit_i8 : 0);
+  L.part = take((size_t)nd * nsplit_cap * mn * c16);
+  L.normp = take((size_t)nd * nsplit_cap * no * d8);
   L.dc = take((size_t)nd * np * no * c16);
   L.cprime = take((size_t)nd * np * no * c16);
   L.s = take((size_t)nd * no * d8);
@@ -160,6 +167,10 @@ Layout layout(const Geometry& g, int num_sms, int nref_max) {
   L.jseq = take((size_t)kGraphChunk * nd * 3 * d8);   // lfd_step_graph: J of the chunk's steps
   L.bsl = L.i8 ? take(lfd::gemm2_i8_bytes(nd, g.ng)) : 0;
   L.bsig = L.i8 ? take(lfd::gemm2_i8_sig_bytes(nd, g.ng)) : 0;
+  L.bsl1 = L.i8 ? take(lfd::gemm1_i8_bytes(nd, g.ng)) : 0;
+  L.bexp = L.i8 ? take((size_t)nd * np * sizeof(int)) : 0;
+  L.colE = L.i8 ? take((size_t)nd * no * sizeof(int)) : 0;
+  L.g1cnt = L.i8 ? take((size_t)nd * sizeof(int)) : 0;
   L.total = o;
   return L;
 }
@@ -263,6 +274,9 @@ struct lfd_ctx {
   // instead of GEMM-1 (cleared by the local propagator, lfd_psi_modified and LFD_FLAG_NO_CARRY).
   bool c_valid = false;
   bool carry = true;
+  // int8-digit GEMM-1: the orbital exponents in the workspace describe the current Psi (set by the K_y K_z
+  // pass that wrote it, consumed -- and cleared on the device -- by GEMM-1)
+  bool colE_valid = false;
   bool exact = false;     // LFD_FLAG_EXACT_NL: exactly unitary nonlocal factor (orthonormal B)
   bool kin_fused = true;  // Phi.K_y K_z in one pass (env LFD_KIN_FUSED=0: separate y and z passes)
   CUtensorMap psi_tmap;   // TMA descriptor of Psi for the fused pass
@@ -495,14 +509,27 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
   a1.ndom = g.ndom; a1.mrows = g.nproj; a1.ncols = g.norb; a1.nsplit = c->L.nsplit;
   a1.ng = g.ng; a1.rows_per_split = c->L.rows_per_split;
   a1.a_dom_stride = g.ng * g.nproj; a1.x_dom_stride = g.ng * g.norb;
-  LFD_TRY(launch(c, LFD_K_NL_PROJ, "k_gemm1", [&] { return gemm1_any(c, a1); }));
+  int nsplit = c->L.nsplit;
+  if (c->L.i8 && c->colE_valid) {  // int8-digit tensor-core GEMM-1 (Psi's orbital exponents from the K_y K_z pass)
+    lfd::Gemm1I8Args ai;
+    ai.psi = c->psi; ai.bsl1 = c->at<int8_t>(c->L.bsl1); ai.bexp = c->at<int>(c->L.bexp);
+    ai.colE = c->at<int>(c->L.colE); ai.counter = c->at<int>(c->L.g1cnt);
+    ai.part = a1.part; ai.norms = a1.norms;
+    ai.ndom = g.ndom; ai.nproj = g.nproj; ai.norb = g.norb; ai.nsplit = c->L.nsplit_i8;
+    ai.ng = g.ng; ai.rps = c->L.rows_per_split_i8;
+    LFD_TRY(launch(c, LFD_K_NL_PROJ, "k_gemm1_i8", [&] { return lfd::launch_gemm1_i8(ai, c->stream); }));
+    c->colE_valid = false;
+    nsplit = c->L.nsplit_i8;
+  } else {
+    LFD_TRY(launch(c, LFD_K_NL_PROJ, "k_gemm1", [&] { return gemm1_any(c, a1); }));
+  }
   lfd::ReduceArgs r;
   r.part = a1.part; r.normp = a1.norms;
   r.D = c->at<double>(c->L.D);
   r.out = c->at<double2>(c->L.dc);
   r.cprime = c->at<double2>(c->L.cprime);
   r.s = c->at<double>(c->L.s);
-  r.ndom = g.ndom; r.mrows = g.nproj; r.ncols = g.norb; r.nsplit = c->L.nsplit;
+  r.ndom = g.ndom; r.mrows = g.nproj; r.ncols = g.norb; r.nsplit = nsplit;
   r.scale = g.dV; r.eps = 0.5 * g.dt;
   if (c->exact) {  // C (undecorated) and C'' = W C; n == 1 (set at init)
     r.D = nullptr;
@@ -542,9 +569,14 @@ lfd_status local_prop(lfd_ctx* c, const double2* src = nullptr) {
   }
   LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin(x)",
                  [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 0, 1, c->scaled, c->stream, src); }));
-  if (c->kin_fused)
-    return launch(c, LFD_K_KIN_YZ, "k_kin_yz",
-                  [&] { return lfd::launch_kin_yz(c->g, &c->psi_tmap, c->psi, c->coef(), c->phi(), c->scaled, c->stream); });
+  if (c->kin_fused) {
+    int* colE = c->L.i8 ? c->at<int>(c->L.colE) : nullptr;
+    LFD_TRY(launch(c, LFD_K_KIN_YZ, "k_kin_yz", [&] {
+      return lfd::launch_kin_yz(c->g, &c->psi_tmap, c->psi, c->coef(), c->phi(), c->scaled, c->stream, colE);
+    }));
+    c->colE_valid = colE != nullptr;
+    return LFD_OK;
+  }
   LFD_TRY(launch(c, LFD_K_KIN_Y, "k_kin(y)",
                  [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 1, 0, c->scaled, c->stream); }));
   return launch(c, LFD_K_KIN_Z, "k_kin(z)",
@@ -927,12 +959,20 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
     s2 = launch(c, LFD_K_NL_REDUCE, "k_reduce(G)", [&] { return lfd::launch_reduce(r, c->stream); });
     if (s2 != LFD_OK) return bail(s2);
   }
-  if (L.i8) {  // int8 digit tiles of B for the tensor-core GEMM-2 (B is constant, like G)
+  if (L.i8) {  // int8 digit tiles of B for the tensor-core GEMM-2 and GEMM-1 (B is constant, like G)
     s2 = launch(c, LFD_K_NL_BACK, "k_bslice_i8", [&] {
       return lfd::launch_bslice_i8(c->proj, g.ndom, g.nproj, g.ng, c->at<int8_t>(L.bsl), c->at<double>(L.bsig),
                                    c->stream);
     });
     if (s2 != LFD_OK) return bail(s2);
+    s2 = launch(c, LFD_K_NL_PROJ, "k_bslice1_i8", [&] {
+      return lfd::launch_bslice1_i8(c->proj, g.ndom, g.nproj, g.ng, c->at<int>(L.bexp), c->at<int8_t>(L.bsl1),
+                                    c->stream);
+    });
+    if (s2 != LFD_OK) return bail(s2);
+    e = cudaMemsetAsync(c->at<int>(L.colE), 0, sizeof(int) * g.ndom * g.norb, c->stream);
+    if (e == cudaSuccess) e = cudaMemsetAsync(c->at<int>(L.g1cnt), 0, sizeof(int) * g.ndom, c->stream);
+    if (e != cudaSuccess) { cuda_fail(c, e, "memset"); return bail(LFD_ECUDA); }
   }
   if (cfg->flags & LFD_FLAG_EXACT_NL) {
     // exactly unitary nonlocal factor: needs dV B^H B = I (checked on G), then
@@ -1394,6 +1434,12 @@ lfd_status lfd_sc_comm_init(lfd_ctx* c, int32_t nranks, int32_t rank, const void
 lfd_status lfd_psi_modified(lfd_ctx* c) {
   LFD_TRY(check_ctx(c));
   c->c_valid = false;
+  if (c->colE_valid) {  // orbital exponents of a Psi that no longer exists: clear them (stream order)
+    DeviceGuard dg(c->device);
+    cudaError_t e = cudaMemsetAsync(c->at<int>(c->L.colE), 0, sizeof(int) * c->g.ndom * c->g.norb, c->stream);
+    if (e != cudaSuccess) return cuda_fail(c, e, "memset");
+    c->colE_valid = false;
+  }
   return LFD_OK;
 }
 

@@ -365,7 +365,7 @@ template <bool kPer, bool kS>
 __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant__ CUtensorMap tmap,
                                                           double2* __restrict__ psi, const DomCoef* __restrict__ coef,
                                                           const double2* __restrict__ phi, int nx, int ny, int nz,
-                                                          int norb, int nchunks, long long ng) {
+                                                          int norb, int nchunks, long long ng, int* __restrict__ colE) {
   pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
   pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   // periodic => nz even (validated), so every thread owns a full pair and every link exists
@@ -467,11 +467,18 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
     __syncwarp();
     if ((tid & 31) == 0) mbar_arrive(&empty[s]);
   };
+  // colE != nullptr: the largest biased FP64 exponent of Re / Im of each orbital's output, for the int8-digit
+  // GEMM-1 that follows (its per-orbital power-of-two scale; nl_i8.cu) -- integer max on the high words
+  int me = 0;
+  auto trk = [&](double2 w) {
+    me = max(me, max(__double2hiint(w.x) & 0x7ff00000, __double2hiint(w.y) & 0x7ff00000));
+    return w;
+  };
   auto put0 = [&](int y, double2 f, double2 v) {
-    if (act) out0[y * yst] = cmul(f, v);
+    if (act) out0[y * yst] = trk(cmul(f, v));
   };
   auto put1 = [&](int y, double2 f, double2 v) {
-    if (act && has1) out1[y * yst] = cmul(f, v);
+    if (act && has1) out1[y * yst] = trk(cmul(f, v));
   };
 
   LineMarch<kS> L0, L1;
@@ -507,10 +514,10 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
       const double2* pb = slot_phi(s_prev + 1);
       const double2 fa0 = pa[pz0], fa1 = pa[pz1], fb0 = pb[pz0], fb1 = pb[pz1];
       L0.steady(cy, wa0, wb0, [&](int k, double2 v) {
-        if (act) o0p[k * yst] = cmul(k == 0 ? fa0 : fb0, v);
+        if (act) o0p[k * yst] = trk(cmul(k == 0 ? fa0 : fb0, v));
       });
       L1.steady(cy, wa1, wb1, [&](int k, double2 v) {
-        if (act) o0p[k * yst + norb] = cmul(k == 0 ? fa1 : fb1, v);
+        if (act) o0p[k * yst + norb] = trk(cmul(k == 0 ? fa1 : fb1, v));
       });
       release(s_prev);
       release(s_prev + 1);
@@ -575,6 +582,11 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
   auto pick1 = [&](int y) { return y == 0 ? f01 : y == 1 ? f11 : y == ny - 1 ? fl1 : fm1; };
   L0.template finish<kPer>(cy, ny, [&](int y, double2 v) { put0(y, pick0(y), v); });
   L1.template finish<kPer>(cy, ny, [&](int y, double2 v) { put1(y, pick1(y), v); });
+  if (colE) {  // max over this orbital's lanes (o = lane % 8), then one global atomicMax per (CTA, orbital)
+    me = max(me, __shfl_xor_sync(0xffffffffu, me, 8));
+    me = max(me, __shfl_xor_sync(0xffffffffu, me, 16));
+    if ((tid & 31) < kYZW && act) atomicMax(colE + (long long)dom * norb + o0 + o, me >> 20);
+  }
 }
 
 bool kin_yz_supported(const Geometry& g) { return g.nz <= 80; }
@@ -600,13 +612,13 @@ cudaError_t kin_yz_set_attributes() {
 }
 
 cudaError_t launch_kin_yz(const Geometry& g, const CUtensorMap* tmap, double2* psi, const DomCoef* coef,
-                          const double2* phi, bool scaled, cudaStream_t st) {
+                          const double2* phi, bool scaled, cudaStream_t st, int* colE) {
   const int nchunks = (g.norb + kYZW - 1) / kYZW;
   const int threads = ((((g.nz + 1) / 2) * kYZW + 31) / 32 + 1) * 32;  // consumer warps + producer warp
   dim3 grid(g.nx * nchunks, g.ndom);
   const size_t sm = yz_smem(g.nz);
 #define LFD_KYZ(P, K) \
-  launch_k(k_kin_yz<P, K>, grid, threads, sm, st, *tmap, psi, coef, phi, g.nx, g.ny, g.nz, g.norb, nchunks, g.ng)
+  launch_k(k_kin_yz<P, K>, grid, threads, sm, st, *tmap, psi, coef, phi, g.nx, g.ny, g.nz, g.norb, nchunks, g.ng, colE)
   if (g.bc == 0) {
     if (scaled) LFD_KYZ(true, true); else LFD_KYZ(true, false);
   } else {

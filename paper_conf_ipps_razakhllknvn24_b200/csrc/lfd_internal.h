@@ -95,8 +95,10 @@ cudaError_t launch_kin_sp(const Geometry& g, float2* psi, const DomCoef* coef, c
 // Fused pass Psi <- Phi . K_y K_z Psi (one read + write of Psi; nz <= 80).
 bool kin_yz_supported(const Geometry& g);
 cudaError_t kin_yz_tensor_map(const Geometry& g, double2* psi, CUtensorMap* out);
+// colE != nullptr: atomicMax of the biased FP64 exponent of every output Re / Im per orbital into
+// colE[dom][norb] (the per-orbital scale of the int8-digit GEMM-1, nl_i8.cu)
 cudaError_t launch_kin_yz(const Geometry& g, const CUtensorMap* tmap, double2* psi, const DomCoef* coef,
-                          const double2* phi, bool scaled, cudaStream_t st);
+                          const double2* phi, bool scaled, cudaStream_t st, int* colE = nullptr);
 cudaError_t kin_yz_set_attributes();
 
 // GEMM-1 split-K: part[dom][split][mrows][ncols] (complex) = sum over the split's grid rows of
@@ -175,6 +177,24 @@ cudaError_t launch_bslice_i8(const double2* B, int ndom, int nproj, long long ng
                              cudaStream_t st);
 cudaError_t launch_gemm2_i8(const Gemm2Args& a, cudaStream_t st);
 cudaError_t gemm_i8_set_attributes();
+// GEMM-1 with FP64 accuracy on the int8 tensor cores (nl_i8.cu): split partials (same layout as launch_gemm1)
+// of C = B^H Psi and the column norms; needs colE[dom][norb] from the K_y K_z pass that wrote Psi.
+struct Gemm1I8Args {
+  const double2* psi;
+  const int8_t* bsl1;   // B digit blocks (launch_bslice1_i8)
+  const int* bexp;      // [dom][nproj] B column exponents
+  int* colE;            // [dom][norb] Psi orbital exponents (cleared by the last CTA)
+  int* counter;         // [dom] CTA completion counters (zero between calls)
+  double2* part;        // [dom][nsplit][nproj][norb]
+  double* norms;        // [dom][nsplit][norb]
+  int ndom, nproj, norb, nsplit;
+  long long ng, rps;
+};
+size_t gemm1_i8_bytes(int ndom, long long ng);
+long long gemm1_i8_rows_per_split(long long ng, int ndom, int num_sms);
+cudaError_t launch_bslice1_i8(const double2* B, int ndom, int nproj, long long ng, int* bexp, int8_t* out,
+                              cudaStream_t st);
+cudaError_t launch_gemm1_i8(const Gemm1I8Args& a, cudaStream_t st);
 int gemm2_smem_bytes();
 cudaError_t gemm_set_attributes();
 

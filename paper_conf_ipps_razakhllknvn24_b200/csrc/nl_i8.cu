@@ -72,15 +72,44 @@ __device__ __forceinline__ void digits4(const double v[4], int e, bool zero, uin
   double x[4];
 #pragma unroll
   for (int q = 0; q < 4; ++q) x[q] = zero ? 0.0 : ldexp(v[q], 6 - e);  // 64 x, exact
+  // rint and the integer conversion in one full-rate DADD: x + 1.5 2^52 rounds x to the nearest integer
+  // (ties to even, as rint) and holds it in the low word; no FRND / F2I (low-rate conversion pipe)
+  constexpr double kM = 6755399441055744.0;
 #pragma unroll
   for (int i = 0; i < kI8S; ++i) {
     uint32_t w = 0;
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
-      const double d = rint(x[q]);
+      const double t = x[q] + kM;
+      const double d = t - kM;
       x[q] = (x[q] - d) * 128.0;  // exact: |x - d| <= 1/2
-      w |= ((uint32_t)(int)d & 0xffu) << (8 * q);
+      w |= ((uint32_t)__double2loint(t) & 0xffu) << (8 * q);
     }
+    out[i] = w;
+  }
+}
+
+// bytewise two's-complement negation of 4 packed int8 digits
+__device__ __forceinline__ uint32_t neg_bytes(uint32_t w) { return __vsub4(0u, w); }
+
+// the 6 balanced base-128 digits of 4 values in integer arithmetic: X = rint(v sc) (one DFMA against
+// 1.5 2^52; |X| < 2^41), X + C with C = 64 (128^6 - 1) / 127 has the unsigned 7-bit fields u_k, and
+// d = u - 64 in [-64, 63] (the top field u_5 <= 128: d_1 in [-64, 64]). X = sum_i d_i 128^(6-i): the same
+// digit weights as digits4 (digit i <-> field 6 - i), a different but exact decomposition.
+__device__ __forceinline__ void digits_i64(const double v[4], double sc, uint32_t out[kI8S]) {
+  constexpr double kM = 6755399441055744.0;
+  constexpr long long kMb = 0x4338000000000000LL;
+  constexpr long long kC = 64LL * ((1LL << 42) - 1) / 127;
+  long long Y[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) Y[q] = (__double_as_longlong(fma(v[q], sc, kM)) - kMb) + kC;
+#pragma unroll
+  for (int i = 0; i < kI8S; ++i) {
+    const int k = 6 - 1 - i;  // digit i + 1 (most significant first) <-> field k
+    uint32_t w = 0;
+#pragma unroll
+    for (int q = 0; q < 4; ++q)  // field k (the top field may be 128: not masked to 7 bits), minus 64
+      w |= ((((uint32_t)(Y[q] >> (7 * k)) & (k == 5 ? 0xffu : 0x7fu)) + 192u) & 0xffu) << (8 * q);
     out[i] = w;
   }
 }
@@ -272,7 +301,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
         v[2] = cn ? x.y : x.x; v[3] = cn ? x.x : -x.y;
       }
       uint32_t d[kI8S];
-      digits4(v, e, !(mx > 0.0), d);
+      digits_i64(v, mx > 0.0 ? ldexp(1.0, 41 - e) : 0.0, d);
 #pragma unroll
       for (int i = 0; i < kI8S; ++i) dg[i][w] = d[i];
     }
@@ -442,6 +471,325 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
   }
 }
 
+// ================================================================================================
+// GEMM-1 (Eq. 7 / Eq. 9): split partials of C[u][s] = sum_r conj(B[r][u]) Psi[r][s]
+// and the column norms sum_r |Psi[r][s]|^2, with the same digit scheme.
+//
+// Real form: D[m][u] = sum_k A[m][k] Bd[u][k] with m = 2s + c (M = 128), k = 2 rr + c' over the grid
+// rows of a 64-row block (K = 128 per block): A[2s][2rr] = Re Psi, A[2s][2rr+1] = Im Psi,
+// A[2s+1][2rr] = Im Psi, A[2s+1][2rr+1] = -Re Psi; Bd[u][2rr] = Re B, Bd[u][2rr+1] = Im B; then
+// D[2s][u] = Re C[u][s], D[2s+1][u] = Im C[u][s]. Scales are global over the domain, so the int32
+// accumulators run over a CTA's whole split (|P_d| <= 6 x 2 rows x 64 x 64 < 2^31 for <= 43,690 rows):
+// sigma_u = 2^e (max_r |Re B|, |Im B| of column u < 2^e, once at lfd_init) and tau_s = 2^(E_s - 1022)
+// with E_s the largest biased exponent of Re / Im Psi of orbital s, recorded by the K_y K_z pass that
+// wrote Psi (k_kin_yz, atomicMax) and cleared here by the last CTA. B's digits: once at lfd_init, per
+// 64-row block [6][64 u][128 B] in the SWIZZLE_128B image (one bulk copy). Psi's digits: per 32-row half
+// block, built by 16 worker warps straight into TMEM (the A operand, 6 x 16 columns), while the MMAs of
+// the previous half run (a single A buffer: the workers hold the next half's digits in registers until
+// the MMA warp releases it). TMEM: A 96 columns + 6 diagonal accumulators x 64 columns.
+// ================================================================================================
+constexpr int kG1Rows = 64;                        // grid rows per B-digit block (K = 128 bytes)
+constexpr int kG1Half = 32;                        // grid rows per A (Psi-digit) half block
+constexpr int kG1SliceB = 64 * 128;                // 8 KB: one digit slice of a B block (64 u rows)
+constexpr int kG1BlkB = kI8S * kG1SliceB;          // 48 KB
+constexpr int kG1Stages = 2;                       // B-digit ring
+constexpr int kG1PsiB = kG1Half * 64 * 16;         // 32 KB: Psi rows of a half block (norb <= 64)
+constexpr int kG1PsiSlots = 3;                     // Psi half-block ring
+constexpr int kG1Smem = kG1Stages * kG1BlkB + kG1PsiSlots * kG1PsiB + 1024;
+constexpr int kG1Workers = 16;                     // worker warps: 4 lane quarters x 4 row groups
+constexpr int kG1Threads = (kG1Workers + 2) * 32;  // + producer + MMA
+constexpr int kG1WProd = kG1Workers, kG1WMma = kG1Workers + 1;
+constexpr int kG1ACols = kI8S * 16;                // TMEM columns of the A buffer (K = 64 bytes per digit)
+constexpr uint32_t kG1Idesc = (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(64 >> 3) << 17) |
+                              ((uint32_t)(128 >> 4) << 24);  // s32 <- s8 x s8, K-major, N = 64, M = 128
+
+__device__ __forceinline__ void umma_g1_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t accumulate) {
+  asm volatile(
+      "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(db), "r"(kG1Idesc), "r"(accumulate));
+}
+__device__ __forceinline__ void tmem_st4(uint32_t taddr, const uint32_t v[4]) {
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1,%2,%3,%4};" ::"r"(taddr), "r"(v[0]), "r"(v[1]),
+               "r"(v[2]), "r"(v[3])
+               : "memory");
+}
+
+// B's GEMM-1 scales: bexp[dom][u] = max over the domain of the biased exponent of Re / Im B[r][u]
+__global__ void __launch_bounds__(256) k_bexp1_i8(const double2* __restrict__ B, int nproj, long long ng,
+                                                  int* __restrict__ bexp) {
+  pdl_wait();
+  pdl_trigger();
+  const int dom = blockIdx.y;
+  int me = 0;
+  const long long n = ng * nproj;
+  const double2* b = B + (long long)dom * n;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+    const double2 v = b[i];
+    const int u = (int)(i % nproj);
+    const int e = max(__double2hiint(v.x) & 0x7ff00000, __double2hiint(v.y) & 0x7ff00000) >> 20;
+    if (e > 0) atomicMax(bexp + (long long)dom * nproj + u, e);
+  }
+  (void)me;
+}
+
+// B's GEMM-1 digits: warp per (64-row block, u); lane l holds rows 2l, 2l+1 (k = 4l .. 4l+3)
+__global__ void __launch_bounds__(256) k_bslice1_i8(const double2* __restrict__ B, int nproj, long long ng,
+                                                    long long nblk, const int* __restrict__ bexp,
+                                                    int8_t* __restrict__ out) {
+  pdl_wait();
+  pdl_trigger();
+  const int dom = blockIdx.y, lane = threadIdx.x & 31;
+  const long long wid = (long long)blockIdx.x * 8 + (threadIdx.x >> 5);
+  if (wid >= nblk * 64) return;
+  const long long blk = wid >> 6;
+  const int u = (int)(wid & 63);
+  double v[4] = {0.0, 0.0, 0.0, 0.0};
+  const int E = u < nproj ? bexp[(long long)dom * nproj + u] : 0;
+  if (u < nproj) {
+    const long long r = blk * kG1Rows + 2 * lane;
+    const double2* col = B + (long long)dom * ng * nproj + u;
+    if (r < ng) { const double2 a = col[r * nproj]; v[0] = a.x; v[1] = a.y; }
+    if (r + 1 < ng) { const double2 a = col[(r + 1) * nproj]; v[2] = a.x; v[3] = a.y; }
+  }
+  uint32_t d[kI8S];
+  digits4(v, E - 1022, E == 0, d);  // |v| < 2^(E - 1022)
+  int8_t* tb = out + ((long long)dom * nblk + blk) * kG1BlkB;
+#pragma unroll
+  for (int i = 0; i < kI8S; ++i) *reinterpret_cast<uint32_t*>(tb + i * kG1SliceB + sw128(u, 4 * lane)) = d[i];
+}
+
+// grid (splits, ndom); CTA = one split of rps rows (a multiple of 64)
+__global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
+  pdl_wait();
+  pdl_trigger();
+  extern __shared__ __align__(1024) unsigned char dsm_raw[];
+  unsigned char* dsm = dsm_raw + ((1024u - (smem_addr(dsm_raw) & 1023u)) & 1023u);
+  unsigned char* Bsm = dsm;                            // [stages][6][64 u][128 B] swizzled B digits
+  unsigned char* Psm = Bsm + kG1Stages * kG1BlkB;      // [slots][32 rows][norb] complex
+  __shared__ __align__(8) uint64_t bfull[kG1Stages], bempty[kG1Stages], pfull[kG1PsiSlots], pempty[kG1PsiSlots];
+  __shared__ __align__(8) uint64_t afull, afree, done;
+  __shared__ uint32_t tmem_base_sh;
+  __shared__ double nsum[4][64];
+  __shared__ int last_sh;
+
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int dom = blockIdx.y, split = blockIdx.x;
+  const int norb = p.norb, nproj = p.nproj;
+  const long long ng = p.ng;
+  const long long nblk = (ng + kG1Rows - 1) / kG1Rows;
+  const long long r0 = (long long)split * p.rps;
+  const long long r1 = min(ng, r0 + p.rps);
+  const int nhalf = (int)((r1 - r0 + kG1Half - 1) / kG1Half);  // half blocks of this split
+  const int rowb = norb * 16;
+
+  if (warp == kG1WMma) {  // TMEM: A (Psi digits, 96 columns) + 6 diagonal accumulators x 64 columns
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_addr(&tmem_base_sh)));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  if (tid == 0) {
+    for (int s = 0; s < kG1Stages; ++s) { mbar_init(&bfull[s], 1); mbar_init(&bempty[s], 1); }
+    for (int s = 0; s < kG1PsiSlots; ++s) { mbar_init(&pfull[s], 1); mbar_init(&pempty[s], kG1Workers); }
+    mbar_init(&afull, kG1Workers);
+    mbar_init(&afree, 1);
+    mbar_init(&done, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_base_sh;
+  const uint32_t tacc = tmem + kG1ACols;
+
+  if (warp == kG1WProd) {  // producer: B-digit blocks and Psi half blocks, in the order the MMAs use them
+    if (lane == 0) {
+      const int8_t* src = p.bsl1 + (long long)dom * nblk * kG1BlkB;
+      const double2* prow = p.psi + (long long)dom * ng * norb;
+      for (int g = 0; g < nhalf; ++g) {
+        if ((g & 1) == 0) {
+          const int b = g >> 1, s = b % kG1Stages;
+          if (b >= kG1Stages) mbar_wait(&bempty[s], (uint32_t)(((b / kG1Stages) - 1) & 1));
+          mbar_expect_tx(&bfull[s], kG1BlkB);
+          tma_row(Bsm + s * kG1BlkB, src + (r0 / kG1Rows + b) * kG1BlkB, kG1BlkB, &bfull[s]);
+        }
+        const int s = g % kG1PsiSlots;
+        if (g >= kG1PsiSlots) mbar_wait(&pempty[s], (uint32_t)(((g / kG1PsiSlots) - 1) & 1));
+        const long long ra = r0 + (long long)g * kG1Half;
+        const long long nr = (r1 - ra) < kG1Half ? (r1 - ra) : kG1Half;
+        mbar_expect_tx(&pfull[s], (uint32_t)(nr * rowb));
+        tma_row(Psm + s * kG1PsiB, prow + ra * norb, (uint32_t)(nr * rowb), &pfull[s]);
+      }
+    }
+  } else if (warp == kG1WMma) {  // MMA issuer
+    if (lane == 0) {
+      const uint32_t bbase = smem_addr(Bsm);
+      for (int g = 0; g < nhalf; ++g) {
+        const int b = g >> 1, s = b % kG1Stages, hb = g & 1;
+        if (hb == 0) mbar_wait(&bfull[s], (uint32_t)((b / kG1Stages) & 1));
+        mbar_wait(&afull, (uint32_t)(g & 1));
+        tc_fence_after();
+        const uint64_t db0 = umma_desc_sw128(bbase + s * kG1BlkB);
+#pragma unroll
+        for (int d = 2; d <= kI8S + 1; ++d) {
+          const uint32_t acc = tacc + (d - 2) * 64;
+#pragma unroll
+          for (int i = 1; i <= kI8S; ++i) {  // i: B digit, j: Psi digit
+            const int j = d - i;
+            if (j < 1 || j > kI8S) continue;
+#pragma unroll
+            for (int kl = 0; kl < 2; ++kl) {
+              const bool first = (g == 0) && (i == (d - 1 < kI8S ? 1 : d - kI8S)) && kl == 0;
+              umma_g1_ts(acc, tmem + (j - 1) * 16 + kl * 8,
+                         db0 + (uint64_t)(((i - 1) * kG1SliceB + (2 * hb + kl) * 32) >> 4), first ? 0u : 1u);
+            }
+          }
+        }
+        umma_commit(&afree);                          // the A buffer may take the next half block
+        if (hb == 1 || g + 1 == nhalf) umma_commit(&bempty[s]);
+      }
+      umma_commit(&done);
+    }
+  } else {  // workers: Psi digits into TMEM, column norms; at the end the accumulators into FP64 partials
+    const int q = warp & 3, h = warp >> 2;    // lane quarter, row group (8 rows of each half block)
+    const int m = 32 * q + lane, sIdx = m >> 1, cm = m & 1;
+    const bool sv = sIdx < norb;
+    const int E = sv ? p.colE[(long long)dom * norb + sIdx] : 0;
+    const bool zc = E == 0;                   // an all-zero orbital (or none): zero digits
+    const double sc41 = zc ? 0.0 : ldexp(1.0, 41 - (E - 1022));  // x 2^41 / tau_s: |v sc41| < 2^41
+    double nrm = 0.0;
+    const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
+    for (int g = 0; g < nhalf; ++g) {
+      const int s = g % kG1PsiSlots;
+      mbar_wait(&pfull[s], (uint32_t)((g / kG1PsiSlots) & 1));
+      const long long ra = r0 + (long long)g * kG1Half;
+      const double2* P = reinterpret_cast<const double2*>(Psm + s * kG1PsiB) + sIdx;
+      // each lane digitises its own component only (even lane m = 2s: Re, odd lane: Im) of its 8 rows, in
+      // integer arithmetic (digits_i64), and the lane pair exchanges them: row 2s of A takes (Re, Im) per
+      // grid row, row 2s+1 takes (Im, -Re) (bytewise negated digits: still an exact decomposition)
+      uint32_t own[kI8S][2];  // [digit][w pair]: bytes (rows 8h+4wp .. +3)
+#pragma unroll
+      for (int wp = 0; wp < 2; ++wp) {
+        double v[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          const int rr = 8 * h + 4 * wp + t;
+          v[t] = 0.0;
+          if (sv && ra + rr < r1) {
+            const double2 x = P[rr * norb];
+            v[t] = cm ? x.y : x.x;
+            nrm = fma(v[t], v[t], nrm);
+          }
+        }
+        uint32_t d[kI8S];
+        digits_i64(v, sc41, d);
+#pragma unroll
+        for (int i = 0; i < kI8S; ++i) own[i][wp] = d[i];
+      }
+      uint32_t dg[kI8S][4];
+#pragma unroll
+      for (int i = 0; i < kI8S; ++i)
+#pragma unroll
+        for (int wp = 0; wp < 2; ++wp) {
+          const uint32_t mine = own[i][wp];
+          const uint32_t other = __shfl_xor_sync(0xffffffffu, mine, 1);
+          // bytes t = 0..3 of mine / other are rows 8h+4wp+t; A row word w = 2 wp + (t >> 1) holds rows
+          // (2w, 2w+1) as [c'=0, c'=1, c'=0, c'=1]
+          const uint32_t a = cm ? mine : mine, b = cm ? neg_bytes(other) : other;
+          // even lane: c'=0 own (Re), c'=1 other (Im); odd lane: c'=0 own (Im), c'=1 -other (-Re)
+          dg[i][2 * wp] = __byte_perm(a, b, 0x5140);      // [a0, b0, a1, b1]
+          dg[i][2 * wp + 1] = __byte_perm(a, b, 0x7362);  // [a2, b2, a3, b3]
+        }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&pempty[s]);  // this warp is done with the Psi rows
+      if (g > 0) mbar_wait(&afree, (uint32_t)((g - 1) & 1));  // the MMAs of half block g - 1 are done with A
+      tc_fence_after();
+#pragma unroll
+      for (int i = 0; i < kI8S; ++i) tmem_st4(trow + i * 16 + 4 * h, dg[i]);
+      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&afull);
+    }
+    // column norms: Re^2 (even lane) + Im^2 (odd lane), then a fixed-order sum over the 4 row groups
+    nrm += __shfl_xor_sync(0xffffffffu, nrm, 1);
+    if (!cm && sv) nsum[h][sIdx] = nrm;
+    mbar_wait(&done, 0);
+    tc_fence_after();
+    // accumulators: warp (q, h) reads lanes 32 q .. (rows m) and columns u = 16 h .. 16 h + 15
+    double cacc[16];
+#pragma unroll
+    for (int c = 0; c < 16; ++c) cacc[c] = 0.0;
+#pragma unroll 1
+    for (int d = 2; d <= kI8S + 1; ++d) {
+      int32_t a[16];
+      tmem_ld16(tacc + (d - 2) * 64 + ((uint32_t)(32 * q) << 16) + 16 * h, a);
+      tmem_wait_ld();
+      const double wd = ldexp(1.0, -7 * (d - 2));
+#pragma unroll
+      for (int c = 0; c < 16; ++c) cacc[c] = fma(i2d(a[c]), wd, cacc[c]);
+    }
+    // C[u][s] = sigma_u tau_s 2^-12 cacc; m = 2 s + cm -> Re (cm 0) / Im (cm 1)
+    const double tau = zc ? 0.0 : ldexp(1.0, E - 1022 - 12);
+    double* part = reinterpret_cast<double*>(p.part + ((long long)dom * p.nsplit + split) * nproj * norb);
+#pragma unroll
+    for (int c = 0; c < 16; ++c) {
+      const int u = 16 * h + c;
+      if (!sv || u >= nproj) continue;
+      const int eb = p.bexp[(long long)dom * nproj + u];
+      const double sig = eb == 0 ? 0.0 : ldexp(1.0, eb - 1022);
+      part[2 * ((long long)u * norb + sIdx) + cm] = sig * tau * cacc[c];
+    }
+    asm volatile("bar.sync 1, %0;" ::"n"(kG1Workers * 32) : "memory");
+    if (tid < norb)
+      p.norms[((long long)dom * p.nsplit + split) * norb + tid] =
+          (nsum[0][tid] + nsum[1][tid]) + (nsum[2][tid] + nsum[3][tid]);
+  }
+  tc_fence_before();
+  __syncthreads();
+  // the last CTA of the domain clears the orbital exponents for the next K_y K_z pass
+  if (tid == 0) {
+    __threadfence();
+    last_sh = atomicAdd(p.counter + dom, 1) == (int)gridDim.x - 1;
+  }
+  __syncthreads();
+  if (last_sh) {
+    for (int i = tid; i < norb; i += blockDim.x) p.colE[(long long)dom * norb + i] = 0;
+    if (tid == 0) p.counter[dom] = 0;
+  }
+  if (warp == kG1WMma) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
+  }
+}
+
+size_t gemm1_i8_bytes(int ndom, long long ng) {
+  const long long nblk = (ng + kG1Rows - 1) / kG1Rows;
+  return (size_t)ndom * nblk * kG1BlkB;
+}
+long long gemm1_i8_rows_per_split(long long ng, int ndom, int num_sms) {
+  int cpd = num_sms / ndom;
+  if (cpd < 1) cpd = 1;
+  long long rps = (ng + cpd - 1) / cpd;
+  rps = (rps + kG1Rows - 1) / kG1Rows * kG1Rows;
+  if (rps > 32768) rps = 32768;  // int32 accumulators: 6 x 2 rps x 64 x 64 < 2^31
+  return rps;
+}
+cudaError_t launch_bslice1_i8(const double2* B, int ndom, int nproj, long long ng, int* bexp, int8_t* out,
+                              cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(bexp, 0, sizeof(int) * ndom * nproj, st);
+  if (e != cudaSuccess) return e;
+  launch_k(k_bexp1_i8, dim3(296, ndom), 256, 0, st, B, nproj, ng, bexp);
+  const long long nblk = (ng + kG1Rows - 1) / kG1Rows;
+  dim3 grid((unsigned)((nblk * 64 + 7) / 8), ndom);
+  launch_k(k_bslice1_i8, grid, 256, 0, st, B, nproj, ng, nblk, (const int*)bexp, out);
+  return cudaGetLastError();
+}
+cudaError_t launch_gemm1_i8(const Gemm1I8Args& a, cudaStream_t st) {
+  dim3 grid(a.nsplit, a.ndom);
+  launch_k(k_gemm1_i8, grid, kG1Threads, kG1Smem, st, a);
+  return cudaGetLastError();
+}
+
 size_t gemm2_i8_bytes(int ndom, long long ng) {
   const long long tiles = (ng + kI8NT - 1) / kI8NT;
   return (size_t)ndom * tiles * kI8TileB;
@@ -473,6 +821,8 @@ cudaError_t launch_gemm2_i8(const Gemm2Args& a, cudaStream_t st) {
 
 cudaError_t gemm_i8_set_attributes() {
   cudaError_t e = cudaFuncSetAttribute(k_gemm2_i8<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kI8Smem);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_gemm1_i8, cudaFuncAttributeMaxDynamicSharedMemorySize, kG1Smem);
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(k_gemm2_i8<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kI8Smem);
 }
