@@ -36,8 +36,9 @@ NCU_NAMES = {"nl_proj": "k_gemm1", "nl_back": "k_gemm2", "kin_x": "k_kin<1, 1, 1
              "kin_z": "k_kin<1, 2>", "kin_yz": "k_kin_yz", "density": "k_density"}
 
 
-def ncu_traffic(kernel):
-    """DRAM bytes per launch (read + write) of `kernel` from the committed ncu --set full summary."""
+def ncu_traffic(kernel, i8=False):
+    """DRAM bytes per launch (read + write) of `kernel` from the committed ncu --set full summary (i8: the
+    int8-digit tensor-core GEMM kernels k_gemm1_i8 / k_gemm2_i8)."""
     import csv
     if not os.path.exists(NCU_SUMMARY) or kernel not in NCU_NAMES:
         return None
@@ -51,7 +52,9 @@ def ncu_traffic(kernel):
     scale = {"[byte]": 1.0, "[Kbyte]": 1e3, "[Mbyte]": 1e6, "[Gbyte]": 1e9}
     vals = []
     for r in rows[1:]:
-        if r[0].replace("void ", "").replace("lfd::", "").startswith(NCU_NAMES[kernel]):
+        name = r[0].replace("void ", "").replace("lfd::", "")
+        want = NCU_NAMES[kernel] + ("_i8" if i8 and kernel in ("nl_proj", "nl_back") else "")
+        if name.startswith(want) and (i8 or "_i8" not in name):
             sr = next((v for k, v in scale.items() if hdr[ir].endswith(k)), 1.0)
             sw = next((v for k, v in scale.items() if hdr[iw].endswith(k)), 1.0)
             vals.append(float(r[ir]) * sr + float(r[iw]) * sw)
@@ -347,10 +350,10 @@ def run_sp_mode(args, w, x, dev, stream, pk):
         e = {"ms_per_launch": avg, "launches": cnt, "share": round(kms / tot, 4)}
         if k in work:
             b, f = work[k]
-            if k == "nl_back" and nl_path == 1:
-                # int8-digit tcgen05 GEMM-2 (FP64 accuracy): the digit products are cheap on the int8 tensor
-                # cores, so the kernel is bound by streaming Psi (read + write) and B -- report it against
-                # HBM with the FP64 operation's algorithmic bytes, and its FP64-equivalent rate alongside
+            if k in ("nl_back", "nl_proj") and nl_path == 1:
+                # int8-digit tcgen05 GEMMs (FP64 accuracy): the digit products are cheap on the int8 tensor
+                # cores, so the kernels are bound by streaming Psi (read, + write for GEMM-2) and B -- report
+                # them against HBM with the FP64 operation's algorithmic bytes, and the FP64-equivalent rate
                 e.update({"bound": "hbm", "achieved": b / (avg * 1e-3) / 1e9, "unit": "GB/s", "peak": pk["hbm_gbs"],
                           "path": "int8-digit tcgen05 (FP64 accuracy)",
                           "fp64_equiv_tflops": f / (avg * 1e-3) / 1e12,
@@ -466,10 +469,10 @@ def main():
         e = {"ms_per_launch": avg, "launches": cnt, "share": kms / total_ms if total_ms else None}
         if k in work:
             b, f = work[k]
-            if k == "nl_back" and nl_path == 1:
-                # int8-digit tcgen05 GEMM-2 (FP64 accuracy): the digit products are cheap on the int8 tensor
-                # cores, so the kernel is bound by streaming Psi (read + write) and B -- report it against
-                # HBM with the FP64 operation's algorithmic bytes, and its FP64-equivalent rate alongside
+            if k in ("nl_back", "nl_proj") and nl_path == 1:
+                # int8-digit tcgen05 GEMMs (FP64 accuracy): the digit products are cheap on the int8 tensor
+                # cores, so the kernels are bound by streaming Psi (read, + write for GEMM-2) and B -- report
+                # them against HBM with the FP64 operation's algorithmic bytes, and the FP64-equivalent rate
                 e.update({"bound": "hbm", "achieved": b / (avg * 1e-3) / 1e9, "unit": "GB/s", "peak": pk["hbm_gbs"],
                           "path": "int8-digit tcgen05 (FP64 accuracy)",
                           "fp64_equiv_tflops": f / (avg * 1e-3) / 1e12,
@@ -485,7 +488,7 @@ def main():
     dom = max((k for k in kernels if "achieved" in kernels[k]), key=lambda k: prof[k][0])
     d = kernels[dom]
     roofline = {"kernel": dom, "bound": d["bound"], "achieved": d["achieved"], "peak": d["peak"], "unit": d["unit"],
-                "frac": d["frac"], "traffic": ncu_traffic(dom),
+                "frac": d["frac"], "traffic": ncu_traffic(dom, nl_path == 1),
                 "traffic_source": "profiles/latest_ncu_full_summary.csv (dram__bytes_read.sum + dram__bytes_write.sum "
                                   "per launch, ncu --set full)",
                 "peak_source": pk["zgemm3m_src"] if d["bound"] == "tensor" else pk["hbm_src"],
