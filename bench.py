@@ -350,15 +350,7 @@ def run_sp_mode(args, w, x, dev, stream, pk):
         e = {"ms_per_launch": avg, "launches": cnt, "share": round(kms / tot, 4)}
         if k in work:
             b, f = work[k]
-            if k in ("nl_back", "nl_proj") and nl_path == 1:
-                # int8-digit tcgen05 GEMMs (FP64 accuracy): the digit products are cheap on the int8 tensor
-                # cores, so the kernels are bound by streaming Psi (read, + write for GEMM-2) and B -- report
-                # them against HBM with the FP64 operation's algorithmic bytes, and the FP64-equivalent rate
-                e.update({"bound": "hbm", "achieved": b / (avg * 1e-3) / 1e9, "unit": "GB/s", "peak": pk["hbm_gbs"],
-                          "path": "int8-digit tcgen05 (FP64 accuracy)",
-                          "fp64_equiv_tflops": f / (avg * 1e-3) / 1e12,
-                          "fp64_equiv_vs_dmma_peak": f / (avg * 1e-3) / 1e12 / pk["zgemm3m_tflops"]})
-            elif f > 0:
+            if f > 0:
                 e.update({"bound": "tensor", "achieved": f / (avg * 1e-3) / 1e12, "unit": "TFLOP/s", "peak": tpeak})
             else:
                 e.update({"bound": "hbm", "achieved": 0.5 * b / (avg * 1e-3) / 1e9, "unit": "GB/s",

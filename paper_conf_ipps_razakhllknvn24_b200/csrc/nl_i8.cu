@@ -520,17 +520,20 @@ __global__ void __launch_bounds__(256) k_bexp1_i8(const double2* __restrict__ B,
                                                   int* __restrict__ bexp) {
   pdl_wait();
   pdl_trigger();
+  __shared__ int sm[64];
   const int dom = blockIdx.y;
-  int me = 0;
+  for (int u = threadIdx.x; u < 64; u += blockDim.x) sm[u] = 0;
+  __syncthreads();
   const long long n = ng * nproj;
   const double2* b = B + (long long)dom * n;
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
     const double2 v = b[i];
-    const int u = (int)(i % nproj);
     const int e = max(__double2hiint(v.x) & 0x7ff00000, __double2hiint(v.y) & 0x7ff00000) >> 20;
-    if (e > 0) atomicMax(bexp + (long long)dom * nproj + u, e);
+    if (e > 0) atomicMax(sm + (int)(i % nproj), e);  // shared-memory atomics, then one global per column
   }
-  (void)me;
+  __syncthreads();
+  for (int u = threadIdx.x; u < nproj; u += blockDim.x)
+    if (sm[u] > 0) atomicMax(bexp + (long long)dom * nproj + u, sm[u]);
 }
 
 // B's GEMM-1 digits: warp per (64-row block, u); lane l holds rows 2l, 2l+1 (k = 4l .. 4l+3)
