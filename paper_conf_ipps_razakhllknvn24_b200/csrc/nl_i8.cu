@@ -489,17 +489,18 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
 // the MMA warp releases it). TMEM: A 96 columns + 6 diagonal accumulators x 64 columns.
 // ================================================================================================
 constexpr int kG1Rows = 64;                        // grid rows per B-digit block (K = 128 bytes)
-constexpr int kG1Half = 32;                        // grid rows per A (Psi-digit) half block
+constexpr int kG1Half = 16;                        // grid rows per A (Psi-digit) quarter block (K = 32 bytes)
 constexpr int kG1SliceB = 64 * 128;                // 8 KB: one digit slice of a B block (64 u rows)
 constexpr int kG1BlkB = kI8S * kG1SliceB;          // 48 KB
 constexpr int kG1Stages = 2;                       // B-digit ring
-constexpr int kG1PsiB = kG1Half * 64 * 16;         // 32 KB: Psi rows of a half block (norb <= 64)
-constexpr int kG1PsiSlots = 3;                     // Psi half-block ring
+constexpr int kG1PsiB = kG1Half * 64 * 16;         // 16 KB: Psi rows of a quarter block (norb <= 64)
+constexpr int kG1PsiSlots = 6;                     // Psi quarter-block ring
 constexpr int kG1Smem = kG1Stages * kG1BlkB + kG1PsiSlots * kG1PsiB + 1024;
 constexpr int kG1Workers = 16;                     // worker warps: 4 lane quarters x 4 row groups
 constexpr int kG1Threads = (kG1Workers + 2) * 32;  // + producer + MMA
 constexpr int kG1WProd = kG1Workers, kG1WMma = kG1Workers + 1;
-constexpr int kG1ACols = kI8S * 16;                // TMEM columns of the A buffer (K = 64 bytes per digit)
+constexpr int kG1ABuf = kI8S * 8;                  // TMEM columns of one A buffer (K = 32 bytes per digit)
+constexpr int kG1ACols = 2 * kG1ABuf;              // double-buffered A
 constexpr uint32_t kG1Idesc = (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(64 >> 3) << 17) |
                               ((uint32_t)(128 >> 4) << 24);  // s32 <- s8 x s8, K-major, N = 64, M = 128
 
@@ -508,6 +509,9 @@ __device__ __forceinline__ void umma_g1_ts(uint32_t tmem_d, uint32_t tmem_a, uin
       "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
       "tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
       "r"(tmem_a), "l"(db), "r"(kG1Idesc), "r"(accumulate));
+}
+__device__ __forceinline__ void tmem_st2(uint32_t taddr, const uint32_t v[2]) {
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0], {%1,%2};" ::"r"(taddr), "r"(v[0]), "r"(v[1]) : "memory");
 }
 __device__ __forceinline__ void tmem_st4(uint32_t taddr, const uint32_t v[4]) {
   asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1,%2,%3,%4};" ::"r"(taddr), "r"(v[0]), "r"(v[1]),
@@ -571,7 +575,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   unsigned char* Bsm = dsm;                            // [stages][6][64 u][128 B] swizzled B digits
   unsigned char* Psm = Bsm + kG1Stages * kG1BlkB;      // [slots][32 rows][norb] complex
   __shared__ __align__(8) uint64_t bfull[kG1Stages], bempty[kG1Stages], pfull[kG1PsiSlots], pempty[kG1PsiSlots];
-  __shared__ __align__(8) uint64_t afull, afree, done;
+  __shared__ __align__(8) uint64_t afull[2], afree[2], done;
   __shared__ uint32_t tmem_base_sh;
   __shared__ double nsum[4][64];
   __shared__ int last_sh;
@@ -583,7 +587,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   const long long nblk = (ng + kG1Rows - 1) / kG1Rows;
   const long long r0 = (long long)split * p.rps;
   const long long r1 = min(ng, r0 + p.rps);
-  const int nhalf = (int)((r1 - r0 + kG1Half - 1) / kG1Half);  // half blocks of this split
+  const int nhalf = (int)((r1 - r0 + kG1Half - 1) / kG1Half);  // quarter blocks of this split
   const int rowb = norb * 16;
 
   if (warp == kG1WMma) {  // TMEM: A (Psi digits, 96 columns) + 6 diagonal accumulators x 64 columns
@@ -593,8 +597,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   if (tid == 0) {
     for (int s = 0; s < kG1Stages; ++s) { mbar_init(&bfull[s], 1); mbar_init(&bempty[s], 1); }
     for (int s = 0; s < kG1PsiSlots; ++s) { mbar_init(&pfull[s], 1); mbar_init(&pempty[s], kG1Workers); }
-    mbar_init(&afull, kG1Workers);
-    mbar_init(&afree, 1);
+    for (int b = 0; b < 2; ++b) { mbar_init(&afull[b], kG1Workers); mbar_init(&afree[b], 1); }
     mbar_init(&done, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -609,8 +612,8 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       const int8_t* src = p.bsl1 + (long long)dom * nblk * kG1BlkB;
       const double2* prow = p.psi + (long long)dom * ng * norb;
       for (int g = 0; g < nhalf; ++g) {
-        if ((g & 1) == 0) {
-          const int b = g >> 1, s = b % kG1Stages;
+        if ((g & 3) == 0) {
+          const int b = g >> 2, s = b % kG1Stages;
           if (b >= kG1Stages) mbar_wait(&bempty[s], (uint32_t)(((b / kG1Stages) - 1) & 1));
           mbar_expect_tx(&bfull[s], kG1BlkB);
           tma_row(Bsm + s * kG1BlkB, src + (r0 / kG1Rows + b) * kG1BlkB, kG1BlkB, &bfull[s]);
@@ -627,9 +630,9 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
     if (lane == 0) {
       const uint32_t bbase = smem_addr(Bsm);
       for (int g = 0; g < nhalf; ++g) {
-        const int b = g >> 1, s = b % kG1Stages, hb = g & 1;
-        if (hb == 0) mbar_wait(&bfull[s], (uint32_t)((b / kG1Stages) & 1));
-        mbar_wait(&afull, (uint32_t)(g & 1));
+        const int b = g >> 2, s = b % kG1Stages, kq = g & 3, ab = g & 1;
+        if (kq == 0) mbar_wait(&bfull[s], (uint32_t)((b / kG1Stages) & 1));
+        mbar_wait(&afull[ab], (uint32_t)((g >> 1) & 1));
         tc_fence_after();
         const uint64_t db0 = umma_desc_sw128(bbase + s * kG1BlkB);
 #pragma unroll
@@ -639,16 +642,13 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
           for (int i = 1; i <= kI8S; ++i) {  // i: B digit, j: Psi digit
             const int j = d - i;
             if (j < 1 || j > kI8S) continue;
-#pragma unroll
-            for (int kl = 0; kl < 2; ++kl) {
-              const bool first = (g == 0) && (i == (d - 1 < kI8S ? 1 : d - kI8S)) && kl == 0;
-              umma_g1_ts(acc, tmem + (j - 1) * 16 + kl * 8,
-                         db0 + (uint64_t)(((i - 1) * kG1SliceB + (2 * hb + kl) * 32) >> 4), first ? 0u : 1u);
-            }
+            const bool first = (g == 0) && (i == (d - 1 < kI8S ? 1 : d - kI8S));
+            umma_g1_ts(acc, tmem + ab * kG1ABuf + (j - 1) * 8,
+                       db0 + (uint64_t)(((i - 1) * kG1SliceB + kq * 32) >> 4), first ? 0u : 1u);
           }
         }
-        umma_commit(&afree);                          // the A buffer may take the next half block
-        if (hb == 1 || g + 1 == nhalf) umma_commit(&bempty[s]);
+        umma_commit(&afree[ab]);                      // A buffer ab may take quarter block g + 2
+        if (kq == 3 || g + 1 == nhalf) umma_commit(&bempty[s]);
       }
       umma_commit(&done);
     }
@@ -662,56 +662,48 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
     double nrm = 0.0;
     const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
     for (int g = 0; g < nhalf; ++g) {
-      const int s = g % kG1PsiSlots;
+      const int s = g % kG1PsiSlots, ab = g & 1;
       mbar_wait(&pfull[s], (uint32_t)((g / kG1PsiSlots) & 1));
       const long long ra = r0 + (long long)g * kG1Half;
       const double2* P = reinterpret_cast<const double2*>(Psm + s * kG1PsiB) + sIdx;
-      // each lane digitises its own component only (even lane m = 2s: Re, odd lane: Im) of its 8 rows, in
-      // integer arithmetic (digits_i64), and the lane pair exchanges them: row 2s of A takes (Re, Im) per
-      // grid row, row 2s+1 takes (Im, -Re) (bytewise negated digits: still an exact decomposition)
-      uint32_t own[kI8S][2];  // [digit][w pair]: bytes (rows 8h+4wp .. +3)
+      // each lane digitises its own component only (even lane m = 2s: Re, odd lane: Im) of its 4 rows
+      // (4h .. 4h + 3 of the quarter block), in integer arithmetic (digits_i64), and the lane pair exchanges
+      // them: row 2s of A takes (Re, Im) per grid row, row 2s+1 takes (Im, -Re) (bytewise negated digits:
+      // still an exact decomposition)
+      double v[4];
 #pragma unroll
-      for (int wp = 0; wp < 2; ++wp) {
-        double v[4];
-#pragma unroll
-        for (int t = 0; t < 4; ++t) {
-          const int rr = 8 * h + 4 * wp + t;
-          v[t] = 0.0;
-          if (sv && ra + rr < r1) {
-            const double2 x = P[rr * norb];
-            v[t] = cm ? x.y : x.x;
-            nrm = fma(v[t], v[t], nrm);
-          }
+      for (int t = 0; t < 4; ++t) {
+        const int rr = 4 * h + t;
+        v[t] = 0.0;
+        if (sv && ra + rr < r1) {
+          const double2 x = P[rr * norb];
+          v[t] = cm ? x.y : x.x;
+          nrm = fma(v[t], v[t], nrm);
         }
-        uint32_t d[kI8S];
-        digits_i64(v, sc41, d);
-#pragma unroll
-        for (int i = 0; i < kI8S; ++i) own[i][wp] = d[i];
       }
-      uint32_t dg[kI8S][4];
+      uint32_t own[kI8S];
+      digits_i64(v, sc41, own);
+      uint32_t dg[kI8S][2];
 #pragma unroll
-      for (int i = 0; i < kI8S; ++i)
-#pragma unroll
-        for (int wp = 0; wp < 2; ++wp) {
-          const uint32_t mine = own[i][wp];
-          const uint32_t other = __shfl_xor_sync(0xffffffffu, mine, 1);
-          // bytes t = 0..3 of mine / other are rows 8h+4wp+t; A row word w = 2 wp + (t >> 1) holds rows
-          // (2w, 2w+1) as [c'=0, c'=1, c'=0, c'=1]
-          const uint32_t a = cm ? mine : mine, b = cm ? neg_bytes(other) : other;
-          // even lane: c'=0 own (Re), c'=1 other (Im); odd lane: c'=0 own (Im), c'=1 -other (-Re)
-          dg[i][2 * wp] = __byte_perm(a, b, 0x5140);      // [a0, b0, a1, b1]
-          dg[i][2 * wp + 1] = __byte_perm(a, b, 0x7362);  // [a2, b2, a3, b3]
-        }
+      for (int i = 0; i < kI8S; ++i) {
+        const uint32_t mine = own[i];
+        const uint32_t other = __shfl_xor_sync(0xffffffffu, mine, 1);
+        // bytes t = 0..3 are rows 4h + t; A word w (K bytes 8h + 4w ..) holds rows (2w, 2w+1) as
+        // [c'=0, c'=1, c'=0, c'=1]; even lane: c'=0 own (Re), c'=1 other (Im); odd lane: own (Im), -other
+        const uint32_t b = cm ? neg_bytes(other) : other;
+        dg[i][0] = __byte_perm(mine, b, 0x5140);  // [a0, b0, a1, b1]
+        dg[i][1] = __byte_perm(mine, b, 0x7362);  // [a2, b2, a3, b3]
+      }
       __syncwarp();
       if (lane == 0) mbar_arrive(&pempty[s]);  // this warp is done with the Psi rows
-      if (g > 0) mbar_wait(&afree, (uint32_t)((g - 1) & 1));  // the MMAs of half block g - 1 are done with A
+      if (g >= 2) mbar_wait(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));  // MMAs of block g - 2 are done with it
       tc_fence_after();
 #pragma unroll
-      for (int i = 0; i < kI8S; ++i) tmem_st4(trow + i * 16 + 4 * h, dg[i]);
+      for (int i = 0; i < kI8S; ++i) tmem_st2(trow + ab * kG1ABuf + i * 8 + 2 * h, dg[i]);
       asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(&afull);
+      if (lane == 0) mbar_arrive(&afull[ab]);
     }
     // column norms: Re^2 (even lane) + Im^2 (odd lane), then a fixed-order sum over the 4 row groups
     nrm += __shfl_xor_sync(0xffffffffu, nrm, 1);
