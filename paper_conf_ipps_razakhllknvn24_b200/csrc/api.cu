@@ -517,7 +517,23 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
     ai.part = a1.part; ai.norms = a1.norms;
     ai.ndom = g.ndom; ai.nproj = g.nproj; ai.norb = g.norb; ai.nsplit = c->L.nsplit_i8;
     ai.ng = g.ng; ai.rps = c->L.rows_per_split_i8;
+    if (std::getenv("LFD_I8_TIMING")) {  // diagnostics: role wait cycles
+      static long long* buf = nullptr;
+      if (!buf) cudaMallocManaged(&buf, 8 * 1024 * sizeof(long long));
+      cudaStreamSynchronize(c->stream);
+      for (int i = 0; i < 8 * 1024; ++i) buf[i] = 0;
+      ai.dbgbuf = buf;
+    }
     LFD_TRY(launch(c, LFD_K_NL_PROJ, "k_gemm1_i8", [&] { return lfd::launch_gemm1_i8(ai, c->stream); }));
+    if (ai.dbgbuf) {
+      cudaStreamSynchronize(c->stream);
+      double s5[5] = {0, 0, 0, 0, 0};
+      for (int b = 0; b < ai.nsplit; ++b)
+        for (int k = 0; k < 5; ++k) s5[k] += (double)ai.dbgbuf[b * 8 + k];
+      std::fprintf(stderr, "g1 timing (avg cycles per CTA): mma loop %.0f  mma-wait-B %.0f  mma-wait-A %.0f  "
+                   "worker-wait-psi %.0f  worker-wait-afree %.0f (per warp)\n", s5[2] / ai.nsplit, s5[0] / ai.nsplit,
+                   s5[1] / ai.nsplit, s5[3] / ai.nsplit / 16, s5[4] / ai.nsplit / 16);
+    }
     c->colE_valid = false;
     nsplit = c->L.nsplit_i8;
   } else {

@@ -100,18 +100,30 @@ __device__ __forceinline__ void digits_i64(const double v[4], double sc, uint32_
   constexpr double kM = 6755399441055744.0;
   constexpr long long kMb = 0x4338000000000000LL;
   constexpr long long kC = 64LL * ((1LL << 42) - 1) / 127;
-  long long Y[4];
+  // per value: the 4 low fields spread into the bytes of one word, the 2 high fields into another, each
+  // byte u -> u - 64 (mod 256); then 4 x 4 byte transposes (PRMT) give the digit words
+  uint32_t sq[4], tq[4];
 #pragma unroll
-  for (int q = 0; q < 4; ++q) Y[q] = (__double_as_longlong(fma(v[q], sc, kM)) - kMb) + kC;
-#pragma unroll
-  for (int i = 0; i < kI8S; ++i) {
-    const int k = 6 - 1 - i;  // digit i + 1 (most significant first) <-> field k
-    uint32_t w = 0;
-#pragma unroll
-    for (int q = 0; q < 4; ++q)  // field k (the top field may be 128: not masked to 7 bits), minus 64
-      w |= ((((uint32_t)(Y[q] >> (7 * k)) & (k == 5 ? 0xffu : 0x7fu)) + 192u) & 0xffu) << (8 * q);
-    out[i] = w;
+  for (int q = 0; q < 4; ++q) {
+    const long long Y = (__double_as_longlong(fma(v[q], sc, kM)) - kMb) + kC;
+    const uint32_t lo = (uint32_t)Y, hi = (uint32_t)(Y >> 32);
+    uint32_t s4 = (lo & 0x7fu) | ((lo << 1) & 0x7f00u) | ((lo << 2) & 0x7f0000u) | ((lo << 3) & 0x7f000000u);
+    s4 = (s4 ^ 0x40404040u) | ((~s4 & 0x40404040u) << 1);  // bytewise u - 64 for u in [0, 127]
+    uint32_t f4 = __funnelshift_r(lo, hi, 28) & 0x7fu;
+    f4 = (f4 ^ 0x40u) | ((~f4 & 0x40u) << 1);
+    const uint32_t f5 = ((hi >> 3) + 192u) & 0xffu;  // top field, may be 128
+    sq[q] = s4;
+    tq[q] = f4 | (f5 << 8);
   }
+  const uint32_t a = __byte_perm(sq[0], sq[1], 0x5140), b = __byte_perm(sq[0], sq[1], 0x7362);
+  const uint32_t c = __byte_perm(sq[2], sq[3], 0x5140), d = __byte_perm(sq[2], sq[3], 0x7362);
+  const uint32_t e = __byte_perm(tq[0], tq[1], 0x5140), f = __byte_perm(tq[2], tq[3], 0x5140);
+  out[0] = __byte_perm(e, f, 0x7632);  // digit 1 = field 5
+  out[1] = __byte_perm(e, f, 0x5410);  // field 4
+  out[2] = __byte_perm(b, d, 0x7632);  // field 3
+  out[3] = __byte_perm(b, d, 0x5410);  // field 2
+  out[4] = __byte_perm(a, c, 0x7632);  // field 1
+  out[5] = __byte_perm(a, c, 0x5410);  // field 0
 }
 
 // exact int32 -> FP64 without the (low-rate) I2F.F64 conversion: 2^52 + (x + 2^31) built from bits, minus
@@ -187,8 +199,8 @@ __device__ __forceinline__ void umma_i8(uint32_t tmem_d, uint64_t da, uint64_t d
 // A (W^T digits) from TMEM, B (digit tile) from shared memory
 __device__ __forceinline__ void umma_i8_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t accumulate) {
   asm volatile(
-      "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
-      "tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "{\n.reg .pred p, e;\nelect.sync _|e, 0xffffffff;\nsetp.ne.b32 p, %4, 0;\n"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
       "r"(tmem_a), "l"(db), "r"(kI8Idesc), "r"(accumulate));
 }
 __device__ __forceinline__ void tmem_st8(uint32_t taddr, const uint32_t v[8]) {
@@ -196,9 +208,12 @@ __device__ __forceinline__ void tmem_st8(uint32_t taddr, const uint32_t v[8]) {
                "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
                : "memory");
 }
+// issued by one elected lane of the (converged) calling warp
 __device__ __forceinline__ void umma_commit(uint64_t* bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_addr(bar))
-               : "memory");
+  asm volatile(
+      "{\n.reg .pred e;\nelect.sync _|e, 0xffffffff;\n"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n}\n" ::"r"(smem_addr(bar))
+      : "memory");
 }
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
@@ -350,7 +365,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
         }
     }
   } else if (warp == kWMma) {  // MMA issuer: D_d += W_j^T (TMEM) x b_i (smem), i + j = d; one ring slot per d
-    if (lane == 0) {
+    {  // the whole warp runs the loop (warp-uniform values stay in uniform registers); one elected lane issues
       const uint32_t tbase = smem_addr(Tsm);
       long long w_full = 0, w_slot = 0;
       const long long t_start = clock64();
@@ -391,7 +406,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
         }
         umma_commit(&empty[s]);  // the digit tile may be overwritten once these MMAs are done
       }
-      if (p.dbgbuf) {
+      if (p.dbgbuf && lane == 0) {
         p.dbgbuf[blockIdx.x * 8 + 0] = w_full;
         p.dbgbuf[blockIdx.x * 8 + 1] = w_slot;
         p.dbgbuf[blockIdx.x * 8 + 2] = clock64() - t_start;
@@ -506,8 +521,8 @@ constexpr uint32_t kG1Idesc = (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(6
 
 __device__ __forceinline__ void umma_g1_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t accumulate) {
   asm volatile(
-      "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
-      "tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "{\n.reg .pred p, e;\nelect.sync _|e, 0xffffffff;\nsetp.ne.b32 p, %4, 0;\n"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
       "r"(tmem_a), "l"(db), "r"(kG1Idesc), "r"(accumulate));
 }
 __device__ __forceinline__ void tmem_st2(uint32_t taddr, const uint32_t v[2]) {
@@ -627,12 +642,18 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       }
     }
   } else if (warp == kG1WMma) {  // MMA issuer
-    if (lane == 0) {
+    {  // the whole warp runs the loop (warp-uniform values stay in uniform registers); one elected lane issues
       const uint32_t bbase = smem_addr(Bsm);
+      long long w_b = 0, w_a = 0;
+      const long long t0 = clock64();
       for (int g = 0; g < nhalf; ++g) {
         const int b = g >> 2, s = b % kG1Stages, kq = g & 3, ab = g & 1;
+        long long c0 = clock64();
         if (kq == 0) mbar_wait(&bfull[s], (uint32_t)((b / kG1Stages) & 1));
+        long long c1 = clock64();
         mbar_wait(&afull[ab], (uint32_t)((g >> 1) & 1));
+        w_b += c1 - c0;
+        w_a += clock64() - c1;
         tc_fence_after();
         const uint64_t db0 = umma_desc_sw128(bbase + s * kG1BlkB);
 #pragma unroll
@@ -651,6 +672,11 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
         if (kq == 3 || g + 1 == nhalf) umma_commit(&bempty[s]);
       }
       umma_commit(&done);
+      if (p.dbgbuf && lane == 0) {
+        p.dbgbuf[blockIdx.x * 8 + 0] = w_b;
+        p.dbgbuf[blockIdx.x * 8 + 1] = w_a;
+        p.dbgbuf[blockIdx.x * 8 + 2] = clock64() - t0;
+      }
     }
   } else {  // workers: Psi digits into TMEM, column norms; at the end the accumulators into FP64 partials
     const int q = warp & 3, h = warp >> 2;    // lane quarter, row group (8 rows of each half block)
@@ -660,10 +686,13 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
     const bool zc = E == 0;                   // an all-zero orbital (or none): zero digits
     const double sc41 = zc ? 0.0 : ldexp(1.0, 41 - (E - 1022));  // x 2^41 / tau_s: |v sc41| < 2^41
     double nrm = 0.0;
+    long long w_p = 0, w_f = 0;
     const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
     for (int g = 0; g < nhalf; ++g) {
       const int s = g % kG1PsiSlots, ab = g & 1;
+      long long c2 = clock64();
       mbar_wait(&pfull[s], (uint32_t)((g / kG1PsiSlots) & 1));
+      w_p += clock64() - c2;
       const long long ra = r0 + (long long)g * kG1Half;
       const double2* P = reinterpret_cast<const double2*>(Psm + s * kG1PsiB) + sIdx;
       // each lane digitises its own component only (even lane m = 2s: Re, odd lane: Im) of its 4 rows
@@ -696,7 +725,9 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(&pempty[s]);  // this warp is done with the Psi rows
+      long long c3 = clock64();
       if (g >= 2) mbar_wait(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));  // MMAs of block g - 2 are done with it
+      w_f += clock64() - c3;
       tc_fence_after();
 #pragma unroll
       for (int i = 0; i < kI8S; ++i) tmem_st2(trow + ab * kG1ABuf + i * 8 + 2 * h, dg[i]);
@@ -704,6 +735,10 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&afull[ab]);
+    }
+    if (p.dbgbuf && lane == 0) {
+      atomicAdd((unsigned long long*)&p.dbgbuf[blockIdx.x * 8 + 3], (unsigned long long)w_p);
+      atomicAdd((unsigned long long*)&p.dbgbuf[blockIdx.x * 8 + 4], (unsigned long long)w_f);
     }
     // column norms: Re^2 (even lane) + Im^2 (odd lane), then a fixed-order sum over the 4 row groups
     nrm += __shfl_xor_sync(0xffffffffu, nrm, 1);
