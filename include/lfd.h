@@ -85,9 +85,10 @@ typedef struct {
  * O(nproj x norb) -- the split reduction, the Gram matrix, n_s, the carry, the energies -- in FP64. Results
  * agree with the FP64 path to single-precision roundoff (DESIGN.md §4 states the tolerance). */
 #define LFD_FLAG_SP 4
-/* lfd_config.flags: run the nonlocal GEMM-2 (Psi <- Psi diag(n) + B C'') as complex FP64 DMMA
- * (mma.sync m8n8k4) instead of the default for FP64 contexts with nproj <= 64 and norb <= 64: the same
- * product with FP64 accuracy on the tcgen05 int8 tensor cores -- B and C'' split exactly into 6 int8
+/* lfd_config.flags: run the nonlocal GEMMs (C = dV B^H Psi; Psi <- Psi diag(n) + B C'') as
+ * complex FP64 DMMA (mma.sync m8n8k4) instead of the default for FP64 contexts with nproj <= 64,
+ * norb <= 64 and >= 65,536 points per domain: the same products with FP64 accuracy on the tcgen05 int8
+ * tensor cores -- B and C'' split exactly into 6 int8
  * digits each with power-of-two row / column scales, the 21 digit-pair products accumulated exactly in
  * int32 in tensor memory, recombined in FP64 (relative error of the product ~3e-12, i.e. ~1e-15 of Psi
  * per factor since the update is O(Delta Delta_sci / 2) of Psi). See lfd_nl_path(). */

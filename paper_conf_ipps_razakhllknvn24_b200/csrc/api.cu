@@ -83,10 +83,15 @@ lfd_status validate(const lfd_config* c, std::string& why) {
 
 // GEMM-2 on the tcgen05 int8 tensor cores with FP64 accuracy (nl_i8.cu): the default for FP64 contexts with
 // nproj, norb <= 64; LFD_FLAG_NL_DMMA (or env LFD_NL_I8=0, an A/B knob) selects the DMMA kernels.
+// Small grids (< 64K points per domain, e.g. C1 / C3) stay on DMMA by default: there the int8 kernels' per-CTA
+// set-up (C'' digits, TMEM allocation, the exponent handshake) is not amortised (C1: 0.084 vs 0.058 ms/step).
+// env LFD_NL_I8=1 forces the int8 path wherever it is supported (tests), 0 disables it.
 bool use_i8(const lfd_config* c) {
   bool on = (c->flags & (LFD_FLAG_NL_DMMA | LFD_FLAG_SP)) == 0;
-  if (const char* v = std::getenv("LFD_NL_I8")) on = on && std::atoi(v) != 0;
-  return on && lfd::gemm2_i8_supported(c->nproj, c->norb);
+  const long long ng = (long long)c->nx * c->ny * c->nz;
+  bool want = ng >= 65536;
+  if (const char* v = std::getenv("LFD_NL_I8")) want = std::atoi(v) != 0;
+  return on && want && lfd::gemm2_i8_supported(c->nproj, c->norb);
 }
 
 Geometry geometry(const lfd_config* c) {

@@ -31,6 +31,12 @@ def _ctx(w, x, flags=0):
     return ctx, psi
 
 
+@pytest.fixture(autouse=True)
+def force_i8(monkeypatch):
+    """the parity shapes are small (< 64K points): force the int8 path where it is supported"""
+    monkeypatch.setenv("LFD_NL_I8", "1")
+
+
 @pytest.mark.parametrize("name,flags,path", [("P0", 0, 1), ("P0", FLAG_DMMA, 0), ("P3", 0, 0), ("C1", 0, 1),
                                              ("P1", 0, 1)])
 def test_nl_path_selection(name, flags, path):
@@ -39,6 +45,18 @@ def test_nl_path_selection(name, flags, path):
     x = make_inputs(w, seed=1)
     ctx, _ = _ctx(w, x, flags)
     assert lfd.lfd_nl_path(ctx.ctx) == path  # P3 has 65 projectors: the DMMA kernels
+    ctx.close()
+
+
+@pytest.mark.parametrize("name,path", [("C1", 0), ("C2", 1)])
+def test_nl_path_default_by_grid_size(name, path, monkeypatch):
+    """default: int8 path from 64K points per domain (C2), DMMA below (C1: set-up not amortised)"""
+    from paper_conf_ipps_razakhllknvn24_b200 import lfd
+    monkeypatch.delenv("LFD_NL_I8")
+    w = workload(name)
+    x = make_inputs(w, seed=1)
+    ctx, _ = _ctx(w, x)
+    assert lfd.lfd_nl_path(ctx.ctx) == path
     ctx.close()
 
 

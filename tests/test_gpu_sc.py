@@ -84,6 +84,17 @@ def test_sc_parity(name, steps, flags, n_corr):
     assert_sc_parity(_gpu(w, x, steps, flags, n_corr), _ref(w, x, steps, flags, n_corr))
 
 
+@pytest.mark.parametrize("name,n_corr", [("P0", 1), ("C3", 2)])
+def test_sc_parity_int8_gemms(name, n_corr, monkeypatch):
+    """the self-consistent step with both nonlocal GEMMs on the int8-digit tensor-core path (forced on these
+    small grids): the out-of-place first factor S = N(Psi(t_n)), the exponent handshake across sweeps"""
+    monkeypatch.setenv("LFD_NL_I8", "1")
+    w = workload(name).with_(vnoise=0.02) if name == "C3" else workload(name)
+    x = make_inputs(w, seed=63)
+    steps = 2 if name == "C3" else 12
+    assert_sc_parity(_gpu(w, x, steps, ALL, n_corr), _ref(w, x, steps, ALL, n_corr))
+
+
 def test_sc_parity_c3_eight_domains():
     """C3: 8 domains of 24^3 tiling the 48^3 global grid of the 2x2x2 supercell (v_H couples them)."""
     w = workload("C3").with_(vnoise=0.02)
