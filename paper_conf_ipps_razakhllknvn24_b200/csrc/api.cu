@@ -522,6 +522,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
     ai.part = a1.part; ai.norms = a1.norms;
     ai.ndom = g.ndom; ai.nproj = g.nproj; ai.norb = g.norb; ai.nsplit = c->L.nsplit_i8;
     ai.ng = g.ng; ai.rps = c->L.rows_per_split_i8;
+    if (const char* v = std::getenv("LFD_I8_DBG1")) ai.dbg = std::atoi(v);
     if (std::getenv("LFD_I8_TIMING")) {  // diagnostics: role wait cycles
       static long long* buf = nullptr;
       if (!buf) cudaMallocManaged(&buf, 8 * 1024 * sizeof(long long));

@@ -190,6 +190,7 @@ struct Gemm1I8Args {
   int ndom, nproj, norb, nsplit;
   long long ng, rps;
   long long* dbgbuf = nullptr;  // diagnostics only (env LFD_I8_TIMING): per-CTA wait cycles of each role
+  int dbg = 0;                  // diagnostics only (env LFD_I8_DBG1): 1 one pair, 4 no TMEM stores, 8 no digits
 };
 size_t gemm1_i8_bytes(int ndom, long long ng);
 long long gemm1_i8_rows_per_split(long long ng, int ndom, int num_sms);
