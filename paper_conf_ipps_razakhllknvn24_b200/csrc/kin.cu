@@ -471,7 +471,7 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
   // GEMM-1 that follows (its per-orbital power-of-two scale; nl_i8.cu) -- integer max on the high words
   int me = 0;
   auto trk = [&](double2 w) {
-    me = max(me, max(__double2hiint(w.x) & 0x7ff00000, __double2hiint(w.y) & 0x7ff00000));
+    me = __vimax3_s32(me, __double2hiint(w.x) & 0x7ff00000, __double2hiint(w.y) & 0x7ff00000);
     return w;
   };
   auto put0 = [&](int y, double2 f, double2 v) {
