@@ -318,7 +318,7 @@ __global__ void __launch_bounds__(kDensThreads) k_density_tma(Geometry g, DensAr
 // mbarriers; the own line y+1 stays resident for the next step. kSub lanes per point split the orbitals
 // and the 7 per-point sums are shuffle reductions with the occupation weights (kept in shared memory).
 // ------------------------------------------------------------------------------------------------
-constexpr int kYOwn = 4, kYXp = 3;  // ring depths (lines); the own line y+1 stays resident for the y links
+constexpr int kYOwn = 6, kYXp = 3;  // ring depths (lines); the own line y+1 stays resident for the y links
 constexpr int kYMaxThreads = 512;  // up to 60 points x kSub + the producer warp
 
 struct DensMaps {
@@ -444,11 +444,14 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
         mbar_expect_tx(&xfull[s], (uint32_t)(zc * norb * (int)sizeof(C)));
         tma_3d(xp_slot(s), &mp.seg, 0, z0, rowxn + y0 + k, &xfull[s]);
       };
-      issue_own(0);
-      if (nown > 1) issue_own(1);
+      // keep the rings full: kYOwn own lines and kYXp x+1 lines in flight (line k + depth reuses the slot
+      // the consumers release after step k)
+      for (int k = 0; k < kYOwn && k < nown; ++k) issue_own(k);
+      if (has_xn)
+        for (int k = 0; k < kYXp && k < ycnt; ++k) issue_xp(k);
       for (int k = 0; k < ycnt; ++k) {
-        if (has_xn) issue_xp(k);
-        if (k + 2 < nown) issue_own(k + 2);
+        if (k + kYOwn < nown) issue_own(k + kYOwn);
+        if (has_xn && k + kYXp < ycnt) issue_xp(k + kYXp);
       }
     }
     return;

@@ -165,7 +165,7 @@ struct Gemm2Args {
   // int8-digit tensor-core path (nl_i8.cu): B's digit tiles and row scales from launch_bslice_i8, or nullptr
   const int8_t* bsl = nullptr;
   const double* bsig = nullptr;
-  int dbg = 0;  // diagnostics only (env LFD_I8_DBG): 1 = one digit pair per tile, 2 = no epilogue math
+  int dbg = 0;  // diagnostics only (env LFD_I8_DBG): 2 = no epilogue math
   long long* dbgbuf = nullptr;  // diagnostics only (env LFD_I8_TIMING): per-CTA wait cycles of each role
 };
 cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st);

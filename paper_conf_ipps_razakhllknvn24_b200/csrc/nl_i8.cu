@@ -392,7 +392,6 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
           for (int i = 1; i <= kI8S; ++i) {
             const int j = d - i;
             if (j < 1 || j > kI8S) continue;
-            if ((p.dbg & 1) && d > 2) continue;
 #pragma unroll
             for (int kk = 0; kk < kI8K / 32; ++kk) {
               // descriptor arithmetic is linear in the (>> 4) start address: one add per MMA (the issuing
@@ -664,7 +663,6 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
             const int j = d - i;
             if (j < 1 || j > kI8S) continue;
             const bool first = (g == 0) && (i == (d - 1 < kI8S ? 1 : d - kI8S));
-            if ((p.dbg & 1) && !first) continue;  // diagnostics: one digit pair per diagonal
             umma_g1_ts(acc, tmem + ab * kG1ABuf + (j - 1) * 8,
                        db0 + (uint64_t)(((i - 1) * kG1SliceB + kq * 32) >> 4), first ? 0u : 1u);
           }
@@ -712,12 +710,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
         }
       }
       uint32_t own[kI8S];
-      if (p.dbg & 8) {  // diagnostics: no digit arithmetic
-#pragma unroll
-        for (int i = 0; i < kI8S; ++i) own[i] = __double2loint(v[i & 3]);
-      } else {
-        digits_i64(v, sc41, own);
-      }
+      digits_i64(v, sc41, own);
       uint32_t dg[kI8S][2];
 #pragma unroll
       for (int i = 0; i < kI8S; ++i) {
@@ -735,11 +728,9 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       if (g >= 2) mbar_wait(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));  // MMAs of block g - 2 are done with it
       w_f += clock64() - c3;
       tc_fence_after();
-      if (!(p.dbg & 4)) {  // (diagnostics: skip the TMEM stores)
 #pragma unroll
-        for (int i = 0; i < kI8S; ++i) tmem_st2(trow + ab * kG1ABuf + i * 8 + 2 * h, dg[i]);
-        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
-      }
+      for (int i = 0; i < kI8S; ++i) tmem_st2(trow + ab * kG1ABuf + i * 8 + 2 * h, dg[i]);
+      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&afull[ab]);
