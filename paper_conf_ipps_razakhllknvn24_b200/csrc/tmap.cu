@@ -17,6 +17,7 @@ bool pdl_enabled() {
 }
 
 void pdl_suspend(bool s) { g_pdl_suspended = s; }
+bool pdl_suspended() { return g_pdl_suspended; }
 
 cudaError_t encode_tmap_f64(CUtensorMap* out, int rank, const void* base, const uint64_t* dims,
                             const uint64_t* strides_bytes, const uint32_t* box) {
