@@ -568,6 +568,14 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
     LFD_TRY(launch(c, LFD_K_NL_REDUCE, "k_reduce", [&] { return lfd::launch_reduce(r, c->stream); }));
     return gemm2(c, out);
   }
+  static const bool fused = [] {
+    const char* v = std::getenv("LFD_REDUCE_FUSED");
+    return v && std::atoi(v) != 0;
+  }();
+  if (!merged && fused)  // split reduction, n_s and C'' in one kernel (A/B knob LFD_REDUCE_FUSED=1)
+    return launch(c, LFD_K_NL_REDUCE, "k_reduce_norm", [&] {
+             return lfd::launch_reduce_norm(r, c->at<double2>(c->L.G), c->at<double>(c->L.nfac), c->stream);
+           }) == LFD_OK ? gemm2(c, out) : LFD_ECUDA;
   LFD_TRY(launch(c, LFD_K_NL_REDUCE, "k_reduce", [&] { return lfd::launch_reduce(r, c->stream); }));
   if (merged)
     LFD_TRY(launch(c, LFD_K_NL_NORM, "k_nlmerge", [&] {

@@ -473,6 +473,102 @@ __global__ void __launch_bounds__(256) k_nlnorm(int nproj, int norb, double eps2
   }
 }
 
+// k_reduce + k_nlnorm for the common factor (real D, no merge), one block per (orbital s, domain): the
+// fixed-order split reduction of column s (DC = dV D C, its norm s_s), then n_s from the Gram closed form
+// and C''_s = -i eps DC_s n_s -- one launch instead of two.
+__global__ void __launch_bounds__(256) k_reduce_norm(ReduceArgs p, const double2* __restrict__ G,
+                                                     double* __restrict__ nfac) {
+  pdl_wait();
+  pdl_trigger();
+  extern __shared__ double2 dcs[];  // DC[:, col]
+  __shared__ double2 part4[4][64];
+  __shared__ double wq[8];
+  const int dom = blockIdx.y, col = blockIdx.x;
+  const int nproj = p.mrows, norb = p.ncols;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const long long per_dom = (long long)nproj * norb;
+  const double2* src = p.part + (long long)dom * p.nsplit * per_dom + col;
+  // 1. split sums: thread (g = tid / 64, u = tid % 64 + 64 k) sums splits g, g + 4, ... in order
+  for (int u0 = 0; u0 < nproj; u0 += 64) {
+    const int u = u0 + (threadIdx.x & 63), g = threadIdx.x >> 6;
+    double sr = 0.0, si = 0.0;
+    if (u < nproj) {
+      const double2* su = src + (long long)u * norb;
+#pragma unroll 8
+      for (int sp = g; sp < p.nsplit; sp += 4) {  // (loads independent: unrolled so they are in flight together)
+        const double2 v = __ldg(su + (long long)sp * per_dom);
+        sr += v.x;
+        si += v.y;
+      }
+    }
+    part4[g][threadIdx.x & 63] = make_double2(sr, si);
+    __syncthreads();
+    if (threadIdx.x < 64 && u < nproj) {
+      const double tr = (part4[0][threadIdx.x].x + part4[1][threadIdx.x].x) + (part4[2][threadIdx.x].x + part4[3][threadIdx.x].x);
+      const double ti = (part4[0][threadIdx.x].y + part4[1][threadIdx.x].y) + (part4[2][threadIdx.x].y + part4[3][threadIdx.x].y);
+      const double f = p.scale * p.D[(long long)dom * nproj + u];
+      const double2 o = make_double2(tr * f, ti * f);
+      dcs[u] = o;
+      p.out[(long long)dom * per_dom + (long long)u * norb + col] = o;
+    }
+    __syncthreads();
+  }
+  // column norm s_s (fixed order over the splits)
+  if (warp == 0) {
+    double a = 0.0;
+    for (int sp = lane; sp < p.nsplit; sp += 32) a += p.normp[((long long)dom * p.nsplit + sp) * norb + col];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
+    if (lane == 0) {
+      a *= p.scale;
+      p.s[(long long)dom * norb + col] = a;
+      wq[7] = a;  // (read by thread 0 after the barrier below)
+    }
+  }
+  // 2. n_s = sqrt(s_s / (s_s + eps^2 Re[(DC)_s^H G (DC)_s]))
+  const double2* Gd = G + (long long)dom * nproj * nproj;
+  double q = 0.0;
+  for (int u = warp; u < nproj; u += 8) {
+    const double2* Gu = Gd + (long long)u * nproj;
+    double tr = 0.0, ti = 0.0;
+    for (int v = lane; v < nproj; v += 32) {
+      const double2 gv = Gu[v], c = dcs[v];
+      tr = fma(gv.x, c.x, fma(-gv.y, c.y, tr));
+      ti = fma(gv.x, c.y, fma(gv.y, c.x, ti));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      tr += __shfl_xor_sync(0xffffffffu, tr, o);
+      ti += __shfl_xor_sync(0xffffffffu, ti, o);
+    }
+    const double2 cu = dcs[u];
+    q = fma(cu.x, tr, fma(cu.y, ti, q));
+  }
+  __shared__ double wq2[8];
+  if (lane == 0) wq2[warp] = q;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double tq = 0.0;
+    for (int w = 0; w < 8; ++w) tq += wq2[w];
+    const double sv = wq[7];
+    const double n = sqrt(sv / (sv + p.eps * p.eps * tq));
+    nfac[(long long)dom * norb + col] = n;
+    wq[0] = n;
+  }
+  __syncthreads();
+  const double n = wq[0];  // C'' = -i eps DC n
+  for (int u = threadIdx.x; u < nproj; u += blockDim.x) {
+    const double2 o = dcs[u];
+    p.cprime[((long long)dom * nproj + u) * norb + col] = make_double2(p.eps * o.y * n, -p.eps * o.x * n);
+  }
+}
+
+cudaError_t launch_reduce_norm(const ReduceArgs& a, const double2* G, double* nfac, cudaStream_t st) {
+  dim3 grid(a.ncols, a.ndom);
+  launch_k(k_reduce_norm, grid, 256, a.mrows * sizeof(double2), st, a, G, nfac);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_nlnorm(int ndom, int nproj, int norb, double eps, const double2* G, const double2* DC,
                           const double* s, double* nfac, double2* Cp, cudaStream_t st) {
   dim3 grid(norb, ndom);
