@@ -144,6 +144,15 @@ __device__ __forceinline__ double pow2mul(double a, double b) {
   return (ea == 0 || eb == 0 || e <= 0) ? 0.0 : __hiloint2double(e << 20, 0);
 }
 
+// x * a * b for powers of two a, b (or zeros) and x = 0 or a normal number whose product stays normal: an
+// integer add on the exponent field instead of FP64 multiplies (the epilogue is FP64-pipe bound)
+__device__ __forceinline__ double scale_pow2(double x, double a, double b) {
+  const int ea = (__double2hiint(a) >> 20) & 0x7ff, eb = (__double2hiint(b) >> 20) & 0x7ff;
+  const int hx = __double2hiint(x);
+  const bool zero = ea == 0 || eb == 0 || (hx & 0x7fffffff) == 0;  // (x = 0: low word 0 too, it is an exact sum)
+  return zero ? 0.0 : __hiloint2double(hx + ((ea + eb - 2046) << 20), __double2loint(x));
+}
+
 __device__ __forceinline__ int row_exponent(double mx) {
   int e = 0;
   frexp(mx, &e);  // mx = m 2^e, m in [0.5, 1): mx < 2^e
@@ -465,7 +474,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
 #pragma unroll
         for (int c = 0; c < kI8Rows; ++c) {
           if (!nvalid || c >= nc || (p.dbg & 2)) continue;
-          pout[(r0 + c) * ld] = fma(nf, ps[c * ld], pow2mul(sg[c], tau) * fa[c]);
+          pout[(r0 + c) * ld] = fma(nf, ps[c * ld], scale_pow2(fa[c], sg[c], tau));
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&pempty[s]);
