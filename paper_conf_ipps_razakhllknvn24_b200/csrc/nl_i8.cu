@@ -128,6 +128,10 @@ __device__ __forceinline__ void digits_i64(const double v[4], double sc, uint32_
 
 // exact int32 -> FP64 without the (low-rate) I2F.F64 conversion: 2^52 + (x + 2^31) built from bits, minus
 // 2^52 + 2^31 (one full-rate DADD)
+constexpr double kI2dM = 4503601774854144.0;  // 2^52 + 2^31
+__device__ __forceinline__ double i2d_raw(int32_t x) {  // 2^52 + 2^31 + x (exact), no subtraction
+  return __hiloint2double(0x43300000, (int)((uint32_t)x ^ 0x80000000u));
+}
 __device__ __forceinline__ double i2d(int32_t x) {
   return __hiloint2double(0x43300000, (int)((uint32_t)x ^ 0x80000000u)) - 4503601774854144.0;
 }
@@ -460,8 +464,13 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
           mbar_arrive(&dempty[s1]);
         }
         const double wd = ldexp(1.0, -14 * dp - 7);
+        if (dp == 0) {  // fa = (m - M) wd in one fma: m = M + x built from bits, exact result x wd
 #pragma unroll
-        for (int c = 0; c < kI8Rows; ++c) fa[c] = fma(i2d(a0[c] * 128 + a1[c]), wd, fa[c]);
+          for (int c = 0; c < kI8Rows; ++c) fa[c] = fma(i2d_raw(a0[c] * 128 + a1[c]), wd, -kI2dM * wd);
+        } else {
+#pragma unroll
+          for (int c = 0; c < kI8Rows; ++c) fa[c] = fma(i2d(a0[c] * 128 + a1[c]), wd, fa[c]);
+        }
       }
       // the warp's staged Psi sub-tile (rows 16 h .. 16 h + 15 of the tile)
       {
