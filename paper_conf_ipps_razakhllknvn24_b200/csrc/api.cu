@@ -451,6 +451,7 @@ lfd_status gemm2(lfd_ctx* c, double2* out = nullptr) {
     a2.bsl = c->at<int8_t>(c->L.bsl);
     a2.bsig = c->at<double>(c->L.bsig);
     if (const char* v = std::getenv("LFD_I8_DBG")) a2.dbg = std::atoi(v);
+    if (const char* v = std::getenv("LFD_EARLY_PDL")) a2.early = std::atoi(v);
     if (std::getenv("LFD_I8_TIMING")) {  // diagnostics: role wait cycles, printed per call (one domain)
       static long long* buf = nullptr;
       if (!buf) cudaMallocManaged(&buf, 8 * 1024 * sizeof(long long));
@@ -532,6 +533,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
     ai.ndom = g.ndom; ai.nproj = g.nproj; ai.norb = g.norb; ai.nsplit = c->L.nsplit_i8;
     ai.ng = g.ng; ai.rps = c->L.rows_per_split_i8;
     if (const char* v = std::getenv("LFD_I8_DBG1")) ai.dbg = std::atoi(v);
+    if (const char* v = std::getenv("LFD_EARLY_PDL")) ai.early = std::atoi(v);
     if (std::getenv("LFD_I8_TIMING")) {  // diagnostics: role wait cycles
       static long long* buf = nullptr;
       if (!buf) cudaMallocManaged(&buf, 8 * 1024 * sizeof(long long));

@@ -168,6 +168,7 @@ struct Gemm2Args {
   // int8-digit tensor-core path (nl_i8.cu): B's digit tiles and row scales from launch_bslice_i8, or nullptr
   const int8_t* bsl = nullptr;
   const double* bsig = nullptr;
+  int early = 1;  // PDL: set-up and the constant-digit loads before griddepcontrol.wait (env LFD_EARLY_PDL=0: off)
   int dbg = 0;  // diagnostics only (env LFD_I8_DBG): 2 = no epilogue math
   long long* dbgbuf = nullptr;  // diagnostics only (env LFD_I8_TIMING): per-CTA wait cycles of each role
 };
@@ -192,6 +193,7 @@ struct Gemm1I8Args {
   double* norms;        // [dom][nsplit][norb]
   int ndom, nproj, norb, nsplit;
   long long ng, rps;
+  int early = 1;  // as Gemm2Args::early
   long long* dbgbuf = nullptr;  // diagnostics only (env LFD_I8_TIMING): per-CTA wait cycles of each role
   int dbg = 0;                  // diagnostics only (env LFD_I8_DBG1): 1 one pair, 4 no TMEM stores, 8 no digits
 };

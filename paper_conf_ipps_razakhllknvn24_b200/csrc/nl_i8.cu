@@ -255,7 +255,9 @@ __device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.
 // grid (CTAs per domain, ndom); CTA b of a domain takes tiles b, b + gridDim.x, ...
 template <bool kOut>
 __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
-  pdl_wait();
+  // programmatic dependent launch: the set-up below (TMEM, barriers) and the digit producer (B's digits are
+  // constant since lfd_init) overlap the previous kernel; every other warp waits for it (C'', n, Psi)
+  if (!p.early) pdl_wait();
   pdl_trigger();
   extern __shared__ __align__(1024) unsigned char dsm_raw[];
   // SWIZZLE_128B images need 1024-byte aligned shared addresses
@@ -292,6 +294,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
   const uint32_t tacc = tmem + kI8WCols;  // accumulator slot columns
+  if (warp != kWDig) pdl_wait();
 
   if (warp < kI8EpiWarps) {
     // W^T digits from C'' (staged by one bulk copy) into TMEM: thread (warp w, lane) owns row
@@ -600,7 +603,9 @@ __global__ void __launch_bounds__(256) k_bslice1_i8(const double2* __restrict__ 
 
 // grid (splits, ndom); CTA = one split of rps rows (a multiple of 64)
 __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
-  pdl_wait();
+  // programmatic dependent launch: set-up and the first B-digit blocks (constant since lfd_init) overlap the
+  // previous kernel; the Psi loads and everything reading colE / writing the partials wait for it
+  if (!p.early) pdl_wait();
   pdl_trigger();
   extern __shared__ __align__(1024) unsigned char dsm_raw[];
   unsigned char* dsm = dsm_raw + ((1024u - (smem_addr(dsm_raw) & 1023u)) & 1023u);
@@ -643,10 +648,16 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
     if (lane == 0) {
       const int8_t* src = p.bsl1 + (long long)dom * nblk * kG1BlkB;
       const double2* prow = p.psi + (long long)dom * ng * norb;
+      const int nb = (nhalf + 3) >> 2;  // B-digit blocks of this split
+      for (int b = 0; b < kG1Stages && b < nb; ++b) {  // before the dependency wait: B is constant
+        mbar_expect_tx(&bfull[b], kG1BlkB);
+        tma_row(Bsm + b * kG1BlkB, src + (r0 / kG1Rows + b) * kG1BlkB, kG1BlkB, &bfull[b]);
+      }
+      pdl_wait();
       for (int g = 0; g < nhalf; ++g) {
-        if ((g & 3) == 0) {
+        if ((g & 3) == 0 && (g >> 2) >= kG1Stages) {
           const int b = g >> 2, s = b % kG1Stages;
-          if (b >= kG1Stages) mbar_wait(&bempty[s], (uint32_t)(((b / kG1Stages) - 1) & 1));
+          mbar_wait(&bempty[s], (uint32_t)(((b / kG1Stages) - 1) & 1));
           mbar_expect_tx(&bfull[s], kG1BlkB);
           tma_row(Bsm + s * kG1BlkB, src + (r0 / kG1Rows + b) * kG1BlkB, kG1BlkB, &bfull[s]);
         }
@@ -696,6 +707,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       }
     }
   } else {  // workers: Psi digits into TMEM, column norms; at the end the accumulators into FP64 partials
+    pdl_wait();
     const int q = warp & 3, h = warp >> 2;    // lane quarter, row group (8 rows of each half block)
     const int m = 32 * q + lane, sIdx = m >> 1, cm = m & 1;
     const bool sv = sIdx < norb;
