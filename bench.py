@@ -590,6 +590,10 @@ def main():
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "dtype_note": ("complex FP64 throughout; the two projector GEMMs as exact int8 digit products "
+                           "(tcgen05 kind::i8, int32 accumulation in TMEM) recombined in FP64: FP64-accurate, "
+                           "1e-10 parity against the FP64 oracle as every path") if nl_path == 1 else
+                          "complex FP64 throughout (projector GEMMs on the FP64 DMMA pipe)",
             "lfd_steps_per_s": world * w.ndom * args.steps / sec,
             "config": run_config(w, world, args.exact_nl),
             "gpu_launches": int(launches),
