@@ -536,14 +536,19 @@ constexpr int kG1Threads = (kG1Workers + 2) * 32;  // + producer + MMA
 constexpr int kG1WProd = kG1Workers, kG1WMma = kG1Workers + 1;
 constexpr int kG1ABuf = kI8S * 8;                  // TMEM columns of one A buffer (K = 32 bytes per digit)
 constexpr int kG1ACols = 2 * kG1ABuf;              // double-buffered A
-constexpr uint32_t kG1Idesc = (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(64 >> 3) << 17) |
-                              ((uint32_t)(128 >> 4) << 24);  // s32 <- s8 x s8, K-major, N = 64, M = 128
+// s32 <- s8 x s8, both K-major, M = 128, N = n (a multiple of 64 here)
+__host__ __device__ constexpr uint32_t g1_idesc(int n) {
+  return (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+}
+constexpr uint32_t kG1Idesc = g1_idesc(64);
+constexpr int kG1Wide = 3;  // B digits stacked along N per MMA (wide schedule)
 
-__device__ __forceinline__ void umma_g1_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t accumulate) {
+__device__ __forceinline__ void umma_g1_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t accumulate,
+                                           uint32_t idesc = kG1Idesc) {
   asm volatile(
       "{\n.reg .pred p, e;\nelect.sync _|e, 0xffffffff;\nsetp.ne.b32 p, %4, 0;\n"
       "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
-      "r"(tmem_a), "l"(db), "r"(kG1Idesc), "r"(accumulate));
+      "r"(tmem_a), "l"(db), "r"(idesc), "r"(accumulate));
 }
 __device__ __forceinline__ void tmem_st2(uint32_t taddr, const uint32_t v[2]) {
   asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0], {%1,%2};" ::"r"(taddr), "r"(v[0]), "r"(v[1]) : "memory");
@@ -684,6 +689,22 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
         w_a += clock64() - c1;
         tc_fence_after();
         const uint64_t db0 = umma_desc_sw128(bbase + s * kG1BlkB);
+        if (p.wide) {
+          // B's digit slices i .. i + w - 1 are consecutive 64-row SWIZZLE_128B tiles (8 KB each), i.e. one
+          // K-major tile of 64 w rows, and the diagonal accumulators d = i + j .. i + j + w - 1 are consecutive
+          // 64-column TMEM blocks: one MMA of N = 64 w computes the w digit pairs (i .. i + w - 1, j) straight
+          // into their diagonals. The two j = 1 MMAs touch every diagonal first (accumulate = 0 at g = 0).
+#pragma unroll
+          for (int j = 1; j <= kI8S; ++j) {
+#pragma unroll
+            for (int i = 1; i <= kI8S + 1 - j; i += kG1Wide) {
+              const int w = (kI8S + 2 - j - i) < kG1Wide ? (kI8S + 2 - j - i) : kG1Wide;
+              umma_g1_ts(tacc + (i + j - 2) * 64, tmem + ab * kG1ABuf + (j - 1) * 8,
+                         db0 + (uint64_t)(((i - 1) * kG1SliceB + kq * 32) >> 4), (g == 0 && j == 1) ? 0u : 1u,
+                         g1_idesc(64 * w));
+            }
+          }
+        } else
 #pragma unroll
         for (int d = 2; d <= kI8S + 1; ++d) {
           const uint32_t acc = tacc + (d - 2) * 64;
