@@ -545,12 +545,13 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
     LFD_TRY(launch(c, LFD_K_NL_PROJ, "k_gemm1_i8", [&] { return lfd::launch_gemm1_i8(ai, c->stream); }));
     if (ai.dbgbuf) {
       cudaStreamSynchronize(c->stream);
-      double s5[5] = {0, 0, 0, 0, 0};
+      double s5[6] = {0, 0, 0, 0, 0, 0};
       for (int b = 0; b < ai.nsplit; ++b)
-        for (int k = 0; k < 5; ++k) s5[k] += (double)ai.dbgbuf[b * 8 + k];
+        for (int k = 0; k < 6; ++k) s5[k] += (double)ai.dbgbuf[b * 8 + k];
       std::fprintf(stderr, "g1 timing (avg cycles per CTA): mma loop %.0f  mma-wait-B %.0f  mma-wait-A %.0f  "
-                   "worker-wait-psi %.0f  worker-wait-afree %.0f (per warp)\n", s5[2] / ai.nsplit, s5[0] / ai.nsplit,
-                   s5[1] / ai.nsplit, s5[3] / ai.nsplit / 16, s5[4] / ai.nsplit / 16);
+                   "worker-wait-psi %.0f  worker-wait-afree %.0f  worker-tmem-store %.0f (per warp)\n",
+                   s5[2] / ai.nsplit, s5[0] / ai.nsplit, s5[1] / ai.nsplit, s5[3] / ai.nsplit / 16,
+                   s5[4] / ai.nsplit / 16, s5[5] / ai.nsplit / 16);
     }
     c->colE_valid = false;
     nsplit = c->L.nsplit_i8;

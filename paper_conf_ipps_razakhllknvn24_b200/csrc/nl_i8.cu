@@ -541,7 +541,6 @@ __host__ __device__ constexpr uint32_t g1_idesc(int n) {
   return (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
 }
 constexpr uint32_t kG1Idesc = g1_idesc(64);
-constexpr int kG1Wide = 3;  // B digits stacked along N per MMA (wide schedule)
 
 __device__ __forceinline__ void umma_g1_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t accumulate,
                                            uint32_t idesc = kG1Idesc) {
@@ -557,6 +556,21 @@ __device__ __forceinline__ void tmem_st4(uint32_t taddr, const uint32_t v[4]) {
   asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1,%2,%3,%4};" ::"r"(taddr), "r"(v[0]), "r"(v[1]),
                "r"(v[2]), "r"(v[3])
                : "memory");
+}
+
+// The wide-N MMA schedule of one quarter block (see k_gemm1_i8): for each Psi digit j, the B digits
+// i = 1 .. 7 - j in chunks of at most W consecutive slices, one MMA of N = 64 w per chunk
+template <int W>
+__device__ __forceinline__ void g1_wide_mmas(uint32_t tacc, uint32_t ta, uint64_t db0, int kq, bool first) {
+#pragma unroll
+  for (int j = 1; j <= kI8S; ++j) {
+#pragma unroll
+    for (int i = 1; i <= kI8S + 1 - j; i += W) {
+      const int w = (kI8S + 2 - j - i) < W ? (kI8S + 2 - j - i) : W;
+      umma_g1_ts(tacc + (i + j - 2) * 64, ta + (j - 1) * 8, db0 + (uint64_t)(((i - 1) * kG1SliceB + kq * 32) >> 4),
+                 (first && j == 1) ? 0u : 1u, g1_idesc(64 * w));
+    }
+  }
 }
 
 // B's GEMM-1 scales: bexp[dom][u] = max over the domain of the biased exponent of Re / Im B[r][u]
@@ -689,19 +703,24 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
         w_a += clock64() - c1;
         tc_fence_after();
         const uint64_t db0 = umma_desc_sw128(bbase + s * kG1BlkB);
-        if (p.wide) {
+        if (p.wide == 1 || p.wide == 2) {
           // B's digit slices i .. i + w - 1 are consecutive 64-row SWIZZLE_128B tiles (8 KB each), i.e. one
           // K-major tile of 64 w rows, and the diagonal accumulators d = i + j .. i + j + w - 1 are consecutive
           // 64-column TMEM blocks: one MMA of N = 64 w computes the w digit pairs (i .. i + w - 1, j) straight
-          // into their diagonals. The two j = 1 MMAs touch every diagonal first (accumulate = 0 at g = 0).
+          // into their diagonals. The j = 1 MMAs touch every diagonal first (accumulate = 0 at g = 0).
+          // wide 1: w <= 3 (9 MMAs); wide 2: w <= 2 (12 MMAs, consecutive ones mostly on disjoint diagonals)
+          if (p.wide == 1) g1_wide_mmas<3>(tacc, tmem + ab * kG1ABuf, db0, kq, g == 0);
+          else g1_wide_mmas<2>(tacc, tmem + ab * kG1ABuf, db0, kq, g == 0);
+        } else if (p.wide == 3) {
+          // N = 64, round-robin over the diagonals: round r takes the pair (r + 1, d - r - 1) of every
+          // diagonal d >= r + 2, so consecutive MMAs accumulate into different TMEM blocks
 #pragma unroll
-          for (int j = 1; j <= kI8S; ++j) {
+          for (int r = 0; r < kI8S; ++r) {
 #pragma unroll
-            for (int i = 1; i <= kI8S + 1 - j; i += kG1Wide) {
-              const int w = (kI8S + 2 - j - i) < kG1Wide ? (kI8S + 2 - j - i) : kG1Wide;
-              umma_g1_ts(tacc + (i + j - 2) * 64, tmem + ab * kG1ABuf + (j - 1) * 8,
-                         db0 + (uint64_t)(((i - 1) * kG1SliceB + kq * 32) >> 4), (g == 0 && j == 1) ? 0u : 1u,
-                         g1_idesc(64 * w));
+            for (int d = r + 2; d <= kI8S + 1; ++d) {
+              const int i = r + 1, j = d - i;
+              umma_g1_ts(tacc + (d - 2) * 64, tmem + ab * kG1ABuf + (j - 1) * 8,
+                         db0 + (uint64_t)(((i - 1) * kG1SliceB + kq * 32) >> 4), (g == 0 && r == 0) ? 0u : 1u);
             }
           }
         } else
@@ -736,7 +755,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
     const bool zc = E == 0;                   // an all-zero orbital (or none): zero digits
     const double sc41 = zc ? 0.0 : ldexp(1.0, 41 - (E - 1022));  // x 2^41 / tau_s: |v sc41| < 2^41
     double nrm = 0.0;
-    long long w_p = 0, w_f = 0;
+    long long w_p = 0, w_f = 0, w_s = 0;
     const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
     for (int g = 0; g < nhalf; ++g) {
       const int s = g % kG1PsiSlots, ab = g & 1;
@@ -744,22 +763,22 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       mbar_wait(&pfull[s], (uint32_t)((g / kG1PsiSlots) & 1));
       w_p += clock64() - c2;
       const long long ra = r0 + (long long)g * kG1Half;
-      const double2* P = reinterpret_cast<const double2*>(Psm + s * kG1PsiB) + sIdx;
+      // this lane's component of Psi[row][sIdx] (Re for cm = 0, Im for cm = 1): 8-byte loads, 2 norb per row
+      const double* P = reinterpret_cast<const double*>(Psm + s * kG1PsiB) + 2 * sIdx + cm;
       // each lane digitises its own component only (even lane m = 2s: Re, odd lane: Im) of its 4 rows
       // (4h .. 4h + 3 of the quarter block), in integer arithmetic (digits_i64), and the lane pair exchanges
       // them: row 2s of A takes (Re, Im) per grid row, row 2s+1 takes (Im, -Re) (bytewise negated digits:
       // still an exact decomposition)
       double v[4];
+      if (sv && ra + 4 * h + 4 <= r1) {  // all 4 rows present (every quarter block but a split's ragged last)
 #pragma unroll
-      for (int t = 0; t < 4; ++t) {
-        const int rr = 4 * h + t;
-        v[t] = 0.0;
-        if (sv && ra + rr < r1) {
-          const double2 x = P[rr * norb];
-          v[t] = cm ? x.y : x.x;
-          nrm = fma(v[t], v[t], nrm);
-        }
+        for (int t = 0; t < 4; ++t) v[t] = P[(4 * h + t) * 2 * norb];
+      } else {
+#pragma unroll
+        for (int t = 0; t < 4; ++t) v[t] = (sv && ra + 4 * h + t < r1) ? P[(4 * h + t) * 2 * norb] : 0.0;
       }
+#pragma unroll
+      for (int t = 0; t < 4; ++t) nrm = fma(v[t], v[t], nrm);  // absent rows add +0 exactly
       uint32_t own[kI8S];
       digits_i64(v, sc41, own);
       uint32_t dg[kI8S][2];
@@ -779,16 +798,19 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       if (g >= 2) mbar_wait(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));  // MMAs of block g - 2 are done with it
       w_f += clock64() - c3;
       tc_fence_after();
+      const long long c4 = clock64();
 #pragma unroll
       for (int i = 0; i < kI8S; ++i) tmem_st2(trow + ab * kG1ABuf + i * 8 + 2 * h, dg[i]);
       asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
       tc_fence_before();
       __syncwarp();
+      w_s += clock64() - c4;
       if (lane == 0) mbar_arrive(&afull[ab]);
     }
     if (p.dbgbuf && lane == 0) {
       atomicAdd((unsigned long long*)&p.dbgbuf[blockIdx.x * 8 + 3], (unsigned long long)w_p);
       atomicAdd((unsigned long long*)&p.dbgbuf[blockIdx.x * 8 + 4], (unsigned long long)w_f);
+      atomicAdd((unsigned long long*)&p.dbgbuf[blockIdx.x * 8 + 5], (unsigned long long)w_s);
     }
     // column norms: Re^2 (even lane) + Im^2 (odd lane), then a fixed-order sum over the 4 row groups
     nrm += __shfl_xor_sync(0xffffffffu, nrm, 1);
