@@ -558,6 +558,12 @@ __device__ __forceinline__ void tmem_st4(uint32_t taddr, const uint32_t v[4]) {
                : "memory");
 }
 
+template <bool T>
+__device__ __forceinline__ long long tclk() {
+  if constexpr (T) return clock64();
+  else return 0;
+}
+
 // The wide-N MMA schedule of one quarter block (see k_gemm1_i8): for each Psi digit j, the B digits
 // i = 1 .. 7 - j in chunks of at most W consecutive slices, one MMA of N = 64 w per chunk
 template <int W>
@@ -621,6 +627,8 @@ __global__ void __launch_bounds__(256) k_bslice1_i8(const double2* __restrict__ 
 }
 
 // grid (splits, ndom); CTA = one split of rps rows (a multiple of 64)
+// kT: role-wait instrumentation compiled in (LFD_I8_TIMING); the clock reads cost issue slots in the worker loop
+template <bool kT>
 __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   // programmatic dependent launch: set-up and the first B-digit blocks (constant since lfd_init) overlap the
   // previous kernel; the Psi loads and everything reading colE / writing the partials wait for it
@@ -692,15 +700,15 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
     {  // the whole warp runs the loop (warp-uniform values stay in uniform registers); one elected lane issues
       const uint32_t bbase = smem_addr(Bsm);
       long long w_b = 0, w_a = 0;
-      const long long t0 = clock64();
+      const long long t0 = tclk<kT>();
       for (int g = 0; g < nhalf; ++g) {
         const int b = g >> 2, s = b % kG1Stages, kq = g & 3, ab = g & 1;
-        long long c0 = clock64();
+        long long c0 = tclk<kT>();
         if (kq == 0) mbar_wait(&bfull[s], (uint32_t)((b / kG1Stages) & 1));
-        long long c1 = clock64();
+        long long c1 = tclk<kT>();
         mbar_wait(&afull[ab], (uint32_t)((g >> 1) & 1));
         w_b += c1 - c0;
-        w_a += clock64() - c1;
+        w_a += tclk<kT>() - c1;
         tc_fence_after();
         const uint64_t db0 = umma_desc_sw128(bbase + s * kG1BlkB);
         if (p.wide == 1 || p.wide == 2) {
@@ -743,7 +751,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       if (p.dbgbuf && lane == 0) {
         p.dbgbuf[blockIdx.x * 8 + 0] = w_b;
         p.dbgbuf[blockIdx.x * 8 + 1] = w_a;
-        p.dbgbuf[blockIdx.x * 8 + 2] = clock64() - t0;
+        p.dbgbuf[blockIdx.x * 8 + 2] = tclk<kT>() - t0;
       }
     }
   } else {  // workers: Psi digits into TMEM, column norms; at the end the accumulators into FP64 partials
@@ -751,17 +759,18 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
     const int q = warp & 3, h = warp >> 2;    // lane quarter, row group (8 rows of each half block)
     const int m = 32 * q + lane, sIdx = m >> 1, cm = m & 1;
     const bool sv = sIdx < norb;
+    const uint32_t nmask = cm ? 0xffffffffu : 0u;
     const int E = sv ? p.colE[(long long)dom * norb + sIdx] : 0;
     const bool zc = E == 0;                   // an all-zero orbital (or none): zero digits
     const double sc41 = zc ? 0.0 : ldexp(1.0, 41 - (E - 1022));  // x 2^41 / tau_s: |v sc41| < 2^41
     double nrm = 0.0;
     long long w_p = 0, w_f = 0, w_s = 0;
     const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
-    for (int g = 0; g < nhalf; ++g) {
-      const int s = g % kG1PsiSlots, ab = g & 1;
-      long long c2 = clock64();
-      mbar_wait(&pfull[s], (uint32_t)((g / kG1PsiSlots) & 1));
-      w_p += clock64() - c2;
+    for (int g = 0, s = 0, ph = 0; g < nhalf; ++g) {  // s = g % kG1PsiSlots, ph = (g / kG1PsiSlots) & 1
+      const int ab = g & 1;
+      long long c2 = tclk<kT>();
+      mbar_wait(&pfull[s], (uint32_t)ph);
+      w_p += tclk<kT>() - c2;
       const long long ra = r0 + (long long)g * kG1Half;
       // this lane's component of Psi[row][sIdx] (Re for cm = 0, Im for cm = 1): 8-byte loads, 2 norb per row
       const double* P = reinterpret_cast<const double*>(Psm + s * kG1PsiB) + 2 * sIdx + cm;
@@ -788,24 +797,27 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
         const uint32_t other = __shfl_xor_sync(0xffffffffu, mine, 1);
         // bytes t = 0..3 are rows 4h + t; A word w (K bytes 8h + 4w ..) holds rows (2w, 2w+1) as
         // [c'=0, c'=1, c'=0, c'=1]; even lane: c'=0 own (Re), c'=1 other (Im); odd lane: own (Im), -other
-        const uint32_t b = cm ? neg_bytes(other) : other;
+        // odd lane: bytewise -other without predication: bytes b in [-64, 64] -> x = b + 128 in [64, 192],
+        // (x ^ 0xff) + 1 = 256 - x has no carry between bytes, ^ 0x80 gives -b
+        const uint32_t b = (((other ^ 0x80808080u ^ nmask) + (nmask & 0x01010101u)) ^ 0x80808080u);
         dg[i][0] = __byte_perm(mine, b, 0x5140);  // [a0, b0, a1, b1]
         dg[i][1] = __byte_perm(mine, b, 0x7362);  // [a2, b2, a3, b3]
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(&pempty[s]);  // this warp is done with the Psi rows
-      long long c3 = clock64();
+      long long c3 = tclk<kT>();
       if (g >= 2) mbar_wait(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));  // MMAs of block g - 2 are done with it
-      w_f += clock64() - c3;
+      w_f += tclk<kT>() - c3;
       tc_fence_after();
-      const long long c4 = clock64();
+      const long long c4 = tclk<kT>();
 #pragma unroll
       for (int i = 0; i < kI8S; ++i) tmem_st2(trow + ab * kG1ABuf + i * 8 + 2 * h, dg[i]);
       asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
       tc_fence_before();
       __syncwarp();
-      w_s += clock64() - c4;
+      w_s += tclk<kT>() - c4;
       if (lane == 0) mbar_arrive(&afull[ab]);
+      if (++s == kG1PsiSlots) { s = 0; ph ^= 1; }
     }
     if (p.dbgbuf && lane == 0) {
       atomicAdd((unsigned long long*)&p.dbgbuf[blockIdx.x * 8 + 3], (unsigned long long)w_p);
@@ -888,7 +900,8 @@ cudaError_t launch_bslice1_i8(const double2* B, int ndom, int nproj, long long n
 }
 cudaError_t launch_gemm1_i8(const Gemm1I8Args& a, cudaStream_t st) {
   dim3 grid(a.nsplit, a.ndom);
-  launch_k(k_gemm1_i8, grid, kG1Threads, kG1Smem, st, a);
+  if (a.dbgbuf) launch_k(k_gemm1_i8<true>, grid, kG1Threads, kG1Smem, st, a);
+  else launch_k(k_gemm1_i8<false>, grid, kG1Threads, kG1Smem, st, a);
   return cudaGetLastError();
 }
 
@@ -924,7 +937,9 @@ cudaError_t launch_gemm2_i8(const Gemm2Args& a, cudaStream_t st) {
 cudaError_t gemm_i8_set_attributes() {
   cudaError_t e = cudaFuncSetAttribute(k_gemm2_i8<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kI8Smem);
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_gemm1_i8, cudaFuncAttributeMaxDynamicSharedMemorySize, kG1Smem);
+  e = cudaFuncSetAttribute(k_gemm1_i8<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kG1Smem);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_gemm1_i8<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kG1Smem);
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(k_gemm2_i8<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kI8Smem);
 }
