@@ -535,6 +535,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
     if (const char* v = std::getenv("LFD_I8_DBG1")) ai.dbg = std::atoi(v);
     if (const char* v = std::getenv("LFD_EARLY_PDL")) ai.early = std::atoi(v);
     if (const char* v = std::getenv("LFD_G1_WIDE")) ai.wide = std::atoi(v);
+    if (const char* v = std::getenv("LFD_G1_SLEEP")) ai.sleep = std::atoi(v);
     if (std::getenv("LFD_I8_TIMING")) {  // diagnostics: role wait cycles
       static long long* buf = nullptr;
       if (!buf) cudaMallocManaged(&buf, 8 * 1024 * sizeof(long long));

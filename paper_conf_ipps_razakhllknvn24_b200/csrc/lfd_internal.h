@@ -194,8 +194,9 @@ struct Gemm1I8Args {
   int ndom, nproj, norb, nsplit;
   long long ng, rps;
   int early = 1;  // as Gemm2Args::early
-  int wide = 0;   // MMA schedule (env LFD_G1_WIDE): 0 = 21 MMAs of N = 64, diagonal-major; 1 / 2 = B digits
+  int wide = 1;   // MMA schedule (env LFD_G1_WIDE): 0 = 21 MMAs of N = 64, diagonal-major; 1 / 2 = B digits
                   // i .. i+2 / i .. i+1 stacked along N (9 / 12 MMAs); 3 = N = 64 round-robin over diagonals
+  int sleep = 0;  // env LFD_G1_SLEEP=1: the A-buffer handshake waits carry a suspend-time hint
   long long* dbgbuf = nullptr;  // diagnostics only (env LFD_I8_TIMING): per-CTA wait cycles of each role
   int dbg = 0;                  // diagnostics only (env LFD_I8_DBG1): 1 one pair, 4 no TMEM stores, 8 no digits
 };

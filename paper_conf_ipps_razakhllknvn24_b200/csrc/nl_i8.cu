@@ -706,7 +706,8 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
         long long c0 = tclk<kT>();
         if (kq == 0) mbar_wait(&bfull[s], (uint32_t)((b / kG1Stages) & 1));
         long long c1 = tclk<kT>();
-        mbar_wait(&afull[ab], (uint32_t)((g >> 1) & 1));
+        if (p.sleep) mbar_wait_sleep(&afull[ab], (uint32_t)((g >> 1) & 1));
+        else mbar_wait(&afull[ab], (uint32_t)((g >> 1) & 1));
         w_b += c1 - c0;
         w_a += tclk<kT>() - c1;
         tc_fence_after();
@@ -806,7 +807,10 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       __syncwarp();
       if (lane == 0) mbar_arrive(&pempty[s]);  // this warp is done with the Psi rows
       long long c3 = tclk<kT>();
-      if (g >= 2) mbar_wait(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));  // MMAs of block g - 2 are done with it
+      if (g >= 2) {  // MMAs of block g - 2 are done with it
+        if (p.sleep) mbar_wait_sleep(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));
+        else mbar_wait(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));
+      }
       w_f += tclk<kT>() - c3;
       tc_fence_after();
       const long long c4 = tclk<kT>();
