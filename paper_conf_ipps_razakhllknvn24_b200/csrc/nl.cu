@@ -439,6 +439,41 @@ __global__ void __launch_bounds__(256) k_nlnorm(int nproj, int norb, double eps2
   for (int u = threadIdx.x; u < nproj; u += blockDim.x) dcs[u] = Cd[(long long)u * norb + col];
   __syncthreads();
   double q = 0.0;
+  if (nproj <= 64) {  // the warp's (up to) 8 rows with all G loads in flight and the shuffle trees interleaved;
+                      // per row the same fma chain and tree as the loop below (bitwise the same q)
+    double tr[8], ti[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int u = warp + 8 * k;
+      tr[k] = 0.0;
+      ti[k] = 0.0;
+#pragma unroll
+      for (int t = 0; t < 2; ++t) {
+        const int v = lane + 32 * t;
+        if (u < nproj && v < nproj) {
+          const double2 gv = Gd[(long long)u * nproj + v], c = dcs[v];
+          tr[k] = fma(gv.x, c.x, fma(-gv.y, c.y, tr[k]));
+          ti[k] = fma(gv.x, c.y, fma(gv.y, c.x, ti[k]));
+        }
+      }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        tr[k] += __shfl_xor_sync(0xffffffffu, tr[k], o);
+        ti[k] += __shfl_xor_sync(0xffffffffu, ti[k], o);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int u = warp + 8 * k;
+      if (u < nproj) {
+        const double2 cu = dcs[u];
+        q = fma(cu.x, tr[k], fma(cu.y, ti[k], q));
+      }
+    }
+  } else
   for (int u = warp; u < nproj; u += 8) {
     const double2* Gu = Gd + (long long)u * nproj;
     double tr = 0.0, ti = 0.0;
@@ -708,9 +743,45 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
       ti += __shfl_xor_sync(0xffffffffu, ti, o);
     }
   };
-  for (int u = warp; u < nproj; u += 8) {
+  // nproj <= 64: the warp's (up to) 8 rows with all their G loads in flight at once and the 16 shuffle trees
+  // interleaved (per row the same fma chain and tree as gdot: bitwise the same values)
+  auto gdot8 = [&](const double2* v, double (&tr)[8], double (&ti)[8]) {
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int u = warp + 8 * k;
+      tr[k] = 0.0;
+      ti[k] = 0.0;
+#pragma unroll
+      for (int t = 0; t < 2; ++t) {
+        const int w = lane + 32 * t;
+        if (u < nproj && w < nproj) {
+          const double2 gv = Gd[(long long)u * nproj + w], x = v[w];
+          tr[k] = fma(gv.x, x.x, fma(-gv.y, x.y, tr[k]));
+          ti[k] = fma(gv.x, x.y, fma(gv.y, x.x, ti[k]));
+        }
+      }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        tr[k] += __shfl_xor_sync(0xffffffffu, tr[k], o);
+        ti[k] += __shfl_xor_sync(0xffffffffu, ti[k], o);
+      }
+    }
+  };
+  const bool small = nproj <= 64;
+  double gr[8], gi[8];
+  if (small) gdot8(xs, gr, gi);
+  for (int u = warp, k = 0; u < nproj; u += 8, ++k) {
     double tr, ti;
-    gdot(u, xs, tr, ti);
+    if (small) {
+#pragma unroll
+      for (int kk = 0; kk < 8; ++kk)
+        if (kk == k) { tr = gr[kk]; ti = gi[kk]; }
+    } else {
+      gdot(u, xs, tr, ti);
+    }
     if (lane == 0) {
       const double du = Dd[u];
       const double2 d = make_double2(fma(n, dcs[u].x, du * tr), fma(n, dcs[u].y, du * ti));
@@ -728,9 +799,16 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
   // n_s of the next factor from the Gram closed form (as k_nlnorm), on DC_new
   __syncthreads();
   double q = 0.0;
-  for (int u = warp; u < nproj; u += 8) {
+  if (small) gdot8(dcs, gr, gi);
+  for (int u = warp, k = 0; u < nproj; u += 8, ++k) {
     double tr, ti;
-    gdot(u, dcs, tr, ti);
+    if (small) {
+#pragma unroll
+      for (int kk = 0; kk < 8; ++kk)
+        if (kk == k) { tr = gr[kk]; ti = gi[kk]; }
+    } else {
+      gdot(u, dcs, tr, ti);
+    }
     const double2 cu = dcs[u];
     q = fma(cu.x, tr, fma(cu.y, ti, q));  // Re(conj(cu) (G DC)_u)
   }
