@@ -715,6 +715,7 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
   extern __shared__ double2 sh[];  // x[np] | dc[np] (dc is overwritten with DC_new)
   double2* xs = sh;
   double2* dcs = sh + nproj;
+  double* ds = reinterpret_cast<double*>(sh + 2 * nproj);  // D[u], staged with x and dc
   __shared__ double wq[8];
   const int dom = blockIdx.y, col = blockIdx.x;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -724,6 +725,7 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
   for (int u = threadIdx.x; u < nproj; u += blockDim.x) {
     xs[u] = X[cb + (long long)u * norb];
     dcs[u] = DC[cb + (long long)u * norb];
+    ds[u] = Dd[u];
   }
   __syncthreads();
   const double n = nfac[(long long)dom * norb + col];
@@ -783,7 +785,7 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
       gdot(u, xs, tr, ti);
     }
     if (lane == 0) {
-      const double du = Dd[u];
+      const double du = ds[u];
       const double2 d = make_double2(fma(n, dcs[u].x, du * tr), fma(n, dcs[u].y, du * ti));
       DC[cb + (long long)u * norb] = d;
       if (W) {  // exactly unitary factor (D == 1 passed, n == 1): C''_new = W C_new
@@ -833,9 +835,9 @@ cudaError_t launch_nlcarry(int ndom, int nproj, int norb, double eps, const doub
                            const double2* W, cudaStream_t st) {
   dim3 grid(norb, ndom);
   if (with_norm && !W)
-    launch_k(k_nlcarry<true>, grid, 256, 2 * nproj * sizeof(double2), st, nproj, norb, eps, G, D, DC, X, s, nfac, W);
+    launch_k(k_nlcarry<true>, grid, 256, 2 * nproj * sizeof(double2) + nproj * sizeof(double), st, nproj, norb, eps, G, D, DC, X, s, nfac, W);
   else
-    launch_k(k_nlcarry<false>, grid, 256, 2 * nproj * sizeof(double2), st, nproj, norb, eps, G, D, DC, X, s, nfac, W);
+    launch_k(k_nlcarry<false>, grid, 256, 2 * nproj * sizeof(double2) + nproj * sizeof(double), st, nproj, norb, eps, G, D, DC, X, s, nfac, W);
   return cudaGetLastError();
 }
 
