@@ -774,16 +774,7 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
   };
   const bool small = nproj <= 64;
   double gr[8], gi[8];
-  if (small) gdot8(xs, gr, gi);
-  for (int u = warp, k = 0; u < nproj; u += 8, ++k) {
-    double tr, ti;
-    if (small) {
-#pragma unroll
-      for (int kk = 0; kk < 8; ++kk)
-        if (kk == k) { tr = gr[kk]; ti = gi[kk]; }
-    } else {
-      gdot(u, xs, tr, ti);
-    }
+  auto row = [&](int u, double tr, double ti) {
     if (lane == 0) {
       const double du = ds[u];
       const double2 d = make_double2(fma(n, dcs[u].x, du * tr), fma(n, dcs[u].y, du * ti));
@@ -796,23 +787,40 @@ __global__ void __launch_bounds__(256) k_nlcarry(int nproj, int norb, double eps
       }
       dcs[u] = d;  // only this lane reads dcs[u] above
     }
+  };
+  if (small) {  // rows u = warp + 8 k, compile-time k (no register-array selects)
+    gdot8(xs, gr, gi);
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+      if (warp + 8 * k < nproj) row(warp + 8 * k, gr[k], gi[k]);
+  } else {
+    for (int u = warp; u < nproj; u += 8) {
+      double tr, ti;
+      gdot(u, xs, tr, ti);
+      row(u, tr, ti);
+    }
   }
   if (!kNorm) return;
   // n_s of the next factor from the Gram closed form (as k_nlnorm), on DC_new
   __syncthreads();
   double q = 0.0;
-  if (small) gdot8(dcs, gr, gi);
-  for (int u = warp, k = 0; u < nproj; u += 8, ++k) {
-    double tr, ti;
-    if (small) {
+  if (small) {
+    gdot8(dcs, gr, gi);
 #pragma unroll
-      for (int kk = 0; kk < 8; ++kk)
-        if (kk == k) { tr = gr[kk]; ti = gi[kk]; }
-    } else {
-      gdot(u, dcs, tr, ti);
+    for (int k = 0; k < 8; ++k) {
+      const int u = warp + 8 * k;
+      if (u < nproj) {
+        const double2 cu = dcs[u];
+        q = fma(cu.x, gr[k], fma(cu.y, gi[k], q));  // Re(conj(cu) (G DC)_u)
+      }
     }
-    const double2 cu = dcs[u];
-    q = fma(cu.x, tr, fma(cu.y, ti, q));  // Re(conj(cu) (G DC)_u)
+  } else {
+    for (int u = warp; u < nproj; u += 8) {
+      double tr, ti;
+      gdot(u, dcs, tr, ti);
+      const double2 cu = dcs[u];
+      q = fma(cu.x, tr, fma(cu.y, ti, q));  // Re(conj(cu) (G DC)_u)
+    }
   }
   if (lane == 0) wq[warp] = q;
   __syncthreads();
