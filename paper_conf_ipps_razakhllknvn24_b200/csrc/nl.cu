@@ -365,7 +365,18 @@ __global__ void __launch_bounds__(256) k_reduce(ReduceArgs p, int eblocks) {
     double sr = 0.0, si = 0.0;
     if (e < per_dom) {
       const double2* src = p.part + (long long)dom * p.nsplit * per_dom + e;
-      for (int s = sg; s < p.nsplit; s += 8) {
+      int s = sg;
+      for (; s + 56 < p.nsplit; s += 64) {  // 8 loads in flight, then added in the same order as one at a time
+        double2 v[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) v[k] = src[(long long)(s + 8 * k) * per_dom];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          sr += v[k].x;
+          si += v[k].y;
+        }
+      }
+      for (; s < p.nsplit; s += 8) {
         const double2 v = src[(long long)s * per_dom];
         sr += v.x;
         si += v.y;
@@ -399,7 +410,15 @@ __global__ void __launch_bounds__(256) k_reduce(ReduceArgs p, int eblocks) {
     double acc = 0.0;
     if (n < p.ncols) {
       const double* ns = p.normp + (long long)dom * p.nsplit * p.ncols + n;
-      for (int s = sg; s < p.nsplit; s += 8) acc += ns[(long long)s * p.ncols];
+      int s = sg;
+      for (; s + 56 < p.nsplit; s += 64) {  // as above: 8 loads in flight, same addition order
+        double v[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) v[k] = ns[(long long)(s + 8 * k) * p.ncols];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) acc += v[k];
+      }
+      for (; s < p.nsplit; s += 8) acc += ns[(long long)s * p.ncols];
     }
     sh[sg][el].x = acc;
     __syncthreads();
