@@ -26,8 +26,12 @@
  *   lfd_ref_nl_half          pinned: norm closed form; Gram closed form; BLAS (numpy) for C.
  *   lfd_ref_nl_half_exact    pinned: dense scipy expm of -i(Delta/2) B D B^H dV; projector columns get
  *                            e^{-i(Delta/2)D_u}; span(B)-orthogonal part unchanged; unitary.
- *   lfd_ref_step_exact       pinned: Gram matrix (orthonormality) conserved for D != 0.
- *   lfd_ref_step             pinned: norm / orthonormality conservation; gauge covariance.
+ *   lfd_ref_step_exact       pinned: Gram matrix (orthonormality) conserved for D != 0; second-order
+ *                            convergence to dense expm(-i T (H_FD + V + B diag(D) B^H dV)).
+ *   lfd_ref_step             pinned: norm / orthonormality conservation; gauge covariance; with the
+ *                            nonlocal factor ON (tests/test_oracle_pins_step.py): closed form on
+ *                            projector plane waves (lambda_u f_u^2, f_u = (1-i eps D_u)/|.|) and on a
+ *                            two-column mix; first-order convergence to the same dense expm.
  *   lfd_ref_density_current  pinned: plane-wave closed forms; sum rule; J = dE_kin/dA / V.
  *   lfd_ref_energy           pinned: plane-wave closed forms (kinetic, local = f mean(v)); nonlocal on
  *                            projector columns = f D_u; O(dt^2) energy drift of the step at A = D = 0.
