@@ -65,7 +65,7 @@ typedef struct {
   int32_t nref_max;    /* max reference-basis columns for lfd_remap_occ, 0..2048 (0: max(norb, nproj)) */
   double dt;           /* Delta_QD [a.u.], finite and nonzero (negative = backward in time) */
   int32_t device;      /* CUDA device ordinal */
-  int32_t flags;       /* 0 or LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP | LFD_FLAG_NL_DMMA */
+  int32_t flags;       /* 0 or LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP | LFD_FLAG_NL_DMMA | LFD_FLAG_NL_I8 */
 } lfd_config;
 
 /* lfd_config.flags: disable the projection carry (lfd_step takes the C of each nonlocal factor that
@@ -86,13 +86,19 @@ typedef struct {
  * agree with the FP64 path to single-precision roundoff (DESIGN.md §4 states the tolerance). */
 #define LFD_FLAG_SP 4
 /* lfd_config.flags: run the nonlocal GEMMs (C = dV B^H Psi; Psi <- Psi diag(n) + B C'') as
- * complex FP64 DMMA (mma.sync m8n8k4) instead of the default for FP64 contexts with nproj <= 64,
- * norb <= 64 and >= 65,536 points per domain: the same products with FP64 accuracy on the tcgen05 int8
- * tensor cores -- B and C'' split exactly into 6 int8
- * digits each with power-of-two row / column scales, the 21 digit-pair products accumulated exactly in
- * int32 in tensor memory, recombined in FP64 (relative error of the product ~3e-12, i.e. ~1e-15 of Psi
- * per factor since the update is O(Delta Delta_sci / 2) of Psi). See lfd_nl_path(). */
+ * strict IEEE complex FP64 on the DMMA pipe (mma.sync m8n8k4) instead of the default for FP64 contexts with
+ * nproj <= 64, norb <= 64 and >= 65,536 points per domain: the same products EMULATED on the tcgen05 int8
+ * tensor cores -- B and C'' split exactly into 6 balanced int8 digits each with power-of-two row / column
+ * scales, the 21 digit pairs i + j <= 7 accumulated exactly in int32 in tensor memory, recombined in FP64.
+ * That arithmetic is narrower than an FP64 product: the truncation (digit remainders and dropped pairs) leaves
+ * an error of ~2^-40 of (row scale x column scale) per output, against ~2^-53 for IEEE FP64 (measured per
+ * GEMM in tests/test_gpu_i8.py). The nonlocal update B C'' is O(Delta Delta_sci / 2 ~ 1.4e-3) of Psi, so at the
+ * paper's scissor size each factor moves Psi by ~1e-15 relative and the FP64 parity contract (1e-10 after 100
+ * steps) holds; bench.py reports the strict-FP64 step (this flag) beside the default. See lfd_nl_path(). */
 #define LFD_FLAG_NL_DMMA 8
+/* lfd_config.flags: use the int8-digit GEMMs wherever they are supported (nproj, norb <= 64), also on small
+ * grids where they are not the default (< 65,536 points per domain: set-up not amortised). */
+#define LFD_FLAG_NL_I8 16
 
 /* Kernel classes, for lfd_profile_read(). */
 typedef enum {
@@ -285,7 +291,7 @@ lfd_status lfd_sync(lfd_ctx* ctx);
 lfd_status lfd_launch_count(const lfd_ctx* ctx, uint64_t* count);
 
 /* Which kernel runs the nonlocal GEMM-2 of this context: *path = 0 complex FP64 DMMA (mma.sync),
- * 1 int8-digit tcgen05 tensor cores with FP64 accuracy (LFD_FLAG_NL_DMMA), 2 SP 3xTF32 (LFD_FLAG_SP),
+ * 1 int8-digit tcgen05 tensor cores, FP64 emulated (see LFD_FLAG_NL_DMMA), 2 SP 3xTF32 (LFD_FLAG_SP),
  * -1 no nonlocal factor (nproj == 0). */
 lfd_status lfd_nl_path(const lfd_ctx* ctx, int32_t* path);
 

@@ -40,6 +40,8 @@ struct Layout {
   size_t total;
   int nsplit;
   long long rows_per_split;
+  int nsplit_g;              // split count of the one-time G = dV B^H B (partials of nproj^2 each)
+  long long rows_per_split_g;
 };
 
 thread_local std::string g_tls_error = "no error";
@@ -68,7 +70,7 @@ lfd_status validate(const lfd_config* c, std::string& why) {
   if (c->norb < 1) { why = "norb must be >= 1"; return LFD_EINVAL; }
   if (c->nproj < 0 || c->nproj > 2048) { why = "nproj must be in [0, 2048]"; return LFD_EINVAL; }
   if (!(c->dt != 0.0) || !std::isfinite(c->dt)) { why = "dt must be finite and nonzero"; return LFD_EINVAL; }
-  if (c->flags & ~(LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP | LFD_FLAG_NL_DMMA)) {
+  if (c->flags & ~(LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP | LFD_FLAG_NL_DMMA | LFD_FLAG_NL_I8)) {
     why = "unknown flags";
     return LFD_EINVAL;
   }
@@ -81,16 +83,15 @@ lfd_status validate(const lfd_config* c, std::string& why) {
   return LFD_OK;
 }
 
-// GEMM-2 on the tcgen05 int8 tensor cores with FP64 accuracy (nl_i8.cu): the default for FP64 contexts with
-// nproj, norb <= 64; LFD_FLAG_NL_DMMA (or env LFD_NL_I8=0, an A/B knob) selects the DMMA kernels.
+// The projector GEMMs on the tcgen05 int8 tensor cores (nl_i8.cu): the default for FP64 contexts with
+// nproj, norb <= 64 and >= 64K points per domain; LFD_FLAG_NL_DMMA selects the FP64 DMMA kernels.
 // Small grids (< 64K points per domain, e.g. C1 / C3) stay on DMMA by default: there the int8 kernels' per-CTA
-// set-up (C'' digits, TMEM allocation, the exponent handshake) is not amortised (C1: 0.084 vs 0.058 ms/step).
-// env LFD_NL_I8=1 forces the int8 path wherever it is supported (tests), 0 disables it.
+// set-up (C'' digits, TMEM allocation, the exponent handshake) is not amortised (C1: 0.084 vs 0.058 ms/step);
+// LFD_FLAG_NL_I8 forces the int8 path wherever it is supported.
 bool use_i8(const lfd_config* c) {
-  bool on = (c->flags & (LFD_FLAG_NL_DMMA | LFD_FLAG_SP)) == 0;
+  const bool on = (c->flags & (LFD_FLAG_NL_DMMA | LFD_FLAG_SP)) == 0;
   const long long ng = (long long)c->nx * c->ny * c->nz;
-  bool want = ng >= 65536;
-  if (const char* v = std::getenv("LFD_NL_I8")) want = std::atoi(v) != 0;
+  const bool want = ng >= 65536 || (c->flags & LFD_FLAG_NL_I8);
   return on && want && lfd::gemm2_i8_supported(c->nproj, c->norb);
 }
 
@@ -139,7 +140,7 @@ Layout layout(const Geometry& g, int num_sms, int nref_max) {
   L.nsplit = nsplit;
   L.rows_per_split = rps;
   const size_t c16 = 16, d8 = 8;
-  const size_t mn = (size_t)std::max(std::max(np * no, np * np), L.nref_cap * no);
+  const size_t mn = (size_t)std::max(np * no, L.nref_cap * no);
   size_t o = 0;
   auto take = [&](size_t bytes) { size_t at = o; o += up(std::max<size_t>(bytes, 1)); return at; };
   L.phi = take((size_t)nd * g.ng * c16);
@@ -152,7 +153,17 @@ Layout layout(const Geometry& g, int num_sms, int nref_max) {
     L.nsplit_i8 = (int)((g.ng + L.rows_per_split_i8 - 1) / L.rows_per_split_i8);
   }
   const int nsplit_cap = std::max(nsplit, L.i8 ? L.nsplit_i8 : 0);
-  L.part = take((size_t)nd * nsplit_cap * mn * c16);
+  // G needs nproj^2 per split: it takes as many splits as fit the per-step partial buffer (at least one), so
+  // the workspace is sized by the per-step GEMM-1, not by the once-only Gram matrix
+  {
+    const long long gsz = std::max<long long>(1, (long long)np * np);
+    long long sg = std::max<long long>(1, std::min<long long>(nsplit, (long long)nsplit_cap * (long long)mn / gsz));
+    long long rg = (g.ng + sg - 1) / sg;
+    rg = std::max<long long>(kKC1, (rg + kKC1 - 1) / kKC1 * kKC1);
+    L.nsplit_g = (int)((g.ng + rg - 1) / rg);
+    L.rows_per_split_g = rg;
+  }
+  L.part = take((size_t)nd * std::max((size_t)nsplit_cap * mn, (size_t)L.nsplit_g * np * np) * c16);
   L.normp = take((size_t)nd * nsplit_cap * no * d8);
   L.dc = take((size_t)nd * np * no * c16);
   L.cprime = take((size_t)nd * np * no * c16);
@@ -273,7 +284,6 @@ struct lfd_ctx {
   int device;
   int num_sms;
   uint64_t launches = 0;
-  int gemm2_variant = 3;  // internal tuning knob, env LFD_GEMM2_VARIANT (3 = TMA tensor maps + warp-half skew)
   // Projection carry: true while the workspace's DC / C' / s / n describe the GEMM-2 that produced the
   // current Psi, so the next nonlocal factor can take C from the exact identity C_new = (C + G X) n
   // instead of GEMM-1 (cleared by the local propagator, lfd_psi_modified and LFD_FLAG_NO_CARRY).
@@ -283,10 +293,10 @@ struct lfd_ctx {
   // pass that wrote it, consumed -- and cleared on the device -- by GEMM-1)
   bool colE_valid = false;
   bool exact = false;     // LFD_FLAG_EXACT_NL: exactly unitary nonlocal factor (orthonormal B)
-  bool kin_fused = true;  // Phi.K_y K_z in one pass (env LFD_KIN_FUSED=0: separate y and z passes)
+  bool kin_fused = true;  // Phi.K_y K_z in one pass (else separate y and z passes: lines too long for the ring)
   CUtensorMap psi_tmap;   // TMA descriptor of Psi for the fused pass
   lfd::DensMaps* dmaps = nullptr;  // TMA descriptors of Psi for the density kernel
-  bool scaled = true;     // scaled pair form of the stencil (env LFD_KIN_SCALED=0: general 2x2 form)
+  bool scaled = true;     // scaled pair form of the stencil (else the general 2x2 form: some cos(tau t) < 1/2)
   std::string err = "no error";
   // density-current global layout cache
   std::vector<long long> gbase_host;
@@ -445,32 +455,10 @@ lfd_status gemm2(lfd_ctx* c, double2* out = nullptr) {
   lfd::Gemm2Args a2;
   a2.psi = c->psi; a2.B = c->proj; a2.Cp = c->at<double2>(c->L.cprime); a2.nfac = c->at<double>(c->L.nfac);
   a2.ndom = g.ndom; a2.nproj = g.nproj; a2.norb = g.norb; a2.ng = g.ng; a2.num_sms = c->num_sms;
-  a2.variant = c->gemm2_variant;
   a2.psi_out = out;
   if (c->L.i8) {
     a2.bsl = c->at<int8_t>(c->L.bsl);
     a2.bsig = c->at<double>(c->L.bsig);
-    if (const char* v = std::getenv("LFD_I8_DBG")) a2.dbg = std::atoi(v);
-    if (const char* v = std::getenv("LFD_EARLY_PDL")) a2.early = std::atoi(v);
-    if (std::getenv("LFD_I8_TIMING")) {  // diagnostics: role wait cycles, printed per call (one domain)
-      static long long* buf = nullptr;
-      if (!buf) cudaMallocManaged(&buf, 8 * 1024 * sizeof(long long));
-      cudaStreamSynchronize(c->stream);
-      for (int i = 0; i < 8 * 1024; ++i) buf[i] = 0;
-      a2.dbgbuf = buf;
-      lfd_status st = LFD_OK;
-      LFD_TRY(launch(c, LFD_K_NL_BACK, "k_gemm2", [&] { return lfd::launch_gemm2(a2, c->stream); }));
-      cudaStreamSynchronize(c->stream);
-      double s[7] = {0, 0, 0, 0, 0, 0, 0};
-      for (int b = 0; b < c->num_sms; ++b)
-        for (int k = 0; k < 7; ++k) s[k] += (double)buf[b * 8 + k];
-      std::fprintf(stderr, "i8 timing (avg cycles per CTA): prologue %.0f  mma loop %.0f  kernel %.0f  mma-wait-digits %.0f  "
-                   "mma-wait-slot %.0f  epi-wait-diag %.0f (per warp)  epi-wait-psi %.0f (per warp)\n",
-                   s[5] / c->num_sms, s[2] / c->num_sms, s[6] / c->num_sms, s[0] / c->num_sms, s[1] / c->num_sms,
-                   s[3] / c->num_sms / 16, s[4] / c->num_sms / 16);
-      c->c_valid = c->carry;
-      return st;
-    }
   }
   c->c_valid = false;
   if (g.sp)
@@ -532,28 +520,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
     ai.part = a1.part; ai.norms = a1.norms;
     ai.ndom = g.ndom; ai.nproj = g.nproj; ai.norb = g.norb; ai.nsplit = c->L.nsplit_i8;
     ai.ng = g.ng; ai.rps = c->L.rows_per_split_i8;
-    if (const char* v = std::getenv("LFD_I8_DBG1")) ai.dbg = std::atoi(v);
-    if (const char* v = std::getenv("LFD_EARLY_PDL")) ai.early = std::atoi(v);
-    if (const char* v = std::getenv("LFD_G1_WIDE")) ai.wide = std::atoi(v);
-    if (const char* v = std::getenv("LFD_G1_SLEEP")) ai.sleep = std::atoi(v);
-    if (std::getenv("LFD_I8_TIMING")) {  // diagnostics: role wait cycles
-      static long long* buf = nullptr;
-      if (!buf) cudaMallocManaged(&buf, 8 * 1024 * sizeof(long long));
-      cudaStreamSynchronize(c->stream);
-      for (int i = 0; i < 8 * 1024; ++i) buf[i] = 0;
-      ai.dbgbuf = buf;
-    }
     LFD_TRY(launch(c, LFD_K_NL_PROJ, "k_gemm1_i8", [&] { return lfd::launch_gemm1_i8(ai, c->stream); }));
-    if (ai.dbgbuf) {
-      cudaStreamSynchronize(c->stream);
-      double s5[6] = {0, 0, 0, 0, 0, 0};
-      for (int b = 0; b < ai.nsplit; ++b)
-        for (int k = 0; k < 6; ++k) s5[k] += (double)ai.dbgbuf[b * 8 + k];
-      std::fprintf(stderr, "g1 timing (avg cycles per CTA): mma loop %.0f  mma-wait-B %.0f  mma-wait-A %.0f  "
-                   "worker-wait-psi %.0f  worker-wait-afree %.0f  worker-tmem-store %.0f (per warp)\n",
-                   s5[2] / ai.nsplit, s5[0] / ai.nsplit, s5[1] / ai.nsplit, s5[3] / ai.nsplit / 16,
-                   s5[4] / ai.nsplit / 16, s5[5] / ai.nsplit / 16);
-    }
     c->colE_valid = false;
     nsplit = c->L.nsplit_i8;
   } else {
@@ -573,14 +540,6 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
     LFD_TRY(launch(c, LFD_K_NL_REDUCE, "k_reduce", [&] { return lfd::launch_reduce(r, c->stream); }));
     return gemm2(c, out);
   }
-  static const bool fused = [] {
-    const char* v = std::getenv("LFD_REDUCE_FUSED");
-    return v && std::atoi(v) != 0;
-  }();
-  if (!merged && fused)  // split reduction, n_s and C'' in one kernel (A/B knob LFD_REDUCE_FUSED=1)
-    return launch(c, LFD_K_NL_REDUCE, "k_reduce_norm", [&] {
-             return lfd::launch_reduce_norm(r, c->at<double2>(c->L.G), c->at<double>(c->L.nfac), c->stream);
-           }) == LFD_OK ? gemm2(c, out) : LFD_ECUDA;
   LFD_TRY(launch(c, LFD_K_NL_REDUCE, "k_reduce", [&] { return lfd::launch_reduce(r, c->stream); }));
   if (merged)
     LFD_TRY(launch(c, LFD_K_NL_NORM, "k_nlmerge", [&] {
@@ -659,7 +618,6 @@ lfd_status density_into(lfd_ctx* c, double* rho, double* j, double* Jmac, const 
   lfd::DensArgs a;
   a.psi = c->psi; a.coef = coef ? coef : c->coef(); a.occ = c->at<double>(c->L.occ);
   a.psi_sp = c->g.sp ? c->psi32() : nullptr;
-  if (const char* v = std::getenv("LFD_DENS_DBG")) a.dbg_nocompute = std::atoi(v);
   a.rho = rho; a.j = j; a.jline = c->at<double>(c->L.jline);
   a.base = base_dev; a.jbase = base_dev + c->g.ndom; a.sx = sx; a.sy = sy; a.jstride = jstride;
   a.v = energy ? c->at<double>(c->L.vstage) : nullptr;
@@ -944,10 +902,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   c->stream = static_cast<cudaStream_t>(stream);
   c->device = cfg->device;
   c->num_sms = prop.multiProcessorCount;
-  if (const char* v = std::getenv("LFD_GEMM2_VARIANT")) c->gemm2_variant = std::atoi(v);
   c->carry = (cfg->flags & LFD_FLAG_NO_CARRY) == 0;
-  if (const char* v = std::getenv("LFD_KIN_FUSED")) c->kin_fused = std::atoi(v) != 0;
-  if (const char* v = std::getenv("LFD_KIN_SCALED")) c->scaled = std::atoi(v) != 0;
   c->scaled = c->scaled && lfd::kin_scaled_ok(g);
   c->kin_fused = c->kin_fused && lfd::kin_yz_supported(g) && !g.sp;
   c->dmaps = lfd::density_maps_create(g, c->psi, active_orbitals(g, occ));
@@ -992,14 +947,14 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   if (g.nproj > 0) {
     lfd::Gemm1Args a1;
     a1.A = c->proj; a1.X = c->proj; a1.part = c->at<double2>(L.part); a1.norms = nullptr;
-    a1.ndom = g.ndom; a1.mrows = g.nproj; a1.ncols = g.nproj; a1.nsplit = L.nsplit;
-    a1.ng = g.ng; a1.rows_per_split = L.rows_per_split;
+    a1.ndom = g.ndom; a1.mrows = g.nproj; a1.ncols = g.nproj; a1.nsplit = L.nsplit_g;
+    a1.ng = g.ng; a1.rows_per_split = L.rows_per_split_g;
     a1.a_dom_stride = g.ng * g.nproj; a1.x_dom_stride = g.ng * g.nproj;
     s2 = launch(c, LFD_K_NL_PROJ, "k_gemm1(G)", [&] { return gemm1_any(c, a1); });
     if (s2 != LFD_OK) return bail(s2);
     lfd::ReduceArgs r{};
     r.part = a1.part; r.normp = nullptr; r.D = nullptr; r.out = c->at<double2>(L.G); r.cprime = nullptr; r.s = nullptr;
-    r.ndom = g.ndom; r.mrows = g.nproj; r.ncols = g.nproj; r.nsplit = L.nsplit; r.scale = g.dV; r.eps = 0;
+    r.ndom = g.ndom; r.mrows = g.nproj; r.ncols = g.nproj; r.nsplit = L.nsplit_g; r.scale = g.dV; r.eps = 0;
     s2 = launch(c, LFD_K_NL_REDUCE, "k_reduce(G)", [&] { return lfd::launch_reduce(r, c->stream); });
     if (s2 != LFD_OK) return bail(s2);
   }

@@ -494,7 +494,7 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
     // per-lane partial sums over this lane's orbitals: rho and the three link products P_d = sum f
     // conj(psi_r) psi_{r+e_d} (f folded into fv = f psi_r)
     double rho = 0.0, pxr = 0.0, pxi = 0.0, pyr = 0.0, pyi = 0.0, pzr = 0.0, pzi = 0.0;
-    if (valid && !a.dbg_nocompute) {
+    if (valid) {
 #pragma unroll
       for (int i = 0; i < (kIt > 0 ? kIt : kItMax); ++i) {
         if (kIt == 0 && i >= nit) break;

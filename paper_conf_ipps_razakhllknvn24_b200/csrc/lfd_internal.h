@@ -132,7 +132,6 @@ struct ReduceArgs {
 };
 cudaError_t launch_reduce(const ReduceArgs& a, cudaStream_t st);
 // launch_reduce + launch_nlnorm in one kernel for the plain factor (D real, cprime = -i eps D C n, no W / merge)
-cudaError_t launch_reduce_norm(const ReduceArgs& a, const double2* G, double* nfac, cudaStream_t st);
 
 // n_s = sqrt( s_s / (s_s + eps^2 * (DC)_s^H G (DC)_s) )   (Gram closed form of the Eq. 6 norm, R11),
 // then C'_s <- C'_s n_s in place: the GEMM-2 coefficient is always C'' = C' diag(n), so its epilogue is
@@ -164,13 +163,9 @@ struct Gemm2Args {
   int ndom, nproj, norb;
   long long ng;
   int num_sms;
-  int variant;  // tuning knob (LFD_GEMM2_VARIANT): 0 = epilogue loads after the K loop, 1 = mid-loop
   // int8-digit tensor-core path (nl_i8.cu): B's digit tiles and row scales from launch_bslice_i8, or nullptr
   const int8_t* bsl = nullptr;
   const double* bsig = nullptr;
-  int early = 1;  // PDL: set-up and the constant-digit loads before griddepcontrol.wait (env LFD_EARLY_PDL=0: off)
-  int dbg = 0;  // diagnostics only (env LFD_I8_DBG): 2 = no epilogue math
-  long long* dbgbuf = nullptr;  // diagnostics only (env LFD_I8_TIMING): per-CTA wait cycles of each role
 };
 cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st);
 // GEMM-2 with FP64 accuracy on the tcgen05 int8 tensor cores (nl_i8.cu): nproj <= 64, norb <= 64.
@@ -193,12 +188,6 @@ struct Gemm1I8Args {
   double* norms;        // [dom][nsplit][norb]
   int ndom, nproj, norb, nsplit;
   long long ng, rps;
-  int early = 1;  // as Gemm2Args::early
-  int wide = 1;   // MMA schedule (env LFD_G1_WIDE): 0 = 21 MMAs of N = 64, diagonal-major; 1 / 2 = B digits
-                  // i .. i+2 / i .. i+1 stacked along N (9 / 12 MMAs); 3 = N = 64 round-robin over diagonals
-  int sleep = 0;  // env LFD_G1_SLEEP=1: the A-buffer handshake waits carry a suspend-time hint
-  long long* dbgbuf = nullptr;  // diagnostics only (env LFD_I8_TIMING): per-CTA wait cycles of each role
-  int dbg = 0;                  // diagnostics only (env LFD_I8_DBG1): 1 one pair, 4 no TMEM stores, 8 no digits
 };
 size_t gemm1_i8_bytes(int ndom, long long ng);
 long long gemm1_i8_rows_per_split(long long ng, int ndom, int num_sms);
@@ -213,7 +202,6 @@ cudaError_t gemm_set_attributes();
 struct DensArgs {
   const double2* psi;
   const float2* psi_sp = nullptr;  // SP variant: complex64 Psi (then psi is unused)
-  int dbg_nocompute = 0;           // diagnostics only (env LFD_DENS_DBG=1): skip the per-point sums
   const DomCoef* coef;
   const double* occ;
   double* rho;

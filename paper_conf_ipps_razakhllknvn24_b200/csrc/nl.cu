@@ -527,102 +527,6 @@ __global__ void __launch_bounds__(256) k_nlnorm(int nproj, int norb, double eps2
   }
 }
 
-// k_reduce + k_nlnorm for the common factor (real D, no merge), one block per (orbital s, domain): the
-// fixed-order split reduction of column s (DC = dV D C, its norm s_s), then n_s from the Gram closed form
-// and C''_s = -i eps DC_s n_s -- one launch instead of two.
-__global__ void __launch_bounds__(256) k_reduce_norm(ReduceArgs p, const double2* __restrict__ G,
-                                                     double* __restrict__ nfac) {
-  pdl_wait();
-  pdl_trigger();
-  extern __shared__ double2 dcs[];  // DC[:, col]
-  __shared__ double2 part4[4][64];
-  __shared__ double wq[8];
-  const int dom = blockIdx.y, col = blockIdx.x;
-  const int nproj = p.mrows, norb = p.ncols;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const long long per_dom = (long long)nproj * norb;
-  const double2* src = p.part + (long long)dom * p.nsplit * per_dom + col;
-  // 1. split sums: thread (g = tid / 64, u = tid % 64 + 64 k) sums splits g, g + 4, ... in order
-  for (int u0 = 0; u0 < nproj; u0 += 64) {
-    const int u = u0 + (threadIdx.x & 63), g = threadIdx.x >> 6;
-    double sr = 0.0, si = 0.0;
-    if (u < nproj) {
-      const double2* su = src + (long long)u * norb;
-#pragma unroll 8
-      for (int sp = g; sp < p.nsplit; sp += 4) {  // (loads independent: unrolled so they are in flight together)
-        const double2 v = __ldg(su + (long long)sp * per_dom);
-        sr += v.x;
-        si += v.y;
-      }
-    }
-    part4[g][threadIdx.x & 63] = make_double2(sr, si);
-    __syncthreads();
-    if (threadIdx.x < 64 && u < nproj) {
-      const double tr = (part4[0][threadIdx.x].x + part4[1][threadIdx.x].x) + (part4[2][threadIdx.x].x + part4[3][threadIdx.x].x);
-      const double ti = (part4[0][threadIdx.x].y + part4[1][threadIdx.x].y) + (part4[2][threadIdx.x].y + part4[3][threadIdx.x].y);
-      const double f = p.scale * p.D[(long long)dom * nproj + u];
-      const double2 o = make_double2(tr * f, ti * f);
-      dcs[u] = o;
-      p.out[(long long)dom * per_dom + (long long)u * norb + col] = o;
-    }
-    __syncthreads();
-  }
-  // column norm s_s (fixed order over the splits)
-  if (warp == 0) {
-    double a = 0.0;
-    for (int sp = lane; sp < p.nsplit; sp += 32) a += p.normp[((long long)dom * p.nsplit + sp) * norb + col];
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
-    if (lane == 0) {
-      a *= p.scale;
-      p.s[(long long)dom * norb + col] = a;
-      wq[7] = a;  // (read by thread 0 after the barrier below)
-    }
-  }
-  // 2. n_s = sqrt(s_s / (s_s + eps^2 Re[(DC)_s^H G (DC)_s]))
-  const double2* Gd = G + (long long)dom * nproj * nproj;
-  double q = 0.0;
-  for (int u = warp; u < nproj; u += 8) {
-    const double2* Gu = Gd + (long long)u * nproj;
-    double tr = 0.0, ti = 0.0;
-    for (int v = lane; v < nproj; v += 32) {
-      const double2 gv = Gu[v], c = dcs[v];
-      tr = fma(gv.x, c.x, fma(-gv.y, c.y, tr));
-      ti = fma(gv.x, c.y, fma(gv.y, c.x, ti));
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      tr += __shfl_xor_sync(0xffffffffu, tr, o);
-      ti += __shfl_xor_sync(0xffffffffu, ti, o);
-    }
-    const double2 cu = dcs[u];
-    q = fma(cu.x, tr, fma(cu.y, ti, q));
-  }
-  __shared__ double wq2[8];
-  if (lane == 0) wq2[warp] = q;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    double tq = 0.0;
-    for (int w = 0; w < 8; ++w) tq += wq2[w];
-    const double sv = wq[7];
-    const double n = sqrt(sv / (sv + p.eps * p.eps * tq));
-    nfac[(long long)dom * norb + col] = n;
-    wq[0] = n;
-  }
-  __syncthreads();
-  const double n = wq[0];  // C'' = -i eps DC n
-  for (int u = threadIdx.x; u < nproj; u += blockDim.x) {
-    const double2 o = dcs[u];
-    p.cprime[((long long)dom * nproj + u) * norb + col] = make_double2(p.eps * o.y * n, -p.eps * o.x * n);
-  }
-}
-
-cudaError_t launch_reduce_norm(const ReduceArgs& a, const double2* G, double* nfac, cudaStream_t st) {
-  dim3 grid(a.ncols, a.ndom);
-  launch_k(k_reduce_norm, grid, 256, a.mrows * sizeof(double2), st, a, G, nfac);
-  return cudaGetLastError();
-}
-
 cudaError_t launch_nlnorm(int ndom, int nproj, int norb, double eps, const double2* G, const double2* DC,
                           const double* s, double* nfac, double2* Cp, cudaStream_t st) {
   dim3 grid(norb, ndom);
@@ -1010,161 +914,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(const __grid_constant__ C
   }
 }
 
-// ------------------------------------------------------------------------------------------------
-// GEMM-2, full-K variant for nproj <= 64 (the paper-shaped case): the whole K = nproj fits one stage.
-// Each work item's 64 B rows arrive by 64 TMA bulk row copies into a 2-deep ring of padded tiles (row
-// stride = nproj rounded to 4, == 4 mod 8 complex, so the A-fragment LDS.128 are conflict free), and
-// C' for the current (domain, column tile) stays resident in shared memory. Items are ordered
-// (domain, column tile, row block) so C' is reloaded only when a CTA crosses into another
-// (domain, tile). The Psi rows of the next item are prefetched into L2 (cp.async.bulk.prefetch) so the
-// epilogue's loads hit L2. kNP = 64 instantiates a fully unrolled K loop; kNP = 0 handles any nproj <= 64.
-// ------------------------------------------------------------------------------------------------
+// Tile geometry of k_gemm2_tma (nproj <= 64): a 2-deep ring of [64 rows][lda] B tiles (lda == 4 mod 8
+// complex: conflict-free A-fragment LDS.128) and C' of one (domain, column tile) resident.
 constexpr int kFullStages = 2;
 constexpr int kFullLdaMax = 68;
 constexpr int kFullABytes = kTile * kFullLdaMax * 16;     // [64 rows][<=68] complex
 constexpr int kFullCBytes = kTile * kLd1 * 16;            // [<=64 proj][66] complex
 constexpr int kFullSmem = kFullStages * kFullABytes + kFullCBytes + 4 * 8;
-
 __host__ __device__ constexpr int full_lda(int np) { return ((np + 3) / 4 * 4) % 8 == 0 ? (np + 3) / 4 * 4 + 4 : (np + 3) / 4 * 4; }
-
-template <int kNP, bool kPvMid>
-__global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
-  pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
-  pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
-  extern __shared__ __align__(128) unsigned char smem[];
-  double2* Cs = reinterpret_cast<double2*>(smem + kFullStages * kFullABytes);
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kFullStages * kFullABytes + kFullCBytes);
-  uint64_t* cbar = bars + kFullStages;
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int g = lane >> 2, t = lane & 3;
-  const int wm = warp >> 2, wn = warp & 3;
-  const int np = kNP > 0 ? kNP : p.nproj;
-  const int lda = full_lda(np);
-  const long long rblocks = (p.ng + kTile - 1) / kTile;
-  const int ntn = (p.norb + kTile - 1) / kTile;
-  const long long items = (long long)p.ndom * ntn * rblocks;
-  const long long my_items = (items > blockIdx.x) ? (items - 1 - blockIdx.x) / gridDim.x + 1 : 0;
-  constexpr int kNK4 = kNP > 0 ? (kNP + 3) / 4 : 16;
-  const int nk4 = (np + 3) / 4;
-
-  if (tid == 0) {
-    for (int s = 0; s < kFullStages + 1; ++s) mbar_init(&bars[s], 1);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-
-  auto decode = [&](long long j, int& dom, int& n0, long long& r0) {
-    const long long item = blockIdx.x + j * gridDim.x;
-    const long long per_dom = (long long)ntn * rblocks;
-    dom = (int)(item / per_dom);
-    const long long rem = item - dom * per_dom;
-    const int nt = (int)(rem / rblocks);
-    n0 = nt * kTile;
-    r0 = (rem - (long long)nt * rblocks) * kTile;
-  };
-  auto issue = [&](long long j, int stage) {  // warp 0
-    int dom, n0;
-    long long r0;
-    decode(j, dom, n0, r0);
-    const int rows = (int)min((long long)kTile, p.ng - r0);
-    if (lane == 0) mbar_expect_tx(&bars[stage], (uint32_t)(rows * np * 16));
-    __syncwarp();
-    double2* As = reinterpret_cast<double2*>(smem + stage * kFullABytes);
-    const double2* src = p.B + ((long long)dom * p.ng + r0) * np;
-    for (int r = lane; r < rows; r += 32) tma_row(As + r * lda, src + (long long)r * np, np * 16, &bars[stage]);
-  };
-
-  if (warp == 0)
-    for (int s = 0; s < kFullStages && s < my_items; ++s) issue(s, s);
-
-  int cur_dom = -1, cur_n0 = -1;
-  uint32_t cphase = 0;
-  for (long long j = 0; j < my_items; ++j) {
-    int dom, n0;
-    long long r0;
-    decode(j, dom, n0, r0);
-    if (dom != cur_dom || n0 != cur_n0) {  // (re)load C'[dom][:, n0:n0+64] (all warps are past Cs)
-      const int nvalid = min(kTile, p.norb - n0);
-      if (warp == 0) {
-        if (lane == 0) mbar_expect_tx(cbar, (uint32_t)(np * nvalid * 16));
-        __syncwarp();
-        for (int r = lane; r < np; r += 32)
-          tma_row(Cs + r * kLd1, p.Cp + ((long long)dom * np + r) * p.norb + n0, nvalid * 16, cbar);
-      }
-      mbar_wait(cbar, cphase);
-      cphase ^= 1;
-      cur_dom = dom;
-      cur_n0 = n0;
-    }
-    // Psi rows of the NEXT item go to L2 now (the epilogue of this item reads rows prefetched during
-    // the previous one), keeping 64 registers free for fragment pipelining.
-    if (tid == 32 && j + 1 < my_items) {
-      int d1, n1;
-      long long q1;
-      decode(j + 1, d1, n1, q1);
-      const long long rows1 = min((long long)kTile, p.ng - q1);
-      l2_prefetch(p.psi + ((long long)d1 * p.ng + q1) * p.norb, (uint32_t)(rows1 * p.norb * 16));
-    }
-    if (tid == 32 && j == 0) {
-      const long long rows0 = min((long long)kTile, p.ng - r0);
-      l2_prefetch(p.psi + ((long long)dom * p.ng + r0) * p.norb, (uint32_t)(rows0 * p.norb * 16));
-    }
-    const int stage = (int)(j % kFullStages);
-    mbar_wait(&bars[stage], (uint32_t)((j / kFullStages) & 1));
-    const double2* As = reinterpret_cast<const double2*>(smem + stage * kFullABytes);
-    Frag acc;
-    acc.zero();
-    const double2* psi = p.psi + (long long)dom * p.ng * p.norb;
-    double2* pout = (p.psi_out ? p.psi_out : p.psi) + (long long)dom * p.ng * p.norb;
-    double2 pv[4][2][2];
-    auto load_pv = [&]() {
-#pragma unroll
-      for (int mi = 0; mi < 4; ++mi) {
-        const long long r = r0 + wm * 32 + mi * 8 + g;
-#pragma unroll
-        for (int ni = 0; ni < 2; ++ni)
-#pragma unroll
-          for (int c = 0; c < 2; ++c) {
-            const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
-            pv[mi][ni][c] = (r < p.ng && col < p.norb) ? psi[r * p.norb + col] : cz();
-          }
-      }
-    };
-#pragma unroll
-    for (int kk = 0; kk < kNK4; ++kk) {
-      if (kNP == 0 && kk >= nk4) break;
-      if (kPvMid && kk == kNK4 / 2) load_pv();  // Psi loads in flight during the second half
-      const int k = kk * 4 + t;
-      const bool ok = (kNP > 0 && kNP % 4 == 0) || k < np;
-      double2 a[4], c[2];
-#pragma unroll
-      for (int mi = 0; mi < 4; ++mi) a[mi] = ok ? As[(wm * 32 + mi * 8 + g) * lda + k] : cz();
-#pragma unroll
-      for (int ni = 0; ni < 2; ++ni) c[ni] = ok ? Cs[k * kLd1 + wn * 16 + ni * 8 + g] : cz();
-      mma_4x2(acc, a, c);
-    }
-    if (!kPvMid || (kNP == 0 && nk4 <= kNK4 / 2)) load_pv();
-    __syncthreads();  // stage and Cs free
-    if (warp == 0 && j + kFullStages < my_items) issue(j + kFullStages, stage);
-    // epilogue: Psi <- n_s (Psi + B C') (the Psi loads were issued above; L2 hits, prefetched)
-    const double* nf = p.nfac + (long long)dom * p.norb;
-#pragma unroll
-    for (int ni = 0; ni < 2; ++ni)
-#pragma unroll
-      for (int c = 0; c < 2; ++c) {
-        const int col = n0 + wn * 16 + ni * 8 + 2 * t + c;
-        if (col >= p.norb) continue;
-        const double f = nf[col];
-#pragma unroll
-        for (int mi = 0; mi < 4; ++mi) {
-          const long long r = r0 + wm * 32 + mi * 8 + g;
-          if (r < p.ng)
-            pout[r * p.norb + col] =
-                make_double2(fma(f, pv[mi][ni][c].x, acc.re(mi, ni, c)), fma(f, pv[mi][ni][c].y, acc.im(mi, ni, c)));
-        }
-      }
-  }
-}
 
 // ------------------------------------------------------------------------------------------------
 // GEMM-2, TMA tensor-map variant for nproj <= 64 (the paper-shaped case). Thread 0 issues, per work item,
@@ -1175,7 +932,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_fullk(Gemm2Args p) {
 // copy when it changes), the K loop is fully unrolled for nproj = 64, the epilogue's Psi loads are
 // issued mid-loop and Psi <- n_s (Psi + B C') is written in place.
 // ------------------------------------------------------------------------------------------------
-template <int kNP, bool kSkew, bool kOut = false>
+template <int kNP, bool kOut>
 __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant__ CUtensorMap tB,
                                                              const __grid_constant__ CUtensorMap tC, Gemm2Args p) {
   pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
@@ -1251,7 +1008,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant
     }
     // skew: the second M-half of the warps starts half a K loop late, so each half's epilogue overlaps
     // the other half's DMMAs (the halves share only the B stage and C')
-    if (kSkew && j == 0 && wm == 1) asm volatile("bar.sync 2, %0;" ::"n"(kThreads));
+    if (j == 0 && wm == 1) asm volatile("bar.sync 2, %0;" ::"n"(kThreads));
     const int s = (int)(j % kFullStages);
     mbar_wait(&full[s], (uint32_t)((j / kFullStages) & 1));
     const double2* As = reinterpret_cast<const double2*>(smem + s * kFullABytes);
@@ -1279,7 +1036,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant
       if (kNP == 0 && kk >= nk4) break;
       if (kk == kmid) {
         load_pv();  // Psi loads (L2 hits) in flight during the second half
-        if (kSkew && j == 0 && wm == 0) asm volatile("bar.arrive 2, %0;" ::"n"(kThreads));
+        if (j == 0 && wm == 0) asm volatile("bar.arrive 2, %0;" ::"n"(kThreads));
       }
       const int k = kk * 4 + t;
       double2 a[4], c[2];
@@ -1335,37 +1092,19 @@ cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
   const long long rblocks = (a.ng + kTile - 1) / kTile;
   const long long items = (long long)a.ndom * rblocks * ((a.norb + kTile - 1) / kTile);
   const int grid = (int)(items < a.num_sms ? items : a.num_sms);
-  if (a.nproj <= kTile && a.variant == 2) {
+  if (a.nproj <= kTile) {
     CUtensorMap tB, tC;
     cudaError_t e = gemm2_maps(a, &tB, &tC);
     if (e != cudaSuccess) return e;
     const bool o = a.psi_out != nullptr;  // out of place (the self-consistent step's first factor)
     if (a.nproj == kTile) {
-      if (o) launch_k(k_gemm2_tma<kTile, false, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
+      if (o) launch_k(k_gemm2_tma<kTile, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
       else launch_k(k_gemm2_tma<kTile, false>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
     } else {
-      if (o) launch_k(k_gemm2_tma<0, false, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
+      if (o) launch_k(k_gemm2_tma<0, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
       else launch_k(k_gemm2_tma<0, false>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
     }
-  } else if (a.nproj <= kTile && a.variant == 3) {
-    CUtensorMap tB, tC;
-    cudaError_t e = gemm2_maps(a, &tB, &tC);
-    if (e != cudaSuccess) return e;
-    const bool o = a.psi_out != nullptr;
-    if (a.nproj == kTile) {
-      if (o) launch_k(k_gemm2_tma<kTile, true, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
-      else launch_k(k_gemm2_tma<kTile, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
-    } else {
-      if (o) launch_k(k_gemm2_tma<0, true, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
-      else launch_k(k_gemm2_tma<0, true>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
-    }
-  } else if (a.nproj == kTile && a.variant == 1)
-    launch_k(k_gemm2_fullk<kTile, true>, grid, kThreads, kFullSmem, st, a);
-  else if (a.nproj == kTile)
-    launch_k(k_gemm2_fullk<kTile, false>, grid, kThreads, kFullSmem, st, a);
-  else if (a.nproj < kTile)
-    launch_k(k_gemm2_fullk<0, false>, grid, kThreads, kFullSmem, st, a);
-  else {
+  } else {
     // B [dom][ng][nproj] (box [1][64 rows][kKC2 + 4 complex]) and C'' [dom][nproj][norb] (box [1][kKC2][66])
     CUtensorMap tA, tC;
     const uint64_t dA[3] = {(uint64_t)2 * a.nproj, (uint64_t)a.ng, (uint64_t)a.ndom};
@@ -1390,18 +1129,19 @@ cudaError_t gemm_set_attributes() {
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_gemm1<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm1_smem_bytes());
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_gemm2_fullk<kTile, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
-  if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_gemm2_fullk<kTile, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
-  if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_gemm2_fullk<0, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem);
-  if (e != cudaSuccess) return e;
-  for (auto f : {k_gemm2_tma<kTile, false>, k_gemm2_tma<0, false>, k_gemm2_tma<kTile, true>, k_gemm2_tma<0, true>,
-                 k_gemm2_tma<kTile, false, true>, k_gemm2_tma<kTile, true, true>, k_gemm2_tma<0, false, true>,
-                 k_gemm2_tma<0, true, true>}) {
+  for (auto f : {k_gemm2_tma<kTile, false>, k_gemm2_tma<0, false>, k_gemm2_tma<kTile, true>, k_gemm2_tma<0, true>}) {
     e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem + 16);
     if (e != cudaSuccess) return e;
   }
+  // the nonlocal-coefficient kernels stage O(nproj) vectors in dynamic shared memory (nproj <= 2048)
+  for (auto f : {k_nlcarry<true>, k_nlcarry<false>}) {
+    e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 40 * 2048);
+    if (e != cudaSuccess) return e;
+  }
+  e = cudaFuncSetAttribute(k_nlmerge, cudaFuncAttributeMaxDynamicSharedMemorySize, 32 * 2048);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_nlnorm, cudaFuncAttributeMaxDynamicSharedMemorySize, 16 * 2048);
+  if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(k_gemm2, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm2_smem_bytes());
 }
 

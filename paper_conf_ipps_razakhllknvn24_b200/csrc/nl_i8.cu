@@ -257,7 +257,6 @@ template <bool kOut>
 __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
   // programmatic dependent launch: the set-up below (TMEM, barriers) and the digit producer (B's digits are
   // constant since lfd_init) overlap the previous kernel; every other warp waits for it (C'', n, Psi)
-  if (!p.early) pdl_wait();
   pdl_trigger();
   extern __shared__ __align__(1024) unsigned char dsm_raw[];
   // SWIZZLE_128B images need 1024-byte aligned shared addresses
@@ -276,7 +275,6 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
   const int norb = p.norb, nproj = p.nproj;
   const long long ng = p.ng;
   const long long tiles = (ng + kI8NT - 1) / kI8NT;
-  const long long t_entry = clock64();
 
   if (warp == kWMma) {  // TMEM: W^T digits (A operand, 6 x 32 columns) + the ring of diagonal accumulators
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_addr(&tmem_base_sh)));
@@ -383,23 +381,17 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
   } else if (warp == kWMma) {  // MMA issuer: D_d += W_j^T (TMEM) x b_i (smem), i + j = d; one ring slot per d
     {  // the whole warp runs the loop (warp-uniform values stay in uniform registers); one elected lane issues
       const uint32_t tbase = smem_addr(Tsm);
-      long long w_full = 0, w_slot = 0;
-      const long long t_start = clock64();
       int it = 0;
       for (long long t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
         const int s = it % kI8Stages;
-        long long c0 = clock64();
         mbar_wait(&full[s], (uint32_t)((it / kI8Stages) & 1));
-        w_full += clock64() - c0;
         tc_fence_after();
         const uint64_t db0 = umma_desc_sw128(tbase + s * kI8TileB);
 #pragma unroll
         for (int d = 2; d <= kI8S + 1; ++d) {
           const int g = it * kI8Acc + (d - 2), sl = g % kI8Slots;
           if (g >= kI8Slots) {
-            long long c1 = clock64();
             mbar_wait(&dempty[sl], (uint32_t)(((g / kI8Slots) - 1) & 1));
-            w_slot += clock64() - c1;
             tc_fence_after();
           }
           const uint32_t acc = tacc + sl * kI8NT;
@@ -421,12 +413,6 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
         }
         umma_commit(&empty[s]);  // the digit tile may be overwritten once these MMAs are done
       }
-      if (p.dbgbuf && lane == 0) {
-        p.dbgbuf[blockIdx.x * 8 + 0] = w_full;
-        p.dbgbuf[blockIdx.x * 8 + 1] = w_slot;
-        p.dbgbuf[blockIdx.x * 8 + 2] = clock64() - t_start;
-        p.dbgbuf[blockIdx.x * 8 + 5] = t_start - t_entry;
-      }
     }
   } else if (warp < kI8EpiWarps) {
     // epilogue: warp w reads TMEM lanes 32 (w & 3) .. + 31 (output double n of a Psi row) and tile rows
@@ -437,7 +423,6 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
     const bool nvalid = n < 2 * norb;
     const double nf = nvalid ? p.nfac[(long long)dom * norb + (n >> 1)] : 0.0;
     const double tau = taus[n];
-    long long w_dfull = 0, w_pfull = 0;
     double* pout = reinterpret_cast<double*>((kOut ? p.psi_out : p.psi) + (long long)dom * ng * norb) + n;
     const int ld = 2 * norb;
     int it = 0;
@@ -450,10 +435,8 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
 #pragma unroll 1
       for (int dp = 0; dp < kI8Acc / 2; ++dp) {  // diagonals d = 2 + 2 dp and d + 1
         const int g = it * kI8Acc + 2 * dp, s0 = g % kI8Slots, s1 = (g + 1) % kI8Slots;
-        long long c2 = clock64();
         mbar_wait(&dfull[s0], (uint32_t)((g / kI8Slots) & 1));
         mbar_wait(&dfull[s1], (uint32_t)(((g + 1) / kI8Slots) & 1));
-        w_dfull += clock64() - c2;
         tc_fence_after();
         int32_t a0[kI8Rows], a1[kI8Rows];
         const uint32_t lb = ((uint32_t)(32 * q) << 16) + kI8Rows * h;
@@ -478,28 +461,21 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
       // the warp's staged Psi sub-tile (rows 16 h .. 16 h + 15 of the tile)
       {
         const int u = it * (kI8NT / kI8SubR) + h, s = u % kI8PsiSlots;
-        long long c3 = clock64();
         mbar_wait(&pfull[s], (uint32_t)((u / kI8PsiSlots) & 1));
-        w_pfull += clock64() - c3;
         const double* ps = reinterpret_cast<const double*>(Psm + s * kI8SubB) + n;
         const double* sg = reinterpret_cast<const double*>(Psm + s * kI8SubB + kI8SubRowsB);
 #pragma unroll
         for (int c = 0; c < kI8Rows; ++c) {
-          if (!nvalid || c >= nc || (p.dbg & 2)) continue;
+          if (!nvalid || c >= nc) continue;
           pout[(r0 + c) * ld] = fma(nf, ps[c * ld], scale_pow2(fa[c], sg[c], tau));
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&pempty[s]);
       }
     }
-    if (p.dbgbuf && lane == 0) {
-      atomicAdd((unsigned long long*)&p.dbgbuf[blockIdx.x * 8 + 3], (unsigned long long)w_dfull);
-      atomicAdd((unsigned long long*)&p.dbgbuf[blockIdx.x * 8 + 4], (unsigned long long)w_pfull);
-    }
   }
   tc_fence_before();
   __syncthreads();
-  if (p.dbgbuf && tid == 0) p.dbgbuf[blockIdx.x * 8 + 6] = clock64() - t_entry;
   if (warp == kWMma) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
@@ -556,12 +532,6 @@ __device__ __forceinline__ void tmem_st4(uint32_t taddr, const uint32_t v[4]) {
   asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1,%2,%3,%4};" ::"r"(taddr), "r"(v[0]), "r"(v[1]),
                "r"(v[2]), "r"(v[3])
                : "memory");
-}
-
-template <bool T>
-__device__ __forceinline__ long long tclk() {
-  if constexpr (T) return clock64();
-  else return 0;
 }
 
 // The wide-N MMA schedule of one quarter block (see k_gemm1_i8): for each Psi digit j, the B digits
@@ -627,12 +597,9 @@ __global__ void __launch_bounds__(256) k_bslice1_i8(const double2* __restrict__ 
 }
 
 // grid (splits, ndom); CTA = one split of rps rows (a multiple of 64)
-// kT: role-wait instrumentation compiled in (LFD_I8_TIMING); the clock reads cost issue slots in the worker loop
-template <bool kT>
 __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   // programmatic dependent launch: set-up and the first B-digit blocks (constant since lfd_init) overlap the
   // previous kernel; the Psi loads and everything reading colE / writing the partials wait for it
-  if (!p.early) pdl_wait();
   pdl_trigger();
   extern __shared__ __align__(1024) unsigned char dsm_raw[];
   unsigned char* dsm = dsm_raw + ((1024u - (smem_addr(dsm_raw) & 1023u)) & 1023u);
@@ -699,61 +666,22 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   } else if (warp == kG1WMma) {  // MMA issuer
     {  // the whole warp runs the loop (warp-uniform values stay in uniform registers); one elected lane issues
       const uint32_t bbase = smem_addr(Bsm);
-      long long w_b = 0, w_a = 0;
-      const long long t0 = tclk<kT>();
       for (int g = 0; g < nhalf; ++g) {
         const int b = g >> 2, s = b % kG1Stages, kq = g & 3, ab = g & 1;
-        long long c0 = tclk<kT>();
         if (kq == 0) mbar_wait(&bfull[s], (uint32_t)((b / kG1Stages) & 1));
-        long long c1 = tclk<kT>();
-        if (p.sleep) mbar_wait_sleep(&afull[ab], (uint32_t)((g >> 1) & 1));
-        else mbar_wait(&afull[ab], (uint32_t)((g >> 1) & 1));
-        w_b += c1 - c0;
-        w_a += tclk<kT>() - c1;
+        mbar_wait(&afull[ab], (uint32_t)((g >> 1) & 1));
         tc_fence_after();
         const uint64_t db0 = umma_desc_sw128(bbase + s * kG1BlkB);
-        if (p.wide == 1 || p.wide == 2) {
-          // B's digit slices i .. i + w - 1 are consecutive 64-row SWIZZLE_128B tiles (8 KB each), i.e. one
-          // K-major tile of 64 w rows, and the diagonal accumulators d = i + j .. i + j + w - 1 are consecutive
-          // 64-column TMEM blocks: one MMA of N = 64 w computes the w digit pairs (i .. i + w - 1, j) straight
-          // into their diagonals. The j = 1 MMAs touch every diagonal first (accumulate = 0 at g = 0).
-          // wide 1: w <= 3 (9 MMAs); wide 2: w <= 2 (12 MMAs, consecutive ones mostly on disjoint diagonals)
-          if (p.wide == 1) g1_wide_mmas<3>(tacc, tmem + ab * kG1ABuf, db0, kq, g == 0);
-          else g1_wide_mmas<2>(tacc, tmem + ab * kG1ABuf, db0, kq, g == 0);
-        } else if (p.wide == 3) {
-          // N = 64, round-robin over the diagonals: round r takes the pair (r + 1, d - r - 1) of every
-          // diagonal d >= r + 2, so consecutive MMAs accumulate into different TMEM blocks
-#pragma unroll
-          for (int r = 0; r < kI8S; ++r) {
-#pragma unroll
-            for (int d = r + 2; d <= kI8S + 1; ++d) {
-              const int i = r + 1, j = d - i;
-              umma_g1_ts(tacc + (d - 2) * 64, tmem + ab * kG1ABuf + (j - 1) * 8,
-                         db0 + (uint64_t)(((i - 1) * kG1SliceB + kq * 32) >> 4), (g == 0 && r == 0) ? 0u : 1u);
-            }
-          }
-        } else
-#pragma unroll
-        for (int d = 2; d <= kI8S + 1; ++d) {
-          const uint32_t acc = tacc + (d - 2) * 64;
-#pragma unroll
-          for (int i = 1; i <= kI8S; ++i) {  // i: B digit, j: Psi digit
-            const int j = d - i;
-            if (j < 1 || j > kI8S) continue;
-            const bool first = (g == 0) && (i == (d - 1 < kI8S ? 1 : d - kI8S));
-            umma_g1_ts(acc, tmem + ab * kG1ABuf + (j - 1) * 8,
-                       db0 + (uint64_t)(((i - 1) * kG1SliceB + kq * 32) >> 4), first ? 0u : 1u);
-          }
-        }
+        // B's digit slices i .. i + w - 1 are consecutive 64-row SWIZZLE_128B tiles (8 KB each), i.e. one
+        // K-major tile of 64 w rows, and the diagonal accumulators d = i + j .. i + j + w - 1 are consecutive
+        // 64-column TMEM blocks: one MMA of N = 64 w (w <= 3) computes the w digit pairs (i .. i + w - 1, j)
+        // straight into their diagonals (9 MMAs per quarter block instead of 21). The j = 1 MMAs touch every
+        // diagonal first (accumulate = 0 at g = 0).
+        g1_wide_mmas<3>(tacc, tmem + ab * kG1ABuf, db0, kq, g == 0);
         umma_commit(&afree[ab]);                      // A buffer ab may take quarter block g + 2
         if (kq == 3 || g + 1 == nhalf) umma_commit(&bempty[s]);
       }
       umma_commit(&done);
-      if (p.dbgbuf && lane == 0) {
-        p.dbgbuf[blockIdx.x * 8 + 0] = w_b;
-        p.dbgbuf[blockIdx.x * 8 + 1] = w_a;
-        p.dbgbuf[blockIdx.x * 8 + 2] = tclk<kT>() - t0;
-      }
     }
   } else {  // workers: Psi digits into TMEM, column norms; at the end the accumulators into FP64 partials
     pdl_wait();
@@ -765,13 +693,10 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
     const bool zc = E == 0;                   // an all-zero orbital (or none): zero digits
     const double sc41 = zc ? 0.0 : ldexp(1.0, 41 - (E - 1022));  // x 2^41 / tau_s: |v sc41| < 2^41
     double nrm = 0.0;
-    long long w_p = 0, w_f = 0, w_s = 0;
     const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
     for (int g = 0, s = 0, ph = 0; g < nhalf; ++g) {  // s = g % kG1PsiSlots, ph = (g / kG1PsiSlots) & 1
       const int ab = g & 1;
-      long long c2 = tclk<kT>();
       mbar_wait(&pfull[s], (uint32_t)ph);
-      w_p += tclk<kT>() - c2;
       const long long ra = r0 + (long long)g * kG1Half;
       // this lane's component of Psi[row][sIdx] (Re for cm = 0, Im for cm = 1): 8-byte loads, 2 norb per row
       const double* P = reinterpret_cast<const double*>(Psm + s * kG1PsiB) + 2 * sIdx + cm;
@@ -806,27 +731,15 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(&pempty[s]);  // this warp is done with the Psi rows
-      long long c3 = tclk<kT>();
-      if (g >= 2) {  // MMAs of block g - 2 are done with it
-        if (p.sleep) mbar_wait_sleep(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));
-        else mbar_wait(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));
-      }
-      w_f += tclk<kT>() - c3;
+      if (g >= 2) mbar_wait(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));  // MMAs of block g - 2 are done with it
       tc_fence_after();
-      const long long c4 = tclk<kT>();
 #pragma unroll
       for (int i = 0; i < kI8S; ++i) tmem_st2(trow + ab * kG1ABuf + i * 8 + 2 * h, dg[i]);
       asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
       tc_fence_before();
       __syncwarp();
-      w_s += tclk<kT>() - c4;
       if (lane == 0) mbar_arrive(&afull[ab]);
       if (++s == kG1PsiSlots) { s = 0; ph ^= 1; }
-    }
-    if (p.dbgbuf && lane == 0) {
-      atomicAdd((unsigned long long*)&p.dbgbuf[blockIdx.x * 8 + 3], (unsigned long long)w_p);
-      atomicAdd((unsigned long long*)&p.dbgbuf[blockIdx.x * 8 + 4], (unsigned long long)w_f);
-      atomicAdd((unsigned long long*)&p.dbgbuf[blockIdx.x * 8 + 5], (unsigned long long)w_s);
     }
     // column norms: Re^2 (even lane) + Im^2 (odd lane), then a fixed-order sum over the 4 row groups
     nrm += __shfl_xor_sync(0xffffffffu, nrm, 1);
@@ -904,8 +817,7 @@ cudaError_t launch_bslice1_i8(const double2* B, int ndom, int nproj, long long n
 }
 cudaError_t launch_gemm1_i8(const Gemm1I8Args& a, cudaStream_t st) {
   dim3 grid(a.nsplit, a.ndom);
-  if (a.dbgbuf) launch_k(k_gemm1_i8<true>, grid, kG1Threads, kG1Smem, st, a);
-  else launch_k(k_gemm1_i8<false>, grid, kG1Threads, kG1Smem, st, a);
+  launch_k(k_gemm1_i8, grid, kG1Threads, kG1Smem, st, a);
   return cudaGetLastError();
 }
 
@@ -941,9 +853,7 @@ cudaError_t launch_gemm2_i8(const Gemm2Args& a, cudaStream_t st) {
 cudaError_t gemm_i8_set_attributes() {
   cudaError_t e = cudaFuncSetAttribute(k_gemm2_i8<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kI8Smem);
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_gemm1_i8<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kG1Smem);
-  if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_gemm1_i8<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kG1Smem);
+  e = cudaFuncSetAttribute(k_gemm1_i8, cudaFuncAttributeMaxDynamicSharedMemorySize, kG1Smem);
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(k_gemm2_i8<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kI8Smem);
 }

@@ -2,19 +2,11 @@
 // entry point, so the library needs no libcuda link). Used by the stencil and GEMM kernels.
 #include "lfd_internal.h"
 
-#include <cstdlib>
-
 namespace lfd {
 
 thread_local bool g_pdl_suspended = false;  // set while a CUDA graph is captured (plain edges measured faster)
 
-bool pdl_enabled() {
-  static const bool on = [] {
-    const char* v = std::getenv("LFD_PDL");
-    return !(v && v[0] == '0');
-  }();
-  return on && !g_pdl_suspended;
-}
+bool pdl_enabled() { return !g_pdl_suspended; }
 
 void pdl_suspend(bool s) { g_pdl_suspended = s; }
 bool pdl_suspended() { return g_pdl_suspended; }

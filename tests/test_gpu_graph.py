@@ -115,14 +115,14 @@ def test_graph_after_occupation_change():
 
 
 @pytest.mark.parametrize("name,steps,chunks", [("P0", 40, (5, 35)), ("C1", 12, (1, 11))])
-def test_graph_bitwise_with_int8_gemms(name, steps, chunks, monkeypatch):
+def test_graph_bitwise_with_int8_gemms(name, steps, chunks):
     """the int8-digit tensor-core GEMMs (forced on these small grids) under capture: the orbital-exponent
     handshake (k_kin_yz -> k_gemm1_i8, cleared by its last CTA) and the completion counters replay exactly"""
-    monkeypatch.setenv("LFD_NL_I8", "1")
+    from paper_conf_ipps_razakhllknvn24_b200 import lfd
     w = workload(name)
     x = make_inputs(w, seed=44)
     A = np.stack([midpoint_A(w, n) for n in range(steps)])
-    a = _eager(w, x, A)
-    b = _graph(w, x, A, chunks)
+    a = _eager(w, x, A, flags=lfd.LFD_FLAG_NL_I8)
+    b = _graph(w, x, A, chunks, flags=lfd.LFD_FLAG_NL_I8)
     for u, v in zip(a, b):
         assert np.array_equal(u, v)

@@ -397,3 +397,41 @@ def test_density_kernel_shapes(name, knobs, monkeypatch):
     x = make_inputs(w, seed=71)
     A = lambda n: midpoint_A(w, n)  # noqa: E731
     assert_parity(w, run_gpu(w, x, 2, A), run_ref(w, x, 2, A))
+
+
+def test_c2_contract_100_steps():
+    """The north-star contract at the bench configuration: C2 (70x70x72, 64 orbitals, 64 projectors, laser;
+    the default int8-digit GEMMs that bench.py times) for 100 steps. The oracle runs the same 100 steps on 6
+    orbital columns spread over both halves of the orbital range (orbitals evolve independently under Eq. 6,
+    so these are exactly those columns of a full run; tests/_oracle_par.py), compared at 1e-10 in Psi; rho, j
+    and J of those columns (occupations moved onto them with lfd_set_occupations) at 1e-10."""
+    torch = _torch()
+    from oracle import ref
+    from paper_conf_ipps_razakhllknvn24_b200 import Context, lfd
+    from tests._oracle_par import oracle_columns
+    w = workload("C2")
+    x = make_inputs(w, seed=5)
+    cols = [0, 1, 17, 31, 32, 63]
+    steps = 100
+    dev = torch.device("cuda:0")
+    psi = torch.from_numpy(x.psi0.copy()).to(dev)
+    ctx = Context(psi, torch.from_numpy(x.proj).to(dev), x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc)
+    assert lfd.lfd_nl_path(ctx.ctx) == 1  # the bench configuration: int8-digit tensor-core GEMMs
+    ctx.set_potential(torch.from_numpy(x.vloc).to(dev))
+    for n in range(steps):
+        ctx.set_vector_potential(midpoint_A(w, n))
+        ctx.step(1)
+    occ = np.zeros((1, w.norb))
+    occ[0, cols] = 2.0
+    ctx.set_occupations(occ)
+    rho, j, J = ctx.density_current()
+    ctx.sync()
+    got = psi.cpu().numpy()[..., cols]
+    rho, j, J = rho.cpu().numpy().reshape(1, -1), j.cpu().numpy().reshape(1, 3, -1), J.cpu().numpy()
+    ctx.close()
+    want, A = oracle_columns("C2", 5, cols, steps)
+    cfg = ref.RefConfig(1, w.nx, w.ny, w.nz, w.hx, w.hy, w.hz, w.bc, len(cols), w.nproj, w.dt)
+    rr, jr, Jr = ref.density_current(cfg, want, np.full((1, len(cols)), 2.0), A)
+    ws = w.with_(norb=len(cols))
+    errs = assert_parity(ws, (got, rho, j, J), (want, rr, jr, Jr))
+    print(f"C2 100 steps (int8 GEMMs) vs oracle: psi {errs[0]:.2e} rho {errs[1]:.2e} j {errs[2]:.2e} J {errs[3]:.2e}")

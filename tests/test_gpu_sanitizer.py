@@ -1,6 +1,8 @@
 """compute-sanitizer over every kernel variant: memcheck (out-of-bounds / misaligned
-accesses) and racecheck (shared-memory hazards, the concern of the in-place sweeps) on tiny
-shapes driven by tools/sanitize_drive.py; the drive itself asserts no NaN appears in Psi."""
+accesses), racecheck (shared-memory hazards, the concern of the in-place sweeps), synccheck (barrier
+misuse) and initcheck (reads of uninitialised device memory), on tiny shapes driven by
+tools/sanitize_drive.py in three modes: the FP64 DMMA kernels, the int8-digit tcgen05 GEMMs forced, and
+the SP variant. The drive itself asserts no NaN appears in Psi."""
 import os
 import shutil
 import subprocess
@@ -13,13 +15,15 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 SAN = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
 
 
-@pytest.mark.parametrize("tool", ["memcheck", "racecheck"])
-def test_compute_sanitizer_clean(tool):
+@pytest.mark.parametrize("mode", ["dmma", "i8", "sp"])
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck", "initcheck"])
+def test_compute_sanitizer_clean(tool, mode):
     if not os.path.exists(SAN):
         pytest.skip("compute-sanitizer not found")
-    r = subprocess.run([SAN, "--tool", tool, "--error-exitcode", "17", sys.executable,
-                        os.path.join(ROOT, "tools", "sanitize_drive.py")],
-                       capture_output=True, text=True, timeout=900)
+    extra = ["--track-unused-memory", "no"] if tool == "initcheck" else []
+    r = subprocess.run([SAN, "--tool", tool, *extra, "--error-exitcode", "17", sys.executable,
+                        os.path.join(ROOT, "tools", "sanitize_drive.py"), mode],
+                       capture_output=True, text=True, timeout=1200)
     out = r.stdout + r.stderr
     assert r.returncode == 0 and "sanitize drive ok" in out, out[-4000:]
     assert ("ERROR SUMMARY: 0 errors" in out or "(0 errors, 0 warnings)" in out), out[-4000:]

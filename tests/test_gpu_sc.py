@@ -36,14 +36,14 @@ def _ref(w, x, steps, flags, n_corr, exact=False, adot0=(3.0, -2.0, 1.0)):
     return st
 
 
-def _gpu(w, x, steps, flags, n_corr, exact=False, adot0=(3.0, -2.0, 1.0), chunks=(None,), nccl=False):
+def _gpu(w, x, steps, flags, n_corr, exact=False, adot0=(3.0, -2.0, 1.0), chunks=(None,), nccl=False, ctx_flags=0):
     import torch
     from paper_conf_ipps_razakhllknvn24_b200 import Context, lfd
     dev = torch.device("cuda:0")
     psi = torch.from_numpy(x.psi0.copy()).to(dev)
     proj = torch.from_numpy(x.proj).to(dev) if w.nproj else None
     ctx = Context(psi, proj, x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc,
-                  flags=lfd.LFD_FLAG_EXACT_NL if exact else 0)
+                  flags=(lfd.LFD_FLAG_EXACT_NL if exact else 0) | ctx_flags)
     offs, gd = domain_tiling(w.ndom, (w.nx, w.ny, w.nz))
     vion = torch.from_numpy(x.vloc.copy()).to(dev)
     A = aext_half(w, steps)
@@ -85,14 +85,14 @@ def test_sc_parity(name, steps, flags, n_corr):
 
 
 @pytest.mark.parametrize("name,n_corr", [("P0", 1), ("C3", 2)])
-def test_sc_parity_int8_gemms(name, n_corr, monkeypatch):
+def test_sc_parity_int8_gemms(name, n_corr):
     """the self-consistent step with both nonlocal GEMMs on the int8-digit tensor-core path (forced on these
     small grids): the out-of-place first factor S = N(Psi(t_n)), the exponent handshake across sweeps"""
-    monkeypatch.setenv("LFD_NL_I8", "1")
+    from paper_conf_ipps_razakhllknvn24_b200 import lfd
     w = workload(name).with_(vnoise=0.02) if name == "C3" else workload(name)
     x = make_inputs(w, seed=63)
     steps = 2 if name == "C3" else 12
-    assert_sc_parity(_gpu(w, x, steps, ALL, n_corr), _ref(w, x, steps, ALL, n_corr))
+    assert_sc_parity(_gpu(w, x, steps, ALL, n_corr, ctx_flags=lfd.LFD_FLAG_NL_I8), _ref(w, x, steps, ALL, n_corr))
 
 
 def test_sc_parity_c3_eight_domains():
