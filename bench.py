@@ -485,10 +485,15 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_ipps_razakhllknvn24_b200 import Context, lfd
+    from paper_conf_ipps_razakhllknvn24_b200 import dist as ldist
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
+        # NCCL's communicator set-up lines (rank count, transports, NVLS) on stderr, for the record
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
         dist.init_process_group("nccl", device_id=dev)
     x = make_inputs(w, seed=args.seed + rank)
     stream = torch.cuda.current_stream()
@@ -500,23 +505,30 @@ def main():
     nd, ng = w.ndom, w.ngrid
     rho = torch.empty((nd, ng), dtype=torch.float64, device=dev)
     J = torch.empty((nd, 3), dtype=torch.float64, device=dev)
-    # global gather buffer of the DC recombination: [world][nd*(ng+3)]
-    send = torch.empty(nd * (ng + 3), dtype=torch.float64, device=dev)
-    recv = torch.empty(world * nd * (ng + 3), dtype=torch.float64, device=dev) if world > 1 else None
+    # N > 1: the DC recombination of [rho | J] (all-gather over NCCL) runs on a side stream, double buffered,
+    # overlapped with the next step's first nonlocal factor (lfd_step_prologue; it needs only Psi, B, D); the
+    # main stream waits for the gather before the next step's v / A (which a real run derives from it)
+    gat = ldist.OverlappedGather(nd * (ng + 3), world, dev) if world > 1 else None
     A_seq = [midpoint_A(w, n) for n in range(args.warmup + args.steps)]
 
-    def step(n):
+    def step(n, last=False):
+        if gat is not None and n > 0:
+            gat.wait(n - 1)
         lfd.lfd_set_vector_potential(ctx.ctx, A_seq[n])
         lfd.lfd_set_potential(ctx.ctx, v_dev)
         lfd.lfd_step(ctx.ctx, 1)
-        if world > 1:
+        if gat is not None:
+            gat.before_write(n)
+            send = gat.send[gat.slot(n)]
             lfd.lfd_density_current(ctx.ctx, send[: nd * ng], None, send[nd * ng:])
-            dist.all_gather_into_tensor(recv, send)
+            gat.start(n)
+            if not last:
+                lfd.lfd_step_prologue(ctx.ctx)
         else:
             lfd.lfd_density_current(ctx.ctx, rho, None, J)
 
     for n in range(args.warmup):
-        step(n)
+        step(n, last=n + 1 == args.warmup)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -527,7 +539,9 @@ def main():
     with Clocks(local) as clk:
         e0.record(stream)
         for n in range(args.steps):
-            step(args.warmup + n)
+            step(args.warmup + n, last=n + 1 == args.steps)
+        if gat is not None:
+            gat.wait(args.warmup + args.steps - 1)
         e1.record(stream)
         torch.cuda.synchronize()
     launches = lfd.lfd_launch_count(ctx.ctx) - l0
@@ -545,7 +559,7 @@ def main():
     torch.cuda.synchronize()
     p0 = time.perf_counter()
     for n in range(args.steps):
-        step(args.warmup + n)
+        step(args.warmup + n, last=n + 1 == args.steps)
     torch.cuda.synchronize()
     prof = lfd.lfd_profile_read(ctx.ctx)
     lfd.lfd_profile_enable(ctx.ctx, False)
@@ -683,8 +697,9 @@ def main():
             lfd.lfd_step(ctx.ctx, 1)
             lfd.lfd_density_current_host(ctx.ctx, rh, Jh)
             if world > 1:
+                send = gat.send[0]
                 lfd.lfd_density_current(ctx.ctx, send[: nd * ng], None, send[nd * ng:])
-                dist.all_gather_into_tensor(recv, send)
+                dist.all_gather_into_tensor(gat.recv[0], send)
             lfd.lfd_sync(ctx.ctx)  # the host reads this step's rho / J
             _ = float(Jh[0, 2])
         f1.record(stream)

@@ -161,6 +161,14 @@ lfd_status lfd_set_vector_potential(lfd_ctx* ctx, const double* A);
 /* Enqueue nsteps LFD steps (Eq. 6) with the current v_loc and A. nsteps == 0 is a no-op; < 0 EINVAL. */
 lfd_status lfd_step(lfd_ctx* ctx, int32_t nsteps);
 
+/* Enqueue the FIRST nonlocal factor of the next Eq.-6 step now (Psi <- N(Psi)). It depends only on Psi,
+ * B, D and Delta -- not on v_loc or A -- so a caller can run it before the inputs of the step are known, e.g.
+ * while the previous step's density is being all-gathered across ranks; the next lfd_step /
+ * lfd_step_sequence then starts with the local factor. The result is bitwise that of the plain call order.
+ * Until that step, Psi holds the intermediate N(Psi): lfd_density_current*, lfd_energy, lfd_remap_occ,
+ * lfd_step_graph, lfd_sc_*, lfd_psi_modified and a second prologue return LFD_ESTATE. */
+lfd_status lfd_step_prologue(lfd_ctx* ctx);
+
 /* Enqueue nsteps LFD steps with one vector potential per step, A_seq HOST double [nsteps][ndom][3]
  * (captured by value; step n uses A_seq[n], Eq. 4 midpoints), and the current v_loc. The result equals
  * nsteps x (lfd_set_vector_potential(A_seq[n]); lfd_step(1)) up to roundoff: the second nonlocal

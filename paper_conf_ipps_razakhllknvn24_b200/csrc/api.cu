@@ -289,6 +289,9 @@ struct lfd_ctx {
   // instead of GEMM-1 (cleared by the local propagator, lfd_psi_modified and LFD_FLAG_NO_CARRY).
   bool c_valid = false;
   bool carry = true;
+  // lfd_step_prologue: the first nonlocal factor of the next step has been applied already (Psi = N(Psi(t_n)));
+  // the next lfd_step / lfd_step_sequence starts with the local factor. Observers of Psi are refused meanwhile.
+  bool nl_pending = false;
   // int8-digit GEMM-1: the orbital exponents in the workspace describe the current Psi (set by the K_y K_z
   // pass that wrote it, consumed -- and cleared on the device -- by GEMM-1)
   bool colE_valid = false;
@@ -1053,10 +1056,20 @@ lfd_status lfd_step(lfd_ctx* c, int32_t nsteps) {
   if (nsteps < 0) return fail(c, LFD_EINVAL, "nsteps must be >= 0");
   DeviceGuard dg(c->device);
   for (int it = 0; it < nsteps; ++it) {
-    if (c->g.nproj > 0) LFD_TRY(nl_half(c));
+    if (c->g.nproj > 0 && !c->nl_pending) LFD_TRY(nl_half(c));
+    c->nl_pending = false;
     LFD_TRY(local_prop(c));
     if (c->g.nproj > 0) LFD_TRY(nl_half(c));
   }
+  return LFD_OK;
+}
+
+lfd_status lfd_step_prologue(lfd_ctx* c) {
+  LFD_TRY(check_ctx(c));
+  if (c->nl_pending) return fail(c, LFD_ESTATE, "a step prologue is already pending");
+  DeviceGuard dg(c->device);
+  if (c->g.nproj > 0) LFD_TRY(nl_half(c));
+  c->nl_pending = true;
   return LFD_OK;
 }
 
@@ -1070,7 +1083,8 @@ lfd_status lfd_step_sequence(lfd_ctx* c, int32_t nsteps, const double* A_seq) {
   const bool nl = c->g.nproj > 0;
   for (int n = 0; n < nsteps; ++n) {
     LFD_TRY(set_A(c, A_seq + 3LL * c->g.ndom * n));
-    if (nl && n == 0) LFD_TRY(nl_half(c));  // first factor of the sequence
+    if (nl && n == 0 && !c->nl_pending) LFD_TRY(nl_half(c));  // first factor of the sequence
+    c->nl_pending = false;
     LFD_TRY(local_prop(c));
     if (nl) LFD_TRY(nl_half(c, n + 1 < nsteps));  // N of step n fused with N of step n+1
   }
@@ -1079,6 +1093,7 @@ lfd_status lfd_step_sequence(lfd_ctx* c, int32_t nsteps, const double* A_seq) {
 
 lfd_status lfd_step_graph(lfd_ctx* c, int32_t nsteps, const double* A_seq, double* rho, double* Jmac_seq) {
   LFD_TRY(check_ctx(c));
+  if (c->nl_pending) return fail(c, LFD_ESTATE, "Psi is between lfd_step_prologue and its step");
   if (nsteps < 0) return fail(c, LFD_EINVAL, "nsteps must be >= 0");
   if (nsteps > 0 && !A_seq) return fail(c, LFD_EINVAL, "A_seq is NULL");
   for (long long i = 0; i < 3LL * c->g.ndom * nsteps; ++i)
@@ -1115,6 +1130,7 @@ lfd_status lfd_step_graph(lfd_ctx* c, int32_t nsteps, const double* A_seq, doubl
 
 lfd_status lfd_density_current(lfd_ctx* c, double* rho, double* j, double* Jmac) {
   LFD_TRY(check_ctx(c));
+  if (c->nl_pending) return fail(c, LFD_ESTATE, "Psi is between lfd_step_prologue and its step");
   if (!rho) return fail(c, LFD_EINVAL, "rho is NULL");
   DeviceGuard dg(c->device);
   if (!is_device_ptr(rho) || (j && !is_device_ptr(j)) || (Jmac && !is_device_ptr(Jmac)))
@@ -1127,6 +1143,7 @@ lfd_status lfd_density_current(lfd_ctx* c, double* rho, double* j, double* Jmac)
 lfd_status lfd_density_current_global(lfd_ctx* c, double* rho_g, double* j_g, double* Jmac, const int32_t* off,
                                       const int32_t* gdims) {
   LFD_TRY(check_ctx(c));
+  if (c->nl_pending) return fail(c, LFD_ESTATE, "Psi is between lfd_step_prologue and its step");
   if (!rho_g || !off || !gdims) return fail(c, LFD_EINVAL, "rho_g, dom_offset and gdims must be non-NULL");
   const Geometry& g = c->g;
   for (int i = 0; i < 3; ++i)
@@ -1157,6 +1174,7 @@ lfd_status lfd_density_current_global(lfd_ctx* c, double* rho_g, double* j_g, do
 
 lfd_status lfd_density_current_host(lfd_ctx* c, double* rho_host, double* Jmac_host) {
   LFD_TRY(check_ctx(c));
+  if (c->nl_pending) return fail(c, LFD_ESTATE, "Psi is between lfd_step_prologue and its step");
   DeviceGuard dg(c->device);
   const Geometry& g = c->g;
   double* rs = c->at<double>(c->L.rhostage);
@@ -1176,6 +1194,7 @@ lfd_status lfd_density_current_host(lfd_ctx* c, double* rho_host, double* Jmac_h
 
 lfd_status lfd_energy(lfd_ctx* c, double* E) {
   LFD_TRY(check_ctx(c));
+  if (c->nl_pending) return fail(c, LFD_ESTATE, "Psi is between lfd_step_prologue and its step");
   if (!E) return fail(c, LFD_EINVAL, "E is NULL");
   DeviceGuard dg(c->device);
   if (!is_device_ptr(E)) return fail(c, LFD_EINVAL, "E must be device memory");
@@ -1195,6 +1214,7 @@ lfd_status lfd_energy(lfd_ctx* c, double* E) {
 
 lfd_status lfd_remap_occ(lfd_ctx* c, const void* ref, int32_t nref, double* occ_out) {
   LFD_TRY(check_ctx(c));
+  if (c->nl_pending) return fail(c, LFD_ESTATE, "Psi is between lfd_step_prologue and its step");
   if (!ref || !occ_out) return fail(c, LFD_EINVAL, "ref and occ_out must be non-NULL");
   if (nref < 1 || nref > c->L.nref_cap) return fail(c, LFD_EINVAL, "nref must be in [1, nref_max]");
   if (reinterpret_cast<uintptr_t>(ref) & (c->celem() - 1))
@@ -1237,6 +1257,7 @@ lfd_status lfd_sc_workspace_size(const lfd_ctx* c, const lfd_sc_config* sc, size
 lfd_status lfd_sc_init(lfd_ctx* c, const lfd_sc_config* sc, const double* vion, void* ws, size_t ws_bytes,
                        const double* Aext0, const double* A_ind0, const double* Adot0) {
   LFD_TRY(check_ctx(c));
+  if (c->nl_pending) return fail(c, LFD_ESTATE, "Psi is between lfd_step_prologue and its step");
   std::string why;
   lfd_status st = sc_validate(c, sc, why);
   if (st != LFD_OK) return fail(c, st, why);
@@ -1320,6 +1341,7 @@ lfd_status lfd_sc_init(lfd_ctx* c, const lfd_sc_config* sc, const double* vion, 
 
 lfd_status lfd_sc_step(lfd_ctx* c, int32_t nsteps, const double* Aext) {
   LFD_TRY(check_ctx(c));
+  if (c->nl_pending) return fail(c, LFD_ESTATE, "Psi is between lfd_step_prologue and its step");
   ScState& S = c->sc;
   if (!S.ready) return fail(c, LFD_ESTATE, "lfd_sc_init has not been called");
   if (nsteps < 0) return fail(c, LFD_EINVAL, "nsteps must be >= 0");
@@ -1432,6 +1454,7 @@ lfd_status lfd_sc_comm_init(lfd_ctx* c, int32_t nranks, int32_t rank, const void
 
 lfd_status lfd_psi_modified(lfd_ctx* c) {
   LFD_TRY(check_ctx(c));
+  if (c->nl_pending) return fail(c, LFD_ESTATE, "Psi is between lfd_step_prologue and its step");
   c->c_valid = false;
   if (c->colE_valid) {  // orbital exponents of a Psi that no longer exists: clear them (stream order)
     DeviceGuard dg(c->device);

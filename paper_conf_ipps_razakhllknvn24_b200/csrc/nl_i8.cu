@@ -464,10 +464,14 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
         mbar_wait(&pfull[s], (uint32_t)((u / kI8PsiSlots) & 1));
         const double* ps = reinterpret_cast<const double*>(Psm + s * kI8SubB) + n;
         const double* sg = reinterpret_cast<const double*>(Psm + s * kI8SubB + kI8SubRowsB);
+        if (nvalid) {  // running row pointers (16 precomputed row offsets would spill)
+          double* po = pout + r0 * ld;
 #pragma unroll
-        for (int c = 0; c < kI8Rows; ++c) {
-          if (!nvalid || c >= nc) continue;
-          pout[(r0 + c) * ld] = fma(nf, ps[c * ld], scale_pow2(fa[c], sg[c], tau));
+          for (int c = 0; c < kI8Rows; ++c) {
+            if (c < nc) *po = fma(nf, *ps, scale_pow2(fa[c], sg[c], tau));
+            po += ld;
+            ps += ld;
+          }
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&pempty[s]);

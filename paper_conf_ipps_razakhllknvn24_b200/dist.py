@@ -62,3 +62,78 @@ def gather(send, world: int, group=None):
     recv = torch.empty(world * send.numel(), dtype=send.dtype, device=send.device)
     dist.all_gather_into_tensor(recv, send, group=group)
     return recv
+
+
+class OverlappedGather:
+    """The per-step DC recombination (all-gather of every rank's packed [rho | J]) on a side stream, double
+    buffered, so it overlaps the next step's first nonlocal factor (lfd_step_prologue: it needs only Psi, B
+    and D, not the v / A the gathered density feeds).
+
+    Per step k:  slot = g.slot(k)  -> the density kernel writes g.send[slot] on the main stream;
+                 g.start(k)        -> the all-gather of g.send[slot] into g.recv[slot] on the side stream;
+                 ... main stream: lfd_step_prologue (overlaps the collective) ...
+                 g.wait(k)         -> the main stream waits for it (before anything reads recv[slot]).
+    A send slot is rewritten two steps later; start() makes the side stream, and slot() the main stream, wait
+    for the previous user of that slot. On CPU tensors (gloo) there are no streams: start() is synchronous."""
+
+    def __init__(self, numel: int, world: int, device, dtype=None, group=None):
+        import torch
+        dtype = dtype or torch.float64
+        self.world, self.group = world, group
+        self.send = [torch.empty(numel, dtype=dtype, device=device) for _ in range(2)]
+        self.recv = [torch.empty(world * numel, dtype=dtype, device=device) for _ in range(2)]
+        self.cuda = torch.device(device).type == "cuda"
+        if self.cuda:
+            self.side = torch.cuda.Stream(device=device)
+            self.done = [None, None]
+
+    @staticmethod
+    def slot(k: int) -> int:
+        return k & 1
+
+    def before_write(self, k: int):
+        """The main stream must not overwrite send[slot] while the gather that read it two steps ago runs."""
+        if self.cuda and self.done[self.slot(k)] is not None:
+            import torch
+            torch.cuda.current_stream().wait_event(self.done[self.slot(k)])
+
+    def start(self, k: int):
+        import torch
+        import torch.distributed as dist
+        s = self.slot(k)
+        if not self.cuda:
+            dist.all_gather_into_tensor(self.recv[s], self.send[s], group=self.group)
+            return
+        ready = torch.cuda.Event()
+        ready.record(torch.cuda.current_stream())
+        self.side.wait_event(ready)
+        with torch.cuda.stream(self.side):
+            dist.all_gather_into_tensor(self.recv[s], self.send[s], group=self.group)
+            ev = torch.cuda.Event()
+            ev.record(self.side)
+        self.done[s] = ev
+
+    def wait(self, k: int):
+        if self.cuda and self.done[self.slot(k)] is not None:
+            import torch
+            torch.cuda.current_stream().wait_event(self.done[self.slot(k)])
+        return self.recv[self.slot(k)]
+
+
+def allgather_occupations(occ_local, counts, group=None, device="cpu"):
+    """The per-MD-step occupation handshake across ranks (only the occupation numbers f cross
+    between QXMD and LFD): every rank contributes f of its domains [ndom_r][norb] and receives
+    f of all domains [ndom_total][norb] (rank-major, i.e. global domain order of `partition`). Blocks are
+    padded to the largest rank's (all-gather needs equal sizes). Returns a host float64 array."""
+    import torch
+    import torch.distributed as dist
+    occ_local = np.ascontiguousarray(occ_local, dtype=np.float64)
+    world = len(counts)
+    norb = occ_local.shape[1]
+    blk = max(counts) * norb
+    send = torch.zeros(blk, dtype=torch.float64, device=device)
+    send[: occ_local.size] = torch.from_numpy(occ_local.reshape(-1)).to(device)
+    recv = torch.empty(world * blk, dtype=torch.float64, device=device)
+    dist.all_gather_into_tensor(recv, send, group=group)
+    r = recv.cpu().numpy()
+    return np.concatenate([r[i * blk: i * blk + counts[i] * norb].reshape(counts[i], norb) for i in range(world)])

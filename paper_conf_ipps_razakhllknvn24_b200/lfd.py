@@ -33,7 +33,7 @@ LFD_SC_HARTREE = 1
 LFD_SC_XC = 2
 LFD_SC_MAXWELL = 4
 EXPORTS = ("lfd_workspace_size", "lfd_init", "lfd_set_potential", "lfd_set_potential_host",
-           "lfd_set_vector_potential", "lfd_step", "lfd_step_sequence", "lfd_density_current", "lfd_density_current_global",
+           "lfd_set_vector_potential", "lfd_step", "lfd_step_prologue", "lfd_step_sequence", "lfd_density_current", "lfd_density_current_global",
            "lfd_density_current_host", "lfd_energy", "lfd_remap_occ", "lfd_psi_modified", "lfd_set_occupations", "lfd_set_stream", "lfd_sync",
            "lfd_launch_count", "lfd_nl_path", "lfd_profile_enable", "lfd_profile_read", "lfd_last_error", "lfd_destroy",
            "lfd_sc_workspace_size", "lfd_sc_init", "lfd_sc_step", "lfd_sc_read", "lfd_comm_unique_id",
@@ -78,6 +78,7 @@ def load():
         "lfd_set_potential_host": [P, P],
         "lfd_set_vector_potential": [P, P],
         "lfd_step": [P, I32],
+        "lfd_step_prologue": [P],
         "lfd_step_sequence": [P, I32, P],
         "lfd_density_current": [P, P, P, P],
         "lfd_density_current_global": [P, P, P, P, P, P],
@@ -184,6 +185,10 @@ def lfd_set_vector_potential(ctx, A):
 
 def lfd_step(ctx, nsteps: int = 1):
     _check(load().lfd_step(ctx, int(nsteps)), ctx)
+
+
+def lfd_step_prologue(ctx):
+    _check(load().lfd_step_prologue(ctx), ctx)
 
 
 def lfd_step_sequence(ctx, A_seq):

@@ -130,6 +130,8 @@ def test_i8_large_scissor_gemm_accuracy(name):
     of the int8-digit emulation, ~2^-40 of the row x column scales) are printed."""
     w = workload(name)
     x = make_inputs(w, seed=9)
+    # projectors overlapping the propagated orbitals (B = B_u + Psi_0 columns: C = O(1) from the first step)
+    x.proj = np.ascontiguousarray(x.proj + x.psi0[..., : w.nproj])
     d = np.ascontiguousarray(np.where(np.arange(x.dnl.size).reshape(x.dnl.shape) % 2, -1.0, 1.0)
                              * 0.3 / (0.5 * w.dt))
     A = laser(w)

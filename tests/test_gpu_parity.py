@@ -435,3 +435,41 @@ def test_c2_contract_100_steps():
     ws = w.with_(norb=len(cols))
     errs = assert_parity(ws, (got, rho, j, J), (want, rr, jr, Jr))
     print(f"C2 100 steps (int8 GEMMs) vs oracle: psi {errs[0]:.2e} rho {errs[1]:.2e} j {errs[2]:.2e} J {errs[3]:.2e}")
+
+
+def test_step_prologue_overlap_schedule_bitwise():
+    """The multi-GPU overlap schedule on one process (a dry run of bench.py's N > 1 loop): the first nonlocal
+    factor of step n+1 enqueued by lfd_step_prologue right after step n's density (where the density
+    all-gather would run on a side stream), then v / A and lfd_step. Bitwise equal to the serial call order
+    (same kernels, same data dependencies), and observers of Psi are refused while a prologue is pending."""
+    torch = _torch()
+    from paper_conf_ipps_razakhllknvn24_b200 import Context, lfd
+    w = workload("P0")
+    x = make_inputs(w, seed=14)
+    dev = torch.device("cuda:0")
+    outs = []
+    for overlap in (False, True):
+        psi = torch.from_numpy(x.psi0.copy()).to(dev)
+        ctx = Context(psi, torch.from_numpy(x.proj).to(dev), x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc)
+        v = torch.from_numpy(x.vloc).to(dev)
+        rhos, Js = [], []
+        for n in range(12):
+            lfd.lfd_set_vector_potential(ctx.ctx, midpoint_A(w, n))
+            lfd.lfd_set_potential(ctx.ctx, v)
+            lfd.lfd_step(ctx.ctx, 1)
+            rho, _, J = ctx.density_current()
+            rhos.append(rho.clone())
+            Js.append(J.clone())
+            if overlap and n < 11:
+                lfd.lfd_step_prologue(ctx.ctx)
+                if n == 3:
+                    with pytest.raises(lfd.LFDError) as e:
+                        ctx.density_current()
+                    assert e.value.status == -4
+                    with pytest.raises(lfd.LFDError):
+                        lfd.lfd_step_prologue(ctx.ctx)
+        ctx.sync()
+        outs.append((psi.cpu().numpy(), torch.stack(rhos).cpu().numpy(), torch.stack(Js).cpu().numpy()))
+        ctx.close()
+    for a, b in zip(*outs):
+        assert np.array_equal(a, b)

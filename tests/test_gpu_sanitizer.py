@@ -20,7 +20,7 @@ SAN = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitize
 def test_compute_sanitizer_clean(tool, mode):
     if not os.path.exists(SAN):
         pytest.skip("compute-sanitizer not found")
-    extra = ["--track-unused-memory", "no"] if tool == "initcheck" else []
+    extra = []
     r = subprocess.run([SAN, "--tool", tool, *extra, "--error-exitcode", "17", sys.executable,
                         os.path.join(ROOT, "tools", "sanitize_drive.py"), mode],
                        capture_output=True, text=True, timeout=1200)

@@ -163,3 +163,45 @@ def test_sc_two_ranks_equal_one_process():
     for r in res:
         assert np.abs(r[2] - st.A_ind).max() < 1e-12 and np.abs(r[3] - st.Adot).max() < 1e-12
         assert np.abs(r[4] - st.rho_g).max() < 1e-13
+
+
+def _occ_worker(rank, world, port, ndom, norb, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    mine = ldist.partition(ndom, rank, world)
+    counts = [len(ldist.partition(ndom, r, world)) for r in range(world)]
+    occ = np.array([[2.0 - 0.01 * (d * norb + s) for s in range(norb)] for d in mine]).reshape(len(mine), norb)
+    got = ldist.allgather_occupations(occ, counts)
+    # the overlapped (double-buffered) density gather on CPU tensors: two steps, slots alternate
+    g = ldist.OverlappedGather(4, world, "cpu")
+    outs = []
+    for k in range(3):
+        s = g.slot(k)
+        g.before_write(k)
+        g.send[s].copy_(torch.arange(4, dtype=torch.float64) + 10 * rank + 100 * k)
+        g.start(k)
+        outs.append(g.wait(k).clone().numpy())
+    q.put((rank, got, outs))
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("ndom", [2, 5])
+def test_occupation_handshake_and_overlapped_gather_two_ranks(ndom):
+    """The per-MD-step occupation all-gather gives every rank f of all domains in global order,
+    and the double-buffered side-stream density gather returns each step's blocks of both ranks."""
+    world, norb = 2, 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_occ_worker, args=(r, world, port, ndom, norb, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    want = np.array([[2.0 - 0.01 * (d * norb + s) for s in range(norb)] for d in range(ndom)])
+    for _, got, outs in res:
+        assert np.array_equal(got, want)
+        for k, o in enumerate(outs):
+            assert np.array_equal(o, np.concatenate([np.arange(4) + 100 * k, np.arange(4) + 10 + 100 * k]))
