@@ -32,6 +32,12 @@
  *                            nonlocal factor ON (tests/test_oracle_pins_step.py): closed form on
  *                            projector plane waves (lambda_u f_u^2, f_u = (1-i eps D_u)/|.|) and on a
  *                            two-column mix; first-order convergence to the same dense expm.
+ *   lfd_ref_nl_half_dense    pinned (tests/test_oracle_pins_dense.py): diagonal D equals lfd_ref_nl_half; a
+ *                            rotated diagonal D equals the diagonal factor on rotated projectors; the step
+ *                            converges (order 1) to dense expm(-i T (H_FD + V + B D B^H dV)).
+ *   lfd_ref_nl_half_exact_dense pinned: dense scipy expm of -i(Delta/2) B D B^H dV on orthonormal B; the
+ *                            exact dense step converges at second order to the same expm.
+ *   lfd_ref_energy_nl_dense  pinned: equals <psi| B D B^H dV |psi> with dense matrices.
  *   lfd_ref_density_current  pinned: plane-wave closed forms; sum rule; J = dE_kin/dA / V.
  *   lfd_ref_energy           pinned: plane-wave closed forms (kinetic, local = f mean(v)); nonlocal on
  *                            projector columns = f D_u; O(dt^2) energy drift of the step at A = D = 0.
@@ -312,6 +318,197 @@ int lfd_ref_step(const lfd_ref_config* c, double complex* psi, const double comp
       e |= lfd_ref_nl_half(&one, p, b, d);
       if (e) return -1;
     }
+  return 0;
+}
+
+/* ---------------------------------------------------------------------------------------------
+ * Dense Hermitian D. Eq. 5 puts the nonlocal ionic pseudopotential into
+ * v_nl; in Kleinman-Bylander form it is  v_nl = sum_{u,v} |b_u> D_uv <b_v|  with a Hermitian coupling
+ * matrix D (the scissor operator of Eq. 7, is the special case D = Delta_sci I). With
+ * <a|b> = dV sum_r conj(a_r) b_r (R12), Eq. 9's BLASified form reads
+ *   C = dV B^H Psi,   Psi' = Psi - i (Delta/2) B (D C),
+ * and N of Eq. 6 renormalises each orbital to its pre-factor norm (R11). Dm: [nproj][nproj] complex,
+ * row-major D[u][v], one domain. Both norms are direct grid sums.
+ * ------------------------------------------------------------------------------------------- */
+static void ref_project(const lfd_ref_config* c, const double complex* psi, const double complex* proj,
+                        double complex* C) {
+  const size_t ng = (size_t)c->nx * c->ny * c->nz;
+  const int no = c->norb, np = c->nproj;
+  const double dV = c->hx * c->hy * c->hz;
+  for (size_t k = 0; k < (size_t)np * no; ++k) C[k] = 0.0;
+  for (size_t r = 0; r < ng; ++r)
+    for (int u = 0; u < np; ++u) {
+      double complex bc = conj(proj[r * np + u]);
+      for (int s = 0; s < no; ++s) C[(size_t)u * no + s] += bc * psi[r * no + s];
+    }
+  for (size_t k = 0; k < (size_t)np * no; ++k) C[k] *= dV;
+}
+
+/* Psi += B Y (Y [nproj][norb]), the back-projection of Eq. 9. */
+static void ref_backproject(const lfd_ref_config* c, double complex* psi, const double complex* proj,
+                            const double complex* Y) {
+  const size_t ng = (size_t)c->nx * c->ny * c->nz;
+  const int no = c->norb, np = c->nproj;
+  for (size_t r = 0; r < ng; ++r)
+    for (int u = 0; u < np; ++u) {
+      double complex b = proj[r * np + u];
+      for (int s = 0; s < no; ++s) psi[r * no + s] += b * Y[(size_t)u * no + s];
+    }
+}
+
+int lfd_ref_nl_half_dense(const lfd_ref_config* c, double complex* psi, const double complex* proj,
+                          const double complex* Dm) {
+  if (ref_check(c) || !psi) return -1;
+  if (c->nproj == 0) return 0;
+  if (!proj || !Dm) return -1;
+  const size_t ng = (size_t)c->nx * c->ny * c->nz;
+  const int no = c->norb, np = c->nproj;
+  const double eps = 0.5 * c->dt;
+  double complex* C = malloc((size_t)np * no * sizeof(double complex));
+  double complex* Y = calloc((size_t)np * no, sizeof(double complex));
+  double* n0 = calloc((size_t)no, sizeof(double));
+  double* n1 = calloc((size_t)no, sizeof(double));
+  if (!C || !Y || !n0 || !n1) { free(C); free(Y); free(n0); free(n1); return -2; }
+  for (size_t r = 0; r < ng; ++r)
+    for (int s = 0; s < no; ++s) {
+      double complex v = psi[r * no + s];
+      n0[s] += creal(v) * creal(v) + cimag(v) * cimag(v);
+    }
+  ref_project(c, psi, proj, C);
+  for (int u = 0; u < np; ++u)  /* Y = -i eps D C */
+    for (int v = 0; v < np; ++v)
+      for (int s = 0; s < no; ++s) Y[(size_t)u * no + s] += -I * eps * Dm[(size_t)u * np + v] * C[(size_t)v * no + s];
+  ref_backproject(c, psi, proj, Y);
+  for (size_t r = 0; r < ng; ++r)
+    for (int s = 0; s < no; ++s) {
+      double complex v = psi[r * no + s];
+      n1[s] += creal(v) * creal(v) + cimag(v) * cimag(v);
+    }
+  for (int s = 0; s < no; ++s) {
+    double f = sqrt(n0[s] / n1[s]);
+    for (size_t r = 0; r < ng; ++r) psi[r * no + s] *= f;
+  }
+  free(C); free(Y); free(n0); free(n1);
+  return 0;
+}
+
+/* exp(M) of an n x n complex matrix by the textbook Taylor series with scaling and squaring:
+ * exp(M) = (exp(M / 2^k))^(2^k), ||M||_1 / 2^k <= 1/2, 30 Taylor terms (truncation < 1e-30). */
+static int ref_expm(int n, const double complex* M, double complex* E) {
+  double nrm = 0.0;
+  for (int j = 0; j < n; ++j) {
+    double col = 0.0;
+    for (int i = 0; i < n; ++i) col += cabs(M[(size_t)i * n + j]);
+    if (col > nrm) nrm = col;
+  }
+  int k = 0;
+  while (nrm > 0.5) { nrm *= 0.5; ++k; }
+  const double sc = ldexp(1.0, -k);
+  double complex* T = malloc((size_t)n * n * sizeof(double complex));
+  double complex* W = malloc((size_t)n * n * sizeof(double complex));
+  if (!T || !W) { free(T); free(W); return -2; }
+  for (int i = 0; i < n; ++i)
+    for (int j = 0; j < n; ++j) {
+      E[(size_t)i * n + j] = (i == j) ? 1.0 : 0.0;
+      T[(size_t)i * n + j] = (i == j) ? 1.0 : 0.0;
+    }
+  for (int t = 1; t <= 30; ++t) {  /* T <- T (M sc) / t ; E += T */
+    for (int i = 0; i < n; ++i)
+      for (int j = 0; j < n; ++j) {
+        double complex a = 0.0;
+        for (int l = 0; l < n; ++l) a += T[(size_t)i * n + l] * M[(size_t)l * n + j] * sc;
+        W[(size_t)i * n + j] = a / (double)t;
+      }
+    for (size_t q = 0; q < (size_t)n * n; ++q) { T[q] = W[q]; E[q] += W[q]; }
+  }
+  for (int it = 0; it < k; ++it) {  /* E <- E E */
+    for (int i = 0; i < n; ++i)
+      for (int j = 0; j < n; ++j) {
+        double complex a = 0.0;
+        for (int l = 0; l < n; ++l) a += E[(size_t)i * n + l] * E[(size_t)l * n + j];
+        W[(size_t)i * n + j] = a;
+      }
+    for (size_t q = 0; q < (size_t)n * n; ++q) E[q] = W[q];
+  }
+  free(T); free(W);
+  return 0;
+}
+
+/* The exactly unitary factor with a dense Hermitian D, for dV-orthonormal projector columns: v_nl =
+ * B D B^H dV acts on span(B) as the matrix D in the basis B, so exp(-i eps v_nl) = 1 + B (exp(-i eps D) - 1)
+ * B^H dV:  C = dV B^H Psi,  Psi' = Psi + B ((exp(-i eps D) - I) C). No renormalisation. One domain. */
+int lfd_ref_nl_half_exact_dense(const lfd_ref_config* c, double complex* psi, const double complex* proj,
+                                const double complex* Dm) {
+  if (ref_check(c) || !psi) return -1;
+  if (c->nproj == 0) return 0;
+  if (!proj || !Dm) return -1;
+  const int no = c->norb, np = c->nproj;
+  const double eps = 0.5 * c->dt;
+  double complex* M = malloc((size_t)np * np * sizeof(double complex));
+  double complex* E = malloc((size_t)np * np * sizeof(double complex));
+  double complex* C = malloc((size_t)np * no * sizeof(double complex));
+  double complex* Y = calloc((size_t)np * no, sizeof(double complex));
+  if (!M || !E || !C || !Y) { free(M); free(E); free(C); free(Y); return -2; }
+  for (size_t q = 0; q < (size_t)np * np; ++q) M[q] = -I * eps * Dm[q];
+  if (ref_expm(np, M, E)) { free(M); free(E); free(C); free(Y); return -2; }
+  for (int u = 0; u < np; ++u) E[(size_t)u * np + u] -= 1.0;
+  ref_project(c, psi, proj, C);
+  for (int u = 0; u < np; ++u)
+    for (int v = 0; v < np; ++v)
+      for (int s = 0; s < no; ++s) Y[(size_t)u * no + s] += E[(size_t)u * np + v] * C[(size_t)v * no + s];
+  ref_backproject(c, psi, proj, Y);
+  free(M); free(E); free(C); free(Y);
+  return 0;
+}
+
+/* nsteps Eq.-6 steps N o Local o N with the dense-D factor (exact != 0: the exactly unitary one) for every
+ * domain; Dm [ndom][nproj][nproj]. */
+int lfd_ref_step_dense(const lfd_ref_config* c, double complex* psi, const double complex* proj,
+                       const double complex* Dm, const double* vloc, const double* A, int nsteps, int exact) {
+  if (ref_check(c) || !psi || !vloc || !A || nsteps < 0) return -1;
+  if (c->nproj > 0 && (!proj || !Dm)) return -1;
+  const size_t ng = (size_t)c->nx * c->ny * c->nz;
+  lfd_ref_config one = *c;
+  one.ndom = 1;
+  for (int it = 0; it < nsteps; ++it)
+    for (int dm = 0; dm < c->ndom; ++dm) {
+      double complex* p = psi + (size_t)dm * ng * c->norb;
+      const double complex* b = proj ? proj + (size_t)dm * ng * c->nproj : NULL;
+      const double complex* d = Dm ? Dm + (size_t)dm * c->nproj * c->nproj : NULL;
+      int e = exact ? lfd_ref_nl_half_exact_dense(&one, p, b, d) : lfd_ref_nl_half_dense(&one, p, b, d);
+      e |= lfd_ref_local(&one, p, vloc + (size_t)dm * ng, A + 3 * dm);
+      e |= exact ? lfd_ref_nl_half_exact_dense(&one, p, b, d) : lfd_ref_nl_half_dense(&one, p, b, d);
+      if (e) return -1;
+    }
+  return 0;
+}
+
+/* Nonlocal energy with a dense D, per domain: E_nl[dm] = sum_s f_s sum_{u,v} conj(C_us) D_uv C_vs
+ * (<psi_s| v_nl |psi_s>, Eq. 5 / P:63). */
+int lfd_ref_energy_nl_dense(const lfd_ref_config* c, const double complex* psi, const double* occ,
+                            const double complex* proj, const double complex* Dm, double* Enl) {
+  if (ref_check(c) || !psi || !occ || !Enl) return -1;
+  const size_t ng = (size_t)c->nx * c->ny * c->nz;
+  const int no = c->norb, np = c->nproj;
+  lfd_ref_config one = *c;
+  one.ndom = 1;
+  double complex* C = malloc(((size_t)np * no + 1) * sizeof(double complex));
+  if (!C) return -2;
+  for (int dm = 0; dm < c->ndom; ++dm) {
+    double e = 0.0;
+    if (np > 0) {
+      ref_project(&one, psi + (size_t)dm * ng * no, proj + (size_t)dm * ng * np, C);
+      const double complex* d = Dm + (size_t)dm * np * np;
+      for (int s = 0; s < no; ++s) {
+        double complex q = 0.0;
+        for (int u = 0; u < np; ++u)
+          for (int v = 0; v < np; ++v) q += conj(C[(size_t)u * no + s]) * d[(size_t)u * np + v] * C[(size_t)v * no + s];
+        e += occ[(size_t)dm * no + s] * creal(q);
+      }
+    }
+    Enl[dm] = e;
+  }
+  free(C);
   return 0;
 }
 

@@ -74,6 +74,12 @@ def lib():
         _lib.lfd_ref_energy.restype = C.c_int
         _lib.lfd_ref_remap_occ.argtypes = [cfgp, P, P, P, C.c_int, P]
         _lib.lfd_ref_remap_occ.restype = C.c_int
+        _lib.lfd_ref_nl_half_dense.argtypes = [cfgp, P, P, P]
+        _lib.lfd_ref_nl_half_exact_dense.argtypes = [cfgp, P, P, P]
+        _lib.lfd_ref_step_dense.argtypes = [cfgp, P, P, P, P, P, C.c_int, C.c_int]
+        _lib.lfd_ref_energy_nl_dense.argtypes = [cfgp, P, P, P, P, P]
+        for f in ("nl_half_dense", "nl_half_exact_dense", "step_dense", "energy_nl_dense"):
+            getattr(_lib, "lfd_ref_" + f).restype = C.c_int
         for f in ("link_sweep", "kinetic", "local", "nl_half", "step", "density_current", "nl_half_exact",
                   "step_exact"):
             getattr(_lib, "lfd_ref_" + f).restype = C.c_int
@@ -189,3 +195,42 @@ def remap_occ(cfg: RefConfig, psi: np.ndarray, occ: np.ndarray, refb: np.ndarray
                                 _ptr(np.ascontiguousarray(occ, np.float64), np.float64),
                                 _ptr(refb, np.complex128), nref, _ptr(out, np.float64)), "remap_occ")
     return out
+
+
+def _dmat(Dm):
+    return np.ascontiguousarray(Dm, np.complex128)
+
+
+def nl_half_dense(cfg: RefConfig, psi: np.ndarray, proj: np.ndarray, Dm: np.ndarray) -> None:
+    """In place: the renormalised first-order factor with a dense Hermitian D [nproj, nproj] (one domain)."""
+    c = cfg.c()
+    _ok(lib().lfd_ref_nl_half_dense(C.byref(c), _ptr(psi, np.complex128), _ptr(proj, np.complex128),
+                                    _ptr(_dmat(Dm), np.complex128)), "nl_half_dense")
+
+
+def nl_half_exact_dense(cfg: RefConfig, psi: np.ndarray, proj: np.ndarray, Dm: np.ndarray) -> None:
+    """In place: exp(-i (Delta/2) B D B^H dV) for dV-orthonormal B (one domain)."""
+    c = cfg.c()
+    _ok(lib().lfd_ref_nl_half_exact_dense(C.byref(c), _ptr(psi, np.complex128), _ptr(proj, np.complex128),
+                                          _ptr(_dmat(Dm), np.complex128)), "nl_half_exact_dense")
+
+
+def step_dense(cfg: RefConfig, psi: np.ndarray, proj: np.ndarray | None, Dm: np.ndarray | None,
+               vloc: np.ndarray, A: np.ndarray, nsteps: int = 1, exact: bool = False) -> None:
+    """In place: nsteps Eq.-6 steps with a dense D [ndom, nproj, nproj] (exact: the unitary factor)."""
+    c = cfg.c()
+    A = np.ascontiguousarray(A, np.float64)
+    _ok(lib().lfd_ref_step_dense(C.byref(c), _ptr(psi, np.complex128), _ptr(proj, np.complex128),
+                                 _ptr(None if Dm is None else _dmat(Dm), np.complex128), _ptr(vloc, np.float64),
+                                 _ptr(A, np.float64), nsteps, 1 if exact else 0), "step_dense")
+
+
+def energy_nl_dense(cfg: RefConfig, psi: np.ndarray, occ: np.ndarray, proj: np.ndarray, Dm: np.ndarray) -> np.ndarray:
+    """[ndom]: sum_s f_s C_s^H D C_s, C = dV B^H Psi."""
+    c = cfg.c()
+    E = np.zeros(cfg.ndom)
+    _ok(lib().lfd_ref_energy_nl_dense(C.byref(c), _ptr(psi, np.complex128),
+                                      _ptr(np.ascontiguousarray(occ, np.float64), np.float64),
+                                      _ptr(proj, np.complex128), _ptr(_dmat(Dm), np.complex128),
+                                      _ptr(E, np.float64)), "energy_nl_dense")
+    return E

@@ -574,7 +574,7 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
   }
   // wrap: planes ny-2, ny-1 (or ny-1 for odd ny; their slots are released at the end) and 0, 1
   const double2* phb = phx + pz0;
-  auto ph = [&](int y, int dz) { return live ? __ldg(phb + y * nz + dz) : cz(); };
+  auto ph = [&](int y, int dz) { return (dz == 0 ? live : has1) ? __ldg(phb + y * nz + dz) : cz(); };
   const double2 f00 = ph(0, 0), f01 = ph(0, 1), f10 = ph(1, 0), f11 = ph(1, 1);
   const double2 fl0 = ph(ny - 1, 0), fl1 = ph(ny - 1, 1);
   const double2 fm0 = ph(ny - 2, 0), fm1 = ph(ny - 2, 1);
