@@ -65,7 +65,7 @@ typedef struct {
   int32_t nref_max;    /* max reference-basis columns for lfd_remap_occ, 0..2048 (0: max(norb, nproj)) */
   double dt;           /* Delta_QD [a.u.], finite and nonzero (negative = backward in time) */
   int32_t device;      /* CUDA device ordinal */
-  int32_t flags;       /* 0 or LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP | LFD_FLAG_NL_DMMA | LFD_FLAG_NL_I8 */
+  int32_t flags;       /* 0 or LFD_FLAG_NO_CARRY | EXACT_NL | SP | NL_DMMA | NL_I8 | DENSE_D (below) */
 } lfd_config;
 
 /* lfd_config.flags: disable the projection carry (lfd_step takes the C of each nonlocal factor that
@@ -99,6 +99,15 @@ typedef struct {
 /* lfd_config.flags: use the int8-digit GEMMs wherever they are supported (nproj, norb <= 64), also on small
  * grids where they are not the default (< 65,536 points per domain: set-up not amortised). */
 #define LFD_FLAG_NL_I8 16
+
+/* lfd_config.flags: a DENSE Hermitian nonlocal coupling (Eq. 5 v_nl, in
+ * Kleinman-Bylander form v_nl = sum_uv |b_u> D_uv <b_v|; Eq. 7's scissor, is D = Delta_sci I): lfd_init's
+ * dnl is then HOST complex128 [ndom][nproj][nproj] (row-major D[u][v], Hermitian to 1e-12 of max |D|, else
+ * LFD_EINVAL), copied. The library diagonalises each D once (D = Q diag(w) Q^H, host Jacobi) and propagates
+ * with the rotated projectors B Q (computed into the workspace by the FP64 GEMM-2) and diagonal couplings w --
+ * the same operator B D B^H, so every path (first-order and exact factors, carry, merged sequences, energy)
+ * applies unchanged. lfd_set_occupations etc. are unaffected. nproj <= 512. */
+#define LFD_FLAG_DENSE_D 32
 
 /* Kernel classes, for lfd_profile_read(). */
 typedef enum {
@@ -134,8 +143,8 @@ lfd_status lfd_workspace_size(const lfd_config* cfg, size_t* bytes);
  *        unoccupied KS orbitals at t = 0, Eq. 7 P:68 / R9); NULL iff nproj == 0. Need not be
  *        orthonormal: the Gram matrix G = dV B^H B is computed here (on the device) and used for n_s.
  *        Must not change while the context lives: G and (default path) B's int8 digits are made here.
- *  dnl   HOST double [ndom][nproj] real couplings D_u (paper: all equal Delta_sci of Eq. 8);
- *        copied. May be NULL iff nproj == 0.
+ *  dnl   HOST double [ndom][nproj] real couplings D_u (paper: all equal Delta_sci of Eq. 8), or with
+ *        LFD_FLAG_DENSE_D complex128 [ndom][nproj][nproj] Hermitian matrices; copied. NULL iff nproj == 0.
  *  occ   HOST double [ndom][norb] occupations f_s (not clamped, R14); copied.
  *  workspace DEVICE, >= lfd_workspace_size bytes, 256-byte aligned; borrowed.
  *  stream cudaStream_t (NULL = legacy default stream); all work is ordered on it.

@@ -7,6 +7,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <complex>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -17,6 +18,7 @@
 #include <vector>
 
 #include "../../include/lfd.h"
+#include "herm_eig.h"
 #include "lfd_internal.h"
 
 using lfd::DomCoef;
@@ -32,7 +34,7 @@ size_t up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 struct Layout {
   size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage, cref,
-      epart, W, ones, x32, aseq, jseq, bsl, bsig, bsl1, bexp, colE, g1cnt;
+      epart, W, ones, x32, aseq, jseq, bsl, bsig, bsl1, bexp, colE, g1cnt, btil, qmat, zero;
   int nref_cap;
   bool i8;  // GEMM-2 on the int8 tensor cores (nl_i8.cu): B digit tiles + row scales in the workspace
   int nsplit_i8;           // GEMM-1 on the int8 tensor cores: splits of rows_per_split_i8 rows
@@ -70,8 +72,13 @@ lfd_status validate(const lfd_config* c, std::string& why) {
   if (c->norb < 1) { why = "norb must be >= 1"; return LFD_EINVAL; }
   if (c->nproj < 0 || c->nproj > 2048) { why = "nproj must be in [0, 2048]"; return LFD_EINVAL; }
   if (!(c->dt != 0.0) || !std::isfinite(c->dt)) { why = "dt must be finite and nonzero"; return LFD_EINVAL; }
-  if (c->flags & ~(LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP | LFD_FLAG_NL_DMMA | LFD_FLAG_NL_I8)) {
+  if (c->flags & ~(LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP | LFD_FLAG_NL_DMMA | LFD_FLAG_NL_I8 |
+                   LFD_FLAG_DENSE_D)) {
     why = "unknown flags";
+    return LFD_EINVAL;
+  }
+  if ((c->flags & LFD_FLAG_DENSE_D) && c->nproj > 512) {
+    why = "LFD_FLAG_DENSE_D supports nproj <= 512";
     return LFD_EINVAL;
   }
   if (c->nref_max < 0 || c->nref_max > 2048) { why = "nref_max must be in [0, 2048]"; return LFD_EINVAL; }
@@ -106,7 +113,7 @@ Geometry geometry(const lfd_config* c) {
   return g;
 }
 
-Layout layout(const Geometry& g, int num_sms, int nref_max) {
+Layout layout(const Geometry& g, int num_sms, int nref_max, bool dense = false) {
   Layout L{};
   L.i8 = g.i8 != 0;
   L.nref_cap = nref_max > 0 ? nref_max : std::max(g.norb, g.nproj);
@@ -178,7 +185,7 @@ Layout layout(const Geometry& g, int num_sms, int nref_max) {
   L.epart = take((size_t)nd * lfd::density_blocks(g) * 2 * d8);
   L.W = take((size_t)2 * nd * np * c16);
   L.ones = take((size_t)nd * std::max(np, no) * d8);
-  L.x32 = g.sp ? take((size_t)nd * np * no * 8) : 0;  // SP: the GEMM-2 coefficient rounded to complex64
+  L.x32 = g.sp ? take((size_t)nd * np * std::max(no, dense ? np : 0) * 8) : 0;  // SP: GEMM-2 coefficient (c64)
   L.aseq = take((size_t)kGraphChunk * nd * 3 * d8);   // lfd_step_graph: A of the chunk's steps
   L.jseq = take((size_t)kGraphChunk * nd * 3 * d8);   // lfd_step_graph: J of the chunk's steps
   L.bsl = L.i8 ? take(lfd::gemm2_i8_bytes(nd, g.ng)) : 0;
@@ -187,6 +194,10 @@ Layout layout(const Geometry& g, int num_sms, int nref_max) {
   L.bexp = L.i8 ? take((size_t)nd * np * sizeof(int)) : 0;
   L.colE = L.i8 ? take((size_t)nd * no * sizeof(int)) : 0;
   L.g1cnt = L.i8 ? take((size_t)nd * sizeof(int)) : 0;
+  // dense D (LFD_FLAG_DENSE_D): the rotated projectors B Q, the eigenvectors Q and a zero vector (GEMM-2's n)
+  L.btil = dense ? take((size_t)nd * g.ng * np * (g.sp ? 8 : c16)) : 0;
+  L.qmat = dense ? take((size_t)nd * np * np * c16) : 0;
+  L.zero = dense ? take((size_t)nd * np * d8) : 0;
   L.total = o;
   return L;
 }
@@ -856,7 +867,7 @@ lfd_status lfd_workspace_size(const lfd_config* cfg, size_t* bytes) {
   if (!bytes) return fail(nullptr, LFD_EINVAL, "bytes is NULL");
   const int sms = query_sms(cfg->device);
   if (sms <= 0) return fail(nullptr, LFD_ECUDA, "no CUDA device (the LFD library has no CPU fallback)");
-  *bytes = layout(geometry(cfg), sms, cfg->nref_max).total;
+  *bytes = layout(geometry(cfg), sms, cfg->nref_max, (cfg->flags & LFD_FLAG_DENSE_D) != 0).total;
   return LFD_OK;
 }
 
@@ -886,7 +897,35 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   if (!is_device_ptr(psi) || !is_device_ptr(workspace) || (proj && !is_device_ptr(proj)))
     return fail(nullptr, LFD_EINVAL, "psi, proj and workspace must be device memory");
   const Geometry g = geometry(cfg);
-  const Layout L = layout(g, prop.multiProcessorCount, cfg->nref_max);
+  const bool dense = (cfg->flags & LFD_FLAG_DENSE_D) != 0;
+  const Layout L = layout(g, prop.multiProcessorCount, cfg->nref_max, dense);
+  // the real couplings the kernels use: D_u, or the eigenvalues w of a dense Hermitian D = Q diag(w) Q^H
+  std::vector<double> dvals((size_t)g.ndom * g.nproj);
+  std::vector<double2> qhost;
+  if (g.nproj > 0 && !dense) std::copy(dnl, dnl + dvals.size(), dvals.begin());
+  if (g.nproj > 0 && dense) {
+    const int np = g.nproj;
+    qhost.resize((size_t)g.ndom * np * np);
+    std::vector<std::complex<double>> Dm((size_t)np * np), Q((size_t)np * np);
+    for (int d = 0; d < g.ndom; ++d) {
+      const double* src = dnl + (size_t)d * np * np * 2;
+      double mx = 0.0, asym = 0.0;
+      for (int u = 0; u < np; ++u)
+        for (int v = 0; v < np; ++v) {
+          Dm[(size_t)u * np + v] = {src[2 * ((size_t)u * np + v)], src[2 * ((size_t)u * np + v) + 1]};
+          mx = std::max(mx, std::abs(Dm[(size_t)u * np + v]));
+        }
+      for (int u = 0; u < np; ++u)
+        for (int v = 0; v < np; ++v)
+          asym = std::max(asym, std::abs(Dm[(size_t)u * np + v] - std::conj(Dm[(size_t)v * np + u])));
+      if (!std::isfinite(mx) || asym > 1e-12 * mx)
+        return fail(nullptr, LFD_EINVAL, "LFD_FLAG_DENSE_D: dnl must be finite Hermitian matrices");
+      if (lfd::herm_eig(np, Dm.data(), dvals.data() + (size_t)d * np, Q.data()) < 0)
+        return fail(nullptr, LFD_EINVAL, "LFD_FLAG_DENSE_D: the eigensolver did not converge");
+      for (size_t k = 0; k < (size_t)np * np; ++k)
+        qhost[(size_t)d * np * np + k] = make_double2(Q[k].real(), Q[k].imag());
+    }
+  }
   if (ws_bytes < L.total) return fail(nullptr, LFD_ENOMEM, "workspace smaller than lfd_workspace_size()");
   cudaError_t e = lfd::gemm_set_attributes();
   if (e == cudaSuccess) e = lfd::density_set_attributes();
@@ -924,7 +963,8 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   };
   // copies of the small host arrays (pageable H2D copies are staged before the call returns)
   if (g.nproj > 0) {
-    e = cudaMemcpyAsync(c->at<double>(L.D), dnl, sizeof(double) * g.ndom * g.nproj, cudaMemcpyHostToDevice, c->stream);
+    e = cudaMemcpyAsync(c->at<double>(L.D), dvals.data(), sizeof(double) * g.ndom * g.nproj, cudaMemcpyHostToDevice,
+                        c->stream);
     if (e != cudaSuccess) { cuda_fail(c, e, "copy dnl"); return bail(LFD_ECUDA); }
   }
   e = cudaMemcpyAsync(c->at<double>(L.occ), occ, sizeof(double) * g.ndom * g.norb, cudaMemcpyHostToDevice, c->stream);
@@ -946,6 +986,31 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   if (s2 != LFD_OK) return bail(s2);
   s2 = set_A(c, nullptr);
   if (s2 != LFD_OK) return bail(s2);
+  if (dense && g.nproj > 0) {
+    // B Q: the projectors rotated into D's eigenbasis (B D B^H = (B Q) diag(w) (B Q)^H), by the FP64 GEMM-2
+    // out of place (Psi := B read-only, n = 0, C'' = Q); from here on the context's projectors are B Q
+    e = cudaMemcpyAsync(c->at<double2>(L.qmat), qhost.data(), sizeof(double2) * qhost.size(), cudaMemcpyHostToDevice,
+                        c->stream);
+    if (e == cudaSuccess) e = cudaMemsetAsync(c->at<double>(L.zero), 0, sizeof(double) * g.ndom * g.nproj, c->stream);
+    if (e != cudaSuccess) { cuda_fail(c, e, "copy Q"); return bail(LFD_ECUDA); }
+    if (g.sp) {
+      s2 = launch(c, LFD_K_NL_BACK, "k_gemm2_sp(BQ)", [&] {
+        return lfd::launch_gemm2_sp(const_cast<float2*>(c->proj32()), c->proj32(), c->at<double2>(L.qmat),
+                                    c->at<float2>(L.x32), c->at<double>(L.zero), g.ndom, g.nproj, g.nproj, g.ng,
+                                    c->stream, c->at<float2>(L.btil));
+      });
+    } else {
+      lfd::Gemm2Args a2;
+      a2.psi = const_cast<double2*>(c->proj); a2.B = c->proj; a2.Cp = c->at<double2>(L.qmat);
+      a2.nfac = c->at<double>(L.zero); a2.ndom = g.ndom; a2.nproj = g.nproj; a2.norb = g.nproj; a2.ng = g.ng;
+      a2.num_sms = c->num_sms; a2.psi_out = c->at<double2>(L.btil);
+      s2 = launch(c, LFD_K_NL_BACK, "k_gemm2(BQ)", [&] { return lfd::launch_gemm2(a2, c->stream); });
+    }
+    if (s2 != LFD_OK) return bail(s2);
+    e = cudaStreamSynchronize(c->stream);  // qhost (host staging) goes out of scope
+    if (e != cudaSuccess) { cuda_fail(c, e, "B Q"); return bail(LFD_ECUDA); }
+    c->proj = c->at<double2>(L.btil);
+  }
   // Gram matrix G = dV B^H B (GEMM-1 with X = B, fixed-order reduction)
   if (g.nproj > 0) {
     lfd::Gemm1Args a1;
@@ -1001,7 +1066,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
       std::vector<double2> Wh((size_t)2 * g.ndom * g.nproj);
       for (size_t i = 0; i < (size_t)g.ndom * g.nproj; ++i)
         for (int k = 0; k < 2; ++k) {  // k = 0: one factor (tau = Delta/2), 1: two merged (tau = Delta)
-          const double ph = -(k + 1) * 0.5 * g.dt * dnl[i];
+          const double ph = -(k + 1) * 0.5 * g.dt * dvals[i];
           Wh[k * (size_t)g.ndom * g.nproj + i] = make_double2(std::cos(ph) - 1.0, std::sin(ph));
         }
       e = cudaMemcpyAsync(c->at<double2>(L.W), Wh.data(), Wh.size() * sizeof(double2), cudaMemcpyHostToDevice,

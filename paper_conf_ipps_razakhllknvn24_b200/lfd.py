@@ -23,6 +23,7 @@ LFD_FLAG_EXACT_NL = 2
 LFD_FLAG_SP = 4
 LFD_FLAG_NL_DMMA = 8
 LFD_FLAG_NL_I8 = 16
+LFD_FLAG_DENSE_D = 32
 LFD_BC_PERIODIC = 0
 LFD_BC_ZERO = 1
 STATUS = {0: "LFD_OK", -1: "LFD_EINVAL", -2: "LFD_ENOMEM", -3: "LFD_ECUDA", -4: "LFD_ESTATE",
@@ -161,7 +162,8 @@ def lfd_workspace_size(cfg: lfd_config) -> int:
 
 
 def lfd_init(cfg, psi, proj, dnl, occ, workspace, stream=None) -> C.c_void_p:
-    pd, _k1 = _hptr(dnl)
+    # dnl: real [ndom][nproj], or with LFD_FLAG_DENSE_D the complex Hermitian matrices [ndom][nproj][nproj]
+    pd, _k1 = _hptr(dnl, np.complex128 if cfg.flags & LFD_FLAG_DENSE_D else np.float64)
     po, _k2 = _hptr(occ)
     ctx = C.c_void_p()
     _check(load().lfd_init(C.byref(cfg), _dptr(psi), _dptr(proj), pd, po, _dptr(workspace),

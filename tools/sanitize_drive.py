@@ -48,4 +48,19 @@ for w in shapes:
     ctx.sync()
     assert not torch.isnan(psi).any(), w.name
     ctx.close()
+if mode == "dmma":  # dense Hermitian D (LFD_FLAG_DENSE_D): the B Q rotation at init, then the diagonal path
+    w = workload("P0")
+    x = make_inputs(w, seed=6)
+    rng = np.random.default_rng(0)
+    M = rng.standard_normal((1, w.nproj, w.nproj)) + 1j * rng.standard_normal((1, w.nproj, w.nproj))
+    Dm = np.ascontiguousarray(0.05 * (M + np.conj(np.swapaxes(M, 1, 2))))
+    psi = torch.from_numpy(x.psi0.copy()).to(dev)
+    ctx = Context(psi, torch.from_numpy(x.proj).to(dev), Dm, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc,
+                  flags=lfd.LFD_FLAG_DENSE_D)
+    ctx.set_potential(torch.from_numpy(x.vloc).to(dev))
+    ctx.step(2)
+    ctx.energy()
+    ctx.sync()
+    assert not torch.isnan(psi).any()
+    ctx.close()
 print("sanitize drive ok")
