@@ -34,7 +34,7 @@ FP64_PEAK_FILE = os.path.join(ROOT, "profiles", "r01_fp64_peaks.jsonl")
 NCU_SUMMARY = os.path.join(ROOT, "profiles", "latest_ncu_full_summary.csv")
 I8_DIGIT_BYTES = 6 * 128  # B digits per grid point of the int8-digit GEMMs (6 digits x K = 128 bytes)
 NCU_NAMES = {"nl_proj": "k_gemm1", "nl_back": "k_gemm2", "kin_x": "k_kin<1, 1, 1", "kin_y": "k_kin<1, 0",
-             "kin_z": "k_kin<1, 2>", "kin_yz": "k_kin_yz", "density": "k_density"}
+             "kin_z": "k_kin<1, 2>", "kin_yz": "k_kin_yz", "density": "k_density", "nl_back_x": "k_gemm2x"}
 
 
 def ncu_traffic(kernel, i8=False):
@@ -168,6 +168,8 @@ def kernel_work(w):
         "kin_yz": (2 * psi + 16.0 * ng * nd, 0.0),
         "nl_proj": (psi + bb, gemm_flops),
         "nl_back": (2 * psi + bb, gemm_flops),
+        # the first factor's GEMM-2 fused with Phi . K_x (nl_fx.cu): Psi read + write, B's int8 digits, Phi
+        "nl_back_x": (2 * psi + I8_DIGIT_BYTES * ng * nd + 16.0 * ng * nd, gemm_flops),
         # the density reads the orbitals up to the last occupied one (f = 0 adds exactly zero) and
         # writes rho (the bench requests rho and J, not j)
         "density": (16.0 * ng * nd * w.nocc + 8.0 * ng * nd, 0.0),
@@ -577,7 +579,11 @@ def main():
         e = {"ms_per_launch": avg, "launches": cnt, "share": kms / total_ms if total_ms else None}
         if k in work:
             b, f = work[k]
-            if k in ("nl_back", "nl_proj") and nl_path == 1:
+            if k == "nl_back_x":  # bytes as stated in kernel_work (the digits, not B's FP64 bytes)
+                e.update({"bound": "hbm", "achieved": b / (avg * 1e-3) / 1e9, "unit": "GB/s", "peak": pk["hbm_gbs"],
+                          "path": "int8-digit tcgen05 GEMM-2 fused with Phi . K_x",
+                          "fp64_equiv_tflops": f / (avg * 1e-3) / 1e12})
+            elif k in ("nl_back", "nl_proj") and nl_path == 1:
                 # int8-digit tcgen05 GEMMs (FP64 emulated): the digit products are cheap on the int8 tensor
                 # cores, so the kernels are bound by streaming Psi (read, + write for GEMM-2) and B's digits
                 # (6 x 128 B per grid point at nproj = 64: 0.75 of B's FP64 bytes) -- reported against HBM

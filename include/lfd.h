@@ -127,7 +127,8 @@ typedef enum {
   LFD_K_KIN_YZ = 13,   /* a6: K_y K_z . Phi fused in one pass (post-phase fused) */
   LFD_K_SC = 14,       /* self-consistent step: Maxwell, potential gather, Poisson filter, v_Hxc */
   LFD_K_FFT = 15,      /* self-consistent step: cuFFT D2Z / Z2D of the Hartree solve (library kernels) */
-  LFD_K_COUNT = 16
+  LFD_K_NL_BACKX = 16, /* a5 + a6: the first factor's GEMM-2 fused with Phi . K_x (int8-digit path, nx <= 80) */
+  LFD_K_COUNT = 17
 } lfd_kernel_id;
 
 /* Bytes of DEVICE workspace lfd_init needs for this configuration. */

@@ -34,9 +34,10 @@ size_t up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 struct Layout {
   size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage, cref,
-      epart, W, ones, x32, aseq, jseq, bsl, bsig, bsl1, bexp, colE, g1cnt, btil, qmat, zero;
+      epart, W, ones, x32, aseq, jseq, bsl, bsig, bsl1, bexp, colE, g1cnt, btil, qmat, zero, bslx, sigx;
   int nref_cap;
   bool i8;  // GEMM-2 on the int8 tensor cores (nl_i8.cu): B digit tiles + row scales in the workspace
+  bool fx;  // the first factor's GEMM-2 fused with the x pass (nl_fx.cu)
   int nsplit_i8;           // GEMM-1 on the int8 tensor cores: splits of rows_per_split_i8 rows
   long long rows_per_split_i8;
   size_t total;
@@ -198,6 +199,10 @@ Layout layout(const Geometry& g, int num_sms, int nref_max, bool dense = false) 
   L.btil = dense ? take((size_t)nd * g.ng * np * (g.sp ? 8 : c16)) : 0;
   L.qmat = dense ? take((size_t)nd * np * np * c16) : 0;
   L.zero = dense ? take((size_t)nd * np * d8) : 0;
+  // the first nonlocal factor's GEMM-2 fused with the x pass (nl_fx.cu): B's digits and scales in x-line order
+  L.fx = lfd::gemm2x_supported(g);
+  L.bslx = L.fx ? take(lfd::gemm2x_digit_bytes(g)) : 0;
+  L.sigx = L.fx ? take(lfd::gemm2x_sig_bytes(g)) : 0;
   L.total = o;
   return L;
 }
@@ -310,6 +315,7 @@ struct lfd_ctx {
   bool kin_fused = true;  // Phi.K_y K_z in one pass (else separate y and z passes: lines too long for the ring)
   CUtensorMap psi_tmap;   // TMA descriptor of Psi for the fused pass
   lfd::DensMaps* dmaps = nullptr;  // TMA descriptors of Psi for the density kernel
+  lfd::FxMaps* fxm = nullptr;      // TMA descriptors of the fused GEMM-2 + x pass (nullptr: not used)
   bool scaled = true;     // scaled pair form of the stencil (else the general 2x2 form: some cos(tau t) < 1/2)
   std::string err = "no error";
   // density-current global layout cache
@@ -491,9 +497,22 @@ const double2* exact_w(lfd_ctx* c, bool merged) {
   return c->at<double2>(c->L.W) + (merged ? (size_t)c->g.ndom * c->g.nproj : 0);
 }
 
-// Eq. 6 nonlocal factor N on every domain (kernels a3, a4, a5); merged = N o N in one pass.
-lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
+// GEMM-2 of a factor that the local propagator's x pass follows, fused with it (nl_fx.cu): Psi <- K_x(Phi .
+// (n Psi + B C'')); afterwards the local propagator runs without its x pass.
+lfd_status gemm2x(lfd_ctx* c) {
+  c->c_valid = false;
+  return launch(c, LFD_K_NL_BACKX, "k_gemm2x_i8", [&] {
+    return lfd::launch_gemm2x_i8(c->g, c->fxm, c->psi, c->coef(), c->at<double>(c->L.nfac),
+                                 c->at<double2>(c->L.cprime), c->at<double>(c->L.sigx), c->scaled, c->num_sms,
+                                 c->stream);
+  });
+}
+
+// Eq. 6 nonlocal factor N on every domain (kernels a3, a4, a5); merged = N o N in one pass; fused = the GEMM-2
+// also applies the next local factor's Phi . K_x (gemm2x; only when c->fxm).
+lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr, bool fused = false) {
   const Geometry& g = c->g;
+  auto finish = [&]() { return fused ? gemm2x(c) : gemm2(c, out); };
   if (c->c_valid) {  // C of the current Psi from the previous factor (no GEMM-1, no reduction)
     double* D = c->at<double>(c->L.D);
     double2* DC = c->at<double2>(c->L.dc);
@@ -505,7 +524,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
         return lfd::launch_nlcarry(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G),
                                    c->at<double>(c->L.ones), DC, X, s, nfac, false, exact_w(c, merged), c->stream);
       }));
-      return gemm2(c, out);
+      return finish();
     }
     LFD_TRY(launch(c, LFD_K_NL_CARRY, "k_nlcarry", [&] {
       return lfd::launch_nlcarry(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), D, DC, X, s, nfac,
@@ -516,7 +535,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
         return lfd::launch_nlmerge(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), D, DC, s, X, nfac,
                                    c->stream);
       }));
-    return gemm2(c, out);
+    return finish();
   }
   lfd::Gemm1Args a1;
   a1.A = c->proj;
@@ -552,7 +571,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
     r.D = nullptr;
     r.W = exact_w(c, merged);
     LFD_TRY(launch(c, LFD_K_NL_REDUCE, "k_reduce", [&] { return lfd::launch_reduce(r, c->stream); }));
-    return gemm2(c, out);
+    return finish();
   }
   LFD_TRY(launch(c, LFD_K_NL_REDUCE, "k_reduce", [&] { return lfd::launch_reduce(r, c->stream); }));
   if (merged)
@@ -565,12 +584,12 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr) {
       return lfd::launch_nlnorm(g.ndom, g.nproj, g.norb, 0.5 * g.dt, c->at<double2>(c->L.G), r.out, r.s,
                                 c->at<double>(c->L.nfac), r.cprime, c->stream);
     }));
-  return gemm2(c, out);
+  return finish();
 }
 
 // Local factor exp(-i Delta h_loc) of Eq. 6: Psi <- Phi . K_z K_y K_x (Phi . Psi) (kernels a6).
 // src != nullptr: the first pass reads src (same layout) and writes Psi (out of place).
-lfd_status local_prop(lfd_ctx* c, const double2* src = nullptr) {
+lfd_status local_prop(lfd_ctx* c, const double2* src = nullptr, bool skip_x = false) {
   c->c_valid = false;
   if (c->g.sp) {  // SP variant: three FP32 line passes Phi.K_x, K_y, K_z.Phi (complex64 Psi)
     LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin_sp(x)", [&] {
@@ -584,8 +603,9 @@ lfd_status local_prop(lfd_ctx* c, const double2* src = nullptr) {
       return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 2, 2, c->scaled, c->stream);
     });
   }
-  LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin(x)",
-                 [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 0, 1, c->scaled, c->stream, src); }));
+  if (!skip_x)
+    LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin(x)",
+                   [&] { return lfd::launch_kin(c->g, c->psi, c->coef(), c->phi(), 0, 1, c->scaled, c->stream, src); }));
   if (c->kin_fused) {
     int* colE = c->L.i8 ? c->at<int>(c->L.colE) : nullptr;
     LFD_TRY(launch(c, LFD_K_KIN_YZ, "k_kin_yz", [&] {
@@ -719,8 +739,10 @@ ScLayout sc_layout(const Geometry& g, const lfd_sc_config* sc, size_t fft_bytes)
 
 // Eq.-6 step of every domain with the context's current Phi and coefficients.
 lfd_status one_step(lfd_ctx* c) {
-  if (c->g.nproj > 0) LFD_TRY(nl_half(c));
-  LFD_TRY(local_prop(c));
+  const bool fx = c->fxm != nullptr && c->g.nproj > 0 && !c->nl_pending;
+  if (c->g.nproj > 0 && !c->nl_pending) LFD_TRY(nl_half(c, false, nullptr, fx));
+  c->nl_pending = false;
+  LFD_TRY(local_prop(c, nullptr, fx));
   if (c->g.nproj > 0) LFD_TRY(nl_half(c));
   return LFD_OK;
 }
@@ -932,6 +954,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   if (e == cudaSuccess) e = lfd::kin_yz_set_attributes();
   if (e == cudaSuccess) e = lfd::gemm_sp_set_attributes();
   if (e == cudaSuccess) e = lfd::gemm_i8_set_attributes();
+  if (e == cudaSuccess) e = lfd::gemm2x_set_attributes();
   if (e != cudaSuccess) return cuda_fail(nullptr, e, "cudaFuncSetAttribute");
 
   lfd_ctx* c = new (std::nothrow) lfd_ctx();
@@ -1041,6 +1064,14 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
     if (e == cudaSuccess) e = cudaMemsetAsync(c->at<int>(L.g1cnt), 0, sizeof(int) * g.ndom, c->stream);
     if (e != cudaSuccess) { cuda_fail(c, e, "memset"); return bail(LFD_ECUDA); }
   }
+  if (L.fx) {  // B's digits in x-line order for the fused first factor
+    s2 = launch(c, LFD_K_NL_BACKX, "k_bslicex_i8", [&] {
+      return lfd::launch_bslicex_i8(g, c->proj, c->at<int8_t>(L.bslx), c->at<double>(L.sigx), c->stream);
+    });
+    if (s2 != LFD_OK) return bail(s2);
+    c->fxm = lfd::gemm2x_maps_create(g, c->at<int8_t>(L.bslx), c->psi, c->phi());
+    // (no descriptors: the unfused GEMM-2 + x pass run instead)
+  }
   if (cfg->flags & LFD_FLAG_EXACT_NL) {
     // exactly unitary nonlocal factor: needs dV B^H B = I (checked on G), then
     // exp(-i (Delta/2) B D B^H dV) = 1 + B diag(e^{-i (Delta/2) D} - 1) B^H dV with n = 1
@@ -1120,12 +1151,7 @@ lfd_status lfd_step(lfd_ctx* c, int32_t nsteps) {
   LFD_TRY(check_ctx(c));
   if (nsteps < 0) return fail(c, LFD_EINVAL, "nsteps must be >= 0");
   DeviceGuard dg(c->device);
-  for (int it = 0; it < nsteps; ++it) {
-    if (c->g.nproj > 0 && !c->nl_pending) LFD_TRY(nl_half(c));
-    c->nl_pending = false;
-    LFD_TRY(local_prop(c));
-    if (c->g.nproj > 0) LFD_TRY(nl_half(c));
-  }
+  for (int it = 0; it < nsteps; ++it) LFD_TRY(one_step(c));
   return LFD_OK;
 }
 
@@ -1146,12 +1172,22 @@ lfd_status lfd_step_sequence(lfd_ctx* c, int32_t nsteps, const double* A_seq) {
     if (!std::isfinite(A_seq[i])) return fail(c, LFD_EINVAL, "A_seq must be finite");
   DeviceGuard dg(c->device);
   const bool nl = c->g.nproj > 0;
+  const bool fx = c->fxm != nullptr && nl;
+  bool x_done = false;  // the x pass of step n already ran inside the preceding factor's GEMM-2
   for (int n = 0; n < nsteps; ++n) {
-    LFD_TRY(set_A(c, A_seq + 3LL * c->g.ndom * n));
-    if (nl && n == 0 && !c->nl_pending) LFD_TRY(nl_half(c));  // first factor of the sequence
+    if (n == 0) LFD_TRY(set_A(c, A_seq));
+    if (nl && n == 0 && !c->nl_pending) {  // first factor of the sequence
+      LFD_TRY(nl_half(c, false, nullptr, fx));
+      x_done = fx;
+    }
     c->nl_pending = false;
-    LFD_TRY(local_prop(c));
-    if (nl) LFD_TRY(nl_half(c, n + 1 < nsteps));  // N of step n fused with N of step n+1
+    LFD_TRY(local_prop(c, nullptr, x_done));
+    x_done = false;
+    if (n + 1 < nsteps) LFD_TRY(set_A(c, A_seq + 3LL * c->g.ndom * (n + 1)));  // before a fused x pass reads it
+    if (nl) {  // N of step n merged with N of step n+1 (and fused with step n+1's x pass)
+      LFD_TRY(nl_half(c, n + 1 < nsteps, nullptr, fx && n + 1 < nsteps));
+      x_done = fx && n + 1 < nsteps;
+    }
   }
   return LFD_OK;
 }
@@ -1602,6 +1638,7 @@ lfd_status lfd_destroy(lfd_ctx* c) {
     }
   }
   lfd::density_maps_destroy(c->dmaps);
+  lfd::gemm2x_maps_destroy(c->fxm);
   sc_release(c->sc);
   release_graphs(c);
   if (c->sc.comm) {

@@ -28,6 +28,7 @@
 #include "lfd_coef.cuh"
 #include "lfd_complex.cuh"
 #include "lfd_internal.h"
+#include "lfd_march.cuh"
 #include "lfd_tma.cuh"
 
 namespace lfd {
@@ -120,156 +121,6 @@ cudaError_t launch_phase_sp(const Geometry& g, const double* v, float2* phi, dou
   return cudaGetLastError();
 }
 
-// ---- pair blocks -------------------------------------------------------------------------------
-// Coefficients of one axis for tau = Delta/2 (1) and Delta (2). General form: a = alpha, u = up,
-// d = dn, s = onsite. Scaled form: u = w_up, d = w_dn, s = (1/c, 0), a unused.
-template <class C>
-struct PairCoefT {
-  C a1, u1, d1, s1, a2, u2, d2, s2;
-};
-using PairCoef = PairCoefT<double2>;
-
-template <bool kS>
-__device__ __forceinline__ PairCoef pair_coef(const DomCoef* cf, int axis) {
-  PairCoef c;
-  if (kS) {
-    c.a1 = c.a2 = make_double2(1.0, 0.0);
-    c.u1 = cf->wu[axis][0]; c.d1 = cf->wd[axis][0]; c.s1 = make_double2(cf->rc[axis][0], 0.0);
-    c.u2 = cf->wu[axis][1]; c.d2 = cf->wd[axis][1]; c.s2 = make_double2(cf->rc[axis][1], 0.0);
-  } else {
-    c.a1 = cf->alpha[axis][0]; c.u1 = cf->up[axis][0]; c.d1 = cf->dn[axis][0]; c.s1 = cf->onsite[axis][0];
-    c.a2 = cf->alpha[axis][1]; c.u2 = cf->up[axis][1]; c.d2 = cf->dn[axis][1]; c.s2 = cf->onsite[axis][1];
-  }
-  return c;
-}
-
-// The SP variant (complex64 Psi) runs the same sweeps in FP32 with the coefficients
-// rounded once from the FP64 table.
-template <bool kS, class C>
-__device__ __forceinline__ PairCoefT<C> pair_coef_t(const DomCoef* cf, int axis) {
-  const PairCoef d = pair_coef<kS>(cf, axis);
-  PairCoefT<C> c;
-  c.a1 = from_d2<C>(d.a1); c.u1 = from_d2<C>(d.u1); c.d1 = from_d2<C>(d.d1); c.s1 = from_d2<C>(d.s1);
-  c.a2 = from_d2<C>(d.a2); c.u2 = from_d2<C>(d.u2); c.d2 = from_d2<C>(d.d2); c.s2 = from_d2<C>(d.s2);
-  return c;
-}
-
-// x + w y
-__device__ __forceinline__ double2 padd(double2 w, double2 x, double2 y) {
-  return make_double2(fma(w.x, y.x, fma(-w.y, y.y, x.x)), fma(w.x, y.y, fma(w.y, y.x, x.y)));
-}
-__device__ __forceinline__ float2 padd(float2 w, float2 x, float2 y) {
-  return make_float2(fmaf(w.x, y.x, fmaf(-w.y, y.y, x.x)), fmaf(w.x, y.y, fmaf(w.y, y.x, x.y)));
-}
-// Two adjacent orbitals of one grid point (the SP passes move 16 bytes per lane, like the FP64 ones).
-struct __align__(16) cf2 {
-  float2 a, b;
-};
-__device__ __forceinline__ cf2 padd(float2 w, cf2 x, cf2 y) { return {padd(w, x.a, y.a), padd(w, x.b, y.b)}; }
-__device__ __forceinline__ cf2 cmul(float2 s, cf2 x) { return {cmul(s, x.a), cmul(s, x.b)}; }
-__device__ __forceinline__ cf2 crow(float2 a, cf2 x, float2 b, cf2 y) {
-  return {crow(a, x.a, b, y.a), crow(a, x.b, b, y.b)};
-}
-__device__ __forceinline__ double2 rscale(double r, double2 x) { return make_double2(r * x.x, r * x.y); }
-__device__ __forceinline__ float2 rscale(float r, float2 x) { return make_float2(r * x.x, r * x.y); }
-__device__ __forceinline__ cf2 rscale(float r, cf2 x) { return {rscale(r, x.a), rscale(r, x.b)}; }
-
-// Left / right output of a link (x at the left point, y at the right point) and a singleton; coefficients
-// of type C, values of type V (V = C, or two complex64 orbitals for the SP passes).
-template <bool kS, class C, class V>
-__device__ __forceinline__ V lk_L(C a, C u, V x, V y) {
-  return kS ? padd(u, x, y) : crow(a, x, u, y);
-}
-template <bool kS, class C, class V>
-__device__ __forceinline__ V lk_R(C a, C d, V x, V y) {
-  return kS ? padd(d, y, x) : crow(d, x, a, y);
-}
-template <bool kS, class C, class V>
-__device__ __forceinline__ V lk_S(C s, V x) {
-  return kS ? rscale(s.x, x) : cmul(s, x);
-}
-
-// Streaming K_d along one line, fed one pair (2p, 2p+1) at a time: first E(Delta/2) on the new pair,
-// O(Delta) on the link (2p-1, 2p), second E(Delta/2) on (2p-2, 2p-1) once both its O outputs exist;
-// points 0, 1 wait for the wrap link (n-1, 0) at the end.
-template <bool kS, class C = double2, class V = C>
-struct LineMarch {
-  V E10, O1, prev_e1, prev_oR;
-  __device__ __forceinline__ void init() { E10 = O1 = prev_e1 = prev_oR = V{}; }
-  template <class St>
-  __device__ __forceinline__ void push(const PairCoefT<C>& c, int p, V a, V b, bool pair, St&& st) {
-    V e0, e1 = V{};
-    if (pair) {
-      e0 = lk_L<kS>(c.a1, c.u1, a, b);
-      e1 = lk_R<kS>(c.a1, c.d1, a, b);
-    } else {
-      e0 = lk_S<kS>(c.s1, a);  // zero-BC singleton (odd n)
-    }
-    if (p == 0) {
-      E10 = e0;
-    } else {
-      const V oL = lk_L<kS>(c.a2, c.u2, prev_e1, e0);
-      const V oR = lk_R<kS>(c.a2, c.d2, prev_e1, e0);
-      if (p == 1) {
-        O1 = oL;
-      } else {
-        st(2 * p - 2, lk_L<kS>(c.a1, c.u1, prev_oR, oL));
-        st(2 * p - 1, lk_R<kS>(c.a1, c.d1, prev_oR, oL));
-      }
-      prev_oR = oR;
-    }
-    prev_e1 = e1;
-  }
-  // The three phases of push() without the p tests (p == 0, p == 1, p >= 2 with a full pair).
-  __device__ __forceinline__ void first(const PairCoefT<C>& c, V a, V b) {
-    E10 = lk_L<kS>(c.a1, c.u1, a, b);
-    prev_e1 = lk_R<kS>(c.a1, c.d1, a, b);
-  }
-  __device__ __forceinline__ void second(const PairCoefT<C>& c, V a, V b) {
-    const V e0 = lk_L<kS>(c.a1, c.u1, a, b);
-    O1 = lk_L<kS>(c.a2, c.u2, prev_e1, e0);
-    prev_oR = lk_R<kS>(c.a2, c.d2, prev_e1, e0);
-    prev_e1 = lk_R<kS>(c.a1, c.d1, a, b);
-  }
-  template <class St>
-  __device__ __forceinline__ void steady(const PairCoefT<C>& c, V a, V b, St&& st) {
-    const V e0 = lk_L<kS>(c.a1, c.u1, a, b);
-    const V oL = lk_L<kS>(c.a2, c.u2, prev_e1, e0);
-    const V oR = lk_R<kS>(c.a2, c.d2, prev_e1, e0);
-    st(0, lk_L<kS>(c.a1, c.u1, prev_oR, oL));
-    st(1, lk_R<kS>(c.a1, c.d1, prev_oR, oL));
-    prev_oR = oR;
-    prev_e1 = lk_R<kS>(c.a1, c.d1, a, b);
-  }
-  template <bool kPer, class St>
-  __device__ __forceinline__ void finish(const PairCoefT<C>& c, int n, St&& st) {
-    if ((n & 1) == 0) {
-      V Olast, O0;
-      if (kPer) {  // wrap link (n-1, 0)
-        Olast = lk_L<kS>(c.a2, c.u2, prev_e1, E10);
-        O0 = lk_R<kS>(c.a2, c.d2, prev_e1, E10);
-      } else {
-        Olast = lk_S<kS>(c.s2, prev_e1);
-        O0 = lk_S<kS>(c.s2, E10);
-      }
-      if (n == 2) {
-        st(0, lk_L<kS>(c.a1, c.u1, O0, Olast));
-        st(1, lk_R<kS>(c.a1, c.d1, O0, Olast));
-      } else {
-        st(n - 2, lk_L<kS>(c.a1, c.u1, prev_oR, Olast));
-        st(n - 1, lk_R<kS>(c.a1, c.d1, prev_oR, Olast));
-        st(0, lk_L<kS>(c.a1, c.u1, O0, O1));
-        st(1, lk_R<kS>(c.a1, c.d1, O0, O1));
-      }
-    } else {  // odd n (zero BC): last point is an E singleton; point 0 an O singleton
-      st(n - 1, lk_S<kS>(c.s1, prev_oR));
-      const V O0 = lk_S<kS>(c.s2, E10);
-      st(0, lk_L<kS>(c.a1, c.u1, O0, O1));
-      st(1, lk_R<kS>(c.a1, c.d1, O0, O1));
-    }
-  }
-};
-
 // One K_axis pass. Column c of domain blockIdx.y: outer = c / inner_len, inner = c % inner_len,
 // element offset = outer*outer_stride + inner; successive points of the line are pt_stride apart.
 // Loads run two pairs ahead of the pair being combined (memory-level parallelism for the HBM stream).
@@ -307,40 +158,7 @@ __global__ void __launch_bounds__(256, 3) k_kin(V* psi, const V* src, const DomC
     line[(long long)i * pt_stride] = v;
   };
 
-  const int P = (n + 1) >> 1;
-  LineMarch<kS, C, V> L;
-  L.init();
-  if (kPeriodic && n >= 6) {  // periodic (even n): first two pairs peeled, then a test-free steady loop
-    V a0 = ld(0), b0 = ld(1), a1 = ld(2), b1 = ld(3), a2 = ld(4), b2 = ld(5);
-    L.first(cf, a0, b0);
-    a0 = a1; b0 = b1; a1 = a2; b1 = b2;
-    if (3 < P) { a2 = ld(6); b2 = ld(7); }
-    L.second(cf, a0, b0);
-    for (int p = 2; p < P; ++p) {
-      a0 = a1; b0 = b1; a1 = a2; b1 = b2;
-      if (p + 2 < P) { a2 = ld(2 * p + 4); b2 = ld(2 * p + 5); }
-      L.steady(cf, a0, b0, [&](int k, V v) { st(2 * p - 2 + k, v); });
-    }
-    L.template finish<kPeriodic>(cf, n, st);
-    return;
-  }
-  V na = ld(0), nb = (n > 1) ? ld(1) : V{};
-  V nc = V{}, nd = V{};
-  if (P > 1) {
-    nc = ld(2);
-    nd = (3 < n) ? ld(3) : V{};
-  }
-  for (int p = 0; p < P; ++p) {
-    const V a = na, b = nb;
-    na = nc;
-    nb = nd;
-    if (p + 2 < P) {
-      nc = ld(2 * p + 4);
-      nd = (2 * p + 5 < n) ? ld(2 * p + 5) : V{};
-    }
-    L.push(cf, p, a, b, 2 * p + 1 < n, st);
-  }
-  L.template finish<kPeriodic>(cf, n, st);
+  march_line<kPeriodic, kS, C, V>(n, cf, ld, st);
 }
 
 // ------------------------------------------------------------------------------------------------

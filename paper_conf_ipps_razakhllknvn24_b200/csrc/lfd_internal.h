@@ -69,6 +69,10 @@ struct Geometry {
 cudaError_t encode_tmap_f64(CUtensorMap* out, int rank, const void* base, const uint64_t* dims,
                             const uint64_t* strides_bytes, const uint32_t* box);
 
+// Any tensor map: dtype a CUtensorMapDataType, swizzle a CUtensorMapSwizzle (tmap.cu).
+cudaError_t encode_tmap(CUtensorMap* out, int dtype, int rank, const void* base, const uint64_t* dims,
+                        const uint64_t* strides_bytes, const uint32_t* box, int swizzle);
+
 // ---- launchers (each returns the cudaError_t of the launch) -------------------------------------
 constexpr int kCoefMaxPerLaunch = 512;
 struct CoefParams {
@@ -189,6 +193,20 @@ struct Gemm1I8Args {
   int ndom, nproj, norb, nsplit;
   long long ng, rps;
 };
+// The first nonlocal factor's GEMM-2 fused with the x pass of the local propagator (nl_fx.cu):
+//   Psi[x][yz] <- K_x (Phi . (n Psi + B C''))  along every x-line (y, z), int8-digit tcgen05 products.
+// B's digits and row scales in x-line order are made once at lfd_init (launch_bslicex_i8).
+struct FxMaps;  // TMA descriptors (digits, Psi, Phi) -- host-owned, built at lfd_init
+bool gemm2x_supported(const Geometry& g);
+size_t gemm2x_digit_bytes(const Geometry& g);
+size_t gemm2x_sig_bytes(const Geometry& g);
+cudaError_t launch_bslicex_i8(const Geometry& g, const double2* B, int8_t* dig, double* sig, cudaStream_t st);
+FxMaps* gemm2x_maps_create(const Geometry& g, const int8_t* dig, double2* psi, const double2* phi);
+void gemm2x_maps_destroy(FxMaps* m);
+cudaError_t launch_gemm2x_i8(const Geometry& g, const FxMaps* m, double2* psi, const DomCoef* coef, const double* nfac,
+                             const double2* Cp, const double* sig, bool scaled, int num_sms, cudaStream_t st);
+cudaError_t gemm2x_set_attributes();
+
 size_t gemm1_i8_bytes(int ndom, long long ng);
 long long gemm1_i8_rows_per_split(long long ng, int ndom, int num_sms);
 cudaError_t launch_bslice1_i8(const double2* B, int ndom, int nproj, long long ng, int* bexp, int8_t* out,

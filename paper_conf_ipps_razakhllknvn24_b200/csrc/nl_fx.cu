@@ -1,0 +1,419 @@
+// nl_fx.cu -- the first nonlocal factor's GEMM-2 fused with the x pass of the local propagator.
+//
+// Eq. 6 applies N, then the local factor Phi . K_z K_y K_x (Phi . ), then N. The GEMM-2 of the first N
+// (Psi <- n Psi + B C'', Eq. 9; nl_i8.cu) writes Psi and the x pass (Psi <- K_x (Phi . Psi), kin.cu)
+// reads it straight back: one full read + write of Psi per step (722 MB at C2) that this kernel removes.
+// A work item is one x-line (y, z) of a domain: all nx points x of all orbitals. The int8-digit products
+// (nl_i8.cu's scheme: 6 balanced digits, 21 digit pairs in int32 TMEM accumulators, FP64 recombination) run
+// with the line as the MMA's N = 80 (zero rows past nx); the epilogue writes n Psi + B C'' into the line's
+// shared-memory copy of Psi, and two march warps (one thread per orbital: the paper's psi_old carry,
+// Alg. 3 l.6, in registers) stream K_x (Phi . ) along the line from shared memory into HBM.
+//
+// Roles (20 warps): 16 epilogue warps (4 TMEM lane quarters x 4 groups of 20 x), the MMA issuer (which also
+// loads B's digit tile of the next line as soon as the previous line's MMAs are done: one 4-D TMA copy
+// [6 digits][80 x][128 B], 128B-swizzled by the TMA, rows past nx zero-filled), a producer of the line (one TMA copy each of Psi [nx][2 norb] and Phi [nx], one bulk copy of
+// B's row scales) and the two march warps. Shared memory: one digit tile (60 KB) + two line buffers
+// (ping-pong: the epilogue fills one while the march drains the other). TMEM: the W digits (A operand,
+// 192 columns) + a 4-slot ring of 80-column diagonal accumulators.
+#include <algorithm>
+#include <new>
+
+#include "lfd_internal.h"
+#include "lfd_march.cuh"
+#include "lfd_tc.cuh"
+#include "lfd_tma.cuh"
+
+namespace lfd {
+
+constexpr int kFxN = 80;                     // MMA N: x points of a line tile (nx <= 80)
+constexpr int kFxK = 128;                    // bytes per digit row (K = 2 nproj padded to 128)
+constexpr int kFxSliceB = kFxN * kFxK;       // 10 KB per digit
+constexpr int kFxTileB = kI8S * kFxSliceB;   // 60 KB
+constexpr int kFxSlots = 4;                  // TMEM ring of diagonal accumulators (80 columns each)
+constexpr int kFxWCols = kI8S * (kFxK / 4);  // 192 TMEM columns of W^T digits
+constexpr int kFxAcc = kI8S;                 // diagonals d = 2 .. S+1
+constexpr int kFxEpi = 16;                   // epilogue warps
+constexpr int kFxXg = kFxN / 4;              // x points per epilogue warp
+constexpr int kFxMarch = 2;                  // march warps (one thread per orbital, norb <= 64)
+constexpr int kFxWMma = kFxEpi, kFxWLine = kFxEpi + 1, kFxWMarch0 = kFxEpi + 2;  // MMA warp also loads B's digits
+constexpr int kFxThreads = (kFxEpi + 2 + kFxMarch) * 32;
+constexpr int kFxMaxSmem = 227 * 1024;
+
+struct FxMaps {
+  CUtensorMap dig, psi, phi;
+};
+
+__host__ __device__ inline int fx_al128(int b) { return (b + 127) & ~127; }
+// bytes of one line buffer: Psi [nx][2 norb] doubles + Phi [nx] complex + B's row scales [80]
+__host__ __device__ inline int fx_line_bytes(int nx, int norb) {
+  return fx_al128(nx * norb * 16) + fx_al128(nx * 16) + kFxN * 8;
+}
+static size_t fx_smem(int nx, int norb) { return (size_t)kFxTileB + 2 * fx_line_bytes(nx, norb) + 1024; }
+
+bool gemm2x_supported(const Geometry& g) {
+  return g.i8 && !g.sp && g.nx <= kFxN && g.nx >= 2 && g.norb <= 64 && g.nproj <= 64 &&
+         (long long)g.ny * g.nz < (1LL << 31) && fx_smem(g.nx, g.norb) <= (size_t)kFxMaxSmem &&
+         (size_t)kFxTileB + (size_t)g.nproj * g.norb * 16 + 1024 <= (size_t)kFxMaxSmem;
+}
+size_t gemm2x_digit_bytes(const Geometry& g) { return (size_t)g.ndom * g.ny * g.nz * kI8S * g.nx * kFxK; }
+size_t gemm2x_sig_bytes(const Geometry& g) { return (size_t)g.ndom * g.ny * g.nz * kFxN * sizeof(double); }
+
+// ---- B's digits in x-line order (once per lfd_init): warp per grid row ------------------------------------
+// dig [dom][line][6][nx][128 B] plain (the TMA applies the 128B swizzle), sig [dom][line][80] (0 past nx)
+__global__ void __launch_bounds__(256) k_bslicex_i8(const double2* __restrict__ B, int nproj, int nx, int nyz,
+                                                    int8_t* __restrict__ out, double* __restrict__ sig) {
+  pdl_wait();
+  pdl_trigger();
+  const int dom = blockIdx.y, lane = threadIdx.x & 31;
+  const long long r = (long long)blockIdx.x * 8 + (threadIdx.x >> 5);  // grid row x * nyz + line
+  const long long ngp = (long long)nx * nyz;
+  if (r >= ngp) return;
+  double v[4] = {0.0, 0.0, 0.0, 0.0};
+  const int u0 = 2 * lane;
+  const double2* row = B + ((long long)dom * ngp + r) * nproj;
+  if (u0 < nproj) { const double2 a = row[u0]; v[0] = a.x; v[1] = a.y; }
+  if (u0 + 1 < nproj) { const double2 a = row[u0 + 1]; v[2] = a.x; v[3] = a.y; }
+  double mx = fmax(fmax(fabs(v[0]), fabs(v[1])), fmax(fabs(v[2]), fabs(v[3])));
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  const int e = mx > 0.0 ? row_exponent(mx) : 0;
+  uint32_t d[kI8S];
+  digits4(v, e, !(mx > 0.0), d);
+  const int x = (int)(r / nyz), line = (int)(r - (long long)x * nyz);
+  int8_t* tb = out + ((long long)dom * nyz + line) * kI8S * nx * kFxK + (long long)x * kFxK + 4 * lane;
+#pragma unroll
+  for (int i = 0; i < kI8S; ++i) *reinterpret_cast<uint32_t*>(tb + (long long)i * nx * kFxK) = d[i];
+  if (lane == 0) sig[((long long)dom * nyz + line) * kFxN + x] = mx > 0.0 ? ldexp(1.0, e) : 0.0;
+}
+
+cudaError_t launch_bslicex_i8(const Geometry& g, const double2* B, int8_t* dig, double* sig, cudaStream_t st) {
+  const int nyz = g.ny * g.nz;
+  cudaError_t e = cudaMemsetAsync(sig, 0, gemm2x_sig_bytes(g), st);
+  if (e != cudaSuccess) return e;
+  dim3 grid((unsigned)((g.ng + 7) / 8), g.ndom);
+  launch_k(k_bslicex_i8, grid, 256, 0, st, B, g.nproj, g.nx, nyz, dig, sig);
+  return cudaGetLastError();
+}
+
+// ---- the fused kernel ------------------------------------------------------------------------------------
+struct FxArgs {
+  double2* psi;
+  const DomCoef* coef;
+  const double* nfac;
+  const double2* Cp;
+  const double* sig;
+  int ndom, nproj, norb, nx, nyz;
+  long long ng;
+};
+
+template <bool kPer, bool kS>
+__global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_constant__ CUtensorMap tDig,
+                                                             const __grid_constant__ CUtensorMap tPsi,
+                                                             const __grid_constant__ CUtensorMap tPhi, FxArgs p) {
+  // programmatic dependent launch: set-up and the first digit tile (B's digits are constant since lfd_init)
+  // overlap the previous kernel; every other load waits for it (C'', n, Psi, Phi)
+  pdl_trigger();
+  extern __shared__ __align__(1024) unsigned char dsm_raw[];
+  unsigned char* dsm = dsm_raw + ((1024u - (smem_addr(dsm_raw) & 1023u)) & 1023u);
+  const int nx = p.nx, norb = p.norb, nproj = p.nproj, nyz = p.nyz;
+  const int psiB = fx_al128(nx * norb * 16), phiB = fx_al128(nx * 16);
+  const int lineB = psiB + phiB + kFxN * 8;
+  unsigned char* Tsm = dsm;             // [6][80][128 B] digit tile (128B-swizzled)
+  unsigned char* Lsm = dsm + kFxTileB;  // 2 line buffers
+  auto lpsi = [&](int b) { return reinterpret_cast<double*>(Lsm + b * lineB); };
+  auto lphi = [&](int b) { return reinterpret_cast<const double2*>(Lsm + b * lineB + psiB); };
+  auto lsig = [&](int b) { return reinterpret_cast<const double*>(Lsm + b * lineB + psiB + phiB); };
+  unsigned char* Csm = Lsm;  // C'' of the domain, staged before the first line load
+  __shared__ __align__(8) uint64_t bfull, bempty, dfull[kFxSlots], dempty[kFxSlots];
+  __shared__ __align__(8) uint64_t lfull[2], lready[2], lempty[2], cbar;
+  __shared__ uint32_t tmem_base_sh;
+  __shared__ double taus[kI8M];
+
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int dom = blockIdx.y;
+
+  if (warp == kFxWMma) {  // TMEM: W^T digits (192 columns) + 4 accumulator slots x 80 columns
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_addr(&tmem_base_sh)));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  if (tid == 0) {
+    mbar_init(&bfull, 1);
+    mbar_init(&bempty, 1);
+    for (int s = 0; s < kFxSlots; ++s) { mbar_init(&dfull[s], 1); mbar_init(&dempty[s], kFxEpi); }
+    for (int b = 0; b < 2; ++b) { mbar_init(&lfull[b], 1); mbar_init(&lready[b], kFxEpi); mbar_init(&lempty[b], kFxMarch); }
+    mbar_init(&cbar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_base_sh;
+  const uint32_t tacc = tmem + kFxWCols;
+  const long long nlines = nyz;
+  if (warp == kFxWMma && lane == 0 && blockIdx.x < nlines) {  // first digit tile, before the dependency wait
+    mbar_expect_tx(&bfull, kFxTileB);
+    tma_4d(Tsm, &tDig, 0, 0, 0, (int)((long long)dom * nyz + blockIdx.x), &bfull);
+  }
+  pdl_wait();
+
+  if (warp < kFxEpi) {
+    // W^T digits from C'' (one bulk copy into shared memory) into TMEM, as in k_gemm2_i8: thread (warp w, lane)
+    // owns row n = 32 (w & 3) + lane of W^T and the 8 columns of chunk c8 = w >> 2 of each digit
+    if (tid == 0) {
+      mbar_expect_tx(&cbar, (uint32_t)(nproj * norb * 16));
+      tma_row(Csm, p.Cp + (long long)dom * nproj * norb, (uint32_t)(nproj * norb * 16), &cbar);
+    }
+    const int q = warp & 3, c8 = warp >> 2;
+    const int n = 32 * q + lane, s = n >> 1, cn = n & 1;
+    const bool sv = s < norb;
+    mbar_wait(&cbar, 0);
+    const double2* X = reinterpret_cast<const double2*>(Csm) + s;
+    double mx = 0.0;
+    if (sv)
+      for (int u = 0; u < nproj; ++u) {
+        const double2 x = X[u * norb];
+        mx = fmax(mx, fmax(fabs(x.x), fabs(x.y)));
+      }
+    const int e = mx > 0.0 ? row_exponent(mx) : 0;
+    if (c8 == 0) taus[n] = mx > 0.0 ? ldexp(1.0, e - 12) : 0.0;
+    const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
+    uint32_t dg[kI8S][8];
+#pragma unroll
+    for (int w = 0; w < 8; ++w) {
+      double v[4] = {0.0, 0.0, 0.0, 0.0};
+      const int u0 = 16 * c8 + 2 * w;
+      if (sv && u0 < nproj) {
+        const double2 x = X[u0 * norb];
+        v[0] = cn ? x.y : x.x; v[1] = cn ? x.x : -x.y;
+      }
+      if (sv && u0 + 1 < nproj) {
+        const double2 x = X[(u0 + 1) * norb];
+        v[2] = cn ? x.y : x.x; v[3] = cn ? x.x : -x.y;
+      }
+      uint32_t d[kI8S];
+      digits_i64(v, mx > 0.0 ? ldexp(1.0, 41 - e) : 0.0, d);
+#pragma unroll
+      for (int i = 0; i < kI8S; ++i) dg[i][w] = d[i];
+    }
+#pragma unroll
+    for (int i = 0; i < kI8S; ++i) tmem_st8(trow + i * 32 + 8 * c8, dg[i]);
+    asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+  }
+  // W ready and the staged C'' consumed (the line producer then reuses its space)
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+
+  if (warp == kFxWLine) {  // the line: Psi [nx][2 norb], Phi [nx], B's row scales
+    if (lane == 0) {
+      int it = 0;
+      for (long long t = blockIdx.x; t < nlines; t += gridDim.x, ++it) {
+        const int b = it & 1;
+        if (it >= 2) mbar_wait(&lempty[b], (uint32_t)(((it >> 1) - 1) & 1));
+        mbar_expect_tx(&lfull[b], (uint32_t)(nx * norb * 16 + nx * 16 + kFxN * 8));
+        tma_4d(lpsi(b), &tPsi, 0, (int)t, 0, dom, &lfull[b]);
+        tma_4d(const_cast<double2*>(lphi(b)), &tPhi, 0, (int)t, 0, dom, &lfull[b]);
+        tma_row(const_cast<double*>(lsig(b)), p.sig + ((long long)dom * nyz + t) * kFxN, kFxN * 8, &lfull[b]);
+      }
+    }
+  } else if (warp == kFxWMma) {  // D_d += W_j^T (TMEM) x b_i (smem), i + j = d; one ring slot per diagonal
+    const uint64_t db0 = umma_desc_sw128(smem_addr(Tsm));
+    int it = 0;
+    for (long long t = blockIdx.x; t < nlines; t += gridDim.x, ++it) {
+      mbar_wait(&bfull, (uint32_t)(it & 1));
+      tc_fence_after();
+#pragma unroll
+      for (int d = 2; d <= kI8S + 1; ++d) {
+        const int g = it * kFxAcc + (d - 2), sl = g % kFxSlots;
+        if (g >= kFxSlots) {
+          mbar_wait(&dempty[sl], (uint32_t)(((g / kFxSlots) - 1) & 1));
+          tc_fence_after();
+        }
+        const uint32_t acc = tacc + sl * kFxN;
+        uint32_t first = 1;
+#pragma unroll
+        for (int i = 1; i <= kI8S; ++i) {
+          const int j = d - i;
+          if (j < 1 || j > kI8S) continue;
+#pragma unroll
+          for (int kk = 0; kk < kFxK / 32; ++kk) {
+            umma_i8_ts(acc, tmem + (j - 1) * 32 + kk * 8, db0 + (uint64_t)(((i - 1) * kFxSliceB + kk * 32) >> 4),
+                       first ? 0u : 1u, i8_idesc(kFxN));
+            first = 0;
+          }
+        }
+        umma_commit(&dfull[sl]);
+      }
+      umma_commit(&bempty);  // the digit tile may be overwritten once these MMAs are done
+      const long long tn = t + gridDim.x;
+      if (tn < nlines) {  // the next line's digit tile
+        mbar_wait(&bempty, (uint32_t)(it & 1));
+        if (lane == 0) {
+          mbar_expect_tx(&bfull, kFxTileB);
+          tma_4d(Tsm, &tDig, 0, 0, 0, (int)((long long)dom * nyz + tn), &bfull);
+        }
+        __syncwarp();
+      }
+    }
+  } else if (warp < kFxEpi) {
+    // epilogue: lanes 32 (w & 3) .. (TMEM lane = output double n of a Psi row), x group 20 (w >> 2) ..;
+    // diagonals drained two at a time ((P_d 2^7 + P_{d+1}) is an exact int32), then Psi1 = n Psi + sigma tau acc
+    // written over the line's staged Psi
+    const int q = warp & 3, h = warp >> 2;
+    const int n = 32 * q + lane;
+    const bool nvalid = n < 2 * norb;
+    const double nf = nvalid ? p.nfac[(long long)dom * norb + (n >> 1)] : 0.0;
+    const double tau = taus[n];
+    const int x0 = kFxXg * h;
+    const int nxc = min(max(nx - x0, 0), kFxXg);  // valid x of this warp
+    const int ld2 = 2 * norb;
+    int it = 0;
+    for (long long t = blockIdx.x; t < nlines; t += gridDim.x, ++it) {
+      const int b = it & 1;
+      double fa[kFxXg];
+#pragma unroll
+      for (int c = 0; c < kFxXg; ++c) fa[c] = 0.0;
+#pragma unroll 1
+      for (int dp = 0; dp < kFxAcc / 2; ++dp) {
+        const int g = it * kFxAcc + 2 * dp, s0 = g % kFxSlots, s1 = (g + 1) % kFxSlots;
+        mbar_wait(&dfull[s0], (uint32_t)((g / kFxSlots) & 1));
+        mbar_wait(&dfull[s1], (uint32_t)(((g + 1) / kFxSlots) & 1));
+        tc_fence_after();
+        const uint32_t lb = ((uint32_t)(32 * q) << 16) + x0;
+        const double wd = ldexp(1.0, -14 * dp - 7);
+        {  // x 0..15 of the warp's group, then 16..19 (two loads keep the register peak low)
+          int32_t a0[16], a1[16];
+          tmem_ld16(tacc + s0 * kFxN + lb, a0);
+          tmem_ld16(tacc + s1 * kFxN + lb, a1);
+          tmem_wait_ld();
+          if (dp == 0) {
+#pragma unroll
+            for (int c = 0; c < 16; ++c) fa[c] = fma(i2d_raw(a0[c] * 128 + a1[c]), wd, -kI2dM * wd);
+          } else {
+#pragma unroll
+            for (int c = 0; c < 16; ++c) fa[c] = fma(i2d(a0[c] * 128 + a1[c]), wd, fa[c]);
+          }
+        }
+        {
+          int32_t c0[4], c1[4];
+          tmem_ld4(tacc + s0 * kFxN + lb + 16, c0);
+          tmem_ld4(tacc + s1 * kFxN + lb + 16, c1);
+          tmem_wait_ld();
+          if (dp == 0) {
+#pragma unroll
+            for (int c = 0; c < 4; ++c) fa[16 + c] = fma(i2d_raw(c0[c] * 128 + c1[c]), wd, -kI2dM * wd);
+          } else {
+#pragma unroll
+            for (int c = 0; c < 4; ++c) fa[16 + c] = fma(i2d(c0[c] * 128 + c1[c]), wd, fa[16 + c]);
+          }
+        }
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) {
+          mbar_arrive(&dempty[s0]);
+          mbar_arrive(&dempty[s1]);
+        }
+      }
+      mbar_wait(&lfull[b], (uint32_t)((it >> 1) & 1));
+      if (nvalid) {
+        double* ps = lpsi(b) + (long long)x0 * ld2 + n;
+        const double* sg = lsig(b) + x0;
+#pragma unroll
+        for (int c = 0; c < kFxXg; ++c) {
+          if (c < nxc) *ps = fma(nf, *ps, scale_pow2(fa[c], sg[c], tau));
+          ps += ld2;
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&lready[b]);
+    }
+  } else {
+    // march warps: thread s streams K_x (Phi . ) along the line for orbital s (smem in, HBM out)
+    const int s = tid - kFxWMarch0 * 32;
+    const bool active = s < norb;
+    const PairCoef cf = pair_coef<kS>(p.coef + dom, 0);
+    int it = 0;
+    for (long long t = blockIdx.x; t < nlines; t += gridDim.x, ++it) {
+      const int b = it & 1;
+      mbar_wait(&lready[b], (uint32_t)((it >> 1) & 1));
+      if (active) {
+        const double2* L = reinterpret_cast<const double2*>(lpsi(b)) + s;
+        const double2* ph = lphi(b);
+        double2* out = p.psi + ((long long)dom * p.ng + t) * norb + s;
+        const long long xs = (long long)nyz * norb;  // element stride between x points
+        march_line<kPer, kS, double2, double2>(
+            nx, cf, [&](int i) { return cmul(ph[i], L[i * norb]); }, [&](int i, double2 v) { out[i * xs] = v; });
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&lempty[b]);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == kFxWMma) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
+  }
+}
+
+FxMaps* gemm2x_maps_create(const Geometry& g, const int8_t* dig, double2* psi, const double2* phi) {
+  FxMaps* m = new (std::nothrow) FxMaps;
+  if (!m) return nullptr;
+  const uint64_t nyz = (uint64_t)g.ny * g.nz;
+  // digits [dom*nyz lines][6][nx][128 B], box [1][6][80][128] with the 128B swizzle (x rows past nx zero)
+  const uint64_t dd[4] = {(uint64_t)kFxK, (uint64_t)g.nx, (uint64_t)kI8S, (uint64_t)g.ndom * nyz};
+  const uint64_t sd[3] = {(uint64_t)kFxK, (uint64_t)g.nx * kFxK, (uint64_t)kI8S * g.nx * kFxK};
+  const uint32_t bd[4] = {(uint32_t)kFxK, (uint32_t)kFxN, (uint32_t)kI8S, 1};
+  // Psi as doubles [dom][x][yz][2 norb], box [1][nx][1][2 norb]: the line (y, z) of all orbitals
+  const uint64_t dp[4] = {(uint64_t)2 * g.norb, nyz, (uint64_t)g.nx, (uint64_t)g.ndom};
+  const uint64_t sp[3] = {(uint64_t)g.norb * 16, nyz * g.norb * 16, (uint64_t)g.ng * g.norb * 16};
+  const uint32_t bp[4] = {(uint32_t)(2 * g.norb), 1, (uint32_t)g.nx, 1};
+  // Phi as doubles [dom][x][yz][2], box [1][nx][1][2]
+  const uint64_t df[4] = {2, nyz, (uint64_t)g.nx, (uint64_t)g.ndom};
+  const uint64_t sf[3] = {16, nyz * 16, (uint64_t)g.ng * 16};
+  const uint32_t bf[4] = {2, 1, (uint32_t)g.nx, 1};
+  if (encode_tmap(&m->dig, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, dig, dd, sd, bd, CU_TENSOR_MAP_SWIZZLE_128B) !=
+          cudaSuccess ||
+      encode_tmap(&m->psi, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, psi, dp, sp, bp, CU_TENSOR_MAP_SWIZZLE_NONE) !=
+          cudaSuccess ||
+      encode_tmap(&m->phi, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, phi, df, sf, bf, CU_TENSOR_MAP_SWIZZLE_NONE) !=
+          cudaSuccess) {
+    delete m;
+    return nullptr;
+  }
+  return m;
+}
+
+void gemm2x_maps_destroy(FxMaps* m) { delete m; }
+
+cudaError_t launch_gemm2x_i8(const Geometry& g, const FxMaps* m, double2* psi, const DomCoef* coef, const double* nfac,
+                             const double2* Cp, const double* sig, bool scaled, int num_sms, cudaStream_t st) {
+  FxArgs a;
+  a.psi = psi; a.coef = coef; a.nfac = nfac; a.Cp = Cp; a.sig = sig;
+  a.ndom = g.ndom; a.nproj = g.nproj; a.norb = g.norb; a.nx = g.nx; a.nyz = g.ny * g.nz; a.ng = g.ng;
+  int cpd = num_sms / g.ndom;
+  if (cpd < 1) cpd = 1;
+  if (cpd > a.nyz) cpd = a.nyz;
+  dim3 grid(cpd, g.ndom);
+  // the C'' staging (nproj x norb complex) lives in the line-buffer region before the first line load
+  const size_t sm = std::max(fx_smem(g.nx, g.norb), (size_t)kFxTileB + (size_t)g.nproj * g.norb * 16 + 1024);
+  if (g.bc == 0) {
+    if (scaled) launch_k(k_gemm2x_i8<true, true>, grid, kFxThreads, sm, st, m->dig, m->psi, m->phi, a);
+    else launch_k(k_gemm2x_i8<true, false>, grid, kFxThreads, sm, st, m->dig, m->psi, m->phi, a);
+  } else {
+    if (scaled) launch_k(k_gemm2x_i8<false, true>, grid, kFxThreads, sm, st, m->dig, m->psi, m->phi, a);
+    else launch_k(k_gemm2x_i8<false, false>, grid, kFxThreads, sm, st, m->dig, m->psi, m->phi, a);
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t gemm2x_set_attributes() {
+  for (auto f : {k_gemm2x_i8<true, true>, k_gemm2x_i8<true, false>, k_gemm2x_i8<false, true>,
+                 k_gemm2x_i8<false, false>}) {
+    cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kFxMaxSmem);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+}  // namespace lfd

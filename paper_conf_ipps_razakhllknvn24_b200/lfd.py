@@ -29,7 +29,7 @@ LFD_BC_ZERO = 1
 STATUS = {0: "LFD_OK", -1: "LFD_EINVAL", -2: "LFD_ENOMEM", -3: "LFD_ECUDA", -4: "LFD_ESTATE",
           -5: "LFD_EUNSUPPORTED"}
 KERNELS = ("coef", "phase", "kin_x", "kin_y", "kin_z", "nl_proj", "nl_reduce", "nl_norm", "nl_back",
-           "density", "jreduce", "energy", "nl_carry", "kin_yz", "sc", "fft")
+           "density", "jreduce", "energy", "nl_carry", "kin_yz", "sc", "fft", "nl_back_x")
 LFD_SC_HARTREE = 1
 LFD_SC_XC = 2
 LFD_SC_MAXWELL = 4

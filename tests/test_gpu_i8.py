@@ -147,3 +147,48 @@ def test_i8_large_scissor_gemm_accuracy(name):
           f"int8 vs dmma {rel(gi8[0], gdm[0]):.2e}; implied per-factor product error "
           f"{e_i8[0] / max(upd, 1e-300) / np.sqrt(2 * steps):.2e}")
     assert upd > 0.1  # the test really exercises O(1) nonlocal updates
+
+
+def test_fused_first_factor_launch_classes_c2():
+    """C2 default path: the first nonlocal factor's GEMM-2 runs fused with Phi . K_x (nl_fx.cu) -- per step one
+    k_gemm2x_i8, no separate x pass, one plain GEMM-2 (the second factor), one GEMM-1 (the first factor's C comes
+    from the projection carry after step 1)."""
+    from paper_conf_ipps_razakhllknvn24_b200 import lfd
+    w = workload("C2")
+    x = make_inputs(w, seed=3)
+    ctx, _ = _ctx(w, x)
+    import torch
+    ctx.set_potential(torch.from_numpy(x.vloc).to("cuda:0"))
+    ctx.step(1)
+    lfd.lfd_profile_enable(ctx.ctx, True)
+    ctx.step(3)
+    prof = lfd.lfd_profile_read(ctx.ctx)
+    ctx.close()
+    assert prof["nl_back_x"][1] == 3 and prof["kin_x"][1] == 0 and prof["nl_back"][1] == 3
+    assert prof["kin_yz"][1] == 3 and prof["nl_proj"][1] == 3 and prof["nl_carry"][1] == 3
+
+
+@pytest.mark.parametrize("name,steps,chunk", [("P0", 40, None), ("P2z", 20, 7), ("C1", 10, None)])
+def test_fused_first_factor_in_sequences(name, steps, chunk):
+    """merged sequences with the int8 path forced: every merged factor N o N feeds the next step's x pass through
+    the fused kernel (set_A of that step enqueued before it); per-step oracle at the FP64 bound"""
+    from .test_gpu_parity import run_gpu_sequence
+    w = workload(name)
+    x = make_inputs(w, seed=4)
+    A = laser(w)
+    assert_parity(w, run_gpu_sequence(w, x, steps, A, chunk, flags=FLAG_I8), run_ref(w, x, steps, A))
+
+
+@pytest.mark.parametrize("name,steps", [("P0", 40), ("C1", 10)])
+def test_fused_first_factor_exact_nl(name, steps):
+    """the exactly unitary factor (n = 1, C'' = W C) through the fused first-factor kernel"""
+    from oracle import ref
+    w = workload(name)
+    x = make_inputs(w, seed=5)
+    A = laser(w)
+    got = run_gpu(w, x, steps, A, flags=FLAG_I8 | 2)  # 2 = LFD_FLAG_EXACT_NL
+    cfg = ref.RefConfig(w.ndom, w.nx, w.ny, w.nz, w.hx, w.hy, w.hz, w.bc, w.norb, w.nproj, w.dt)
+    p = x.psi0.copy()
+    for n in range(steps):
+        ref.step_exact(cfg, p, x.proj, x.dnl, x.vloc, A(n), 1)
+    assert rel(got[0], p) < 1e-10

@@ -265,13 +265,13 @@ def test_launch_count_and_profile():
     ctx.close()
 
 
-def run_gpu_sequence(w, x, steps, A_fn, chunk=None):
+def run_gpu_sequence(w, x, steps, A_fn, chunk=None, flags=0):
     torch = _torch()
     from paper_conf_ipps_razakhllknvn24_b200 import Context
     dev = torch.device("cuda:0")
     psi = torch.from_numpy(x.psi0.copy()).to(dev)
     proj = torch.from_numpy(x.proj).to(dev) if w.nproj > 0 else None
-    ctx = Context(psi, proj, x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc)
+    ctx = Context(psi, proj, x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt, bc=w.bc, flags=flags)
     ctx.set_potential(torch.from_numpy(x.vloc).to(dev))
     A_seq = np.stack([A_fn(n) for n in range(steps)])
     chunk = chunk or steps
