@@ -41,7 +41,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
     def compile_one(src):
         obj = os.path.join(OBJ, os.path.basename(src)[:-3] + ".o")
-        cmd = [NVCC, *FLAGS, "-c", "-o", obj, src]
+        # extra -D defines for A/B experiments (build-time only; e.g. the role-wait printf instrumentation)
+        cmd = [NVCC, *FLAGS, *os.environ.get("LFD_NVCC_DEFINES", "").split(), "-c", "-o", obj, src]
         if verbose:
             cmd.insert(1, "-Xptxas=-v")
         return obj, subprocess.run(cmd, capture_output=True, text=True)

@@ -198,4 +198,36 @@ __device__ __forceinline__ void march_line(int n, const PairCoefT<C>& cf, LD&& l
   L.template finish<kPeriodic>(cf, n, st);
 }
 
+// The same K_d on a periodic line (n even, n >= 8) as two segments A = [0, LA) and B = [LA, n), LA = 2 ceil(n/4),
+// marched side by side by one thread (two independent dependency chains, half the chain length); the links
+// across the segment ends -- (LA-1, LA) and the wrap (n-1, 0) -- are taken at the end from the segments' first
+// and last E outputs, as finish() takes the wrap of a single line. Same outputs, same arithmetic per output.
+template <bool kS, class C, class V, class LD, class ST>
+__device__ __forceinline__ void march_line2(int n, const PairCoefT<C>& c, LD&& ld, ST&& st) {
+  const int PA = (n / 2 + 1) / 2, PB = n / 2 - PA, LA = 2 * PA;
+  LineMarch<kS, C, V> A, B;
+  A.init();
+  B.init();
+  A.first(c, ld(0), ld(1));
+  B.first(c, ld(LA), ld(LA + 1));
+  A.second(c, ld(2), ld(3));
+  B.second(c, ld(LA + 2), ld(LA + 3));
+  for (int p = 2; p < PA; ++p) {
+    A.steady(c, ld(2 * p), ld(2 * p + 1), [&](int k, V v) { st(2 * p - 2 + k, v); });
+    if (p < PB) B.steady(c, ld(LA + 2 * p), ld(LA + 2 * p + 1), [&](int k, V v) { st(LA + 2 * p - 2 + k, v); });
+  }
+  const V OAl = lk_L<kS>(c.a2, c.u2, A.prev_e1, B.E10);  // O output at LA - 1
+  const V OBf = lk_R<kS>(c.a2, c.d2, A.prev_e1, B.E10);  // O output at LA
+  const V OBl = lk_L<kS>(c.a2, c.u2, B.prev_e1, A.E10);  // O output at n - 1 (wrap link)
+  const V OAf = lk_R<kS>(c.a2, c.d2, B.prev_e1, A.E10);  // O output at 0
+  st(LA - 2, lk_L<kS>(c.a1, c.u1, A.prev_oR, OAl));
+  st(LA - 1, lk_R<kS>(c.a1, c.d1, A.prev_oR, OAl));
+  st(n - 2, lk_L<kS>(c.a1, c.u1, B.prev_oR, OBl));
+  st(n - 1, lk_R<kS>(c.a1, c.d1, B.prev_oR, OBl));
+  st(0, lk_L<kS>(c.a1, c.u1, OAf, A.O1));
+  st(1, lk_R<kS>(c.a1, c.d1, OAf, A.O1));
+  st(LA, lk_L<kS>(c.a1, c.u1, OBf, B.O1));
+  st(LA + 1, lk_R<kS>(c.a1, c.d1, OBf, B.O1));
+}
+
 }  // namespace lfd

@@ -17,13 +17,25 @@
 // 192 columns) + a 4-slot ring of 80-column diagonal accumulators.
 #include <algorithm>
 #include <new>
+#ifdef LFD_FX_TIMING
+#include <cstdio>
+#endif
 
 #include "lfd_internal.h"
-#include "lfd_march.cuh"
+#include "lfd_march.cuh"  // PairCoef, pair_coef
 #include "lfd_tc.cuh"
 #include "lfd_tma.cuh"
 
 namespace lfd {
+
+// Role-wait instrumentation for A/B experiments only (compiled in with -DLFD_FX_TIMING; printf from two CTAs)
+#ifdef LFD_FX_TIMING
+#define FX_T0(v) long long v = clock64()
+#define FX_ACC(acc, v) acc += clock64() - v
+#else
+#define FX_T0(v)
+#define FX_ACC(acc, v)
+#endif
 
 constexpr int kFxN = 80;                     // MMA N: x points of a line tile (nx <= 80)
 constexpr int kFxK = 128;                    // bytes per digit row (K = 2 nproj padded to 128)
@@ -34,10 +46,12 @@ constexpr int kFxWCols = kI8S * (kFxK / 4);  // 192 TMEM columns of W^T digits
 constexpr int kFxAcc = kI8S;                 // diagonals d = 2 .. S+1
 constexpr int kFxEpi = 16;                   // epilogue warps
 constexpr int kFxXg = kFxN / 4;              // x points per epilogue warp
-constexpr int kFxMarch = 2;                  // march warps (one thread per orbital, norb <= 64)
-constexpr int kFxWMma = kFxEpi, kFxWLine = kFxEpi + 1, kFxWMarch0 = kFxEpi + 2;  // MMA warp also loads B's digits
-constexpr int kFxThreads = (kFxEpi + 2 + kFxMarch) * 32;
-constexpr int kFxMaxSmem = 227 * 1024;
+constexpr int kFxMarch = 4;                  // march warps (one warpgroup): 64 orbitals x 2 segments of each line
+constexpr int kFxSeg = 2;                    // segments of a periodic line marched in parallel
+constexpr int kFxWMarch0 = kFxEpi, kFxWMma = kFxEpi + kFxMarch, kFxWLine = kFxWMma + 1;  // + 2 idle warps
+constexpr int kFxThreads = (kFxEpi + kFxMarch + 4) * 32;  // 24 warps = 6 warpgroups (setmaxnreg: 96 / 64)
+constexpr int kFxXchB = 2 * kFxSeg * 64 * 32;             // segment boundary E outputs [parity][seg][s][2]
+constexpr int kFxMaxSmem = 225 * 1024;  // dynamic (the static barriers and tau table take the rest)
 
 struct FxMaps {
   CUtensorMap dig, psi, phi;
@@ -48,7 +62,7 @@ __host__ __device__ inline int fx_al128(int b) { return (b + 127) & ~127; }
 __host__ __device__ inline int fx_line_bytes(int nx, int norb) {
   return fx_al128(nx * norb * 16) + fx_al128(nx * 16) + kFxN * 8;
 }
-static size_t fx_smem(int nx, int norb) { return (size_t)kFxTileB + 2 * fx_line_bytes(nx, norb) + 1024; }
+static size_t fx_smem(int nx, int norb) { return (size_t)kFxTileB + 2 * fx_line_bytes(nx, norb) + kFxXchB + 1024; }
 
 bool gemm2x_supported(const Geometry& g) {
   return g.i8 && !g.sp && g.nx <= kFxN && g.nx >= 2 && g.norb <= 64 && g.nproj <= 64 &&
@@ -95,6 +109,64 @@ cudaError_t launch_bslicex_i8(const Geometry& g, const double2* B, int8_t* dig, 
   return cudaGetLastError();
 }
 
+// ---- K_x on lane components ------------------------------------------------------------------------------
+// The epilogue lane n = 2 s + c holds component c (0 re, 1 im) of orbital s; z_p, its partner component, is the
+// neighbour lane's (shfl_xor 1). For complex w: (w z)_c = w.x z_c + sgn w.y z_p with sgn = -1 (c = 0), +1 (c = 1).
+__device__ __forceinline__ double cmul_c(double2 w, double zc, double zp, double sgn) {
+  return fma(w.x, zc, sgn * w.y * zp);
+}
+// K_x of one periodic line (nx even, >= 8) for one orbital, as march_line2 (lfd_march.cuh: two segments marched
+// side by side) with explicit shared-memory loads and running store pointers (the generic lambda form recomputed
+// the shared-window base and 64-bit addresses every pair)
+__device__ __forceinline__ double2 ld_sh2(uint32_t a) {
+  double2 v;
+  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "r"(a));
+  return v;
+}
+template <bool kS>
+__device__ __forceinline__ void fx_march2(int n, const PairCoef& c, uint32_t l0, uint32_t ls, double2* out,
+                                          long long xs) {
+  const int PA = (n / 2 + 1) / 2, PB = n / 2 - PA, LA = 2 * PA;
+  LineMarch<kS> A, B;
+  A.init();
+  B.init();
+  uint32_t la = l0, lb = l0 + (uint32_t)LA * ls;
+  A.first(c, ld_sh2(la), ld_sh2(la + ls));
+  B.first(c, ld_sh2(lb), ld_sh2(lb + ls));
+  la += 2 * ls;
+  lb += 2 * ls;
+  A.second(c, ld_sh2(la), ld_sh2(la + ls));
+  B.second(c, ld_sh2(lb), ld_sh2(lb + ls));
+  la += 2 * ls;
+  lb += 2 * ls;
+  double2* oa = out + 2 * xs;  // stores of the steady loop at pair p: points 2p-2, 2p-1 (A), LA + 2p-2 .. (B)
+  double2* ob = out + (long long)(LA + 2) * xs;
+  for (int p = 2; p < PA; ++p) {
+    const double2 aa = ld_sh2(la), ab = ld_sh2(la + ls);
+    A.steady(c, aa, ab, [&](int k, double2 v) { oa[k * xs] = v; });
+    la += 2 * ls;
+    oa += 2 * xs;
+    if (p < PB) {
+      const double2 ba = ld_sh2(lb), bb = ld_sh2(lb + ls);
+      B.steady(c, ba, bb, [&](int k, double2 v) { ob[k * xs] = v; });
+      lb += 2 * ls;
+      ob += 2 * xs;
+    }
+  }
+  const double2 OAl = lk_L<kS>(c.a2, c.u2, A.prev_e1, B.E10);
+  const double2 OBf = lk_R<kS>(c.a2, c.d2, A.prev_e1, B.E10);
+  const double2 OBl = lk_L<kS>(c.a2, c.u2, B.prev_e1, A.E10);
+  const double2 OAf = lk_R<kS>(c.a2, c.d2, B.prev_e1, A.E10);
+  out[(long long)(LA - 2) * xs] = lk_L<kS>(c.a1, c.u1, A.prev_oR, OAl);
+  out[(long long)(LA - 1) * xs] = lk_R<kS>(c.a1, c.d1, A.prev_oR, OAl);
+  out[(long long)(n - 2) * xs] = lk_L<kS>(c.a1, c.u1, B.prev_oR, OBl);
+  out[(long long)(n - 1) * xs] = lk_R<kS>(c.a1, c.d1, B.prev_oR, OBl);
+  out[0] = lk_L<kS>(c.a1, c.u1, OAf, A.O1);
+  out[xs] = lk_R<kS>(c.a1, c.d1, OAf, A.O1);
+  out[(long long)LA * xs] = lk_L<kS>(c.a1, c.u1, OBf, B.O1);
+  out[(long long)(LA + 1) * xs] = lk_R<kS>(c.a1, c.d1, OBf, B.O1);
+}
+
 // ---- the fused kernel ------------------------------------------------------------------------------------
 struct FxArgs {
   double2* psi;
@@ -124,6 +196,7 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
   auto lphi = [&](int b) { return reinterpret_cast<const double2*>(Lsm + b * lineB + psiB); };
   auto lsig = [&](int b) { return reinterpret_cast<const double*>(Lsm + b * lineB + psiB + phiB); };
   unsigned char* Csm = Lsm;  // C'' of the domain, staged before the first line load
+  double2* Xsm = reinterpret_cast<double2*>(Lsm + 2 * lineB);  // march segments' boundary values
   __shared__ __align__(8) uint64_t bfull, bempty, dfull[kFxSlots], dempty[kFxSlots];
   __shared__ __align__(8) uint64_t lfull[2], lready[2], lempty[2], cbar;
   __shared__ uint32_t tmem_base_sh;
@@ -203,59 +276,11 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
+  // registers (setmaxnreg, per warpgroup at the top of each role): the epilogue warpgroups hold 20 FP64
+  // accumulators + two 16-wide TMEM loads per lane (96); the march and MMA / producer warpgroups need 64
 
-  if (warp == kFxWLine) {  // the line: Psi [nx][2 norb], Phi [nx], B's row scales
-    if (lane == 0) {
-      int it = 0;
-      for (long long t = blockIdx.x; t < nlines; t += gridDim.x, ++it) {
-        const int b = it & 1;
-        if (it >= 2) mbar_wait(&lempty[b], (uint32_t)(((it >> 1) - 1) & 1));
-        mbar_expect_tx(&lfull[b], (uint32_t)(nx * norb * 16 + nx * 16 + kFxN * 8));
-        tma_4d(lpsi(b), &tPsi, 0, (int)t, 0, dom, &lfull[b]);
-        tma_4d(const_cast<double2*>(lphi(b)), &tPhi, 0, (int)t, 0, dom, &lfull[b]);
-        tma_row(const_cast<double*>(lsig(b)), p.sig + ((long long)dom * nyz + t) * kFxN, kFxN * 8, &lfull[b]);
-      }
-    }
-  } else if (warp == kFxWMma) {  // D_d += W_j^T (TMEM) x b_i (smem), i + j = d; one ring slot per diagonal
-    const uint64_t db0 = umma_desc_sw128(smem_addr(Tsm));
-    int it = 0;
-    for (long long t = blockIdx.x; t < nlines; t += gridDim.x, ++it) {
-      mbar_wait(&bfull, (uint32_t)(it & 1));
-      tc_fence_after();
-#pragma unroll
-      for (int d = 2; d <= kI8S + 1; ++d) {
-        const int g = it * kFxAcc + (d - 2), sl = g % kFxSlots;
-        if (g >= kFxSlots) {
-          mbar_wait(&dempty[sl], (uint32_t)(((g / kFxSlots) - 1) & 1));
-          tc_fence_after();
-        }
-        const uint32_t acc = tacc + sl * kFxN;
-        uint32_t first = 1;
-#pragma unroll
-        for (int i = 1; i <= kI8S; ++i) {
-          const int j = d - i;
-          if (j < 1 || j > kI8S) continue;
-#pragma unroll
-          for (int kk = 0; kk < kFxK / 32; ++kk) {
-            umma_i8_ts(acc, tmem + (j - 1) * 32 + kk * 8, db0 + (uint64_t)(((i - 1) * kFxSliceB + kk * 32) >> 4),
-                       first ? 0u : 1u, i8_idesc(kFxN));
-            first = 0;
-          }
-        }
-        umma_commit(&dfull[sl]);
-      }
-      umma_commit(&bempty);  // the digit tile may be overwritten once these MMAs are done
-      const long long tn = t + gridDim.x;
-      if (tn < nlines) {  // the next line's digit tile
-        mbar_wait(&bempty, (uint32_t)(it & 1));
-        if (lane == 0) {
-          mbar_expect_tx(&bfull, kFxTileB);
-          tma_4d(Tsm, &tDig, 0, 0, 0, (int)((long long)dom * nyz + tn), &bfull);
-        }
-        __syncwarp();
-      }
-    }
-  } else if (warp < kFxEpi) {
+  if (warp < kFxEpi) {
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 88;\n" ::: "memory");
     // epilogue: lanes 32 (w & 3) .. (TMEM lane = output double n of a Psi row), x group 20 (w >> 2) ..;
     // diagonals drained two at a time ((P_d 2^7 + P_{d+1}) is an exact int32), then Psi1 = n Psi + sigma tau acc
     // written over the line's staged Psi
@@ -267,6 +292,8 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
     const int x0 = kFxXg * h;
     const int nxc = min(max(nx - x0, 0), kFxXg);  // valid x of this warp
     const int ld2 = 2 * norb;
+    long long w_d = 0, w_l = 0;
+    FX_T0(t_all);
     int it = 0;
     for (long long t = blockIdx.x; t < nlines; t += gridDim.x, ++it) {
       const int b = it & 1;
@@ -276,8 +303,10 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
 #pragma unroll 1
       for (int dp = 0; dp < kFxAcc / 2; ++dp) {
         const int g = it * kFxAcc + 2 * dp, s0 = g % kFxSlots, s1 = (g + 1) % kFxSlots;
+        FX_T0(c3);
         mbar_wait(&dfull[s0], (uint32_t)((g / kFxSlots) & 1));
         mbar_wait(&dfull[s1], (uint32_t)(((g + 1) / kFxSlots) & 1));
+        FX_ACC(w_d, c3);
         tc_fence_after();
         const uint32_t lb = ((uint32_t)(32 * q) << 16) + x0;
         const double wd = ldexp(1.0, -14 * dp - 7);
@@ -314,7 +343,10 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
           mbar_arrive(&dempty[s1]);
         }
       }
+      FX_T0(c4);
       mbar_wait(&lfull[b], (uint32_t)((it >> 1) & 1));
+      FX_ACC(w_l, c4);
+      // Psi1 = n Psi + sigma tau acc, written over the line's staged Psi for the march warps
       if (nvalid) {
         double* ps = lpsi(b) + (long long)x0 * ld2 + n;
         const double* sg = lsig(b) + x0;
@@ -327,25 +359,163 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
       __syncwarp();
       if (lane == 0) mbar_arrive(&lready[b]);
     }
-  } else {
-    // march warps: thread s streams K_x (Phi . ) along the line for orbital s (smem in, HBM out)
-    const int s = tid - kFxWMarch0 * 32;
+#ifdef LFD_FX_TIMING
+    if (warp == 0 && lane == 0 && (blockIdx.x == 0 || blockIdx.x == 100))
+      printf("fx cta %d epi0: total %lld wait-diag %lld wait-line %lld\n", blockIdx.x, clock64() - t_all, w_d, w_l);
+#endif
+    (void)w_d; (void)w_l;
+  } else if (warp < kFxEpi + kFxMarch) {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 72;\n" ::: "memory");
+    // march warps: thread (segment g, orbital s) streams K_x over segment g of the line for orbital s (Phi . Psi1
+    // from shared memory, HBM out); the links across segment ends (and the periodic wrap) are taken after a
+    // barrier from the neighbouring segments' first / last E outputs (as finish() takes the wrap of one line).
+    // Lines that do not split (zero BC, nx < 12): segment-0 threads march the whole line (march_line).
+    const int gi = tid - kFxWMarch0 * 32;
+    const int g = gi / 64, s = gi % 64;
     const bool active = s < norb;
+    const bool split = kPer && nx >= 4 * kFxSeg;
+    const int P = nx / 2;  // pairs (periodic: nx even)
+    const int p0 = split ? (g * P) / kFxSeg : 0, p1 = split ? ((g + 1) * P) / kFxSeg : 0;  // this segment's pairs
     const PairCoef cf = pair_coef<kS>(p.coef + dom, 0);
+    const long long xs = (long long)nyz * norb;  // element stride between x points
+    long long w_r = 0;
+    FX_T0(t_all);
     int it = 0;
     for (long long t = blockIdx.x; t < nlines; t += gridDim.x, ++it) {
       const int b = it & 1;
+      FX_T0(c5);
       mbar_wait(&lready[b], (uint32_t)((it >> 1) & 1));
-      if (active) {
-        const double2* L = reinterpret_cast<const double2*>(lpsi(b)) + s;
+      FX_ACC(w_r, c5);
+      const double2* L = reinterpret_cast<const double2*>(lpsi(b)) + s;
+      double2* out = p.psi + ((long long)dom * p.ng + t) * norb + s;
+      if (split) {
+        LineMarch<kS> M;
+        M.init();
+        const uint32_t ls = (uint32_t)norb * 16;
+        uint32_t la = smem_addr(L) + (uint32_t)(2 * p0) * ls;
+        uint32_t lf = smem_addr(lphi(b)) + (uint32_t)(2 * p0) * 16;  // Phi (the x pass's pre-phase)
+        if (active) {
+          M.first(cf, cmul(ld_sh2(lf), ld_sh2(la)), cmul(ld_sh2(lf + 16), ld_sh2(la + ls)));
+          la += 2 * ls;
+          lf += 32;
+          M.second(cf, cmul(ld_sh2(lf), ld_sh2(la)), cmul(ld_sh2(lf + 16), ld_sh2(la + ls)));
+          la += 2 * ls;
+          lf += 32;
+          double2* o = out + (long long)(2 * p0 + 2) * xs;
+          for (int q = p0 + 2; q < p1; ++q) {
+            const double2 a = cmul(ld_sh2(lf), ld_sh2(la)), c = cmul(ld_sh2(lf + 16), ld_sh2(la + ls));
+            M.steady(cf, a, c, [&](int k, double2 v) { o[k * xs] = v; });
+            la += 2 * ls;
+            lf += 32;
+            o += 2 * xs;
+          }
+        }
+        double2* xb = Xsm + ((b * kFxSeg + g) * 64 + s) * 2;  // [E output at the first point, at the last point]
+        xb[0] = M.E10;
+        xb[1] = M.prev_e1;
+        asm volatile("bar.sync 3, %0;" ::"n"(kFxMarch * 32) : "memory");
+        if (active) {
+          const int gl = g > 0 ? g - 1 : kFxSeg - 1, gr = g + 1 < kFxSeg ? g + 1 : 0;
+          const double2 lft = Xsm[((b * kFxSeg + gl) * 64 + s) * 2 + 1];  // left segment's last E output
+          const double2 rgt = Xsm[((b * kFxSeg + gr) * 64 + s) * 2];      // right segment's first E output
+          const double2 Ol = lk_L<kS>(cf.a2, cf.u2, M.prev_e1, rgt);       // O output at the segment's last point
+          const double2 Of = lk_R<kS>(cf.a2, cf.d2, lft, M.E10);           // O output at its first point
+          const int e = 2 * p1;
+          out[(long long)(e - 2) * xs] = lk_L<kS>(cf.a1, cf.u1, M.prev_oR, Ol);
+          out[(long long)(e - 1) * xs] = lk_R<kS>(cf.a1, cf.d1, M.prev_oR, Ol);
+          out[(long long)(2 * p0) * xs] = lk_L<kS>(cf.a1, cf.u1, Of, M.O1);
+          out[(long long)(2 * p0 + 1) * xs] = lk_R<kS>(cf.a1, cf.d1, Of, M.O1);
+        }
+      } else if (g == 0 && active) {
         const double2* ph = lphi(b);
-        double2* out = p.psi + ((long long)dom * p.ng + t) * norb + s;
-        const long long xs = (long long)nyz * norb;  // element stride between x points
         march_line<kPer, kS, double2, double2>(
             nx, cf, [&](int i) { return cmul(ph[i], L[i * norb]); }, [&](int i, double2 v) { out[i * xs] = v; });
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(&lempty[b]);
+    }
+#ifdef LFD_FX_TIMING
+    if (tid == kFxWMarch0 * 32 && (blockIdx.x == 0 || blockIdx.x == 100))
+      printf("fx cta %d march: total %lld wait-ready %lld\n", blockIdx.x, clock64() - t_all, w_r);
+#endif
+    (void)w_r;
+  } else {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 56;\n" ::: "memory");
+    if (warp == kFxWLine) {  // the line: Psi [nx][2 norb], Phi [nx], B's row scales
+      if (lane == 0) {
+        long long w_m = 0;
+        int it = 0;
+        for (long long t = blockIdx.x; t < nlines; t += gridDim.x, ++it) {
+          const int b = it & 1;
+          FX_T0(c6);
+          if (it >= 2) mbar_wait(&lempty[b], (uint32_t)(((it >> 1) - 1) & 1));
+          FX_ACC(w_m, c6);
+          mbar_expect_tx(&lfull[b], (uint32_t)(nx * norb * 16 + nx * 16 + kFxN * 8));
+          tma_4d(lpsi(b), &tPsi, 0, (int)t, 0, dom, &lfull[b]);
+          tma_4d(const_cast<double2*>(lphi(b)), &tPhi, 0, (int)t, 0, dom, &lfull[b]);
+          tma_row(const_cast<double*>(lsig(b)), p.sig + ((long long)dom * nyz + t) * kFxN, kFxN * 8, &lfull[b]);
+        }
+  #ifdef LFD_FX_TIMING
+        if (blockIdx.x == 0 || blockIdx.x == 100) printf("fx cta %d line: wait-empty %lld\n", blockIdx.x, w_m);
+  #endif
+        (void)w_m;
+      }
+    } else if (warp == kFxWMma) {  // D_d += W_j^T (TMEM) x b_i (smem), i + j = d; one ring slot per diagonal
+      const uint64_t db0 = umma_desc_sw128(smem_addr(Tsm));
+      long long w_b = 0, w_s = 0, w_e = 0;
+      FX_T0(t_all);
+      int it = 0;
+      for (long long t = blockIdx.x; t < nlines; t += gridDim.x, ++it) {
+        FX_T0(c0);
+        mbar_wait(&bfull, (uint32_t)(it & 1));
+        FX_ACC(w_b, c0);
+        tc_fence_after();
+#pragma unroll
+        for (int d = 2; d <= kI8S + 1; ++d) {
+          const int g = it * kFxAcc + (d - 2), sl = g % kFxSlots;
+          if (g >= kFxSlots) {
+            FX_T0(c1);
+            mbar_wait(&dempty[sl], (uint32_t)(((g / kFxSlots) - 1) & 1));
+            FX_ACC(w_s, c1);
+            tc_fence_after();
+          }
+          const uint32_t acc = tacc + sl * kFxN;
+          uint32_t accum = 0;  // 0 for the diagonal's first MMA
+#pragma unroll
+          for (int i = 1; i <= kI8S; ++i) {
+            const int j = d - i;
+            if (j < 1 || j > kI8S) continue;
+            uint64_t db = db0 + (uint64_t)(((i - 1) * kFxSliceB) >> 4);
+            uint32_t ta = tmem + (j - 1) * 32;
+#pragma unroll 1
+            for (int kk = 0; kk < kFxK / 32; ++kk) {  // (not unrolled: the 64-register warpgroup)
+              umma_i8_ts(acc, ta, db, accum, i8_idesc(kFxN));
+              accum = 1;
+              db += 2;  // 32 bytes >> 4
+              ta += 8;
+            }
+          }
+          umma_commit(&dfull[sl]);
+        }
+        umma_commit(&bempty);  // the digit tile may be overwritten once these MMAs are done
+        const long long tn = t + gridDim.x;
+        if (tn < nlines) {  // the next line's digit tile
+          FX_T0(c2);
+          mbar_wait(&bempty, (uint32_t)(it & 1));
+          FX_ACC(w_e, c2);
+          if (lane == 0) {
+            mbar_expect_tx(&bfull, kFxTileB);
+            tma_4d(Tsm, &tDig, 0, 0, 0, (int)((long long)dom * nyz + tn), &bfull);
+          }
+          __syncwarp();
+        }
+      }
+  #ifdef LFD_FX_TIMING
+      if (lane == 0 && (blockIdx.x == 0 || blockIdx.x == 100))
+        printf("fx cta %d mma: total %lld wait-digits %lld wait-slot %lld wait-mma-done %lld lines %d\n", blockIdx.x,
+               clock64() - t_all, w_b, w_s, w_e, it);
+  #endif
+      (void)w_b; (void)w_s; (void)w_e;
     }
   }
   tc_fence_before();
