@@ -51,6 +51,9 @@ constexpr int kFxSeg = 2;                    // segments of a periodic line marc
 constexpr int kFxWMarch0 = kFxEpi, kFxWMma = kFxEpi + kFxMarch, kFxWLine = kFxWMma + 1;  // + 2 idle warps
 constexpr int kFxThreads = (kFxEpi + kFxMarch + 4) * 32;  // 24 warps = 6 warpgroups (setmaxnreg: 96 / 64)
 constexpr int kFxXchB = 2 * kFxSeg * 64 * 32;             // segment boundary E outputs [parity][seg][s][2]
+// named barriers: epilogue -> march "ready" (2, 3 by line parity), march -> epilogue "free" (4, 5), march only (6)
+constexpr int kFxBarReady = 2, kFxBarFree = 4, kFxBarMarch = 6;
+constexpr int kFxHandoff = (kFxEpi + kFxMarch) * 32;
 constexpr int kFxMaxSmem = 225 * 1024;  // dynamic (the static barriers and tau table take the rest)
 
 struct FxMaps {
@@ -198,7 +201,7 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
   unsigned char* Csm = Lsm;  // C'' of the domain, staged before the first line load
   double2* Xsm = reinterpret_cast<double2*>(Lsm + 2 * lineB);  // march segments' boundary values
   __shared__ __align__(8) uint64_t bfull, bempty, dfull[kFxSlots], dempty[kFxSlots];
-  __shared__ __align__(8) uint64_t lfull[2], lready[2], lempty[2], cbar;
+  __shared__ __align__(8) uint64_t lfull[2], lempty[2], cbar;
   __shared__ uint32_t tmem_base_sh;
   __shared__ double taus[kI8M];
 
@@ -213,7 +216,7 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
     mbar_init(&bfull, 1);
     mbar_init(&bempty, 1);
     for (int s = 0; s < kFxSlots; ++s) { mbar_init(&dfull[s], 1); mbar_init(&dempty[s], kFxEpi); }
-    for (int b = 0; b < 2; ++b) { mbar_init(&lfull[b], 1); mbar_init(&lready[b], kFxEpi); mbar_init(&lempty[b], kFxMarch); }
+    for (int b = 0; b < 2; ++b) { mbar_init(&lfull[b], 1); mbar_init(&lempty[b], kFxMarch); }
     mbar_init(&cbar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -346,7 +349,10 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
       FX_T0(c4);
       mbar_wait(&lfull[b], (uint32_t)((it >> 1) & 1));
       FX_ACC(w_l, c4);
-      // Psi1 = n Psi + sigma tau acc, written over the line's staged Psi for the march warps
+      // Psi1 = n Psi + sigma tau acc, written over the line's staged Psi for the march warps. The handoffs with the
+      // march warps are named barriers (epilogue + march warps): "free" b (the march of line it - 2 is done with
+      // the buffer -- also implied by lfull, whose load waited for it) and "ready" b (Psi1 written)
+      if (it >= 2) asm volatile("bar.sync %0, %1;" ::"r"(kFxBarFree + b), "n"(kFxHandoff) : "memory");
       if (nvalid) {
         double* ps = lpsi(b) + (long long)x0 * ld2 + n;
         const double* sg = lsig(b) + x0;
@@ -356,8 +362,7 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
           ps += ld2;
         }
       }
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&lready[b]);
+      asm volatile("bar.arrive %0, %1;" ::"r"(kFxBarReady + b), "n"(kFxHandoff) : "memory");
     }
 #ifdef LFD_FX_TIMING
     if (warp == 0 && lane == 0 && (blockIdx.x == 0 || blockIdx.x == 100))
@@ -384,7 +389,7 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
     for (long long t = blockIdx.x; t < nlines; t += gridDim.x, ++it) {
       const int b = it & 1;
       FX_T0(c5);
-      mbar_wait(&lready[b], (uint32_t)((it >> 1) & 1));
+      asm volatile("bar.sync %0, %1;" ::"r"(kFxBarReady + b), "n"(kFxHandoff) : "memory");
       FX_ACC(w_r, c5);
       const double2* L = reinterpret_cast<const double2*>(lpsi(b)) + s;
       double2* out = p.psi + ((long long)dom * p.ng + t) * norb + s;
@@ -413,7 +418,7 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
         double2* xb = Xsm + ((b * kFxSeg + g) * 64 + s) * 2;  // [E output at the first point, at the last point]
         xb[0] = M.E10;
         xb[1] = M.prev_e1;
-        asm volatile("bar.sync 3, %0;" ::"n"(kFxMarch * 32) : "memory");
+        asm volatile("bar.sync %0, %1;" ::"n"(kFxBarMarch), "n"(kFxMarch * 32) : "memory");
         if (active) {
           const int gl = g > 0 ? g - 1 : kFxSeg - 1, gr = g + 1 < kFxSeg ? g + 1 : 0;
           const double2 lft = Xsm[((b * kFxSeg + gl) * 64 + s) * 2 + 1];  // left segment's last E output
@@ -432,7 +437,9 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
             nx, cf, [&](int i) { return cmul(ph[i], L[i * norb]); }, [&](int i, double2 v) { out[i * xs] = v; });
       }
       __syncwarp();
-      if (lane == 0) mbar_arrive(&lempty[b]);
+      if (lane == 0) mbar_arrive(&lempty[b]);  // the line producer may reload the buffer
+      if (t + 2 * (long long)gridDim.x < nlines)  // the epilogue syncs on this for line it + 2
+        asm volatile("bar.arrive %0, %1;" ::"r"(kFxBarFree + b), "n"(kFxHandoff) : "memory");
     }
 #ifdef LFD_FX_TIMING
     if (tid == kFxWMarch0 * 32 && (blockIdx.x == 0 || blockIdx.x == 100))
