@@ -469,8 +469,71 @@ def run_small_config(name, args, dev, stream):
     return out
 
 
+def run_c5(args):
+    """--config C5 (BASELINE configs[4]): the nonlocal-projector sweep at Ngrid = 352,800 (the C2 mesh), norb in
+    {32..512} x nproj in {64..1024}. One JSON line per shape: per-launch device time of GEMM-1 (C = dV B^H Psi) and
+    GEMM-2 (Psi <- (Psi + B C') n) from the library's CUDA-event profiler over `steps` LFD steps, the FP64-equivalent
+    rate (8 flops per complex MAC) against the FP64 DMMA peak, the path that ran (FP64 DMMA 3M, or the int8-digit
+    emulation where nproj, norb <= 64), and a GEMM-level accuracy check: one nonlocal factor (lfd_step_prologue)
+    against the same factor computed with cuBLAS ZGEMM (torch.matmul, complex128), as the relative error of the
+    nonlocal update."""
+    import torch
+    from lfd_workloads.configs import C5_NORB, C5_NPROJ, workload
+    from paper_conf_ipps_razakhllknvn24_b200 import Context, lfd
+    pk = peaks()
+    w = workload("C2")
+    ng = w.ngrid
+    shape = (1, w.nx, w.ny, w.nz)
+    for no in C5_NORB:
+        for npj in C5_NPROJ:
+            g = torch.Generator(device="cuda").manual_seed(no * 7919 + npj)
+            psi = torch.randn(shape + (no,), dtype=torch.complex128, device="cuda", generator=g)
+            psi *= (1.0 / (w.dV * ng)) ** 0.5
+            proj = torch.randn(shape + (npj,), dtype=torch.complex128, device="cuda", generator=g)
+            proj *= (1.0 / (w.dV * ng)) ** 0.5
+            dnl = np.full((1, npj), 0.07)
+            ctx = Context(psi, proj, dnl, np.full((1, no), 2.0), (w.hx, w.hy, w.hz), w.dt)
+            path = {0: "fp64-dmma-3m", 1: "int8-digit-tcgen05 (FP64 emulated)"}[lfd.lfd_nl_path(ctx.ctx)]
+            for _ in range(max(1, args.warmup)):
+                ctx.step(1)
+            lfd.lfd_profile_enable(ctx.ctx, True)
+            ctx.step(args.steps)
+            prof = lfd.lfd_profile_read(ctx.ctx)
+            lfd.lfd_profile_enable(ctx.ctx, False)
+            # accuracy: one factor N(Psi) = (Psi - i eps B (D dV B^H Psi)) n, n restoring each column's norm
+            ctx.psi_modified()
+            before = psi.clone()
+            lfd.lfd_step_prologue(ctx.ctx)
+            ctx.sync()
+            P = before.reshape(ng, no)
+            B = proj.reshape(ng, npj)
+            C = w.dV * (B.mH @ P)
+            R = P + B @ ((-0.5j * w.dt * 0.07) * C)
+            R = R * (torch.linalg.vector_norm(P, dim=0) / torch.linalg.vector_norm(R, dim=0))
+            got = psi.reshape(ng, no)
+            acc = float(torch.linalg.vector_norm(got - R) / torch.linalg.vector_norm(R - P))
+            ctx.close()
+            flops = 8.0 * ng * no * npj
+            rec = {"metric": "C5 nonlocal GEMM sweep", "config": {"workload": "C5", "ngrid": ng, "norb": no,
+                                                                  "nproj": npj}, "path": path,
+                   "gflop_per_gemm": flops / 1e9, "update_rel_error_vs_cublas_zgemm": acc,
+                   "peak": {"fp64_dmma_tflops": pk["fp64_tflops"], "source": pk["fp64_src"]}}
+            for k, name in (("nl_proj", "gemm1"), ("nl_back", "gemm2")):
+                ms = prof[k][0] / max(prof[k][1], 1)
+                tf = flops / (ms * 1e-3) / 1e12
+                rec[name] = {"ms": ms, "launches": prof[k][1], "fp64_equiv_tflops": tf,
+                             "frac_of_fp64_dmma_peak": tf / pk["fp64_tflops"],
+                             "frac_of_dmma_pipe_3m": tf / pk["zgemm3m_tflops"]}
+            print(json.dumps(rec), flush=True)
+            del psi, proj, before, P, B, C, R, got
+            torch.cuda.empty_cache()
+
+
 def main():
     args = parse()
+    if args.config == "C5":
+        run_c5(args)
+        return
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))

@@ -212,7 +212,6 @@ long long gemm1_i8_rows_per_split(long long ng, int ndom, int num_sms);
 cudaError_t launch_bslice1_i8(const double2* B, int ndom, int nproj, long long ng, int* bexp, int8_t* out,
                               cudaStream_t st);
 cudaError_t launch_gemm1_i8(const Gemm1I8Args& a, cudaStream_t st);
-int gemm2_smem_bytes();
 cudaError_t gemm_set_attributes();
 
 // Density / current (a7). Output addressing: out index = base[dom] + x*sx + y*sy + z,

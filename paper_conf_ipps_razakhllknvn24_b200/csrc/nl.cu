@@ -37,8 +37,6 @@ constexpr int kThreads1 = kConsWarps1 * 32 + 32;  // + producer warp
 // GEMM-2 stage: A rows [64][kLdA2] (B rows, k = projector along the row) and C' rows [KC2][kLd1].
 constexpr int kKC2 = 32;
 constexpr int kLdA2 = kKC2 + 4;  // 36 == 4 mod 8: conflict-free A-fragment loads
-constexpr int kStages2 = 3;
-constexpr int kStage2Bytes = kTile * kLdA2 * 16 + kKC2 * kLd1 * 16;
 
 __device__ __forceinline__ void dmma(double& c0, double& c1, double a, double b) {
   asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
@@ -191,33 +189,36 @@ __device__ __forceinline__ void mma_conj(FragT<MI, NI>& acc, const double2 (&a)[
     for (int ni = 0; ni < NI; ++ni) dmma(acc.t3[mi][ni][0], acc.t3[mi][ni][1], as[mi], xs[ni]);
 }
 
-template <int kMT>
+// kNT = 32: the N tile for narrow orbital sets (norb <= 32, C5's first row): 4 x 2 warps of 16 x 16, so no DMMA
+// work is spent on empty orbital columns either
+template <int kMT, int kNT = kTile>
 struct G1Shape {
-  static constexpr int WM = kMT == 64 ? 2 : 1;   // warps along M
+  static constexpr int WM = kNT == 32 ? (kMT >= 64 ? 4 : 2) : (kMT == 64 ? 2 : 1);  // warps along M
   static constexpr int WN = 8 / WM;              // warps along N
   static constexpr int MI = kMT / WM / 8;        // 8-row fragments per warp
-  static constexpr int NI = kTile / WN / 8;      // 8-column fragments per warp
+  static constexpr int NI = kNT / WN / 8;        // 8-column fragments per warp
   static constexpr int LDA = kMT + 2;            // smem row pitch of the A block (complex)
+  static constexpr int LDX = kNT + 2;            // smem row pitch of the X block (== 2 mod 8 complex)
   static constexpr int ABytes = kKC1 * LDA * 16;
-  static constexpr int StageBytes = ABytes + kKC1 * kLd1 * 16;
+  static constexpr int StageBytes = ABytes + kKC1 * LDX * 16;
 };
 
-template <int kMT>
+template <int kMT, int kNT = kTile>
 __global__ void __launch_bounds__(kThreads1, 1) k_gemm1(const __grid_constant__ CUtensorMap tA,
                                                          const __grid_constant__ CUtensorMap tX, Gemm1Args p) {
   pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
   pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
-  using S = G1Shape<kMT>;
+  using S = G1Shape<kMT, kNT>;
   extern __shared__ __align__(128) unsigned char smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages1 * S::StageBytes);
   uint64_t* empty = full + kStages1;
-  __shared__ double nsh[2][kTile];
+  __shared__ double nsh[4][kNT];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int split = blockIdx.x;
-  const int ntn = (p.ncols + kTile - 1) / kTile;
+  const int ntn = (p.ncols + kNT - 1) / kNT;
   const int mt = blockIdx.y / ntn, nt = blockIdx.y - (blockIdx.y / ntn) * ntn;
   const int dom = blockIdx.z;
-  const int m0 = mt * kMT, n0 = nt * kTile;
+  const int m0 = mt * kMT, n0 = nt * kNT;
   const long long kbeg = (long long)split * p.rows_per_split;
   const long long kend = min(p.ng, kbeg + p.rows_per_split);
   const int nchunks = (kend > kbeg) ? (int)((kend - kbeg + kKC1 - 1) / kKC1) : 0;
@@ -248,7 +249,7 @@ __global__ void __launch_bounds__(kThreads1, 1) k_gemm1(const __grid_constant__ 
 
   const int g = lane >> 2, t = lane & 3;
   const int wm = warp / S::WN, wn = warp - (warp / S::WN) * S::WN;
-  const int mvalid = min(kMT, p.mrows - m0), nvalid = min(kTile, p.ncols - n0);
+  const int mvalid = min(kMT, p.mrows - m0), nvalid = min(kNT, p.ncols - n0);
   FragT<S::MI, S::NI> acc;
   acc.zero();
   double nrm[S::NI];
@@ -268,7 +269,7 @@ __global__ void __launch_bounds__(kThreads1, 1) k_gemm1(const __grid_constant__ 
 #pragma unroll
       for (int mi = 0; mi < S::MI; ++mi) a[mi] = As[k * S::LDA + wm * (kMT / S::WM) + mi * 8 + g];
 #pragma unroll
-      for (int ni = 0; ni < S::NI; ++ni) x[ni] = Xs[k * kLd1 + wn * (kTile / S::WN) + ni * 8 + g];
+      for (int ni = 0; ni < S::NI; ++ni) x[ni] = Xs[k * S::LDX + wn * (kNT / S::WN) + ni * 8 + g];
       if (do_norm && ((kk >> 2) % S::WM) == wm) {
 #pragma unroll
         for (int ni = 0; ni < S::NI; ++ni) nrm[ni] = fma(x[ni].x, x[ni].x, fma(x[ni].y, x[ni].y, nrm[ni]));
@@ -290,7 +291,7 @@ __global__ void __launch_bounds__(kThreads1, 1) k_gemm1(const __grid_constant__ 
     for (int ni = 0; ni < S::NI; ++ni)
 #pragma unroll
       for (int c = 0; c < 2; ++c) {
-        const int col = wn * (kTile / S::WN) + ni * 8 + 2 * t + c;
+        const int col = wn * (kNT / S::WN) + ni * 8 + 2 * t + c;
         if (col < nvalid) {
           const double t1 = acc.t1[mi][ni][c], t2 = acc.t2[mi][ni][c], t3 = acc.t3[mi][ni][c];
           out[(long long)(m0 + row) * p.ncols + n0 + col] = make_double2(t1 + t2, t3 - t1 + t2);
@@ -303,12 +304,13 @@ __global__ void __launch_bounds__(kThreads1, 1) k_gemm1(const __grid_constant__ 
       double v = nrm[ni];
       v += __shfl_xor_sync(0xffffffffu, v, 1);
       v += __shfl_xor_sync(0xffffffffu, v, 2);
-      if (t == 0) nsh[wm][wn * (kTile / S::WN) + ni * 8 + g] = v;
+      if (t == 0) nsh[wm][wn * (kNT / S::WN) + ni * 8 + g] = v;
     }
     asm volatile("bar.sync 1, %0;" ::"n"(kConsWarps1 * 32));  // consumer warps only
     if (tid < nvalid) {
       double v = nsh[0][tid];
-      if (S::WM == 2) v += nsh[1][tid];
+#pragma unroll
+      for (int q = 1; q < S::WM; ++q) v += nsh[q][tid];
       p.norms[((long long)dom * p.nsplit + split) * p.ncols + n0 + tid] = v;
     }
   }
@@ -317,9 +319,9 @@ __global__ void __launch_bounds__(kThreads1, 1) k_gemm1(const __grid_constant__ 
 static int gemm1_mt(int mrows) { return mrows <= 16 ? 16 : mrows <= 32 ? 32 : 64; }
 
 // A [dom][ng][mrows] / X [dom][ng][ncols] complex as 3-D float64 tensors, boxes [1][kKC1][tile + 2].
-static cudaError_t gemm1_maps(const Gemm1Args& a, int mt, CUtensorMap* tA, CUtensorMap* tX) {
+static cudaError_t gemm1_maps(const Gemm1Args& a, int mt, int nt, CUtensorMap* tA, CUtensorMap* tX) {
   const uint32_t boxA[3] = {(uint32_t)(2 * (mt + 2)), kKC1, 1};
-  const uint32_t boxX[3] = {2 * kLd1, kKC1, 1};
+  const uint32_t boxX[3] = {(uint32_t)(2 * (nt + 2)), kKC1, 1};
   const uint64_t dA[3] = {(uint64_t)2 * a.mrows, (uint64_t)a.ng, (uint64_t)a.ndom};
   const uint64_t sA[2] = {(uint64_t)a.mrows * 16, (uint64_t)a.a_dom_stride * 16};
   cudaError_t e = encode_tmap_f64(tA, 3, a.A, dA, sA, boxA);
@@ -330,21 +332,27 @@ static cudaError_t gemm1_maps(const Gemm1Args& a, int mt, CUtensorMap* tA, CUten
 }
 
 int gemm1_smem_bytes() { return kStages1 * G1Shape<64>::StageBytes + 2 * kStages1 * 8; }
-int gemm2_smem_bytes() { return kStages2 * kStage2Bytes + 2 * kStages2 * 8; }
 
 cudaError_t launch_gemm1(const Gemm1Args& a, cudaStream_t st) {
   const int mt = gemm1_mt(a.mrows);
-  const int tiles = ((a.mrows + mt - 1) / mt) * ((a.ncols + kTile - 1) / kTile);
+  const int nt = a.ncols <= 32 ? 32 : kTile;
+  const int tiles = ((a.mrows + mt - 1) / mt) * ((a.ncols + nt - 1) / nt);
   dim3 grid(a.nsplit, tiles, a.ndom);
   CUtensorMap tA, tX;
-  cudaError_t e = gemm1_maps(a, mt, &tA, &tX);
+  cudaError_t e = gemm1_maps(a, mt, nt, &tA, &tX);
   if (e != cudaSuccess) return e;
-  if (mt == 16)
-    launch_k(k_gemm1<16>, grid, kThreads1, kStages1 * G1Shape<16>::StageBytes + 2 * kStages1 * 8, st, tA, tX, a);
-  else if (mt == 32)
-    launch_k(k_gemm1<32>, grid, kThreads1, kStages1 * G1Shape<32>::StageBytes + 2 * kStages1 * 8, st, tA, tX, a);
-  else
-    launch_k(k_gemm1<64>, grid, kThreads1, gemm1_smem_bytes(), st, tA, tX, a);
+#define LFD_G1(M, N) launch_k(k_gemm1<M, N>, grid, kThreads1, kStages1 * G1Shape<M, N>::StageBytes + 2 * kStages1 * 8, \
+                              st, tA, tX, a)
+  if (nt == 32) {
+    if (mt == 16) LFD_G1(16, 32);
+    else if (mt == 32) LFD_G1(32, 32);
+    else LFD_G1(64, 32);
+  } else {
+    if (mt == 16) LFD_G1(16, 64);
+    else if (mt == 32) LFD_G1(32, 64);
+    else LFD_G1(64, 64);
+  }
+#undef LFD_G1
   return cudaGetLastError();
 }
 
@@ -777,39 +785,52 @@ cudaError_t launch_nlcarry(int ndom, int nproj, int norb, double eps, const doub
 // (dom, 64-row block, 64-column tile) work item; K = nproj in chunks of kKC2 through a TMA tensor-map
 // ring (full/empty mbarriers; thread 0 refills a stage once every warp has released it).
 // ------------------------------------------------------------------------------------------------
-template <bool kTail>
-__device__ __forceinline__ void gemm2_chunk(const double2* As, const double2* Cs, int kv, int wm, int wn, int g,
-                                            int t, Frag& acc) {
+// Tile shapes of k_gemm2: kRT rows x kCT orbital columns, 8 warps of 32 x 16 (the same fragments): 64 x 64 (2 x 4
+// warps, 3-stage ring) or, for narrow orbital sets (norb <= 32, C5's first row), 128 x 32 (4 x 2 warps, 2 stages)
+template <int kRT, int kCT>
+struct G2Shape {
+  static constexpr int WN = kCT / 16, WM = 8 / WN;
+  static constexpr int LDC = kCT + 2;                       // == 2 mod 8 complex: conflict-free fragment loads
+  static constexpr int Stages = kRT == 64 ? 3 : 2;
+  static constexpr int StageBytes = kRT * kLdA2 * 16 + kKC2 * LDC * 16;
+  static constexpr int Smem = Stages * StageBytes + 2 * Stages * 8;
+};
+
+template <int kLDC>
+__device__ __forceinline__ void gemm2_chunk(const double2* As, const double2* Cs, int wm, int wn, int g, int t,
+                                            Frag& acc) {
 #pragma unroll
   for (int kk = 0; kk < kKC2; kk += 4) {
     const int k = kk + t;
-    const bool ok = !kTail || (k < kv);
     double2 a[4], c[2];
 #pragma unroll
-    for (int mi = 0; mi < 4; ++mi) a[mi] = ok ? As[(wm * 32 + mi * 8 + g) * kLdA2 + k] : cz();
+    for (int mi = 0; mi < 4; ++mi) a[mi] = As[(wm * 32 + mi * 8 + g) * kLdA2 + k];
 #pragma unroll
-    for (int ni = 0; ni < 2; ++ni) c[ni] = ok ? Cs[k * kLd1 + wn * 16 + ni * 8 + g] : cz();
+    for (int ni = 0; ni < 2; ++ni) c[ni] = Cs[k * kLDC + wn * 16 + ni * 8 + g];
     mma_4x2(acc, a, c);
   }
 }
 
+template <int kRT, int kCT>
 __global__ void __launch_bounds__(kThreads, 1) k_gemm2(const __grid_constant__ CUtensorMap tA,
                                                        const __grid_constant__ CUtensorMap tC, Gemm2Args p) {
   pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
   pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
+  using S = G2Shape<kRT, kCT>;
+  constexpr int kSt = S::Stages;
   extern __shared__ __align__(128) unsigned char smem[];
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages2 * kStage2Bytes);
-  uint64_t* empty = full + kStages2;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kSt * S::StageBytes);
+  uint64_t* empty = full + kSt;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int g = lane >> 2, t = lane & 3;
-  const int wm = warp >> 2, wn = warp & 3;
-  const int rblocks = (int)((p.ng + kTile - 1) / kTile);
-  const int ntn = (p.norb + kTile - 1) / kTile;
+  const int wm = warp / S::WN, wn = warp % S::WN;
+  const int rblocks = (int)((p.ng + kRT - 1) / kRT);
+  const int ntn = (p.norb + kCT - 1) / kCT;
   const long long items = (long long)p.ndom * rblocks * ntn;
   const int nk = (p.nproj + kKC2 - 1) / kKC2;
 
   if (tid == 0) {
-    for (int s = 0; s < kStages2; ++s) {
+    for (int s = 0; s < kSt; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], kConsWarps1);
     }
@@ -826,28 +847,28 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(const __grid_constant__ C
     dom = (int)(item / per_dom);
     const long long rem = item - dom * per_dom;
     const long long rb = rem / ntn;
-    r0 = rb * kTile;
-    n0 = (int)(rem - rb * ntn) * kTile;
+    r0 = rb * kRT;
+    n0 = (int)(rem - rb * ntn) * kCT;
   };
 
-  // chunk gc -> stage gc % kStages2: two tiled tensor copies, the B block [64 rows][kKC2 + 4 complex]
-  // (columns past nproj and rows past ng are zero fill) and the C'' block [kKC2 rows][66 complex]
+  // chunk gc -> stage gc % kSt: two tiled tensor copies, the B block [kRT rows][kKC2 + 4 complex]
+  // (columns past nproj and rows past ng are zero fill) and the C'' block [kKC2 rows][kCT + 2 complex]
   auto issue = [&](long long gc) {  // thread 0 only
-    const int stage = (int)(gc % kStages2);
+    const int stage = (int)(gc % kSt);
     const long long item = blockIdx.x + (gc / nk) * gridDim.x;
     const int kc = (int)(gc % nk);
     int dom, n0;
     long long r0;
     decode(item, dom, r0, n0);
-    double2* As = reinterpret_cast<double2*>(smem + stage * kStage2Bytes);
-    double2* Cs = As + kTile * kLdA2;
-    mbar_expect_tx(&full[stage], (uint32_t)kStage2Bytes);
+    double2* As = reinterpret_cast<double2*>(smem + stage * S::StageBytes);
+    double2* Cs = As + kRT * kLdA2;
+    mbar_expect_tx(&full[stage], (uint32_t)S::StageBytes);
     tma_3d(As, &tA, 2 * kc * kKC2, (int)r0, dom, &full[stage]);
     tma_3d(Cs, &tC, 2 * n0, kc * kKC2, dom, &full[stage]);
   };
 
   if (tid == 0)
-    for (long long s = 0; s < kStages2 && s < total; ++s) issue(s);
+    for (long long s = 0; s < kSt && s < total; ++s) issue(s);
 
   long long gc = 0;
   for (long long it = 0; it < my_items; ++it) {
@@ -858,28 +879,28 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(const __grid_constant__ C
     const double2* psi = p.psi + (long long)dom * p.ng * p.norb;
     double2* pout = (p.psi_out ? p.psi_out : p.psi) + (long long)dom * p.ng * p.norb;
     if (tid == 32) {  // Psi rows of this item (first) and of the next one -> L2, read in the epilogue
-      if (it == 0) l2_prefetch(psi + r0 * p.norb, (uint32_t)(min((long long)kTile, p.ng - r0) * p.norb * 16));
+      if (it == 0) l2_prefetch(psi + r0 * p.norb, (uint32_t)(min((long long)kRT, p.ng - r0) * p.norb * 16));
       if (it + 1 < my_items) {
         int d1, n1;
         long long q1;
         decode(item + gridDim.x, d1, q1, n1);
         l2_prefetch(p.psi + ((long long)d1 * p.ng + q1) * p.norb,
-                    (uint32_t)(min((long long)kTile, p.ng - q1) * p.norb * 16));
+                    (uint32_t)(min((long long)kRT, p.ng - q1) * p.norb * 16));
       }
     }
     Frag acc;
     acc.zero();
     for (int kc = 0; kc < nk; ++kc, ++gc) {
-      const int stage = (int)(gc % kStages2);
-      mbar_wait(&full[stage], (uint32_t)((gc / kStages2) & 1));
-      const double2* As = reinterpret_cast<const double2*>(smem + stage * kStage2Bytes);
-      const double2* Cs = As + kTile * kLdA2;
-      gemm2_chunk<false>(As, Cs, kKC2, wm, wn, g, t, acc);  // the K tail is zero fill
+      const int stage = (int)(gc % kSt);
+      mbar_wait(&full[stage], (uint32_t)((gc / kSt) & 1));
+      const double2* As = reinterpret_cast<const double2*>(smem + stage * S::StageBytes);
+      const double2* Cs = As + kRT * kLdA2;
+      gemm2_chunk<S::LDC>(As, Cs, wm, wn, g, t, acc);  // the K tail is zero fill
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);
-      if (tid == 0 && gc + kStages2 < total) {  // refill once every warp has released the stage
-        mbar_wait(&empty[stage], (uint32_t)((gc / kStages2) & 1));
-        issue(gc + kStages2);
+      if (tid == 0 && gc + kSt < total) {  // refill once every warp has released the stage
+        mbar_wait(&empty[stage], (uint32_t)((gc / kSt) & 1));
+        issue(gc + kSt);
       }
     }
     // epilogue: Psi <- n_s (Psi + B C'); all 16 loads (L2 hits) are issued before any store
@@ -1105,30 +1126,35 @@ cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st) {
       else launch_k(k_gemm2_tma<0, false>, grid, kThreads, kFullSmem + 16, st, tB, tC, a);
     }
   } else {
-    // B [dom][ng][nproj] (box [1][64 rows][kKC2 + 4 complex]) and C'' [dom][nproj][norb] (box [1][kKC2][66])
+    // B [dom][ng][nproj] (box [1][kRT rows][kKC2 + 4 complex]) and C'' [dom][nproj][norb] (box [1][kKC2][kCT + 2])
+    const bool narrow = a.norb <= 32;
+    const int rt = narrow ? 128 : kTile, ct = narrow ? 32 : kTile;
     CUtensorMap tA, tC;
     const uint64_t dA[3] = {(uint64_t)2 * a.nproj, (uint64_t)a.ng, (uint64_t)a.ndom};
     const uint64_t sA[2] = {(uint64_t)a.nproj * 16, (uint64_t)a.ng * a.nproj * 16};
-    const uint32_t bA[3] = {2 * kLdA2, kTile, 1};
+    const uint32_t bA[3] = {2 * kLdA2, (uint32_t)rt, 1};
     cudaError_t e = encode_tmap_f64(&tA, 3, a.B, dA, sA, bA);
     if (e != cudaSuccess) return e;
     const uint64_t dC[3] = {(uint64_t)2 * a.norb, (uint64_t)a.nproj, (uint64_t)a.ndom};
     const uint64_t sC[2] = {(uint64_t)a.norb * 16, (uint64_t)a.nproj * a.norb * 16};
-    const uint32_t bC[3] = {2 * kLd1, kKC2, 1};
+    const uint32_t bC[3] = {(uint32_t)(2 * (ct + 2)), kKC2, 1};
     e = encode_tmap_f64(&tC, 3, a.Cp, dC, sC, bC);
     if (e != cudaSuccess) return e;
-    launch_k(k_gemm2, grid, kThreads, gemm2_smem_bytes(), st, tA, tC, a);
+    const long long items2 = (long long)a.ndom * ((a.ng + rt - 1) / rt) * ((a.norb + ct - 1) / ct);
+    const int grid2 = (int)(items2 < a.num_sms ? items2 : a.num_sms);
+    if (narrow) launch_k(k_gemm2<128, 32>, grid2, kThreads, G2Shape<128, 32>::Smem, st, tA, tC, a);
+    else launch_k(k_gemm2<64, 64>, grid2, kThreads, G2Shape<64, 64>::Smem, st, tA, tC, a);
   }
   return cudaGetLastError();
 }
 
 cudaError_t gemm_set_attributes() {
-  cudaError_t e = cudaFuncSetAttribute(k_gemm1<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm1_smem_bytes());
-  if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_gemm1<32>, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm1_smem_bytes());
-  if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_gemm1<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm1_smem_bytes());
-  if (e != cudaSuccess) return e;
+  cudaError_t e = cudaSuccess;
+  for (auto f : {k_gemm1<64, 64>, k_gemm1<32, 64>, k_gemm1<16, 64>, k_gemm1<64, 32>, k_gemm1<32, 32>,
+                 k_gemm1<16, 32>}) {
+    e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm1_smem_bytes());
+    if (e != cudaSuccess) return e;
+  }
   for (auto f : {k_gemm2_tma<kTile, false>, k_gemm2_tma<0, false>, k_gemm2_tma<kTile, true>, k_gemm2_tma<0, true>}) {
     e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kFullSmem + 16);
     if (e != cudaSuccess) return e;
@@ -1142,7 +1168,9 @@ cudaError_t gemm_set_attributes() {
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(k_nlnorm, cudaFuncAttributeMaxDynamicSharedMemorySize, 16 * 2048);
   if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(k_gemm2, cudaFuncAttributeMaxDynamicSharedMemorySize, gemm2_smem_bytes());
+  e = cudaFuncSetAttribute(k_gemm2<128, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, G2Shape<128, 32>::Smem);
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(k_gemm2<64, 64>, cudaFuncAttributeMaxDynamicSharedMemorySize, G2Shape<64, 64>::Smem);
 }
 
 }  // namespace lfd

@@ -473,3 +473,12 @@ def test_step_prologue_overlap_schedule_bitwise():
         ctx.close()
     for a, b in zip(*outs):
         assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("norb,nproj,dims", [(20, 100, (8, 10, 12)), (32, 65, (10, 12, 14)), (9, 40, (8, 6, 10))])
+def test_narrow_orbital_tiles(norb, nproj, dims):
+    """norb <= 32 (C5's first row): GEMM-1 with 32-wide orbital tiles and, for nproj > 64, the 128 x 32 GEMM-2
+    tile -- ragged in every direction -- against the oracle."""
+    w = workload("P0").with_(nx=dims[0], ny=dims[1], nz=dims[2], norb=norb, nocc=min(norb, 12), nproj=nproj)
+    x = make_inputs(w, seed=15)
+    assert_parity(w, run_gpu(w, x, 4, laser(w)), run_ref(w, x, 4, laser(w)))
