@@ -80,9 +80,11 @@ typedef struct {
 #define LFD_FLAG_EXACT_NL 2
 /* lfd_config.flags: the SP variant (the paper's SP column, and its
  * complex<float> listings): psi, proj (and lfd_remap_occ's ref) are complex64 [.. same layouts ..]
- * (two floats, 8-byte aligned). The stencil sweeps run in FP32 (three line passes), the projector GEMMs in
- * 3xTF32 on the tensor pipe (FP32-accurate products, FP32 accumulation per split), and everything
- * O(nproj x norb) -- the split reduction, the Gram matrix, n_s, the carry, the energies -- in FP64. Results
+ * (two floats, 8-byte aligned). The stencil sweeps run in FP32 (three line passes); the projector GEMMs run on
+ * the tcgen05 int8 tensor cores with 4 balanced digits per operand (products to ~2^-27 of the row / column
+ * scales, below FP32 rounding; the default where nproj, norb <= 64 and >= 65,536 points, or LFD_FLAG_NL_I8),
+ * else as 3xTF32 on the warp-level mma.sync path (LFD_FLAG_NL_DMMA selects the latter); everything
+ * O(nproj x norb) -- the split reduction, the Gram matrix, n_s, the carry, the energies -- runs in FP64. Results
  * agree with the FP64 path to single-precision roundoff (DESIGN.md §4 states the tolerance). */
 #define LFD_FLAG_SP 4
 /* lfd_config.flags: run the nonlocal GEMMs (C = dV B^H Psi; Psi <- Psi diag(n) + B C'') as
@@ -310,6 +312,7 @@ lfd_status lfd_launch_count(const lfd_ctx* ctx, uint64_t* count);
 
 /* Which kernel runs the nonlocal GEMM-2 of this context: *path = 0 complex FP64 DMMA (mma.sync),
  * 1 int8-digit tcgen05 tensor cores, FP64 emulated (see LFD_FLAG_NL_DMMA), 2 SP 3xTF32 (LFD_FLAG_SP),
+ * 3 SP on the int8-digit tcgen05 tensor cores (4 digits),
  * -1 no nonlocal factor (nproj == 0). */
 lfd_status lfd_nl_path(const lfd_ctx* ctx, int32_t* path);
 

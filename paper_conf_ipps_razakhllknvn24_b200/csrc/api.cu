@@ -97,7 +97,7 @@ lfd_status validate(const lfd_config* c, std::string& why) {
 // set-up (C'' digits, TMEM allocation, the exponent handshake) is not amortised (C1: 0.084 vs 0.058 ms/step);
 // LFD_FLAG_NL_I8 forces the int8 path wherever it is supported.
 bool use_i8(const lfd_config* c) {
-  const bool on = (c->flags & (LFD_FLAG_NL_DMMA | LFD_FLAG_SP)) == 0;
+  const bool on = (c->flags & LFD_FLAG_NL_DMMA) == 0;  // (SP contexts: 4-digit int8 GEMMs, else 3xTF32 mma.sync)
   const long long ng = (long long)c->nx * c->ny * c->nz;
   const bool want = ng >= 65536 || (c->flags & LFD_FLAG_NL_I8);
   return on && want && lfd::gemm2_i8_supported(c->nproj, c->norb);
@@ -189,9 +189,10 @@ Layout layout(const Geometry& g, int num_sms, int nref_max, bool dense = false) 
   L.x32 = g.sp ? take((size_t)nd * np * std::max(no, dense ? np : 0) * 8) : 0;  // SP: GEMM-2 coefficient (c64)
   L.aseq = take((size_t)kGraphChunk * nd * 3 * d8);   // lfd_step_graph: A of the chunk's steps
   L.jseq = take((size_t)kGraphChunk * nd * 3 * d8);   // lfd_step_graph: J of the chunk's steps
-  L.bsl = L.i8 ? take(lfd::gemm2_i8_bytes(nd, g.ng)) : 0;
+  const int S = g.sp ? 4 : 6;  // int8 digits per operand
+  L.bsl = L.i8 ? take(lfd::gemm2_i8_bytes(nd, g.ng, S)) : 0;
   L.bsig = L.i8 ? take(lfd::gemm2_i8_sig_bytes(nd, g.ng)) : 0;
-  L.bsl1 = L.i8 ? take(lfd::gemm1_i8_bytes(nd, g.ng)) : 0;
+  L.bsl1 = L.i8 ? take(lfd::gemm1_i8_bytes(nd, g.ng, S)) : 0;
   L.bexp = L.i8 ? take((size_t)nd * np * sizeof(int)) : 0;
   L.colE = L.i8 ? take((size_t)nd * no * sizeof(int)) : 0;
   L.g1cnt = L.i8 ? take((size_t)nd * sizeof(int)) : 0;
@@ -405,8 +406,8 @@ lfd_status launch(lfd_ctx* c, int kid, const char* name, F&& f) {
     cudaEventRecord(s->a, c->stream);
   }
   cudaError_t e;
-  if (c->g.sp) {  // SP contexts launch without PDL (C2 SP step 0.98 ms without, 1.12 ms with: the early-resident
-                  // CTAs of the next kernel slow the SP GEMMs' cp.async rings)
+  if (c->g.sp && !c->L.i8) {  // the 3xTF32 SP contexts launch without PDL (C2 SP step 0.98 ms without, 1.12 ms
+                             // with: the early-resident CTAs of the next kernel slow the SP GEMMs' cp.async rings)
     const bool prev = lfd::pdl_suspended();
     lfd::pdl_suspend(true);
     e = f();
@@ -479,9 +480,10 @@ lfd_status gemm2(lfd_ctx* c, double2* out = nullptr) {
   if (c->L.i8) {
     a2.bsl = c->at<int8_t>(c->L.bsl);
     a2.bsig = c->at<double>(c->L.bsig);
+    a2.sp = g.sp;
   }
   c->c_valid = false;
-  if (g.sp)
+  if (g.sp && !c->L.i8)
     LFD_TRY(launch(c, LFD_K_NL_BACK, "k_gemm2_sp", [&] {
       return lfd::launch_gemm2_sp(c->psi32(), c->proj32(), a2.Cp, c->at<float2>(c->L.x32), a2.nfac, g.ndom, g.nproj,
                                   g.norb, g.ng, c->stream, reinterpret_cast<float2*>(out));
@@ -552,7 +554,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr, bool
     ai.colE = c->at<int>(c->L.colE); ai.counter = c->at<int>(c->L.g1cnt);
     ai.part = a1.part; ai.norms = a1.norms;
     ai.ndom = g.ndom; ai.nproj = g.nproj; ai.norb = g.norb; ai.nsplit = c->L.nsplit_i8;
-    ai.ng = g.ng; ai.rps = c->L.rows_per_split_i8;
+    ai.ng = g.ng; ai.rps = c->L.rows_per_split_i8; ai.sp = g.sp;
     LFD_TRY(launch(c, LFD_K_NL_PROJ, "k_gemm1_i8", [&] { return lfd::launch_gemm1_i8(ai, c->stream); }));
     c->colE_valid = false;
     nsplit = c->L.nsplit_i8;
@@ -599,9 +601,12 @@ lfd_status local_prop(lfd_ctx* c, const double2* src = nullptr, bool skip_x = fa
     LFD_TRY(launch(c, LFD_K_KIN_Y, "k_kin_sp(y)", [&] {
       return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 1, 0, c->scaled, c->stream);
     }));
-    return launch(c, LFD_K_KIN_Z, "k_kin_sp(z)", [&] {
-      return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 2, 2, c->scaled, c->stream);
-    });
+    int* colE = c->L.i8 ? c->at<int>(c->L.colE) : nullptr;  // exponents for the int8-digit GEMM-1
+    LFD_TRY(launch(c, LFD_K_KIN_Z, "k_kin_sp(z)", [&] {
+      return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 2, 2, c->scaled, c->stream, nullptr, colE);
+    }));
+    c->colE_valid = colE != nullptr;
+    return LFD_OK;
   }
   if (!skip_x)
     LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin(x)",
@@ -1051,12 +1056,12 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   }
   if (L.i8) {  // int8 digit tiles of B for the tensor-core GEMM-2 and GEMM-1 (B is constant, like G)
     s2 = launch(c, LFD_K_NL_BACK, "k_bslice_i8", [&] {
-      return lfd::launch_bslice_i8(c->proj, g.ndom, g.nproj, g.ng, c->at<int8_t>(L.bsl), c->at<double>(L.bsig),
+      return lfd::launch_bslice_i8(c->proj, g.sp, g.ndom, g.nproj, g.ng, c->at<int8_t>(L.bsl), c->at<double>(L.bsig),
                                    c->stream);
     });
     if (s2 != LFD_OK) return bail(s2);
     s2 = launch(c, LFD_K_NL_PROJ, "k_bslice1_i8", [&] {
-      return lfd::launch_bslice1_i8(c->proj, g.ndom, g.nproj, g.ng, c->at<int>(L.bexp), c->at<int8_t>(L.bsl1),
+      return lfd::launch_bslice1_i8(c->proj, g.sp, g.ndom, g.nproj, g.ng, c->at<int>(L.bexp), c->at<int8_t>(L.bsl1),
                                     c->stream);
     });
     if (s2 != LFD_OK) return bail(s2);
@@ -1584,7 +1589,7 @@ lfd_status lfd_sync(lfd_ctx* c) {
 lfd_status lfd_nl_path(const lfd_ctx* c, int32_t* path) {
   LFD_TRY(check_ctx(c));
   if (!path) return LFD_EINVAL;
-  *path = c->g.nproj == 0 ? -1 : c->g.sp ? 2 : c->L.i8 ? 1 : 0;
+  *path = c->g.nproj == 0 ? -1 : c->g.sp ? (c->L.i8 ? 3 : 2) : c->L.i8 ? 1 : 0;
   return LFD_OK;
 }
 

@@ -24,6 +24,7 @@
 // operator; used when every c >= 1/2 (else the general 2x2 form runs). The FP64 pipe (not tensor) is
 // what bounds these sweeps next to HBM on B200 (DFMA 34 TF/s), so halving the FP64 work matters.
 #include <cmath>
+#include <type_traits>
 
 #include "lfd_coef.cuh"
 #include "lfd_complex.cuh"
@@ -129,14 +130,67 @@ cudaError_t launch_phase_sp(const Geometry& g, const double* v, float2* phi, dou
 // src: the input (== psi for the usual in-place pass; another buffer for the out-of-place first pass of the
 // self-consistent sweeps). In place is safe: each line belongs to one lane, whose reads of a point precede
 // its write of that point.
+// FP64 biased exponent bound of a complex64 value's components (0 for zero): |re|, |im| < 2^(E - 1022)
+__device__ __forceinline__ int exp64_of(float2 v) {
+  const uint32_t m = max(__float_as_uint(v.x) & 0x7fffffffu, __float_as_uint(v.y) & 0x7fffffffu);
+  const int e8 = (int)(m >> 23);
+  return m == 0 ? 0 : (e8 == 0 ? 897 : e8 + 896);
+}
+
+// colE (SP z pass with the int8-digit GEMMs only): the largest exponent of each orbital over the domain, for
+// the next GEMM-1's digit scales (as k_kin_yz records it for FP64; a shared-memory max per CTA, then one global
+// atomicMax per orbital).
 template <bool kPeriodic, int kPhase, bool kS, class C = double2, class V = C>
 __global__ void __launch_bounds__(256, 3) k_kin(V* psi, const V* src, const DomCoef* __restrict__ coef,
                                              const C* __restrict__ phi, int axis, int n, int pt_stride,
                                              int inner_len, int outer_stride, int ncols, int norb,
-                                             long long dom_stride, long long ng) {
+                                             long long dom_stride, long long ng, int* __restrict__ colE) {
   pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
   pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if constexpr (std::is_same<C, float2>::value) {
+    if (colE) {
+      __shared__ int smax[128];
+      for (int i = threadIdx.x; i < 128; i += blockDim.x) smax[i] = 0;
+      __syncthreads();
+      int ea = 0, eb = 0;
+      if (c < ncols) {
+        const int dom = blockIdx.y;
+        const int outer = c / inner_len;
+        const int inner = c - outer * inner_len;
+        const int off = outer * outer_stride + inner;
+        V* line = psi + dom * dom_stride + off;
+        const V* sline = src + dom * dom_stride + off;
+        const C* ph = phi + dom * ng + off / norb;
+        const int ph_stride = pt_stride / norb;
+        const PairCoefT<C> cf = pair_coef_t<kS, C>(coef + dom, axis);
+        auto ld = [&](int i) -> V {
+          V v = sline[(long long)i * pt_stride];
+          if (kPhase == 1) v = cmul(ph[(long long)i * ph_stride], v);
+          return v;
+        };
+        auto st = [&](int i, V v) {
+          if (kPhase == 2) v = cmul(ph[(long long)i * ph_stride], v);
+          line[(long long)i * pt_stride] = v;
+          if constexpr (std::is_same<V, cf2>::value) {
+            ea = max(ea, exp64_of(v.a));
+            eb = max(eb, exp64_of(v.b));
+          } else {
+            ea = max(ea, exp64_of(v));
+          }
+        };
+        march_line<kPeriodic, kS, C, V>(n, cf, ld, st);
+        const int orb = std::is_same<V, cf2>::value ? 2 * inner : inner;  // (the z pass: inner = orbital unit)
+        atomicMax(smax + orb, ea);
+        if (std::is_same<V, cf2>::value) atomicMax(smax + orb + 1, eb);
+      }
+      __syncthreads();
+      const int no = std::is_same<V, cf2>::value ? 2 * norb : norb;  // (norb is in units of V)
+      for (int i = threadIdx.x; i < no; i += blockDim.x)
+        if (smax[i] > 0) atomicMax(colE + (long long)blockIdx.y * no + i, smax[i]);
+      return;
+    }
+  }
   if (c >= ncols) return;
   const int dom = blockIdx.y;
   const int outer = c / inner_len;
@@ -448,7 +502,7 @@ cudaError_t launch_kin_yz(const Geometry& g, const CUtensorMap* tmap, double2* p
 
 template <class C, class V>
 static cudaError_t launch_kin_t(const Geometry& g, V* psi, const DomCoef* coef, const C* phi, int axis,
-                                int phase_mode, bool scaled, cudaStream_t st, const V* src) {
+                                int phase_mode, bool scaled, cudaStream_t st, const V* src, int* colE = nullptr) {
   if (!src) src = psi;
   const int nd[3] = {g.nx, g.ny, g.nz};
   const int norb = g.norb / (int)(sizeof(V) / sizeof(C));  // values of type V per grid point
@@ -472,7 +526,7 @@ static cudaError_t launch_kin_t(const Geometry& g, V* psi, const DomCoef* coef, 
   const long long dom_stride = g.ng * norb;
 #define LFD_KIN(P, M, K)                                                                                       \
   launch_k(k_kin<P, M, K, C, V>, grid, 256, 0, st, psi, src, coef, phi, axis, n, pt_stride, inner_len, outer_stride, ncols, \
-                                          norb, dom_stride, g.ng)
+                                          norb, dom_stride, g.ng, colE)
 #define LFD_KIN_M(P, K) \
   if (phase_mode == 1) LFD_KIN(P, 1, K); else if (phase_mode == 2) LFD_KIN(P, 2, K); else LFD_KIN(P, 0, K)
   if (g.bc == 0) {
@@ -491,12 +545,12 @@ cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, con
 }
 
 cudaError_t launch_kin_sp(const Geometry& g, float2* psi, const DomCoef* coef, const float2* phi, int axis,
-                          int phase_mode, bool scaled, cudaStream_t st, const float2* src) {
+                          int phase_mode, bool scaled, cudaStream_t st, const float2* src, int* colE) {
   if (!src) src = psi;
   if (g.norb % 2 == 0 && ((reinterpret_cast<uintptr_t>(psi) | reinterpret_cast<uintptr_t>(src)) & 15) == 0)
     return launch_kin_t<float2, cf2>(g, reinterpret_cast<cf2*>(psi), coef, phi, axis, phase_mode, scaled, st,
-                                     reinterpret_cast<const cf2*>(src));  // two orbitals (16 bytes) per lane
-  return launch_kin_t<float2, float2>(g, psi, coef, phi, axis, phase_mode, scaled, st, src);
+                                     reinterpret_cast<const cf2*>(src), colE);  // two orbitals (16 bytes) per lane
+  return launch_kin_t<float2, float2>(g, psi, coef, phi, axis, phase_mode, scaled, st, src, colE);
 }
 
 }  // namespace lfd

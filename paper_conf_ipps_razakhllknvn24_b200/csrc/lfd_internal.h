@@ -94,8 +94,11 @@ bool kin_scaled_ok(const Geometry& g);
 cudaError_t launch_kin(const Geometry& g, double2* psi, const DomCoef* coef, const double2* phi,
                        int axis, int phase_mode, bool scaled, cudaStream_t st, const double2* src = nullptr);
 // SP variant (complex64 Psi and Phi, FP32 sweeps)
+// colE != nullptr (the z pass on the int8-digit path): also records each orbital's largest exponent (k_kin_yz's
+// role for FP64) for the next GEMM-1
 cudaError_t launch_kin_sp(const Geometry& g, float2* psi, const DomCoef* coef, const float2* phi,
-                          int axis, int phase_mode, bool scaled, cudaStream_t st, const float2* src = nullptr);
+                          int axis, int phase_mode, bool scaled, cudaStream_t st, const float2* src = nullptr,
+                          int* colE = nullptr);
 
 // Fused pass Psi <- Phi . K_y K_z Psi (one read + write of Psi; nz <= 80).
 bool kin_yz_supported(const Geometry& g);
@@ -170,13 +173,14 @@ struct Gemm2Args {
   // int8-digit tensor-core path (nl_i8.cu): B's digit tiles and row scales from launch_bslice_i8, or nullptr
   const int8_t* bsl = nullptr;
   const double* bsig = nullptr;
+  int sp = 0;  // the SP variant: Psi, B complex64, 4 digits per operand
 };
 cudaError_t launch_gemm2(const Gemm2Args& a, cudaStream_t st);
 // GEMM-2 with FP64 accuracy on the tcgen05 int8 tensor cores (nl_i8.cu): nproj <= 64, norb <= 64.
 bool gemm2_i8_supported(int nproj, int norb);
-size_t gemm2_i8_bytes(int ndom, long long ng);      // B digit tiles
+size_t gemm2_i8_bytes(int ndom, long long ng, int S);  // B digit tiles (S digits: 6 FP64, 4 SP)
 size_t gemm2_i8_sig_bytes(int ndom, long long ng);  // B row scales
-cudaError_t launch_bslice_i8(const double2* B, int ndom, int nproj, long long ng, int8_t* out, double* sig,
+cudaError_t launch_bslice_i8(const void* B, bool sp, int ndom, int nproj, long long ng, int8_t* out, double* sig,
                              cudaStream_t st);
 cudaError_t launch_gemm2_i8(const Gemm2Args& a, cudaStream_t st);
 cudaError_t gemm_i8_set_attributes();
@@ -192,6 +196,7 @@ struct Gemm1I8Args {
   double* norms;        // [dom][nsplit][norb]
   int ndom, nproj, norb, nsplit;
   long long ng, rps;
+  int sp = 0;  // the SP variant (complex64 Psi, 4 digits; colE from the SP z pass)
 };
 // The first nonlocal factor's GEMM-2 fused with the x pass of the local propagator (nl_fx.cu):
 //   Psi[x][yz] <- K_x (Phi . (n Psi + B C''))  along every x-line (y, z), int8-digit tcgen05 products.
@@ -207,9 +212,9 @@ cudaError_t launch_gemm2x_i8(const Geometry& g, const FxMaps* m, double2* psi, c
                              const double2* Cp, const double* sig, bool scaled, int num_sms, cudaStream_t st);
 cudaError_t gemm2x_set_attributes();
 
-size_t gemm1_i8_bytes(int ndom, long long ng);
+size_t gemm1_i8_bytes(int ndom, long long ng, int S);
 long long gemm1_i8_rows_per_split(long long ng, int ndom, int num_sms);
-cudaError_t launch_bslice1_i8(const double2* B, int ndom, int nproj, long long ng, int* bexp, int8_t* out,
+cudaError_t launch_bslice1_i8(const void* B, bool sp, int ndom, int nproj, long long ng, int* bexp, int8_t* out,
                               cudaStream_t st);
 cudaError_t launch_gemm1_i8(const Gemm1I8Args& a, cudaStream_t st);
 cudaError_t gemm_set_attributes();

@@ -17,8 +17,9 @@ __host__ __device__ __forceinline__ int sw128(int row, int k) {
   return ((row >> 3) << 10) + ((row & 7) << 7) + ((((k >> 4) ^ (row & 7))) << 4) + (k & 15);
 }
 
-// the digits of 4 consecutive values of one row; the scale exponent e is shared by the row (x = v 2^-e)
-__device__ __forceinline__ void digits4(const double v[4], int e, bool zero, uint32_t out[kI8S]) {
+// the S digits of 4 consecutive values of one row; the scale exponent e is shared by the row (x = v 2^-e)
+template <int S = kI8S>
+__device__ __forceinline__ void digits4(const double v[4], int e, bool zero, uint32_t out[S]) {
   double x[4];
 #pragma unroll
   for (int q = 0; q < 4; ++q) x[q] = zero ? 0.0 : ldexp(v[q], 6 - e);  // 64 x, exact
@@ -26,7 +27,7 @@ __device__ __forceinline__ void digits4(const double v[4], int e, bool zero, uin
   // (ties to even, as rint) and holds it in the low word; no FRND / F2I (low-rate conversion pipe)
   constexpr double kM = 6755399441055744.0;
 #pragma unroll
-  for (int i = 0; i < kI8S; ++i) {
+  for (int i = 0; i < S; ++i) {
     uint32_t w = 0;
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
@@ -74,6 +75,35 @@ __device__ __forceinline__ void digits_i64(const double v[4], double sc, uint32_
   out[3] = __byte_perm(b, d, 0x5410);  // field 2
   out[4] = __byte_perm(a, c, 0x7632);  // field 1
   out[5] = __byte_perm(a, c, 0x5410);  // field 0
+}
+
+// The same with 4 digits (the SP variant: complex64 operands, products accurate to ~2^-27 of the scales, below
+// FP32 rounding): X = rint(v sc), |X| < 2^27, X + C4 (C4 = 64 (128^4 - 1) / 127) fits one 32-bit word with the
+// fields u_0 .. u_3 (u_3 <= 128), d = u - 64; digit i <-> field 4 - i.
+__device__ __forceinline__ void digits_s4(const double v[4], double sc, uint32_t out[4]) {
+  constexpr double kM = 6755399441055744.0;
+  constexpr long long kMb = 0x4338000000000000LL;
+  constexpr int kC4 = 64 * ((1 << 28) - 1) / 127;
+  uint32_t w[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const uint32_t lo = (uint32_t)((__double_as_longlong(fma(v[q], sc, kM)) - kMb) + kC4);
+    uint32_t s3 = (lo & 0x7fu) | ((lo << 1) & 0x7f00u) | ((lo << 2) & 0x7f0000u);
+    s3 = (s3 ^ 0x404040u) | ((~s3 & 0x404040u) << 1);  // bytewise u - 64 (fields 0..2, u in [0, 127])
+    w[q] = s3 | ((((lo >> 21) + 192u) & 0xffu) << 24);  // top field, may be 128
+  }
+  const uint32_t a = __byte_perm(w[0], w[1], 0x5140), b = __byte_perm(w[0], w[1], 0x7362);
+  const uint32_t c = __byte_perm(w[2], w[3], 0x5140), d = __byte_perm(w[2], w[3], 0x7362);
+  out[0] = __byte_perm(b, d, 0x7632);  // digit 1 = field 3
+  out[1] = __byte_perm(b, d, 0x5410);  // field 2
+  out[2] = __byte_perm(a, c, 0x7632);  // field 1
+  out[3] = __byte_perm(a, c, 0x5410);  // field 0
+}
+// S-digit dispatch (S = 6: FP64 contexts, 4: SP); sc = 2^(7 S - 1 - e) for |v| < 2^e
+template <int S>
+__device__ __forceinline__ void digits_x(const double v[4], double sc, uint32_t out[S]) {
+  if constexpr (S == 6) digits_i64(v, sc, out);
+  else digits_s4(v, sc, out);
 }
 
 // exact int32 -> FP64 without the (low-rate) I2F.F64 conversion: 2^52 + (x + 2^31) built from bits, minus

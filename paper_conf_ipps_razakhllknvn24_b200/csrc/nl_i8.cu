@@ -45,23 +45,30 @@ namespace lfd {
 constexpr int kI8NT = 64;                           // grid points per tile (MMA N)
 constexpr int kI8K = 128;                           // bytes per digit row: K = 2 nproj padded to 128
 constexpr int kI8Stages = 2;                        // digit-tile ring
-constexpr int kI8Slots = 5;                         // TMEM ring of diagonal accumulators (kI8NT columns each)
 constexpr int kI8EpiWarps = 16;                     // epilogue warps: 4 lane quarters x 4 row quarters
 constexpr int kI8Rows = kI8NT / 4;                  // tile rows per epilogue warp
 constexpr int kI8SliceB = kI8NT * kI8K;             // 8 KB: one digit slice of a tile
-constexpr int kI8TileB = kI8S * kI8SliceB;          // 48 KB: all digits of a tile
 constexpr int kI8SubR = 16;                         // Psi rows per staged sub-tile (= rows per epilogue warp)
-constexpr int kI8SubRowsB = kI8SubR * 64 * 16;      // 16 KB (norb <= 64)
-constexpr int kI8SubB = kI8SubRowsB + kI8SubR * 8;  // + the sub-tile's row scales sigma_r
 constexpr int kI8PsiSlots = 7;                      // Psi sub-tile ring (the first 64 KB also stage C'')
-constexpr int kI8Smem = kI8Stages * kI8TileB + kI8PsiSlots * kI8SubB + 1024;  // + alignment slack
-constexpr int kI8WCols = kI8S * (kI8K / 4);        // 192 TMEM columns: W^T digits (4 int8 per column)
-constexpr int kI8Acc = kI8S;                        // diagonals d = 2 .. S+1
+// Shapes depending on the digit count S (6: FP64 contexts, 4: the SP variant) and the element type T of Psi
+// (double2 / float2): digit tile, TMEM columns of W^T (4 int8 per column), diagonal accumulators d = 2 .. S+1 and
+// the TMEM ring of them, the staged Psi sub-tile
+template <int S, class T>
+struct I8G2 {
+  static constexpr int TileB = S * kI8SliceB;             // 48 KB (S = 6)
+  static constexpr int WCols = S * (kI8K / 4);            // 192 (S = 6)
+  static constexpr int Acc = S;
+  static constexpr int Slots = (512 - WCols) / kI8NT;     // 5 (S = 6), 6 (S = 4)
+  static constexpr int SubRowsB = kI8SubR * 64 * (int)sizeof(T);  // norb <= 64
+  static constexpr int SubB = SubRowsB + kI8SubR * 8;     // + the sub-tile's row scales sigma_r
+  static constexpr int Smem = kI8Stages * TileB + kI8PsiSlots * SubB + 1024;  // + alignment slack
+};
 constexpr int kI8Threads = (kI8EpiWarps + 3) * 32;  // epilogue warps + 2 producers + MMA
 constexpr int kWDig = kI8EpiWarps, kWMma = kI8EpiWarps + 1, kWPsi = kI8EpiWarps + 2;  // role warps
 
 // ---- B digits (once per lfd_init): warp per grid row -------------------------------------------------
-__global__ void __launch_bounds__(256) k_bslice_i8(const double2* __restrict__ B, int nproj, long long ng,
+template <class T, int S>
+__global__ void __launch_bounds__(256) k_bslice_i8(const T* __restrict__ B, int nproj, long long ng,
                                                    long long tiles, int8_t* __restrict__ out,
                                                    double* __restrict__ sig) {
   pdl_wait();
@@ -72,28 +79,32 @@ __global__ void __launch_bounds__(256) k_bslice_i8(const double2* __restrict__ B
   double v[4] = {0.0, 0.0, 0.0, 0.0};
   const int u0 = 2 * lane;
   if (r < ng) {
-    const double2* row = B + ((long long)dom * ng + r) * nproj;
-    if (u0 < nproj) { const double2 a = row[u0]; v[0] = a.x; v[1] = a.y; }
-    if (u0 + 1 < nproj) { const double2 a = row[u0 + 1]; v[2] = a.x; v[3] = a.y; }
+    const T* row = B + ((long long)dom * ng + r) * nproj;
+    if (u0 < nproj) { const T a = row[u0]; v[0] = a.x; v[1] = a.y; }
+    if (u0 + 1 < nproj) { const T a = row[u0 + 1]; v[2] = a.x; v[3] = a.y; }
   }
   double mx = fmax(fmax(fabs(v[0]), fabs(v[1])), fmax(fabs(v[2]), fabs(v[3])));
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
   const int e = mx > 0.0 ? row_exponent(mx) : 0;
-  uint32_t d[kI8S];
-  digits4(v, e, !(mx > 0.0), d);
+  uint32_t d[S];
+  digits4<S>(v, e, !(mx > 0.0), d);
   const long long t = r / kI8NT;
   const int rr = (int)(r - t * kI8NT);
-  int8_t* tb = out + ((long long)dom * tiles + t) * kI8TileB;
+  int8_t* tb = out + ((long long)dom * tiles + t) * (S * kI8SliceB);
 #pragma unroll
-  for (int i = 0; i < kI8S; ++i) *reinterpret_cast<uint32_t*>(tb + i * kI8SliceB + sw128(rr, 4 * lane)) = d[i];
+  for (int i = 0; i < S; ++i) *reinterpret_cast<uint32_t*>(tb + i * kI8SliceB + sw128(rr, 4 * lane)) = d[i];
   if (lane == 0) sig[(long long)dom * tiles * kI8NT + r] = mx > 0.0 ? ldexp(1.0, e) : 0.0;
 }
 
 // ---- GEMM-2 -----------------------------------------------------------------------------------------
 // grid (CTAs per domain, ndom); CTA b of a domain takes tiles b, b + gridDim.x, ...
-template <bool kOut>
+template <bool kOut, class T, int S>
 __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
+  using G = I8G2<S, T>;
+  using R = decltype(T::x);  // real component type of Psi (double / float)
+  constexpr int kI8TileB = G::TileB, kI8WCols = G::WCols, kI8Acc = G::Acc, kI8Slots = G::Slots;
+  constexpr int kI8SubRowsB = G::SubRowsB, kI8SubB = G::SubB;
   // programmatic dependent launch: the set-up below (TMEM, barriers) and the digit producer (B's digits are
   // constant since lfd_init) overlap the previous kernel; every other warp waits for it (C'', n, Psi)
   pdl_trigger();
@@ -155,7 +166,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
     const int e = mx > 0.0 ? row_exponent(mx) : 0;
     if (c8 == 0) taus[n] = mx > 0.0 ? ldexp(1.0, e - 12) : 0.0;  // x 2^-12: the weight of diagonal 2
     const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
-    uint32_t dg[kI8S][8];
+    uint32_t dg[S][8];
 #pragma unroll
     for (int w = 0; w < 8; ++w) {
       double v[4] = {0.0, 0.0, 0.0, 0.0};
@@ -168,13 +179,13 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
         const double2 x = X[(u0 + 1) * norb];
         v[2] = cn ? x.y : x.x; v[3] = cn ? x.x : -x.y;
       }
-      uint32_t d[kI8S];
-      digits_i64(v, mx > 0.0 ? ldexp(1.0, 41 - e) : 0.0, d);
+      uint32_t d[S];
+      digits_x<S>(v, mx > 0.0 ? ldexp(1.0, 7 * S - 1 - e) : 0.0, d);
 #pragma unroll
-      for (int i = 0; i < kI8S; ++i) dg[i][w] = d[i];
+      for (int i = 0; i < S; ++i) dg[i][w] = d[i];
     }
 #pragma unroll
-    for (int i = 0; i < kI8S; ++i) tmem_st8(trow + i * 32 + 8 * c8, dg[i]);
+    for (int i = 0; i < S; ++i) tmem_st8(trow + i * 32 + 8 * c8, dg[i]);
     asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
   }
   // W ready (TMEM digits, taus[]) and the staged C'' consumed: named barrier 1 over every warp except the
@@ -185,7 +196,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
     tc_fence_after();
   }
 
-  const int rowb = norb * 16;  // bytes per Psi row
+  const int rowb = norb * (int)sizeof(T);  // bytes per Psi row
   if (warp == kWDig) {  // producer of the digit tiles (one bulk copy each)
     if (lane == 0) {
       const int8_t* src = p.bsl + (long long)dom * tiles * kI8TileB;
@@ -199,7 +210,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
     }
   } else if (warp == kWPsi) {  // producer of the Psi sub-tiles (16 contiguous rows + their 16 row scales)
     if (lane == 0) {
-      const double2* prow = p.psi + (long long)dom * ng * norb;
+      const T* prow = reinterpret_cast<const T*>(p.psi) + (long long)dom * ng * norb;
       const double* sig = p.bsig + (long long)dom * tiles * kI8NT;
       int u = 0;
       for (long long t = blockIdx.x; t < tiles; t += gridDim.x)
@@ -227,7 +238,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
         tc_fence_after();
         const uint64_t db0 = umma_desc_sw128(tbase + s * kI8TileB);
 #pragma unroll
-        for (int d = 2; d <= kI8S + 1; ++d) {
+        for (int d = 2; d <= S + 1; ++d) {
           const int g = it * kI8Acc + (d - 2), sl = g % kI8Slots;
           if (g >= kI8Slots) {
             mbar_wait(&dempty[sl], (uint32_t)(((g / kI8Slots) - 1) & 1));
@@ -236,9 +247,9 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
           const uint32_t acc = tacc + sl * kI8NT;
           uint32_t first = 1;
 #pragma unroll
-          for (int i = 1; i <= kI8S; ++i) {
+          for (int i = 1; i <= S; ++i) {
             const int j = d - i;
-            if (j < 1 || j > kI8S) continue;
+            if (j < 1 || j > S) continue;
 #pragma unroll
             for (int kk = 0; kk < kI8K / 32; ++kk) {
               // descriptor arithmetic is linear in the (>> 4) start address: one add per MMA (the issuing
@@ -262,7 +273,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
     const bool nvalid = n < 2 * norb;
     const double nf = nvalid ? p.nfac[(long long)dom * norb + (n >> 1)] : 0.0;
     const double tau = taus[n];
-    double* pout = reinterpret_cast<double*>((kOut ? p.psi_out : p.psi) + (long long)dom * ng * norb) + n;
+    R* pout = reinterpret_cast<R*>(reinterpret_cast<T*>(kOut ? p.psi_out : p.psi) + (long long)dom * ng * norb) + n;
     const int ld = 2 * norb;
     int it = 0;
     for (long long t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
@@ -301,13 +312,13 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
       {
         const int u = it * (kI8NT / kI8SubR) + h, s = u % kI8PsiSlots;
         mbar_wait(&pfull[s], (uint32_t)((u / kI8PsiSlots) & 1));
-        const double* ps = reinterpret_cast<const double*>(Psm + s * kI8SubB) + n;
+        const R* ps = reinterpret_cast<const R*>(Psm + s * kI8SubB) + n;
         const double* sg = reinterpret_cast<const double*>(Psm + s * kI8SubB + kI8SubRowsB);
         if (nvalid) {  // running row pointers (16 precomputed row offsets would spill)
-          double* po = pout + r0 * ld;
+          R* po = pout + r0 * ld;
 #pragma unroll
           for (int c = 0; c < kI8Rows; ++c) {
-            if (c < nc) *po = fma(nf, *ps, scale_pow2(fa[c], sg[c], tau));
+            if (c < nc) *po = (R)fma(nf, (double)*ps, scale_pow2(fa[c], sg[c], tau));
             po += ld;
             ps += ld;
           }
@@ -345,16 +356,20 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
 constexpr int kG1Rows = 64;                        // grid rows per B-digit block (K = 128 bytes)
 constexpr int kG1Half = 16;                        // grid rows per A (Psi-digit) quarter block (K = 32 bytes)
 constexpr int kG1SliceB = 64 * 128;                // 8 KB: one digit slice of a B block (64 u rows)
-constexpr int kG1BlkB = kI8S * kG1SliceB;          // 48 KB
 constexpr int kG1Stages = 2;                       // B-digit ring
-constexpr int kG1PsiB = kG1Half * 64 * 16;         // 16 KB: Psi rows of a quarter block (norb <= 64)
 constexpr int kG1PsiSlots = 6;                     // Psi quarter-block ring
-constexpr int kG1Smem = kG1Stages * kG1BlkB + kG1PsiSlots * kG1PsiB + 1024;
 constexpr int kG1Workers = 16;                     // worker warps: 4 lane quarters x 4 row groups
 constexpr int kG1Threads = (kG1Workers + 2) * 32;  // + producer + MMA
 constexpr int kG1WProd = kG1Workers, kG1WMma = kG1Workers + 1;
-constexpr int kG1ABuf = kI8S * 8;                  // TMEM columns of one A buffer (K = 32 bytes per digit)
-constexpr int kG1ACols = 2 * kG1ABuf;              // double-buffered A
+// shapes depending on the digit count S and Psi's element type T (see I8G2)
+template <int S, class T>
+struct I8G1 {
+  static constexpr int BlkB = S * kG1SliceB;                     // 48 KB (S = 6)
+  static constexpr int PsiB = kG1Half * 64 * (int)sizeof(T);     // Psi rows of a quarter block (norb <= 64)
+  static constexpr int Smem = kG1Stages * BlkB + kG1PsiSlots * PsiB + 1024;
+  static constexpr int ABuf = S * 8;                             // TMEM columns of one A buffer (K = 32 bytes)
+  static constexpr int ACols = 2 * ABuf;                         // double-buffered A
+};
 // s32 <- s8 x s8, both K-major, M = 128, N = n (a multiple of 64 here)
 __host__ __device__ constexpr uint32_t g1_idesc(int n) {
   return (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
@@ -379,13 +394,13 @@ __device__ __forceinline__ void tmem_st4(uint32_t taddr, const uint32_t v[4]) {
 
 // The wide-N MMA schedule of one quarter block (see k_gemm1_i8): for each Psi digit j, the B digits
 // i = 1 .. 7 - j in chunks of at most W consecutive slices, one MMA of N = 64 w per chunk
-template <int W>
+template <int W, int S>
 __device__ __forceinline__ void g1_wide_mmas(uint32_t tacc, uint32_t ta, uint64_t db0, int kq, bool first) {
 #pragma unroll
-  for (int j = 1; j <= kI8S; ++j) {
+  for (int j = 1; j <= S; ++j) {
 #pragma unroll
-    for (int i = 1; i <= kI8S + 1 - j; i += W) {
-      const int w = (kI8S + 2 - j - i) < W ? (kI8S + 2 - j - i) : W;
+    for (int i = 1; i <= S + 1 - j; i += W) {
+      const int w = (S + 2 - j - i) < W ? (S + 2 - j - i) : W;
       umma_g1_ts(tacc + (i + j - 2) * 64, ta + (j - 1) * 8, db0 + (uint64_t)(((i - 1) * kG1SliceB + kq * 32) >> 4),
                  (first && j == 1) ? 0u : 1u, g1_idesc(64 * w));
     }
@@ -393,7 +408,8 @@ __device__ __forceinline__ void g1_wide_mmas(uint32_t tacc, uint32_t ta, uint64_
 }
 
 // B's GEMM-1 scales: bexp[dom][u] = max over the domain of the biased exponent of Re / Im B[r][u]
-__global__ void __launch_bounds__(256) k_bexp1_i8(const double2* __restrict__ B, int nproj, long long ng,
+template <class T>
+__global__ void __launch_bounds__(256) k_bexp1_i8(const T* __restrict__ B, int nproj, long long ng,
                                                   int* __restrict__ bexp) {
   pdl_wait();
   pdl_trigger();
@@ -402,10 +418,11 @@ __global__ void __launch_bounds__(256) k_bexp1_i8(const double2* __restrict__ B,
   for (int u = threadIdx.x; u < 64; u += blockDim.x) sm[u] = 0;
   __syncthreads();
   const long long n = ng * nproj;
-  const double2* b = B + (long long)dom * n;
+  const T* b = B + (long long)dom * n;
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
-    const double2 v = b[i];
-    const int e = max(__double2hiint(v.x) & 0x7ff00000, __double2hiint(v.y) & 0x7ff00000) >> 20;
+    const T v = b[i];
+    const double vx = v.x, vy = v.y;  // (complex64 values widened exactly)
+    const int e = max(__double2hiint(vx) & 0x7ff00000, __double2hiint(vy) & 0x7ff00000) >> 20;
     if (e > 0) atomicMax(sm + (int)(i % nproj), e);  // shared-memory atomics, then one global per column
   }
   __syncthreads();
@@ -414,7 +431,8 @@ __global__ void __launch_bounds__(256) k_bexp1_i8(const double2* __restrict__ B,
 }
 
 // B's GEMM-1 digits: warp per (64-row block, u); lane l holds rows 2l, 2l+1 (k = 4l .. 4l+3)
-__global__ void __launch_bounds__(256) k_bslice1_i8(const double2* __restrict__ B, int nproj, long long ng,
+template <class T, int S>
+__global__ void __launch_bounds__(256) k_bslice1_i8(const T* __restrict__ B, int nproj, long long ng,
                                                     long long nblk, const int* __restrict__ bexp,
                                                     int8_t* __restrict__ out) {
   pdl_wait();
@@ -428,19 +446,23 @@ __global__ void __launch_bounds__(256) k_bslice1_i8(const double2* __restrict__ 
   const int E = u < nproj ? bexp[(long long)dom * nproj + u] : 0;
   if (u < nproj) {
     const long long r = blk * kG1Rows + 2 * lane;
-    const double2* col = B + (long long)dom * ng * nproj + u;
-    if (r < ng) { const double2 a = col[r * nproj]; v[0] = a.x; v[1] = a.y; }
-    if (r + 1 < ng) { const double2 a = col[(r + 1) * nproj]; v[2] = a.x; v[3] = a.y; }
+    const T* col = B + (long long)dom * ng * nproj + u;
+    if (r < ng) { const T a = col[r * nproj]; v[0] = a.x; v[1] = a.y; }
+    if (r + 1 < ng) { const T a = col[(r + 1) * nproj]; v[2] = a.x; v[3] = a.y; }
   }
-  uint32_t d[kI8S];
-  digits4(v, E - 1022, E == 0, d);  // |v| < 2^(E - 1022)
-  int8_t* tb = out + ((long long)dom * nblk + blk) * kG1BlkB;
+  uint32_t d[S];
+  digits4<S>(v, E - 1022, E == 0, d);  // |v| < 2^(E - 1022)
+  int8_t* tb = out + ((long long)dom * nblk + blk) * (S * kG1SliceB);
 #pragma unroll
-  for (int i = 0; i < kI8S; ++i) *reinterpret_cast<uint32_t*>(tb + i * kG1SliceB + sw128(u, 4 * lane)) = d[i];
+  for (int i = 0; i < S; ++i) *reinterpret_cast<uint32_t*>(tb + i * kG1SliceB + sw128(u, 4 * lane)) = d[i];
 }
 
 // grid (splits, ndom); CTA = one split of rps rows (a multiple of 64)
+template <class T, int S>
 __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
+  using G = I8G1<S, T>;
+  using R = decltype(T::x);
+  constexpr int kG1BlkB = G::BlkB, kG1PsiB = G::PsiB, kG1ABuf = G::ABuf, kG1ACols = G::ACols;
   // programmatic dependent launch: set-up and the first B-digit blocks (constant since lfd_init) overlap the
   // previous kernel; the Psi loads and everything reading colE / writing the partials wait for it
   pdl_trigger();
@@ -462,9 +484,9 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   const long long r0 = (long long)split * p.rps;
   const long long r1 = min(ng, r0 + p.rps);
   const int nhalf = (int)((r1 - r0 + kG1Half - 1) / kG1Half);  // quarter blocks of this split
-  const int rowb = norb * 16;
+  const int rowb = norb * (int)sizeof(T);
 
-  if (warp == kG1WMma) {  // TMEM: A (Psi digits, 96 columns) + 6 diagonal accumulators x 64 columns
+  if (warp == kG1WMma) {  // TMEM: A (Psi digits, 2 x 8 S columns) + S diagonal accumulators x 64 columns
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_addr(&tmem_base_sh)));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
@@ -484,7 +506,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   if (warp == kG1WProd) {  // producer: B-digit blocks and Psi half blocks, in the order the MMAs use them
     if (lane == 0) {
       const int8_t* src = p.bsl1 + (long long)dom * nblk * kG1BlkB;
-      const double2* prow = p.psi + (long long)dom * ng * norb;
+      const T* prow = reinterpret_cast<const T*>(p.psi) + (long long)dom * ng * norb;
       const int nb = (nhalf + 3) >> 2;  // B-digit blocks of this split
       for (int b = 0; b < kG1Stages && b < nb; ++b) {  // before the dependency wait: B is constant
         mbar_expect_tx(&bfull[b], kG1BlkB);
@@ -520,7 +542,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
         // 64-column TMEM blocks: one MMA of N = 64 w (w <= 3) computes the w digit pairs (i .. i + w - 1, j)
         // straight into their diagonals (9 MMAs per quarter block instead of 21). The j = 1 MMAs touch every
         // diagonal first (accumulate = 0 at g = 0).
-        g1_wide_mmas<3>(tacc, tmem + ab * kG1ABuf, db0, kq, g == 0);
+        g1_wide_mmas<3, S>(tacc, tmem + ab * kG1ABuf, db0, kq, g == 0);
         umma_commit(&afree[ab]);                      // A buffer ab may take quarter block g + 2
         if (kq == 3 || g + 1 == nhalf) umma_commit(&bempty[s]);
       }
@@ -534,7 +556,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
     const uint32_t nmask = cm ? 0xffffffffu : 0u;
     const int E = sv ? p.colE[(long long)dom * norb + sIdx] : 0;
     const bool zc = E == 0;                   // an all-zero orbital (or none): zero digits
-    const double sc41 = zc ? 0.0 : ldexp(1.0, 41 - (E - 1022));  // x 2^41 / tau_s: |v sc41| < 2^41
+    const double sc41 = zc ? 0.0 : ldexp(1.0, 7 * S - 1 - (E - 1022));  // x 2^(7S-1) / tau_s
     double nrm = 0.0;
     const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
     for (int g = 0, s = 0, ph = 0; g < nhalf; ++g) {  // s = g % kG1PsiSlots, ph = (g / kG1PsiSlots) & 1
@@ -542,7 +564,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       mbar_wait(&pfull[s], (uint32_t)ph);
       const long long ra = r0 + (long long)g * kG1Half;
       // this lane's component of Psi[row][sIdx] (Re for cm = 0, Im for cm = 1): 8-byte loads, 2 norb per row
-      const double* P = reinterpret_cast<const double*>(Psm + s * kG1PsiB) + 2 * sIdx + cm;
+      const R* P = reinterpret_cast<const R*>(Psm + s * kG1PsiB) + 2 * sIdx + cm;
       // each lane digitises its own component only (even lane m = 2s: Re, odd lane: Im) of its 4 rows
       // (4h .. 4h + 3 of the quarter block), in integer arithmetic (digits_i64), and the lane pair exchanges
       // them: row 2s of A takes (Re, Im) per grid row, row 2s+1 takes (Im, -Re) (bytewise negated digits:
@@ -557,11 +579,11 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       }
 #pragma unroll
       for (int t = 0; t < 4; ++t) nrm = fma(v[t], v[t], nrm);  // absent rows add +0 exactly
-      uint32_t own[kI8S];
-      digits_i64(v, sc41, own);
-      uint32_t dg[kI8S][2];
+      uint32_t own[S];
+      digits_x<S>(v, sc41, own);
+      uint32_t dg[S][2];
 #pragma unroll
-      for (int i = 0; i < kI8S; ++i) {
+      for (int i = 0; i < S; ++i) {
         const uint32_t mine = own[i];
         const uint32_t other = __shfl_xor_sync(0xffffffffu, mine, 1);
         // bytes t = 0..3 are rows 4h + t; A word w (K bytes 8h + 4w ..) holds rows (2w, 2w+1) as
@@ -577,7 +599,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       if (g >= 2) mbar_wait(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));  // MMAs of block g - 2 are done with it
       tc_fence_after();
 #pragma unroll
-      for (int i = 0; i < kI8S; ++i) tmem_st2(trow + ab * kG1ABuf + i * 8 + 2 * h, dg[i]);
+      for (int i = 0; i < S; ++i) tmem_st2(trow + ab * kG1ABuf + i * 8 + 2 * h, dg[i]);
       asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
       tc_fence_before();
       __syncwarp();
@@ -594,7 +616,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
 #pragma unroll
     for (int c = 0; c < 16; ++c) cacc[c] = 0.0;
 #pragma unroll 1
-    for (int d = 2; d <= kI8S + 1; ++d) {
+    for (int d = 2; d <= S + 1; ++d) {
       int32_t a[16];
       tmem_ld16(tacc + (d - 2) * 64 + ((uint32_t)(32 * q) << 16) + 16 * h, a);
       tmem_wait_ld();
@@ -636,9 +658,9 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   }
 }
 
-size_t gemm1_i8_bytes(int ndom, long long ng) {
+size_t gemm1_i8_bytes(int ndom, long long ng, int S) {
   const long long nblk = (ng + kG1Rows - 1) / kG1Rows;
-  return (size_t)ndom * nblk * kG1BlkB;
+  return (size_t)ndom * nblk * S * kG1SliceB;
 }
 long long gemm1_i8_rows_per_split(long long ng, int ndom, int num_sms) {
   int cpd = num_sms / ndom;
@@ -648,25 +670,33 @@ long long gemm1_i8_rows_per_split(long long ng, int ndom, int num_sms) {
   if (rps > 32768) rps = 32768;  // int32 accumulators: 6 x 2 rps x 64 x 64 < 2^31
   return rps;
 }
-cudaError_t launch_bslice1_i8(const double2* B, int ndom, int nproj, long long ng, int* bexp, int8_t* out,
+cudaError_t launch_bslice1_i8(const void* B, bool sp, int ndom, int nproj, long long ng, int* bexp, int8_t* out,
                               cudaStream_t st) {
   cudaError_t e = cudaMemsetAsync(bexp, 0, sizeof(int) * ndom * nproj, st);
   if (e != cudaSuccess) return e;
-  launch_k(k_bexp1_i8, dim3(296, ndom), 256, 0, st, B, nproj, ng, bexp);
   const long long nblk = (ng + kG1Rows - 1) / kG1Rows;
   dim3 grid((unsigned)((nblk * 64 + 7) / 8), ndom);
-  launch_k(k_bslice1_i8, grid, 256, 0, st, B, nproj, ng, nblk, (const int*)bexp, out);
+  if (sp) {
+    const float2* b = static_cast<const float2*>(B);
+    launch_k(k_bexp1_i8<float2>, dim3(296, ndom), 256, 0, st, b, nproj, ng, bexp);
+    launch_k(k_bslice1_i8<float2, 4>, grid, 256, 0, st, b, nproj, ng, nblk, (const int*)bexp, out);
+  } else {
+    const double2* b = static_cast<const double2*>(B);
+    launch_k(k_bexp1_i8<double2>, dim3(296, ndom), 256, 0, st, b, nproj, ng, bexp);
+    launch_k(k_bslice1_i8<double2, 6>, grid, 256, 0, st, b, nproj, ng, nblk, (const int*)bexp, out);
+  }
   return cudaGetLastError();
 }
 cudaError_t launch_gemm1_i8(const Gemm1I8Args& a, cudaStream_t st) {
   dim3 grid(a.nsplit, a.ndom);
-  launch_k(k_gemm1_i8, grid, kG1Threads, kG1Smem, st, a);
+  if (a.sp) launch_k(k_gemm1_i8<float2, 4>, grid, kG1Threads, I8G1<4, float2>::Smem, st, a);
+  else launch_k(k_gemm1_i8<double2, 6>, grid, kG1Threads, I8G1<6, double2>::Smem, st, a);
   return cudaGetLastError();
 }
 
-size_t gemm2_i8_bytes(int ndom, long long ng) {
+size_t gemm2_i8_bytes(int ndom, long long ng, int S) {
   const long long tiles = (ng + kI8NT - 1) / kI8NT;
-  return (size_t)ndom * tiles * kI8TileB;
+  return (size_t)ndom * tiles * S * kI8SliceB;
 }
 size_t gemm2_i8_sig_bytes(int ndom, long long ng) {
   const long long tiles = (ng + kI8NT - 1) / kI8NT;
@@ -674,11 +704,12 @@ size_t gemm2_i8_sig_bytes(int ndom, long long ng) {
 }
 bool gemm2_i8_supported(int nproj, int norb) { return nproj >= 1 && nproj <= 64 && norb >= 1 && norb <= 64; }
 
-cudaError_t launch_bslice_i8(const double2* B, int ndom, int nproj, long long ng, int8_t* out, double* sig,
+cudaError_t launch_bslice_i8(const void* B, bool sp, int ndom, int nproj, long long ng, int8_t* out, double* sig,
                              cudaStream_t st) {
   const long long tiles = (ng + kI8NT - 1) / kI8NT;
   dim3 grid((unsigned)((tiles * kI8NT + 7) / 8), ndom);
-  launch_k(k_bslice_i8, grid, 256, 0, st, B, nproj, ng, tiles, out, sig);
+  if (sp) launch_k(k_bslice_i8<float2, 4>, grid, 256, 0, st, static_cast<const float2*>(B), nproj, ng, tiles, out, sig);
+  else launch_k(k_bslice_i8<double2, 6>, grid, 256, 0, st, static_cast<const double2*>(B), nproj, ng, tiles, out, sig);
   return cudaGetLastError();
 }
 
@@ -688,17 +719,30 @@ cudaError_t launch_gemm2_i8(const Gemm2Args& a, cudaStream_t st) {
   if (cpd < 1) cpd = 1;
   if (cpd > tiles) cpd = (int)tiles;
   dim3 grid(cpd, a.ndom);
-  if (a.psi_out) launch_k(k_gemm2_i8<true>, grid, kI8Threads, kI8Smem, st, a);
-  else launch_k(k_gemm2_i8<false>, grid, kI8Threads, kI8Smem, st, a);
+  if (a.sp) {
+    constexpr int sm = I8G2<4, float2>::Smem;
+    if (a.psi_out) launch_k(k_gemm2_i8<true, float2, 4>, grid, kI8Threads, sm, st, a);
+    else launch_k(k_gemm2_i8<false, float2, 4>, grid, kI8Threads, sm, st, a);
+  } else {
+    constexpr int sm = I8G2<6, double2>::Smem;
+    if (a.psi_out) launch_k(k_gemm2_i8<true, double2, 6>, grid, kI8Threads, sm, st, a);
+    else launch_k(k_gemm2_i8<false, double2, 6>, grid, kI8Threads, sm, st, a);
+  }
   return cudaGetLastError();
 }
 
 cudaError_t gemm_i8_set_attributes() {
-  cudaError_t e = cudaFuncSetAttribute(k_gemm2_i8<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kI8Smem);
-  if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_gemm1_i8, cudaFuncAttributeMaxDynamicSharedMemorySize, kG1Smem);
-  if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(k_gemm2_i8<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kI8Smem);
+  cudaError_t e = cudaSuccess;
+#define LFD_ATTR(f, sm) \
+  if ((e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, sm)) != cudaSuccess) return e
+  LFD_ATTR((k_gemm2_i8<false, double2, 6>), (I8G2<6, double2>::Smem));
+  LFD_ATTR((k_gemm2_i8<true, double2, 6>), (I8G2<6, double2>::Smem));
+  LFD_ATTR((k_gemm2_i8<false, float2, 4>), (I8G2<4, float2>::Smem));
+  LFD_ATTR((k_gemm2_i8<true, float2, 4>), (I8G2<4, float2>::Smem));
+  LFD_ATTR((k_gemm1_i8<double2, 6>), (I8G1<6, double2>::Smem));
+  LFD_ATTR((k_gemm1_i8<float2, 4>), (I8G1<4, float2>::Smem));
+#undef LFD_ATTR
+  return cudaSuccess;
 }
 
 }  // namespace lfd

@@ -1,4 +1,4 @@
-"""GPU parity of the SP variant (LFD_FLAG_SP: complex64 Psi / B, FP32 sweeps, 3xTF32 tensor-core projector
+"""GPU parity of the SP variant (LFD_FLAG_SP: complex64 Psi / B, FP32 sweeps, int8-digit or 3xTF32 tensor-core projector
 GEMMs, FP64 small kernels) against the FP64 oracle, through the C ABI.
 
 Tolerance: every step rounds each orbital value O(30) times at the FP32 unit roundoff
@@ -118,3 +118,37 @@ def test_sp_c2_full_size_two_steps():
     for n in range(2):
         ref.step(cfg, p, x.proj.astype(np.complex128), x.dnl, x.vloc, midpoint_A(w, n), 1)
     assert rel(got[0][..., cols], p) <= sp_tol(2)
+
+
+@pytest.mark.parametrize("name,steps", [("P0", 100), ("P1", 20), ("P2z", 20), ("C1", 10)])
+def test_sp_parity_int8_digit_gemms(name, steps):
+    """the SP projector GEMMs on the tcgen05 int8 tensor cores (4 digits per operand; forced on these small grids,
+    the default at C2): same bound; the orbital exponents for GEMM-1 come from the SP z pass"""
+    from paper_conf_ipps_razakhllknvn24_b200 import lfd
+    w = workload(name)
+    x = _inputs(w, 85)
+    assert_sp(w, _gpu(w, x, steps, flags=lfd.LFD_FLAG_NL_I8), _ref(w, x, steps), steps)
+
+
+def test_sp_int8_sequence_energy_exact():
+    from paper_conf_ipps_razakhllknvn24_b200 import lfd
+    w = workload("P0")
+    x = _inputs(w, 86)
+    got = _gpu(w, x, 40, flags=lfd.LFD_FLAG_NL_I8, sequence=True, energy=True)
+    want = _ref(w, x, 40)
+    assert_sp(w, got, want, 40)
+    assert np.abs(got[4] - want[4]).max() <= sp_tol(40) * np.abs(want[4]).max()
+    want_x = _ref(w, x, 30, exact=True)
+    assert_sp(w, _gpu(w, x, 30, flags=lfd.LFD_FLAG_NL_I8 | lfd.LFD_FLAG_EXACT_NL), want_x, 30)
+
+
+def test_sp_c2_default_path_is_int8_tensor_cores():
+    import torch
+    from paper_conf_ipps_razakhllknvn24_b200 import Context, lfd
+    w = workload("C2")
+    x = _inputs(w, 87)
+    dev = torch.device("cuda:0")
+    ctx = Context(torch.from_numpy(x.psi0).to(dev), torch.from_numpy(x.proj).to(dev), x.dnl, x.occ,
+                  (w.hx, w.hy, w.hz), w.dt)
+    assert lfd.lfd_nl_path(ctx.ctx) == 3
+    ctx.close()
