@@ -33,6 +33,7 @@ PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FP64_PEAK_FILE = os.path.join(ROOT, "profiles", "r01_fp64_peaks.jsonl")
 NCU_SUMMARY = os.path.join(ROOT, "profiles", "latest_ncu_full_summary.csv")
 I8_DIGIT_BYTES = 6 * 128  # B digits per grid point of the int8-digit GEMMs (6 digits x K = 128 bytes)
+SP_DIGIT_BYTES = 4 * 128  # the same for the SP variant (4 digits)
 NCU_NAMES = {"nl_proj": "k_gemm1", "nl_back": "k_gemm2", "kin_x": "k_kin<1, 1, 1", "kin_y": "k_kin<1, 0",
              "kin_z": "k_kin<1, 2>", "kin_yz": "k_kin_yz", "density": "k_density", "nl_back_x": "k_gemm2x"}
 
@@ -341,6 +342,7 @@ def run_sp_mode(args, w, x, dev, stream, pk):
     for n in range(args.steps):
         step(args.warmup + n)
     prof = lfd.lfd_profile_read(ctx.ctx)
+    nl_path = lfd.lfd_nl_path(ctx.ctx)
     ctx.close()
     del psi, proj
     tot = sum(v[0] for v in prof.values()) or 1.0
@@ -355,7 +357,13 @@ def run_sp_mode(args, w, x, dev, stream, pk):
         e = {"ms_per_launch": avg, "launches": cnt, "share": round(kms / tot, 4)}
         if k in work:
             b, f = work[k]
-            if f > 0:
+            if f > 0 and nl_path == 3:
+                # int8-digit tcgen05 GEMMs with 4 digits (nl_i8.cu, S = 4): bound by streaming complex64 Psi
+                # (half the FP64 bytes) and B's digits (4 x 128 B per grid point)
+                b = 0.5 * (b - 16.0 * w.ngrid * w.nproj * w.ndom) + SP_DIGIT_BYTES * w.ngrid * w.ndom
+                e.update({"bound": "hbm", "achieved": b / (avg * 1e-3) / 1e9, "unit": "GB/s", "peak": pk["hbm_gbs"],
+                          "bytes_per_launch": b, "c64_equiv_tflops": f / (avg * 1e-3) / 1e12})
+            elif f > 0:
                 e.update({"bound": "tensor", "achieved": f / (avg * 1e-3) / 1e12, "unit": "TFLOP/s", "peak": tpeak})
             else:
                 e.update({"bound": "hbm", "achieved": 0.5 * b / (avg * 1e-3) / 1e9, "unit": "GB/s",
@@ -363,7 +371,9 @@ def run_sp_mode(args, w, x, dev, stream, pk):
             e["frac"] = e["achieved"] / e["peak"]
         kern[k] = e
     return {"value": w.ogp_per_step * args.steps / (ms / 1e3), "unit": UNIT, "ms_per_step": ms / args.steps,
-            "dtype": "c64 (FP32 sweeps, 3xTF32 tensor-core GEMMs, FP64 reductions)", "kernels": kern,
+            "dtype": "c64 (FP32 sweeps, " + ("int8-digit tcgen05 GEMMs (4 digits)" if nl_path == 3 else
+                                             "3xTF32 tensor-core GEMMs") + ", FP64 reductions)", "kernels": kern,
+            "nl_path": {2: "sp-3xtf32", 3: "sp-int8-digit-tcgen05", -1: "none"}.get(nl_path, nl_path),
             "tensor_peak_source": f"measured mma.sync tf32 {pk['tf32_tflops']} TF/s (profiles/r01_sp_peaks.txt) "
                                   "x 8/18 (3M x 3xTF32)",
             "note": "same step loop as the headline on complex64 copies of Psi / B (LFD_FLAG_SP); parity vs the "

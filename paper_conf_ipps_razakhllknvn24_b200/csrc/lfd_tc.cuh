@@ -83,7 +83,7 @@ __device__ __forceinline__ void digits_i64(const double v[4], double sc, uint32_
 __device__ __forceinline__ void digits_s4(const double v[4], double sc, uint32_t out[4]) {
   constexpr double kM = 6755399441055744.0;
   constexpr long long kMb = 0x4338000000000000LL;
-  constexpr int kC4 = 64 * ((1 << 28) - 1) / 127;
+  constexpr int kC4 = 64 * (((1 << 28) - 1) / 127);  // 64 (1 + 128 + 128^2 + 128^3): the fields' 64s
   uint32_t w[4];
 #pragma unroll
   for (int q = 0; q < 4; ++q) {

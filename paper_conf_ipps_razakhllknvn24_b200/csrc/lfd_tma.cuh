@@ -37,6 +37,21 @@ __device__ __forceinline__ void tma_row(void* dst, const void* src, uint32_t byt
       : "memory");
 }
 
+// Row copy of any multiple of 8 bytes (complex64 rows of odd length): cp.async.bulk takes multiples of 16, so an
+// 8-byte tail goes by a plain load / shared store, made visible to the async proxy and ordered before the
+// arrive (release) that the consumers acquire; the barrier expects the bulk bytes plus `extra` (other copies
+// completing on it). One thread.
+__device__ __forceinline__ void tma_row8(void* dst, const void* src, uint32_t bytes, uint64_t* bar, uint32_t extra) {
+  const uint32_t bulk = bytes & ~15u;
+  if (bulk != bytes) {
+    *reinterpret_cast<uint2*>(static_cast<char*>(dst) + bulk) =
+        *reinterpret_cast<const uint2*>(static_cast<const char*>(src) + bulk);
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  mbar_expect_tx(bar, bulk + extra);
+  if (bulk) tma_row(dst, src, bulk, bar);
+}
+
 // Tiled tensor copy (3-D tensor map, coordinates innermost first) into shared memory.
 __device__ __forceinline__ void tma_3d(void* dst, const void* tmap, int c0, int c1, int c2, uint64_t* bar) {
   asm volatile(

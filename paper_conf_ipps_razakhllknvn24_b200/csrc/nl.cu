@@ -26,7 +26,6 @@ namespace {
 
 constexpr int kThreads = 256;  // 8 warps: 2 (M) x 4 (N), warp tile 32 x 16 complex
 constexpr int kTile = 64;      // CTA tile 64 x 64 complex
-constexpr int kStages = 4;
 
 // GEMM-1 stage: A rows [KC1][kLd1] (B rows, m along the row) and X rows [KC1][kLd1].
 constexpr int kKC1 = 32;
@@ -77,21 +76,6 @@ struct Frag {
   __device__ __forceinline__ double im(int i, int j, int c) const {
 #if LFD_3M
     return t3[i][j][c] - t1[i][j][c] - t2[i][j][c];
-#else
-    return t2[i][j][c];
-#endif
-  }
-  // GEMM-1 (conjugated A) results
-  __device__ __forceinline__ double re_conj(int i, int j, int c) const {
-#if LFD_3M
-    return t1[i][j][c] + t2[i][j][c];
-#else
-    return t1[i][j][c];
-#endif
-  }
-  __device__ __forceinline__ double im_conj(int i, int j, int c) const {
-#if LFD_3M
-    return t3[i][j][c] - t1[i][j][c] + t2[i][j][c];
 #else
     return t2[i][j][c];
 #endif

@@ -61,7 +61,9 @@ struct I8G2 {
   static constexpr int Slots = (512 - WCols) / kI8NT;     // 5 (S = 6), 6 (S = 4)
   static constexpr int SubRowsB = kI8SubR * 64 * (int)sizeof(T);  // norb <= 64
   static constexpr int SubB = SubRowsB + kI8SubR * 8;     // + the sub-tile's row scales sigma_r
-  static constexpr int Smem = kI8Stages * TileB + kI8PsiSlots * SubB + 1024;  // + alignment slack
+  // (the Psi ring's space first stages C'' -- FP64, up to 64 x 64 complex -- for the W digits)
+  static constexpr int RingB = kI8PsiSlots * SubB > 64 * 64 * 16 ? kI8PsiSlots * SubB : 64 * 64 * 16;
+  static constexpr int Smem = kI8Stages * TileB + RingB + 1024;  // + alignment slack
 };
 constexpr int kI8Threads = (kI8EpiWarps + 3) * 32;  // epilogue warps + 2 producers + MMA
 constexpr int kWDig = kI8EpiWarps, kWMma = kI8EpiWarps + 1, kWPsi = kI8EpiWarps + 2;  // role warps
@@ -223,8 +225,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
             mbar_arrive(&pfull[s]);
             continue;
           }
-          mbar_expect_tx(&pfull[s], (uint32_t)(nr * rowb + kI8SubR * 8));
-          tma_row(Psm + s * kI8SubB, prow + r0 * norb, (uint32_t)(nr * rowb), &pfull[s]);
+          tma_row8(Psm + s * kI8SubB, prow + r0 * norb, (uint32_t)(nr * rowb), &pfull[s], kI8SubR * 8);
           tma_row(Psm + s * kI8SubB + kI8SubRowsB, sig + r0, kI8SubR * 8, &pfull[s]);
         }
     }
@@ -524,8 +525,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
         if (g >= kG1PsiSlots) mbar_wait(&pempty[s], (uint32_t)(((g / kG1PsiSlots) - 1) & 1));
         const long long ra = r0 + (long long)g * kG1Half;
         const long long nr = (r1 - ra) < kG1Half ? (r1 - ra) : kG1Half;
-        mbar_expect_tx(&pfull[s], (uint32_t)(nr * rowb));
-        tma_row(Psm + s * kG1PsiB, prow + ra * norb, (uint32_t)(nr * rowb), &pfull[s]);
+        tma_row8(Psm + s * kG1PsiB, prow + ra * norb, (uint32_t)(nr * rowb), &pfull[s], 0);
       }
     }
   } else if (warp == kG1WMma) {  // MMA issuer

@@ -45,7 +45,6 @@ __device__ __forceinline__ TF split_tf32(float x) {
   const unsigned xb = __float_as_uint(x);
   return {xb, __float_as_uint(x - __uint_as_float(xb & 0xffffe000u))};
 }
-__device__ __forceinline__ TF neg(TF v) { return {v.hi ^ 0x80000000u, v.lo ^ 0x80000000u}; }
 // Not volatile: the compiler may interleave the independent HMMAs of different accumulators.
 __device__ __forceinline__ void hmma(float* c, unsigned a0, unsigned a1, unsigned a2, unsigned a3, unsigned b0,
                                      unsigned b1) {

@@ -482,3 +482,12 @@ def test_narrow_orbital_tiles(norb, nproj, dims):
     w = workload("P0").with_(nx=dims[0], ny=dims[1], nz=dims[2], norb=norb, nocc=min(norb, 12), nproj=nproj)
     x = make_inputs(w, seed=15)
     assert_parity(w, run_gpu(w, x, 4, laser(w)), run_ref(w, x, 4, laser(w)))
+
+
+@pytest.mark.parametrize("norb,nproj,dims", [(512, 64, (8, 10, 12)), (130, 64, (8, 6, 10)), (200, 30, (10, 8, 6))])
+def test_wide_orbital_sets_short_projector_tile(norb, nproj, dims):
+    """norb > 64 with nproj <= 64 (C5's nproj = 64 column: the TMA GEMM-2 over several orbital tiles, GEMM-1 with
+    one projector tile and several orbital tiles) against the oracle."""
+    w = workload("P0").with_(nx=dims[0], ny=dims[1], nz=dims[2], norb=norb, nocc=min(norb, 40), nproj=nproj)
+    x = make_inputs(w, seed=16)
+    assert_parity(w, run_gpu(w, x, 3, laser(w)), run_ref(w, x, 3, laser(w)))
