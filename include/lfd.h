@@ -65,7 +65,7 @@ typedef struct {
   int32_t nref_max;    /* max reference-basis columns for lfd_remap_occ, 0..2048 (0: max(norb, nproj)) */
   double dt;           /* Delta_QD [a.u.], finite and nonzero (negative = backward in time) */
   int32_t device;      /* CUDA device ordinal */
-  int32_t flags;       /* 0 or LFD_FLAG_NO_CARRY | EXACT_NL | SP | NL_DMMA | NL_I8 | DENSE_D (below) */
+  int32_t flags;       /* 0 or LFD_FLAG_NO_CARRY | EXACT_NL | SP | NL_DMMA | NL_I8 | DENSE_D | NO_PDL (below) */
 } lfd_config;
 
 /* lfd_config.flags: disable the projection carry (lfd_step takes the C of each nonlocal factor that
@@ -110,6 +110,11 @@ typedef struct {
  * the same operator B D B^H, so every path (first-order and exact factors, carry, merged sequences, energy)
  * applies unchanged. lfd_set_occupations etc. are unaffected. nproj <= 512. */
 #define LFD_FLAG_DENSE_D 32
+
+/* lfd_config.flags: launch every kernel in plain stream order, without programmatic dependent launch (PDL lets
+ * a kernel's set-up overlap its predecessor's tail; the results are the same either way). For debugging and
+ * measurement. */
+#define LFD_FLAG_NO_PDL 64
 
 /* Kernel classes, for lfd_profile_read(). */
 typedef enum {

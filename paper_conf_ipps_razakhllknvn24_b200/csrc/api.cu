@@ -74,7 +74,7 @@ lfd_status validate(const lfd_config* c, std::string& why) {
   if (c->nproj < 0 || c->nproj > 2048) { why = "nproj must be in [0, 2048]"; return LFD_EINVAL; }
   if (!(c->dt != 0.0) || !std::isfinite(c->dt)) { why = "dt must be finite and nonzero"; return LFD_EINVAL; }
   if (c->flags & ~(LFD_FLAG_NO_CARRY | LFD_FLAG_EXACT_NL | LFD_FLAG_SP | LFD_FLAG_NL_DMMA | LFD_FLAG_NL_I8 |
-                   LFD_FLAG_DENSE_D)) {
+                   LFD_FLAG_DENSE_D | LFD_FLAG_NO_PDL)) {
     why = "unknown flags";
     return LFD_EINVAL;
   }
@@ -312,6 +312,7 @@ struct lfd_ctx {
   // int8-digit GEMM-1: the orbital exponents in the workspace describe the current Psi (set by the K_y K_z
   // pass that wrote it, consumed -- and cleared on the device -- by GEMM-1)
   bool colE_valid = false;
+  bool no_pdl = false;    // LFD_FLAG_NO_PDL: plain stream order for every launch
   bool exact = false;     // LFD_FLAG_EXACT_NL: exactly unitary nonlocal factor (orthonormal B)
   bool kin_fused = true;  // Phi.K_y K_z in one pass (else separate y and z passes: lines too long for the ring)
   CUtensorMap psi_tmap;   // TMA descriptor of Psi for the fused pass
@@ -406,7 +407,7 @@ lfd_status launch(lfd_ctx* c, int kid, const char* name, F&& f) {
     cudaEventRecord(s->a, c->stream);
   }
   cudaError_t e;
-  if (c->g.sp && !c->L.i8) {  // the 3xTF32 SP contexts launch without PDL (C2 SP step 0.98 ms without, 1.12 ms
+  if ((c->g.sp && !c->L.i8) || c->no_pdl) {  // the 3xTF32 SP contexts launch without PDL (C2 SP step 0.98 ms without, 1.12 ms
                              // with: the early-resident CTAs of the next kernel slow the SP GEMMs' cp.async rings)
     const bool prev = lfd::pdl_suspended();
     lfd::pdl_suspend(true);
@@ -973,6 +974,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   c->device = cfg->device;
   c->num_sms = prop.multiProcessorCount;
   c->carry = (cfg->flags & LFD_FLAG_NO_CARRY) == 0;
+  c->no_pdl = (cfg->flags & LFD_FLAG_NO_PDL) != 0;
   c->scaled = c->scaled && lfd::kin_scaled_ok(g);
   c->kin_fused = c->kin_fused && lfd::kin_yz_supported(g) && !g.sp;
   c->dmaps = lfd::density_maps_create(g, c->psi, active_orbitals(g, occ));

@@ -519,11 +519,8 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
         }
       }
     }
-    __syncwarp();
-    if ((tid & 31) == 0) {  // this warp is done with own line y and x+1 line y
-      mbar_arrive(&oempty[so]);
-      if (has_xn) mbar_arrive(&xempty[sx]);
-    }
+    // this warp is done with own line y and x+1 line y (once its loads have returned: lfd_tma.cuh)
+    mbar_release2(&oempty[so], &xempty[sx], has_xn, ((rho + pxr) + (pyr + pzr)) + (pxi + pyi + pzi), (tid & 31) == 0);
     // the currents and the kinetic energy density are linear in the P_d: form them per lane first
     // (Im(e^{i theta} P) = cos Im P + sin Re P, Re(e^{i theta} P) = cos Re P - sin Im P)
     const double jx = (kPer || has_x) ? (ex.x * pxi + ex.y * pxr) * ihx : 0.0;

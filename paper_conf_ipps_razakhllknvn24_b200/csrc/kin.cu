@@ -335,10 +335,8 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
       w1 = cz();
     }
   };
-  auto release = [&](int s) {
-    __syncwarp();
-    if ((tid & 31) == 0) mbar_arrive(&empty[s]);
-  };
+  // dep: computed from this warp's last loads of the slot (they must have returned: lfd_tma.cuh)
+  auto release = [&](int s, double dep) { mbar_release(&empty[s], dep, (tid & 31) == 0); };
   // colE != nullptr: the largest biased FP64 exponent of Re / Im of each orbital's output, for the int8-digit
   // GEMM-1 that follows (its per-orbital power-of-two scale; nl_i8.cu) -- integer max on the high words
   int me = 0;
@@ -364,8 +362,8 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
     kz(0, wa0, wa1);
     mbar_wait(&full[1], 0);
     kz(1, wb0, wb1);
-    release(0);
-    release(1);
+    release(0, wa0.x + wa1.x);
+    release(1, wb0.x + wb1.x);
     L0.first(cy, wa0, wb0);
     L1.first(cy, wa1, wb1);
     mbar_wait(&full[2], 0);
@@ -391,8 +389,8 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
       L1.steady(cy, wa1, wb1, [&](int k, double2 v) {
         if (act) o0p[k * yst + norb] = trk(cmul(k == 0 ? fa1 : fb1, v));
       });
-      release(s_prev);
-      release(s_prev + 1);
+      release(s_prev, fa0.x + fa1.x);
+      release(s_prev + 1, fb0.x + fb1.x);
       o0p += 2 * yst;
       s_prev = s_a;
       s_a += 2;
@@ -419,8 +417,8 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
         kz(s_b, wb0, wb1);
       }
       if (p == 0) {
-        release(s_a);
-        if (hb) release(s_b);
+        release(s_a, wa0.x + wa1.x);
+        if (hb) release(s_b, wb0.x + wb1.x);
       }
       // Phi of the planes this march step stores (2p-2 in slot s_prev, 2p-1 in the next slot)
       int s_pb = s_prev + 1;
@@ -435,8 +433,8 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
       L0.push(cy, p, wa0, wb0, hb, [&](int y, double2 v) { put0(y, y == ya - 2 ? fa0 : fb0, v); });
       L1.push(cy, p, wa1, wb1, hb, [&](int y, double2 v) { put1(y, y == ya - 2 ? fa1 : fb1, v); });
       if (p >= 2) {
-        release(s_prev);
-        release(s_pb);
+        release(s_prev, fa0.x + fa1.x);
+        release(s_pb, fb0.x + fb1.x);
       }
       s_prev = s_a;
       s_a = s_b + 1;

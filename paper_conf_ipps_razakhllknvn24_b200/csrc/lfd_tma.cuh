@@ -18,6 +18,38 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
 }
+// Warp-collective release of a shared-memory stage that TMA refills. An mbarrier.arrive is not held back for the
+// warp's shared loads still in flight (measured: one 8-lane phase of a k_gemm2_tma LDS.128 returned the bytes of
+// the next refill -- two rows of a DMMA tile wrong, a few times per 10^5 tiles), and the TMA write does not queue
+// behind them. So the arrive waits for a value computed from the warp's last loads of the stage (`dep`): every
+// lane turns it into an always-zero integer (+-0 or NaN times 0 is never > 1), a warp-wide OR (redux) needs every
+// lane's value, and the arrive's count is 1 + that zero. Lane `leader` arrives on each of the n barriers.
+__device__ __forceinline__ uint32_t lds_done_count(double dep) {
+  uint32_t cnt;
+  asm volatile(
+      "{\n.reg .f64 t;\n.reg .pred p;\n.reg .b32 z;\n"
+      "mul.f64 t, %1, 0d0000000000000000;\n"
+      "setp.gt.f64 p, t, 0d3FF0000000000000;\n"
+      "selp.b32 z, 1, 0, p;\n"
+      "redux.sync.or.b32 z, z, 0xffffffff;\n"
+      "add.u32 %0, z, 1;\n}\n"
+      : "=r"(cnt)
+      : "d"(dep)
+      : "memory");
+  return cnt;
+}
+__device__ __forceinline__ void mbar_release(uint64_t* bar, double dep, bool leader) {
+  const uint32_t cnt = lds_done_count(dep);
+  if (leader) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(cnt) : "memory");
+}
+__device__ __forceinline__ void mbar_release2(uint64_t* bar0, uint64_t* bar1, bool two, double dep, bool leader) {
+  const uint32_t cnt = lds_done_count(dep);
+  if (leader) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar0)), "r"(cnt) : "memory");
+    if (two) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar1)), "r"(cnt) : "memory");
+  }
+}
+
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   asm volatile(
       "{\n"

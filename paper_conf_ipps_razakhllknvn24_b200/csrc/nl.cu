@@ -246,10 +246,10 @@ __global__ void __launch_bounds__(kThreads1, 1) k_gemm1(const __grid_constant__ 
     mbar_wait(&full[s], (uint32_t)((i / kStages1) & 1));
     const double2* As = reinterpret_cast<const double2*>(smem + s * S::StageBytes);
     const double2* Xs = reinterpret_cast<const double2*>(smem + s * S::StageBytes + S::ABytes);
+    double2 a[S::MI], x[S::NI];
 #pragma unroll
     for (int kk = 0; kk < kKC1; kk += 4) {
       const int k = kk + t;
-      double2 a[S::MI], x[S::NI];
 #pragma unroll
       for (int mi = 0; mi < S::MI; ++mi) a[mi] = As[k * S::LDA + wm * (kMT / S::WM) + mi * 8 + g];
 #pragma unroll
@@ -260,8 +260,12 @@ __global__ void __launch_bounds__(kThreads1, 1) k_gemm1(const __grid_constant__ 
       }
       mma_conj(acc, a, x);
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[s]);
+    double dep = 0.0;  // the stage's last loads have returned before it is released (lfd_tma.cuh)
+#pragma unroll
+    for (int mi = 0; mi < S::MI; ++mi) dep += a[mi].x;
+#pragma unroll
+    for (int ni = 0; ni < S::NI; ++ni) dep += x[ni].x;
+    mbar_release(&empty[s], dep, lane == 0);
   }
 
   // epilogue: split partials (fixed positions, reduced in order by k_reduce); 3M recombination for
@@ -780,19 +784,21 @@ struct G2Shape {
   static constexpr int Smem = Stages * StageBytes + 2 * Stages * 8;
 };
 
+// returns a value computed from the chunk's last shared loads (for mbar_release)
 template <int kLDC>
-__device__ __forceinline__ void gemm2_chunk(const double2* As, const double2* Cs, int wm, int wn, int g, int t,
-                                            Frag& acc) {
+__device__ __forceinline__ double gemm2_chunk(const double2* As, const double2* Cs, int wm, int wn, int g, int t,
+                                              Frag& acc) {
+  double2 a[4], c[2];
 #pragma unroll
   for (int kk = 0; kk < kKC2; kk += 4) {
     const int k = kk + t;
-    double2 a[4], c[2];
 #pragma unroll
     for (int mi = 0; mi < 4; ++mi) a[mi] = As[(wm * 32 + mi * 8 + g) * kLdA2 + k];
 #pragma unroll
     for (int ni = 0; ni < 2; ++ni) c[ni] = Cs[k * kLDC + wn * 16 + ni * 8 + g];
     mma_4x2(acc, a, c);
   }
+  return ((a[0].x + a[1].x) + (a[2].x + a[3].x)) + (c[0].x + c[1].x);
 }
 
 template <int kRT, int kCT>
@@ -879,9 +885,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2(const __grid_constant__ C
       mbar_wait(&full[stage], (uint32_t)((gc / kSt) & 1));
       const double2* As = reinterpret_cast<const double2*>(smem + stage * S::StageBytes);
       const double2* Cs = As + kRT * kLdA2;
-      gemm2_chunk<S::LDC>(As, Cs, wm, wn, g, t, acc);  // the K tail is zero fill
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&empty[stage]);
+      const double dep = gemm2_chunk<S::LDC>(As, Cs, wm, wn, g, t, acc);  // the K tail is zero fill
+      mbar_release(&empty[stage], dep, lane == 0);
       if (tid == 0 && gc + kSt < total) {  // refill once every warp has released the stage
         mbar_wait(&empty[stage], (uint32_t)((gc / kSt) & 1));
         issue(gc + kSt);
@@ -1036,6 +1041,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant
           }
       }
     };
+    double2 a[4], c[2];
 #pragma unroll
     for (int kk = 0; kk < kNK4; ++kk) {
       if (kNP == 0 && kk >= nk4) break;
@@ -1044,15 +1050,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemm2_tma(const __grid_constant
         if (j == 0 && wm == 0) asm volatile("bar.arrive 2, %0;" ::"n"(kThreads));
       }
       const int k = kk * 4 + t;
-      double2 a[4], c[2];
 #pragma unroll
       for (int mi = 0; mi < 4; ++mi) a[mi] = As[(wm * 32 + mi * 8 + g) * lda + k];
 #pragma unroll
       for (int ni = 0; ni < 2; ++ni) c[ni] = Cs[k * kLd1 + wn * 16 + ni * 8 + g];
       mma_4x2(acc, a, c);
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[s]);
+    // the stage's last loads have returned before it is released (lfd_tma.cuh)
+    mbar_release(&empty[s], ((a[0].x + a[1].x) + (a[2].x + a[3].x)) + (c[0].x + c[1].x), lane == 0);
     if (tid == 0 && j + kFullStages < my_items) {  // refill the stage once every warp has released it
       mbar_wait(&empty[s], (uint32_t)((j / kFullStages) & 1));
       issue(j + kFullStages);

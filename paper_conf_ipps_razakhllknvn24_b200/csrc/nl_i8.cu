@@ -594,8 +594,8 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
         dg[i][0] = __byte_perm(mine, b, 0x5140);  // [a0, b0, a1, b1]
         dg[i][1] = __byte_perm(mine, b, 0x7362);  // [a2, b2, a3, b3]
       }
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&pempty[s]);  // this warp is done with the Psi rows
+      // this warp is done with the Psi rows (its loads have returned: nrm depends on every one, lfd_tma.cuh)
+      mbar_release(&pempty[s], nrm, lane == 0);
       if (g >= 2) mbar_wait(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));  // MMAs of block g - 2 are done with it
       tc_fence_after();
 #pragma unroll

@@ -24,6 +24,7 @@ LFD_FLAG_SP = 4
 LFD_FLAG_NL_DMMA = 8
 LFD_FLAG_NL_I8 = 16
 LFD_FLAG_DENSE_D = 32
+LFD_FLAG_NO_PDL = 64
 LFD_BC_PERIODIC = 0
 LFD_BC_ZERO = 1
 STATUS = {0: "LFD_OK", -1: "LFD_EINVAL", -2: "LFD_ENOMEM", -3: "LFD_ECUDA", -4: "LFD_ESTATE",
