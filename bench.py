@@ -32,8 +32,10 @@ UNIT = "orbital-gridpoint updates/s"
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FP64_PEAK_FILE = os.path.join(ROOT, "profiles", "r01_fp64_peaks.jsonl")
 NCU_SUMMARY = os.path.join(ROOT, "profiles", "latest_ncu_full_summary.csv")
-I8_DIGIT_BYTES = 6 * 128  # B digits per grid point of the int8-digit GEMMs (6 digits x K = 128 bytes)
-SP_DIGIT_BYTES = 4 * 128  # the same for the SP variant (4 digits)
+I8_DIGIT_BYTES = 6 * 128  # B digits per grid point of the int8-digit GEMM-2 (6 base-128 digits x K = 128 bytes)
+G1_DIGIT_BYTES = 5 * 128  # ... of GEMM-1 (5 base-256 digits, nl_i8.cu)
+SP_DIGIT_BYTES = 4 * 128  # the SP variant's GEMM-2 (4 digits)
+SP_G1_DIGIT_BYTES = 3 * 128  # the SP variant's GEMM-1 (3 digits)
 NCU_NAMES = {"nl_proj": "k_gemm1", "nl_back": "k_gemm2", "kin_x": "k_kin<1, 1, 1", "kin_y": "k_kin<1, 0",
              "kin_z": "k_kin<1, 2>", "kin_yz": "k_kin_yz", "density": "k_density", "nl_back_x": "k_gemm2x"}
 
@@ -360,7 +362,8 @@ def run_sp_mode(args, w, x, dev, stream, pk):
             if f > 0 and nl_path == 3:
                 # int8-digit tcgen05 GEMMs with 4 digits (nl_i8.cu, S = 4): bound by streaming complex64 Psi
                 # (half the FP64 bytes) and B's digits (4 x 128 B per grid point)
-                b = 0.5 * (b - 16.0 * w.ngrid * w.nproj * w.ndom) + SP_DIGIT_BYTES * w.ngrid * w.ndom
+                dig = SP_G1_DIGIT_BYTES if k == "nl_proj" else SP_DIGIT_BYTES
+                b = 0.5 * (b - 16.0 * w.ngrid * w.nproj * w.ndom) + dig * w.ngrid * w.ndom
                 e.update({"bound": "hbm", "achieved": b / (avg * 1e-3) / 1e9, "unit": "GB/s", "peak": pk["hbm_gbs"],
                           "bytes_per_launch": b, "c64_equiv_tflops": f / (avg * 1e-3) / 1e12})
             elif f > 0:
@@ -659,11 +662,12 @@ def main():
             elif k in ("nl_back", "nl_proj") and nl_path == 1:
                 # int8-digit tcgen05 GEMMs (FP64 emulated): the digit products are cheap on the int8 tensor
                 # cores, so the kernels are bound by streaming Psi (read, + write for GEMM-2) and B's digits
-                # (6 x 128 B per grid point at nproj = 64: 0.75 of B's FP64 bytes) -- reported against HBM
+                # (GEMM-2: 6 x 128 B per grid point at nproj = 64, GEMM-1: 5 x 128 B) -- reported against HBM
                 # with the bytes the kernel must move, and the FP64-equivalent rate alongside
-                b = b - 16.0 * w.ngrid * w.nproj * w.ndom + I8_DIGIT_BYTES * w.ngrid * w.ndom
+                dig = G1_DIGIT_BYTES if k == "nl_proj" else I8_DIGIT_BYTES
+                b = b - 16.0 * w.ngrid * w.nproj * w.ndom + dig * w.ngrid * w.ndom
                 e.update({"bound": "hbm", "achieved": b / (avg * 1e-3) / 1e9, "unit": "GB/s", "peak": pk["hbm_gbs"],
-                          "path": "int8-digit tcgen05 (FP64 emulated, ~2^-40 product error)",
+                          "path": "int8-digit tcgen05 (FP64 emulated, ~2^-38 (GEMM-1) / ~2^-40 (GEMM-2) product error)",
                           "fp64_equiv_tflops": f / (avg * 1e-3) / 1e12,
                           "fp64_equiv_vs_dmma_peak": f / (avg * 1e-3) / 1e12 / pk["zgemm3m_tflops"]})
             elif f > 0:

@@ -34,7 +34,7 @@ size_t up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 struct Layout {
   size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage, cref,
-      epart, W, ones, x32, aseq, jseq, bsl, bsig, bsl1, bexp, colE, g1cnt, btil, qmat, zero, bslx, sigx;
+      epart, W, ones, x32, aseq, jseq, bsl, bsig, bsl1, bexp, colE, g1cnt, g1cs, btil, qmat, zero, bslx, sigx;
   int nref_cap;
   bool i8;  // GEMM-2 on the int8 tensor cores (nl_i8.cu): B digit tiles + row scales in the workspace
   bool fx;  // the first factor's GEMM-2 fused with the x pass (nl_fx.cu)
@@ -192,7 +192,8 @@ Layout layout(const Geometry& g, int num_sms, int nref_max, bool dense = false) 
   const int S = g.sp ? 4 : 6;  // int8 digits per operand
   L.bsl = L.i8 ? take(lfd::gemm2_i8_bytes(nd, g.ng, S)) : 0;
   L.bsig = L.i8 ? take(lfd::gemm2_i8_sig_bytes(nd, g.ng)) : 0;
-  L.bsl1 = L.i8 ? take(lfd::gemm1_i8_bytes(nd, g.ng, S)) : 0;
+  L.bsl1 = L.i8 ? take(lfd::gemm1_i8_bytes(nd, g.ng, g.sp)) : 0;
+  L.g1cs = L.i8 ? take(lfd::gemm1_i8_colsum_bytes(nd, L.nsplit_i8, np, g.sp)) : 0;
   L.bexp = L.i8 ? take((size_t)nd * np * sizeof(int)) : 0;
   L.colE = L.i8 ? take((size_t)nd * no * sizeof(int)) : 0;
   L.g1cnt = L.i8 ? take((size_t)nd * sizeof(int)) : 0;
@@ -552,7 +553,7 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr, bool
   if (c->L.i8 && c->colE_valid) {  // int8-digit tensor-core GEMM-1 (Psi's orbital exponents from the K_y K_z pass)
     lfd::Gemm1I8Args ai;
     ai.psi = c->psi; ai.bsl1 = c->at<int8_t>(c->L.bsl1); ai.bexp = c->at<int>(c->L.bexp);
-    ai.colE = c->at<int>(c->L.colE); ai.counter = c->at<int>(c->L.g1cnt);
+    ai.colE = c->at<int>(c->L.colE); ai.counter = c->at<int>(c->L.g1cnt); ai.colsum = c->at<int>(c->L.g1cs);
     ai.part = a1.part; ai.norms = a1.norms;
     ai.ndom = g.ndom; ai.nproj = g.nproj; ai.norb = g.norb; ai.nsplit = c->L.nsplit_i8;
     ai.ng = g.ng; ai.rps = c->L.rows_per_split_i8; ai.sp = g.sp;
@@ -1063,8 +1064,8 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
     });
     if (s2 != LFD_OK) return bail(s2);
     s2 = launch(c, LFD_K_NL_PROJ, "k_bslice1_i8", [&] {
-      return lfd::launch_bslice1_i8(c->proj, g.sp, g.ndom, g.nproj, g.ng, c->at<int>(L.bexp), c->at<int8_t>(L.bsl1),
-                                    c->stream);
+      return lfd::launch_bslice1_i8(c->proj, g.sp, g.ndom, g.nproj, g.ng, L.rows_per_split_i8, L.nsplit_i8,
+                                    c->at<int>(L.bexp), c->at<int8_t>(L.bsl1), c->at<int>(L.g1cs), c->stream);
     });
     if (s2 != LFD_OK) return bail(s2);
     e = cudaMemsetAsync(c->at<int>(L.colE), 0, sizeof(int) * g.ndom * g.norb, c->stream);

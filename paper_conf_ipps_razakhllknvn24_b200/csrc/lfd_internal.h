@@ -192,11 +192,12 @@ struct Gemm1I8Args {
   const int* bexp;      // [dom][nproj] B column exponents
   int* colE;            // [dom][norb] Psi orbital exponents (cleared by the last CTA)
   int* counter;         // [dom] CTA completion counters (zero between calls)
+  const int* colsum;    // [dom][nsplit][S][nproj] column sums of B's digits per split (launch_bslice1_i8)
   double2* part;        // [dom][nsplit][nproj][norb]
   double* norms;        // [dom][nsplit][norb]
   int ndom, nproj, norb, nsplit;
   long long ng, rps;
-  int sp = 0;  // the SP variant (complex64 Psi, 4 digits; colE from the SP z pass)
+  int sp = 0;  // the SP variant (complex64 Psi, 3 digits; colE from the SP z pass)
 };
 // The first nonlocal factor's GEMM-2 fused with the x pass of the local propagator (nl_fx.cu):
 //   Psi[x][yz] <- K_x (Phi . (n Psi + B C''))  along every x-line (y, z), int8-digit tcgen05 products.
@@ -212,10 +213,11 @@ cudaError_t launch_gemm2x_i8(const Geometry& g, const FxMaps* m, double2* psi, c
                              const double2* Cp, const double* sig, bool scaled, int num_sms, cudaStream_t st);
 cudaError_t gemm2x_set_attributes();
 
-size_t gemm1_i8_bytes(int ndom, long long ng, int S);
+size_t gemm1_i8_bytes(int ndom, long long ng, bool sp);
+size_t gemm1_i8_colsum_bytes(int ndom, int nsplit, int nproj, bool sp);
 long long gemm1_i8_rows_per_split(long long ng, int ndom, int num_sms);
-cudaError_t launch_bslice1_i8(const void* B, bool sp, int ndom, int nproj, long long ng, int* bexp, int8_t* out,
-                              cudaStream_t st);
+cudaError_t launch_bslice1_i8(const void* B, bool sp, int ndom, int nproj, long long ng, long long rps, int nsplit,
+                              int* bexp, int8_t* out, int* colsum, cudaStream_t st);
 cudaError_t launch_gemm1_i8(const Gemm1I8Args& a, cudaStream_t st);
 cudaError_t gemm_set_attributes();
 

@@ -339,20 +339,35 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
 
 // ================================================================================================
 // GEMM-1 (Eq. 7 / Eq. 9): split partials of C[u][s] = sum_r conj(B[r][u]) Psi[r][s]
-// and the column norms sum_r |Psi[r][s]|^2, with the same digit scheme.
+// and the column norms sum_r |Psi[r][s]|^2, on the int8 tensor cores with base-256 digits.
 //
-// Real form: D[m][u] = sum_k A[m][k] Bd[u][k] with m = 2s + c (M = 128), k = 2 rr + c' over the grid
-// rows of a 64-row block (K = 128 per block): A[2s][2rr] = Re Psi, A[2s][2rr+1] = Im Psi,
-// A[2s+1][2rr] = Im Psi, A[2s+1][2rr+1] = -Re Psi; Bd[u][2rr] = Re B, Bd[u][2rr+1] = Im B; then
-// D[2s][u] = Re C[u][s], D[2s+1][u] = Im C[u][s]. Scales are global over the domain, so the int32
-// accumulators run over a CTA's whole split (|P_d| <= 6 x 2 rows x 64 x 64 < 2^31 for <= 43,690 rows):
-// sigma_u = 2^e (max_r |Re B|, |Im B| of column u < 2^e, once at lfd_init) and tau_s = 2^(E_s - 1022)
-// with E_s the largest biased exponent of Re / Im Psi of orbital s, recorded by the K_y K_z pass that
-// wrote Psi (k_kin_yz, atomicMax) and cleared here by the last CTA. B's digits: once at lfd_init, per
-// 64-row block [6][64 u][128 B] in the SWIZZLE_128B image (one bulk copy). Psi's digits: per 32-row half
-// block, built by 16 worker warps straight into TMEM (the A operand, 6 x 16 columns), while the MMAs of
-// the previous half run (a single A buffer: the workers hold the next half's digits in registers until
-// the MMA warp releases it). TMEM: A 96 columns + 6 diagonal accumulators x 64 columns.
+// Real form: D[m][u] = sum_k A[m][k] Bd[u][k] with m = 2s + c (M = 128) and k over the grid rows of a 64-row
+// block in groups of 4 rows, k = 8 (rr / 4) + 4 c' + rr % 4 (K = 128 per block): A[2s][.] = (Re Psi, Im Psi)
+// of the group's 4 rows, A[2s+1][.] = (Im Psi, -Re Psi), Bd[u][.] = (Re B, Im B); then D[2s][u] = Re C[u][s],
+// D[2s+1][u] = Im C[u][s].
+//
+// Digits (S bytes per value: S = 5 for FP64 contexts, 3 for the SP variant). Psi, per orbital scale
+// tau_s = 2^(E_s - 1022) (every |Re|, |Im| < tau_s; E_s recorded by the K_y K_z pass that wrote Psi, k_kin_yz /
+// the SP z pass, integer max of the FP64 exponent fields, cleared here by the last CTA):
+// X = rint(x 2^(8S-2) / tau_s), written OFFSET-BINARY -- the S bytes u_k of X + 2^(8S-1) are unsigned digits
+// (tcgen05 kind::i8 takes u8 A x s8 B), and they are the low mantissa bytes of ONE DFMA against
+// 1.5 2^52 + 2^(8S-1) (the sum is an integer below 2^53, so the DFMA rounds to it exactly). B, per column scale
+// sigma_u (once at lfd_init): Y = rint(b 2^(8S-2) / sigma_u) as balanced base-256 digits d_i in [-128, 127]
+// (the bytes of Y + 128 (1 + 256 + ... + 256^(S-1)) minus 128, from one DFMA the same way). With a_k the
+// signed digits of X (a_k = u_k below the top byte, a_{S-1} = u_{S-1} - 128):
+//   sum_K X Y = sum_{k,i} 256^(k+i) sum_K u_k d_i  -  128 sum_i 256^(S-1+i) sum_K d_i,
+// the second term from the column sums of B's digits over the CTA's rows (exact, once at lfd_init). The pairs
+// with k + i >= S - 2 are kept (19 of 25 for S = 5), grouped by diagonal d = k + i into S + 1 exact int32
+// accumulators in TMEM (|P_d| <= S x 2 rps x 255 x 128 < 2^31 for rps <= 6144); the dropped pairs and the
+// digit remainders are ~2^-38 relative to sigma_u tau_s (S = 5; the old base-128 scheme: ~2^-40), so the
+// update B C'' stays within ~1e-15 of Psi per factor. C = sigma_u tau_s 2^-12 sum_d 256^(d-2S+2) (P_d - corr_d).
+//
+// Kernel: B's digits per 64-row block [S][64 u][128 B] in the SWIZZLE_128B image (one bulk copy, 2-stage
+// ring); Psi rows staged per 16-row quarter block (bulk copies, 6-slot ring). 16 worker warps: lane (m, h)
+// loads its orbital's two components of 4 grid rows, makes their digits (2 DFMA per row: digits, norm) and
+// transposes them with byte permutes into the A words of its TMEM lane (2 per digit), into one of NBuf A
+// buffers; one thread issues the quarter block's MMAs (S = 5: 7 MMAs of N = 64 w, w <= 4 consecutive
+// diagonals each) as soon as its buffer is full. TMEM: NBuf x 8S A columns + (S + 1) x 64 accumulators.
 // ================================================================================================
 constexpr int kG1Rows = 64;                        // grid rows per B-digit block (K = 128 bytes)
 constexpr int kG1Half = 16;                        // grid rows per A (Psi-digit) quarter block (K = 32 bytes)
@@ -362,23 +377,55 @@ constexpr int kG1PsiSlots = 6;                     // Psi quarter-block ring
 constexpr int kG1Workers = 16;                     // worker warps: 4 lane quarters x 4 row groups
 constexpr int kG1Threads = (kG1Workers + 2) * 32;  // + producer + MMA
 constexpr int kG1WProd = kG1Workers, kG1WMma = kG1Workers + 1;
-// shapes depending on the digit count S and Psi's element type T (see I8G2)
+constexpr long long kG1MaxRps = 6144;              // int32 diagonals: S x 2 rps x 255 x 128 < 2^31 (S <= 5)
+__host__ __device__ constexpr int g1_digits(bool sp) { return sp ? 3 : 5; }
+// shapes depending on the digit count S and Psi's element type T
 template <int S, class T>
 struct I8G1 {
-  static constexpr int BlkB = S * kG1SliceB;                     // 48 KB (S = 6)
-  static constexpr int PsiB = kG1Half * 64 * (int)sizeof(T);     // Psi rows of a quarter block (norb <= 64)
+  static constexpr int Acc = S + 1;                           // diagonals d = S-2 .. 2S-2
+  static constexpr int NBuf = S >= 5 ? 3 : 4;                 // TMEM A buffers
+  static constexpr int ABuf = S * 8;                          // TMEM columns of one A buffer (K = 32 bytes)
+  static constexpr int BlkB = S * kG1SliceB;                  // 40 KB (S = 5)
+  static constexpr int PsiB = kG1Half * 64 * (int)sizeof(T);  // Psi rows of a quarter block (norb <= 64)
   static constexpr int Smem = kG1Stages * BlkB + kG1PsiSlots * PsiB + 1024;
-  static constexpr int ABuf = S * 8;                             // TMEM columns of one A buffer (K = 32 bytes)
-  static constexpr int ACols = 2 * ABuf;                         // double-buffered A
+  static_assert(NBuf * ABuf + 64 * Acc <= 512, "TMEM columns");
 };
-// s32 <- s8 x s8, both K-major, M = 128, N = n (a multiple of 64 here)
+// s32 <- u8 (A, Psi digits) x s8 (B digits), both K-major, M = 128, N = n (a multiple of 64 here)
 __host__ __device__ constexpr uint32_t g1_idesc(int n) {
-  return (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+  return (2u << 4) | (0u << 7) | (1u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
 }
-constexpr uint32_t kG1Idesc = g1_idesc(64);
+// 1.5 2^52 + the digit offset: the low 8S mantissa bits of fma(x, sc, M) are the integer rint(x sc) + offset
+template <int S>
+__host__ __device__ constexpr double g1_madd_a() { return 6755399441055744.0 + (double)(1LL << (8 * S - 1)); }
+template <int S>
+__host__ __device__ constexpr double g1_madd_b() {  // offset 128 (1 + 256 + ... + 256^(S-1))
+  long long c = 0;
+  for (int k = 0; k < S; ++k) c = (c << 8) | 128;
+  return 6755399441055744.0 + (double)c;
+}
+
+// the S low bytes of rint(v[q] sc) + offset (q = 0..3) transposed: out[k] = byte k of the four values
+template <int S>
+__device__ __forceinline__ void g1_bytes(const double v[4], double sc, double madd, uint32_t out[S]) {
+  uint32_t lo[4], hi[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const long long b = __double_as_longlong(fma(v[q], sc, madd));
+    lo[q] = (uint32_t)b;
+    hi[q] = (uint32_t)(b >> 32);
+  }
+  const uint32_t a = __byte_perm(lo[0], lo[1], 0x5140), b = __byte_perm(lo[0], lo[1], 0x7362);
+  const uint32_t c = __byte_perm(lo[2], lo[3], 0x5140), d = __byte_perm(lo[2], lo[3], 0x7362);
+  out[0] = __byte_perm(a, c, 0x5410);
+  out[1] = __byte_perm(a, c, 0x7632);
+  out[2] = __byte_perm(b, d, 0x5410);
+  if constexpr (S >= 4) out[3] = __byte_perm(b, d, 0x7632);
+  if constexpr (S >= 5) out[4] = __byte_perm(__byte_perm(hi[0], hi[1], 0x0040), __byte_perm(hi[2], hi[3], 0x0040), 0x5410);
+  (void)hi;
+}
 
 __device__ __forceinline__ void umma_g1_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t accumulate,
-                                           uint32_t idesc = kG1Idesc) {
+                                           uint32_t idesc) {
   asm volatile(
       "{\n.reg .pred p, e;\nelect.sync _|e, 0xffffffff;\nsetp.ne.b32 p, %4, 0;\n"
       "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
@@ -387,24 +434,31 @@ __device__ __forceinline__ void umma_g1_ts(uint32_t tmem_d, uint32_t tmem_a, uin
 __device__ __forceinline__ void tmem_st2(uint32_t taddr, const uint32_t v[2]) {
   asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0], {%1,%2};" ::"r"(taddr), "r"(v[0]), "r"(v[1]) : "memory");
 }
-__device__ __forceinline__ void tmem_st4(uint32_t taddr, const uint32_t v[4]) {
-  asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1,%2,%3,%4};" ::"r"(taddr), "r"(v[0]), "r"(v[1]),
-               "r"(v[2]), "r"(v[3])
-               : "memory");
-}
 
-// The wide-N MMA schedule of one quarter block (see k_gemm1_i8): for each Psi digit j, the B digits
-// i = 1 .. 7 - j in chunks of at most W consecutive slices, one MMA of N = 64 w per chunk
-template <int W, int S>
-__device__ __forceinline__ void g1_wide_mmas(uint32_t tacc, uint32_t ta, uint64_t db0, int kq, bool first) {
+// The MMAs of one quarter block: entry j = (A digit k, first B digit i0, width w) is one MMA of N = 64 w into the
+// consecutive diagonals k + i0 .. k + i0 + w - 1 (B's digit slices i0 .. are consecutive 64-row K-major tiles,
+// the diagonals consecutive 64-column TMEM blocks). The first two entries cover every diagonal exactly once
+// (accumulate = 0 at a split's first quarter block); all pairs k + i >= S - 2 appear once.
+template <int S>
+__host__ __device__ constexpr int g1_sched_n() { return S == 5 ? 7 : 4; }
+template <int S>
+__host__ __device__ constexpr int g1_sched(int j) {  // k | i0 << 4 | w << 8
+  if (S == 5) {
+    constexpr int t[7] = {3 | 0 << 4 | 4 << 8, 4 | 3 << 4 | 2 << 8, 3 | 4 << 4 | 1 << 8, 4 | 0 << 4 | 3 << 8,
+                          0 | 3 << 4 | 2 << 8, 1 | 2 << 4 | 3 << 8, 2 | 1 << 4 | 4 << 8};
+    return t[j];
+  }
+  constexpr int t[4] = {1 | 0 << 4 | 3 << 8, 2 | 2 << 4 | 1 << 8, 2 | 0 << 4 | 2 << 8, 0 | 1 << 4 | 2 << 8};
+  return t[j];
+}
+template <int S>
+__device__ __forceinline__ void g1_mmas(uint32_t tacc, uint32_t ta, uint64_t db0, int kq, bool first) {
 #pragma unroll
-  for (int j = 1; j <= S; ++j) {
-#pragma unroll
-    for (int i = 1; i <= S + 1 - j; i += W) {
-      const int w = (S + 2 - j - i) < W ? (S + 2 - j - i) : W;
-      umma_g1_ts(tacc + (i + j - 2) * 64, ta + (j - 1) * 8, db0 + (uint64_t)(((i - 1) * kG1SliceB + kq * 32) >> 4),
-                 (first && j == 1) ? 0u : 1u, g1_idesc(64 * w));
-    }
+  for (int j = 0; j < g1_sched_n<S>(); ++j) {
+    const int e = g1_sched<S>(j);
+    const int k = e & 15, i0 = (e >> 4) & 15, w = e >> 8;
+    umma_g1_ts(tacc + (k + i0 - (S - 2)) * 64, ta + k * 8, db0 + (uint64_t)((i0 * kG1SliceB + kq * 32) >> 4),
+               (first && j < 2) ? 0u : 1u, g1_idesc(64 * w));
   }
 }
 
@@ -431,11 +485,12 @@ __global__ void __launch_bounds__(256) k_bexp1_i8(const T* __restrict__ B, int n
     if (sm[u] > 0) atomicMax(bexp + (long long)dom * nproj + u, sm[u]);
 }
 
-// B's GEMM-1 digits: warp per (64-row block, u); lane l holds rows 2l, 2l+1 (k = 4l .. 4l+3)
+// B's GEMM-1 digits: warp per (64-row block, u); lane l holds K bytes 4l .. 4l+3, i.e. component c' = l & 1 of
+// rows 4 (l >> 1) .. + 3. Also the per-split column sums of each digit (integer atomics: order-independent).
 template <class T, int S>
 __global__ void __launch_bounds__(256) k_bslice1_i8(const T* __restrict__ B, int nproj, long long ng,
-                                                    long long nblk, const int* __restrict__ bexp,
-                                                    int8_t* __restrict__ out) {
+                                                    long long nblk, const int* __restrict__ bexp, int blk_per_split,
+                                                    int nsplit, int8_t* __restrict__ out, int* __restrict__ colsum) {
   pdl_wait();
   pdl_trigger();
   const int dom = blockIdx.y, lane = threadIdx.x & 31;
@@ -446,16 +501,34 @@ __global__ void __launch_bounds__(256) k_bslice1_i8(const T* __restrict__ B, int
   double v[4] = {0.0, 0.0, 0.0, 0.0};
   const int E = u < nproj ? bexp[(long long)dom * nproj + u] : 0;
   if (u < nproj) {
-    const long long r = blk * kG1Rows + 2 * lane;
     const T* col = B + (long long)dom * ng * nproj + u;
-    if (r < ng) { const T a = col[r * nproj]; v[0] = a.x; v[1] = a.y; }
-    if (r + 1 < ng) { const T a = col[(r + 1) * nproj]; v[2] = a.x; v[3] = a.y; }
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {
+      const long long r = blk * kG1Rows + 4 * (lane >> 1) + t;
+      if (r < ng) {
+        const T a = col[r * nproj];
+        v[t] = (lane & 1) ? a.y : a.x;
+      }
+    }
   }
   uint32_t d[S];
-  digits4<S>(v, E - 1022, E == 0, d);  // |v| < 2^(E - 1022)
+  g1_bytes<S>(v, E == 0 ? 0.0 : ldexp(1.0, 8 * S - 2 - (E - 1022)), g1_madd_b<S>(), d);  // |Y| <= 2^(8S-2)
   int8_t* tb = out + ((long long)dom * nblk + blk) * (S * kG1SliceB);
 #pragma unroll
-  for (int i = 0; i < S; ++i) *reinterpret_cast<uint32_t*>(tb + i * kG1SliceB + sw128(u, 4 * lane)) = d[i];
+  for (int i = 0; i < S; ++i) {
+    d[i] ^= 0x80808080u;  // byte f -> digit f - 128 (balanced)
+    *reinterpret_cast<uint32_t*>(tb + i * kG1SliceB + sw128(u, 4 * lane)) = d[i];
+  }
+  if (u < nproj) {
+    const int split = (int)(blk / blk_per_split);
+#pragma unroll
+    for (int i = 0; i < S; ++i) {
+      int s = __dp4a((int)d[i], 0x01010101, 0);  // the 4 signed digits
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+      if (lane == 0 && s != 0) atomicAdd(colsum + (((long long)dom * nsplit + split) * S + i) * nproj + u, s);
+    }
+  }
 }
 
 // grid (splits, ndom); CTA = one split of rps rows (a multiple of 64)
@@ -463,16 +536,16 @@ template <class T, int S>
 __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   using G = I8G1<S, T>;
   using R = decltype(T::x);
-  constexpr int kG1BlkB = G::BlkB, kG1PsiB = G::PsiB, kG1ABuf = G::ABuf, kG1ACols = G::ACols;
+  constexpr int kG1BlkB = G::BlkB, kG1PsiB = G::PsiB, kG1ABuf = G::ABuf, kNBuf = G::NBuf;
   // programmatic dependent launch: set-up and the first B-digit blocks (constant since lfd_init) overlap the
   // previous kernel; the Psi loads and everything reading colE / writing the partials wait for it
   pdl_trigger();
   extern __shared__ __align__(1024) unsigned char dsm_raw[];
   unsigned char* dsm = dsm_raw + ((1024u - (smem_addr(dsm_raw) & 1023u)) & 1023u);
-  unsigned char* Bsm = dsm;                            // [stages][6][64 u][128 B] swizzled B digits
-  unsigned char* Psm = Bsm + kG1Stages * kG1BlkB;      // [slots][32 rows][norb] complex
+  unsigned char* Bsm = dsm;                            // [stages][S][64 u][128 B] swizzled B digits
+  unsigned char* Psm = Bsm + kG1Stages * kG1BlkB;      // [slots][16 rows][norb] complex
   __shared__ __align__(8) uint64_t bfull[kG1Stages], bempty[kG1Stages], pfull[kG1PsiSlots], pempty[kG1PsiSlots];
-  __shared__ __align__(8) uint64_t afull[2], afree[2], done;
+  __shared__ __align__(8) uint64_t afull[kNBuf], afree[kNBuf], done;
   __shared__ uint32_t tmem_base_sh;
   __shared__ double nsum[4][64];
   __shared__ int last_sh;
@@ -487,14 +560,14 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   const int nhalf = (int)((r1 - r0 + kG1Half - 1) / kG1Half);  // quarter blocks of this split
   const int rowb = norb * (int)sizeof(T);
 
-  if (warp == kG1WMma) {  // TMEM: A (Psi digits, 2 x 8 S columns) + S diagonal accumulators x 64 columns
+  if (warp == kG1WMma) {  // TMEM: NBuf A buffers (Psi digits, 8 S columns each) + S + 1 accumulators x 64 columns
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_addr(&tmem_base_sh)));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   if (tid == 0) {
     for (int s = 0; s < kG1Stages; ++s) { mbar_init(&bfull[s], 1); mbar_init(&bempty[s], 1); }
     for (int s = 0; s < kG1PsiSlots; ++s) { mbar_init(&pfull[s], 1); mbar_init(&pempty[s], kG1Workers); }
-    for (int b = 0; b < 2; ++b) { mbar_init(&afull[b], kG1Workers); mbar_init(&afree[b], 1); }
+    for (int b = 0; b < kNBuf; ++b) { mbar_init(&afull[b], kG1Workers); mbar_init(&afree[b], 1); }
     mbar_init(&done, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -502,9 +575,9 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
-  const uint32_t tacc = tmem + kG1ACols;
+  const uint32_t tacc = tmem + kNBuf * kG1ABuf;
 
-  if (warp == kG1WProd) {  // producer: B-digit blocks and Psi half blocks, in the order the MMAs use them
+  if (warp == kG1WProd) {  // producer: B-digit blocks and Psi quarter blocks, in the order the MMAs use them
     if (lane == 0) {
       const int8_t* src = p.bsl1 + (long long)dom * nblk * kG1BlkB;
       const T* prow = reinterpret_cast<const T*>(p.psi) + (long long)dom * ng * norb;
@@ -531,98 +604,93 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   } else if (warp == kG1WMma) {  // MMA issuer
     {  // the whole warp runs the loop (warp-uniform values stay in uniform registers); one elected lane issues
       const uint32_t bbase = smem_addr(Bsm);
-      for (int g = 0; g < nhalf; ++g) {
-        const int b = g >> 2, s = b % kG1Stages, kq = g & 3, ab = g & 1;
+      for (int g = 0, ab = 0, aph = 0; g < nhalf; ++g) {  // ab = g % NBuf, aph = (g / NBuf) & 1
+        const int b = g >> 2, s = b % kG1Stages, kq = g & 3;
         if (kq == 0) mbar_wait(&bfull[s], (uint32_t)((b / kG1Stages) & 1));
-        mbar_wait(&afull[ab], (uint32_t)((g >> 1) & 1));
+        mbar_wait(&afull[ab], (uint32_t)aph);
         tc_fence_after();
-        const uint64_t db0 = umma_desc_sw128(bbase + s * kG1BlkB);
-        // B's digit slices i .. i + w - 1 are consecutive 64-row SWIZZLE_128B tiles (8 KB each), i.e. one
-        // K-major tile of 64 w rows, and the diagonal accumulators d = i + j .. i + j + w - 1 are consecutive
-        // 64-column TMEM blocks: one MMA of N = 64 w (w <= 3) computes the w digit pairs (i .. i + w - 1, j)
-        // straight into their diagonals (9 MMAs per quarter block instead of 21). The j = 1 MMAs touch every
-        // diagonal first (accumulate = 0 at g = 0).
-        g1_wide_mmas<3, S>(tacc, tmem + ab * kG1ABuf, db0, kq, g == 0);
-        umma_commit(&afree[ab]);                      // A buffer ab may take quarter block g + 2
+        g1_mmas<S>(tacc, tmem + ab * kG1ABuf, umma_desc_sw128(bbase + s * kG1BlkB), kq, g == 0);
+        umma_commit(&afree[ab]);  // A buffer ab may take quarter block g + NBuf
         if (kq == 3 || g + 1 == nhalf) umma_commit(&bempty[s]);
+        if (++ab == kNBuf) { ab = 0; aph ^= 1; }
       }
       umma_commit(&done);
     }
   } else {  // workers: Psi digits into TMEM, column norms; at the end the accumulators into FP64 partials
     pdl_wait();
-    const int q = warp & 3, h = warp >> 2;    // lane quarter, row group (8 rows of each half block)
+    const int q = warp & 3, h = warp >> 2;    // lane quarter, row group (4 rows of each quarter block)
     const int m = 32 * q + lane, sIdx = m >> 1, cm = m & 1;
     const bool sv = sIdx < norb;
-    const uint32_t nmask = cm ? 0xffffffffu : 0u;
     const int E = sv ? p.colE[(long long)dom * norb + sIdx] : 0;
-    const bool zc = E == 0;                   // an all-zero orbital (or none): zero digits
-    const double sc41 = zc ? 0.0 : ldexp(1.0, 7 * S - 1 - (E - 1022));  // x 2^(7S-1) / tau_s
+    const bool zc = E == 0;                   // an all-zero orbital (or none): tau = 0
+    const double sc = zc ? 0.0 : ldexp(1.0, 8 * S - 2 - (E - 1022));  // x 2^(8S-2) / tau_s
+    const double sc2 = cm ? -sc : sc;         // the odd row's second component is -Re
+    constexpr double kMA = g1_madd_a<S>();
     double nrm = 0.0;
     const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
-    for (int g = 0, s = 0, ph = 0; g < nhalf; ++g) {  // s = g % kG1PsiSlots, ph = (g / kG1PsiSlots) & 1
-      const int ab = g & 1;
+    for (int g = 0, s = 0, ph = 0, ab = 0, aph = 0; g < nhalf; ++g) {
       mbar_wait(&pfull[s], (uint32_t)ph);
       const long long ra = r0 + (long long)g * kG1Half;
-      // this lane's component of Psi[row][sIdx] (Re for cm = 0, Im for cm = 1): 8-byte loads, 2 norb per row
-      const R* P = reinterpret_cast<const R*>(Psm + s * kG1PsiB) + 2 * sIdx + cm;
-      // each lane digitises its own component only (even lane m = 2s: Re, odd lane: Im) of its 4 rows
-      // (4h .. 4h + 3 of the quarter block), in integer arithmetic (digits_i64), and the lane pair exchanges
-      // them: row 2s of A takes (Re, Im) per grid row, row 2s+1 takes (Im, -Re) (bytewise negated digits:
-      // still an exact decomposition)
-      double v[4];
+      // this lane's components of Psi[row][sIdx] for rows 4h .. 4h+3: (Re, Im) for the even row m = 2s, (Im, Re)
+      // for the odd row (its Re enters negated: sc2)
+      const R* P = reinterpret_cast<const R*>(Psm + s * kG1PsiB) + 2 * sIdx + 8 * h * norb;
+      double v1[4], v2[4];
       if (sv && ra + 4 * h + 4 <= r1) {  // all 4 rows present (every quarter block but a split's ragged last)
 #pragma unroll
-        for (int t = 0; t < 4; ++t) v[t] = P[(4 * h + t) * 2 * norb];
+        for (int t = 0; t < 4; ++t) { v1[t] = P[t * 2 * norb + cm]; v2[t] = P[t * 2 * norb + 1 - cm]; }
       } else {
 #pragma unroll
-        for (int t = 0; t < 4; ++t) v[t] = (sv && ra + 4 * h + t < r1) ? P[(4 * h + t) * 2 * norb] : 0.0;
+        for (int t = 0; t < 4; ++t) {
+          const bool ok = sv && ra + 4 * h + t < r1;
+          v1[t] = ok ? P[t * 2 * norb + cm] : 0.0;
+          v2[t] = ok ? P[t * 2 * norb + 1 - cm] : 0.0;
+        }
       }
 #pragma unroll
-      for (int t = 0; t < 4; ++t) nrm = fma(v[t], v[t], nrm);  // absent rows add +0 exactly
-      uint32_t own[S];
-      digits_x<S>(v, sc41, own);
-      uint32_t dg[S][2];
-#pragma unroll
-      for (int i = 0; i < S; ++i) {
-        const uint32_t mine = own[i];
-        const uint32_t other = __shfl_xor_sync(0xffffffffu, mine, 1);
-        // bytes t = 0..3 are rows 4h + t; A word w (K bytes 8h + 4w ..) holds rows (2w, 2w+1) as
-        // [c'=0, c'=1, c'=0, c'=1]; even lane: c'=0 own (Re), c'=1 other (Im); odd lane: own (Im), -other
-        // odd lane: bytewise -other without predication: bytes b in [-64, 64] -> x = b + 128 in [64, 192],
-        // (x ^ 0xff) + 1 = 256 - x has no carry between bytes, ^ 0x80 gives -b
-        const uint32_t b = (((other ^ 0x80808080u ^ nmask) + (nmask & 0x01010101u)) ^ 0x80808080u);
-        dg[i][0] = __byte_perm(mine, b, 0x5140);  // [a0, b0, a1, b1]
-        dg[i][1] = __byte_perm(mine, b, 0x7362);  // [a2, b2, a3, b3]
-      }
-      // this warp is done with the Psi rows (its loads have returned: nrm depends on every one, lfd_tma.cuh)
-      mbar_release(&pempty[s], nrm, lane == 0);
-      if (g >= 2) mbar_wait(&afree[ab], (uint32_t)(((g >> 1) - 1) & 1));  // MMAs of block g - 2 are done with it
+      for (int t = 0; t < 4; ++t) nrm = fma(v1[t], v1[t], fma(v2[t], v2[t], nrm));  // absent rows add +0
+      uint32_t d1[S], d2[S];
+      g1_bytes<S>(v1, sc, kMA, d1);
+      g1_bytes<S>(v2, sc2, kMA, d2);
+      // this warp is done with the Psi rows (its loads have returned: lfd_tma.cuh)
+      mbar_release(&pempty[s], (v1[0] + v1[3]) + (v2[0] + v2[3]) + (v1[1] + v1[2]) + (v2[1] + v2[2]), lane == 0);
+      if (g >= kNBuf) mbar_wait(&afree[ab], (uint32_t)(aph ^ 1));  // the MMAs of quarter block g - NBuf are done
       tc_fence_after();
 #pragma unroll
-      for (int i = 0; i < S; ++i) tmem_st2(trow + ab * kG1ABuf + i * 8 + 2 * h, dg[i]);
+      for (int k = 0; k < S; ++k) {
+        const uint32_t w2[2] = {d1[k], d2[k]};
+        tmem_st2(trow + ab * kG1ABuf + k * 8 + 2 * h, w2);
+      }
       asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&afull[ab]);
       if (++s == kG1PsiSlots) { s = 0; ph ^= 1; }
+      if (++ab == kNBuf) { ab = 0; aph ^= 1; }
     }
-    // column norms: Re^2 (even lane) + Im^2 (odd lane), then a fixed-order sum over the 4 row groups
-    nrm += __shfl_xor_sync(0xffffffffu, nrm, 1);
+    // column norms: both lanes of a pair hold the orbital's full |Psi|^2; the even lane writes it (fixed-order
+    // sum over the 4 row groups below)
     if (!cm && sv) nsum[h][sIdx] = nrm;
     mbar_wait(&done, 0);
     tc_fence_after();
     // accumulators: warp (q, h) reads lanes 32 q .. (rows m) and columns u = 16 h .. 16 h + 15
+    const int* cs = p.colsum + ((long long)dom * p.nsplit + split) * S * nproj;  // [S][nproj]
     double cacc[16];
 #pragma unroll
     for (int c = 0; c < 16; ++c) cacc[c] = 0.0;
 #pragma unroll 1
-    for (int d = 2; d <= S + 1; ++d) {
+    for (int d = S - 2; d <= 2 * S - 2; ++d) {
       int32_t a[16];
-      tmem_ld16(tacc + (d - 2) * 64 + ((uint32_t)(32 * q) << 16) + 16 * h, a);
+      tmem_ld16(tacc + (d - (S - 2)) * 64 + ((uint32_t)(32 * q) << 16) + 16 * h, a);
       tmem_wait_ld();
-      const double wd = ldexp(1.0, -7 * (d - 2));
+      const double wd = ldexp(1.0, -8 * (2 * S - 2 - d));
+      const int i = d - (S - 1);  // the pair (S-1, i) carries the offset of the top A digit
 #pragma unroll
-      for (int c = 0; c < 16; ++c) cacc[c] = fma(i2d(a[c]), wd, cacc[c]);
+      for (int c = 0; c < 16; ++c) {
+        const int u = 16 * h + c;
+        double pd = i2d(a[c]);
+        if (i >= 0 && u < nproj) pd -= 128.0 * (double)cs[i * nproj + u];
+        cacc[c] = fma(pd, wd, cacc[c]);
+      }
     }
     // C[u][s] = sigma_u tau_s 2^-12 cacc; m = 2 s + cm -> Re (cm 0) / Im (cm 1)
     const double tau = zc ? 0.0 : ldexp(1.0, E - 1022 - 12);
@@ -658,39 +726,44 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
   }
 }
 
-size_t gemm1_i8_bytes(int ndom, long long ng, int S) {
+size_t gemm1_i8_bytes(int ndom, long long ng, bool sp) {
   const long long nblk = (ng + kG1Rows - 1) / kG1Rows;
-  return (size_t)ndom * nblk * S * kG1SliceB;
+  return (size_t)ndom * nblk * g1_digits(sp) * kG1SliceB;
+}
+size_t gemm1_i8_colsum_bytes(int ndom, int nsplit, int nproj, bool sp) {
+  return (size_t)ndom * nsplit * g1_digits(sp) * nproj * sizeof(int);
 }
 long long gemm1_i8_rows_per_split(long long ng, int ndom, int num_sms) {
   int cpd = num_sms / ndom;
   if (cpd < 1) cpd = 1;
   long long rps = (ng + cpd - 1) / cpd;
   rps = (rps + kG1Rows - 1) / kG1Rows * kG1Rows;
-  if (rps > 32768) rps = 32768;  // int32 accumulators: 6 x 2 rps x 64 x 64 < 2^31
+  if (rps > kG1MaxRps) rps = kG1MaxRps;
   return rps;
 }
-cudaError_t launch_bslice1_i8(const void* B, bool sp, int ndom, int nproj, long long ng, int* bexp, int8_t* out,
-                              cudaStream_t st) {
+cudaError_t launch_bslice1_i8(const void* B, bool sp, int ndom, int nproj, long long ng, long long rps, int nsplit,
+                              int* bexp, int8_t* out, int* colsum, cudaStream_t st) {
   cudaError_t e = cudaMemsetAsync(bexp, 0, sizeof(int) * ndom * nproj, st);
+  if (e == cudaSuccess) e = cudaMemsetAsync(colsum, 0, gemm1_i8_colsum_bytes(ndom, nsplit, nproj, sp), st);
   if (e != cudaSuccess) return e;
   const long long nblk = (ng + kG1Rows - 1) / kG1Rows;
+  const int bps = (int)(rps / kG1Rows);
   dim3 grid((unsigned)((nblk * 64 + 7) / 8), ndom);
   if (sp) {
     const float2* b = static_cast<const float2*>(B);
     launch_k(k_bexp1_i8<float2>, dim3(296, ndom), 256, 0, st, b, nproj, ng, bexp);
-    launch_k(k_bslice1_i8<float2, 4>, grid, 256, 0, st, b, nproj, ng, nblk, (const int*)bexp, out);
+    launch_k(k_bslice1_i8<float2, 3>, grid, 256, 0, st, b, nproj, ng, nblk, (const int*)bexp, bps, nsplit, out, colsum);
   } else {
     const double2* b = static_cast<const double2*>(B);
     launch_k(k_bexp1_i8<double2>, dim3(296, ndom), 256, 0, st, b, nproj, ng, bexp);
-    launch_k(k_bslice1_i8<double2, 6>, grid, 256, 0, st, b, nproj, ng, nblk, (const int*)bexp, out);
+    launch_k(k_bslice1_i8<double2, 5>, grid, 256, 0, st, b, nproj, ng, nblk, (const int*)bexp, bps, nsplit, out, colsum);
   }
   return cudaGetLastError();
 }
 cudaError_t launch_gemm1_i8(const Gemm1I8Args& a, cudaStream_t st) {
   dim3 grid(a.nsplit, a.ndom);
-  if (a.sp) launch_k(k_gemm1_i8<float2, 4>, grid, kG1Threads, I8G1<4, float2>::Smem, st, a);
-  else launch_k(k_gemm1_i8<double2, 6>, grid, kG1Threads, I8G1<6, double2>::Smem, st, a);
+  if (a.sp) launch_k(k_gemm1_i8<float2, 3>, grid, kG1Threads, I8G1<3, float2>::Smem, st, a);
+  else launch_k(k_gemm1_i8<double2, 5>, grid, kG1Threads, I8G1<5, double2>::Smem, st, a);
   return cudaGetLastError();
 }
 
@@ -739,8 +812,8 @@ cudaError_t gemm_i8_set_attributes() {
   LFD_ATTR((k_gemm2_i8<true, double2, 6>), (I8G2<6, double2>::Smem));
   LFD_ATTR((k_gemm2_i8<false, float2, 4>), (I8G2<4, float2>::Smem));
   LFD_ATTR((k_gemm2_i8<true, float2, 4>), (I8G2<4, float2>::Smem));
-  LFD_ATTR((k_gemm1_i8<double2, 6>), (I8G1<6, double2>::Smem));
-  LFD_ATTR((k_gemm1_i8<float2, 4>), (I8G1<4, float2>::Smem));
+  LFD_ATTR((k_gemm1_i8<double2, 5>), (I8G1<5, double2>::Smem));
+  LFD_ATTR((k_gemm1_i8<float2, 3>), (I8G1<3, float2>::Smem));
 #undef LFD_ATTR
   return cudaSuccess;
 }
