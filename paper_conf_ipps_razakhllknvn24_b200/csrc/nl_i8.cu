@@ -39,8 +39,21 @@
 #include "lfd_tma.cuh"
 
 #include <type_traits>
+#ifdef LFD_G1_TIMING
+#include <cstdio>
+#endif
 
 namespace lfd {
+
+// Role-wait instrumentation of k_gemm1_i8 for A/B experiments only (compiled in with -DLFD_G1_TIMING; printf
+// from two CTAs)
+#ifdef LFD_G1_TIMING
+#define G1_T0(v) long long v = clock64()
+#define G1_ACC(acc, v) acc += clock64() - v
+#else
+#define G1_T0(v)
+#define G1_ACC(acc, v)
+#endif
 
 constexpr int kI8NT = 64;                           // grid points per tile (MMA N)
 constexpr int kI8K = 128;                           // bytes per digit row: K = 2 nproj padded to 128
@@ -587,27 +600,45 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
         tma_row(Bsm + b * kG1BlkB, src + (r0 / kG1Rows + b) * kG1BlkB, kG1BlkB, &bfull[b]);
       }
       pdl_wait();
+      long long w_be = 0, w_pe = 0;
+      G1_T0(t_all);
       for (int g = 0; g < nhalf; ++g) {
         if ((g & 3) == 0 && (g >> 2) >= kG1Stages) {
           const int b = g >> 2, s = b % kG1Stages;
+          G1_T0(c0);
           mbar_wait(&bempty[s], (uint32_t)(((b / kG1Stages) - 1) & 1));
+          G1_ACC(w_be, c0);
           mbar_expect_tx(&bfull[s], kG1BlkB);
           tma_row(Bsm + s * kG1BlkB, src + (r0 / kG1Rows + b) * kG1BlkB, kG1BlkB, &bfull[s]);
         }
         const int s = g % kG1PsiSlots;
+        G1_T0(c1);
         if (g >= kG1PsiSlots) mbar_wait(&pempty[s], (uint32_t)(((g / kG1PsiSlots) - 1) & 1));
+        G1_ACC(w_pe, c1);
         const long long ra = r0 + (long long)g * kG1Half;
         const long long nr = (r1 - ra) < kG1Half ? (r1 - ra) : kG1Half;
         tma_row8(Psm + s * kG1PsiB, prow + ra * norb, (uint32_t)(nr * rowb), &pfull[s], 0);
       }
+#ifdef LFD_G1_TIMING
+      if (blockIdx.x == 0 || blockIdx.x == 100)
+        printf("g1 cta %d prod: total %lld wait-bempty %lld wait-pempty %lld blocks %d\n", blockIdx.x,
+               clock64() - t_all, w_be, w_pe, nhalf);
+#endif
+      (void)w_be; (void)w_pe;
     }
   } else if (warp == kG1WMma) {  // MMA issuer
     {  // the whole warp runs the loop (warp-uniform values stay in uniform registers); one elected lane issues
       const uint32_t bbase = smem_addr(Bsm);
+      long long w_bf = 0, w_af = 0;
+      G1_T0(t_all);
       for (int g = 0, ab = 0, aph = 0; g < nhalf; ++g) {  // ab = g % NBuf, aph = (g / NBuf) & 1
         const int b = g >> 2, s = b % kG1Stages, kq = g & 3;
+        G1_T0(c0);
         if (kq == 0) mbar_wait(&bfull[s], (uint32_t)((b / kG1Stages) & 1));
+        G1_ACC(w_bf, c0);
+        G1_T0(c1);
         mbar_wait(&afull[ab], (uint32_t)aph);
+        G1_ACC(w_af, c1);
         tc_fence_after();
         g1_mmas<S>(tacc, tmem + ab * kG1ABuf, umma_desc_sw128(bbase + s * kG1BlkB), kq, g == 0);
         umma_commit(&afree[ab]);  // A buffer ab may take quarter block g + NBuf
@@ -615,6 +646,11 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
         if (++ab == kNBuf) { ab = 0; aph ^= 1; }
       }
       umma_commit(&done);
+#ifdef LFD_G1_TIMING
+      if (lane == 0 && (blockIdx.x == 0 || blockIdx.x == 100))
+        printf("g1 cta %d mma: total %lld wait-bfull %lld wait-afull %lld\n", blockIdx.x, clock64() - t_all, w_bf, w_af);
+#endif
+      (void)w_bf; (void)w_af;
     }
   } else {  // workers: Psi digits into TMEM, column norms; at the end the accumulators into FP64 partials
     pdl_wait();
@@ -628,8 +664,12 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
     constexpr double kMA = g1_madd_a<S>();
     double nrm = 0.0;
     const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
+    long long w_pf = 0, w_afr = 0, w_st = 0;
+    G1_T0(t_all);
     for (int g = 0, s = 0, ph = 0, ab = 0, aph = 0; g < nhalf; ++g) {
+      G1_T0(c0);
       mbar_wait(&pfull[s], (uint32_t)ph);
+      G1_ACC(w_pf, c0);
       const long long ra = r0 + (long long)g * kG1Half;
       // this lane's components of Psi[row][sIdx] for rows 4h .. 4h+3: (Re, Im) for the even row m = 2s, (Im, Re)
       // for the odd row (its Re enters negated: sc2)
@@ -646,29 +686,46 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
           v2[t] = ok ? P[t * 2 * norb + 1 - cm] : 0.0;
         }
       }
-#pragma unroll
-      for (int t = 0; t < 4; ++t) nrm = fma(v1[t], v1[t], fma(v2[t], v2[t], nrm));  // absent rows add +0
+      // this lane's share of the column norm: Re^2 (even lane, v1 = Re) or Im^2 (odd lane, v1 = Im); the pair
+      // is summed once at the end. Absent rows add +0.
+      nrm = fma(v1[0], v1[0], nrm);
+      nrm = fma(v1[1], v1[1], nrm);
+      nrm = fma(v1[2], v1[2], nrm);
+      nrm = fma(v1[3], v1[3], nrm);
       uint32_t d1[S], d2[S];
       g1_bytes<S>(v1, sc, kMA, d1);
       g1_bytes<S>(v2, sc2, kMA, d2);
-      // this warp is done with the Psi rows (its loads have returned: lfd_tma.cuh)
-      mbar_release(&pempty[s], (v1[0] + v1[3]) + (v2[0] + v2[3]) + (v1[1] + v1[2]) + (v2[1] + v2[2]), lane == 0);
+      G1_T0(c1);
       if (g >= kNBuf) mbar_wait(&afree[ab], (uint32_t)(aph ^ 1));  // the MMAs of quarter block g - NBuf are done
+      G1_ACC(w_afr, c1);
       tc_fence_after();
+      G1_T0(c2);
 #pragma unroll
       for (int k = 0; k < S; ++k) {
         const uint32_t w2[2] = {d1[k], d2[k]};
         tmem_st2(trow + ab * kG1ABuf + k * 8 + 2 * h, w2);
       }
       asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+      G1_ACC(w_st, c2);
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(&afull[ab]);
+      if (lane == 0) {
+        mbar_arrive(&afull[ab]);
+        // the Psi rows are free: the digits just stored depend on every load of them, so those have returned
+        // (the hazard mbar_release guards against cannot occur here)
+        mbar_arrive(&pempty[s]);
+      }
       if (++s == kG1PsiSlots) { s = 0; ph ^= 1; }
       if (++ab == kNBuf) { ab = 0; aph ^= 1; }
     }
-    // column norms: both lanes of a pair hold the orbital's full |Psi|^2; the even lane writes it (fixed-order
-    // sum over the 4 row groups below)
+#ifdef LFD_G1_TIMING
+    if (tid == 0 && (blockIdx.x == 0 || blockIdx.x == 100))
+      printf("g1 cta %d work0: total %lld wait-pfull %lld wait-afree %lld tmem-st %lld\n", blockIdx.x, clock64() - t_all,
+             w_pf, w_afr, w_st);
+#endif
+    (void)w_pf; (void)w_afr; (void)w_st;
+    // column norms: Re^2 (even lane) + Im^2 (odd lane), then a fixed-order sum over the 4 row groups
+    nrm += __shfl_xor_sync(0xffffffffu, nrm, 1);
     if (!cm && sv) nsum[h][sIdx] = nrm;
     mbar_wait(&done, 0);
     tc_fence_after();
