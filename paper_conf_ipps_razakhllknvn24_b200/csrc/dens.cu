@@ -318,7 +318,7 @@ __global__ void __launch_bounds__(kDensThreads) k_density_tma(Geometry g, DensAr
 // mbarriers; the own line y+1 stays resident for the next step. kSub lanes per point split the orbitals
 // and the 7 per-point sums are shuffle reductions with the occupation weights (kept in shared memory).
 // ------------------------------------------------------------------------------------------------
-constexpr int kYOwn = 6, kYXp = 3;  // ring depths (lines); the own line y+1 stays resident for the y links
+// ring depths (lines): DensMaps::nso / nsx; the own line y+1 stays resident for the y links
 constexpr int kYMaxThreads = 512;  // up to 60 points x kSub + the producer warp
 
 struct DensMaps {
@@ -329,37 +329,49 @@ struct DensMaps {
   int nyc;           // y chunks per (plane group, z chunk)
   int nact;          // active orbitals: 1 + the last index with f != 0 (f = 0 contributes exactly 0)
   int esz;           // bytes per complex value: 16 (complex128) or 8 (complex64, the SP variant)
+  int nso, nsx;      // ring depths: own lines, x+px lines
 };
 
 // shared-memory layout of the y-marching kernel (every TMA destination 128-byte aligned): an own slot
 // holds px (segment, halo point) pairs
 struct YLayout {
   size_t seg_b, halo_b, pl_b, own_b, xp_b, fsh_off, bar_off, total;
-  __host__ __device__ YLayout(int zc, int norb, int px, int esz = 16) {  // esz: bytes per complex value
+  __host__ __device__ YLayout(int zc, int norb, int px, int esz, int nso, int nsx) {  // esz: bytes per complex value
     seg_b = ((size_t)zc * norb * esz + 127) & ~(size_t)127;
     halo_b = ((size_t)norb * esz + 127) & ~(size_t)127;
     pl_b = seg_b + halo_b;
     own_b = px * pl_b;
     xp_b = seg_b;
-    fsh_off = kYOwn * own_b + kYXp * xp_b;
+    fsh_off = nso * own_b + nsx * xp_b;
     bar_off = fsh_off + (((size_t)norb * 8 + 15) & ~(size_t)15);
-    total = bar_off + (2 * kYOwn + 2 * kYXp) * 8;
+    total = bar_off + (2 * nso + 2 * nsx) * 8;
   }
 };
 
 struct YShape {
-  int zc, px, nyc;
+  int zc, px, nyc, nso, nsx;
 };
 
-// Tuning knobs LFD_DENS_ZCMAX (points per plane), LFD_DENS_PX (planes per CTA), LFD_DENS_YC (y chunks).
+// The shape measured best on C2 inside the step loop (bench, ncu launch lists): 18 points per plane and CTA,
+// one y chunk, rings of 6 own / 3 x+1 lines. Sweeps of density calls alone (tools/dens_sweep.py,
+// profiles/r02_dens_sweep*.jsonl) favour smaller shapes with 4 resident CTAs per SM (12 points, 2 y chunks, rings
+// 3 / 2, <= 80 registers: 0.058 vs 0.066 ms there) because repeated calls find part of Psi in L2; inside the step
+// that shape measured 59.5 vs 56.7 us (ncu launch list r02h). A build with -DLFD_TUNING_KNOBS reads
+// LFD_DENS_ZCMAX / _PX / _YC / _OWN / _XP at lfd_init for such sweeps; the library proper reads no environment.
 static YShape ymarch_shape(const Geometry& g) {
-  YShape sh{0, 1, 1};
+  YShape sh{0, 1, 1, 6, 3};
   if (g.norb > 128) return sh;
   if (g.sp && (g.norb & 1)) return sh;  // TMA global strides must be multiples of 16 bytes
-  int zmax = 18, pxmax = 1, yc = 1;  // measured on C2 (tools/dens_tune.sh): 1 plane, 18 points
+  int zmax = 18, pxmax = 1, yc = 1;
+#ifdef LFD_TUNING_KNOBS
+  constexpr int kYOwnMax = 8, kYXpMax = 4;
   if (const char* v = std::getenv("LFD_DENS_ZCMAX")) zmax = std::max(1, std::min(60, std::atoi(v)));
   if (const char* v = std::getenv("LFD_DENS_PX")) pxmax = std::max(1, std::atoi(v));
   if (const char* v = std::getenv("LFD_DENS_YC")) yc = std::max(1, std::atoi(v));
+  if (const char* v = std::getenv("LFD_DENS_OWN")) sh.nso = std::max(3, std::min(kYOwnMax, std::atoi(v)));
+  if (const char* v = std::getenv("LFD_DENS_XP")) sh.nsx = std::max(1, std::min(kYXpMax, std::atoi(v)));
+#endif
+  const int esz = g.sp ? 8 : 16;
   int px = 1;
   for (int d = std::min(pxmax, g.nx); d >= 1; --d)
     if (g.nx % d == 0) { px = d; break; }
@@ -367,7 +379,7 @@ static YShape ymarch_shape(const Geometry& g) {
     if (g.nz % nzc) continue;
     const int zc = g.nz / nzc;
     if (zc > zmax || zc * px * kSub + 32 > kYMaxThreads) continue;
-    if (YLayout(zc, g.norb, px).total <= 200 * 1024) { sh.zc = zc; break; }
+    if (YLayout(zc, g.norb, px, esz, sh.nso, sh.nsx).total <= 200 * 1024) { sh.zc = zc; break; }
   }
   if (sh.zc == 0 && px > 1) {  // fall back to one plane per CTA
     sh.px = 1;
@@ -375,7 +387,7 @@ static YShape ymarch_shape(const Geometry& g) {
       if (g.nz % nzc) continue;
       const int zc = g.nz / nzc;
       if (zc > std::min(zmax, 40)) continue;
-      if (YLayout(zc, g.norb, 1).total <= 200 * 1024) { sh.zc = zc; break; }
+      if (YLayout(zc, g.norb, 1, esz, sh.nso, sh.nsx).total <= 200 * 1024) { sh.zc = zc; break; }
     }
     px = 1;
   }
@@ -391,7 +403,8 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
   pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   extern __shared__ __align__(128) unsigned char dsm[];
   const int norb = mp.nact, zc = mp.zc, px = mp.px;  // smem rows hold the nact active orbitals of each point
-  const YLayout Ly(zc, norb, px, (int)sizeof(C));
+  const int kYOwn = mp.nso, kYXp = mp.nsx;
+  const YLayout Ly(zc, norb, px, (int)sizeof(C), kYOwn, kYXp);
   auto own_seg = [&](int s, int p) { return reinterpret_cast<C*>(dsm + s * Ly.own_b + p * Ly.pl_b); };
   auto halo_of = [&](int s, int p) {
     return reinterpret_cast<C*>(dsm + s * Ly.own_b + p * Ly.pl_b + Ly.seg_b);
@@ -585,7 +598,7 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
   }
 }
 
-static size_t ymarch_smem(int zc, int nact, int px, int esz) { return YLayout(zc, nact, px, esz).total; }
+static size_t ymarch_smem(const DensMaps& m) { return YLayout(m.zc, m.nact, m.px, m.esz, m.nso, m.nsx).total; }
 
 // Psi as a 3-D tensor of 8-byte elements [rows][nz][norb * esz / 8] (the TMA only moves bytes: a
 // complex64 value is one 8-byte element, a complex128 value two).
@@ -609,6 +622,8 @@ DensMaps* density_maps_create(const Geometry& g, const double2* psi, int nact) {
   m->zc = sh.zc;
   m->px = sh.px;
   m->nyc = sh.nyc;
+  m->nso = sh.nso;
+  m->nsx = sh.nsx;
   m->esz = g.sp ? 8 : 16;
   if (density_maps_encode(m, g, psi, std::min(std::max(nact, 1), g.norb)) != cudaSuccess) {
     delete m;
@@ -638,7 +653,7 @@ cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps*
   dim3 grid(density_blocks(g), g.ndom);
   if (maps) {
     const int threads = ((maps->zc * maps->px * kSub + 31) / 32 + 1) * 32;
-    const size_t sm = ymarch_smem(maps->zc, maps->nact, maps->px, maps->esz);
+    const size_t sm = ymarch_smem(*maps);
     if (maps->esz == 8) {  // SP variant (complex64 Psi)
       if (g.bc == 0 && maps->nact == 32)
         launch_k(k_density_y<true, 4, float2>, grid, threads, sm, st, *maps, g, a);
