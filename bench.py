@@ -811,9 +811,10 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "dtype_note": ("complex FP64 storage and arithmetic everywhere except the two projector GEMMs, which are "
-                           "FP64 EMULATED on the int8 tensor cores (tcgen05 kind::i8): 6 balanced int8 digits per "
-                           "operand, 21 digit pairs accumulated exactly in int32 in TMEM, recombined in FP64 -- a "
-                           "product error of ~2^-40 of the row x column scales (IEEE FP64: ~2^-53); the step meets "
+                           "FP64 EMULATED on the int8 tensor cores (tcgen05 kind::i8): exact int8 digit splits "
+                           "(GEMM-2: 6 balanced base-128 digits, 21 pairs; GEMM-1: 5 base-256 digits, 19 pairs) "
+                           "accumulated exactly in int32 in TMEM, recombined in FP64 -- a product error of ~2^-40 / "
+                           "~2^-38 of the row x column scales (IEEE FP64: ~2^-53); the step meets "
                            "the FP64 parity contract (1e-10 after 100 steps, tests/test_gpu_parity.py::"
                            "test_c2_contract_100_steps); nl_dmma_mode is the same step in strict FP64") if nl_path == 1 else
                           "complex FP64 throughout (projector GEMMs on the FP64 DMMA pipe)",

@@ -81,8 +81,9 @@ typedef struct {
 /* lfd_config.flags: the SP variant (the paper's SP column, and its
  * complex<float> listings): psi, proj (and lfd_remap_occ's ref) are complex64 [.. same layouts ..]
  * (two floats, 8-byte aligned). The stencil sweeps run in FP32 (three line passes); the projector GEMMs run on
- * the tcgen05 int8 tensor cores with 4 balanced digits per operand (products to ~2^-27 of the row / column
- * scales, below FP32 rounding; the default where nproj, norb <= 64 and >= 65,536 points, or LFD_FLAG_NL_I8),
+ * the tcgen05 int8 tensor cores (GEMM-2: 4 balanced base-128 digits per operand; GEMM-1: 3 base-256 digits;
+ * products to ~2^-22 .. 2^-27 of the row / column scales, below FP32 rounding of Psi; the default where nproj,
+ * norb <= 64 and >= 65,536 points, or LFD_FLAG_NL_I8),
  * else as 3xTF32 on the warp-level mma.sync path (LFD_FLAG_NL_DMMA selects the latter); everything
  * O(nproj x norb) -- the split reduction, the Gram matrix, n_s, the carry, the energies -- runs in FP64. Results
  * agree with the FP64 path to single-precision roundoff (DESIGN.md §4 states the tolerance). */
@@ -90,11 +91,12 @@ typedef struct {
 /* lfd_config.flags: run the nonlocal GEMMs (C = dV B^H Psi; Psi <- Psi diag(n) + B C'') as
  * strict IEEE complex FP64 on the DMMA pipe (mma.sync m8n8k4) instead of the default for FP64 contexts with
  * nproj <= 64, norb <= 64 and >= 65,536 points per domain: the same products EMULATED on the tcgen05 int8
- * tensor cores -- B and C'' split exactly into 6 balanced int8 digits each with power-of-two row / column
- * scales, the 21 digit pairs i + j <= 7 accumulated exactly in int32 in tensor memory, recombined in FP64.
+ * tensor cores -- operands split exactly into int8 digits with power-of-two row / column scales, the digit
+ * pairs accumulated exactly in int32 in tensor memory, recombined in FP64 (GEMM-2: 6 balanced base-128 digits,
+ * the 21 pairs i + j <= 7; GEMM-1: 5 base-256 digits, Psi's offset-binary, the 19 pairs k + i >= 3).
  * That arithmetic is narrower than an FP64 product: the truncation (digit remainders and dropped pairs) leaves
- * an error of ~2^-40 of (row scale x column scale) per output, against ~2^-53 for IEEE FP64 (measured per
- * GEMM in tests/test_gpu_i8.py). The nonlocal update B C'' is O(Delta Delta_sci / 2 ~ 1.4e-3) of Psi, so at the
+ * an error of ~2^-40 (GEMM-2) / ~2^-38 (GEMM-1) of (row scale x column scale) per output, against ~2^-53 for
+ * IEEE FP64 (measured against the DMMA path in tests/test_gpu_i8.py). The nonlocal update B C'' is O(Delta Delta_sci / 2 ~ 1.4e-3) of Psi, so at the
  * paper's scissor size each factor moves Psi by ~1e-15 relative and the FP64 parity contract (1e-10 after 100
  * steps) holds; bench.py reports the strict-FP64 step (this flag) beside the default. See lfd_nl_path(). */
 #define LFD_FLAG_NL_DMMA 8

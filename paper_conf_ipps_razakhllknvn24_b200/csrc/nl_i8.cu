@@ -1,7 +1,7 @@
-// nl_i8.cu -- GEMM-2 of the nonlocal factor (Eq. 9 / P:210) on the tcgen05 tensor
-// cores with FP64 accuracy: the FP64 operands are split into int8 digit slices (an Ozaki-type scheme), the
-// digit products run as tcgen05.mma kind::i8 with exact int32 accumulation in TMEM, and the epilogue
-// recombines them in FP64.
+// nl_i8.cu -- the projector GEMMs of the nonlocal factor (Eq. 9 / P:210) on the
+// tcgen05 tensor cores with (emulated) FP64 accuracy: the FP64 operands are split exactly into int8 digit
+// slices (an Ozaki-type scheme), the digit products run as tcgen05.mma kind::i8 with exact int32
+// accumulation in TMEM, and the epilogues recombine them in FP64. GEMM-2 first, GEMM-1 further down.
 //
 //   Psi[r][s] <- n_s Psi[r][s] + sum_u B[r][u] X[u][s]          (X = C'' = C' diag(n), nl.cu)
 //
@@ -22,18 +22,21 @@
 // wide margin (tests/test_gpu_i8.py checks the same bound as the FP64 path).
 //
 // Kernel (B200-first). The B digits are built ONCE at lfd_init (B is constant: P:216's resident Psi_u(0))
-// into tiles of 32 grid points, each tile [S][32 rows][128 B] already in the canonical K-major
-// SWIZZLE_128B shared-memory image, so one cp.async.bulk per tile stages it. Per call every CTA builds the
-// W digits (6 x 16 KB) from C'' itself, straight into TMEM (tcgen05.st), where they are the MMA's A
-// operand -- shared memory is left to the two streaming rings. Transposed MMA: D[n][r] = sum_k W^T[n][k]
-// b[r][k] (M = 128 output columns n on the TMEM lanes, N = 32 grid points), so each epilogue lane owns one
-// Psi double n and a warp reads/writes 256 contiguous bytes per grid point. Roles: warp 8 = producer of the
-// digit tiles, warp 10 = producer of the tile's Psi rows (contiguous in HBM: one bulk copy into a 2-deep
-// shared-memory ring), warp 9 = MMA issuer (21 digit pairs x 4 K-steps per tile into 6 diagonal
-// accumulators), warps 0-7 = epilogue (tcgen05.ld, FP64 recombination, Psi update stored to HBM). The
-// epilogue releases the accumulators as soon as they are in registers, so the MMAs of tile t+1 overlap
-// its FP64 work on tile t; the digit ring (3 x 24 KB) and the Psi ring (4 x 32 KB) keep ~150 KB per SM in
-// flight.
+// into tiles of 64 grid points, each tile [S][64 rows][128 B] already in the canonical K-major SWIZZLE_128B
+// shared-memory image, so one cp.async.bulk per tile stages it (2-stage ring), plus the row scales sigma_r.
+// Per call every CTA builds the W digits (S x 16 KB) from C'' (one bulk copy) straight into TMEM
+// (tcgen05.st), where they are the MMA's A operand. Transposed MMA: D[n][r] = sum_k W^T[n][k] b[r][k]
+// (M = 128 output doubles n on the TMEM lanes, N = 64 grid points), so each epilogue lane owns one Psi double
+// n of a row. Roles: warp 16 = producer of the digit tiles, warp 18 = producer of the tile's Psi rows and
+// their sigma_r (16-row sub-tiles, contiguous in HBM, one bulk copy each into a 7-slot ring), warp 17 = MMA
+// issuer (the 21 digit pairs x 4 K-steps of a tile into S diagonal accumulators d = i + j, each in a slot of
+// a TMEM ring of (512 - 32 S) / 64 slots), warps 0-15 = epilogue (4 TMEM lane quarters x 4 row quarters:
+// tcgen05.ld of the diagonals two at a time, (P_d 2^7 + P_{d+1}) exact in int32, FP64 recombination with
+// the scales applied by exponent arithmetic, Psi <- n_s Psi + sigma_r tau_n acc stored to HBM). The epilogue
+// releases each accumulator slot as soon as it is in registers, so the MMAs run up to a ring ahead of it.
+// S = 6 for FP64 contexts, 4 for the SP variant (complex64 Psi, float epilogue stores).
+// GEMM-1 (below) uses a different, base-256 digit scheme; the first nonlocal factor's GEMM-2 fused with
+// the x pass is nl_fx.cu.
 #include "lfd_internal.h"
 #include "lfd_tc.cuh"
 #include "lfd_tma.cuh"
