@@ -766,12 +766,15 @@ def main():
             except Exception as ex:
                 small[nm] = {"error": f"{type(ex).__name__}: {ex}"}
 
-    # end to end through the C ABI with HOST buffers: pinned v in, pinned rho + J out, every step
+    # end to end through the C ABI with HOST buffers: pinned v in, pinned rho + J out, every step. The host
+    # double-buffers both (the library's copies run on side streams, overlapping the kernels): it refills v for
+    # step n and reads step n-1's rho / J (lfd_wait_host_outputs(1)) while step n runs.
     e2e = None
     if not args.no_e2e:
-        vh = torch.from_numpy(x.vloc.copy()).pin_memory()
-        rh = torch.empty((nd, ng), dtype=torch.float64).pin_memory()
-        Jh = torch.empty((nd, 3), dtype=torch.float64).pin_memory()
+        vh = [torch.from_numpy(x.vloc.copy()).pin_memory() for _ in range(2)]
+        rh = [torch.empty((nd, ng), dtype=torch.float64).pin_memory() for _ in range(2)]
+        Jh = [torch.empty((nd, 3), dtype=torch.float64).pin_memory() for _ in range(2)]
+        vsrc = torch.from_numpy(x.vloc)
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
@@ -780,16 +783,20 @@ def main():
         t0 = time.perf_counter()
         f0.record(stream)
         for n in range(args.steps):
+            vh[n % 2].copy_(vsrc)  # this step's input (its slot's previous H2D, step n-2, has run)
             lfd.lfd_set_vector_potential(ctx.ctx, A_seq[args.warmup + n])
-            lfd.lfd_set_potential_host(ctx.ctx, vh)
+            lfd.lfd_set_potential_host(ctx.ctx, vh[n % 2])
             lfd.lfd_step(ctx.ctx, 1)
-            lfd.lfd_density_current_host(ctx.ctx, rh, Jh)
+            lfd.lfd_density_current_host(ctx.ctx, rh[n % 2], Jh[n % 2])
             if world > 1:
                 send = gat.send[0]
                 lfd.lfd_density_current(ctx.ctx, send[: nd * ng], None, send[nd * ng:])
                 dist.all_gather_into_tensor(gat.recv[0], send)
-            lfd.lfd_sync(ctx.ctx)  # the host reads this step's rho / J
-            _ = float(Jh[0, 2])
+            if n >= 1:
+                lfd.lfd_wait_host_outputs(ctx.ctx, 1)  # step n-1's rho / J are on the host
+                _ = float(Jh[(n - 1) % 2][0, 2])
+        lfd.lfd_wait_host_outputs(ctx.ctx, 0)
+        _ = float(Jh[(args.steps - 1) % 2][0, 2])
         f1.record(stream)
         torch.cuda.synchronize()
         ems = max(f0.elapsed_time(f1), 1e3 * (time.perf_counter() - t0))
@@ -798,8 +805,10 @@ def main():
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
         e2e = {"value": ogp / (float(te.item()) / 1e3), "unit": UNIT, "h2d_bytes_per_step": int(nd * ng * 8),
                "d2h_bytes_per_step": int(nd * ng * 8 + nd * 3 * 8),
-               "note": "per step: H2D v_loc (pinned) -> a1..a7 -> D2H rho + J (pinned) -> host sync; "
-                       "Psi and B stay resident in HBM (the paper's GPU-resident design, P:216)"}
+               "note": "per step: host refills a pinned v_loc buffer -> H2D (library side stream) -> a1..a7 -> D2H rho "
+                       "+ J into pinned buffers (side stream) -> the host reads them one step later (double-buffered, "
+                       "lfd_wait_host_outputs); Psi and B stay resident in HBM (the paper's GPU-resident design, "
+                       "P:216)"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

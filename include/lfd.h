@@ -169,8 +169,10 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
  * call's work has run). */
 lfd_status lfd_set_potential(lfd_ctx* ctx, const double* vloc);
 
-/* As lfd_set_potential, but vloc is a HOST buffer (pinned recommended): an async H2D copy into the
- * workspace is enqueued. The host buffer must stay unchanged until that copy has run (lfd_sync). */
+/* As lfd_set_potential, but vloc is a HOST buffer (pinned recommended): an async H2D copy into one of two
+ * workspace staging slots is enqueued on a side stream (so it overlaps the kernels already queued, e.g. the
+ * previous step), and the potential-phase kernel waits for it in stream order. The host buffer must stay
+ * unchanged until that copy has run (lfd_sync; callers that refill it every step double-buffer it). */
 lfd_status lfd_set_potential_host(lfd_ctx* ctx, const double* vloc_host);
 
 /* A_X(alpha)(t) at the step midpoint (Eq. 2 / Eq. 5; Eq. 4 midpoint), HOST double [ndom][3] a.u.;
@@ -229,6 +231,12 @@ lfd_status lfd_density_current_global(lfd_ctx* ctx, double* rho_g, double* j_g, 
 /* As lfd_density_current for rho and Jmac, into HOST buffers (pinned recommended) via async D2H
  * copies; read them after lfd_sync(). Either pointer may be NULL to skip it. */
 lfd_status lfd_density_current_host(lfd_ctx* ctx, double* rho_host, double* Jmac_host);
+
+/* Wait on the host until the D2H copies of an lfd_density_current_host call have landed: lag 0 = the latest
+ * call, lag 1 = the one before it (its copies ran on a side stream while later work was queued: a caller that
+ * double-buffers its host outputs reads step n's while step n+1 runs). LFD_EINVAL for another lag,
+ * LFD_ESTATE if there is no such call; asynchronous CUDA errors as lfd_sync. */
+lfd_status lfd_wait_host_outputs(lfd_ctx* ctx, int32_t lag);
 
 /* calc_energy (Fig. 5): E[dom][4] = {kinetic, local, nonlocal,
  * total} of the current Psi with the current v_loc and A, DEVICE double, stream-ordered:

@@ -33,7 +33,7 @@ constexpr int kKC1 = 32;  // GEMM-1 rows per chunk (nl.cu)
 size_t up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 struct Layout {
-  size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage, cref,
+  size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage, hv[2], hrho[2], hJ[2], cref,
       epart, W, ones, x32, aseq, jseq, bsl, bsig, bsl1, bexp, colE, g1cnt, g1cs, btil, qmat, zero, bslx, sigx;
   int nref_cap;
   bool i8;  // GEMM-2 on the int8 tensor cores (nl_i8.cu): B digit tiles + row scales in the workspace
@@ -182,6 +182,11 @@ Layout layout(const Geometry& g, int num_sms, int nref_max, bool dense = false) 
   L.vstage = take((size_t)nd * g.ng * d8);
   L.rhostage = take((size_t)nd * g.ng * d8);
   L.Jstage = take((size_t)nd * 3 * d8);
+  for (int k = 0; k < 2; ++k) {  // double-buffered staging of the host-buffer calls (copies on side streams)
+    L.hv[k] = take((size_t)nd * g.ng * d8);
+    L.hrho[k] = take((size_t)nd * g.ng * d8);
+    L.hJ[k] = take((size_t)nd * 3 * d8);
+  }
   L.cref = take((size_t)nd * std::max(L.nref_cap, np) * no * c16);
   L.epart = take((size_t)nd * lfd::density_blocks(g) * 2 * d8);
   L.W = take((size_t)2 * nd * np * c16);
@@ -341,6 +346,10 @@ struct lfd_ctx {
   };
   std::vector<Graph> graphs;
   cudaStream_t cap_stream = nullptr;  // private stream for capture only (the legacy stream cannot capture)
+  // host-buffer calls: H2D / D2H on two side streams, double-buffered staging, created on first use
+  cudaStream_t h2d = nullptr, d2h = nullptr;
+  cudaEvent_t ev_vcopy[2] = {}, ev_vfree[2] = {}, ev_dens[2] = {}, ev_d2h[2] = {};
+  long long nvh = 0, ndh = 0;  // host-buffer calls so far (slot = count % 2)
 
   template <class T>
   T* at(size_t off) const { return reinterpret_cast<T*>(ws + off); }
@@ -1135,15 +1144,42 @@ lfd_status lfd_set_potential(lfd_ctx* c, const double* vloc) {
   });
 }
 
+// The side streams and events of the host-buffer calls (created once; the copies then overlap the kernels
+// of the context stream: the H2D of step n+1's v_loc runs during step n, the D2H of step n's rho / J during
+// step n+1).
+static lfd_status host_copy_init(lfd_ctx* c) {
+  if (c->h2d) return LFD_OK;
+  cudaError_t e = cudaStreamCreateWithFlags(&c->h2d, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->d2h, cudaStreamNonBlocking);
+  for (int k = 0; k < 2 && e == cudaSuccess; ++k) {
+    e = cudaEventCreateWithFlags(&c->ev_vcopy[k], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_vfree[k], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_dens[k], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_d2h[k], cudaEventDisableTiming);
+  }
+  if (e != cudaSuccess) return cuda_fail(c, e, "host copy streams");
+  return LFD_OK;
+}
+
 lfd_status lfd_set_potential_host(lfd_ctx* c, const double* vloc_host) {
   LFD_TRY(check_ctx(c));
   if (!vloc_host) return fail(c, LFD_EINVAL, "vloc_host is NULL");
   DeviceGuard dg(c->device);
-  double* stage = c->at<double>(c->L.vstage);
-  cudaError_t e = cudaMemcpyAsync(stage, vloc_host, sizeof(double) * c->g.ndom * c->g.ng, cudaMemcpyHostToDevice,
-                                  c->stream);
+  LFD_TRY(host_copy_init(c));
+  const int k = (int)(c->nvh & 1);
+  double* stage = c->at<double>(c->L.hv[k]);
+  // the H2D into slot k waits for the k_phase that read slot k two calls ago; k_phase waits for the H2D
+  cudaError_t e = c->nvh >= 2 ? cudaStreamWaitEvent(c->h2d, c->ev_vfree[k], 0) : cudaSuccess;
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(stage, vloc_host, sizeof(double) * c->g.ndom * c->g.ng, cudaMemcpyHostToDevice, c->h2d);
+  if (e == cudaSuccess) e = cudaEventRecord(c->ev_vcopy[k], c->h2d);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(c->stream, c->ev_vcopy[k], 0);
   if (e != cudaSuccess) return cuda_fail(c, e, "H2D vloc");
-  return launch(c, LFD_K_PHASE, "k_phase", [&] { return phase_any(c, stage, stage); });
+  LFD_TRY(launch(c, LFD_K_PHASE, "k_phase", [&] { return phase_any(c, stage, c->at<double>(c->L.vstage)); }));
+  e = cudaEventRecord(c->ev_vfree[k], c->stream);
+  if (e != cudaSuccess) return cuda_fail(c, e, "event");
+  ++c->nvh;
+  return LFD_OK;
 }
 
 lfd_status lfd_set_vector_potential(lfd_ctx* c, const double* A) {
@@ -1286,18 +1322,33 @@ lfd_status lfd_density_current_host(lfd_ctx* c, double* rho_host, double* Jmac_h
   if (c->nl_pending) return fail(c, LFD_ESTATE, "Psi is between lfd_step_prologue and its step");
   DeviceGuard dg(c->device);
   const Geometry& g = c->g;
-  double* rs = c->at<double>(c->L.rhostage);
-  double* Js = c->at<double>(c->L.Jstage);
+  LFD_TRY(host_copy_init(c));
+  const int k = (int)(c->ndh & 1);
+  double* rs = c->at<double>(c->L.hrho[k]);
+  double* Js = c->at<double>(c->L.hJ[k]);
+  // staging slot k is rewritten only after its D2H of two calls ago; the D2H waits for this density
+  cudaError_t e = c->ndh >= 2 ? cudaStreamWaitEvent(c->stream, c->ev_d2h[k], 0) : cudaSuccess;
+  if (e != cudaSuccess) return cuda_fail(c, e, "event wait");
   LFD_TRY(density_into(c, rs, nullptr, Js, c->at<long long>(c->L.base), (long long)g.ny * g.nz, g.nz, g.ng));
-  cudaError_t e;
-  if (rho_host) {
-    e = cudaMemcpyAsync(rho_host, rs, sizeof(double) * g.ndom * g.ng, cudaMemcpyDeviceToHost, c->stream);
-    if (e != cudaSuccess) return cuda_fail(c, e, "D2H rho");
-  }
-  if (Jmac_host) {
-    e = cudaMemcpyAsync(Jmac_host, Js, sizeof(double) * g.ndom * 3, cudaMemcpyDeviceToHost, c->stream);
-    if (e != cudaSuccess) return cuda_fail(c, e, "D2H J");
-  }
+  e = cudaEventRecord(c->ev_dens[k], c->stream);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(c->d2h, c->ev_dens[k], 0);
+  if (e == cudaSuccess && rho_host)
+    e = cudaMemcpyAsync(rho_host, rs, sizeof(double) * g.ndom * g.ng, cudaMemcpyDeviceToHost, c->d2h);
+  if (e == cudaSuccess && Jmac_host)
+    e = cudaMemcpyAsync(Jmac_host, Js, sizeof(double) * g.ndom * 3, cudaMemcpyDeviceToHost, c->d2h);
+  if (e == cudaSuccess) e = cudaEventRecord(c->ev_d2h[k], c->d2h);
+  if (e != cudaSuccess) return cuda_fail(c, e, "D2H rho / J");
+  ++c->ndh;
+  return LFD_OK;
+}
+
+lfd_status lfd_wait_host_outputs(lfd_ctx* c, int32_t lag) {
+  LFD_TRY(check_ctx(c));
+  if (lag < 0 || lag > 1) return fail(c, LFD_EINVAL, "lag must be 0 or 1");
+  if (c->ndh <= lag) return fail(c, LFD_ESTATE, "no such lfd_density_current_host call");
+  DeviceGuard dg(c->device);
+  cudaError_t e = cudaEventSynchronize(c->ev_d2h[(int)((c->ndh - 1 - lag) & 1)]);
+  if (e != cudaSuccess) return cuda_fail(c, e, "asynchronous CUDA error");
   return LFD_OK;
 }
 
@@ -1584,6 +1635,8 @@ lfd_status lfd_sync(lfd_ctx* c) {
   LFD_TRY(check_ctx(c));
   DeviceGuard dg(c->device);
   cudaError_t e = cudaStreamSynchronize(c->stream);
+  if (e == cudaSuccess && c->h2d) e = cudaStreamSynchronize(c->h2d);
+  if (e == cudaSuccess && c->d2h) e = cudaStreamSynchronize(c->d2h);
   if (e == cudaSuccess) e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "asynchronous CUDA error");
   return LFD_OK;
@@ -1640,6 +1693,18 @@ lfd_status lfd_destroy(lfd_ctx* c) {
   {
     DeviceGuard dg(c->device);
     cudaStreamSynchronize(c->stream);
+    if (c->h2d) {
+      cudaStreamSynchronize(c->h2d);
+      cudaStreamSynchronize(c->d2h);
+      for (int k = 0; k < 2; ++k) {
+        cudaEventDestroy(c->ev_vcopy[k]);
+        cudaEventDestroy(c->ev_vfree[k]);
+        cudaEventDestroy(c->ev_dens[k]);
+        cudaEventDestroy(c->ev_d2h[k]);
+      }
+      cudaStreamDestroy(c->h2d);
+      cudaStreamDestroy(c->d2h);
+    }
     for (auto& s : c->slots) {
       cudaEventDestroy(s.a);
       cudaEventDestroy(s.b);

@@ -36,7 +36,7 @@ LFD_SC_XC = 2
 LFD_SC_MAXWELL = 4
 EXPORTS = ("lfd_workspace_size", "lfd_init", "lfd_set_potential", "lfd_set_potential_host",
            "lfd_set_vector_potential", "lfd_step", "lfd_step_prologue", "lfd_step_sequence", "lfd_density_current", "lfd_density_current_global",
-           "lfd_density_current_host", "lfd_energy", "lfd_remap_occ", "lfd_psi_modified", "lfd_set_occupations", "lfd_set_stream", "lfd_sync",
+           "lfd_density_current_host", "lfd_wait_host_outputs", "lfd_energy", "lfd_remap_occ", "lfd_psi_modified", "lfd_set_occupations", "lfd_set_stream", "lfd_sync",
            "lfd_launch_count", "lfd_nl_path", "lfd_profile_enable", "lfd_profile_read", "lfd_last_error", "lfd_destroy",
            "lfd_sc_workspace_size", "lfd_sc_init", "lfd_sc_step", "lfd_sc_read", "lfd_comm_unique_id",
            "lfd_sc_comm_init", "lfd_step_graph")
@@ -85,6 +85,7 @@ def load():
         "lfd_density_current": [P, P, P, P],
         "lfd_density_current_global": [P, P, P, P, P, P],
         "lfd_density_current_host": [P, P, P],
+        "lfd_wait_host_outputs": [P, I32],
         "lfd_energy": [P, P],
         "lfd_remap_occ": [P, P, I32, P],
         "lfd_set_occupations": [P, P],
@@ -142,6 +143,21 @@ def _hptr(a, dtype=np.float64):
     return C.c_void_p(arr.ctypes.data), arr
 
 
+def _hptr_async(a):
+    """Host pointer for an ASYNC copy (lfd_set_potential_host / lfd_density_current_host): the buffer itself must
+    be contiguous float64 (a converted temporary would be freed before the copy runs)."""
+    if a is None:
+        return None
+    if hasattr(a, "data_ptr") and not getattr(a, "is_cuda", False):
+        import torch
+        if not a.is_contiguous() or a.dtype != torch.float64:
+            raise TypeError("expected a contiguous float64 host tensor")
+        return C.c_void_p(a.data_ptr())
+    if not isinstance(a, np.ndarray) or a.dtype != np.float64 or not a.flags["C_CONTIGUOUS"]:
+        raise TypeError("expected a C-contiguous float64 numpy array")
+    return C.c_void_p(a.ctypes.data)
+
+
 def _stream_ptr(stream=None):
     import torch
     s = stream if stream is not None else torch.cuda.current_stream()
@@ -177,8 +193,9 @@ def lfd_set_potential(ctx, vloc):
 
 
 def lfd_set_potential_host(ctx, vloc_host):
-    p, _k = _hptr(vloc_host)
-    _check(load().lfd_set_potential_host(ctx, p), ctx)
+    """vloc_host: contiguous float64 host buffer (pinned recommended), copied asynchronously: keep it unchanged
+    until lfd_sync (or double-buffer it)."""
+    _check(load().lfd_set_potential_host(ctx, _hptr_async(vloc_host)), ctx)
 
 
 def lfd_set_vector_potential(ctx, A):
@@ -219,9 +236,13 @@ def lfd_density_current_global(ctx, rho_g, j_g, Jmac, dom_offset, gdims):
 
 
 def lfd_density_current_host(ctx, rho_host=None, Jmac_host=None):
-    pr, _k1 = _hptr(rho_host)
-    pj, _k2 = _hptr(Jmac_host)
-    _check(load().lfd_density_current_host(ctx, pr, pj), ctx)
+    """rho_host / Jmac_host: contiguous float64 host buffers (pinned recommended), written asynchronously: read
+    them after lfd_sync or lfd_wait_host_outputs."""
+    _check(load().lfd_density_current_host(ctx, _hptr_async(rho_host), _hptr_async(Jmac_host)), ctx)
+
+
+def lfd_wait_host_outputs(ctx, lag=0):
+    _check(load().lfd_wait_host_outputs(ctx, lag), ctx)
 
 
 def lfd_energy(ctx, E):

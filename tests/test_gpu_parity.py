@@ -168,6 +168,56 @@ def test_norm_conservation_on_gpu():
     assert np.abs(w.dV * np.einsum("rs,rs->s", P.conj(), P).real - 1).max() < 1e-12
 
 
+def test_host_buffer_pipeline_double_buffered():
+    """the host-buffer calls with their copies on side streams: a caller that double-buffers v_loc and the
+    outputs and reads step n's rho / J (lfd_wait_host_outputs(1)) while step n+1 runs gets, step by step,
+    exactly the device-path values"""
+    torch = _torch()
+    from paper_conf_ipps_razakhllknvn24_b200 import Context, lfd
+    w = workload("C1")
+    x = make_inputs(w, seed=12)
+    dev = torch.device("cuda:0")
+    nsteps = 6
+    vs = [x.vloc * (1.0 + 0.02 * n) for n in range(nsteps)]
+    # reference: device buffers, synchronous reads
+    psi = torch.from_numpy(x.psi0.copy()).to(dev)
+    ctx = Context(psi, torch.from_numpy(x.proj).to(dev), x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt)
+    want = []
+    for n in range(nsteps):
+        ctx.set_potential(torch.from_numpy(vs[n]).to(dev))
+        ctx.set_vector_potential(midpoint_A(w, n))
+        ctx.step(1)
+        rho, _, J = ctx.density_current()
+        ctx.sync()
+        want.append((rho.cpu().clone(), J.cpu().clone()))
+    ctx.close()
+    # pipelined host-buffer loop
+    psi2 = torch.from_numpy(x.psi0.copy()).to(dev)
+    ctx2 = Context(psi2, torch.from_numpy(x.proj).to(dev), x.dnl, x.occ, (w.hx, w.hy, w.hz), w.dt)
+    vh = [torch.empty(vs[0].shape, dtype=torch.float64).pin_memory() for _ in range(2)]
+    rh = [torch.empty((w.ndom, w.nx, w.ny, w.nz), dtype=torch.float64).pin_memory() for _ in range(2)]
+    Jh = [torch.empty((w.ndom, 3), dtype=torch.float64).pin_memory() for _ in range(2)]
+    got = []
+    for n in range(nsteps):
+        vh[n % 2].copy_(torch.from_numpy(vs[n]))  # its previous H2D (step n-2) has run: see the wait below
+        lfd.lfd_set_potential_host(ctx2.ctx, vh[n % 2])
+        lfd.lfd_set_vector_potential(ctx2.ctx, midpoint_A(w, n))
+        lfd.lfd_step(ctx2.ctx, 1)
+        lfd.lfd_density_current_host(ctx2.ctx, rh[n % 2], Jh[n % 2])
+        if n >= 1:
+            lfd.lfd_wait_host_outputs(ctx2.ctx, 1)
+            got.append((rh[(n - 1) % 2].clone(), Jh[(n - 1) % 2].clone()))
+    lfd.lfd_wait_host_outputs(ctx2.ctx, 0)
+    got.append((rh[(nsteps - 1) % 2].clone(), Jh[(nsteps - 1) % 2].clone()))
+    with pytest.raises(lfd.LFDError):
+        lfd.lfd_wait_host_outputs(ctx2.ctx, 2)
+    ctx2.sync()
+    assert torch.equal(psi, psi2)
+    for (r1, J1), (r2, J2) in zip(want, got):
+        assert torch.equal(r1.reshape(r2.shape), r2) and torch.equal(J1, J2)
+    ctx2.close()
+
+
 def test_global_layout_and_host_variants():
     torch = _torch()
     from paper_conf_ipps_razakhllknvn24_b200 import Context, lfd
