@@ -604,6 +604,18 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr, bool
 // src != nullptr: the first pass reads src (same layout) and writes Psi (out of place).
 lfd_status local_prop(lfd_ctx* c, const double2* src = nullptr, bool skip_x = false) {
   c->c_valid = false;
+  if (c->g.sp && c->kin_fused) {  // SP variant: Phi.K_x, then Phi.K_y K_z fused (FP32, complex64 Psi)
+    LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin_sp(x)", [&] {
+      return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 0, 1, c->scaled, c->stream,
+                                reinterpret_cast<const float2*>(src));
+    }));
+    int* colE = c->L.i8 ? c->at<int>(c->L.colE) : nullptr;  // exponents for the int8-digit GEMM-1
+    LFD_TRY(launch(c, LFD_K_KIN_YZ, "k_kin_yz_sp", [&] {
+      return lfd::launch_kin_yz_sp(c->g, &c->psi_tmap, c->psi32(), c->coef(), c->phi32(), c->scaled, c->stream, colE);
+    }));
+    c->colE_valid = colE != nullptr;
+    return LFD_OK;
+  }
   if (c->g.sp) {  // SP variant: three FP32 line passes Phi.K_x, K_y, K_z.Phi (complex64 Psi)
     LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin_sp(x)", [&] {
       return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 0, 1, c->scaled, c->stream,
@@ -986,7 +998,7 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   c->carry = (cfg->flags & LFD_FLAG_NO_CARRY) == 0;
   c->no_pdl = (cfg->flags & LFD_FLAG_NO_PDL) != 0;
   c->scaled = c->scaled && lfd::kin_scaled_ok(g);
-  c->kin_fused = c->kin_fused && lfd::kin_yz_supported(g) && !g.sp;
+  c->kin_fused = c->kin_fused && lfd::kin_yz_supported(g);
   c->dmaps = lfd::density_maps_create(g, c->psi, active_orbitals(g, occ));
   if (c->kin_fused && lfd::kin_yz_tensor_map(g, c->psi, &c->psi_tmap) != cudaSuccess) {
     cudaGetLastError();

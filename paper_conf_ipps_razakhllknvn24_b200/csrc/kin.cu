@@ -226,6 +226,11 @@ __global__ void __launch_bounds__(256, 3) k_kin(V* psi, const V* src, const DomC
 // orbital o0 + o and recomputes its neighbours' first-E outputs from the ring instead of exchanging
 // them, so consumer warps never synchronise with each other.
 // ------------------------------------------------------------------------------------------------
+// a value of a loaded register, for mbar_release (lfd_tma.cuh)
+__device__ __forceinline__ double dep_of(double2 v) { return v.x; }
+__device__ __forceinline__ double dep_of(float2 v) { return (double)v.x; }
+__device__ __forceinline__ double dep_of(cf2 v) { return (double)v.a.x; }
+
 constexpr int kYZW = 8;
 constexpr int kYZMaxThreads = 352;  // up to 40 z pairs x 8 orbitals + the producer warp
 constexpr int kYZS = 10;            // ring depth (planes); even, so a y pair never straddles the wrap
@@ -233,10 +238,10 @@ constexpr int kYZS = 10;            // ring depth (planes); even, so a y pair ne
 // bytes of one ring slot: the Psi segment [nz][8 orbitals] + the Phi row [nz], 128-byte aligned
 __host__ __device__ __forceinline__ int yz_slot_bytes(int nz) { return (nz * kYZW * 16 + nz * 16 + 127) & ~127; }
 
-template <bool kPer, bool kS>
+template <bool kPer, bool kS, class C = double2, class V = C>
 __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant__ CUtensorMap tmap,
-                                                          double2* __restrict__ psi, const DomCoef* __restrict__ coef,
-                                                          const double2* __restrict__ phi, int nx, int ny, int nz,
+                                                          V* __restrict__ psi, const DomCoef* __restrict__ coef,
+                                                          const C* __restrict__ phi, int nx, int ny, int nz,
                                                           int norb, int nchunks, long long ng, int* __restrict__ colE) {
   pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
   pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
@@ -245,8 +250,8 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
   extern __shared__ __align__(128) unsigned char smem[];
   const int seg = nz * kYZW;                               // complex elements of the Psi segment
   const int slot_b = yz_slot_bytes(nz);                    // Psi segment + Phi row, 128-byte aligned
-  auto slot_psi = [&](int s) { return reinterpret_cast<const double2*>(smem + s * slot_b); };
-  auto slot_phi = [&](int s) { return reinterpret_cast<const double2*>(smem + s * slot_b + seg * 16); };
+  auto slot_psi = [&](int s) { return reinterpret_cast<const V*>(smem + s * slot_b); };
+  auto slot_phi = [&](int s) { return reinterpret_cast<const C*>(smem + s * slot_b + seg * 16); };
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + kYZS * slot_b);
   uint64_t* empty = full + kYZS;
   const int dom = blockIdx.y;
@@ -255,13 +260,13 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
   const int npz = (nz + 1) >> 1;                 // z pairs (the last one a singleton for odd nz)
   const int nconsw = (npz * kYZW + 31) >> 5;     // consumer warps; the next warp is the producer
   // coefficients live in shared memory (broadcast LDS) to keep registers for the march state
-  __shared__ PairCoef sc[2];
-  const PairCoef& cz_ = sc[0];
-  const PairCoef& cy = sc[1];
+  __shared__ PairCoefT<C> sc[2];
+  const PairCoefT<C>& cz_ = sc[0];
+  const PairCoefT<C>& cy = sc[1];
   const int tid = threadIdx.x;
   if (tid == 0) {
-    sc[0] = pair_coef<kS>(coef + dom, 2);
-    sc[1] = pair_coef<kS>(coef + dom, 1);
+    sc[0] = pair_coef_t<kS, C>(coef + dom, 2);
+    sc[1] = pair_coef_t<kS, C>(coef + dom, 1);
     for (int s = 0; s < kYZS; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], nconsw);
@@ -269,7 +274,7 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  const double2* phx = phi + (long long)dom * ng + (long long)x * ny * nz;  // Phi(x, y = 0, z = 0)
+  const C* phx = phi + (long long)dom * ng + (long long)x * ny * nz;  // Phi(x, y = 0, z = 0)
 
   if (tid >= nconsw * 32) {  // producer warp: plane y -> slot y % kYZS (Psi: one tensor copy; Phi: one row)
     if (tid == nconsw * 32) {
@@ -278,9 +283,9 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
       uint32_t ph = 0;
       for (int y = 0; y < ny; ++y) {
         if (y >= kYZS) mbar_wait(&empty[s], ph ^ 1);
-        mbar_expect_tx(&full[s], (uint32_t)(seg * 16 + nz * 16));
+        mbar_expect_tx(&full[s], (uint32_t)(seg * 16 + nz * (int)sizeof(C)));
         tma_3d(smem + s * slot_b, &tmap, 2 * o0, 0, row0 + y, &full[s]);
-        tma_row(smem + s * slot_b + seg * 16, phx + (long long)y * nz, (uint32_t)(nz * 16), &full[s]);
+        tma_row(smem + s * slot_b + seg * 16, phx + (long long)y * nz, (uint32_t)(nz * (int)sizeof(C)), &full[s]);
         if (++s == kYZS) { s = 0; ph ^= 1; }
       }
     }
@@ -303,27 +308,27 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
   const int ozr = has_r ? zr * kYZW + o : o, ozr1 = (has_r && !r_single) ? (zr + 1) * kYZW + o : o;
   const int pz0 = live ? z0 : 0, pz1 = has1 ? z1 : 0;          // Phi offsets in the slot's Phi row
   const int yst = nz * norb;  // element stride between y planes (< 2^31 per domain, validated)
-  double2* out0 = psi + (long long)dom * ng * norb + (long long)x * ny * yst + o0 + z0 * norb + o;
-  double2* out1 = out0 + norb;
+  V* out0 = psi + (long long)dom * ng * norb + (long long)x * ny * yst + o0 + z0 * norb + o;
+  V* out1 = out0 + norb;
 
   // K_z of plane y (slot s) for this thread's pair: the first E(Delta/2) on pairs m-1, m, m+1 (the
   // neighbours' outputs recomputed here), O(Delta) on the links (2m-1, 2m), (2m+1, 2m+2), then the
   // second E(Delta/2) on (2m, 2m+1).
-  auto kz = [&](int s, double2& w0, double2& w1) {
-    const double2* r = slot_psi(s);
-    const double2 a = r[oz0], b = r[oz1], vl = r[ozl], vl1 = r[ozl1], vr = r[ozr], vr1 = r[ozr1];
-    double2 e0, e1 = cz();
+  auto kz = [&](int s, V& w0, V& w1) {
+    const V* r = slot_psi(s);
+    const V a = r[oz0], b = r[oz1], vl = r[ozl], vl1 = r[ozl1], vr = r[ozr], vr1 = r[ozr1];
+    V e0, e1 = V{};
     if (has1) {
       e0 = lk_L<kS>(cz_.a1, cz_.u1, a, b);
       e1 = lk_R<kS>(cz_.a1, cz_.d1, a, b);
     } else {
       e0 = lk_S<kS>(cz_.s1, a);
     }
-    const double2 q0 = has_l ? lk_R<kS>(cz_.a2, cz_.d2, lk_R<kS>(cz_.a1, cz_.d1, vl, vl1), e0) : lk_S<kS>(cz_.s2, e0);
+    const V q0 = has_l ? lk_R<kS>(cz_.a2, cz_.d2, lk_R<kS>(cz_.a1, cz_.d1, vl, vl1), e0) : lk_S<kS>(cz_.s2, e0);
     if (has1) {
-      double2 q1;
+      V q1;
       if (has_r) {
-        const double2 r0 = r_single ? lk_S<kS>(cz_.s1, vr) : lk_L<kS>(cz_.a1, cz_.u1, vr, vr1);
+        const V r0 = r_single ? lk_S<kS>(cz_.s1, vr) : lk_L<kS>(cz_.a1, cz_.u1, vr, vr1);
         q1 = lk_L<kS>(cz_.a2, cz_.u2, e1, r0);
       } else {
         q1 = lk_S<kS>(cz_.s2, e1);
@@ -332,38 +337,43 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
       w1 = lk_R<kS>(cz_.a1, cz_.d1, q0, q1);
     } else {
       w0 = lk_S<kS>(cz_.s1, q0);
-      w1 = cz();
+      w1 = V{};
     }
   };
   // dep: computed from this warp's last loads of the slot (they must have returned: lfd_tma.cuh)
   auto release = [&](int s, double dep) { mbar_release(&empty[s], dep, (tid & 31) == 0); };
   // colE != nullptr: the largest biased FP64 exponent of Re / Im of each orbital's output, for the int8-digit
   // GEMM-1 that follows (its per-orbital power-of-two scale; nl_i8.cu) -- integer max on the high words
-  int me = 0;
-  auto trk = [&](double2 w) {
-    me = __vimax3_s32(me, __double2hiint(w.x) & 0x7ff00000, __double2hiint(w.y) & 0x7ff00000);
+  int me = 0, me2 = 0;  // (complex64 pairs: the exponents of the lane's two orbitals, FP64-biased)
+  auto trk = [&](V w) {
+    if constexpr (std::is_same<V, cf2>::value) {
+      me = max(me, exp64_of(w.a));
+      me2 = max(me2, exp64_of(w.b));
+    } else {
+      me = __vimax3_s32(me, __double2hiint(w.x) & 0x7ff00000, __double2hiint(w.y) & 0x7ff00000);
+    }
     return w;
   };
-  auto put0 = [&](int y, double2 f, double2 v) {
+  auto put0 = [&](int y, C f, V v) {
     if (act) out0[y * yst] = trk(cmul(f, v));
   };
-  auto put1 = [&](int y, double2 f, double2 v) {
+  auto put1 = [&](int y, C f, V v) {
     if (act && has1) out1[y * yst] = trk(cmul(f, v));
   };
 
-  LineMarch<kS> L0, L1;
+  LineMarch<kS, C, V> L0, L1;
   L0.init();
   L1.init();
   const int npairs = (ny + 1) >> 1;
   if (kFull && ny >= 4) {
     // periodic (even ny): pairs 0 and 1 peeled, then a steady loop without p / parity tests
-    double2 wa0, wa1, wb0, wb1;
+    V wa0, wa1, wb0, wb1;
     mbar_wait(&full[0], 0);
     kz(0, wa0, wa1);
     mbar_wait(&full[1], 0);
     kz(1, wb0, wb1);
-    release(0, wa0.x + wa1.x);
-    release(1, wb0.x + wb1.x);
+    release(0, dep_of(wa0) + dep_of(wa1));
+    release(1, dep_of(wb0) + dep_of(wb1));
     L0.first(cy, wa0, wb0);
     L1.first(cy, wa1, wb1);
     mbar_wait(&full[2], 0);
@@ -374,23 +384,23 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
     L1.second(cy, wa1, wb1);
     int s_prev = 2, s_a = 4;  // slot of plane 2p-2 and of plane 2p (kYZS is even: pairs never straddle)
     uint32_t ph_a = 0;
-    double2* o0p = out0 + 2 * yst;  // plane 2p-2
+    V* o0p = out0 + 2 * yst;  // plane 2p-2
     for (int p = 2; p < npairs; ++p) {
       mbar_wait(&full[s_a], ph_a);
       kz(s_a, wa0, wa1);
       mbar_wait(&full[s_a + 1], ph_a);
       kz(s_a + 1, wb0, wb1);
-      const double2* pa = slot_phi(s_prev);
-      const double2* pb = slot_phi(s_prev + 1);
-      const double2 fa0 = pa[pz0], fa1 = pa[pz1], fb0 = pb[pz0], fb1 = pb[pz1];
-      L0.steady(cy, wa0, wb0, [&](int k, double2 v) {
+      const C* pa = slot_phi(s_prev);
+      const C* pb = slot_phi(s_prev + 1);
+      const C fa0 = pa[pz0], fa1 = pa[pz1], fb0 = pb[pz0], fb1 = pb[pz1];
+      L0.steady(cy, wa0, wb0, [&](int k, V v) {
         if (act) o0p[k * yst] = trk(cmul(k == 0 ? fa0 : fb0, v));
       });
-      L1.steady(cy, wa1, wb1, [&](int k, double2 v) {
+      L1.steady(cy, wa1, wb1, [&](int k, V v) {
         if (act) o0p[k * yst + norb] = trk(cmul(k == 0 ? fa1 : fb1, v));
       });
-      release(s_prev, fa0.x + fa1.x);
-      release(s_prev + 1, fb0.x + fb1.x);
+      release(s_prev, dep_of(fa0) + dep_of(fa1));
+      release(s_prev + 1, dep_of(fb0) + dep_of(fb1));
       o0p += 2 * yst;
       s_prev = s_a;
       s_a += 2;
@@ -409,7 +419,7 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
       int s_b = s_a + 1;
       uint32_t ph_b = ph_a;
       if (s_b == kYZS) { s_b = 0; ph_b ^= 1; }
-      double2 wa0, wa1, wb0 = cz(), wb1 = cz();
+      V wa0, wa1, wb0 = V{}, wb1 = V{};
       mbar_wait(&full[s_a], ph_a);
       kz(s_a, wa0, wa1);
       if (hb) {
@@ -417,24 +427,24 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
         kz(s_b, wb0, wb1);
       }
       if (p == 0) {
-        release(s_a, wa0.x + wa1.x);
-        if (hb) release(s_b, wb0.x + wb1.x);
+        release(s_a, dep_of(wa0) + dep_of(wa1));
+        if (hb) release(s_b, dep_of(wb0) + dep_of(wb1));
       }
       // Phi of the planes this march step stores (2p-2 in slot s_prev, 2p-1 in the next slot)
       int s_pb = s_prev + 1;
       if (s_pb == kYZS) s_pb = 0;
-      double2 fa0 = cz(), fa1 = cz(), fb0 = cz(), fb1 = cz();
+      C fa0 = C{}, fa1 = C{}, fb0 = C{}, fb1 = C{};
       if (p >= 2) {
-        const double2* pa = slot_phi(s_prev);
-        const double2* pb = slot_phi(s_pb);
+        const C* pa = slot_phi(s_prev);
+        const C* pb = slot_phi(s_pb);
         fa0 = pa[pz0]; fa1 = pa[pz1];
         fb0 = pb[pz0]; fb1 = pb[pz1];
       }
-      L0.push(cy, p, wa0, wb0, hb, [&](int y, double2 v) { put0(y, y == ya - 2 ? fa0 : fb0, v); });
-      L1.push(cy, p, wa1, wb1, hb, [&](int y, double2 v) { put1(y, y == ya - 2 ? fa1 : fb1, v); });
+      L0.push(cy, p, wa0, wb0, hb, [&](int y, V v) { put0(y, y == ya - 2 ? fa0 : fb0, v); });
+      L1.push(cy, p, wa1, wb1, hb, [&](int y, V v) { put1(y, y == ya - 2 ? fa1 : fb1, v); });
       if (p >= 2) {
-        release(s_prev, fa0.x + fa1.x);
-        release(s_pb, fb0.x + fb1.x);
+        release(s_prev, dep_of(fa0) + dep_of(fa1));
+        release(s_pb, dep_of(fb0) + dep_of(fb1));
       }
       s_prev = s_a;
       s_a = s_b + 1;
@@ -443,31 +453,45 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
     }
   }
   // wrap: planes ny-2, ny-1 (or ny-1 for odd ny; their slots are released at the end) and 0, 1
-  const double2* phb = phx + pz0;
-  auto ph = [&](int y, int dz) { return (dz == 0 ? live : has1) ? __ldg(phb + y * nz + dz) : cz(); };
-  const double2 f00 = ph(0, 0), f01 = ph(0, 1), f10 = ph(1, 0), f11 = ph(1, 1);
-  const double2 fl0 = ph(ny - 1, 0), fl1 = ph(ny - 1, 1);
-  const double2 fm0 = ph(ny - 2, 0), fm1 = ph(ny - 2, 1);
+  const C* phb = phx + pz0;
+  auto ph = [&](int y, int dz) { return (dz == 0 ? live : has1) ? __ldg(phb + y * nz + dz) : C{}; };
+  const C f00 = ph(0, 0), f01 = ph(0, 1), f10 = ph(1, 0), f11 = ph(1, 1);
+  const C fl0 = ph(ny - 1, 0), fl1 = ph(ny - 1, 1);
+  const C fm0 = ph(ny - 2, 0), fm1 = ph(ny - 2, 1);
   auto pick0 = [&](int y) { return y == 0 ? f00 : y == 1 ? f10 : y == ny - 1 ? fl0 : fm0; };
   auto pick1 = [&](int y) { return y == 0 ? f01 : y == 1 ? f11 : y == ny - 1 ? fl1 : fm1; };
-  L0.template finish<kPer>(cy, ny, [&](int y, double2 v) { put0(y, pick0(y), v); });
-  L1.template finish<kPer>(cy, ny, [&](int y, double2 v) { put1(y, pick1(y), v); });
+  L0.template finish<kPer>(cy, ny, [&](int y, V v) { put0(y, pick0(y), v); });
+  L1.template finish<kPer>(cy, ny, [&](int y, V v) { put1(y, pick1(y), v); });
   if (colE) {  // max over this orbital's lanes (o = lane % 8), then one global atomicMax per (CTA, orbital)
     me = max(me, __shfl_xor_sync(0xffffffffu, me, 8));
     me = max(me, __shfl_xor_sync(0xffffffffu, me, 16));
-    if ((tid & 31) < kYZW && act) atomicMax(colE + (long long)dom * norb + o0 + o, me >> 20);
+    if constexpr (std::is_same<V, cf2>::value) {  // norb counts cf2 pairs here: orbitals 2 (o0 + o), + 1
+      me2 = max(me2, __shfl_xor_sync(0xffffffffu, me2, 8));
+      me2 = max(me2, __shfl_xor_sync(0xffffffffu, me2, 16));
+      if ((tid & 31) < kYZW && act) {
+        int* ce = colE + (long long)dom * 2 * norb + 2 * (o0 + o);
+        if (me > 0) atomicMax(ce, me);
+        if (me2 > 0) atomicMax(ce + 1, me2);
+      }
+    } else {
+      if ((tid & 31) < kYZW && act) atomicMax(colE + (long long)dom * norb + o0 + o, me >> 20);
+    }
   }
 }
 
-bool kin_yz_supported(const Geometry& g) { return g.nz <= 80; }
+// (SP: two complex64 orbitals per lane (cf2), so norb must be even; the Phi row of nz complex64 must be a
+// multiple of 16 bytes for its bulk copy: nz even)
+bool kin_yz_supported(const Geometry& g) { return g.nz <= 80 && (!g.sp || (g.norb % 2 == 0 && g.nz % 2 == 0)); }
 
 static size_t yz_smem(int nz) { return (size_t)kYZS * yz_slot_bytes(nz) + (size_t)kYZS * 16; }
 
 // Tensor map of Psi for k_kin_yz: 3-D view [ndom*nx*ny planes][nz rows][2*norb doubles], box
 // [1][nz][16 doubles] (one (x, y) plane segment of 8 orbitals), no swizzle (dense rows of 128 B).
-cudaError_t kin_yz_tensor_map(const Geometry& g, double2* psi, CUtensorMap* out) {
-  const uint64_t dims[3] = {(uint64_t)2 * g.norb, (uint64_t)g.nz, (uint64_t)g.ndom * g.nx * g.ny};
-  const uint64_t strides[2] = {(uint64_t)g.norb * 16, (uint64_t)g.nz * g.norb * 16};
+// (SP: the same bytes, [planes][nz rows][norb 8-byte elements = complex64], box 16 elements = 8 cf2 pairs)
+cudaError_t kin_yz_tensor_map(const Geometry& g, void* psi, CUtensorMap* out) {
+  const uint64_t esz = g.sp ? 8 : 16;  // bytes per complex value
+  const uint64_t dims[3] = {(uint64_t)g.norb * esz / 8, (uint64_t)g.nz, (uint64_t)g.ndom * g.nx * g.ny};
+  const uint64_t strides[2] = {(uint64_t)g.norb * esz, (uint64_t)g.nz * g.norb * esz};
   const uint32_t box[3] = {2 * kYZW, (uint32_t)g.nz, 1};
   return encode_tmap_f64(out, 3, psi, dims, strides, box);
 }
@@ -478,6 +502,10 @@ cudaError_t kin_yz_set_attributes() {
   if (e == cudaSuccess) e = cudaFuncSetAttribute(k_kin_yz<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(k_kin_yz<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(k_kin_yz<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(k_kin_yz<true, true, float2, cf2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(k_kin_yz<true, false, float2, cf2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(k_kin_yz<false, true, float2, cf2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(k_kin_yz<false, false, float2, cf2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
   return e;
 }
 
@@ -489,6 +517,28 @@ cudaError_t launch_kin_yz(const Geometry& g, const CUtensorMap* tmap, double2* p
   const size_t sm = yz_smem(g.nz);
 #define LFD_KYZ(P, K) \
   launch_k(k_kin_yz<P, K>, grid, threads, sm, st, *tmap, psi, coef, phi, g.nx, g.ny, g.nz, g.norb, nchunks, g.ng, colE)
+  if (g.bc == 0) {
+    if (scaled) LFD_KYZ(true, true); else LFD_KYZ(true, false);
+  } else {
+    if (scaled) LFD_KYZ(false, true); else LFD_KYZ(false, false);
+  }
+#undef LFD_KYZ
+  return cudaGetLastError();
+}
+
+// SP: the same pass on complex64 Psi, two orbitals (16 bytes) per lane, FP32 arithmetic; colE gets the FP64-biased
+// exponents of each complex64 orbital
+cudaError_t launch_kin_yz_sp(const Geometry& g, const CUtensorMap* tmap, float2* psi, const DomCoef* coef,
+                             const float2* phi, bool scaled, cudaStream_t st, int* colE) {
+  const int nv = g.norb / 2;  // cf2 pairs per grid point
+  const int nchunks = (nv + kYZW - 1) / kYZW;
+  const int threads = ((((g.nz + 1) / 2) * kYZW + 31) / 32 + 1) * 32;
+  dim3 grid(g.nx * nchunks, g.ndom);
+  const size_t sm = yz_smem(g.nz);
+  cf2* pv = reinterpret_cast<cf2*>(psi);
+#define LFD_KYZ(P, K)                                                                                            \
+  launch_k(k_kin_yz<P, K, float2, cf2>, grid, threads, sm, st, *tmap, pv, coef, phi, g.nx, g.ny, g.nz, nv, nchunks, \
+           g.ng, colE)
   if (g.bc == 0) {
     if (scaled) LFD_KYZ(true, true); else LFD_KYZ(true, false);
   } else {

@@ -102,11 +102,13 @@ cudaError_t launch_kin_sp(const Geometry& g, float2* psi, const DomCoef* coef, c
 
 // Fused pass Psi <- Phi . K_y K_z Psi (one read + write of Psi; nz <= 80).
 bool kin_yz_supported(const Geometry& g);
-cudaError_t kin_yz_tensor_map(const Geometry& g, double2* psi, CUtensorMap* out);
+cudaError_t kin_yz_tensor_map(const Geometry& g, void* psi, CUtensorMap* out);
 // colE != nullptr: atomicMax of the biased FP64 exponent of every output Re / Im per orbital into
 // colE[dom][norb] (the per-orbital scale of the int8-digit GEMM-1, nl_i8.cu)
 cudaError_t launch_kin_yz(const Geometry& g, const CUtensorMap* tmap, double2* psi, const DomCoef* coef,
                           const double2* phi, bool scaled, cudaStream_t st, int* colE = nullptr);
+cudaError_t launch_kin_yz_sp(const Geometry& g, const CUtensorMap* tmap, float2* psi, const DomCoef* coef,
+                             const float2* phi, bool scaled, cudaStream_t st, int* colE);
 cudaError_t kin_yz_set_attributes();
 
 // GEMM-1 split-K: part[dom][split][mrows][ncols] (complex) = sum over the split's grid rows of
