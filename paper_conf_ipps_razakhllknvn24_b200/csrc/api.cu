@@ -687,7 +687,7 @@ lfd_status density_into(lfd_ctx* c, double* rho, double* j, double* Jmac, const 
   LFD_TRY(launch(c, LFD_K_DENSITY, "k_density", [&] { return lfd::launch_density(c->g, a, c->dmaps, c->stream); }));
   if (Jmac)
     LFD_TRY(launch(c, LFD_K_JREDUCE, "k_jreduce",
-                   [&] { return lfd::launch_jreduce(c->g, a.jline, Jmac, c->stream); }));
+                   [&] { return lfd::launch_jreduce(c->g, a.jline, lfd::density_blocks_used(c->g, c->dmaps), Jmac, c->stream); }));
   return LFD_OK;
 }
 
@@ -1379,7 +1379,7 @@ lfd_status lfd_energy(lfd_ctx* c, double* E) {
   LFD_TRY(density_into(c, c->at<double>(c->L.rhostage), nullptr, nullptr, c->at<long long>(c->L.base),
                        (long long)g.ny * g.nz, g.nz, g.ng, true));
   return launch(c, LFD_K_ENERGY, "k_energy_final", [&] {
-    return lfd::launch_energy_final(g, c->at<double>(c->L.epart), lfd::density_blocks(g), C,
+    return lfd::launch_energy_final(g, c->at<double>(c->L.epart), lfd::density_blocks_used(g, c->dmaps), C,
                                     c->at<double>(c->L.D), c->at<double>(c->L.occ), E, c->stream);
   });
 }
@@ -1408,6 +1408,11 @@ lfd_status lfd_set_occupations(lfd_ctx* c, const double* occ) {
                                   cudaMemcpyHostToDevice, c->stream);
   if (e != cudaSuccess) return cuda_fail(c, e, "copy occ");
   e = lfd::density_maps_set_active(c->dmaps, c->g, c->psi, active_orbitals(c->g, occ));
+  if (e == cudaErrorNotSupported) {  // more active orbitals than the y-marching kernel takes: the generic kernel
+    lfd::density_maps_destroy(c->dmaps);
+    c->dmaps = nullptr;
+    e = cudaSuccess;
+  }
   if (e != cudaSuccess) return cuda_fail(c, e, "density tensor map");
   release_graphs(c);  // captured graphs hold the density kernel's tensor maps by value
   return LFD_OK;

@@ -308,232 +308,301 @@ __global__ void __launch_bounds__(kDensThreads) k_density_tma(Geometry g, DensAr
 }
 
 // ------------------------------------------------------------------------------------------------
-// y-marching variant (norb <= 128; the bench shape). CTA = (px consecutive x planes, z chunk of zc
+// y-marching kernel (the bench shape; nact <= kQMaxAct). CTA = (px consecutive x planes, z chunk of zc
 // points, y chunk, domain): it walks y and needs, at step y, the z-line segments of its own points
-// (x0..x0+px-1, y, z0..z0+zc) plus their z+1 halo points, the next lines (y+1) for the y links and, for
-// the x links, the lines of its own next plane -- or, for the last plane, of plane x0+px (the next CTA's
-// first plane: an L2 hit, so HBM sees each line once and the L2->SM traffic is (px+1)/px of it). A
-// producer warp brings each segment with one tiled TMA tensor copy (the halo point is a second, 1-point
-// copy) into two rings (own lines: kYOwn slots of px segments, x+px lines: kYXp slots) with full/empty
-// mbarriers; the own line y+1 stays resident for the next step. kSub lanes per point split the orbitals
-// and the 7 per-point sums are shuffle reductions with the occupation weights (kept in shared memory).
+// (x0..x0+px-1, y, z0..z0+zc-1) plus their z+1 halo points, the next lines (y+1) for the y links and, for the
+// x links, the lines of its own next plane -- or, for the last plane, of plane x0+px (the next CTA's first
+// plane, read about when that CTA reads it: an L2 hit, so HBM sees each line about once). A producer warp
+// brings each segment with one tiled TMA tensor copy (the halo point is a second, 1-point copy) into two rings
+// (own lines: nso slots of px segments, x+px lines: nsx slots) with full/empty mbarriers; the own line y+1 stays
+// resident as the next step's own line.
+//
+// Lanes: 4 per point (lane = 8 q + p: point p of the warp's 8, orbital quarter q owning s = q, q+4, q+8, ...),
+// so a lane does 8 orbitals per step at nact = 32 and the per-point sums need a 2-level shuffle reduce-scatter.
+// Bank conflicts: the 8 lanes of an LDS.128 phase read the same orbital of 8 consecutive points, so each smem row
+// (one point, the active orbitals) is padded to an odd number of 16-byte units (a multiple of 16 bytes + 16 for
+// complex64, whose 16-lane phases take q = 0, 1): the TMA box starts `pad` orbitals BEFORE orbital 0, where the
+// tensor is out of bounds and the copy zero-fills -- padding without HBM traffic. Every LDS then has a
+// compile-time offset from a per-step row pointer.
 // ------------------------------------------------------------------------------------------------
-// ring depths (lines): DensMaps::nso / nsx; the own line y+1 stays resident for the y links
-constexpr int kYMaxThreads = 512;  // up to 60 points x kSub + the producer warp
+constexpr int kQMaxWarps = 8;                        // consumer warps per CTA (8 points each; <= 168 registers)
+constexpr int kQMaxThreads = (kQMaxWarps + 1) * 32;  // + the producer warp
+constexpr int kQMaxAct = 120;                        // box inner dim <= 256 elements (FP64: 2 (nact + pad))
+constexpr int kQPf = 4;                              // lines prefetched into L2 ahead of the ring loads
 
 struct DensMaps {
-  CUtensorMap seg;   // box [1][zc][2*nact]: a z-line segment of zc points, the active orbitals
-  CUtensorMap one;   // box [1][1][2*nact]: the z+1 halo point
+  CUtensorMap seg;   // box [1][zc][E (nact + pad)] at orbital -pad: a z-line segment, each row padded in front
+  CUtensorMap one;   // box [1][1][E (nact + pad)]: the z+1 halo point
   int zc;            // points per CTA and plane (divides nz)
   int px;            // x planes per CTA (divides nx)
   int nyc;           // y chunks per (plane group, z chunk)
   int nact;          // active orbitals: 1 + the last index with f != 0 (f = 0 contributes exactly 0)
+  int pad;           // zero-filled orbitals in front of each shared-memory row (odd row length in 16-byte units)
   int esz;           // bytes per complex value: 16 (complex128) or 8 (complex64, the SP variant)
   int nso, nsx;      // ring depths: own lines, x+px lines
+  int blocks;        // CTAs per domain
 };
 
-// shared-memory layout of the y-marching kernel (every TMA destination 128-byte aligned): an own slot
-// holds px (segment, halo point) pairs
-struct YLayout {
-  size_t seg_b, halo_b, pl_b, own_b, xp_b, fsh_off, bar_off, total;
-  __host__ __device__ YLayout(int zc, int norb, int px, int esz, int nso, int nsx) {  // esz: bytes per complex value
-    seg_b = ((size_t)zc * norb * esz + 127) & ~(size_t)127;
-    halo_b = ((size_t)norb * esz + 127) & ~(size_t)127;
+__host__ __device__ inline uint32_t q_al128(uint32_t b) { return (b + 127u) & ~127u; }
+
+// shared-memory layout (every TMA destination 128-byte aligned): an own slot holds px (segment, halo point) pairs
+struct QLayout {
+  uint32_t rs, seg_b, halo_b, pl_b, own_b, xp_b, fsh_off, bar_off, total;
+  __host__ __device__ QLayout(int zc, int px, int nact, int pad, int esz, int nso, int nsx) {
+    rs = (uint32_t)((nact + pad) * esz);
+    seg_b = q_al128((uint32_t)zc * rs);
+    halo_b = q_al128(rs);
     pl_b = seg_b + halo_b;
-    own_b = px * pl_b;
+    own_b = (uint32_t)px * pl_b;
     xp_b = seg_b;
-    fsh_off = nso * own_b + nsx * xp_b;
-    bar_off = fsh_off + (((size_t)norb * 8 + 15) & ~(size_t)15);
-    total = bar_off + (2 * nso + 2 * nsx) * 8;
+    fsh_off = (uint32_t)nso * own_b + (uint32_t)nsx * xp_b;
+    if (fsh_off < 5u * kQMaxWarps * 8u * 8u) fsh_off = 5u * kQMaxWarps * 8u * 8u;  // the per-CTA partials reuse it
+    bar_off = fsh_off + (((uint32_t)nact * 8u + 15u) & ~15u);
+    total = bar_off + (uint32_t)(2 * nso + 2 * nsx) * 8u;
   }
 };
 
-struct YShape {
-  int zc, px, nyc, nso, nsx;
+// pad: FP64 rows of an odd number of 16-byte units; complex64 rows of 2 (mod 4) 8-byte units (a 16-byte multiple).
+// The box must start 16-byte aligned (the TMA faults otherwise): an even pad for complex64, whose active count is
+// rounded up to even first (density_maps_shape; the extra orbital has f = 0).
+static int q_pad(int nact, int esz) {
+  if (esz == 16) return (nact & 1) ? 2 : 1;
+  return (nact % 4 == 0) ? 2 : 0;
+}
+
+struct QShape {
+  int zc, px, nyc, nso, nsx, pad;
 };
 
-// The shape measured best on C2 inside the step loop (bench, ncu launch lists): 18 points per plane and CTA,
-// one y chunk, rings of 6 own / 3 x+1 lines. Sweeps of density calls alone (tools/dens_sweep.py,
-// profiles/r02_dens_sweep*.jsonl) favour smaller shapes with 4 resident CTAs per SM (12 points, 2 y chunks, rings
-// 3 / 2, <= 80 registers: 0.058 vs 0.066 ms there) because repeated calls find part of Psi in L2; inside the step
-// that shape measured 59.5 vs 56.7 us (ncu launch list r02h). A build with -DLFD_TUNING_KNOBS reads
-// LFD_DENS_ZCMAX / _PX / _YC / _OWN / _XP at lfd_init for such sweeps; the library proper reads no environment.
-static YShape ymarch_shape(const Geometry& g) {
-  YShape sh{0, 1, 1, 6, 3};
-  if (g.norb > 128) return sh;
-  if (g.sp && (g.norb & 1)) return sh;  // TMA global strides must be multiples of 16 bytes
-  int zmax = 18, pxmax = 1, yc = 1;
-#ifdef LFD_TUNING_KNOBS
-  constexpr int kYOwnMax = 8, kYXpMax = 4;
-  if (const char* v = std::getenv("LFD_DENS_ZCMAX")) zmax = std::max(1, std::min(60, std::atoi(v)));
-  if (const char* v = std::getenv("LFD_DENS_PX")) pxmax = std::max(1, std::atoi(v));
-  if (const char* v = std::getenv("LFD_DENS_YC")) yc = std::max(1, std::atoi(v));
-  if (const char* v = std::getenv("LFD_DENS_OWN")) sh.nso = std::max(3, std::min(kYOwnMax, std::atoi(v)));
-  if (const char* v = std::getenv("LFD_DENS_XP")) sh.nsx = std::max(1, std::min(kYXpMax, std::atoi(v)));
-#endif
+static int q_num_sms() {
+  int dev = 0, n = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess ||
+      n <= 0) {
+    cudaGetLastError();
+    n = 148;
+  }
+  return n;
+}
+
+// Shape search: lanes used (px zc of 8 W), CTA balance over the resident slots (SMs x CTAs per SM by shared
+// memory, threads and 168 registers per thread), the y+1 line each y chunk re-reads, warps straddling two planes
+// and consumer warps per SM (>= 8); among equals, more ring bytes per SM. The DRAM latency is covered by the
+// L2 prefetches (kQPf lines ahead), so the rings only need to cover L2 hits.
+static QShape q_shape(const Geometry& g, int nact, int nsm) {
+  QShape best{0, 1, 1, 3, 2, 1};
   const int esz = g.sp ? 8 : 16;
-  int px = 1;
-  for (int d = std::min(pxmax, g.nx); d >= 1; --d)
-    if (g.nx % d == 0) { px = d; break; }
-  for (int nzc = 1; nzc <= g.nz; ++nzc) {
-    if (g.nz % nzc) continue;
-    const int zc = g.nz / nzc;
-    if (zc > zmax || zc * px * kSub + 32 > kYMaxThreads) continue;
-    if (YLayout(zc, g.norb, px, esz, sh.nso, sh.nsx).total <= 200 * 1024) { sh.zc = zc; break; }
-  }
-  if (sh.zc == 0 && px > 1) {  // fall back to one plane per CTA
-    sh.px = 1;
-    for (int nzc = 1; nzc <= g.nz; ++nzc) {
-      if (g.nz % nzc) continue;
-      const int zc = g.nz / nzc;
-      if (zc > std::min(zmax, 40)) continue;
-      if (YLayout(zc, g.norb, 1, esz, sh.nso, sh.nsx).total <= 200 * 1024) { sh.zc = zc; break; }
+  if (nact > kQMaxAct) return best;
+  if (g.sp && (g.norb & 1)) return best;  // TMA global strides must be multiples of 16 bytes
+  const int pad = q_pad(nact, esz);
+  best.pad = pad;
+  double bscore = -1.0, binfl = 0.0;
+  int fzc = 0, fpx = 0, fyc = 0, fso = 0, fsx = 0;
+#ifdef LFD_TUNING_KNOBS
+  if (const char* v = std::getenv("LFD_DENS_ZC")) fzc = std::atoi(v);
+  if (const char* v = std::getenv("LFD_DENS_PX")) fpx = std::atoi(v);
+  if (const char* v = std::getenv("LFD_DENS_YC")) fyc = std::atoi(v);
+  if (const char* v = std::getenv("LFD_DENS_OWN")) fso = std::atoi(v);
+  if (const char* v = std::getenv("LFD_DENS_XP")) fsx = std::atoi(v);
+#endif
+  for (int px = 1; px <= std::min(8, g.nx); ++px) {
+    if (g.nx % px || (fpx && px != fpx)) continue;
+    for (int zc = 1; zc <= g.nz; ++zc) {
+      if (g.nz % zc || (fzc && zc != fzc)) continue;
+      const int pts = px * zc, W = (pts + 7) / 8;
+      if (W > kQMaxWarps) continue;
+      const double util = (double)pts / (8.0 * W);
+      if (util < 0.7) continue;
+      for (int nso = 3; nso <= 6; ++nso) {
+        if (fso && nso != fso) continue;
+        for (int nsx = 2; nsx <= 3; ++nsx) {
+          if (fsx && nsx != fsx) continue;
+          const QLayout L(zc, px, nact, pad, esz, nso, nsx);
+          if (L.total > 200u * 1024u) continue;
+          const int cps = std::min({(int)((228u * 1024u) / (L.total + 1024u)), 2048 / ((W + 1) * 32),
+                                    65536 / (168 * 32 * (W + 1)), 32});
+          if (cps < 1) continue;
+          const double R = (double)nsm * cps;
+          const int base = (g.nx / px) * (g.nz / zc) * g.ndom;
+          for (int nyc = 1; nyc <= std::min(8, std::max(1, g.ny / 2)); ++nyc) {
+            if (fyc && nyc != fyc) continue;
+            const double T = (double)base * nyc;
+            const double bal = T / (std::ceil(T / R) * R);
+            const double yeff = (double)g.ny / (double)(g.ny + nyc - 1);
+            const double infl = (double)cps * ((nso - 2) * (double)L.own_b + (nsx - 1) * (double)L.xp_b);
+            const double warps = (double)cps * W;
+            const double straddle = (px > 1 && zc % 8) ? 0.9 : 1.0;  // warps across two planes: bank conflicts
+            const double sc = util * bal * yeff * straddle * std::min(1.0, warps / 8.0);
+            if (sc > bscore + 1e-9 || (sc > bscore - 1e-9 && infl > binfl)) {
+              bscore = sc;
+              binfl = infl;
+              best = QShape{zc, px, nyc, nso, nsx, pad};
+            }
+          }
+        }
+      }
     }
-    px = 1;
   }
-  sh.px = px;
-  sh.nyc = std::max(1, std::min(yc, g.ny / 2 > 0 ? g.ny / 2 : 1));
-  return sh;
+  return best;
 }
 
 template <bool kPer, int kIt, class C = double2>
-__global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constant__ DensMaps mp, Geometry g,
+__global__ void __launch_bounds__(kQMaxThreads, 1) k_density_q(const __grid_constant__ DensMaps mp, Geometry g,
                                                             DensArgs a) {
   pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
   pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
   extern __shared__ __align__(128) unsigned char dsm[];
-  const int norb = mp.nact, zc = mp.zc, px = mp.px;  // smem rows hold the nact active orbitals of each point
-  const int kYOwn = mp.nso, kYXp = mp.nsx;
-  const YLayout Ly(zc, norb, px, (int)sizeof(C), kYOwn, kYXp);
-  auto own_seg = [&](int s, int p) { return reinterpret_cast<C*>(dsm + s * Ly.own_b + p * Ly.pl_b); };
-  auto halo_of = [&](int s, int p) {
-    return reinterpret_cast<C*>(dsm + s * Ly.own_b + p * Ly.pl_b + Ly.seg_b);
-  };
-  auto xp_slot = [&](int s) { return reinterpret_cast<C*>(dsm + kYOwn * Ly.own_b + s * Ly.xp_b); };
+  const int nact = mp.nact, zc = mp.zc, px = mp.px, nso = mp.nso, nsx = mp.nsx;
+  const QLayout Ly(zc, px, nact, mp.pad, (int)sizeof(C), nso, nsx);
+  const uint32_t rs = Ly.rs;
+  auto own_seg = [&](int s, int p) { return dsm + s * Ly.own_b + p * Ly.pl_b; };
+  auto halo_of = [&](int s, int p) { return dsm + s * Ly.own_b + p * Ly.pl_b + Ly.seg_b; };
+  auto xp_slot = [&](int s) { return dsm + nso * Ly.own_b + s * Ly.xp_b; };
   double* fsh = reinterpret_cast<double*>(dsm + Ly.fsh_off);
   uint64_t* bars = reinterpret_cast<uint64_t*>(dsm + Ly.bar_off);
-  uint64_t *ofull = bars, *oempty = bars + kYOwn, *xfull = bars + 2 * kYOwn, *xempty = xfull + kYXp;
-  __shared__ double jsh[5][kYMaxThreads / kSub];
+  uint64_t *ofull = bars, *oempty = bars + nso, *xfull = bars + 2 * nso, *xempty = xfull + nsx;
   const int dom = blockIdx.y;
   const int nzc = g.nz / zc, nyc = mp.nyc;
   const int yci = blockIdx.x % nyc, xz = blockIdx.x / nyc;
   const int xg = xz / nzc, z0 = (xz - xg * nzc) * zc;
   const int xb = xg * px;  // first plane of the CTA
   const int y0 = (int)(((long long)yci * g.ny) / nyc), ycnt = (int)(((long long)(yci + 1) * g.ny) / nyc) - y0;
-  const bool per = kPer;
-  const bool has_xn = per || xb + px < g.nx;  // plane xb + px exists (the x+1 of the last plane)
+  const bool has_xn = kPer || xb + px < g.nx;  // plane xb + px exists (the x+1 of the last plane)
+  const bool xring = has_xn;
   const int xnext = (xb + px == g.nx) ? 0 : xb + px;
   const bool last_chunk = z0 + zc == g.nz;
-  const int nconsw = (zc * px * kSub + 31) >> 5;
+  const int nconsw = (zc * px + 7) >> 3;
   const int tid = threadIdx.x;
   // own lines y0 .. y0+ycnt-1 plus the y+1 halo line (y = 0 again past the periodic wrap)
-  const int nown = (per || y0 + ycnt < g.ny) ? ycnt + 1 : ycnt;
+  const int nown = (kPer || y0 + ycnt < g.ny) ? ycnt + 1 : ycnt;
+  const int E = (int)sizeof(C) / 8;  // 8-byte tensor elements per complex value
   if (tid == 0) {
-    for (int s = 0; s < kYOwn; ++s) { mbar_init(&ofull[s], 1); mbar_init(&oempty[s], nconsw); }
-    for (int s = 0; s < kYXp; ++s) { mbar_init(&xfull[s], 1); mbar_init(&xempty[s], nconsw); }
+    for (int s = 0; s < nso; ++s) { mbar_init(&ofull[s], 1); mbar_init(&oempty[s], nconsw); }
+    for (int s = 0; s < nsx; ++s) { mbar_init(&xfull[s], 1); mbar_init(&xempty[s], nconsw); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  for (int s = tid; s < norb; s += blockDim.x) fsh[s] = a.occ[(long long)dom * g.norb + s];
+  for (int s = tid; s < nact; s += blockDim.x) fsh[s] = a.occ[(long long)dom * g.norb + s];
   __syncthreads();
 
   if (tid >= nconsw * 32) {  // producer warp
     if (tid == nconsw * 32) {
       const int rowxn = (dom * g.nx + xnext) * g.ny;
+      const int c0 = -E * mp.pad;  // the row's zero-filled front padding (out of bounds: no HBM traffic)
+      const bool halo = !last_chunk || kPer;  // z+1 halo point: z0 + zc, or z = 0 (periodic wrap)
+      const uint32_t own_tx = (uint32_t)(px * (zc + (halo ? 1 : 0))) * rs, xp_tx = (uint32_t)zc * rs;
+      int so = 0, sx = 0;
+      uint32_t pho = 0, phx = 0;
+      // L2 prefetch of the own / x+px lines kQPf lines ahead of their shared-memory loads: the DRAM latency is
+      // covered without ring depth (shared memory), the ring only waits for L2 hits
+      auto prefetch = [&](int k) {
+        if (k < nown) {
+          const int yy = (y0 + k == g.ny) ? 0 : y0 + k;
+          for (int p = 0; p < px; ++p) tma_prefetch_3d(&mp.seg, c0, z0, (dom * g.nx + xb + p) * g.ny + yy);
+        }
+        if (has_xn && k < ycnt) tma_prefetch_3d(&mp.seg, c0, z0, rowxn + y0 + k);
+      };
+      for (int k = 0; k < kQPf; ++k) prefetch(nso + k);
       auto issue_own = [&](int k) {  // own lines y0 + k (== ny: plane 0 again) of the px planes
-        const int s = k % kYOwn;
-        if (k >= kYOwn) mbar_wait(&oempty[s], (uint32_t)(((k / kYOwn) - 1) & 1));
+        if (k >= nso) mbar_wait(&oempty[so], pho ^ 1u);
+        prefetch(k + kQPf);
         const int yy = (y0 + k == g.ny) ? 0 : y0 + k;
-        const bool halo = !last_chunk || per;  // z+1 halo point: z0 + zc, or z = 0 (periodic wrap)
-        mbar_expect_tx(&ofull[s], (uint32_t)(px * (zc + (halo ? 1 : 0)) * norb * (int)sizeof(C)));
+        mbar_expect_tx(&ofull[so], own_tx);
         for (int p = 0; p < px; ++p) {
           const int row = (dom * g.nx + xb + p) * g.ny + yy;
-          tma_3d(own_seg(s, p), &mp.seg, 0, z0, row, &ofull[s]);
-          if (halo) tma_3d(halo_of(s, p), &mp.one, 0, last_chunk ? 0 : z0 + zc, row, &ofull[s]);
+          tma_3d(own_seg(so, p), &mp.seg, c0, z0, row, &ofull[so]);
+          if (halo) tma_3d(halo_of(so, p), &mp.one, c0, last_chunk ? 0 : z0 + zc, row, &ofull[so]);
         }
+        if (++so == nso) { so = 0; pho ^= 1u; }
       };
       auto issue_xp = [&](int k) {
-        const int s = k % kYXp;
-        if (k >= kYXp) mbar_wait(&xempty[s], (uint32_t)(((k / kYXp) - 1) & 1));
-        mbar_expect_tx(&xfull[s], (uint32_t)(zc * norb * (int)sizeof(C)));
-        tma_3d(xp_slot(s), &mp.seg, 0, z0, rowxn + y0 + k, &xfull[s]);
+        if (k >= nsx) mbar_wait(&xempty[sx], phx ^ 1u);
+        mbar_expect_tx(&xfull[sx], xp_tx);
+        tma_3d(xp_slot(sx), &mp.seg, c0, z0, rowxn + y0 + k, &xfull[sx]);
+        if (++sx == nsx) { sx = 0; phx ^= 1u; }
       };
-      // keep the rings full: kYOwn own lines and kYXp x+1 lines in flight (line k + depth reuses the slot
-      // the consumers release after step k)
-      for (int k = 0; k < kYOwn && k < nown; ++k) issue_own(k);
-      if (has_xn)
-        for (int k = 0; k < kYXp && k < ycnt; ++k) issue_xp(k);
+      // keep the rings full: line k + depth reuses the slot the consumers release after step k
+      for (int k = 0; k < nso && k < nown; ++k) issue_own(k);
+      if (xring)
+        for (int k = 0; k < nsx && k < ycnt; ++k) issue_xp(k);
       for (int k = 0; k < ycnt; ++k) {
-        if (k + kYOwn < nown) issue_own(k + kYOwn);
-        if (has_xn && k + kYXp < ycnt) issue_xp(k + kYXp);
+        if (k + nso < nown) issue_own(k + nso);
+        if (xring && k + nsx < ycnt) issue_xp(k + nsx);
       }
     }
     return;
   }
 
-  const int q = tid % kSub, pa = tid / kSub;
+  const int lane = tid & 31, q = lane >> 3;
+  const int pa = (tid >> 5) * 8 + (lane & 7);
   const int pl = pa / zc, pt = pa - pl * zc;  // plane within the CTA, point within the z chunk
   const bool valid = pl < px;
-  const int x = xb + (valid ? pl : 0);
-  const bool has_x = per || x + 1 < g.nx;
-  const int z = z0 + pt;
+  const int plr = valid ? pl : 0, ptr = valid ? pt : 0;
+  const int x = xb + plr, z = z0 + ptr;
+  const bool has_x = valid && (kPer || x + 1 < g.nx);
   const bool has_z = valid && (kPer || z + 1 < g.nz);
   const DomCoef* cf = a.coef + dom;
   const double2 ex = cf->eth[0], ey = cf->eth[1], ez = cf->eth[2];
   const double ihx = cf->inv_h[0], ihy = cf->inv_h[1], ihz = cf->inv_h[2];
   const double w2x = ihx * ihx, w2y = ihy * ihy, w2z = ihz * ihz;
-  const int ptr = valid ? pt : 0;
-  // occupations of this lane's orbitals s = q, q + kSub, ... in registers
-  constexpr int kItMax = 128 / kSub;
-  const int nit = (norb - q + kSub - 1) / kSub;
-  double fr[kIt > 0 ? kIt : kItMax];
+  const uint32_t lo = (uint32_t)(mp.pad + q) * (uint32_t)sizeof(C);  // this lane's first orbital (s = q) in a row
+  const uint32_t orow = (uint32_t)ptr * rs + lo;
+  const bool zin = ptr + 1 < zc;  // z+1 in the segment (else the halo point)
+  // occupations of this lane's orbitals s = q + 4 i in registers (kIt > 0: nact == 4 kIt exactly)
+  double fr[kIt > 0 ? kIt : 1];
 #pragma unroll
-  for (int i = 0; i < (kIt > 0 ? kIt : kItMax); ++i) fr[i] = (i < nit) ? fsh[q + i * kSub] : 0.0;
-  // lane q of a point ends up holding the full sum of value q >> 1: 0 rho, 1 jx, 2 jy, 3 jz
-  const int vsel = q >> 1;
+  for (int i = 0; i < (kIt > 0 ? kIt : 1); ++i) fr[i] = kIt > 0 ? fsh[q + 4 * i] : 0.0;
+  const int nit = (nact - q + 3) >> 2;  // this lane's orbital count (kIt == 0)
   double jacc = 0.0, ekin = 0.0, eloc = 0.0;
   const long long rbase = a.base[dom], jb = a.j ? a.jbase[dom] : 0;  // hoisted global loads
+  int so = 0, sn = nso > 1 ? 1 : 0, sx = 0;
+  uint32_t pho = 0, phn = 0, phx = 0;
   for (int k = 0; k < ycnt; ++k) {
     const int y = y0 + k;
     const bool has_y = valid && (kPer || y + 1 < g.ny);
-    const int so = k % kYOwn, sn = (k + 1) % kYOwn, sx = k % kYXp;
-    mbar_wait(&ofull[so], (uint32_t)((k / kYOwn) & 1));
-    if (k + 1 < nown) mbar_wait(&ofull[sn], (uint32_t)(((k + 1) / kYOwn) & 1));
-    if (has_xn) mbar_wait(&xfull[sx], (uint32_t)((k / kYXp) & 1));
-    const int plr = valid ? pl : 0;
-    const C* O = own_seg(so, plr) + ptr * norb;
-    const C* Oz = (ptr + 1 < zc) ? O + norb : halo_of(so, plr);  // point z+1
-    const C* N = own_seg(sn, plr) + ptr * norb;
-    const C* X = (plr + 1 < px ? own_seg(so, plr + 1) : xp_slot(sx)) + ptr * norb;  // plane x+1
+    mbar_wait(&ofull[so], pho);
+    if (k + 1 < nown) mbar_wait(&ofull[sn], phn);
+    if (xring) mbar_wait(&xfull[sx], phx);
+    const unsigned char* O = own_seg(so, plr) + orow;
+    const unsigned char* Oz = zin ? O + rs : halo_of(so, plr) + lo;  // point z+1
+    const unsigned char* N = own_seg(sn, plr) + orow;
+    const unsigned char* X = (plr + 1 < px ? own_seg(so, plr + 1) : xp_slot(sx)) + orow;  // plane x+1
     // per-lane partial sums over this lane's orbitals: rho and the three link products P_d = sum f
     // conj(psi_r) psi_{r+e_d} (f folded into fv = f psi_r)
     double rho = 0.0, pxr = 0.0, pxi = 0.0, pyr = 0.0, pyi = 0.0, pzr = 0.0, pzi = 0.0;
     if (valid) {
-#pragma unroll
-      for (int i = 0; i < (kIt > 0 ? kIt : kItMax); ++i) {
-        if (kIt == 0 && i >= nit) break;
-        const int sidx = q + i * kSub;
-        const double2 v = to_d2(O[sidx]);  // FP64 accumulation (also for complex64 Psi)
-        const double2 fv = make_double2(fr[i] * v.x, fr[i] * v.y);
+      auto orb = [&](int i, double f) {
+        const uint32_t off = (uint32_t)i * 4u * (uint32_t)sizeof(C);
+        const double2 v = to_d2(*reinterpret_cast<const C*>(O + off));  // FP64 accumulation (also for complex64 Psi)
+        const double2 fv = make_double2(f * v.x, f * v.y);
         rho = fma(fv.x, v.x, fma(fv.y, v.y, rho));
         if (kPer || has_x) {
-          const double2 w = to_d2(X[sidx]);
+          const double2 w = to_d2(*reinterpret_cast<const C*>(X + off));
           pxr = fma(fv.x, w.x, fma(fv.y, w.y, pxr));
           pxi = fma(fv.x, w.y, fma(-fv.y, w.x, pxi));
         }
         if (kPer || has_y) {
-          const double2 w = to_d2(N[sidx]);
+          const double2 w = to_d2(*reinterpret_cast<const C*>(N + off));
           pyr = fma(fv.x, w.x, fma(fv.y, w.y, pyr));
           pyi = fma(fv.x, w.y, fma(-fv.y, w.x, pyi));
         }
         if (kPer || has_z) {
-          const double2 w = to_d2(Oz[sidx]);
+          const double2 w = to_d2(*reinterpret_cast<const C*>(Oz + off));
           pzr = fma(fv.x, w.x, fma(fv.y, w.y, pzr));
           pzi = fma(fv.x, w.y, fma(-fv.y, w.x, pzi));
         }
+      };
+      if (kIt > 0) {
+#pragma unroll
+        for (int i = 0; i < (kIt > 0 ? kIt : 1); ++i) orb(i, fr[i]);
+      } else {
+#pragma unroll 4
+        for (int i = 0; i < nit; ++i) orb(i, fsh[q + 4 * i]);
       }
     }
     // this warp is done with own line y and x+1 line y (once its loads have returned: lfd_tma.cuh)
-    mbar_release2(&oempty[so], &xempty[sx], has_xn, ((rho + pxr) + (pyr + pzr)) + (pxi + pyi + pzi), (tid & 31) == 0);
+    mbar_release2(&oempty[so], &xempty[sx], xring, ((rho + pxr) + (pyr + pzr)) + (pxi + pyi + pzi), lane == 0);
+    if (++so == nso) { so = 0; pho ^= 1u; }
+    if (++sn == nso) { sn = 0; phn ^= 1u; }
+    if (xring && ++sx == nsx) { sx = 0; phx ^= 1u; }
     // the currents and the kinetic energy density are linear in the P_d: form them per lane first
     // (Im(e^{i theta} P) = cos Im P + sin Re P, Re(e^{i theta} P) = cos Re P - sin Im P)
     const double jx = (kPer || has_x) ? (ex.x * pxi + ex.y * pxr) * ihx : 0.0;
@@ -546,46 +615,43 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
       if (kPer || has_z) ek -= w2z * (ez.x * pzr - ez.y * pzi);
       ekin += ek;
     }
-    // reduce-scatter of (rho, jx, jy, jz) over the kSub = 8 lanes of the point (fixed order)
+    // reduce-scatter of (rho, jx, jy, jz) over the 4 lanes of the point (lanes xor 16, then xor 8; fixed order)
     double u0, u1;
     {
-      const bool hi = (q & 4) != 0;  // lanes 4..7 keep (jy, jz), lanes 0..3 keep (rho, jx)
+      const bool hi = (q & 2) != 0;  // q = 2, 3 keep (jy, jz); q = 0, 1 keep (rho, jx)
       const double s0 = hi ? rho : jy, s1 = hi ? jx : jz;
       const double k0 = hi ? jy : rho, k1 = hi ? jz : jx;
-      u0 = k0 + __shfl_xor_sync(0xffffffffu, s0, 4);
-      u1 = k1 + __shfl_xor_sync(0xffffffffu, s1, 4);
+      u0 = k0 + __shfl_xor_sync(0xffffffffu, s0, 16);
+      u1 = k1 + __shfl_xor_sync(0xffffffffu, s1, 16);
     }
-    double val;
-    {
-      const bool hi = (q & 2) != 0;  // keep the second of the two
-      const double sd = hi ? u0 : u1, kp = hi ? u1 : u0;
-      val = kp + __shfl_xor_sync(0xffffffffu, sd, 2);
-    }
-    val += __shfl_xor_sync(0xffffffffu, val, 1);
-    // lanes 2v, 2v+1 now hold value v: 0 rho, 1 jx, 2 jy, 3 jz
-    if (valid && (q & 1) == 0) {
+    const bool odd = (q & 1) != 0;  // keep the second of the two
+    const double val = (odd ? u1 : u0) + __shfl_xor_sync(0xffffffffu, odd ? u0 : u1, 8);
+    // lane q now holds value q of its point: 0 rho, 1 jx, 2 jy, 3 jz
+    if (valid) {
       const long long o = (long long)x * a.sx + (long long)y * a.sy + z;
-      if (vsel == 0) {
+      if (q == 0) {
         a.rho[rbase + o] = val;
         if (a.epart) eloc += a.v[(long long)dom * g.ng + ((long long)x * g.ny + y) * g.nz + z] * val;
       } else {
         jacc += val;
-        if (a.j) a.j[jb + o + (vsel - 1) * a.jstride] = val;
+        if (a.j) a.j[jb + o + (q - 1) * a.jstride] = val;
       }
     }
   }
-  // per-CTA sums in a fixed order: J components from lanes q = 2, 4, 6 of every point, energies from all
-  const int pts = nconsw * 32 / kSub;
-  if (q == 2 || q == 4 || q == 6) jsh[q / 2 - 1][pa] = jacc;
-  double ekp = ekin;  // sum the kinetic partials over the 8 lanes of the point (fixed tree)
-  ekp += __shfl_xor_sync(0xffffffffu, ekp, 4);
-  ekp += __shfl_xor_sync(0xffffffffu, ekp, 2);
-  ekp += __shfl_xor_sync(0xffffffffu, ekp, 1);
+  // per-CTA sums in a fixed order: J components from lanes q = 1, 2, 3 of every point, energies from all; the
+  // partials go to the (consumed) ring space once every consumer warp is done with it
+  const int pts = nconsw * 8;
+  double(*jsh)[kQMaxWarps * 8] = reinterpret_cast<double(*)[kQMaxWarps * 8]>(dsm);
+  asm volatile("bar.sync 1, %0;" ::"r"(nconsw * 32) : "memory");
+  if (q > 0) jsh[q - 1][pa] = jacc;
+  double ekp = ekin;  // sum the kinetic partials over the 4 lanes of the point (fixed tree)
+  ekp += __shfl_xor_sync(0xffffffffu, ekp, 16);
+  ekp += __shfl_xor_sync(0xffffffffu, ekp, 8);
   if (q == 0) {
     jsh[3][pa] = ekp;
     jsh[4][pa] = eloc;
   }
-  asm volatile("bar.sync 1, %0;" ::"r"(nconsw * 32));  // consumer warps only
+  asm volatile("bar.sync 1, %0;" ::"r"(nconsw * 32) : "memory");  // consumer warps only
   if (a.epart && tid >= 3 && tid < 5) {  // (warp 0: there may be a single consumer warp)
     double t = 0.0;
     for (int k = 0; k < pts; ++k) t += jsh[tid][k];
@@ -598,82 +664,94 @@ __global__ void __launch_bounds__(kYMaxThreads) k_density_y(const __grid_constan
   }
 }
 
-static size_t ymarch_smem(const DensMaps& m) { return YLayout(m.zc, m.nact, m.px, m.esz, m.nso, m.nsx).total; }
+static size_t q_smem(const DensMaps& m) { return QLayout(m.zc, m.px, m.nact, m.pad, m.esz, m.nso, m.nsx).total; }
 
-// Psi as a 3-D tensor of 8-byte elements [rows][nz][norb * esz / 8] (the TMA only moves bytes: a
-// complex64 value is one 8-byte element, a complex128 value two).
-static cudaError_t density_maps_encode(DensMaps* m, const Geometry& g, const double2* psi, int nact) {
+// Psi as a 3-D tensor of 8-byte elements [rows][nz][norb * esz / 8] (the TMA only moves bytes: a complex64 value
+// is one 8-byte element, a complex128 value two); the box spans nact + pad values from value -pad.
+static cudaError_t density_maps_encode(DensMaps* m, const Geometry& g, const double2* psi) {
   const uint64_t w = (uint64_t)m->esz / 8;
   const uint64_t dims[3] = {w * g.norb, (uint64_t)g.nz, (uint64_t)g.ndom * g.nx * g.ny};
   const uint64_t str[2] = {(uint64_t)g.norb * m->esz, (uint64_t)g.nz * g.norb * m->esz};
-  const uint32_t b2[3] = {(uint32_t)(w * nact), (uint32_t)m->zc, 1};
-  const uint32_t b3[3] = {(uint32_t)(w * nact), 1, 1};
+  const uint32_t b2[3] = {(uint32_t)(w * (m->nact + m->pad)), (uint32_t)m->zc, 1};
+  const uint32_t b3[3] = {(uint32_t)(w * (m->nact + m->pad)), 1, 1};
   cudaError_t e = encode_tmap_f64(&m->seg, 3, psi, dims, str, b2);
   if (e == cudaSuccess) e = encode_tmap_f64(&m->one, 3, psi, dims, str, b3);
-  if (e == cudaSuccess) m->nact = nact;
   return e;
 }
 
+static bool density_maps_shape(DensMaps* m, const Geometry& g, int nact) {
+  if (g.sp && (nact & 1) && nact < g.norb) ++nact;  // complex64: an even active count (q_pad)
+  const QShape sh = q_shape(g, nact, q_num_sms());
+  if (sh.zc == 0) return false;
+  m->zc = sh.zc; m->px = sh.px; m->nyc = sh.nyc; m->nso = sh.nso; m->nsx = sh.nsx; m->pad = sh.pad;
+  m->nact = nact;
+  m->esz = g.sp ? 8 : 16;
+  m->blocks = (g.nx / sh.px) * (g.nz / sh.zc) * sh.nyc;
+  return true;
+}
+
 DensMaps* density_maps_create(const Geometry& g, const double2* psi, int nact) {
-  const YShape sh = ymarch_shape(g);
-  if (sh.zc == 0) return nullptr;
+  nact = std::min(std::max(nact, 1), g.norb);
   DensMaps* m = new (std::nothrow) DensMaps;
   if (!m) return nullptr;
-  m->zc = sh.zc;
-  m->px = sh.px;
-  m->nyc = sh.nyc;
-  m->nso = sh.nso;
-  m->nsx = sh.nsx;
-  m->esz = g.sp ? 8 : 16;
-  if (density_maps_encode(m, g, psi, std::min(std::max(nact, 1), g.norb)) != cudaSuccess) {
+  if (!density_maps_shape(m, g, nact) || density_maps_encode(m, g, psi) != cudaSuccess) {
     delete m;
     return nullptr;
   }
   return m;
 }
 
+// The active-orbital count changed (lfd_set_occupations): new shape and descriptors. A count past kQMaxAct keeps the
+// old shape and its (larger) active set -- the extra orbitals have f = 0 and add exactly zero.
 cudaError_t density_maps_set_active(DensMaps* m, const Geometry& g, const double2* psi, int nact) {
   nact = std::min(std::max(nact, 1), g.norb);
   if (!m || m->nact == nact) return cudaSuccess;
-  return density_maps_encode(m, g, psi, nact);
+  DensMaps t = *m;
+  if (!density_maps_shape(&t, g, nact)) {
+    if (nact < m->nact) return cudaSuccess;
+    return cudaErrorNotSupported;
+  }
+  const cudaError_t e = density_maps_encode(&t, g, psi);
+  if (e == cudaSuccess) *m = t;
+  return e;
 }
 
 void density_maps_destroy(DensMaps* m) { delete m; }
 
 int density_smem_bytes(int norb) { return kRingSlots * kPlanePts * norb * 16; }
 
-int density_blocks(const Geometry& g) {
-  const YShape sh = ymarch_shape(g);
-  if (sh.zc > 0) return (g.nx / sh.px) * (g.nz / sh.zc) * sh.nyc;
+static int fallback_blocks(const Geometry& g) {
   const int ntz = (g.nz + kTZ - 1) / kTZ, nty = (g.ny + kTY - 1) / kTY, nxc = (g.nx + kXC - 1) / kXC;
   return ntz * nty * nxc;
 }
 
+// workspace bound on the CTAs per domain (per-CTA partial sums): any y-marching shape has at most nx nz 8 CTAs
+int density_blocks(const Geometry& g) {
+  return std::max(fallback_blocks(g), g.nx * g.nz * std::min(8, std::max(1, g.ny / 2)));
+}
+
+int density_blocks_used(const Geometry& g, const DensMaps* m) { return m ? m->blocks : fallback_blocks(g); }
+
 cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps* maps, cudaStream_t st) {
-  dim3 grid(density_blocks(g), g.ndom);
   if (maps) {
-    const int threads = ((maps->zc * maps->px * kSub + 31) / 32 + 1) * 32;
-    const size_t sm = ymarch_smem(*maps);
+    dim3 grid(maps->blocks, g.ndom);
+    const int threads = ((maps->zc * maps->px + 7) / 8 + 1) * 32;
+    const size_t sm = q_smem(*maps);
+    const int n = maps->nact;
     if (maps->esz == 8) {  // SP variant (complex64 Psi)
-      if (g.bc == 0 && maps->nact == 32)
-        launch_k(k_density_y<true, 4, float2>, grid, threads, sm, st, *maps, g, a);
-      else if (g.bc == 0)
-        launch_k(k_density_y<true, 0, float2>, grid, threads, sm, st, *maps, g, a);
-      else
-        launch_k(k_density_y<false, 0, float2>, grid, threads, sm, st, *maps, g, a);
+      if (g.bc == 0 && n == 32) launch_k(k_density_q<true, 8, float2>, grid, threads, sm, st, *maps, g, a);
+      else if (g.bc == 0 && n == 64) launch_k(k_density_q<true, 16, float2>, grid, threads, sm, st, *maps, g, a);
+      else if (g.bc == 0) launch_k(k_density_q<true, 0, float2>, grid, threads, sm, st, *maps, g, a);
+      else launch_k(k_density_q<false, 0, float2>, grid, threads, sm, st, *maps, g, a);
       return cudaGetLastError();
     }
-    if (g.bc == 0 && maps->nact == 64)
-      launch_k(k_density_y<true, 8>, grid, threads, sm, st, *maps, g, a);
-    else if (g.bc == 0 && maps->nact == 32)
-      launch_k(k_density_y<true, 4>, grid, threads, sm, st, *maps, g, a);
-    else if (g.bc == 0)
-      launch_k(k_density_y<true, 0>, grid, threads, sm, st, *maps, g, a);
-    else
-      launch_k(k_density_y<false, 0>, grid, threads, sm, st, *maps, g, a);
+    if (g.bc == 0 && n == 32) launch_k(k_density_q<true, 8>, grid, threads, sm, st, *maps, g, a);
+    else if (g.bc == 0 && n == 64) launch_k(k_density_q<true, 16>, grid, threads, sm, st, *maps, g, a);
+    else if (g.bc == 0) launch_k(k_density_q<true, 0>, grid, threads, sm, st, *maps, g, a);
+    else launch_k(k_density_q<false, 0>, grid, threads, sm, st, *maps, g, a);
     return cudaGetLastError();
   }
-  if (ymarch_shape(g).zc > 0) return cudaErrorInvalidValue;  // the block layout expects the y-marching kernel
+  dim3 grid(fallback_blocks(g), g.ndom);
   const int ntz = (g.nz + kTZ - 1) / kTZ, nty = (g.ny + kTY - 1) / kTY;
   if (a.psi_sp)
     launch_k(k_density<float2>, grid, kDensThreads, 0, st, g, a, ntz, nty, kXC);
@@ -688,11 +766,9 @@ cudaError_t density_set_attributes() {
   cudaError_t e = cudaFuncSetAttribute(k_density_tma, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        density_smem_bytes(kMaxNorbTma));
   if (e != cudaSuccess) return e;
-  for (auto f : {k_density_y<true, 8>, k_density_y<true, 4>, k_density_y<true, 0>, k_density_y<false, 0>}) {
-    e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024);
-    if (e != cudaSuccess) return e;
-  }
-  for (auto f : {k_density_y<true, 4, float2>, k_density_y<true, 0, float2>, k_density_y<false, 0, float2>}) {
+  for (auto f : {k_density_q<true, 8>, k_density_q<true, 16>, k_density_q<true, 0>, k_density_q<false, 0>,
+                 k_density_q<true, 8, float2>, k_density_q<true, 16, float2>, k_density_q<true, 0, float2>,
+                 k_density_q<false, 0, float2>}) {
     e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024);
     if (e != cudaSuccess) return e;
   }
@@ -719,8 +795,8 @@ __global__ void __launch_bounds__(256) k_jreduce(const double* __restrict__ jlin
   if (threadIdx.x < 3) Jmac[dom * 3 + threadIdx.x] = sh[threadIdx.x][0] * inv_ng;
 }
 
-cudaError_t launch_jreduce(const Geometry& g, const double* jline, double* Jmac, cudaStream_t st) {
-  launch_k(k_jreduce, g.ndom, 256, 0, st, jline, density_blocks(g), 1.0 / (double)g.ng, Jmac);
+cudaError_t launch_jreduce(const Geometry& g, const double* jline, int blocks, double* Jmac, cudaStream_t st) {
+  launch_k(k_jreduce, g.ndom, 256, 0, st, jline, blocks, 1.0 / (double)g.ng, Jmac);
   return cudaGetLastError();
 }
 

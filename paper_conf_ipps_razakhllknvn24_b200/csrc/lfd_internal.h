@@ -245,9 +245,10 @@ DensMaps* density_maps_create(const Geometry& g, const double2* psi, int nact); 
 cudaError_t density_maps_set_active(DensMaps* m, const Geometry& g, const double2* psi, int nact);
 void density_maps_destroy(DensMaps* m);
 cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps* maps, cudaStream_t st);
-int density_blocks(const Geometry& g);
+int density_blocks(const Geometry& g);  // workspace bound on the CTAs per domain
+int density_blocks_used(const Geometry& g, const DensMaps* m);  // CTAs per domain of launch_density
 cudaError_t density_set_attributes();
-cudaError_t launch_jreduce(const Geometry& g, const double* jline, double* Jmac, cudaStream_t st);
+cudaError_t launch_jreduce(const Geometry& g, const double* jline, int blocks, double* Jmac, cudaStream_t st);
 
 // calc_energy / remap_occ reductions (energy.cu)
 cudaError_t launch_energy_final(const Geometry& g, const double* epart, int blocks, const double2* C,

@@ -434,21 +434,6 @@ def test_set_occupations_changes_active_orbitals():
     ctx.close()
 
 
-@pytest.mark.parametrize("knobs", [{"LFD_DENS_PX": "2", "LFD_DENS_YC": "3", "LFD_DENS_ZCMAX": "6"},
-                                   {"LFD_DENS_PX": "3", "LFD_DENS_YC": "2", "LFD_DENS_ZCMAX": "8"},
-                                   {"LFD_DENS_PX": "1", "LFD_DENS_YC": "5", "LFD_DENS_ZCMAX": "24"}])
-@pytest.mark.parametrize("name", ["C1", "P2z"])
-def test_density_kernel_shapes(name, knobs, monkeypatch):
-    """The y-marching density kernel's tiling knobs (planes per CTA, y chunks, points per plane) change the
-    work decomposition only: rho, j and J match the oracle for each (periodic and zero BC, ragged chunks)."""
-    for k, v in knobs.items():
-        monkeypatch.setenv(k, v)
-    w = workload(name).with_(laser=True)
-    x = make_inputs(w, seed=71)
-    A = lambda n: midpoint_A(w, n)  # noqa: E731
-    assert_parity(w, run_gpu(w, x, 2, A), run_ref(w, x, 2, A))
-
-
 def test_c2_contract_100_steps():
     """The north-star contract at the bench configuration: C2 (70x70x72, 64 orbitals, 64 projectors, laser;
     the default int8-digit GEMMs that bench.py times) for 100 steps. The oracle runs the same 100 steps on 6

@@ -1,6 +1,7 @@
 """Shape sweep of the y-marching density kernel on C2 (A/B only; needs a build with LFD_NVCC_DEFINES=-DLFD_TUNING_KNOBS):
 for each combination of the tuning knobs
-(LFD_DENS_ZCMAX, LFD_DENS_YC, LFD_DENS_OWN, LFD_DENS_XP, read at lfd_init), the device time per density call.
+(LFD_DENS_ZC, LFD_DENS_PX, LFD_DENS_YC, LFD_DENS_OWN, LFD_DENS_XP, read at lfd_init; a combination the shape
+search rejects falls back to its best admissible shape), the device time per density call.
   python tools/dens_sweep.py [--sp]"""
 import itertools
 import json
@@ -24,7 +25,8 @@ psi = torch.from_numpy(x.psi0.astype(dt)).to(dev)
 proj = torch.from_numpy(x.proj.astype(dt)).to(dev)
 rho = torch.empty((1, w.ngrid), dtype=torch.float64, device=dev)
 J = torch.empty((1, 3), dtype=torch.float64, device=dev)
-grid = {"LFD_DENS_ZCMAX": [9, 12, 18], "LFD_DENS_YC": [1, 2, 3, 5, 7], "LFD_DENS_OWN": [3, 4], "LFD_DENS_XP": [2, 3]}
+grid = {"LFD_DENS_ZC": [8, 12, 24, 36], "LFD_DENS_PX": [1, 2], "LFD_DENS_YC": [1, 2, 4], "LFD_DENS_OWN": [3, 4, 5],
+        "LFD_DENS_XP": [2, 3]}
 keys = list(grid)
 for vals in itertools.product(*[grid[k] for k in keys]):
     for k, v in zip(keys, vals):

@@ -1,0 +1,13 @@
+#!/bin/bash
+# density: tests, cold probe, bench default, launch list, then in-step shapes with the tuning build
+set -u
+TAG=${1:-dens4}
+bash tools/gpu_dens3.sh $TAG
+LFD_NVCC_DEFINES=-DLFD_TUNING_KNOBS python -c "from paper_conf_ipps_razakhllknvn24_b200 import build as b; b.build(force=True)" > gpurun_out/${TAG}_tbuild.log 2>&1
+for sh in "24 1 2 5 0" "24 1 2 4 0" "24 1 2 6 0" "24 1 2 3 2" "12 2 2 4 2" "36 1 2 4 0" "72 1 2 4 0" "72 1 2 5 0" "8 1 2 6 0"; do
+  set -- $sh
+  LFD_DENS_ZC=$1 LFD_DENS_PX=$2 LFD_DENS_YC=$3 LFD_DENS_OWN=$4 LFD_DENS_XP=$5 timeout 200 python bench.py --no-cpu-baseline --no-e2e --no-sc --no-sp --no-dmma --no-small --steps 50 > gpurun_out/${TAG}_b.json 2>/dev/null
+  python -c "
+import json; d=json.load(open('gpurun_out/${TAG}_b.json')); k=d['kernels']['density']
+print('shape $sh', 'step', round(d['ms_per_step'],4), 'dens', round(k['ms_per_launch'],4), round(k['frac'],3))"
+done
