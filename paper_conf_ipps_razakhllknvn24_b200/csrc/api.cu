@@ -325,6 +325,10 @@ struct lfd_ctx {
   lfd::DensMaps* dmaps = nullptr;  // TMA descriptors of Psi for the density kernel
   lfd::FxMaps* fxm = nullptr;      // TMA descriptors of the fused GEMM-2 + x pass (nullptr: not used)
   bool scaled = true;     // scaled pair form of the stencil (else the general 2x2 form: some cos(tau t) < 1/2)
+  // lfd_set_vector_potential (ndom <= kCoefFuse) only records A; the coefficient tables are written by the next
+  // phase kernel (lfd_set_potential) or, before any other kernel, by k_coef (launch())
+  bool a_pending = false;
+  double a_pend[3 * lfd::kCoefFuse];
   std::string err = "no error";
   // density-current global layout cache
   std::vector<long long> gbase_host;
@@ -398,8 +402,13 @@ void prof_flush(lfd_ctx* c) {
   c->nslot = 0;
 }
 
+lfd_status flush_A(lfd_ctx* c);
 template <class F>
 lfd_status launch(lfd_ctx* c, int kid, const char* name, F&& f) {
+  if (c->a_pending && kid != LFD_K_PHASE) {  // every other kernel may read the coefficients
+    const lfd_status fs = flush_A(c);
+    if (fs != LFD_OK) return fs;
+  }
   ProfSlot* s = nullptr;
   if (c->prof) {
     if (c->nslot == c->slots.size()) {
@@ -476,8 +485,15 @@ cudaError_t gemm1_any(lfd_ctx* c, const lfd::Gemm1Args& a) {
 
 // Phi from v in the context's precision (vcopy as lfd::launch_phase).
 cudaError_t phase_any(lfd_ctx* c, const double* v, double* vcopy) {
-  if (c->g.sp) return lfd::launch_phase_sp(c->g, v, c->phi32(), vcopy, c->scaled, c->stream);
-  return lfd::launch_phase(c->g, v, c->phi(), vcopy, c->scaled, c->stream);
+  lfd::CoefFuse cf{};
+  if (c->a_pending) {  // the pending coefficient tables in the same launch
+    for (int i = 0; i < 3 * c->g.ndom; ++i) cf.A[i / 3][i % 3] = c->a_pend[i];
+    cf.count = c->g.ndom;
+    cf.coef = c->coef();
+    c->a_pending = false;
+  }
+  if (c->g.sp) return lfd::launch_phase_sp(c->g, v, c->phi32(), vcopy, c->scaled, c->stream, &cf);
+  return lfd::launch_phase(c->g, v, c->phi(), vcopy, c->scaled, c->stream, &cf);
 }
 
 // GEMM-2 of a nonlocal factor: Psi <- (Psi + B C') diag(n), C' and n from the workspace; with out != nullptr
@@ -664,6 +680,7 @@ lfd_status project(lfd_ctx* c, const double2* A, int mrows, double2* out) {
 }
 
 lfd_status set_A(lfd_ctx* c, const double* A) {
+  c->a_pending = false;
   thread_local lfd::CoefParams tp;  // 12 KB kernel-parameter block (A captured by value)
   for (int d0 = 0; d0 < c->g.ndom; d0 += lfd::kCoefMaxPerLaunch) {
     const int cnt = std::min(lfd::kCoefMaxPerLaunch, c->g.ndom - d0);
@@ -673,6 +690,11 @@ lfd_status set_A(lfd_ctx* c, const double* A) {
                    [&] { return lfd::launch_coef(c->g, tp, d0, cnt, c->coef(), c->stream); }));
   }
   return LFD_OK;
+}
+
+lfd_status flush_A(lfd_ctx* c) {
+  c->a_pending = false;
+  return set_A(c, c->a_pend);
 }
 
 lfd_status density_into(lfd_ctx* c, double* rho, double* j, double* Jmac, const long long* base_dev, long long sx,
@@ -871,6 +893,7 @@ lfd_status get_graph(lfd_ctx* c, int K, double* rho, bool dens, lfd_ctx::Graph**
     cudaError_t e = cudaStreamCreateWithFlags(&c->cap_stream, cudaStreamNonBlocking);
     if (e != cudaSuccess) return cuda_fail(c, e, "cudaStreamCreate (graph capture)");
   }
+  if (c->a_pending) LFD_TRY(flush_A(c));  // (not into the captured graph)
   lfd_ctx::Graph gr;
   gr.K = K; gr.cv0 = c->c_valid; gr.rho = rho; gr.dens = dens;
   cudaStream_t orig = c->stream;
@@ -1200,8 +1223,14 @@ lfd_status lfd_set_vector_potential(lfd_ctx* c, const double* A) {
   for (int i = 0; i < 3 * c->g.ndom; ++i)
     if (!std::isfinite(A[i])) return fail(c, LFD_EINVAL, "A must be finite");
   DeviceGuard dg(c->device);
+  if (c->g.ndom <= lfd::kCoefFuse) {  // recorded now (by value), applied by the next kernel launch
+    std::copy(A, A + 3 * c->g.ndom, c->a_pend);
+    c->a_pending = true;
+    return LFD_OK;
+  }
   return set_A(c, A);
 }
+
 
 lfd_status lfd_step(lfd_ctx* c, int32_t nsteps) {
   LFD_TRY(check_ctx(c));

@@ -69,11 +69,13 @@ cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int co
 // Phi(r) = e^{-i (Delta/2) v_loc(r)} (Strang placement of the potential, reading R7), times the
 // constant sqrt(g) of the scaled pair form (1 for the general form).
 // The kernel also keeps a copy of v_loc for lfd_energy (vcopy may alias v: then it is not written).
+// With cf.count > 0 the first block also writes the coefficient tables of a pending lfd_set_vector_potential.
 template <class C>
 __global__ void k_phase(const double* __restrict__ v, C* __restrict__ phi, double* vcopy, long long n,
-                        double half_dt, double2 sg) {
+                        double half_dt, double2 sg, CoefFuse cf, double hx, double hy, double hz) {
   pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
   pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
+  if (blockIdx.x == 0 && threadIdx.x < cf.count) cf.coef[threadIdx.x] = make_coef(cf.A[threadIdx.x], hx, hy, hz, 2.0 * half_dt);
   long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   const double vi = v[i];
@@ -107,18 +109,24 @@ static double2 scaled_sqrt_g(const Geometry& g) {
 }
 
 cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, double* vcopy, bool scaled,
-                         cudaStream_t st) {
+                         cudaStream_t st, const CoefFuse* cf) {
   long long n = g.ng * g.ndom;
   const double2 sg = scaled ? scaled_sqrt_g(g) : make_double2(1.0, 0.0);
-  launch_k(k_phase<double2>, (unsigned)((n + 255) / 256), 256, 0, st, v, phi, vcopy, n, 0.5 * g.dt, sg);
+  CoefFuse c{};
+  if (cf) c = *cf;
+  launch_k(k_phase<double2>, (unsigned)((n + 255) / 256), 256, 0, st, v, phi, vcopy, n, 0.5 * g.dt, sg, c, g.hx, g.hy,
+           g.hz);
   return cudaGetLastError();
 }
 
 cudaError_t launch_phase_sp(const Geometry& g, const double* v, float2* phi, double* vcopy, bool scaled,
-                            cudaStream_t st) {
+                            cudaStream_t st, const CoefFuse* cf) {
   long long n = g.ng * g.ndom;
   const double2 sg = scaled ? scaled_sqrt_g(g) : make_double2(1.0, 0.0);
-  launch_k(k_phase<float2>, (unsigned)((n + 255) / 256), 256, 0, st, v, phi, vcopy, n, 0.5 * g.dt, sg);
+  CoefFuse c{};
+  if (cf) c = *cf;
+  launch_k(k_phase<float2>, (unsigned)((n + 255) / 256), 256, 0, st, v, phi, vcopy, n, 0.5 * g.dt, sg, c, g.hx, g.hy,
+           g.hz);
   return cudaGetLastError();
 }
 

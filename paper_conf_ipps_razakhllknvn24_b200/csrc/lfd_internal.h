@@ -82,10 +82,18 @@ cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int co
                         cudaStream_t st);
 cudaError_t launch_coef_dev(const Geometry& g, const double* A, DomCoef* coef, cudaStream_t st);
 // Phi = e^{-i (Delta/2) v} (times sqrt(g) when the scaled pair form is used, kin.cu).
+// The coefficient table of a pending lfd_set_vector_potential (up to kCoefFuse domains), computed by the phase
+// kernel that runs next (one launch instead of two; count = 0: none pending).
+constexpr int kCoefFuse = 8;
+struct CoefFuse {
+  double A[kCoefFuse][3];
+  int count;
+  DomCoef* coef;
+};
 cudaError_t launch_phase(const Geometry& g, const double* v, double2* phi, double* vcopy, bool scaled,
-                         cudaStream_t st);
+                         cudaStream_t st, const CoefFuse* cf = nullptr);
 cudaError_t launch_phase_sp(const Geometry& g, const double* v, float2* phi, double* vcopy, bool scaled,
-                            cudaStream_t st);
+                            cudaStream_t st, const CoefFuse* cf = nullptr);
 // True when the scaled pair form applies (cos(tau t_d) >= 1/2 for every axis and tau).
 bool kin_scaled_ok(const Geometry& g);
 

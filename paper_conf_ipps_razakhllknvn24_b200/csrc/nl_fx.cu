@@ -358,7 +358,7 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
         const double* sg = lsig(b) + x0;
 #pragma unroll
         for (int c = 0; c < kFxXg; ++c) {
-          if (c < nxc) *ps = fma(nf, *ps, scale_pow2(fa[c], sg[c], tau));
+          if (c < nxc) *ps = fma(nf, *ps, fa[c] * (sg[c] * tau));  // (powers of two: exact scaling)
           ps += ld2;
         }
       }
@@ -396,22 +396,23 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
       if (split) {
         LineMarch<kS> M;
         M.init();
-        const uint32_t ls = (uint32_t)norb * 16;
-        uint32_t la = smem_addr(L) + (uint32_t)(2 * p0) * ls;
-        uint32_t lf = smem_addr(lphi(b)) + (uint32_t)(2 * p0) * 16;  // Phi (the x pass's pre-phase)
+        // plain shared-memory loads (ordered by the named barriers' memory clobbers, free to be scheduled early)
+        const double2* la = L + (2 * p0) * norb;
+        const double2* lf = lphi(b) + 2 * p0;  // Phi (the x pass's pre-phase)
         if (active) {
-          M.first(cf, cmul(ld_sh2(lf), ld_sh2(la)), cmul(ld_sh2(lf + 16), ld_sh2(la + ls)));
-          la += 2 * ls;
-          lf += 32;
-          M.second(cf, cmul(ld_sh2(lf), ld_sh2(la)), cmul(ld_sh2(lf + 16), ld_sh2(la + ls)));
-          la += 2 * ls;
-          lf += 32;
+          M.first(cf, cmul(lf[0], la[0]), cmul(lf[1], la[norb]));
+          la += 2 * norb;
+          lf += 2;
+          M.second(cf, cmul(lf[0], la[0]), cmul(lf[1], la[norb]));
+          la += 2 * norb;
+          lf += 2;
           double2* o = out + (long long)(2 * p0 + 2) * xs;
+#pragma unroll 2
           for (int q = p0 + 2; q < p1; ++q) {
-            const double2 a = cmul(ld_sh2(lf), ld_sh2(la)), c = cmul(ld_sh2(lf + 16), ld_sh2(la + ls));
+            const double2 a = cmul(lf[0], la[0]), c = cmul(lf[1], la[norb]);
             M.steady(cf, a, c, [&](int k, double2 v) { o[k * xs] = v; });
-            la += 2 * ls;
-            lf += 32;
+            la += 2 * norb;
+            lf += 2;
             o += 2 * xs;
           }
         }

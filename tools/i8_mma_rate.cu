@@ -146,7 +146,8 @@ int main() {
   int sms; cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
   long long* d; cudaMalloc(&d, sizeof(long long) * 256);
   run<16, false>(sms, d); run<32, false>(sms, d); run<64, false>(sms, d); run<128, false>(sms, d); run<256, false>(sms, d);
-  run<16, true>(sms, d); run<32, true>(sms, d); run<64, true>(sms, d); run<128, true>(sms, d); run<256, true>(sms, d);
+  run<16, true>(sms, d); run<32, true>(sms, d); run<64, true>(sms, d); run<80, true>(sms, d); run<96, true>(sms, d);
+  run<128, true>(sms, d); run<160, true>(sms, d); run<256, true>(sms, d); run<80, false>(sms, d);
   cudaMalloc(&d, sizeof(long long) * 2048);
   runpat(sms, d, 0); runpat(sms, d, 4); runpat(sms, d, 16);
   return 0;
