@@ -328,7 +328,6 @@ __global__ void __launch_bounds__(kDensThreads) k_density_tma(Geometry g, DensAr
 constexpr int kQMaxWarps = 8;                        // consumer warps per CTA (8 points each; <= 168 registers)
 constexpr int kQMaxThreads = (kQMaxWarps + 1) * 32;  // + the producer warp
 constexpr int kQMaxAct = 120;                        // box inner dim <= 256 elements (FP64: 2 (nact + pad))
-constexpr int kQPf = 4;                              // lines prefetched into L2 ahead of the ring loads
 
 struct DensMaps {
   CUtensorMap seg;   // box [1][zc][E (nact + pad)] at orbital -pad: a z-line segment, each row padded in front
@@ -386,8 +385,8 @@ static int q_num_sms() {
 
 // Shape search: lanes used (px zc of 8 W), CTA balance over the resident slots (SMs x CTAs per SM by shared
 // memory, threads and 168 registers per thread), the y+1 line each y chunk re-reads, warps straddling two planes
-// and consumer warps per SM (>= 8); among equals, more ring bytes per SM. The DRAM latency is covered by the
-// L2 prefetches (kQPf lines ahead), so the rings only need to cover L2 hits.
+// and consumer warps per SM (>= 8); among equals, more ring bytes per SM. (L2 tensor prefetches of lines ahead
+// of the ring loads measured slower in the step: C2 48.8 -> 55.9 us at 4 lines ahead.)
 static QShape q_shape(const Geometry& g, int nact, int nsm) {
   QShape best{0, 1, 1, 3, 2, 1};
   const int esz = g.sp ? 8 : 16;
@@ -491,19 +490,8 @@ __global__ void __launch_bounds__(kQMaxThreads, 1) k_density_q(const __grid_cons
       const uint32_t own_tx = (uint32_t)(px * (zc + (halo ? 1 : 0))) * rs, xp_tx = (uint32_t)zc * rs;
       int so = 0, sx = 0;
       uint32_t pho = 0, phx = 0;
-      // L2 prefetch of the own / x+px lines kQPf lines ahead of their shared-memory loads: the DRAM latency is
-      // covered without ring depth (shared memory), the ring only waits for L2 hits
-      auto prefetch = [&](int k) {
-        if (k < nown) {
-          const int yy = (y0 + k == g.ny) ? 0 : y0 + k;
-          for (int p = 0; p < px; ++p) tma_prefetch_3d(&mp.seg, c0, z0, (dom * g.nx + xb + p) * g.ny + yy);
-        }
-        if (has_xn && k < ycnt) tma_prefetch_3d(&mp.seg, c0, z0, rowxn + y0 + k);
-      };
-      for (int k = 0; k < kQPf; ++k) prefetch(nso + k);
       auto issue_own = [&](int k) {  // own lines y0 + k (== ny: plane 0 again) of the px planes
         if (k >= nso) mbar_wait(&oempty[so], pho ^ 1u);
-        prefetch(k + kQPf);
         const int yy = (y0 + k == g.ny) ? 0 : y0 + k;
         mbar_expect_tx(&ofull[so], own_tx);
         for (int p = 0; p < px; ++p) {
@@ -558,7 +546,7 @@ __global__ void __launch_bounds__(kQMaxThreads, 1) k_density_q(const __grid_cons
   for (int k = 0; k < ycnt; ++k) {
     const int y = y0 + k;
     const bool has_y = valid && (kPer || y + 1 < g.ny);
-    mbar_wait(&ofull[so], pho);
+    if (k == 0) mbar_wait(&ofull[so], pho);  // (later own lines were waited for as the previous step's y+1 line)
     if (k + 1 < nown) mbar_wait(&ofull[sn], phn);
     if (xring) mbar_wait(&xfull[sx], phx);
     const unsigned char* O = own_seg(so, plr) + orow;
@@ -567,37 +555,41 @@ __global__ void __launch_bounds__(kQMaxThreads, 1) k_density_q(const __grid_cons
     const unsigned char* X = (plr + 1 < px ? own_seg(so, plr + 1) : xp_slot(sx)) + orow;  // plane x+1
     // per-lane partial sums over this lane's orbitals: rho and the three link products P_d = sum f
     // conj(psi_r) psi_{r+e_d} (f folded into fv = f psi_r)
-    double rho = 0.0, pxr = 0.0, pxi = 0.0, pyr = 0.0, pyi = 0.0, pzr = 0.0, pzi = 0.0;
+    // (two accumulator sets over alternate orbitals halve the FP64 dependency chains; summed in a fixed order)
+    double acc[2][7] = {};
     if (valid) {
-      auto orb = [&](int i, double f) {
+      auto orb = [&](int i, double f, double* r) {
         const uint32_t off = (uint32_t)i * 4u * (uint32_t)sizeof(C);
         const double2 v = to_d2(*reinterpret_cast<const C*>(O + off));  // FP64 accumulation (also for complex64 Psi)
         const double2 fv = make_double2(f * v.x, f * v.y);
-        rho = fma(fv.x, v.x, fma(fv.y, v.y, rho));
+        r[0] = fma(fv.x, v.x, fma(fv.y, v.y, r[0]));
         if (kPer || has_x) {
           const double2 w = to_d2(*reinterpret_cast<const C*>(X + off));
-          pxr = fma(fv.x, w.x, fma(fv.y, w.y, pxr));
-          pxi = fma(fv.x, w.y, fma(-fv.y, w.x, pxi));
+          r[1] = fma(fv.x, w.x, fma(fv.y, w.y, r[1]));
+          r[2] = fma(fv.x, w.y, fma(-fv.y, w.x, r[2]));
         }
         if (kPer || has_y) {
           const double2 w = to_d2(*reinterpret_cast<const C*>(N + off));
-          pyr = fma(fv.x, w.x, fma(fv.y, w.y, pyr));
-          pyi = fma(fv.x, w.y, fma(-fv.y, w.x, pyi));
+          r[3] = fma(fv.x, w.x, fma(fv.y, w.y, r[3]));
+          r[4] = fma(fv.x, w.y, fma(-fv.y, w.x, r[4]));
         }
         if (kPer || has_z) {
           const double2 w = to_d2(*reinterpret_cast<const C*>(Oz + off));
-          pzr = fma(fv.x, w.x, fma(fv.y, w.y, pzr));
-          pzi = fma(fv.x, w.y, fma(-fv.y, w.x, pzi));
+          r[5] = fma(fv.x, w.x, fma(fv.y, w.y, r[5]));
+          r[6] = fma(fv.x, w.y, fma(-fv.y, w.x, r[6]));
         }
       };
       if (kIt > 0) {
 #pragma unroll
-        for (int i = 0; i < (kIt > 0 ? kIt : 1); ++i) orb(i, fr[i]);
+        for (int i = 0; i < (kIt > 0 ? kIt : 1); ++i) orb(i, fr[i], acc[i & 1]);
       } else {
 #pragma unroll 4
-        for (int i = 0; i < nit; ++i) orb(i, fsh[q + 4 * i]);
+        for (int i = 0; i < nit; ++i) orb(i, fsh[q + 4 * i], acc[0]);
       }
     }
+    const double rho = acc[0][0] + acc[1][0], pxr = acc[0][1] + acc[1][1], pxi = acc[0][2] + acc[1][2];
+    const double pyr = acc[0][3] + acc[1][3], pyi = acc[0][4] + acc[1][4];
+    const double pzr = acc[0][5] + acc[1][5], pzi = acc[0][6] + acc[1][6];
     // this warp is done with own line y and x+1 line y (once its loads have returned: lfd_tma.cuh)
     mbar_release2(&oempty[so], &xempty[sx], xring, ((rho + pxr) + (pyr + pzr)) + (pxi + pyi + pzi), lane == 0);
     if (++so == nso) { so = 0; pho ^= 1u; }
