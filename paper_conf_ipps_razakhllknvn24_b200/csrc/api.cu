@@ -34,7 +34,7 @@ size_t up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 struct Layout {
   size_t phi, coef, G, D, occ, part, normp, dc, cprime, s, nfac, jline, base, vstage, rhostage, Jstage, hv[2], hrho[2], hJ[2], cref,
-      epart, W, ones, x32, aseq, jseq, bsl, bsig, bsl1, bexp, colE, g1cnt, g1cs, btil, qmat, zero, bslx, sigx;
+      epart, W, ones, x32, aseq, jseq, bsl, bsig, bsl1, bexp, colE, g1cnt, g1cs, btil, qmat, zero, bslx, sigx, dcount;
   int nref_cap;
   bool i8;  // GEMM-2 on the int8 tensor cores (nl_i8.cu): B digit tiles + row scales in the workspace
   bool fx;  // the first factor's GEMM-2 fused with the x pass (nl_fx.cu)
@@ -178,6 +178,7 @@ Layout layout(const Geometry& g, int num_sms, int nref_max, bool dense = false) 
   L.s = take((size_t)nd * no * d8);
   L.nfac = take((size_t)nd * no * d8);
   L.jline = take((size_t)nd * lfd::density_blocks(g) * 3 * d8);
+  L.dcount = take((size_t)nd * sizeof(int));  // density CTA completion counters (zero between launches)
   L.base = take((size_t)4 * nd * sizeof(long long));
   L.vstage = take((size_t)nd * g.ng * d8);
   L.rhostage = take((size_t)nd * g.ng * d8);
@@ -706,8 +707,10 @@ lfd_status density_into(lfd_ctx* c, double* rho, double* j, double* Jmac, const 
   a.base = base_dev; a.jbase = base_dev + c->g.ndom; a.sx = sx; a.sy = sy; a.jstride = jstride;
   a.v = energy ? c->at<double>(c->L.vstage) : nullptr;
   a.epart = energy ? c->at<double>(c->L.epart) : nullptr;
+  a.Jmac = Jmac;
+  a.dcount = c->at<int>(c->L.dcount);
   LFD_TRY(launch(c, LFD_K_DENSITY, "k_density", [&] { return lfd::launch_density(c->g, a, c->dmaps, c->stream); }));
-  if (Jmac)
+  if (Jmac && !lfd::density_reduces_J(c->dmaps))
     LFD_TRY(launch(c, LFD_K_JREDUCE, "k_jreduce",
                    [&] { return lfd::launch_jreduce(c->g, a.jline, lfd::density_blocks_used(c->g, c->dmaps), Jmac, c->stream); }));
   return LFD_OK;
@@ -1053,8 +1056,9 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   e = cudaMemcpyAsync(c->at<long long>(L.base), base.data(), sizeof(long long) * base.size(), cudaMemcpyHostToDevice,
                       c->stream);
   if (e != cudaSuccess) { cuda_fail(c, e, "copy base"); return bail(LFD_ECUDA); }
-  // initial state: v = 0 (Phi = 1), A = 0
+  // initial state: v = 0 (Phi = 1), A = 0; density completion counters 0
   e = cudaMemsetAsync(c->at<double>(L.vstage), 0, sizeof(double) * g.ndom * g.ng, c->stream);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->at<int>(L.dcount), 0, sizeof(int) * g.ndom, c->stream);
   if (e != cudaSuccess) { cuda_fail(c, e, "memset"); return bail(LFD_ECUDA); }
   lfd_status s2 = launch(c, LFD_K_PHASE, "k_phase",
                          [&] { return phase_any(c, c->at<double>(L.vstage), c->at<double>(L.vstage)); });

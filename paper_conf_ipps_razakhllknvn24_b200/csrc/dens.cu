@@ -355,7 +355,7 @@ struct QLayout {
     own_b = (uint32_t)px * pl_b;
     xp_b = seg_b;
     fsh_off = (uint32_t)nso * own_b + (uint32_t)nsx * xp_b;
-    if (fsh_off < 5u * kQMaxWarps * 8u * 8u) fsh_off = 5u * kQMaxWarps * 8u * 8u;  // the per-CTA partials reuse it
+    if (fsh_off < 3u * (kQMaxWarps * 32u) * 8u) fsh_off = 3u * (kQMaxWarps * 32u) * 8u;  // the end-of-kernel sums reuse it
     bar_off = fsh_off + (((uint32_t)nact * 8u + 15u) & ~15u);
     total = bar_off + (uint32_t)(2 * nso + 2 * nsx) * 8u;
   }
@@ -653,8 +653,34 @@ __global__ void __launch_bounds__(kQMaxThreads, 1) k_density_q(const __grid_cons
     double t = 0.0;
     for (int k = 0; k < pts; ++k) t += jsh[tid][k];
     a.jline[((long long)dom * gridDim.x + blockIdx.x) * 3 + tid] = t;
+    __threadfence();  // (before the CTA's completion count below)
   }
+  if (!a.Jmac) return;
+  // the domain's last CTA to finish reduces the per-CTA partials into J_d = (1/Ngrid) sum (fixed order: by CTA
+  // index, whatever the arrival order) and re-arms the counter -- the k_jreduce launch folded in
+  __shared__ int last;
+  asm volatile("bar.sync 1, %0;" ::"r"(nconsw * 32) : "memory");
+  if (tid == 0) last = atomicAdd(a.dcount + dom, 1) == (int)gridDim.x - 1;
+  asm volatile("bar.sync 1, %0;" ::"r"(nconsw * 32) : "memory");
+  if (!last) return;
+  __threadfence();
+  const int nt = nconsw * 32;
+  double sj[3] = {0.0, 0.0, 0.0};
+  const volatile double* jl = a.jline + (long long)dom * gridDim.x * 3;
+  for (int l = tid; l < (int)gridDim.x; l += nt)
+    for (int d = 0; d < 3; ++d) sj[d] += jl[l * 3 + d];
+  double* red = reinterpret_cast<double*>(dsm);  // (the ring is consumed)
+  for (int d = 0; d < 3; ++d) red[d * nt + tid] = sj[d];
+  asm volatile("bar.sync 1, %0;" ::"r"(nt) : "memory");
+  if (tid < 3) {
+    double t = 0.0;
+    for (int k = 0; k < nt; ++k) t += red[tid * nt + k];
+    a.Jmac[dom * 3 + tid] = t / (double)g.ng;
+  }
+  if (tid == 0) a.dcount[dom] = 0;
 }
+
+bool density_reduces_J(const DensMaps* m) { return m != nullptr; }
 
 static size_t q_smem(const DensMaps& m) { return QLayout(m.zc, m.px, m.nact, m.pad, m.esz, m.nso, m.nsx).total; }
 
@@ -724,7 +750,9 @@ int density_blocks(const Geometry& g) {
 
 int density_blocks_used(const Geometry& g, const DensMaps* m) { return m ? m->blocks : fallback_blocks(g); }
 
-cudaError_t launch_density(const Geometry& g, const DensArgs& a, const DensMaps* maps, cudaStream_t st) {
+cudaError_t launch_density(const Geometry& g, const DensArgs& a_in, const DensMaps* maps, cudaStream_t st) {
+  DensArgs a = a_in;
+  if (!maps) a.Jmac = nullptr;  // (the generic kernels leave J to k_jreduce)
   if (maps) {
     dim3 grid(maps->blocks, g.ndom);
     const int threads = ((maps->zc * maps->px + 7) / 8 + 1) * 32;

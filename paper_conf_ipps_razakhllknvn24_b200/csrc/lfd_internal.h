@@ -246,8 +246,11 @@ struct DensArgs {
   long long sx, sy, jstride;
   const double* v;      // v_loc copy [dom][ng] when energy partials are wanted, else nullptr
   double* epart;        // [dom][density_blocks][2] per-CTA sums of (kinetic, local) energy densities
+  double* Jmac = nullptr;  // [dom][3]: the y-marching kernel's last CTA reduces jline into J (else k_jreduce)
+  int* dcount = nullptr;   // [dom] CTA completion counters for that reduction (zero between launches)
 };
 struct DensMaps;  // TMA descriptors of Psi for the y-marching density kernel (dens.cu)
+bool density_reduces_J(const DensMaps* m);  // launch_density writes J itself (no k_jreduce)
 // nact: active orbitals (1 + last index with f != 0); f = 0 orbitals add exactly zero to rho, j, E
 DensMaps* density_maps_create(const Geometry& g, const double2* psi, int nact);  // nullptr: generic kernel
 cudaError_t density_maps_set_active(DensMaps* m, const Geometry& g, const double2* psi, int nact);
