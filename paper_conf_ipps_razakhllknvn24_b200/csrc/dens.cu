@@ -13,6 +13,7 @@
 #include <algorithm>
 #include <cstdlib>
 #include <new>
+#include <type_traits>
 
 namespace lfd {
 
@@ -556,40 +557,44 @@ __global__ void __launch_bounds__(kQMaxThreads, 1) k_density_q(const __grid_cons
     // per-lane partial sums over this lane's orbitals: rho and the three link products P_d = sum f
     // conj(psi_r) psi_{r+e_d} (f folded into fv = f psi_r)
     // (two accumulator sets over alternate orbitals halve the FP64 dependency chains; summed in a fixed order)
-    double acc[2][7] = {};
+    // (complex64 Psi, the SP variant: FP32 products and partial sums over the lane's orbitals -- <= 16 terms, a
+    // relative error ~2^-20, far below the SP contract n 30 2^-24 -- then FP64 for the reduction over lanes)
+    using A = typename std::conditional<sizeof(C) == 8, float, double>::type;
+    A acc[2][7] = {};
     if (valid) {
-      auto orb = [&](int i, double f, double* r) {
+      auto orb = [&](int i, A f, A* r) {
         const uint32_t off = (uint32_t)i * 4u * (uint32_t)sizeof(C);
-        const double2 v = to_d2(*reinterpret_cast<const C*>(O + off));  // FP64 accumulation (also for complex64 Psi)
-        const double2 fv = make_double2(f * v.x, f * v.y);
-        r[0] = fma(fv.x, v.x, fma(fv.y, v.y, r[0]));
+        const C v = *reinterpret_cast<const C*>(O + off);
+        const A fx = f * v.x, fy = f * v.y;
+        r[0] = fma(fx, v.x, fma(fy, v.y, r[0]));
         if (kPer || has_x) {
-          const double2 w = to_d2(*reinterpret_cast<const C*>(X + off));
-          r[1] = fma(fv.x, w.x, fma(fv.y, w.y, r[1]));
-          r[2] = fma(fv.x, w.y, fma(-fv.y, w.x, r[2]));
+          const C w = *reinterpret_cast<const C*>(X + off);
+          r[1] = fma(fx, w.x, fma(fy, w.y, r[1]));
+          r[2] = fma(fx, w.y, fma(-fy, w.x, r[2]));
         }
         if (kPer || has_y) {
-          const double2 w = to_d2(*reinterpret_cast<const C*>(N + off));
-          r[3] = fma(fv.x, w.x, fma(fv.y, w.y, r[3]));
-          r[4] = fma(fv.x, w.y, fma(-fv.y, w.x, r[4]));
+          const C w = *reinterpret_cast<const C*>(N + off);
+          r[3] = fma(fx, w.x, fma(fy, w.y, r[3]));
+          r[4] = fma(fx, w.y, fma(-fy, w.x, r[4]));
         }
         if (kPer || has_z) {
-          const double2 w = to_d2(*reinterpret_cast<const C*>(Oz + off));
-          r[5] = fma(fv.x, w.x, fma(fv.y, w.y, r[5]));
-          r[6] = fma(fv.x, w.y, fma(-fv.y, w.x, r[6]));
+          const C w = *reinterpret_cast<const C*>(Oz + off);
+          r[5] = fma(fx, w.x, fma(fy, w.y, r[5]));
+          r[6] = fma(fx, w.y, fma(-fy, w.x, r[6]));
         }
       };
       if (kIt > 0) {
 #pragma unroll
-        for (int i = 0; i < (kIt > 0 ? kIt : 1); ++i) orb(i, fr[i], acc[i & 1]);
+        for (int i = 0; i < (kIt > 0 ? kIt : 1); ++i) orb(i, (A)fr[i], acc[i & 1]);
       } else {
 #pragma unroll 4
-        for (int i = 0; i < nit; ++i) orb(i, fsh[q + 4 * i], acc[0]);
+        for (int i = 0; i < nit; ++i) orb(i, (A)fsh[q + 4 * i], acc[0]);
       }
     }
-    const double rho = acc[0][0] + acc[1][0], pxr = acc[0][1] + acc[1][1], pxi = acc[0][2] + acc[1][2];
-    const double pyr = acc[0][3] + acc[1][3], pyi = acc[0][4] + acc[1][4];
-    const double pzr = acc[0][5] + acc[1][5], pzi = acc[0][6] + acc[1][6];
+    const double rho = (double)acc[0][0] + acc[1][0], pxr = (double)acc[0][1] + acc[1][1];
+    const double pxi = (double)acc[0][2] + acc[1][2], pyr = (double)acc[0][3] + acc[1][3];
+    const double pyi = (double)acc[0][4] + acc[1][4], pzr = (double)acc[0][5] + acc[1][5];
+    const double pzi = (double)acc[0][6] + acc[1][6];
     // this warp is done with own line y and x+1 line y (once its loads have returned: lfd_tma.cuh)
     mbar_release2(&oempty[so], &xempty[sx], xring, ((rho + pxr) + (pyr + pzr)) + (pxi + pyi + pzi), lane == 0);
     if (++so == nso) { so = 0; pho ^= 1u; }

@@ -13,6 +13,7 @@ from lfd_workloads import make_inputs, workload
 
 pytestmark = pytest.mark.gpu
 TOL = 1e-12
+TOL_SP = 1e-5
 
 CASES = [  # (nx, ny, nz, bc, norb, nact)
     (70, 6, 72, 0, 64, 32),    # the bench's shape class (C2 planes, 32 of 64 active)
@@ -57,4 +58,5 @@ def test_density_current_shapes(case, sp):
     e_rho = np.linalg.norm(rho - rr) / np.linalg.norm(rr)
     e_j = np.linalg.norm(j - jr) / max(np.linalg.norm(jr), 1e-3 * np.linalg.norm(rr))
     e_J = np.abs(J - Jr).max() / max(np.abs(jr).mean(), 1e-3 * np.abs(rr).mean())
-    assert e_rho < TOL and e_j < TOL and e_J < TOL, (case, sp, e_rho, e_j, e_J)
+    tol = TOL_SP if sp else TOL
+    assert e_rho < tol and e_j < tol and e_J < tol, (case, sp, e_rho, e_j, e_J)
