@@ -544,6 +544,7 @@ __global__ void __launch_bounds__(kQMaxThreads, 1) k_density_q(const __grid_cons
   const long long rbase = a.base[dom], jb = a.j ? a.jbase[dom] : 0;  // hoisted global loads
   int so = 0, sn = nso > 1 ? 1 : 0, sx = 0;
   uint32_t pho = 0, phn = 0, phx = 0;
+  C ocur[kIt > 0 ? kIt : 1];  // this lane's own values of the current line (kIt > 0)
   for (int k = 0; k < ycnt; ++k) {
     const int y = y0 + k;
     const bool has_y = valid && (kPer || y + 1 < g.ny);
@@ -562,9 +563,8 @@ __global__ void __launch_bounds__(kQMaxThreads, 1) k_density_q(const __grid_cons
     using A = typename std::conditional<sizeof(C) == 8, float, double>::type;
     A acc[2][7] = {};
     if (valid) {
-      auto orb = [&](int i, A f, A* r) {
+      auto orb = [&](int i, A f, A* r, const C v, C& nv) {
         const uint32_t off = (uint32_t)i * 4u * (uint32_t)sizeof(C);
-        const C v = *reinterpret_cast<const C*>(O + off);
         const A fx = f * v.x, fy = f * v.y;
         r[0] = fma(fx, v.x, fma(fy, v.y, r[0]));
         if (kPer || has_x) {
@@ -574,6 +574,7 @@ __global__ void __launch_bounds__(kQMaxThreads, 1) k_density_q(const __grid_cons
         }
         if (kPer || has_y) {
           const C w = *reinterpret_cast<const C*>(N + off);
+          nv = w;
           r[3] = fma(fx, w.x, fma(fy, w.y, r[3]));
           r[4] = fma(fx, w.y, fma(-fy, w.x, r[4]));
         }
@@ -583,12 +584,21 @@ __global__ void __launch_bounds__(kQMaxThreads, 1) k_density_q(const __grid_cons
           r[6] = fma(fx, w.y, fma(-fy, w.x, r[6]));
         }
       };
-      if (kIt > 0) {
+      if (kIt > 0) {  // the own values come from registers: the y+1 values of the previous step
+        if (k == 0) {
 #pragma unroll
-        for (int i = 0; i < (kIt > 0 ? kIt : 1); ++i) orb(i, (A)fr[i], acc[i & 1]);
+          for (int i = 0; i < (kIt > 0 ? kIt : 1); ++i) ocur[i] = *reinterpret_cast<const C*>(O + i * 4 * (int)sizeof(C));
+        }
+        C nn[kIt > 0 ? kIt : 1];
+#pragma unroll
+        for (int i = 0; i < (kIt > 0 ? kIt : 1); ++i) orb(i, (A)fr[i], acc[i & 1], ocur[i], nn[i]);
+#pragma unroll
+        for (int i = 0; i < (kIt > 0 ? kIt : 1); ++i) ocur[i] = nn[i];
       } else {
+        C nn;
 #pragma unroll 4
-        for (int i = 0; i < nit; ++i) orb(i, (A)fsh[q + 4 * i], acc[0]);
+        for (int i = 0; i < nit; ++i)
+          orb(i, (A)fsh[q + 4 * i], acc[0], *reinterpret_cast<const C*>(O + i * 4 * (int)sizeof(C)), nn);
       }
     }
     const double rho = (double)acc[0][0] + acc[1][0], pxr = (double)acc[0][1] + acc[1][1];
