@@ -60,3 +60,35 @@ def test_density_current_shapes(case, sp):
     e_J = np.abs(J - Jr).max() / max(np.abs(jr).mean(), 1e-3 * np.abs(rr).mean())
     tol = TOL_SP if sp else TOL
     assert e_rho < tol and e_j < tol and e_J < tol, (case, sp, e_rho, e_j, e_J)
+
+
+def test_density_active_count_changes():
+    """lfd_set_occupations moves the active-orbital count across the y-marching kernel's limit (32 -> 126 -> 20 of
+    128): the shape is re-chosen, then the generic kernel takes over (and stays), with the same results."""
+    import torch
+    from oracle import ref
+    from paper_conf_ipps_razakhllknvn24_b200 import Context
+    nx, ny, nz, norb = 8, 6, 24, 128
+    w = workload("P0").with_(nx=nx, ny=ny, nz=nz, norb=norb, nocc=32, nproj=0)
+    x = make_inputs(w, seed=17)
+    dev = torch.device("cuda:0")
+    psi = torch.from_numpy(x.psi0.copy()).to(dev)
+    occ0 = np.zeros((1, norb))
+    occ0[0, :32] = 2.0
+    ctx = Context(psi, None, None, occ0, (w.hx, w.hy, w.hz), w.dt, bc=w.bc)
+    A = np.array([[0.2, 0.1, -0.3]])
+    ctx.set_vector_potential(A)
+    cfg = ref.RefConfig(1, nx, ny, nz, w.hx, w.hy, w.hz, w.bc, norb, 0, w.dt)
+    rng = np.random.default_rng(3)
+    for nact in (32, 126, 20):
+        occ = np.zeros((1, norb))
+        occ[0, :nact] = rng.uniform(0.5, 2.0, size=nact)
+        ctx.set_occupations(np.ascontiguousarray(occ))
+        rho, j, J = ctx.density_current()
+        ctx.sync()
+        rr, jr, Jr = ref.density_current(cfg, x.psi0, occ, A)
+        rho, j = rho.cpu().numpy().reshape(1, -1), j.cpu().numpy().reshape(1, 3, -1)
+        assert np.linalg.norm(rho - rr) / np.linalg.norm(rr) < TOL, nact
+        assert np.linalg.norm(j - jr) / max(np.linalg.norm(jr), 1e-3 * np.linalg.norm(rr)) < TOL, nact
+        assert np.abs(J.cpu().numpy() - Jr).max() / max(np.abs(jr).mean(), 1e-3 * np.abs(rr).mean()) < TOL, nact
+    ctx.close()
