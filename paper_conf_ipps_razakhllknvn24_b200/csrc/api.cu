@@ -532,7 +532,8 @@ const double2* exact_w(lfd_ctx* c, bool merged) {
 lfd_status gemm2x(lfd_ctx* c) {
   c->c_valid = false;
   return launch(c, LFD_K_NL_BACKX, "k_gemm2x_i8", [&] {
-    return lfd::launch_gemm2x_i8(c->g, c->fxm, c->psi, c->coef(), c->at<double>(c->L.nfac),
+    return lfd::launch_gemm2x_i8(c->g, c->fxm, c->g.sp ? (void*)c->psi32() : (void*)c->psi, c->coef(),
+                                 c->at<double>(c->L.nfac),
                                  c->at<double2>(c->L.cprime), c->at<double>(c->L.sigx), c->scaled, c->num_sms,
                                  c->stream);
   });
@@ -621,11 +622,12 @@ lfd_status nl_half(lfd_ctx* c, bool merged = false, double2* out = nullptr, bool
 // src != nullptr: the first pass reads src (same layout) and writes Psi (out of place).
 lfd_status local_prop(lfd_ctx* c, const double2* src = nullptr, bool skip_x = false) {
   c->c_valid = false;
-  if (c->g.sp && c->kin_fused) {  // SP variant: Phi.K_x, then Phi.K_y K_z fused (FP32, complex64 Psi)
-    LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin_sp(x)", [&] {
-      return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 0, 1, c->scaled, c->stream,
-                                reinterpret_cast<const float2*>(src));
-    }));
+  if (c->g.sp && c->kin_fused) {  // SP variant: Phi.K_x (unless fused into the GEMM-2), then Phi.K_y K_z fused
+    if (!skip_x)
+      LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin_sp(x)", [&] {
+        return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 0, 1, c->scaled, c->stream,
+                                  reinterpret_cast<const float2*>(src));
+      }));
     int* colE = c->L.i8 ? c->at<int>(c->L.colE) : nullptr;  // exponents for the int8-digit GEMM-1
     LFD_TRY(launch(c, LFD_K_KIN_YZ, "k_kin_yz_sp", [&] {
       return lfd::launch_kin_yz_sp(c->g, &c->psi_tmap, c->psi32(), c->coef(), c->phi32(), c->scaled, c->stream, colE);
@@ -634,10 +636,11 @@ lfd_status local_prop(lfd_ctx* c, const double2* src = nullptr, bool skip_x = fa
     return LFD_OK;
   }
   if (c->g.sp) {  // SP variant: three FP32 line passes Phi.K_x, K_y, K_z.Phi (complex64 Psi)
-    LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin_sp(x)", [&] {
-      return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 0, 1, c->scaled, c->stream,
-                                reinterpret_cast<const float2*>(src));
-    }));
+    if (!skip_x)
+      LFD_TRY(launch(c, LFD_K_KIN_X, "k_kin_sp(x)", [&] {
+        return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 0, 1, c->scaled, c->stream,
+                                  reinterpret_cast<const float2*>(src));
+      }));
     LFD_TRY(launch(c, LFD_K_KIN_Y, "k_kin_sp(y)", [&] {
       return lfd::launch_kin_sp(c->g, c->psi32(), c->coef(), c->phi32(), 1, 0, c->scaled, c->stream);
     }));
@@ -1122,10 +1125,12 @@ lfd_status lfd_init(const lfd_config* cfg, void* psi, const void* proj, const do
   }
   if (L.fx) {  // B's digits in x-line order for the fused first factor
     s2 = launch(c, LFD_K_NL_BACKX, "k_bslicex_i8", [&] {
-      return lfd::launch_bslicex_i8(g, c->proj, c->at<int8_t>(L.bslx), c->at<double>(L.sigx), c->stream);
+      return lfd::launch_bslicex_i8(g, g.sp ? (const void*)c->proj32() : (const void*)c->proj, c->at<int8_t>(L.bslx),
+                                    c->at<double>(L.sigx), c->stream);
     });
     if (s2 != LFD_OK) return bail(s2);
-    c->fxm = lfd::gemm2x_maps_create(g, c->at<int8_t>(L.bslx), c->psi, c->phi());
+    c->fxm = g.sp ? lfd::gemm2x_maps_create(g, c->at<int8_t>(L.bslx), c->psi32(), c->phi32())
+                  : lfd::gemm2x_maps_create(g, c->at<int8_t>(L.bslx), c->psi, c->phi());
     // (no descriptors: the unfused GEMM-2 + x pass run instead)
   }
   if (cfg->flags & LFD_FLAG_EXACT_NL) {

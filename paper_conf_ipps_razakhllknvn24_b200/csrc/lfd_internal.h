@@ -216,10 +216,10 @@ struct FxMaps;  // TMA descriptors (digits, Psi, Phi) -- host-owned, built at lf
 bool gemm2x_supported(const Geometry& g);
 size_t gemm2x_digit_bytes(const Geometry& g);
 size_t gemm2x_sig_bytes(const Geometry& g);
-cudaError_t launch_bslicex_i8(const Geometry& g, const double2* B, int8_t* dig, double* sig, cudaStream_t st);
-FxMaps* gemm2x_maps_create(const Geometry& g, const int8_t* dig, double2* psi, const double2* phi);
+cudaError_t launch_bslicex_i8(const Geometry& g, const void* B, int8_t* dig, double* sig, cudaStream_t st);
+FxMaps* gemm2x_maps_create(const Geometry& g, const int8_t* dig, void* psi, const void* phi);
 void gemm2x_maps_destroy(FxMaps* m);
-cudaError_t launch_gemm2x_i8(const Geometry& g, const FxMaps* m, double2* psi, const DomCoef* coef, const double* nfac,
+cudaError_t launch_gemm2x_i8(const Geometry& g, const FxMaps* m, void* psi, const DomCoef* coef, const double* nfac,
                              const double2* Cp, const double* sig, bool scaled, int num_sms, cudaStream_t st);
 cudaError_t gemm2x_set_attributes();
 

@@ -40,10 +40,15 @@ namespace lfd {
 constexpr int kFxN = 80;                     // MMA N: x points of a line tile (nx <= 80)
 constexpr int kFxK = 128;                    // bytes per digit row (K = 2 nproj padded to 128)
 constexpr int kFxSliceB = kFxN * kFxK;       // 10 KB per digit
-constexpr int kFxTileB = kI8S * kFxSliceB;   // 60 KB
 constexpr int kFxSlots = 4;                  // TMEM ring of diagonal accumulators (80 columns each)
-constexpr int kFxWCols = kI8S * (kFxK / 4);  // 192 TMEM columns of W^T digits
-constexpr int kFxAcc = kI8S;                 // diagonals d = 2 .. S+1
+// shapes by the digit count S (6 for FP64 contexts, 4 for the SP variant)
+template <int S>
+struct FxG {
+  static constexpr int TileB = S * kFxSliceB;     // 60 KB / 40 KB
+  static constexpr int WCols = S * (kFxK / 4);    // TMEM columns of W^T digits
+  static constexpr int Acc = S;                   // diagonals d = 2 .. S+1
+};
+constexpr int fx_digits(bool sp) { return sp ? 4 : kI8S; }
 constexpr int kFxEpi = 16;                   // epilogue warps
 constexpr int kFxXg = kFxN / 4;              // x points per epilogue warp
 constexpr int kFxMarch = 4;                  // march warps (one warpgroup): 64 orbitals x 2 segments of each line
@@ -54,30 +59,39 @@ constexpr int kFxXchB = 2 * kFxSeg * 64 * 32;             // segment boundary E 
 // named barriers: epilogue -> march "ready" (2, 3 by line parity), march -> epilogue "free" (4, 5), march only (6)
 constexpr int kFxBarReady = 2, kFxBarFree = 4, kFxBarMarch = 6;
 constexpr int kFxHandoff = (kFxEpi + kFxMarch) * 32;
-constexpr int kFxMaxSmem = 225 * 1024;  // dynamic (the static barriers and tau table take the rest)
+constexpr int kFxMaxSmem = 225 * 1024;  // dynamic (the static barriers, tau table and coefficients take the rest)
 
 struct FxMaps {
   CUtensorMap dig, psi, phi;
 };
 
 __host__ __device__ inline int fx_al128(int b) { return (b + 127) & ~127; }
-// bytes of one line buffer: Psi [nx][2 norb] doubles + Phi [nx] complex + B's row scales [80]
-__host__ __device__ inline int fx_line_bytes(int nx, int norb) {
-  return fx_al128(nx * norb * 16) + fx_al128(nx * 16) + kFxN * 8;
+// bytes of one line buffer: Psi [nx][norb] complex (esz bytes each) + Phi [nx] x 16 bytes (complex128, or two
+// complex64: the TMA box needs 16 bytes) + B's row scales [80]
+__host__ __device__ inline int fx_line_bytes(int nx, int norb, int esz) {
+  return fx_al128(nx * norb * esz) + fx_al128(nx * 16) + kFxN * 8;
 }
-static size_t fx_smem(int nx, int norb) { return (size_t)kFxTileB + 2 * fx_line_bytes(nx, norb) + kFxXchB + 1024; }
+static size_t fx_smem(int nx, int norb, bool sp) {
+  return (size_t)fx_digits(sp) * kFxSliceB + 2 * fx_line_bytes(nx, norb, sp ? 8 : 16) + kFxXchB + 1024;
+}
 
 bool gemm2x_supported(const Geometry& g) {
-  return g.i8 && !g.sp && g.nx <= kFxN && g.nx >= 2 && g.norb <= 64 && g.nproj <= 64 &&
-         (long long)g.ny * g.nz < (1LL << 31) && fx_smem(g.nx, g.norb) <= (size_t)kFxMaxSmem &&
-         (size_t)kFxTileB + (size_t)g.nproj * g.norb * 16 + 1024 <= (size_t)kFxMaxSmem;
+  const size_t tile = (size_t)fx_digits(g.sp) * kFxSliceB;
+  // (complex64: TMA strides of 16-byte multiples -- norb even, and ny nz even for the Phi map)
+  return g.i8 && g.nx <= kFxN && g.nx >= 2 && g.norb <= 64 && g.nproj <= 64 &&
+         (!g.sp || (g.norb % 2 == 0 && (g.ny * g.nz) % 2 == 0)) &&
+         (long long)g.ny * g.nz < (1LL << 31) && fx_smem(g.nx, g.norb, g.sp) <= (size_t)kFxMaxSmem &&
+         tile + (size_t)g.nproj * g.norb * 16 + 1024 <= (size_t)kFxMaxSmem;
 }
-size_t gemm2x_digit_bytes(const Geometry& g) { return (size_t)g.ndom * g.ny * g.nz * kI8S * g.nx * kFxK; }
+size_t gemm2x_digit_bytes(const Geometry& g) {
+  return (size_t)g.ndom * g.ny * g.nz * fx_digits(g.sp) * g.nx * kFxK;
+}
 size_t gemm2x_sig_bytes(const Geometry& g) { return (size_t)g.ndom * g.ny * g.nz * kFxN * sizeof(double); }
 
 // ---- B's digits in x-line order (once per lfd_init): warp per grid row ------------------------------------
-// dig [dom][line][6][nx][128 B] plain (the TMA applies the 128B swizzle), sig [dom][line][80] (0 past nx)
-__global__ void __launch_bounds__(256) k_bslicex_i8(const double2* __restrict__ B, int nproj, int nx, int nyz,
+// dig [dom][line][S][nx][128 B] plain (the TMA applies the 128B swizzle), sig [dom][line][80] (0 past nx)
+template <class T, int S>
+__global__ void __launch_bounds__(256) k_bslicex_i8(const T* __restrict__ B, int nproj, int nx, int nyz,
                                                     int8_t* __restrict__ out, double* __restrict__ sig) {
   pdl_wait();
   pdl_trigger();
@@ -87,92 +101,37 @@ __global__ void __launch_bounds__(256) k_bslicex_i8(const double2* __restrict__ 
   if (r >= ngp) return;
   double v[4] = {0.0, 0.0, 0.0, 0.0};
   const int u0 = 2 * lane;
-  const double2* row = B + ((long long)dom * ngp + r) * nproj;
-  if (u0 < nproj) { const double2 a = row[u0]; v[0] = a.x; v[1] = a.y; }
-  if (u0 + 1 < nproj) { const double2 a = row[u0 + 1]; v[2] = a.x; v[3] = a.y; }
+  const T* row = B + ((long long)dom * ngp + r) * nproj;
+  if (u0 < nproj) { const T a = row[u0]; v[0] = a.x; v[1] = a.y; }
+  if (u0 + 1 < nproj) { const T a = row[u0 + 1]; v[2] = a.x; v[3] = a.y; }
   double mx = fmax(fmax(fabs(v[0]), fabs(v[1])), fmax(fabs(v[2]), fabs(v[3])));
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
   const int e = mx > 0.0 ? row_exponent(mx) : 0;
-  uint32_t d[kI8S];
-  digits4(v, e, !(mx > 0.0), d);
+  uint32_t d[S];
+  digits4<S>(v, e, !(mx > 0.0), d);
   const int x = (int)(r / nyz), line = (int)(r - (long long)x * nyz);
-  int8_t* tb = out + ((long long)dom * nyz + line) * kI8S * nx * kFxK + (long long)x * kFxK + 4 * lane;
+  int8_t* tb = out + ((long long)dom * nyz + line) * S * nx * kFxK + (long long)x * kFxK + 4 * lane;
 #pragma unroll
-  for (int i = 0; i < kI8S; ++i) *reinterpret_cast<uint32_t*>(tb + (long long)i * nx * kFxK) = d[i];
+  for (int i = 0; i < S; ++i) *reinterpret_cast<uint32_t*>(tb + (long long)i * nx * kFxK) = d[i];
   if (lane == 0) sig[((long long)dom * nyz + line) * kFxN + x] = mx > 0.0 ? ldexp(1.0, e) : 0.0;
 }
 
-cudaError_t launch_bslicex_i8(const Geometry& g, const double2* B, int8_t* dig, double* sig, cudaStream_t st) {
+cudaError_t launch_bslicex_i8(const Geometry& g, const void* B, int8_t* dig, double* sig, cudaStream_t st) {
   const int nyz = g.ny * g.nz;
   cudaError_t e = cudaMemsetAsync(sig, 0, gemm2x_sig_bytes(g), st);
   if (e != cudaSuccess) return e;
   dim3 grid((unsigned)((g.ng + 7) / 8), g.ndom);
-  launch_k(k_bslicex_i8, grid, 256, 0, st, B, g.nproj, g.nx, nyz, dig, sig);
+  if (g.sp)
+    launch_k(k_bslicex_i8<float2, 4>, grid, 256, 0, st, static_cast<const float2*>(B), g.nproj, g.nx, nyz, dig, sig);
+  else
+    launch_k(k_bslicex_i8<double2, kI8S>, grid, 256, 0, st, static_cast<const double2*>(B), g.nproj, g.nx, nyz, dig, sig);
   return cudaGetLastError();
-}
-
-// ---- K_x on lane components ------------------------------------------------------------------------------
-// The epilogue lane n = 2 s + c holds component c (0 re, 1 im) of orbital s; z_p, its partner component, is the
-// neighbour lane's (shfl_xor 1). For complex w: (w z)_c = w.x z_c + sgn w.y z_p with sgn = -1 (c = 0), +1 (c = 1).
-__device__ __forceinline__ double cmul_c(double2 w, double zc, double zp, double sgn) {
-  return fma(w.x, zc, sgn * w.y * zp);
-}
-// K_x of one periodic line (nx even, >= 8) for one orbital, as march_line2 (lfd_march.cuh: two segments marched
-// side by side) with explicit shared-memory loads and running store pointers (the generic lambda form recomputed
-// the shared-window base and 64-bit addresses every pair)
-__device__ __forceinline__ double2 ld_sh2(uint32_t a) {
-  double2 v;
-  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "r"(a));
-  return v;
-}
-template <bool kS>
-__device__ __forceinline__ void fx_march2(int n, const PairCoef& c, uint32_t l0, uint32_t ls, double2* out,
-                                          long long xs) {
-  const int PA = (n / 2 + 1) / 2, PB = n / 2 - PA, LA = 2 * PA;
-  LineMarch<kS> A, B;
-  A.init();
-  B.init();
-  uint32_t la = l0, lb = l0 + (uint32_t)LA * ls;
-  A.first(c, ld_sh2(la), ld_sh2(la + ls));
-  B.first(c, ld_sh2(lb), ld_sh2(lb + ls));
-  la += 2 * ls;
-  lb += 2 * ls;
-  A.second(c, ld_sh2(la), ld_sh2(la + ls));
-  B.second(c, ld_sh2(lb), ld_sh2(lb + ls));
-  la += 2 * ls;
-  lb += 2 * ls;
-  double2* oa = out + 2 * xs;  // stores of the steady loop at pair p: points 2p-2, 2p-1 (A), LA + 2p-2 .. (B)
-  double2* ob = out + (long long)(LA + 2) * xs;
-  for (int p = 2; p < PA; ++p) {
-    const double2 aa = ld_sh2(la), ab = ld_sh2(la + ls);
-    A.steady(c, aa, ab, [&](int k, double2 v) { oa[k * xs] = v; });
-    la += 2 * ls;
-    oa += 2 * xs;
-    if (p < PB) {
-      const double2 ba = ld_sh2(lb), bb = ld_sh2(lb + ls);
-      B.steady(c, ba, bb, [&](int k, double2 v) { ob[k * xs] = v; });
-      lb += 2 * ls;
-      ob += 2 * xs;
-    }
-  }
-  const double2 OAl = lk_L<kS>(c.a2, c.u2, A.prev_e1, B.E10);
-  const double2 OBf = lk_R<kS>(c.a2, c.d2, A.prev_e1, B.E10);
-  const double2 OBl = lk_L<kS>(c.a2, c.u2, B.prev_e1, A.E10);
-  const double2 OAf = lk_R<kS>(c.a2, c.d2, B.prev_e1, A.E10);
-  out[(long long)(LA - 2) * xs] = lk_L<kS>(c.a1, c.u1, A.prev_oR, OAl);
-  out[(long long)(LA - 1) * xs] = lk_R<kS>(c.a1, c.d1, A.prev_oR, OAl);
-  out[(long long)(n - 2) * xs] = lk_L<kS>(c.a1, c.u1, B.prev_oR, OBl);
-  out[(long long)(n - 1) * xs] = lk_R<kS>(c.a1, c.d1, B.prev_oR, OBl);
-  out[0] = lk_L<kS>(c.a1, c.u1, OAf, A.O1);
-  out[xs] = lk_R<kS>(c.a1, c.d1, OAf, A.O1);
-  out[(long long)LA * xs] = lk_L<kS>(c.a1, c.u1, OBf, B.O1);
-  out[(long long)(LA + 1) * xs] = lk_R<kS>(c.a1, c.d1, OBf, B.O1);
 }
 
 // ---- the fused kernel ------------------------------------------------------------------------------------
 struct FxArgs {
-  double2* psi;
+  void* psi;  // complex128, or complex64 (SP)
   const DomCoef* coef;
   const double* nfac;
   const double2* Cp;
@@ -181,7 +140,8 @@ struct FxArgs {
   long long ng;
 };
 
-template <bool kPer, bool kS>
+// T = double2 (S = 6 digits) or float2 (the SP variant: S = 4 digits, complex64 Psi, the march in FP32)
+template <bool kPer, bool kS, class T = double2, int S = kI8S>
 __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_constant__ CUtensorMap tDig,
                                                              const __grid_constant__ CUtensorMap tPsi,
                                                              const __grid_constant__ CUtensorMap tPhi, FxArgs p) {
@@ -190,16 +150,19 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
   pdl_trigger();
   extern __shared__ __align__(1024) unsigned char dsm_raw[];
   unsigned char* dsm = dsm_raw + ((1024u - (smem_addr(dsm_raw) & 1023u)) & 1023u);
+  using R = decltype(T::x);  // real component type of Psi
+  constexpr int kTileB = FxG<S>::TileB, kWCols = FxG<S>::WCols, kAcc = FxG<S>::Acc;
+  constexpr int kPhiStep = sizeof(T) == 8 ? 2 : 1;  // complex64 Phi staged two lines at a time (16-byte box)
   const int nx = p.nx, norb = p.norb, nproj = p.nproj, nyz = p.nyz;
-  const int psiB = fx_al128(nx * norb * 16), phiB = fx_al128(nx * 16);
+  const int psiB = fx_al128(nx * norb * (int)sizeof(T)), phiB = fx_al128(nx * 16);
   const int lineB = psiB + phiB + kFxN * 8;
-  unsigned char* Tsm = dsm;             // [6][80][128 B] digit tile (128B-swizzled)
-  unsigned char* Lsm = dsm + kFxTileB;  // 2 line buffers
-  auto lpsi = [&](int b) { return reinterpret_cast<double*>(Lsm + b * lineB); };
-  auto lphi = [&](int b) { return reinterpret_cast<const double2*>(Lsm + b * lineB + psiB); };
+  unsigned char* Tsm = dsm;           // [S][80][128 B] digit tile (128B-swizzled)
+  unsigned char* Lsm = dsm + kTileB;  // 2 line buffers
+  auto lpsi = [&](int b) { return reinterpret_cast<R*>(Lsm + b * lineB); };
+  auto lphi = [&](int b) { return reinterpret_cast<const T*>(Lsm + b * lineB + psiB); };  // Phi(x) at [x kPhiStep]
   auto lsig = [&](int b) { return reinterpret_cast<const double*>(Lsm + b * lineB + psiB + phiB); };
   unsigned char* Csm = Lsm;  // C'' of the domain, staged before the first line load
-  double2* Xsm = reinterpret_cast<double2*>(Lsm + 2 * lineB);  // march segments' boundary values
+  T* Xsm = reinterpret_cast<T*>(Lsm + 2 * lineB);  // march segments' boundary values
   __shared__ __align__(8) uint64_t bfull, bempty, dfull[kFxSlots], dempty[kFxSlots];
   __shared__ __align__(8) uint64_t lfull[2], lempty[2], cbar;
   __shared__ uint32_t tmem_base_sh;
@@ -224,10 +187,10 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = tmem_base_sh;
-  const uint32_t tacc = tmem + kFxWCols;
+  const uint32_t tacc = tmem + kWCols;
   const long long nlines = nyz;
   if (warp == kFxWMma && lane == 0 && blockIdx.x < nlines) {  // first digit tile, before the dependency wait
-    mbar_expect_tx(&bfull, kFxTileB);
+    mbar_expect_tx(&bfull, kTileB);
     tma_4d(Tsm, &tDig, 0, 0, 0, (int)((long long)dom * nyz + blockIdx.x), &bfull);
   }
   pdl_wait();
@@ -253,7 +216,7 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
     const int e = mx > 0.0 ? row_exponent(mx) : 0;
     if (c8 == 0) taus[n] = mx > 0.0 ? ldexp(1.0, e - 12) : 0.0;
     const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
-    uint32_t dg[kI8S][8];
+    uint32_t dg[S][8];
 #pragma unroll
     for (int w = 0; w < 8; ++w) {
       double v[4] = {0.0, 0.0, 0.0, 0.0};
@@ -266,13 +229,13 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
         const double2 x = X[(u0 + 1) * norb];
         v[2] = cn ? x.y : x.x; v[3] = cn ? x.x : -x.y;
       }
-      uint32_t d[kI8S];
-      digits_i64(v, mx > 0.0 ? ldexp(1.0, 41 - e) : 0.0, d);
+      uint32_t d[S];
+      digits_x<S>(v, mx > 0.0 ? ldexp(1.0, 7 * S - 1 - e) : 0.0, d);
 #pragma unroll
-      for (int i = 0; i < kI8S; ++i) dg[i][w] = d[i];
+      for (int i = 0; i < S; ++i) dg[i][w] = d[i];
     }
 #pragma unroll
-    for (int i = 0; i < kI8S; ++i) tmem_st8(trow + i * 32 + 8 * c8, dg[i]);
+    for (int i = 0; i < S; ++i) tmem_st8(trow + i * 32 + 8 * c8, dg[i]);
     asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
   }
   // W ready and the staged C'' consumed (the line producer then reuses its space)
@@ -304,8 +267,8 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
 #pragma unroll
       for (int c = 0; c < kFxXg; ++c) fa[c] = 0.0;
 #pragma unroll 1
-      for (int dp = 0; dp < kFxAcc / 2; ++dp) {
-        const int g = it * kFxAcc + 2 * dp, s0 = g % kFxSlots, s1 = (g + 1) % kFxSlots;
+      for (int dp = 0; dp < kAcc / 2; ++dp) {
+        const int g = it * kAcc + 2 * dp, s0 = g % kFxSlots, s1 = (g + 1) % kFxSlots;
         FX_T0(c3);
         mbar_wait(&dfull[s0], (uint32_t)((g / kFxSlots) & 1));
         mbar_wait(&dfull[s1], (uint32_t)(((g + 1) / kFxSlots) & 1));
@@ -354,11 +317,11 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
       // the buffer -- also implied by lfull, whose load waited for it) and "ready" b (Psi1 written)
       if (it >= 2) asm volatile("bar.sync %0, %1;" ::"r"(kFxBarFree + b), "n"(kFxHandoff) : "memory");
       if (nvalid) {
-        double* ps = lpsi(b) + (long long)x0 * ld2 + n;
+        R* ps = lpsi(b) + (long long)x0 * ld2 + n;
         const double* sg = lsig(b) + x0;
 #pragma unroll
         for (int c = 0; c < kFxXg; ++c) {
-          if (c < nxc) *ps = fma(nf, *ps, fa[c] * (sg[c] * tau));  // (powers of two: exact scaling)
+          if (c < nxc) *ps = (R)fma(nf, (double)*ps, fa[c] * (sg[c] * tau));  // (powers of two: exact scaling)
           ps += ld2;
         }
       }
@@ -381,7 +344,7 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
     const bool split = kPer && nx >= 4 * kFxSeg;
     const int P = nx / 2;  // pairs (periodic: nx even)
     const int p0 = split ? (g * P) / kFxSeg : 0, p1 = split ? ((g + 1) * P) / kFxSeg : 0;  // this segment's pairs
-    const PairCoef cf = pair_coef<kS>(p.coef + dom, 0);
+    const PairCoefT<T> cf = pair_coef_t<kS, T>(p.coef + dom, 0);  // (complex64: rounded once from FP64)
     const long long xs = (long long)nyz * norb;  // element stride between x points
     long long w_r = 0;
     FX_T0(t_all);
@@ -391,41 +354,41 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
       FX_T0(c5);
       asm volatile("bar.sync %0, %1;" ::"r"(kFxBarReady + b), "n"(kFxHandoff) : "memory");
       FX_ACC(w_r, c5);
-      const double2* L = reinterpret_cast<const double2*>(lpsi(b)) + s;
-      double2* out = p.psi + ((long long)dom * p.ng + t) * norb + s;
+      const T* L = reinterpret_cast<const T*>(lpsi(b)) + s;
+      T* out = static_cast<T*>(p.psi) + ((long long)dom * p.ng + t) * norb + s;
       if (split) {
-        LineMarch<kS> M;
+        LineMarch<kS, T, T> M;
         M.init();
         // plain shared-memory loads (ordered by the named barriers' memory clobbers, free to be scheduled early)
-        const double2* la = L + (2 * p0) * norb;
-        const double2* lf = lphi(b) + 2 * p0;  // Phi (the x pass's pre-phase)
+        const T* la = L + (2 * p0) * norb;
+        const T* lf = lphi(b) + 2 * p0 * kPhiStep + (kPhiStep == 2 ? (int)(t & 1) : 0);  // Phi (the pre-phase)
         if (active) {
-          M.first(cf, cmul(lf[0], la[0]), cmul(lf[1], la[norb]));
+          M.first(cf, cmul(lf[0], la[0]), cmul(lf[kPhiStep], la[norb]));
           la += 2 * norb;
-          lf += 2;
-          M.second(cf, cmul(lf[0], la[0]), cmul(lf[1], la[norb]));
+          lf += 2 * kPhiStep;
+          M.second(cf, cmul(lf[0], la[0]), cmul(lf[kPhiStep], la[norb]));
           la += 2 * norb;
-          lf += 2;
-          double2* o = out + (long long)(2 * p0 + 2) * xs;
+          lf += 2 * kPhiStep;
+          T* o = out + (long long)(2 * p0 + 2) * xs;
 #pragma unroll 2
           for (int q = p0 + 2; q < p1; ++q) {
-            const double2 a = cmul(lf[0], la[0]), c = cmul(lf[1], la[norb]);
-            M.steady(cf, a, c, [&](int k, double2 v) { o[k * xs] = v; });
+            const T a = cmul(lf[0], la[0]), c = cmul(lf[kPhiStep], la[norb]);
+            M.steady(cf, a, c, [&](int k, T v) { o[k * xs] = v; });
             la += 2 * norb;
-            lf += 2;
+            lf += 2 * kPhiStep;
             o += 2 * xs;
           }
         }
-        double2* xb = Xsm + ((b * kFxSeg + g) * 64 + s) * 2;  // [E output at the first point, at the last point]
+        T* xb = Xsm + ((b * kFxSeg + g) * 64 + s) * 2;  // [E output at the first point, at the last point]
         xb[0] = M.E10;
         xb[1] = M.prev_e1;
         asm volatile("bar.sync %0, %1;" ::"n"(kFxBarMarch), "n"(kFxMarch * 32) : "memory");
         if (active) {
           const int gl = g > 0 ? g - 1 : kFxSeg - 1, gr = g + 1 < kFxSeg ? g + 1 : 0;
-          const double2 lft = Xsm[((b * kFxSeg + gl) * 64 + s) * 2 + 1];  // left segment's last E output
-          const double2 rgt = Xsm[((b * kFxSeg + gr) * 64 + s) * 2];      // right segment's first E output
-          const double2 Ol = lk_L<kS>(cf.a2, cf.u2, M.prev_e1, rgt);       // O output at the segment's last point
-          const double2 Of = lk_R<kS>(cf.a2, cf.d2, lft, M.E10);           // O output at its first point
+          const T lft = Xsm[((b * kFxSeg + gl) * 64 + s) * 2 + 1];  // left segment's last E output
+          const T rgt = Xsm[((b * kFxSeg + gr) * 64 + s) * 2];      // right segment's first E output
+          const T Ol = lk_L<kS>(cf.a2, cf.u2, M.prev_e1, rgt);       // O output at the segment's last point
+          const T Of = lk_R<kS>(cf.a2, cf.d2, lft, M.E10);           // O output at its first point
           const int e = 2 * p1;
           out[(long long)(e - 2) * xs] = lk_L<kS>(cf.a1, cf.u1, M.prev_oR, Ol);
           out[(long long)(e - 1) * xs] = lk_R<kS>(cf.a1, cf.d1, M.prev_oR, Ol);
@@ -433,9 +396,9 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
           out[(long long)(2 * p0 + 1) * xs] = lk_R<kS>(cf.a1, cf.d1, Of, M.O1);
         }
       } else if (g == 0 && active) {
-        const double2* ph = lphi(b);
-        march_line<kPer, kS, double2, double2>(
-            nx, cf, [&](int i) { return cmul(ph[i], L[i * norb]); }, [&](int i, double2 v) { out[i * xs] = v; });
+        const T* ph = lphi(b) + (kPhiStep == 2 ? (int)(t & 1) : 0);
+        march_line<kPer, kS, T, T>(
+            nx, cf, [&](int i) { return cmul(ph[i * kPhiStep], L[i * norb]); }, [&](int i, T v) { out[i * xs] = v; });
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(&lempty[b]);  // the line producer may reload the buffer
@@ -458,9 +421,10 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
           FX_T0(c6);
           if (it >= 2) mbar_wait(&lempty[b], (uint32_t)(((it >> 1) - 1) & 1));
           FX_ACC(w_m, c6);
-          mbar_expect_tx(&lfull[b], (uint32_t)(nx * norb * 16 + nx * 16 + kFxN * 8));
+          mbar_expect_tx(&lfull[b], (uint32_t)(nx * norb * (int)sizeof(T) + nx * 16 + kFxN * 8));
           tma_4d(lpsi(b), &tPsi, 0, (int)t, 0, dom, &lfull[b]);
-          tma_4d(const_cast<double2*>(lphi(b)), &tPhi, 0, (int)t, 0, dom, &lfull[b]);
+          if (sizeof(T) == 16) tma_4d(const_cast<T*>(lphi(b)), &tPhi, 0, (int)t, 0, dom, &lfull[b]);
+          else tma_4d(const_cast<T*>(lphi(b)), &tPhi, (int)(t & ~1LL), 0, dom, 0, &lfull[b]);  // (16-byte aligned)
           tma_row(const_cast<double*>(lsig(b)), p.sig + ((long long)dom * nyz + t) * kFxN, kFxN * 8, &lfull[b]);
         }
   #ifdef LFD_FX_TIMING
@@ -479,8 +443,8 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
         FX_ACC(w_b, c0);
         tc_fence_after();
 #pragma unroll
-        for (int d = 2; d <= kI8S + 1; ++d) {
-          const int g = it * kFxAcc + (d - 2), sl = g % kFxSlots;
+        for (int d = 2; d <= S + 1; ++d) {
+          const int g = it * kAcc + (d - 2), sl = g % kFxSlots;
           if (g >= kFxSlots) {
             FX_T0(c1);
             mbar_wait(&dempty[sl], (uint32_t)(((g / kFxSlots) - 1) & 1));
@@ -490,9 +454,9 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
           const uint32_t acc = tacc + sl * kFxN;
           uint32_t accum = 0;  // 0 for the diagonal's first MMA
 #pragma unroll
-          for (int i = 1; i <= kI8S; ++i) {
+          for (int i = 1; i <= S; ++i) {
             const int j = d - i;
-            if (j < 1 || j > kI8S) continue;
+            if (j < 1 || j > S) continue;
             uint64_t db = db0 + (uint64_t)(((i - 1) * kFxSliceB) >> 4);
             uint32_t ta = tmem + (j - 1) * 32;
 #pragma unroll 1
@@ -512,7 +476,7 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
           mbar_wait(&bempty, (uint32_t)(it & 1));
           FX_ACC(w_e, c2);
           if (lane == 0) {
-            mbar_expect_tx(&bfull, kFxTileB);
+            mbar_expect_tx(&bfull, kTileB);
             tma_4d(Tsm, &tDig, 0, 0, 0, (int)((long long)dom * nyz + tn), &bfull);
           }
           __syncwarp();
@@ -534,28 +498,34 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
   }
 }
 
-FxMaps* gemm2x_maps_create(const Geometry& g, const int8_t* dig, double2* psi, const double2* phi) {
+FxMaps* gemm2x_maps_create(const Geometry& g, const int8_t* dig, void* psi, const void* phi) {
   FxMaps* m = new (std::nothrow) FxMaps;
   if (!m) return nullptr;
-  const uint64_t nyz = (uint64_t)g.ny * g.nz;
-  // digits [dom*nyz lines][6][nx][128 B], box [1][6][80][128] with the 128B swizzle (x rows past nx zero)
-  const uint64_t dd[4] = {(uint64_t)kFxK, (uint64_t)g.nx, (uint64_t)kI8S, (uint64_t)g.ndom * nyz};
-  const uint64_t sd[3] = {(uint64_t)kFxK, (uint64_t)g.nx * kFxK, (uint64_t)kI8S * g.nx * kFxK};
-  const uint32_t bd[4] = {(uint32_t)kFxK, (uint32_t)kFxN, (uint32_t)kI8S, 1};
-  // Psi as doubles [dom][x][yz][2 norb], box [1][nx][1][2 norb]: the line (y, z) of all orbitals
-  const uint64_t dp[4] = {(uint64_t)2 * g.norb, nyz, (uint64_t)g.nx, (uint64_t)g.ndom};
-  const uint64_t sp[3] = {(uint64_t)g.norb * 16, nyz * g.norb * 16, (uint64_t)g.ng * g.norb * 16};
-  const uint32_t bp[4] = {(uint32_t)(2 * g.norb), 1, (uint32_t)g.nx, 1};
-  // Phi as doubles [dom][x][yz][2], box [1][nx][1][2]
+  const uint64_t nyz = (uint64_t)g.ny * g.nz, S = (uint64_t)fx_digits(g.sp);
+  // digits [dom*nyz lines][S][nx][128 B], box [1][S][80][128] with the 128B swizzle (x rows past nx zero)
+  const uint64_t dd[4] = {(uint64_t)kFxK, (uint64_t)g.nx, S, (uint64_t)g.ndom * nyz};
+  const uint64_t sd[3] = {(uint64_t)kFxK, (uint64_t)g.nx * kFxK, S * g.nx * kFxK};
+  const uint32_t bd[4] = {(uint32_t)kFxK, (uint32_t)kFxN, (uint32_t)S, 1};
+  // Psi as 8-byte elements [dom][x][yz][E norb] (E = 2 doubles per complex128, 1 per complex64), box [1][nx][1][E norb]:
+  // the line (y, z) of all orbitals
+  const uint64_t E = g.sp ? 1 : 2, esz = g.sp ? 8 : 16;
+  const uint64_t dp[4] = {E * g.norb, nyz, (uint64_t)g.nx, (uint64_t)g.ndom};
+  const uint64_t sp[3] = {(uint64_t)g.norb * esz, nyz * g.norb * esz, (uint64_t)g.ng * g.norb * esz};
+  const uint32_t bp[4] = {(uint32_t)(E * g.norb), 1, (uint32_t)g.nx, 1};
+  // Phi: complex128 [dom][x][yz][2 doubles], box [1][nx][1][2]; complex64 [1][dom][x][yz] (8-byte elements), box
+  // [1][1][nx][2]: the line pair (2k, 2k + 1) holding the line (a 16-byte box that starts 16-byte aligned)
   const uint64_t df[4] = {2, nyz, (uint64_t)g.nx, (uint64_t)g.ndom};
   const uint64_t sf[3] = {16, nyz * 16, (uint64_t)g.ng * 16};
   const uint32_t bf[4] = {2, 1, (uint32_t)g.nx, 1};
+  const uint64_t df32[4] = {nyz, (uint64_t)g.nx, (uint64_t)g.ndom, 1};
+  const uint64_t sf32[3] = {nyz * 8, (uint64_t)g.ng * 8, (uint64_t)g.ndom * g.ng * 8};
+  const uint32_t bf32[4] = {2, (uint32_t)g.nx, 1, 1};
   if (encode_tmap(&m->dig, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, dig, dd, sd, bd, CU_TENSOR_MAP_SWIZZLE_128B) !=
           cudaSuccess ||
       encode_tmap(&m->psi, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, psi, dp, sp, bp, CU_TENSOR_MAP_SWIZZLE_NONE) !=
           cudaSuccess ||
-      encode_tmap(&m->phi, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, phi, df, sf, bf, CU_TENSOR_MAP_SWIZZLE_NONE) !=
-          cudaSuccess) {
+      encode_tmap(&m->phi, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, phi, g.sp ? df32 : df, g.sp ? sf32 : sf,
+                  g.sp ? bf32 : bf, CU_TENSOR_MAP_SWIZZLE_NONE) != cudaSuccess) {
     delete m;
     return nullptr;
   }
@@ -564,7 +534,7 @@ FxMaps* gemm2x_maps_create(const Geometry& g, const int8_t* dig, double2* psi, c
 
 void gemm2x_maps_destroy(FxMaps* m) { delete m; }
 
-cudaError_t launch_gemm2x_i8(const Geometry& g, const FxMaps* m, double2* psi, const DomCoef* coef, const double* nfac,
+cudaError_t launch_gemm2x_i8(const Geometry& g, const FxMaps* m, void* psi, const DomCoef* coef, const double* nfac,
                              const double2* Cp, const double* sig, bool scaled, int num_sms, cudaStream_t st) {
   FxArgs a;
   a.psi = psi; a.coef = coef; a.nfac = nfac; a.Cp = Cp; a.sig = sig;
@@ -573,21 +543,26 @@ cudaError_t launch_gemm2x_i8(const Geometry& g, const FxMaps* m, double2* psi, c
   if (cpd < 1) cpd = 1;
   if (cpd > a.nyz) cpd = a.nyz;
   dim3 grid(cpd, g.ndom);
-  // the C'' staging (nproj x norb complex) lives in the line-buffer region before the first line load
-  const size_t sm = std::max(fx_smem(g.nx, g.norb), (size_t)kFxTileB + (size_t)g.nproj * g.norb * 16 + 1024);
+  // the C'' staging (nproj x norb complex128) lives in the line-buffer region before the first line load
+  const size_t sm = std::max(fx_smem(g.nx, g.norb, g.sp),
+                             (size_t)fx_digits(g.sp) * kFxSliceB + (size_t)g.nproj * g.norb * 16 + 1024);
+#define LFD_FX(P, K)                                                                                             \
+  (g.sp ? launch_k(k_gemm2x_i8<P, K, float2, 4>, grid, kFxThreads, sm, st, m->dig, m->psi, m->phi, a)         \
+        : launch_k(k_gemm2x_i8<P, K, double2, kI8S>, grid, kFxThreads, sm, st, m->dig, m->psi, m->phi, a))
   if (g.bc == 0) {
-    if (scaled) launch_k(k_gemm2x_i8<true, true>, grid, kFxThreads, sm, st, m->dig, m->psi, m->phi, a);
-    else launch_k(k_gemm2x_i8<true, false>, grid, kFxThreads, sm, st, m->dig, m->psi, m->phi, a);
+    if (scaled) LFD_FX(true, true); else LFD_FX(true, false);
   } else {
-    if (scaled) launch_k(k_gemm2x_i8<false, true>, grid, kFxThreads, sm, st, m->dig, m->psi, m->phi, a);
-    else launch_k(k_gemm2x_i8<false, false>, grid, kFxThreads, sm, st, m->dig, m->psi, m->phi, a);
+    if (scaled) LFD_FX(false, true); else LFD_FX(false, false);
   }
+#undef LFD_FX
   return cudaGetLastError();
 }
 
 cudaError_t gemm2x_set_attributes() {
-  for (auto f : {k_gemm2x_i8<true, true>, k_gemm2x_i8<true, false>, k_gemm2x_i8<false, true>,
-                 k_gemm2x_i8<false, false>}) {
+  for (auto f : {k_gemm2x_i8<true, true, double2, kI8S>, k_gemm2x_i8<true, false, double2, kI8S>,
+                 k_gemm2x_i8<false, true, double2, kI8S>, k_gemm2x_i8<false, false, double2, kI8S>,
+                 k_gemm2x_i8<true, true, float2, 4>, k_gemm2x_i8<true, false, float2, 4>,
+                 k_gemm2x_i8<false, true, float2, 4>, k_gemm2x_i8<false, false, float2, 4>}) {
     cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kFxMaxSmem);
     if (e != cudaSuccess) return e;
   }

@@ -152,3 +152,18 @@ def test_sp_c2_default_path_is_int8_tensor_cores():
                   (w.hx, w.hy, w.hz), w.dt)
     assert lfd.lfd_nl_path(ctx.ctx) == 3
     ctx.close()
+
+
+@pytest.mark.parametrize("case", ["periodic", "zero_bc_odd_nx"])
+def test_sp_fused_first_factor(case):
+    """The SP first factor's GEMM-2 fused with Phi . K_x (k_gemm2x_i8 on complex64 lines, 4 digits, the march in
+    FP32): shapes that select it (even orbital count, ny nz even) with the int8-digit GEMMs forced -- periodic
+    (segmented march) and zero BC with an odd nx (whole-line march) -- at the SP bound over 60 steps."""
+    from paper_conf_ipps_razakhllknvn24_b200 import lfd
+    if case == "periodic":
+        w = workload("P0").with_(nx=20, norb=8, nocc=6)
+    else:
+        w = workload("P2z").with_(ny=6, nz=10, norb=4, nocc=4)
+    x = _inputs(w, 88)
+    steps = 60
+    assert_sp(w, _gpu(w, x, steps, flags=lfd.LFD_FLAG_NL_I8), _ref(w, x, steps), steps)
