@@ -266,7 +266,7 @@ __global__ void __launch_bounds__(kFxThreads, 1) k_gemm2x_i8(const __grid_consta
       double fa[kFxXg];
 #pragma unroll
       for (int c = 0; c < kFxXg; ++c) fa[c] = 0.0;
-#pragma unroll 1
+#pragma unroll  // (unrolled: 223 -> 221 us; in k_gemm2_i8 the same unroll took 174 -> 165 us)
       for (int dp = 0; dp < kAcc / 2; ++dp) {
         const int g = it * kAcc + 2 * dp, s0 = g % kFxSlots, s1 = (g + 1) % kFxSlots;
         FX_T0(c3);

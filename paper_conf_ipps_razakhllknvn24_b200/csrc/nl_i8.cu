@@ -299,7 +299,7 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
       double fa[kI8Rows];
 #pragma unroll
       for (int c = 0; c < kI8Rows; ++c) fa[c] = 0.0;
-#pragma unroll 1
+#pragma unroll  // (unrolled: C2 174 -> 165 us, the loads of the next pair overlap this pair's FP64 work)
       for (int dp = 0; dp < kI8Acc / 2; ++dp) {  // diagonals d = 2 + 2 dp and d + 1
         const int g = it * kI8Acc + 2 * dp, s0 = g % kI8Slots, s1 = (g + 1) % kI8Slots;
         mbar_wait(&dfull[s0], (uint32_t)((g / kI8Slots) & 1));
