@@ -393,6 +393,7 @@ __global__ void __launch_bounds__(kYZMaxThreads) k_kin_yz(const __grid_constant_
     int s_prev = 2, s_a = 4;  // slot of plane 2p-2 and of plane 2p (kYZS is even: pairs never straddle)
     uint32_t ph_a = 0;
     V* o0p = out0 + 2 * yst;  // plane 2p-2
+#pragma unroll 2  // (C2 148.3 -> 145.6 us)
     for (int p = 2; p < npairs; ++p) {
       mbar_wait(&full[s_a], ph_a);
       kz(s_a, wa0, wa1);
