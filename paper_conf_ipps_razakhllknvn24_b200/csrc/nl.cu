@@ -349,10 +349,13 @@ cudaError_t launch_gemm1(const Gemm1Args& a, cudaStream_t st) {
 // (e, sg) sums splits sg, sg+8, ... of element e (coalesced over e), then the 8 group sums are added in
 // group order. Blocks past the element range reduce the column norms the same way. Deterministic.
 // ------------------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(256) k_reduce(ReduceArgs p, int eblocks) {
+// 1024 threads: 32 split groups x 32 elements; a thread sums its groups' partials (s = sg, sg + 32, ...: <= 5 at
+// C2, all loads in flight) in order, then one thread per element the 32 group sums in order (deterministic).
+constexpr int kRedSG = 32;
+__global__ void __launch_bounds__(1024) k_reduce(ReduceArgs p, int eblocks) {
   pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
   pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
-  __shared__ double2 sh[8][32];
+  __shared__ double2 sh[kRedSG][32];
   const int dom = blockIdx.y;
   const int el = threadIdx.x & 31, sg = threadIdx.x >> 5;
   const long long per_dom = (long long)p.mrows * p.ncols;
@@ -362,17 +365,17 @@ __global__ void __launch_bounds__(256) k_reduce(ReduceArgs p, int eblocks) {
     if (e < per_dom) {
       const double2* src = p.part + (long long)dom * p.nsplit * per_dom + e;
       int s = sg;
-      for (; s + 56 < p.nsplit; s += 64) {  // 8 loads in flight, then added in the same order as one at a time
-        double2 v[8];
+      for (; s + 3 * kRedSG < p.nsplit; s += 4 * kRedSG) {  // 4 loads in flight, added in order
+        double2 v[4];
 #pragma unroll
-        for (int k = 0; k < 8; ++k) v[k] = src[(long long)(s + 8 * k) * per_dom];
+        for (int k = 0; k < 4; ++k) v[k] = src[(long long)(s + kRedSG * k) * per_dom];
 #pragma unroll
-        for (int k = 0; k < 8; ++k) {
+        for (int k = 0; k < 4; ++k) {
           sr += v[k].x;
           si += v[k].y;
         }
       }
-      for (; s < p.nsplit; s += 8) {
+      for (; s < p.nsplit; s += kRedSG) {
         const double2 v = src[(long long)s * per_dom];
         sr += v.x;
         si += v.y;
@@ -382,8 +385,8 @@ __global__ void __launch_bounds__(256) k_reduce(ReduceArgs p, int eblocks) {
     __syncthreads();
     if (sg == 0 && e < per_dom) {
       double tr = 0.0, ti = 0.0;
-#pragma unroll
-      for (int q = 0; q < 8; ++q) {
+#pragma unroll 8
+      for (int q = 0; q < kRedSG; ++q) {
         tr += sh[q][el].x;
         ti += sh[q][el].y;
       }
@@ -406,22 +409,13 @@ __global__ void __launch_bounds__(256) k_reduce(ReduceArgs p, int eblocks) {
     double acc = 0.0;
     if (n < p.ncols) {
       const double* ns = p.normp + (long long)dom * p.nsplit * p.ncols + n;
-      int s = sg;
-      for (; s + 56 < p.nsplit; s += 64) {  // as above: 8 loads in flight, same addition order
-        double v[8];
-#pragma unroll
-        for (int k = 0; k < 8; ++k) v[k] = ns[(long long)(s + 8 * k) * p.ncols];
-#pragma unroll
-        for (int k = 0; k < 8; ++k) acc += v[k];
-      }
-      for (; s < p.nsplit; s += 8) acc += ns[(long long)s * p.ncols];
+      for (int s = sg; s < p.nsplit; s += kRedSG) acc += ns[(long long)s * p.ncols];
     }
     sh[sg][el].x = acc;
     __syncthreads();
     if (sg == 0 && n < p.ncols) {
       double t = 0.0;
-#pragma unroll
-      for (int q = 0; q < 8; ++q) t += sh[q][el].x;
+      for (int q = 0; q < kRedSG; ++q) t += sh[q][el].x;
       p.s[(long long)dom * p.ncols + n] = p.scale * t;
     }
   }
@@ -432,7 +426,7 @@ cudaError_t launch_reduce(const ReduceArgs& a, cudaStream_t st) {
   const int eblocks = (int)((per_dom + 31) / 32);
   const int nblocks = a.s ? (a.ncols + 31) / 32 : 0;
   dim3 grid(eblocks + nblocks, a.ndom);
-  launch_k(k_reduce, grid, 256, 0, st, a, eblocks);
+  launch_k(k_reduce, grid, kRedSG * 32, 0, st, a, eblocks);
   return cudaGetLastError();
 }
 
