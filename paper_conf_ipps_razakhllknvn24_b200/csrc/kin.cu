@@ -241,7 +241,7 @@ __device__ __forceinline__ double dep_of(cf2 v) { return (double)v.a.x; }
 
 constexpr int kYZW = 8;
 constexpr int kYZMaxThreads = 352;  // up to 40 z pairs x 8 orbitals + the producer warp
-constexpr int kYZS = 10;            // ring depth (planes); even, so a y pair never straddles the wrap
+constexpr int kYZS = 16;            // ring depth (planes); even, so a y pair never straddles the wrap
 
 // bytes of one ring slot: the Psi segment [nz][8 orbitals] + the Phi row [nz], 128-byte aligned
 __host__ __device__ __forceinline__ int yz_slot_bytes(int nz) { return (nz * kYZW * 16 + nz * 16 + 127) & ~127; }
