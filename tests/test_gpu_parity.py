@@ -526,3 +526,14 @@ def test_wide_orbital_sets_short_projector_tile(norb, nproj, dims):
     w = workload("P0").with_(nx=dims[0], ny=dims[1], nz=dims[2], norb=norb, nocc=min(norb, 40), nproj=nproj)
     x = make_inputs(w, seed=16)
     assert_parity(w, run_gpu(w, x, 3, laser(w)), run_ref(w, x, 3, laser(w)))
+
+
+def test_large_nproj_carry_and_sequence():
+    """nproj = 1300 (> 1228: the projection carry's D / x / DC staging needs more than the 48 KB default dynamic
+    shared memory, k_nlmerge too): steps with the carry and a merged-factor sequence against the oracle."""
+    w = workload("P0").with_(nx=8, ny=8, nz=8, norb=4, nocc=4, nproj=1300)
+    x = make_inputs(w, seed=97)
+    dnl = np.ascontiguousarray(np.full((1, w.nproj), 0.07))
+    A = laser(w)
+    assert_parity(w, run_gpu(w, x, 2, A, dnl=dnl), run_ref(w, x, 2, A, dnl=dnl))
+    assert_parity(w, run_gpu_sequence(w, x, 2, A), run_ref(w, x, 2, A))
