@@ -669,7 +669,7 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
     const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
     long long w_pf = 0, w_afr = 0, w_st = 0;
     G1_T0(t_all);
-#pragma unroll(S == 5 ? 2 : 4)  // (129.1 -> 128.1 us)
+#pragma unroll(S == 5 ? 2 : 4)  // (FP64 129.1 -> 128.1 us; SP by 4: 89.4 -> 87.9)
     for (int g = 0, s = 0, ph = 0, ab = 0, aph = 0; g < nhalf; ++g) {
       G1_T0(c0);
       mbar_wait(&pfull[s], (uint32_t)ph);
