@@ -148,7 +148,6 @@ struct ReduceArgs {
   const double2* W = nullptr;  // [dom][mrows]: cprime = W out instead of -i eps out (exact factor)
 };
 cudaError_t launch_reduce(const ReduceArgs& a, cudaStream_t st);
-// launch_reduce + launch_nlnorm in one kernel for the plain factor (D real, cprime = -i eps D C n, no W / merge)
 
 // n_s = sqrt( s_s / (s_s + eps^2 * (DC)_s^H G (DC)_s) )   (Gram closed form of the Eq. 6 norm, R11),
 // then C'_s <- C'_s n_s in place: the GEMM-2 coefficient is always C'' = C' diag(n), so its epilogue is
