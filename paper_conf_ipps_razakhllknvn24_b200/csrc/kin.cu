@@ -70,8 +70,10 @@ cudaError_t launch_coef(const Geometry& g, const CoefParams& p, int dom0, int co
 // constant sqrt(g) of the scaled pair form (1 for the general form).
 // The kernel also keeps a copy of v_loc for lfd_energy (vcopy may alias v: then it is not written).
 // With cf.count > 0 the first block also writes the coefficient tables of a pending lfd_set_vector_potential.
+// (__launch_bounds__(256, 4): 64 registers instead of 126 -- the coefficient write of block 0 and sincos's
+// never-taken large-argument path spill instead; 4 CTAs per SM: ncu 7.7 -> 6.6 us at C2)
 template <class C>
-__global__ void k_phase(const double* __restrict__ v, C* __restrict__ phi, double* vcopy, long long n,
+__global__ void __launch_bounds__(256, 4) k_phase(const double* __restrict__ v, C* __restrict__ phi, double* vcopy, long long n,
                         double half_dt, double2 sg, CoefFuse cf, double hx, double hy, double hz) {
   pdl_wait();     // programmatic dependent launch: the previous kernel's writes are visible
   pdl_trigger();  // let the next kernel launch (its CTAs wait in pdl_wait)
