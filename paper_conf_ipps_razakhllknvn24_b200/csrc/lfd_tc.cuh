@@ -137,6 +137,17 @@ __device__ __forceinline__ double scale_pow2(double x, double a, double b) {
   return zero ? 0.0 : __hiloint2double(hx + ((ea + eb - 2046) << 20), __double2loint(x));
 }
 
+// x sigma tau for power-of-two FP64 scales, on an FP32 x (the SP epilogues): exponent-field arithmetic; a result
+// below the FP32 normal range flushes to 0 (an SP update that small is far below the SP rounding of Psi)
+__device__ __forceinline__ float scale_pow2f(float x, double a, double b) {
+  const int ea = (__double2hiint(a) >> 20) & 0x7ff, eb = (__double2hiint(b) >> 20) & 0x7ff;
+  const int hx = __float_as_int(x), k = ea + eb - 2046;
+  const int ex = (hx >> 23) & 0xff;
+  return (ea == 0 || eb == 0 || ex == 0 || ex + k <= 0) ? 0.0f : __int_as_float(hx + (k << 23));
+}
+// exact int32 -> float for |x| < 2^22: 1.5 2^23 + x built from bits, minus 1.5 2^23
+__device__ __forceinline__ float i2f(int32_t x) { return __int_as_float(0x4B400000 + x) - 12582912.0f; }
+
 __device__ __forceinline__ int row_exponent(double mx) {
   int e = 0;
   frexp(mx, &e);  // mx = m 2^e, m in [0.5, 1): mx < 2^e

@@ -296,9 +296,13 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
     for (long long t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
       const long long r0 = t * kI8NT + kI8Rows * h;
       const int nc = (int)((ng - r0) < kI8Rows ? (ng - r0) : kI8Rows);  // valid rows of this warp
-      double fa[kI8Rows];
+      // SP (R = float): each diagonal converted exactly (|P_d| < 2^21 for S = 4) and accumulated in FP32, the
+      // scaling by exponent arithmetic on the float -- no FP64 pipe work in the SP epilogue
+      constexpr bool kF32 = sizeof(R) == 4;
+      using A = std::conditional_t<kF32, float, double>;
+      A fa[kI8Rows];
 #pragma unroll
-      for (int c = 0; c < kI8Rows; ++c) fa[c] = 0.0;
+      for (int c = 0; c < kI8Rows; ++c) fa[c] = A(0);
 #pragma unroll  // (unrolled: C2 174 -> 165 us, the loads of the next pair overlap this pair's FP64 work)
       for (int dp = 0; dp < kI8Acc / 2; ++dp) {  // diagonals d = 2 + 2 dp and d + 1
         const int g = it * kI8Acc + 2 * dp, s0 = g % kI8Slots, s1 = (g + 1) % kI8Slots;
@@ -316,13 +320,19 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
           mbar_arrive(&dempty[s0]);
           mbar_arrive(&dempty[s1]);
         }
-        const double wd = ldexp(1.0, -14 * dp - 7);
-        if (dp == 0) {  // fa = (m - M) wd in one fma: m = M + x built from bits, exact result x wd
+        if constexpr (kF32) {
+          const float w0 = __int_as_float((127 - 14 * dp) << 23), w1 = __int_as_float((120 - 14 * dp) << 23);
 #pragma unroll
-          for (int c = 0; c < kI8Rows; ++c) fa[c] = fma(i2d_raw(a0[c] * 128 + a1[c]), wd, -kI2dM * wd);
+          for (int c = 0; c < kI8Rows; ++c) fa[c] = fmaf(i2f(a1[c]), w1, fmaf(i2f(a0[c]), w0, fa[c]));
         } else {
+          const double wd = ldexp(1.0, -14 * dp - 7);
+          if (dp == 0) {  // fa = (m - M) wd in one fma: m = M + x built from bits, exact result x wd
 #pragma unroll
-          for (int c = 0; c < kI8Rows; ++c) fa[c] = fma(i2d(a0[c] * 128 + a1[c]), wd, fa[c]);
+            for (int c = 0; c < kI8Rows; ++c) fa[c] = fma(i2d_raw(a0[c] * 128 + a1[c]), wd, -kI2dM * wd);
+          } else {
+#pragma unroll
+            for (int c = 0; c < kI8Rows; ++c) fa[c] = fma(i2d(a0[c] * 128 + a1[c]), wd, fa[c]);
+          }
         }
       }
       // the warp's staged Psi sub-tile (rows 16 h .. 16 h + 15 of the tile)
@@ -335,7 +345,11 @@ __global__ void __launch_bounds__(kI8Threads, 1) k_gemm2_i8(Gemm2Args p) {
           R* po = pout + r0 * ld;
 #pragma unroll
           for (int c = 0; c < kI8Rows; ++c) {
-            if (c < nc) *po = (R)fma(nf, (double)*ps, scale_pow2(fa[c], sg[c], tau));
+            if constexpr (kF32) {
+              if (c < nc) *po = fmaf((float)nf, (float)*ps, scale_pow2f(fa[c], sg[c], tau));
+            } else {
+              if (c < nc) *po = (R)fma(nf, (double)*ps, scale_pow2(fa[c], sg[c], tau));
+            }
             po += ld;
             ps += ld;
           }
