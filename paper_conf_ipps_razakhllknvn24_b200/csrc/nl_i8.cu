@@ -454,6 +454,20 @@ __device__ __forceinline__ void g1_bytes(const double v[4], double sc, double ma
   (void)hi;
 }
 
+// The SP variant (S = 3) from FP32 values: fma(v, sc, 1.5 2^23) is 1.5 2^23 + X exactly for |X| <= 2^22, its
+// low 24 bits are X + 2^22 (the exponent's low bit is 0 below 2^24 and 1 at X = 2^22 exactly), so adding 2^22
+// to the word gives the offset-binary X + 2^23 in the low 3 bytes, as the FP64 form's low bytes (g1_madd_a<3>).
+__device__ __forceinline__ void g1_bytes3f(const float v[4], float sc, uint32_t out[3]) {
+  uint32_t lo[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) lo[q] = __float_as_uint(fmaf(v[q], sc, 12582912.0f)) + 0x400000u;
+  const uint32_t a = __byte_perm(lo[0], lo[1], 0x5140), b = __byte_perm(lo[0], lo[1], 0x7362);
+  const uint32_t c = __byte_perm(lo[2], lo[3], 0x5140), d = __byte_perm(lo[2], lo[3], 0x7362);
+  out[0] = __byte_perm(a, c, 0x5410);
+  out[1] = __byte_perm(a, c, 0x7632);
+  out[2] = __byte_perm(b, d, 0x5410);
+}
+
 __device__ __forceinline__ void umma_g1_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t accumulate,
                                            uint32_t idesc) {
   asm volatile(
@@ -679,6 +693,14 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
     const double sc = zc ? 0.0 : ldexp(1.0, 8 * S - 2 - (E - 1022));  // x 2^(8S-2) / tau_s
     const double sc2 = cm ? -sc : sc;         // the odd row's second component is -Re
     constexpr double kMA = g1_madd_a<S>();
+    // SP: the digits from the FP32 values (g1_bytes3f) and the norm per quarter block in FP32, so the workers do
+    // no FP64 conversions; the scale 2^(22 - (E - 1022)) is a normal float unless max |psi_s| < 2^-106, and such
+    // an orbital is taken as zero (its contribution to C is below 1e-32)
+    constexpr bool kF = sizeof(R) == 4;
+    static_assert(!kF || S == 3, "the FP32 digit path is the 3-digit SP scheme");
+    const int esc = 8 * S - 2 - (E - 1022);
+    const float scf = (zc || esc > 127) ? 0.0f : __int_as_float((esc + 127) << 23);
+    const float scf2 = cm ? -scf : scf;
     double nrm = 0.0;
     const uint32_t trow = tmem + ((uint32_t)(32 * q) << 16);
     long long w_pf = 0, w_afr = 0, w_st = 0;
@@ -692,7 +714,8 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
       // this lane's components of Psi[row][sIdx] for rows 4h .. 4h+3: (Re, Im) for the even row m = 2s, (Im, Re)
       // for the odd row (its Re enters negated: sc2)
       const R* P = reinterpret_cast<const R*>(Psm + s * kG1PsiB) + 2 * sIdx + 8 * h * norb;
-      double v1[4], v2[4];
+      using V = std::conditional_t<kF, float, double>;
+      V v1[4], v2[4];
       if (sv && ra + 4 * h + 4 <= r1) {  // all 4 rows present (every quarter block but a split's ragged last)
 #pragma unroll
         for (int t = 0; t < 4; ++t) { v1[t] = P[t * 2 * norb + cm]; v2[t] = P[t * 2 * norb + 1 - cm]; }
@@ -700,19 +723,26 @@ __global__ void __launch_bounds__(kG1Threads, 1) k_gemm1_i8(Gemm1I8Args p) {
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
           const bool ok = sv && ra + 4 * h + t < r1;
-          v1[t] = ok ? P[t * 2 * norb + cm] : 0.0;
-          v2[t] = ok ? P[t * 2 * norb + 1 - cm] : 0.0;
+          v1[t] = ok ? (V)P[t * 2 * norb + cm] : V(0);
+          v2[t] = ok ? (V)P[t * 2 * norb + 1 - cm] : V(0);
         }
       }
       // this lane's share of the column norm: Re^2 (even lane, v1 = Re) or Im^2 (odd lane, v1 = Im); the pair
       // is summed once at the end. Absent rows add +0.
-      nrm = fma(v1[0], v1[0], nrm);
-      nrm = fma(v1[1], v1[1], nrm);
-      nrm = fma(v1[2], v1[2], nrm);
-      nrm = fma(v1[3], v1[3], nrm);
       uint32_t d1[S], d2[S];
-      g1_bytes<S>(v1, sc, kMA, d1);
-      g1_bytes<S>(v2, sc2, kMA, d2);
+      if constexpr (kF) {
+        const float nq = fmaf(v1[3], v1[3], fmaf(v1[2], v1[2], fmaf(v1[1], v1[1], v1[0] * v1[0])));
+        nrm += (double)nq;
+        g1_bytes3f(v1, scf, d1);
+        g1_bytes3f(v2, scf2, d2);
+      } else {
+        nrm = fma(v1[0], v1[0], nrm);
+        nrm = fma(v1[1], v1[1], nrm);
+        nrm = fma(v1[2], v1[2], nrm);
+        nrm = fma(v1[3], v1[3], nrm);
+        g1_bytes<S>(v1, sc, kMA, d1);
+        g1_bytes<S>(v2, sc2, kMA, d2);
+      }
       G1_T0(c1);
       if (g >= kNBuf) mbar_wait(&afree[ab], (uint32_t)(aph ^ 1));  // the MMAs of quarter block g - NBuf are done
       G1_ACC(w_afr, c1);

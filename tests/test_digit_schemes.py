@@ -120,3 +120,28 @@ def test_gemm2_balanced_digits_and_error():
     got = acc * 2.0 ** (ex + ew - 2 * (7 * S - 1))
     want = float(np.dot(x, w))
     assert abs(got - want) <= K * 2.0 ** -39 * 2.0 ** (ex + ew)
+
+
+def test_gemm1_sp_fp32_digit_trick():
+    """The SP GEMM-1's digits from FP32 values (g1_bytes3f): the float bits of v*sc + 1.5 2^23, plus 2^22, hold
+    the offset-binary X + 2^23 (X = rint(v sc), |X| <= 2^22) in their low 24 bits -- the same bytes as the
+    FP64 form with g1_madd_a<3> -- including both ends X = -2^22 and X = +2^22 (where the float reaches 2^24 and
+    its exponent's low bit becomes the 2^23 bit)."""
+    rng = np.random.default_rng(7)
+    e = -3  # tau = 2^e > max |v|
+    sc = np.float32(2.0 ** (22 - e))
+    v = rng.uniform(-1, 1, 200000).astype(np.float32) * np.float32(2.0 ** e)
+    edge = (np.array([-2.0 ** 22, 2.0 ** 22, -2.0 ** 22 + 1, 2.0 ** 22 - 1, 0.5, -0.5, 1.5, -1.5, 0.0]) /
+            float(sc)).astype(np.float32)
+    v = np.concatenate([v, edge])
+    f = v * sc + np.float32(12582912.0)  # v*sc exact (power of two); the add rounds to nearest even = rint
+    assert f.dtype == np.float32
+    low = (f.view(np.uint32).astype(np.int64) + (1 << 22)) & ((1 << 24) - 1)
+    X = np.rint(v.astype(np.float64) * float(sc)).astype(np.int64)
+    assert np.abs(X).max() <= 1 << 22
+    assert np.array_equal(low, X + (1 << 23))
+    # the same three bytes as the FP64 route of the 3-digit scheme
+    Xd, bytes_d = g1_a_digits(v.astype(np.float64), 3, e)
+    assert np.array_equal(Xd, X)
+    for k in range(3):
+        assert np.array_equal((low >> (8 * k)) & 255, bytes_d[k])
