@@ -532,6 +532,11 @@ __global__ void __launch_bounds__(kQMaxThreads, 1) k_density_q(const __grid_cons
   const double2 ex = cf->eth[0], ey = cf->eth[1], ez = cf->eth[2];
   const double ihx = cf->inv_h[0], ihy = cf->inv_h[1], ihz = cf->inv_h[2];
   const double w2x = ihx * ihx, w2y = ihy * ihy, w2z = ihz * ihz;
+  // the per-point combination (rho, the link products, j, the lane reduce-scatter) in the accumulators' type:
+  // FP32 for the SP variant (no FP64 pipe work per point but the final store conversion), FP64 otherwise
+  using PA = typename std::conditional<sizeof(C) == 8, float, double>::type;
+  const PA exx = (PA)ex.x, exy = (PA)ex.y, eyx = (PA)ey.x, eyy = (PA)ey.y, ezx = (PA)ez.x, ezy = (PA)ez.y;
+  const PA ihxa = (PA)ihx, ihya = (PA)ihy, ihza = (PA)ihz;
   const uint32_t lo = (uint32_t)(mp.pad + q) * (uint32_t)sizeof(C);  // this lane's first orbital (s = q) in a row
   const uint32_t orow = (uint32_t)ptr * rs + lo;
   const bool zin = ptr + 1 < zc;  // z+1 in the segment (else the halo point)
@@ -601,10 +606,10 @@ __global__ void __launch_bounds__(kQMaxThreads, 1) k_density_q(const __grid_cons
           orb(i, (A)fsh[q + 4 * i], acc[0], *reinterpret_cast<const C*>(O + i * 4 * (int)sizeof(C)), nn);
       }
     }
-    const double rho = (double)acc[0][0] + acc[1][0], pxr = (double)acc[0][1] + acc[1][1];
-    const double pxi = (double)acc[0][2] + acc[1][2], pyr = (double)acc[0][3] + acc[1][3];
-    const double pyi = (double)acc[0][4] + acc[1][4], pzr = (double)acc[0][5] + acc[1][5];
-    const double pzi = (double)acc[0][6] + acc[1][6];
+    const PA rho = (PA)acc[0][0] + acc[1][0], pxr = (PA)acc[0][1] + acc[1][1];
+    const PA pxi = (PA)acc[0][2] + acc[1][2], pyr = (PA)acc[0][3] + acc[1][3];
+    const PA pyi = (PA)acc[0][4] + acc[1][4], pzr = (PA)acc[0][5] + acc[1][5];
+    const PA pzi = (PA)acc[0][6] + acc[1][6];
     // this warp is done with own line y and x+1 line y (once its loads have returned: lfd_tma.cuh)
     mbar_release2(&oempty[so], &xempty[sx], xring, ((rho + pxr) + (pyr + pzr)) + (pxi + pyi + pzi), lane == 0);
     if (++so == nso) { so = 0; pho ^= 1u; }
@@ -612,27 +617,27 @@ __global__ void __launch_bounds__(kQMaxThreads, 1) k_density_q(const __grid_cons
     if (xring && ++sx == nsx) { sx = 0; phx ^= 1u; }
     // the currents and the kinetic energy density are linear in the P_d: form them per lane first
     // (Im(e^{i theta} P) = cos Im P + sin Re P, Re(e^{i theta} P) = cos Re P - sin Im P)
-    const double jx = (kPer || has_x) ? (ex.x * pxi + ex.y * pxr) * ihx : 0.0;
-    const double jy = (kPer || has_y) ? (ey.x * pyi + ey.y * pyr) * ihy : 0.0;
-    const double jz = (kPer || has_z) ? (ez.x * pzi + ez.y * pzr) * ihz : 0.0;
+    const PA jx = (kPer || has_x) ? (exx * pxi + exy * pxr) * ihxa : PA(0);
+    const PA jy = (kPer || has_y) ? (eyx * pyi + eyy * pyr) * ihya : PA(0);
+    const PA jz = (kPer || has_z) ? (ezx * pzi + ezy * pzr) * ihza : PA(0);
     if (a.epart) {  // kinetic energy density (FD Peierls form) summed per lane; reduced per CTA at the end
-      double ek = (w2x + w2y + w2z) * rho;
-      if (kPer || has_x) ek -= w2x * (ex.x * pxr - ex.y * pxi);
-      if (kPer || has_y) ek -= w2y * (ey.x * pyr - ey.y * pyi);
-      if (kPer || has_z) ek -= w2z * (ez.x * pzr - ez.y * pzi);
+      double ek = (w2x + w2y + w2z) * (double)rho;
+      if (kPer || has_x) ek -= w2x * (ex.x * (double)pxr - ex.y * (double)pxi);
+      if (kPer || has_y) ek -= w2y * (ey.x * (double)pyr - ey.y * (double)pyi);
+      if (kPer || has_z) ek -= w2z * (ez.x * (double)pzr - ez.y * (double)pzi);
       ekin += ek;
     }
     // reduce-scatter of (rho, jx, jy, jz) over the 4 lanes of the point (lanes xor 16, then xor 8; fixed order)
-    double u0, u1;
+    PA u0, u1;
     {
       const bool hi = (q & 2) != 0;  // q = 2, 3 keep (jy, jz); q = 0, 1 keep (rho, jx)
-      const double s0 = hi ? rho : jy, s1 = hi ? jx : jz;
-      const double k0 = hi ? jy : rho, k1 = hi ? jz : jx;
+      const PA s0 = hi ? rho : jy, s1 = hi ? jx : jz;
+      const PA k0 = hi ? jy : rho, k1 = hi ? jz : jx;
       u0 = k0 + __shfl_xor_sync(0xffffffffu, s0, 16);
       u1 = k1 + __shfl_xor_sync(0xffffffffu, s1, 16);
     }
     const bool odd = (q & 1) != 0;  // keep the second of the two
-    const double val = (odd ? u1 : u0) + __shfl_xor_sync(0xffffffffu, odd ? u0 : u1, 8);
+    const double val = (double)((odd ? u1 : u0) + __shfl_xor_sync(0xffffffffu, odd ? u0 : u1, 8));
     // lane q now holds value q of its point: 0 rho, 1 jx, 2 jy, 3 jz
     if (valid) {
       const long long o = (long long)x * a.sx + (long long)y * a.sy + z;
